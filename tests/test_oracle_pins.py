@@ -1,0 +1,297 @@
+"""Pins for the CPU oracle (oracle/dbg_oracle.cpp) against what the paper and the mathematics fix.
+
+None of these re-types the oracle's own formula: each one checks it against a value printed in
+the paper (tests/golden/), an independent closed form, an invariant, or a string brute force.
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+
+from oracle import brute
+from synth import genome, make_reads, random_reads, ReadSet
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _as_dict(recs, k):
+    d = {}
+    for r in recs:
+        code = (int(r["key_hi"]) << 64) | int(r["key_lo"])
+        s = "".join("ACGT"[(code >> (2 * (k - 1 - t))) & 3] for t in range(k))
+        d[s] = [int(r["count"]), [int(x) for x in r["out"]], [int(x) for x in r["in"]], int(r["pid"])]
+    return d
+
+
+def _readset(reads):
+    b = "".join(reads).encode()
+    offs = np.zeros(len(reads) + 1, dtype=np.uint64)
+    offs[1:] = np.cumsum([len(r) for r in reads])
+    return ReadSet(np.frombuffer(b, dtype=np.uint8).copy(), offs)
+
+
+# ---------------------------------------------------------------- paper-printed values
+
+
+def test_fig1_worked_example(oracle_lib):
+    """PAPER.md Fig. 1 (L186-197): edge multiplicities 2 and 1 (tests/golden/fig1_edges.txt)."""
+    lines = [l.split() for l in open(os.path.join(GOLD, "fig1_edges.txt")) if l.strip() and l[0] != "#"]
+    k = int(lines[0][1])
+    np_ = int(lines[1][1])
+    reads = lines[2][1:]
+    expect = {l[0]: [int(l[1]), [int(x) for x in l[2:6]], [int(x) for x in l[6:10]]] for l in lines[3:]}
+    rs = _readset(reads)
+    got = _as_dict(oracle_lib.graph(rs.seq, rs.offsets, k, 3, np_), k)
+    assert {v: e[:3] for v, e in got.items()} == expect
+
+
+def test_fig1_kmer_count():
+    """Fig. 1: reads of length 23 with K=5 give 19 K-mers each (L187-190); N(L-K+1) (L176-177)."""
+    rs = random_reads(7, 23, 23, seed=11)
+    import oracle
+
+    recs = oracle.graph(rs.seq, rs.offsets, 5, 3, 4)
+    assert int(recs["count"].sum()) == 7 * 19
+
+
+def test_fig4_encoding(oracle_lib):
+    """Fig. 4 (L598-606): the 2-word K-mer "00100101,01110011" is AGCCCTAT under reading A."""
+    lines = dict(l.split() for l in open(os.path.join(GOLD, "fig4_encoding.txt")) if l.strip() and l[0] != "#")
+    assert oracle_lib.canonical(lines["KMER"]) == int(lines["BITS"], 2)
+
+
+def test_table1_occurrence_formula():
+    """Table I (L925-935): # duplicate vertices = N (L-K+1) within the 2 % rounding of N."""
+    for l in open(os.path.join(GOLD, "table1_table2.txt")):
+        f = l.split()
+        if f and f[0] == "TABLE1":
+            L, n_m, dup_m = int(f[2]), float(f[3]), float(f[4])
+            assert abs(n_m * (L - 27 + 1) - dup_m) / dup_m < 0.02
+
+
+def test_table1_occurrences_on_oracle(oracle_lib):
+    """I1 at a Table-I read length: sum of vertex counts = N (L-K+1) (K=27, L=101)."""
+    g = genome(20_000, seed=7)
+    seq, offs = make_reads(g, 300, 101, 0.005, seed=8)
+    recs = oracle_lib.graph(seq, offs, 27, 11, 8)
+    assert int(recs["count"].sum()) == 300 * (101 - 27 + 1)
+
+
+def test_property1_appendix_closed_form():
+    """Appendix, Eqs. (4)/(5) (L1349-1434): E[#erroneous K-mers | one error] by enumeration."""
+    for L in (23, 50, 100, 101, 124):
+        for K in range(1, L + 1):
+            # exact: average over the error position of the K-mers covering it
+            cover = [min(e, L - K) - max(0, e - K + 1) + 1 for e in range(L)]
+            exact = sum(cover) / L
+            if K <= (L + 1) // 2:
+                paper = K * (L - 2 * K + 2) / L + sum(m * 2 / L for m in range(1, K))
+            else:
+                paper = (L - K + 1) * (2 * K - L) / L + sum(m * 2 / L for m in range(1, L - K + 1))
+            assert math.isclose(exact, paper, rel_tol=1e-12), (L, K)
+            assert math.isclose(exact, K * (L - K + 1) / L, rel_tol=1e-12)
+            assert exact <= (L + 1) ** 2 / (4 * L) + 1e-12  # the Theta(L/4) bound of (4)/(5)
+
+
+def test_property1_distinct_vertices_statistical(oracle_lib):
+    """Property 1 (L540-555): distinct vertices ~ covered genome K-mers + erroneous K-mers."""
+    G, N, L, K, e = 40_000, 4_000, 100, 31, 0.01
+    g = genome(G, seed=21)
+    seq, offs = make_reads(g, N, L, e, seed=22)
+    recs = oracle_lib.graph(seq, offs, K, 11, 4, n_threads=4)
+    p_ok = (1 - e) ** K
+    starts = G - L + 1
+    covered = 0.0
+    for x in range(G - K + 1):
+        n_cov = min(x, G - L) - max(0, x + K - L) + 1
+        q = n_cov / starts
+        covered += 1 - (1 - q * p_ok) ** N
+    erroneous = N * (L - K + 1) * (1 - p_ok)
+    expect = covered + erroneous
+    assert abs(len(recs) - expect) / expect < 0.01, (len(recs), expect)
+
+
+# ---------------------------------------------------------------- brute force
+
+
+@pytest.mark.parametrize(
+    "k,p,np_,seed",
+    [(3, 1, 1, 1), (3, 3, 3, 2), (5, 3, 3, 3), (5, 5, 16, 4), (7, 1, 16, 5), (7, 3, 2, 6),
+     (31, 11, 16, 7), (31, 31, 3, 8), (9, 4, 5, 9), (33, 13, 7, 10), (63, 19, 16, 11),
+     (63, 1, 4, 12)],
+)
+def test_oracle_vs_string_brute_force(oracle_lib, k, p, np_, seed):
+    rs = random_reads(40, 1, 2 * k + 40, seed=seed, n_rate=0.02, lower_rate=0.05)
+    got = _as_dict(oracle_lib.graph(rs.seq, rs.offsets, k, p, np_), k)
+    want = brute.graph(rs.reads(), k, p, np_)
+    assert got == want
+
+
+def test_oracle_threads_equal(oracle_lib):
+    rs = random_reads(300, 20, 120, seed=13)
+    a = oracle_lib.graph(rs.seq, rs.offsets, 11, 5, 7, n_threads=1)
+    b = oracle_lib.graph(rs.seq, rs.offsets, 11, 5, 7, n_threads=5)
+    assert a.tobytes() == b.tobytes()
+
+
+def test_oracle_msp_vs_brute(oracle_lib):
+    for (k, p, np_, seed) in [(5, 3, 4, 1), (31, 11, 16, 2), (21, 7, 3, 3), (9, 9, 5, 4)]:
+        rs = random_reads(30, 1, 90, seed=seed)
+        sk = oracle_lib.msp(rs.seq, rs.offsets, k, p, np_)
+        want = brute.superkmers(rs.reads(), k, p, np_)
+        got = [(int(s["read"]), int(s["start"]), int(s["n_kmers"]), int(s["pid"]), int(s["has_left"]),
+                int(s["has_right"])) for s in sk]
+        assert got == [w[:6] for w in want]
+        assert [int(s["minimizer"]) for s in sk] == [brute.code(w[6]) for w in want]
+
+
+# ---------------------------------------------------------------- closed form and invariants
+
+
+@pytest.mark.parametrize("k,seed", [(3, 1), (5, 2), (7, 3), (11, 4), (31, 5)])
+def test_kplus1_closed_form(oracle_lib, k, seed):
+    """Edge multiplicities equal (K+1)-mer counts (north star; odd K, no palindromes)."""
+    rs = random_reads(60, 1, 80, seed=seed, alphabet=b"ACGT" if k > 5 else b"ACGTAC")
+    got = {v: e[:3] for v, e in _as_dict(oracle_lib.graph(rs.seq, rs.offsets, k, 1, 1), k).items()}
+    assert got == brute.kplus1_closed_form(rs.reads(), k)
+
+
+def test_kplus1_closed_form_with_palindromic_kplus1mers(oracle_lib):
+    """A palindromic (K+1)-mer (even length) increments the same counter twice (reading K)."""
+    reads = ["ACGT", "AACGTT", "TTAA", "GAATTC", "ACGTACGT"]
+    rs = _readset(reads)
+    got = {v: e[:3] for v, e in _as_dict(oracle_lib.graph(rs.seq, rs.offsets, 3, 1, 1), 3).items()}
+    assert got == brute.kplus1_closed_form(reads, 3)
+
+
+def _tiny_erroneous():
+    g = genome(30_000, seed=31)
+    seq, offs = make_reads(g, 2_000, 100, 0.01, seed=32)
+    return ReadSet(seq, offs)
+
+
+def test_invariants_I1_I2_I3_I4(oracle_lib):
+    rs = _tiny_erroneous()
+    K, P, NP = 31, 11, 16
+    recs = oracle_lib.graph(rs.seq, rs.offsets, K, P, NP, n_threads=4)
+    L = rs.lengths()
+    # I1: total vertex occurrences
+    assert int(recs["count"].sum()) == int(np.maximum(L - K + 1, 0).sum())
+    # I2: every adjacent K-mer pair counts once at each endpoint
+    assert int(recs["out"].sum() + recs["in"].sum()) == 2 * int(np.maximum(L - K, 0).sum())
+    d = _as_dict(recs, K)
+    # I3 mirror: out_v[c] > 0 -> w = v[1:]+c has the matching in-edge (or out-edge if w is not canonical)
+    for v, (cnt, out, inn, pid) in d.items():
+        for ci, c in enumerate("ACGT"):
+            if out[ci]:
+                w = v[1:] + c
+                cw = brute.canonical_string(w)
+                if cw == w:
+                    assert d[cw][2]["ACGT".index(v[0])] == out[ci]
+                else:
+                    assert d[cw][1][3 - "ACGT".index(v[0])] == out[ci]
+            if inn[ci]:
+                w = c + v[:-1]
+                cw = brute.canonical_string(w)
+                if cw == w:
+                    assert d[cw][1]["ACGT".index(v[-1])] == inn[ci]
+                else:
+                    assert d[cw][2][3 - "ACGT".index(v[-1])] == inn[ci]
+    # I4 placement, recomputed from the vertex string alone with the string brute force
+    for v, e in list(d.items())[:3000]:
+        assert e[3] == brute.partition(v, P, NP)
+
+
+def test_invariant_I5_strand_symmetry(oracle_lib):
+    rs = random_reads(100, 10, 90, seed=41)
+    reads = rs.reads()
+    a = oracle_lib.graph(rs.seq, rs.offsets, 15, 5, 9)
+    rr = _readset([brute.rc(r) for r in reads])
+    b = oracle_lib.graph(rr.seq, rr.offsets, 15, 5, 9)
+    assert a.tobytes() == b.tobytes()
+
+
+def test_invariant_I6_partition_independence(oracle_lib):
+    rs = _tiny_erroneous().subset(0, 600)
+    base = None
+    for P in (1, 5, 11, 31):
+        for NP in (1, 16, 512):
+            r = oracle_lib.graph(rs.seq, rs.offsets, 31, P, NP, n_threads=2)
+            key = b"".join(r[f].tobytes() for f in ("key_hi", "key_lo", "count", "out", "in"))
+            base = base or key
+            assert key == base
+
+
+def test_read_permutation_and_union(oracle_lib):
+    rs = random_reads(80, 5, 70, seed=51)
+    reads = rs.reads()
+    perm = np.random.default_rng(3).permutation(len(reads))
+    rp = _readset([reads[i] for i in perm])
+    a = oracle_lib.graph(rs.seq, rs.offsets, 9, 3, 5)
+    b = oracle_lib.graph(rp.seq, rp.offsets, 9, 3, 5)
+    assert a.tobytes() == b.tobytes()
+    # additivity under read-set union
+    h1, h2 = _readset(reads[:40]), _readset(reads[40:])
+    d1 = _as_dict(oracle_lib.graph(h1.seq, h1.offsets, 9, 3, 5), 9)
+    d2 = _as_dict(oracle_lib.graph(h2.seq, h2.offsets, 9, 3, 5), 9)
+    da = _as_dict(a, 9)
+    for v, e in da.items():
+        e1 = d1.get(v, [0, [0] * 4, [0] * 4, e[3]])
+        e2 = d2.get(v, [0, [0] * 4, [0] * 4, e[3]])
+        assert e[0] == e1[0] + e2[0]
+        assert e[1] == [x + y for x, y in zip(e1[1], e2[1])]
+        assert e[2] == [x + y for x, y in zip(e1[2], e2[2])]
+
+
+def test_special_case_P_equals_K(oracle_lib):
+    """P = K (L1101-1103): every superkmer holds one K-mer on random reads."""
+    rs = random_reads(50, 100, 100, seed=61)
+    sk = oracle_lib.msp(rs.seq, rs.offsets, 31, 31, 8)
+    assert len(sk) == 50 * 70 and set(sk["n_kmers"].tolist()) == {1}
+
+
+def test_superkmers_cover_all_kmers(oracle_lib):
+    rs = _tiny_erroneous().subset(0, 300)
+    sk = oracle_lib.msp(rs.seq, rs.offsets, 31, 11, 16)
+    assert int(sk["n_kmers"].sum()) == rs.n_kmers(31)
+    # Def. 2 with reading G: consecutive superkmers of a read have different minimizers
+    same_read = sk["read"][1:] == sk["read"][:-1]
+    assert np.all(sk["minimizer"][1:][same_read] != sk["minimizer"][:-1][same_read])
+    # average superkmer length near the SURVEY.md simulation (8.85 K-mers, K=31 P=11)
+    assert 7.0 < rs.n_kmers(31) / len(sk) < 11.0
+
+
+def test_edge_cases_short_reads(oracle_lib):
+    """Reading N: L<K gives nothing, L=K one vertex without edges; empty input."""
+    rs = _readset(["ACG", "ACGTA", "", "TTTTT"])
+    d = _as_dict(oracle_lib.graph(rs.seq, rs.offsets, 5, 2, 3), 5)
+    assert d["ACGTA"][:3] == [1, [0] * 4, [0] * 4]
+    assert d["AAAAA"][:3] == [1, [0] * 4, [0] * 4]
+    assert len(d) == 2
+    empty = oracle_lib.graph(np.zeros(0, np.uint8), np.zeros(1, np.uint64), 5, 2, 3)
+    assert len(empty) == 0
+
+
+def test_unknown_bases_become_A(oracle_lib):
+    """L205-206: unknown bases -> A; lower case as upper (reading B)."""
+    a = _readset(["ACGNNTRYacgt"])
+    b = _readset(["ACGAATAAACGT"])
+    ga = oracle_lib.graph(a.seq, a.offsets, 5, 3, 4)
+    gb = oracle_lib.graph(b.seq, b.offsets, 5, 3, 4)
+    assert ga.tobytes() == gb.tobytes()
+
+
+def test_checksum_order_independent(oracle_lib):
+    rs = random_reads(50, 30, 60, seed=71)
+    r = oracle_lib.graph(rs.seq, rs.offsets, 11, 5, 4)
+    c = oracle_lib.checksum(r)
+    assert c == oracle_lib.checksum(r[::-1].copy())
+    r2 = r.copy()
+    r2["out"][0, 0] += 1
+    assert oracle_lib.checksum(r2) != c
+    # fmix64 (reading I) agrees with the string-side twin; the partition function is a free
+    # choice (reading I), so this is consistency, not a pin -- placement is pinned by I4.
+    for x in (0, 1, 2, 0xDEADBEEF, (1 << 64) - 1):
+        assert oracle_lib.fmix64(x) == brute.fmix64(x)
+    assert brute.fmix64(0) == 0
