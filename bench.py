@@ -1,0 +1,325 @@
+#!/usr/bin/env python
+"""Benchmark of the ParaHash hot path on B200: K-mers hashed per second (graph build, device-timed).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config ecoli] [--impl ours|reference]
+
+One step = one pass of the whole hot path over the synthetic read set
+of the chosen configuration: MSP count pass -> size readback -> MSP emit pass -> table plan ->
+table zero-fill -> hash build.  Extraction (a7) is timed separately (``extract_ms``) and is part of
+the ``e2e`` number, which also includes the H2D of the packed reads and the D2H of the stats.
+
+Prints ONE JSON line (rank 0).  See DESIGN.md Sec. 7 for the roofline arithmetic.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "K-mers hashed/sec (graph build, device-timed) at 1/2/4/8 B200; HBM roofline %"
+UNIT = "kmers/s"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        return False
+
+    def summary(self):
+        rows = [r for r in self.rows if len(r) >= 8]
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[4 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def _workload(args):
+    from synth import make_config
+
+    t = time.time()
+    rs = make_config(args.config, scale=args.scale, num_partitions=args.np)
+    return rs, time.time() - t
+
+
+def _config_json(rs, args, extra=None):
+    c = {"workload": rs.name, "genome_bp": rs.meta["genome"], "reads": rs.n_reads,
+         "read_len": rs.meta["read_len"], "error_rate": rs.meta["error"], "k": rs.k, "p": rs.p,
+         "num_partitions": rs.num_partitions, "lambda": args.lam, "alpha": args.alpha,
+         "kmers_per_step": rs.n_kmers(), "scale": args.scale,
+         "l2": "flushed between timed steps (512 MiB write); step working set > L2",
+         "parallelism": f"partitions sharded over {args.gpus} GPU(s)"}
+    if extra:
+        c.update(extra)
+    return c
+
+
+# ------------------------------------------------------------------------------- oracle arm
+def _oracle_rate(rs, seconds: float, threads: int):
+    """Times the oracle (as it stands) on a bounded prefix of the workload's reads."""
+    import oracle
+
+    oracle.build()
+    n = min(rs.n_reads, 2000)
+    t = time.time()
+    sub = rs.subset(0, n)
+    oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
+    dt = max(time.time() - t, 1e-3)
+    rate = sub.n_kmers() / dt
+    n2 = int(min(rs.n_reads, max(n, n * seconds / dt)))
+    sub = rs.subset(0, n2)
+    t = time.time()
+    oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
+    dt = time.time() - t
+    return sub.n_kmers() / dt, sub, dt
+
+
+def run_reference(args):
+    ws, rank, _ = _dist()
+    if rank != 0:
+        return 0
+    rs, _ = _workload(args)
+    threads = os.cpu_count() or 1
+    import oracle
+
+    oracle.build()
+    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    _, sub, _ = _oracle_rate(rs, per_step, threads)
+    for _ in range(args.warmup):
+        oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
+    times = []
+    for _ in range(args.steps):
+        t = time.time()
+        oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
+        times.append(time.time() - t)
+    total = sum(times)
+    value = sub.n_kmers() * args.steps / total
+    sample = f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers) per step"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic", "config": _config_json(rs, args),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------- our arm
+def run_ours(args):
+    import torch
+
+    ws, rank, local = _dist()
+    if ws > 1:
+        from paper_conf_icdcs_qiul17_b200 import multi
+
+        return multi.bench_main(args, METRIC, UNIT)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    from paper_conf_icdcs_qiul17_b200 import DbgBuilder, encode_reads, _lib
+
+    rs, gen_s = _workload(args)
+    packed = encode_reads(rs.seq, pin=True)
+    offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
+    n_kmers = rs.n_kmers()
+    stream = torch.cuda.current_stream(dev)
+    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget)
+    d_bases, d_off = b.upload(packed, offsets, stream)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+
+    def step(ev):
+        """One pass of rows a2-a6 (plus extraction when the tables are processed in batches)."""
+        ev["start"].record(stream)
+        b.msp(d_bases, d_off, stream)
+        ev["msp_end"].record(stream)
+        batches = b.plan(stream)
+        multi = len(batches) > 1
+        if multi:
+            b.reset_output(n_kmers // 2 + 1, stream)
+        for (lo, hi) in batches:
+            b.hash_batch(lo, hi, stream)  # zero-fill + hash_build_kernel
+            if multi:
+                b.extract_batch(lo, hi, stream)
+        ev["end"].record(stream)
+        return batches
+
+    for _ in range(args.warmup):
+        step({"start": E(), "msp_end": E(), "end": E()})
+    torch.cuda.synchronize()
+    b.hash_timer = []
+
+    step_ms, msp_ms = [], []
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            flush.zero_()
+            ev = {"start": E(), "msp_end": E(), "end": E()}
+            torch.cuda.synchronize()
+            batches = step(ev)
+            torch.cuda.synchronize()
+            step_ms.append(ev["start"].elapsed_time(ev["end"]))
+            msp_ms.append(ev["start"].elapsed_time(ev["msp_end"]))
+    hev = b.hash_timer
+    b.hash_timer = None
+    hash_ms_per_step = [sum(a.elapsed_time(c) for a, c in hev[i * len(batches):(i + 1) * len(batches)])
+                        for i in range(args.steps)]
+
+    # extraction (a7) + stats, timed separately; also validates invariants I1/I2
+    single = len(batches) == 1
+    x0, x1 = E(), E()
+    if single:
+        b.reset_output(max(1, n_kmers // 2), stream)
+        x0.record(stream)
+        b.extract_batch(0, rs.num_partitions, stream)
+        x1.record(stream)
+    st = _lib.dbg_sync_status(b.d_status, stream)
+    extract_ms = x0.elapsed_time(x1) if single else None
+    stats = b.stats()
+    L = rs.lengths()
+    inv_ok = (st == 0 and stats["sum_count"] == n_kmers
+              and stats["sum_edges"] == 2 * int(np.maximum(L - rs.k, 0).sum()))
+
+    # e2e through the public API: H2D of the packed reads (pinned) + path + extract + D2H stats
+    e2e_ms = []
+    for _ in range(max(1, min(args.steps, 5))):
+        flush.zero_()
+        torch.cuda.synchronize()
+        e0, e1 = E(), E()
+        e0.record(stream)
+        db, do = b.upload(packed, offsets, stream)
+        b.msp(db, do, stream)
+        bt = b.plan(stream)
+        b.reset_output(max(1, n_kmers // 2), stream)
+        for (lo, hi) in bt:
+            b.hash_batch(lo, hi, stream)
+            b.extract_batch(lo, hi, stream)
+        host_stats = b.d_stats.to("cpu", non_blocking=False)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms.append(e0.elapsed_time(e1))
+    h2d = packed.numel() * 8 + offsets.numel() * 8
+    d2h = 32 + 16 * rs.num_partitions
+
+    ms = statistics.mean(step_ms)
+    hash_ms = statistics.mean(hash_ms_per_step)
+    n_records = int(b.part_records.sum())
+    alg_bytes = n_kmers * 64 + n_records * 4 * b.rec_words
+    peak, peak_kind = _peaks()
+    achieved = alg_bytes / (hash_ms * 1e-3) / 1e9
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            traffic = json.load(f).get(rs.name, {}).get("hash_build_dram_bytes")
+    except Exception:
+        pass
+    cpu = None
+    if not args.no_cpu_baseline:
+        threads = os.cpu_count() or 1
+        rate, sub, dt = _oracle_rate(rs, args.cpu_seconds, threads)
+        cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
+               "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
+    line = {
+        "metric": METRIC, "value": n_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": _config_json(rs, args, {"batches": len(batches)}),
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "kernel": "hash_build_kernel",
+                     "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
+                     "hash_kmers_per_s": n_kmers / (hash_ms * 1e-3)},
+        "cpu_baseline": cpu,
+        "e2e": {"value": n_kmers / (statistics.mean(e2e_ms) * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h, "ms": statistics.mean(e2e_ms)},
+        "gpu_launches": args.steps * (4 + len(batches) * (2 if len(batches) > 1 else 1)),
+        "clocks": clk.summary(),
+        "breakdown_ms": {"msp": statistics.mean(msp_ms), "hash_build": hash_ms,
+                         "plan_fill_other": ms - statistics.mean(msp_ms) - hash_ms, "extract": extract_ms},
+        "stats": stats, "invariants_ok": bool(inv_ok), "gen_s": gen_s,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="ecoli")
+    ap.add_argument("--scale", type=float, default=1.0)
+    ap.add_argument("--np", type=int, default=None, help="override the number of partitions")
+    ap.add_argument("--lam", type=float, default=2.0)
+    ap.add_argument("--alpha", type=float, default=0.5)
+    ap.add_argument("--table-budget", type=int, default=None)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

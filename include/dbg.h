@@ -1,0 +1,174 @@
+/*
+ * dbg.h -- C ABI of the B200 hot path of ParaHash (Qiu & Luo, ICDCS 2017):
+ * MSP partitioning of reads into superkmer partitions, then one shared
+ * open-addressing hash table of <canonical K-mer, in/out edge multiplicities>
+ * per partition.  Citations "P:L<a>-<b>" are lines of the paper text
+ * (PAPER.md); readings A..T are listed in DESIGN.md Sec. 2.
+ *
+ * Conventions (all calls):
+ *  - The library never allocates or frees device memory: the caller (the
+ *    Python binding uses PyTorch tensors) owns every buffer and passes device
+ *    pointers ("d_" prefix) or host pointers ("h_" prefix).
+ *  - Device calls are stream-ordered and asynchronous; they validate their
+ *    arguments on the host and return before any launch on error.  Launch
+ *    failures return DBG_ECUDA.  Device-side conditions (table overflow,
+ *    output overflow) are recorded in a caller-owned uint32 status word and
+ *    reported by dbg_sync_status, the only call that synchronizes.
+ *  - Thread-safe across distinct buffers; one host thread per device.
+ *  - K must be odd (reading C), 1 <= K <= 63; 1 <= P <= min(K, 31);
+ *    1 <= num_partitions <= 4,194,303.  Reads shorter than K contribute
+ *    nothing and are not an error (reading N).
+ */
+#ifndef PARAHASH_DBG_H
+#define PARAHASH_DBG_H
+
+#include <stdint.h>
+#include <cuda_runtime_api.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define DBG_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define DBG_API __attribute__((visibility("default")))
+#else
+#define DBG_API
+#endif
+
+typedef enum {
+  DBG_OK = 0,
+  DBG_EINVAL = 1,      /* invalid argument (nothing launched) */
+  DBG_ENOSPACE = 2,    /* output buffer too small (count still written) */
+  DBG_ETABLEFULL = 3,  /* a probe sequence wrapped: table unusable, rebuild larger (reading O) */
+  DBG_ECUDA = 4        /* CUDA launch / runtime error */
+} dbg_status;
+
+/* Parameters of Sec. IV-A and Sec. V-A. */
+typedef struct {
+  int32_t k;              /* K-mer length, odd, 1..63 (reading C, T) */
+  int32_t p;              /* minimizer length P, 1..min(k,31) (Def. 1) */
+  int32_t num_partitions; /* NP, number of superkmer partitions (Sec. III-B) */
+  float lambda;           /* average errors per read (Property 1); default 2 */
+  float alpha;            /* load ratio; default 0.5 => capacity = N^i_kmer */
+} dbg_params;
+
+/* One vertex of Definition 3: the canonical K-mer (the
+ * lexicographically smaller of a K-mer and its reverse complement,
+ * P:L197-201) as a 2K-bit code, first base most significant, split into two
+ * 64-bit halves (K <= 31: kmer_hi = 0); its multiplicity; and the
+ * multiplicities of its out- and in-edges indexed by the neighbour's extreme
+ * base A,C,G,T in the vertex's canonical orientation
+ * (reading J); pid = its MSP partition.  56 bytes. */
+typedef struct {
+  uint64_t kmer_hi, kmer_lo;
+  uint32_t count;
+  uint32_t out[4];
+  uint32_t in[4];
+  uint32_t pid;
+} dbg_vertex;
+
+/* Totals; checksum = sum over vertices of h, h = fmix64 chained over
+ * (kmer_hi, kmer_lo, count, out[0..3], in[0..3]). */
+typedef struct {
+  uint64_t distinct, sum_count, sum_edges, checksum;
+} dbg_stats;
+
+/* Superkmer partitions (Sec. III-A Fig. 3) resident in HBM.
+ * All arrays are device memory owned by the caller.  Records of partition i
+ * occupy record slots [d_record_offset[i], d_record_offset[i+1]) of
+ * d_records; one record is dbg_record_words() uint32 words:
+ *   word 0: n_kmers (bits 0-7) | has_left (bit 8) | has_right (bit 9) | pid (bits 10-31)
+ *   words 1..: the bases S[s-has_left .. e+K-1+has_right], 2-bit, 16 per word,
+ *              first base in the most significant bits (Sec. III-B).
+ * A superkmer longer than the record holds is stored as consecutive pieces,
+ * each with its own adjacency bases (the graph is unchanged). */
+typedef struct {
+  uint64_t* d_n_records;     /* [NP]   records per partition (count pass) */
+  uint64_t* d_n_kmers;       /* [NP]   N^i_kmer, K-mers per partition (count pass; sizes tables) */
+  uint64_t* d_record_offset; /* [NP+1] exclusive prefix sum of d_n_records (count pass) */
+  uint64_t* d_fill;          /* [NP]   emission cursors (emit pass; zeroed by the call) */
+  uint32_t* d_records;       /* record buffer, d_record_offset[NP] records; NULL => count pass */
+} dbg_partition_set;
+
+/* ---- sizes ------------------------------------------------------------ */
+DBG_API int dbg_abi_version(void);
+/* uint32 words per superkmer record for these params (4 for K <= 39, else 8). */
+DBG_API uint32_t dbg_record_words(const dbg_params* prm);
+/* K-mers a record holds at most. */
+DBG_API uint32_t dbg_record_max_kmers(const dbg_params* prm);
+/* Bytes per hash-table slot (64). */
+DBG_API uint32_t dbg_slot_bytes(const dbg_params* prm);
+/* Table capacity for a partition with n_kmers K-mers: ceil(lambda/(4 alpha) * n_kmers)
+ * (Sec. IV-A), at least 1 when n_kmers > 0 (Property 1 sizing). */
+DBG_API uint64_t dbg_table_capacity(const dbg_params* prm, uint64_t n_kmers);
+/* uint64 words of the packed 2-bit stream for n_bases bases, including one pad word. */
+DBG_API uint64_t dbg_packed_words(uint64_t n_bases);
+
+/* ---- a0: host encoder (Sec. II-A; Sec. III-B) ---- */
+/* seq: n_bases ASCII characters (all reads concatenated).  Writes
+ * dbg_packed_words(n_bases) words to h_words: base i at word i/32, bits
+ * 63-2(i%32) .. 62-2(i%32); A=0 C=1 G=2 T=3, anything else -> A (reading A, B). */
+DBG_API dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64_t* h_words);
+
+/* ---- a2-a4: Step 1, MSP (Sec. III-B; Defs. 1-2) ------------
+ * d_bases: packed stream (dbg_packed_words(total) words), d_offsets: [n_reads+1]
+ * base offsets of the reads in the stream.
+ * part->d_records == NULL: count pass -- zeroes and fills d_n_records, d_n_kmers
+ *   and d_record_offset (size query; the caller reads d_record_offset[NP],
+ *   allocates and calls again).
+ * part->d_records != NULL: emit pass -- requires d_record_offset from a count
+ *   pass over the same reads; zeroes d_fill and writes every record. */
+DBG_API dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
+                             const uint64_t* d_offsets, uint64_t n_reads,
+                             const dbg_partition_set* part, cudaStream_t stream);
+
+/* ---- a5: sizing (Property 1; Sec. IV-A) ----------------------
+ * d_table_offset[NP+1] = exclusive prefix sum of dbg_table_capacity(N^i_kmer)
+ * (in slots).  Tables of partitions [b, e) need d_table_offset[e]-d_table_offset[b]
+ * slots of dbg_slot_bytes each, zero-filled before dbg_hash_build (EMPTY = 0). */
+DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers,
+                          uint64_t* d_table_offset, cudaStream_t stream);
+
+/* ---- a6: Step 2, hash build (Sec. III-C; Sec. III-D)
+ * Inserts every K-mer occurrence of partitions [pid_begin, pid_end) into that
+ * partition's table: one insertion per distinct vertex (a 64- or 128-bit
+ * CAS claims an EMPTY slot), multiple updates (atomic adds on the edge
+ * counters).  Partition i's table starts at
+ *   (char*)d_slots + (d_table_offset[i] - slot_base) * dbg_slot_bytes().
+ * Overflow sets bit 0 of *d_status (reported by dbg_sync_status). */
+DBG_API dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                          int32_t pid_end, void* d_slots, const uint64_t* d_table_offset,
+                          uint64_t slot_base, uint32_t* d_status, cudaStream_t stream);
+
+/* ---- a7: output (Def. 3) -------------------------------------
+ * Compacts the occupied slots of partitions [pid_begin, pid_end) into
+ * d_out[*d_n_out ...] (appends; the caller zeroes *d_n_out and *d_stats
+ * once) and accumulates *d_stats.  Records beyond out_cap are dropped and
+ * set bit 1 of *d_status (DBG_ENOSPACE; *d_n_out still counts them).
+ * Record order is unspecified (reading S): use dbg_sort_vertices. */
+DBG_API dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_slots,
+                             const uint64_t* d_table_offset, uint64_t slot_base,
+                             int32_t pid_begin, int32_t pid_end, dbg_vertex* d_out,
+                             uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
+                             uint32_t* d_status, cudaStream_t stream);
+
+/* Sorts n vertices ascending by (kmer_hi, kmer_lo) (reading Q) from d_in to
+ * d_out (distinct buffers) using a caller workspace of
+ * dbg_sort_workspace_bytes(n) bytes. */
+DBG_API uint64_t dbg_sort_workspace_bytes(const dbg_params* prm, uint64_t n);
+DBG_API dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_in, dbg_vertex* d_out,
+                             uint64_t n, void* d_workspace, uint64_t workspace_bytes,
+                             cudaStream_t stream);
+
+/* Synchronizes the stream, then decodes *d_status: bit 0 -> DBG_ETABLEFULL,
+ * bit 1 -> DBG_ENOSPACE; also returns DBG_ECUDA on a sticky CUDA error. */
+DBG_API dbg_status dbg_sync_status(const uint32_t* d_status, cudaStream_t stream);
+
+DBG_API const char* dbg_status_string(dbg_status s);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PARAHASH_DBG_H */

@@ -77,6 +77,12 @@ def _load():
             ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(ctypes.c_void_p), u64p,
         ]
         lib.oracle_graph.restype = ctypes.c_int
+        lib.oracle_graph_filtered.argtypes = [
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_int,
+            ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+            ctypes.POINTER(ctypes.c_void_p), u64p,
+        ]
+        lib.oracle_graph_filtered.restype = ctypes.c_int
         lib.oracle_msp.argtypes = [
             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_int,
             ctypes.c_int, ctypes.POINTER(ctypes.c_void_p), u64p,
@@ -102,10 +108,12 @@ def _as_inputs(seq, offsets):
     return seq, offsets
 
 
-def graph(seq, offsets, k: int, p: int, num_partitions: int, n_threads: int = 1, pids=None):
+def graph(seq, offsets, k: int, p: int, num_partitions: int, n_threads: int = 1, pids=None,
+          keys=None):
     """Sorted vertex records (VERTEX_DTYPE) of the reads ``seq[offsets[r]:offsets[r+1]]``.
 
-    ``pids``: optional iterable of partition ids to keep (sampled parity).
+    ``pids``: optional iterable of partition ids to keep; ``keys``: optional
+    (hi, lo) uint64 pairs of canonical codes to keep (sampled parity at full size).
     """
     lib = _load()
     seq, offsets = _as_inputs(seq, offsets)
@@ -114,11 +122,17 @@ def graph(seq, offsets, k: int, p: int, num_partitions: int, n_threads: int = 1,
     if pids is not None:
         filt = np.zeros(num_partitions, dtype=np.uint8)
         filt[np.asarray(list(pids), dtype=np.int64)] = 1
+    kf = None
+    if keys is not None:
+        kf = np.ascontiguousarray(np.asarray(keys, dtype=np.uint64).reshape(-1, 2))
+        order = np.lexsort((kf[:, 1], kf[:, 0]))
+        kf = np.ascontiguousarray(kf[order])
     out = ctypes.c_void_p()
     n = ctypes.c_uint64()
-    rc = lib.oracle_graph(
+    rc = lib.oracle_graph_filtered(
         seq.ctypes.data if seq.size else None, offsets.ctypes.data, n_reads, k, p,
         num_partitions, n_threads, filt.ctypes.data if filt is not None else None,
+        kf.ctypes.data if kf is not None else None, 0 if kf is None else len(kf),
         ctypes.byref(out), ctypes.byref(n),
     )
     if rc != 0:

@@ -206,11 +206,15 @@ uint64_t oracle_kmer_minimizer(const char* kmer, int K, int P) {
 // The graph.  Returns 0 on success, 1 on invalid arguments, 2 if a vertex
 // was found in two partitions (violates Sec. III-B), 3 on OOM.
 // pid_filter: NULL for all partitions, else one byte per partition (nonzero =
-// keep); used for sampled parity at full size.  *out is malloc'ed; release it
-// with oracle_free.  Records are sorted ascending by the 2K-bit code (reading Q).
-int oracle_graph(const char* seq, const uint64_t* offs, uint64_t n_reads, int K,
-                 int P, int NP, int n_threads, const uint8_t* pid_filter,
-                 oracle_vertex** out, uint64_t* n_out) {
+// keep); key_filter: NULL, or n_keys canonical codes as (hi, lo) pairs sorted
+// ascending -- only those vertices are counted.  Both are for sampled parity
+// at full size; they drop occurrences, never change the per-occurrence rule.
+// *out is malloc'ed; release it with oracle_free.  Records are sorted
+// ascending by the 2K-bit code (reading Q).
+int oracle_graph_filtered(const char* seq, const uint64_t* offs, uint64_t n_reads, int K,
+                          int P, int NP, int n_threads, const uint8_t* pid_filter,
+                          const uint64_t* key_filter, uint64_t n_keys,
+                          oracle_vertex** out, uint64_t* n_out) {
   *out = nullptr;
   *n_out = 0;
   if (K < 1 || K > 63 || P < 1 || P > K || P > 31 || NP < 1) return 1;
@@ -226,6 +230,20 @@ int oracle_graph(const char* seq, const uint64_t* offs, uint64_t n_reads, int K,
       std::string S = read_string(seq, offs, r);
       if (S.size() < (size_t)K) continue;  // reading N: no K-mers
       for (size_t i = 0; i + K <= S.size(); ++i) {
+        if (key_filter) {
+          std::string x = S.substr(i, K);
+          u128 fx = encode(x), ry = encode(reverse_complement(x));
+          u128 v = fx <= ry ? fx : ry;
+          uint64_t hi = (uint64_t)(v >> 64), lo = (uint64_t)v;
+          uint64_t a = 0, b = n_keys;  // binary search in the sorted (hi, lo) list
+          while (a < b) {
+            uint64_t m = (a + b) / 2;
+            uint64_t mh = key_filter[2 * m], ml = key_filter[2 * m + 1];
+            if (mh < hi || (mh == hi && ml < lo)) a = m + 1;
+            else b = m;
+          }
+          if (a == n_keys || key_filter[2 * a] != hi || key_filter[2 * a + 1] != lo) continue;
+        }
         uint32_t pid = partition_of(canonical_minimizer(S, i, K, P), NP);
         if (pid_filter && !pid_filter[pid]) continue;
         add_occurrence(S, i, K, maps[t][pid]);
@@ -279,6 +297,12 @@ int oracle_graph(const char* seq, const uint64_t* offs, uint64_t n_reads, int K,
   *out = v;
   *n_out = n;
   return 0;
+}
+
+int oracle_graph(const char* seq, const uint64_t* offs, uint64_t n_reads, int K, int P, int NP,
+                 int n_threads, const uint8_t* pid_filter, oracle_vertex** out, uint64_t* n_out) {
+  return oracle_graph_filtered(seq, offs, n_reads, K, P, NP, n_threads, pid_filter, nullptr, 0,
+                               out, n_out);
 }
 
 // MSP diagnostics (Sec. III-B): per read, the K-mers' canonical minimizers

@@ -1,0 +1,12 @@
+"""B200-native hot path of ParaHash (Qiu & Luo, ICDCS 2017): MSP partitioning + per-partition
+hash-table De Bruijn graph construction, behind the C ABI of include/dbg.h (libdbg.so, sm_100a).
+
+The Python layer only marshals arguments and owns device memory (PyTorch); there is no CPU
+fallback -- if libdbg.so is missing, calls raise.
+"""
+from . import _lib
+from ._lib import VERTEX_DTYPE, DbgError, load
+from .graph import DbgBuilder, GraphResult, build_graph, encode_reads
+
+__all__ = ["_lib", "VERTEX_DTYPE", "DbgError", "load", "DbgBuilder", "GraphResult", "build_graph",
+           "encode_reads"]

@@ -1,0 +1,199 @@
+"""ctypes binding of libdbg.so (include/dbg.h) -- argument marshalling only.
+
+Every function here has the name of the C entry point it calls and only turns
+torch tensors / numpy arrays into pointers; all work runs in libdbg.so.  The
+library is loaded from this package's lib/ directory (built in-tree by
+``paper_conf_icdcs_qiul17_b200.build``); if it is missing, loading fails
+loudly -- there is no fallback path.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "lib", "libdbg.so")
+
+DBG_OK, DBG_EINVAL, DBG_ENOSPACE, DBG_ETABLEFULL, DBG_ECUDA = range(5)
+
+
+class DbgError(RuntimeError):
+    def __init__(self, name: str, status: int, msg: str):
+        super().__init__(f"{name} failed: status {status} ({msg})")
+        self.status = status
+
+
+class dbg_params(ctypes.Structure):
+    _fields_ = [("k", ctypes.c_int32), ("p", ctypes.c_int32), ("num_partitions", ctypes.c_int32),
+                ("lambda_", ctypes.c_float), ("alpha", ctypes.c_float)]
+
+
+class dbg_partition_set(ctypes.Structure):
+    _fields_ = [("d_n_records", ctypes.c_void_p), ("d_n_kmers", ctypes.c_void_p),
+                ("d_record_offset", ctypes.c_void_p), ("d_fill", ctypes.c_void_p),
+                ("d_records", ctypes.c_void_p)]
+
+
+# dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
+VERTEX_DTYPE = np.dtype([("kmer_hi", "<u8"), ("kmer_lo", "<u8"), ("count", "<u4"),
+                         ("out", "<u4", (4,)), ("in", "<u4", (4,)), ("pid", "<u4")])
+STATS_FIELDS = ("distinct", "sum_count", "sum_edges", "checksum")
+assert VERTEX_DTYPE.itemsize == 56
+
+_P = ctypes.c_void_p
+_U64 = ctypes.c_uint64
+_I32 = ctypes.c_int32
+_PRM = ctypes.POINTER(dbg_params)
+_PART = ctypes.POINTER(dbg_partition_set)
+
+# name -> (restype, argtypes); mirrors include/dbg.h
+SIGNATURES = {
+    "dbg_abi_version": (ctypes.c_int, []),
+    "dbg_record_words": (ctypes.c_uint32, [_PRM]),
+    "dbg_record_max_kmers": (ctypes.c_uint32, [_PRM]),
+    "dbg_slot_bytes": (ctypes.c_uint32, [_PRM]),
+    "dbg_table_capacity": (_U64, [_PRM, _U64]),
+    "dbg_packed_words": (_U64, [_U64]),
+    "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
+    "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
+    "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P]),
+    "dbg_hash_build": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _U64, _P, _P]),
+    "dbg_extract_graph": (ctypes.c_int, [_PRM, _P, _P, _U64, _I32, _I32, _P, _U64, _P, _P, _P, _P]),
+    "dbg_sort_workspace_bytes": (_U64, [_PRM, _U64]),
+    "dbg_sort_vertices": (ctypes.c_int, [_PRM, _P, _P, _U64, _P, _U64, _P]),
+    "dbg_sync_status": (ctypes.c_int, [_P, _P]),
+    "dbg_status_string": (ctypes.c_char_p, [ctypes.c_int]),
+}
+
+_lib = None
+
+
+def load():
+    """Loads libdbg.so; raises if it has not been built."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run `python -m paper_conf_icdcs_qiul17_b200.build` "
+                              "(there is no CPU fallback)")
+        lib = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in SIGNATURES.items():
+            f = getattr(lib, name)
+            f.restype = res
+            f.argtypes = args
+        if lib.dbg_abi_version() != 1:
+            raise ImportError("libdbg.so ABI version mismatch")
+        _lib = lib
+    return _lib
+
+
+def _ptr(x) -> int | None:
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    raise TypeError(type(x))
+
+
+def _check(name: str, status: int):
+    if status != DBG_OK:
+        raise DbgError(name, status, load().dbg_status_string(status).decode())
+
+
+def _stream(stream) -> int | None:
+    if stream is None:
+        return None
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def params(k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5) -> dbg_params:
+    return dbg_params(k, p, num_partitions, lam, alpha)
+
+
+def partition_set(n_records, n_kmers, record_offset, fill, records=None) -> dbg_partition_set:
+    return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(records))
+
+
+# --------------------------------------------------------------------------- entry points
+
+
+def dbg_abi_version() -> int:
+    return load().dbg_abi_version()
+
+
+def dbg_record_words(prm: dbg_params) -> int:
+    return load().dbg_record_words(ctypes.byref(prm))
+
+
+def dbg_record_max_kmers(prm: dbg_params) -> int:
+    return load().dbg_record_max_kmers(ctypes.byref(prm))
+
+
+def dbg_slot_bytes(prm: dbg_params) -> int:
+    return load().dbg_slot_bytes(ctypes.byref(prm))
+
+
+def dbg_table_capacity(prm: dbg_params, n_kmers: int) -> int:
+    return load().dbg_table_capacity(ctypes.byref(prm), n_kmers)
+
+
+def dbg_packed_words(n_bases: int) -> int:
+    return load().dbg_packed_words(n_bases)
+
+
+def dbg_encode_ascii(seq, h_words) -> None:
+    """seq: uint8 ASCII array (numpy or CPU tensor); h_words: uint64 host buffer of
+    dbg_packed_words(len(seq)) words (numpy or pinned CPU tensor)."""
+    n = seq.numel() if hasattr(seq, "numel") else len(seq)
+    _check("dbg_encode_ascii", load().dbg_encode_ascii(_ptr(seq), n, _ptr(h_words)))
+
+
+def dbg_msp_partition(prm, d_bases, n_words: int, d_offsets, n_reads: int, part: dbg_partition_set,
+                      stream=None) -> None:
+    _check("dbg_msp_partition", load().dbg_msp_partition(
+        ctypes.byref(prm), _ptr(d_bases), n_words, _ptr(d_offsets), n_reads, ctypes.byref(part),
+        _stream(stream)))
+
+
+def dbg_table_plan(prm, d_n_kmers, d_table_offset, stream=None) -> None:
+    _check("dbg_table_plan", load().dbg_table_plan(ctypes.byref(prm), _ptr(d_n_kmers),
+                                                   _ptr(d_table_offset), _stream(stream)))
+
+
+def dbg_hash_build(prm, part, pid_begin: int, pid_end: int, d_slots, d_table_offset, slot_base: int,
+                   d_status, stream=None) -> None:
+    _check("dbg_hash_build", load().dbg_hash_build(
+        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_slots), _ptr(d_table_offset),
+        slot_base, _ptr(d_status), _stream(stream)))
+
+
+def dbg_extract_graph(prm, d_slots, d_table_offset, slot_base: int, pid_begin: int, pid_end: int,
+                      d_out, out_cap: int, d_n_out, d_stats, d_status, stream=None) -> None:
+    _check("dbg_extract_graph", load().dbg_extract_graph(
+        ctypes.byref(prm), _ptr(d_slots), _ptr(d_table_offset), slot_base, pid_begin, pid_end,
+        _ptr(d_out), out_cap, _ptr(d_n_out), _ptr(d_stats), _ptr(d_status), _stream(stream)))
+
+
+def dbg_sort_workspace_bytes(prm, n: int) -> int:
+    return load().dbg_sort_workspace_bytes(ctypes.byref(prm), n)
+
+
+def dbg_sort_vertices(prm, d_in, d_out, n: int, d_workspace, workspace_bytes: int, stream=None) -> None:
+    _check("dbg_sort_vertices", load().dbg_sort_vertices(
+        ctypes.byref(prm), _ptr(d_in), _ptr(d_out), n, _ptr(d_workspace), workspace_bytes,
+        _stream(stream)))
+
+
+def dbg_sync_status(d_status, stream=None) -> int:
+    return load().dbg_sync_status(_ptr(d_status), _stream(stream))
+
+
+def dbg_status_string(status: int) -> str:
+    return load().dbg_status_string(status).decode()

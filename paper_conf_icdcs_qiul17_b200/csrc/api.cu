@@ -1,0 +1,87 @@
+// api.cu -- host side of libdbg.so: sizes, the host 2-bit encoder (row a0) and
+// status handling.  See include/dbg.h for the contract of every entry point.
+#include <cmath>
+#include <cstring>
+
+#include "dbg_device.cuh"
+
+using namespace dbg;
+
+extern "C" int dbg_abi_version(void) { return DBG_ABI_VERSION; }
+
+extern "C" uint32_t dbg_record_words(const dbg_params* prm) {
+  return prm ? record_words(prm->k) : 0u;
+}
+
+extern "C" uint32_t dbg_record_max_kmers(const dbg_params* prm) {
+  return prm ? record_max_kmers(prm->k) : 0u;
+}
+
+extern "C" uint32_t dbg_slot_bytes(const dbg_params* prm) {
+  (void)prm;
+  return kSlotBytes;
+}
+
+// Sec. IV-A: "we use [N^i_kmer] with a load ratio alpha to set the
+// hash table size as lambda/(4 alpha) N^i_kmer"; lambda = 2, alpha = 0.5 by
+// default, which makes the capacity N^i_kmer (Table II).
+// The same double-precision expression runs on the device in dbg_table_plan.
+extern "C" uint64_t dbg_table_capacity(const dbg_params* prm, uint64_t n_kmers) {
+  if (!prm || n_kmers == 0 || !(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return 0;
+  const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
+  const double c = std::ceil(ratio * (double)n_kmers);
+  return c < 1.0 ? 1ull : (uint64_t)c;
+}
+
+extern "C" uint64_t dbg_packed_words(uint64_t n_bases) { return (n_bases + 31) / 32 + 1; }
+
+// Sec. II-A: characters are transformed into {A,C,G,T}, unknown
+// bases to A; Sec. III-B: 2 bits per base.
+extern "C" dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64_t* h_words) {
+  if (!h_words || (n_bases && !seq)) return DBG_EINVAL;
+  uint8_t lut[256];
+  memset(lut, 0, sizeof(lut));  // reading B: anything else -> A
+  lut['C'] = lut['c'] = 1;
+  lut['G'] = lut['g'] = 2;
+  lut['T'] = lut['t'] = 3;
+  const uint64_t nw = dbg_packed_words(n_bases);
+  const unsigned char* s = reinterpret_cast<const unsigned char*>(seq);
+  const uint64_t full = n_bases / 32;
+  for (uint64_t w = 0; w < full; ++w) {
+    uint64_t v = 0;
+    const unsigned char* p = s + 32 * w;
+    for (int t = 0; t < 32; ++t) v = (v << 2) | lut[p[t]];
+    h_words[w] = v;
+  }
+  for (uint64_t w = full; w < nw; ++w) {
+    uint64_t v = 0;
+    for (int t = 0; t < 32; ++t) {
+      const uint64_t i = 32 * w + t;
+      v = (v << 2) | (i < n_bases ? lut[s[i]] : 0u);
+    }
+    h_words[w] = v;
+  }
+  return DBG_OK;
+}
+
+extern "C" dbg_status dbg_sync_status(const uint32_t* d_status, cudaStream_t stream) {
+  if (!d_status) return DBG_EINVAL;
+  uint32_t h = 0;
+  if (cudaMemcpyAsync(&h, d_status, sizeof(h), cudaMemcpyDeviceToHost, stream) != cudaSuccess)
+    return DBG_ECUDA;
+  if (cudaStreamSynchronize(stream) != cudaSuccess) return DBG_ECUDA;
+  if (h & kStatusTableFull) return DBG_ETABLEFULL;
+  if (h & kStatusNoSpace) return DBG_ENOSPACE;
+  return DBG_OK;
+}
+
+extern "C" const char* dbg_status_string(dbg_status s) {
+  switch (s) {
+    case DBG_OK: return "ok";
+    case DBG_EINVAL: return "invalid argument";
+    case DBG_ENOSPACE: return "output buffer too small";
+    case DBG_ETABLEFULL: return "hash table full (probe sequence wrapped)";
+    case DBG_ECUDA: return "CUDA error";
+  }
+  return "unknown status";
+}

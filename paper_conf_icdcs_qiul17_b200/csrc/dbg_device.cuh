@@ -1,0 +1,60 @@
+// dbg_device.cuh -- device helpers shared by the sm_100a kernels of libdbg.so.
+// Product code: never includes or links anything under oracle/.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/dbg.h"
+
+namespace dbg {
+
+constexpr int kWarp = 32;
+constexpr uint32_t kFull = 0xffffffffu;
+constexpr uint32_t kSlotBytes = 64;     // one 64-B aligned slot = 2 sectors, 1/2 line
+constexpr uint32_t kMaxPid = (1u << 22) - 1;
+constexpr uint64_t kOccupied = 1ull << 63;
+
+// Status bits (dbg_sync_status).
+constexpr uint32_t kStatusTableFull = 1u;
+constexpr uint32_t kStatusNoSpace = 2u;
+
+// Record geometry (dbg.h): 4 words (48 bases) for K <= 39, else 8 (112 bases).
+__host__ __device__ inline uint32_t record_words(int k) { return k <= 39 ? 4u : 8u; }
+__host__ __device__ inline uint32_t record_max_kmers(int k) {
+  // bases = 16 * (R - 1) >= has_left + n + K - 1 + has_right
+  return 16u * (record_words(k) - 1u) - (uint32_t)k - 1u;
+}
+
+// MurmurHash3 64-bit finaliser: the partition function of reading I
+// ("superkmer ID ... from the minimizer's hash bit value with a modulo",
+// P:L455-459), and the slot hash of the tables.
+__host__ __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
+  k ^= k >> 33;
+  k *= 0xff51afd7ed558ccdULL;
+  k ^= k >> 33;
+  k *= 0xc4ceb9fe1a85ec53ULL;
+  k ^= k >> 33;
+  return k;
+}
+
+// Reverse complement of a P-mer held in the low 2P bits (reading A:
+// complement = 3 - c = c ^ 3; the 2-bit groups are reversed).
+__device__ __forceinline__ uint64_t revcomp64(uint64_t x, int p) {
+  uint64_t y = __brevll(~x);
+  y = ((y >> 1) & 0x5555555555555555ull) | ((y & 0x5555555555555555ull) << 1);
+  return y >> (64 - 2 * p);
+}
+
+// 64 bases starting at base position pos of the packed stream (MSB-first),
+// i.e. the bits that follow; positions past the end read as A.
+__device__ __forceinline__ uint64_t window64(const uint64_t* __restrict__ words, uint64_t n_words,
+                                             uint64_t pos) {
+  uint64_t wi = pos >> 5;
+  uint32_t sh = (uint32_t)(pos & 31) * 2;
+  uint64_t hi = wi < n_words ? __ldg(words + wi) : 0;
+  if (sh == 0) return hi;
+  uint64_t lo = wi + 1 < n_words ? __ldg(words + wi + 1) : 0;
+  return (hi << sh) | (lo >> (64 - sh));
+}
+
+}  // namespace dbg

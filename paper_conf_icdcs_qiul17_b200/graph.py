@@ -1,0 +1,243 @@
+"""Host orchestration of the hot path over the C ABI (include/dbg.h).
+
+PyTorch provides device memory and the stream; every step of the path runs in
+libdbg.so kernels:
+
+    a0  encode_reads         dbg_encode_ascii (host C)
+    a1  DbgBuilder.upload    H2D copy of the packed reads
+    a2-a4 DbgBuilder.msp     dbg_msp_partition (count pass -> sizes -> emit pass)
+    a5  DbgBuilder.plan      dbg_table_plan (lambda/(4 alpha) N^i_kmer)
+    a5-a6 DbgBuilder.hash    zero-fill + dbg_hash_build, batch by batch
+    a7  DbgBuilder.extract   dbg_extract_graph (+ dbg_sort_vertices)
+
+Partitions are processed in batches of consecutive partition ids whose tables
+fit ``table_budget_bytes`` (the paper's "one partition at a time", P:L359-367,
+generalised to as many partitions as HBM holds); each batch is extracted before
+its table memory is reused.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import VERTEX_DTYPE, STATS_FIELDS
+
+
+def encode_reads(seq: np.ndarray, pin: bool = False) -> torch.Tensor:
+    """Row a0: ASCII reads (concatenated) -> packed 2-bit words (uint64 as int64 tensor)."""
+    seq = np.ascontiguousarray(seq, dtype=np.uint8)
+    n_words = _lib.dbg_packed_words(len(seq))
+    out = torch.empty(n_words, dtype=torch.int64, pin_memory=pin)
+    _lib.dbg_encode_ascii(seq, out.data_ptr())
+    return out
+
+
+@dataclass
+class GraphResult:
+    vertices: np.ndarray | None          # VERTEX_DTYPE records (sorted if requested), or None
+    n_vertices: int
+    stats: dict
+    n_kmers: int
+    part_kmers: np.ndarray
+    part_records: np.ndarray
+    batches: list = field(default_factory=list)
+
+
+class DbgBuilder:
+    """Reusable buffers + the call sequence of the path for one (K, P, NP) setting."""
+
+    def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
+                 device: str | torch.device = "cuda", table_budget_bytes: int | None = None):
+        if k % 2 == 0 or not 1 <= k <= 63:
+            raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
+        if not 1 <= p <= min(k, 31):
+            raise ValueError("P must be in 1..min(K, 31)")
+        self.k, self.p, self.np = k, p, num_partitions
+        self.prm = _lib.params(k, p, num_partitions, lam, alpha)
+        self.device = torch.device(device)
+        _lib.load()
+        self.rec_words = _lib.dbg_record_words(self.prm)
+        self.slot_bytes = _lib.dbg_slot_bytes(self.prm)
+        dev = self.device
+        NP = num_partitions
+        self.d_n_records = torch.zeros(NP, dtype=torch.int64, device=dev)
+        self.d_n_kmers = torch.zeros(NP, dtype=torch.int64, device=dev)
+        self.d_rec_off = torch.zeros(NP + 1, dtype=torch.int64, device=dev)
+        self.d_fill = torch.zeros(NP, dtype=torch.int64, device=dev)
+        self.d_tab_off = torch.zeros(NP + 1, dtype=torch.int64, device=dev)
+        self.d_status = torch.zeros(1, dtype=torch.int32, device=dev)
+        self.d_n_out = torch.zeros(1, dtype=torch.int64, device=dev)
+        self.d_stats = torch.zeros(4, dtype=torch.int64, device=dev)
+        self.records = torch.empty(0, dtype=torch.int32, device=dev)
+        self.slots = torch.empty(0, dtype=torch.uint8, device=dev)
+        self.out = torch.empty(0, dtype=torch.uint8, device=dev)
+        self.table_budget_bytes = table_budget_bytes
+        self.part_kmers = np.zeros(NP, dtype=np.int64)
+        self.part_records = np.zeros(NP, dtype=np.int64)
+        self.tab_host = np.zeros(NP + 1, dtype=np.int64)
+        self.batches: list[tuple[int, int]] = []
+        self._caps_key = None
+        self._caps = None
+        self.hash_timer: list | None = None  # if a list: (start, end) CUDA events per hash launch
+
+    # ------------------------------------------------------------------ a1
+    def upload(self, packed: torch.Tensor, offsets: np.ndarray | torch.Tensor, stream=None):
+        """H2D of the packed reads and base offsets (row a1)."""
+        if not isinstance(offsets, torch.Tensor):
+            offsets = torch.from_numpy(np.ascontiguousarray(offsets, dtype=np.uint64).view(np.int64))
+        with torch.cuda.stream(stream) if stream is not None else _null():
+            d_bases = packed.to(self.device, non_blocking=True)
+            d_offsets = offsets.to(self.device, non_blocking=True)
+        return d_bases, d_offsets
+
+    # ------------------------------------------------------------------ a2-a4
+    def part_set(self, with_records: bool) -> _lib.dbg_partition_set:
+        return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill,
+                                  self.records if with_records else None)
+
+    def msp(self, d_bases: torch.Tensor, d_offsets: torch.Tensor, stream=None) -> None:
+        stream = stream or torch.cuda.current_stream(self.device)
+        n_reads = d_offsets.numel() - 1
+        n_words = d_bases.numel()
+        _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(False), stream)
+        with torch.cuda.stream(stream):
+            sizes = torch.cat([self.d_n_records, self.d_n_kmers]).cpu()  # the one size readback
+        sizes = sizes.numpy()
+        self.part_records = sizes[:self.np].copy()
+        self.part_kmers = sizes[self.np:].copy()
+        total = int(self.part_records.sum())
+        need = total * self.rec_words
+        if self.records.numel() < need:
+            self.records = torch.empty(int(need * 1.05) + 16, dtype=torch.int32, device=self.device)
+        _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
+
+    # ------------------------------------------------------------------ a5
+    def plan(self, stream=None) -> list[tuple[int, int]]:
+        stream = stream or torch.cuda.current_stream(self.device)
+        _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, stream)
+        key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha)
+        if self._caps_key != key:  # host copy of the same C sizing function (dbg_table_capacity)
+            self._caps = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in self.part_kmers],
+                                  dtype=np.int64)
+            self._caps_key = key
+        caps = self._caps
+        self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
+        self.tab_host[1:] = np.cumsum(caps)
+        budget = self.table_budget_bytes
+        if budget is None:
+            free, _ = torch.cuda.mem_get_info(self.device)
+            budget = max(int(free * 0.6), 1 << 26)
+        max_slots = max(budget // self.slot_bytes, int(caps.max(initial=0)))
+        batches, b = [], 0
+        while b < self.np:
+            e = b + 1
+            while e < self.np and self.tab_host[e + 1] - self.tab_host[b] <= max_slots:
+                e += 1
+            batches.append((b, e))
+            b = e
+        self.batches = batches
+        need = max((self.tab_host[e] - self.tab_host[b] for b, e in batches), default=0) * self.slot_bytes
+        if self.slots.numel() < need:
+            self.slots = torch.empty(0, dtype=torch.uint8, device=self.device)
+            self.slots = torch.empty(int(need), dtype=torch.uint8, device=self.device)
+        return batches
+
+    # ------------------------------------------------------------------ a5-a6
+    def hash_batch(self, b: int, e: int, stream=None) -> None:
+        stream = stream or torch.cuda.current_stream(self.device)
+        n_slots = int(self.tab_host[e] - self.tab_host[b])
+        with torch.cuda.stream(stream):
+            self.slots[: n_slots * self.slot_bytes].zero_()  # EMPTY = 0 (hash.cu slot layout)
+        if self.hash_timer is not None:
+            ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+            ev[0].record(stream)
+        _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.slots, self.d_tab_off,
+                            int(self.tab_host[b]), self.d_status, stream)
+        if self.hash_timer is not None:
+            ev[1].record(stream)
+            self.hash_timer.append(ev)
+
+    # ------------------------------------------------------------------ a7
+    def reset_output(self, cap: int, stream=None) -> None:
+        with torch.cuda.stream(stream or torch.cuda.current_stream(self.device)):
+            self.d_n_out.zero_()
+            self.d_stats.zero_()
+            self.d_status.zero_()
+        if self.out.numel() < cap * VERTEX_DTYPE.itemsize:
+            self.out = torch.empty(cap * VERTEX_DTYPE.itemsize, dtype=torch.uint8, device=self.device)
+
+    def extract_batch(self, b: int, e: int, stream=None) -> None:
+        stream = stream or torch.cuda.current_stream(self.device)
+        cap = self.out.numel() // VERTEX_DTYPE.itemsize
+        _lib.dbg_extract_graph(self.prm, self.slots, self.d_tab_off, int(self.tab_host[b]), b, e, self.out,
+                               cap, self.d_n_out, self.d_stats, self.d_status, stream)
+
+    def stats(self) -> dict:
+        s = self.d_stats.cpu().numpy().view(np.uint64)
+        return {f: int(v) for f, v in zip(STATS_FIELDS, s)}
+
+    def vertices(self, sort: bool = True, stream=None) -> np.ndarray:
+        """D2H of the compacted records (sorted on the device by dbg_sort_vertices)."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        n = int(self.d_n_out.item())
+        nbytes = n * VERTEX_DTYPE.itemsize
+        src = self.out[:nbytes]
+        if sort and n:
+            dst = torch.empty(nbytes, dtype=torch.uint8, device=self.device)
+            wsb = _lib.dbg_sort_workspace_bytes(self.prm, n)
+            ws = torch.empty(wsb, dtype=torch.uint8, device=self.device)
+            _lib.dbg_sort_vertices(self.prm, src, dst, n, ws, wsb, stream)
+            src = dst
+        return src.cpu().numpy().view(VERTEX_DTYPE)
+
+    # ------------------------------------------------------------------ whole path
+    def build(self, d_bases, d_offsets, stream=None, out_cap: int | None = None,
+              want_vertices: bool = True, sort: bool = True) -> GraphResult:
+        stream = stream or torch.cuda.current_stream(self.device)
+        self.msp(d_bases, d_offsets, stream)
+        batches = self.plan(stream)
+        n_kmers = int(self.part_kmers.sum())
+        cap = out_cap if out_cap is not None else n_kmers
+        while True:
+            self.reset_output(cap, stream)
+            cap = self.out.numel() // VERTEX_DTYPE.itemsize
+            for b, e in batches:
+                self.hash_batch(b, e, stream)
+                self.extract_batch(b, e, stream)
+            st = _lib.dbg_sync_status(self.d_status, stream)
+            if st == _lib.DBG_ENOSPACE:
+                cap = int(self.d_n_out.item())
+                continue
+            if st == _lib.DBG_ETABLEFULL:  # reading O: rebuild at capacity N^i_kmer
+                if self.prm.lambda_ / (4 * self.prm.alpha) >= 1.0:
+                    raise _lib.DbgError("dbg_hash_build", st, "table full at capacity >= N^i_kmer")
+                self.prm = _lib.params(self.k, self.p, self.np, 2.0, 0.5)
+                batches = self.plan(stream)
+                continue
+            if st != _lib.DBG_OK:
+                raise _lib.DbgError("dbg_sync_status", st, _lib.dbg_status_string(st))
+            break
+        verts = self.vertices(sort=sort, stream=stream) if want_vertices else None
+        return GraphResult(verts, int(self.d_n_out.item()), self.stats(), n_kmers, self.part_kmers.copy(),
+                           self.part_records.copy(), list(batches))
+
+
+class _null:
+    def __enter__(self):
+        return None
+
+    def __exit__(self, *a):
+        return False
+
+
+def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
+                lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
+                table_budget_bytes: int | None = None) -> GraphResult:
+    """ASCII reads -> De Bruijn graph records (the public one-call API)."""
+    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes)
+    packed = encode_reads(seq)
+    d_bases, d_offsets = builder.upload(packed, offsets)
+    return builder.build(d_bases, d_offsets, sort=sort)

@@ -1,0 +1,115 @@
+"""C-ABI library (libdbg.so): loads, exports every symbol include/dbg.h declares, and its host-only
+entry points behave (no GPU needed: no compute call launches a kernel here)."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+GOLD = os.path.join(ROOT, "tests", "golden")
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_icdcs_qiul17_b200 import build
+
+    build.build()
+    from paper_conf_icdcs_qiul17_b200 import _lib
+
+    _lib.load()
+    return _lib
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "dbg.h")).read()
+    return re.findall(r"DBG_API\s+[\w\s\*]+?\b(dbg_\w+)\s*\(", src)
+
+
+def test_exports_every_declared_symbol(lib):
+    names = _declared()
+    assert len(names) == 15
+    raw = lib.load()
+    for n in names:
+        assert hasattr(raw, n), n
+        assert n in lib.SIGNATURES, n
+
+
+def test_abi_and_sizes(lib):
+    assert lib.dbg_abi_version() == 1
+    p31 = lib.params(31, 11, 16)
+    p63 = lib.params(63, 19, 16)
+    assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
+    assert lib.dbg_record_words(p63) == 8 and lib.dbg_record_max_kmers(p63) == 48
+    assert lib.dbg_slot_bytes(p31) == 64
+    assert lib.dbg_packed_words(0) == 1 and lib.dbg_packed_words(32) == 2 and lib.dbg_packed_words(33) == 3
+
+
+def test_table2_sizing_pin(lib):
+    """Table II (L1005-1013): with lambda=2, alpha=0.5 the capacity is N^i_kmer, so at the 32 B per
+    entry of L1242 the max table per partition is 32 B x (2725 M / NP) within 7 %."""
+    prm = lib.params(27, 11, 16, 2.0, 0.5)
+    for l in open(os.path.join(GOLD, "table1_table2.txt")):
+        f = l.split()
+        if f and f[0] == "TABLE2":
+            np_, kmers_m, size_mb = int(f[1]), float(f[2]), float(f[3])
+            n_i = int(2725e6 / np_)
+            assert abs(n_i / 1e6 - kmers_m) <= 0.5 + 0.01 * kmers_m
+            cap = lib.dbg_table_capacity(prm, n_i)
+            assert cap == n_i
+            assert abs(cap * 32 / 1e6 - size_mb) / size_mb < 0.07
+    # lambda/(4 alpha) scaling (L783-788)
+    assert lib.dbg_table_capacity(lib.params(31, 11, 16, 2.0, 0.8), 1000) == 625
+    assert lib.dbg_table_capacity(lib.params(31, 11, 16, 1.0, 0.5), 1001) == 501
+    assert lib.dbg_table_capacity(prm, 0) == 0
+    assert lib.dbg_table_capacity(lib.params(31, 11, 16, 0.001, 0.5), 10) == 1
+
+
+def test_encoder_fig4_and_rules(lib):
+    """Fig. 4 (L598-606) bits; unknown -> A and lower case (L205-206)."""
+    lines = dict(l.split() for l in open(os.path.join(GOLD, "fig4_encoding.txt")) if l.strip() and l[0] != "#")
+    seq = np.frombuffer(lines["KMER"].encode(), dtype=np.uint8)
+    out = np.zeros(lib.dbg_packed_words(len(seq)), dtype=np.uint64)
+    lib.dbg_encode_ascii(seq, out)
+    assert int(out[0]) >> 48 == int(lines["BITS"], 2)
+    s = np.frombuffer(b"acgtNRYX" * 5, dtype=np.uint8)
+    o1 = np.zeros(lib.dbg_packed_words(len(s)), dtype=np.uint64)
+    lib.dbg_encode_ascii(s, o1)
+    t = np.frombuffer(b"ACGTAAAA" * 5, dtype=np.uint8)
+    o2 = np.zeros(lib.dbg_packed_words(len(t)), dtype=np.uint64)
+    lib.dbg_encode_ascii(t, o2)
+    assert (o1 == o2).all()
+    # base i at word i/32, most significant first; pad word zero
+    rng = np.random.default_rng(0)
+    codes = rng.integers(0, 4, 1000)
+    seq = np.frombuffer(b"ACGT", dtype=np.uint8)[codes]
+    w = np.zeros(lib.dbg_packed_words(1000), dtype=np.uint64)
+    lib.dbg_encode_ascii(seq, w)
+    for i in range(0, 1000, 7):
+        assert (int(w[i // 32]) >> (62 - 2 * (i % 32))) & 3 == codes[i]
+    assert int(w[-1]) == 0
+
+
+def test_invalid_arguments_return_before_launch(lib):
+    from paper_conf_icdcs_qiul17_b200._lib import DbgError, partition_set
+
+    part = partition_set(1, 1, 1, 1, None)
+    for prm in (lib.params(30, 11, 16), lib.params(31, 0, 16), lib.params(31, 32, 16), lib.params(31, 11, 0),
+                lib.params(65, 11, 16)):
+        with pytest.raises(DbgError) as e:
+            lib.dbg_msp_partition(prm, 1, 1, 1, 1, part, None)
+        assert e.value.status == lib.DBG_EINVAL
+    with pytest.raises(DbgError):
+        lib.dbg_hash_build(lib.params(31, 11, 16), part, 5, 2, 1, 1, 0, 1, None)
+    assert lib.dbg_status_string(lib.DBG_ETABLEFULL).startswith("hash table full")
+
+
+def test_product_has_no_oracle_dependency():
+    """The product package never imports, loads or calls anything under oracle/ (DESIGN.md Sec. 3)."""
+    pkg = os.path.join(ROOT, "paper_conf_icdcs_qiul17_b200")
+    bad = re.compile(r"(import\s+oracle|from\s+oracle|liboracle|oracle_\w+\s*\(|oracle/\w+\.(cpp|py))")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                src = open(os.path.join(dirpath, f)).read()
+                assert not bad.search(src), f

@@ -1,0 +1,207 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bar: bit-exact -- integer work.  Sorted (kmer_hi, kmer_lo, count, out[4], in[4],
+pid) records must equal the oracle's; totals and the order-independent checksum too.
+"""
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover - CPU box
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import oracle  # noqa: E402
+from paper_conf_icdcs_qiul17_b200 import DbgBuilder, build_graph, encode_reads, _lib  # noqa: E402
+from paper_conf_icdcs_qiul17_b200 import build as _build  # noqa: E402
+from synth import ReadSet, genome, make_config, make_reads, random_reads  # noqa: E402
+
+from gpu_helpers import (compare_vertices, decode_records, occurrences_from_oracle_msp,  # noqa: E402
+                         occurrences_from_records)
+
+NT = os.cpu_count() or 1
+_build.build()
+
+
+def _readset(reads):
+    b = "".join(reads).encode()
+    offs = np.zeros(len(reads) + 1, dtype=np.uint64)
+    offs[1:] = np.cumsum([len(r) for r in reads])
+    return ReadSet(np.frombuffer(b, dtype=np.uint8).copy(), offs)
+
+
+def _check(rs, k, p, np_, **kw):
+    res = build_graph(rs.seq, rs.offsets, k, p, np_, **kw)
+    orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT)
+    compare_vertices(res.vertices, orc)
+    st = res.stats
+    assert st["distinct"] == len(orc)
+    assert st["sum_count"] == int(orc["count"].sum())
+    assert st["sum_edges"] == int(orc["out"].sum() + orc["in"].sum())
+    assert st["checksum"] == oracle.checksum(orc)
+    return res, orc
+
+
+def test_tiny_config_bitexact():
+    rs = make_config("tiny")
+    res, orc = _check(rs, rs.k, rs.p, rs.num_partitions)
+    # I1: sum of counts = sum(L-K+1)
+    assert res.stats["sum_count"] == rs.n_kmers()
+    assert res.n_kmers == rs.n_kmers()
+    assert np.array_equal(res.part_kmers, np.bincount(orc["pid"], weights=orc["count"],
+                                                      minlength=rs.num_partitions).astype(np.int64))
+
+
+CASES = [(3, 1, 1), (5, 3, 3), (7, 7, 16), (11, 4, 5), (31, 11, 16), (31, 31, 3), (31, 1, 7),
+         (33, 13, 7), (39, 15, 9), (41, 17, 11), (63, 19, 16), (63, 1, 4), (63, 31, 64), (21, 9, 1)]
+
+
+@pytest.mark.parametrize("k,p,np_", CASES)
+def test_ragged_random_reads(k, p, np_):
+    rs = random_reads(400, 1, 2 * k + 150, seed=k * 100 + p, n_rate=0.01, lower_rate=0.02)
+    _check(rs, k, p, np_)
+
+
+@pytest.mark.parametrize("k,p", [(31, 11), (63, 19), (31, 31), (9, 3)])
+def test_long_reads_and_repeats(k, p):
+    rs = random_reads(20, 300, 3000, seed=7 + k)
+    reads = rs.reads()
+    reads += ["A" * 700, "AC" * 400, "ACGTTGCA" * 90, "T" * (k + 1), "G" * k, "ACG"]
+    _check(_readset(reads), k, p, 13)
+
+
+def test_hot_key_stress():
+    """One K-mer repeated ~10^5 times (poly-A), plus its reverse complement."""
+    reads = ["A" * 2000] * 30 + ["T" * 2000] * 30 + ["C" * 200]
+    res, orc = _check(_readset(reads), 31, 11, 8)
+    assert res.vertices["count"].max() == 60 * (2000 - 31 + 1)
+
+
+def test_edge_cases_empty_short():
+    empty = ReadSet(np.zeros(0, np.uint8), np.zeros(1, np.uint64))
+    res = build_graph(empty.seq, empty.offsets, 31, 11, 16)
+    assert res.n_vertices == 0 and res.stats["distinct"] == 0
+    _check(_readset(["ACGT", "", "ACGTACGTA", "TTTTTTTTT"]), 9, 3, 4)
+    _check(_readset(["A" * 31]), 31, 11, 16)
+
+
+def test_msp_records_vs_oracle_superkmers():
+    """Kernel (a): per-partition multisets of (K-mer, pred, succ) occurrences from the emitted
+    records equal the oracle's MSP superkmers (reading S: buffer order is not unique)."""
+    for (k, p, np_, seed) in [(31, 11, 16, 1), (63, 19, 8, 2), (15, 5, 3, 3), (31, 31, 5, 4)]:
+        rs = random_reads(200, 1, 300, seed=seed, n_rate=0.01)
+        b = DbgBuilder(k, p, np_)
+        d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+        b.msp(d_bases, d_off)
+        torch.cuda.synchronize()
+        nrec = int(b.part_records.sum())
+        words = b.records[: nrec * b.rec_words].cpu().numpy().view(np.uint32)
+        recs = decode_records(words, b.rec_words, k)
+        sk = oracle.msp(rs.seq, rs.offsets, k, p, np_)
+        nmax = _lib.dbg_record_max_kmers(b.prm)
+        # sizes per partition (count pass)
+        want_k = np.bincount(sk["pid"], weights=sk["n_kmers"], minlength=np_).astype(np.int64)
+        want_r = np.bincount(sk["pid"], weights=(sk["n_kmers"] + nmax - 1) // nmax,
+                             minlength=np_).astype(np.int64)
+        assert np.array_equal(b.part_kmers, want_k)
+        assert np.array_equal(b.part_records, want_r)
+        # records sit in their partition's range
+        off = b.d_rec_off.cpu().numpy()
+        pids = np.array([r[0] for r in recs])
+        for q in range(np_):
+            assert (pids[off[q]:off[q + 1]] == q).all()
+        assert occurrences_from_records(recs, k) == occurrences_from_oracle_msp(sk, rs.reads(), k)
+
+
+def test_table_overflow_detected_and_rebuilt():
+    """Reading O: an undersized table (lambda/(4 alpha) << distinct/N) overflows; the status word
+    reports DBG_ETABLEFULL and the builder rebuilds at capacity N^i_kmer with the same result."""
+    g = genome(20_000, seed=5)
+    seq, offs = make_reads(g, 3000, 100, 0.01, seed=6)
+    rs = ReadSet(seq, offs)
+    b = DbgBuilder(31, 11, 4, lam=0.04, alpha=0.5)
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    b.msp(d_bases, d_off)
+    for (lo, hi) in b.plan():
+        b.reset_output(1 << 20)
+        b.hash_batch(lo, hi)
+    assert _lib.dbg_sync_status(b.d_status) == _lib.DBG_ETABLEFULL
+    _check(rs, 31, 11, 4, lam=0.04, alpha=0.5)
+
+
+def test_batches_give_same_graph():
+    rs = make_config("tiny", scale=0.5)
+    a = build_graph(rs.seq, rs.offsets, 31, 11, 16)
+    b = build_graph(rs.seq, rs.offsets, 31, 11, 16, table_budget_bytes=64 * 2000)
+    assert len(b.batches) > 4
+    assert a.vertices.tobytes() == b.vertices.tobytes()
+    assert a.stats == b.stats
+
+
+def test_repeat_runs_deterministic():
+    rs = random_reads(2000, 50, 150, seed=99)
+    b = DbgBuilder(31, 11, 32)
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    r1 = b.build(d_bases, d_off)
+    r2 = b.build(d_bases, d_off)
+    assert r1.vertices.tobytes() == r2.vertices.tobytes() and r1.stats == r2.stats
+
+
+def test_strand_symmetry_on_gpu():
+    """I5: graph(R) = graph(rc(R)) on the GPU output alone."""
+    rs = random_reads(300, 40, 200, seed=3)
+    comp = str.maketrans("ACGT", "TGCA")
+    rr = _readset([r.translate(comp)[::-1] for r in rs.reads()])
+    a = build_graph(rs.seq, rs.offsets, 31, 11, 16)
+    b = build_graph(rr.seq, rr.offsets, 31, 11, 16)
+    assert a.vertices.tobytes() == b.vertices.tobytes()
+
+
+def _mirror_violations(v, k):
+    """I3 on a vertex array: every out-edge has its mirror in-edge (or out-edge) at the neighbour."""
+    code = v["kmer_lo"].astype(object) + (v["kmer_hi"].astype(object) << 64)
+    idx = {int(c): i for i, c in enumerate(code)}
+    mask = (1 << (2 * k)) - 1
+    bad = 0
+    for i in range(0, len(v), max(1, len(v) // 3000)):
+        c = int(code[i])
+        first = c >> (2 * k - 2)
+        for b in range(4):
+            m = int(v["out"][i][b])
+            if not m:
+                continue
+            w = ((c << 2) | b) & mask
+            rcw = 0
+            x = w
+            for _ in range(k):
+                rcw = (rcw << 2) | (3 - (x & 3))
+                x >>= 2
+            if w <= rcw:
+                bad += int(v["in"][idx[w]][first] != m)
+            else:
+                bad += int(v["out"][idx[rcw]][3 - first] != m)
+    return bad
+
+
+@pytest.mark.parametrize("name", ["ecoli"])
+def test_full_size_config_sampled(name):
+    """BASELINE configs[1] at full size, in the launch configuration bench.py times: invariants at
+    any size (I1, I2, I3 mirror on a sample) and oracle parity on 4000 sampled vertices."""
+    rs = make_config(name)
+    k, p, np_ = rs.k, rs.p, rs.num_partitions
+    res = build_graph(rs.seq, rs.offsets, k, p, np_)
+    v = res.vertices
+    L = rs.lengths()
+    assert res.stats["sum_count"] == int(np.maximum(L - k + 1, 0).sum())             # I1
+    assert res.stats["sum_edges"] == 2 * int(np.maximum(L - k, 0).sum())             # I2
+    assert res.stats["distinct"] == len(v)
+    assert np.all(v["kmer_lo"][1:] > v["kmer_lo"][:-1])                               # sorted, unique
+    assert _mirror_violations(v, k) == 0                                               # I3
+    rng = np.random.default_rng(17)
+    sel = v[np.sort(rng.choice(len(v), size=4000, replace=False))]
+    orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT,
+                       keys=np.stack([sel["kmer_hi"], sel["kmer_lo"]], 1))
+    compare_vertices(sel, orc)
