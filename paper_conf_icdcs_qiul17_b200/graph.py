@@ -110,7 +110,7 @@ class DbgBuilder:
         self.part_kmers = sizes[self.np:].copy()
         total = int(self.part_records.sum())
         need = total * self.rec_words
-        if self.records.numel() < need:
+        if self.records.numel() < max(need, 16):
             self.records = torch.empty(int(need * 1.05) + 16, dtype=torch.int32, device=self.device)
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
 
