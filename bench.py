@@ -184,63 +184,44 @@ def run_ours(args):
     offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
     n_kmers = rs.n_kmers()
     stream = torch.cuda.current_stream(dev)
-    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget)
+    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode)
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
 
-    def step(ev):
-        """One pass of rows a2-a6 (plus extraction when the tables are processed in batches)."""
-        ev["start"].record(stream)
+    def step():
+        """One pass of rows a2-a7 (MSP, sizing, fused zero/hash/extract)."""
         b.msp(d_bases, d_off, stream)
-        ev["msp_end"].record(stream)
-        batches = b.plan(stream)
-        multi = len(batches) > 1
-        if multi:
-            b.reset_output(n_kmers // 2 + 1, stream)
-        for (lo, hi) in batches:
-            b.hash_batch(lo, hi, stream)  # zero-fill + hash_build_kernel
-            if multi:
-                b.extract_batch(lo, hi, stream)
-        ev["end"].record(stream)
-        return batches
+        b.plan(stream)
+        b.reset_output(n_kmers // 2 + 1024, stream)
+        b.step2(stream)
 
     for _ in range(args.warmup):
-        step({"start": E(), "msp_end": E(), "end": E()})
-    torch.cuda.synchronize()
-    b.hash_timer = []
+        step()
+    st = _lib.dbg_sync_status(b.d_status, stream)
+    assert st == 0, _lib.dbg_status_string(st)
 
-    step_ms, msp_ms = [], []
+    b.timer = {}
+    step_ms = []
     with ClockSampler(local) as clk:
         for _ in range(args.steps):
             flush.zero_()
-            ev = {"start": E(), "msp_end": E(), "end": E()}
+            e0, e1 = E(), E()
             torch.cuda.synchronize()
-            batches = step(ev)
+            e0.record(stream)
+            step()
+            e1.record(stream)
             torch.cuda.synchronize()
-            step_ms.append(ev["start"].elapsed_time(ev["end"]))
-            msp_ms.append(ev["start"].elapsed_time(ev["msp_end"]))
-    hev = b.hash_timer
-    b.hash_timer = None
-    hash_ms_per_step = [sum(a.elapsed_time(c) for a, c in hev[i * len(batches):(i + 1) * len(batches)])
-                        for i in range(args.steps)]
-
-    # extraction (a7) + stats, timed separately; also validates invariants I1/I2
-    single = len(batches) == 1
-    x0, x1 = E(), E()
-    if single:
-        b.reset_output(max(1, n_kmers // 2), stream)
-        x0.record(stream)
-        b.extract_batch(0, rs.num_partitions, stream)
-        x1.record(stream)
+            step_ms.append(e0.elapsed_time(e1))
+    phases = {k: statistics.mean(a.elapsed_time(c) for a, c in v) for k, v in b.timer.items()}
+    b.timer = None
     st = _lib.dbg_sync_status(b.d_status, stream)
-    extract_ms = x0.elapsed_time(x1) if single else None
     stats = b.stats()
     L = rs.lengths()
     inv_ok = (st == 0 and stats["sum_count"] == n_kmers
               and stats["sum_edges"] == 2 * int(np.maximum(L - rs.k, 0).sum()))
 
-    # e2e through the public API: H2D of the packed reads (pinned) + path + extract + D2H stats
+    # e2e through the public API: H2D of the packed reads (pinned) + path + D2H of the stats
     e2e_ms = []
     for _ in range(max(1, min(args.steps, 5))):
         flush.zero_()
@@ -249,12 +230,10 @@ def run_ours(args):
         e0.record(stream)
         db, do = b.upload(packed, offsets, stream)
         b.msp(db, do, stream)
-        bt = b.plan(stream)
-        b.reset_output(max(1, n_kmers // 2), stream)
-        for (lo, hi) in bt:
-            b.hash_batch(lo, hi, stream)
-            b.extract_batch(lo, hi, stream)
-        host_stats = b.d_stats.to("cpu", non_blocking=False)
+        b.plan(stream)
+        b.reset_output(n_kmers // 2 + 1024, stream)
+        b.step2(stream)
+        b.d_stats.to("cpu")
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
@@ -262,15 +241,18 @@ def run_ours(args):
     d2h = 32 + 16 * rs.num_partitions
 
     ms = statistics.mean(step_ms)
-    hash_ms = statistics.mean(hash_ms_per_step)
+    key = "step2" if args.mode == "fused" else "hash_build"
+    hash_ms = phases.get(key, float("nan"))
     n_records = int(b.part_records.sum())
-    alg_bytes = n_kmers * 64 + n_records * 4 * b.rec_words
+    # one 32-B sector read + write-back per K-mer occurrence (the paper's
+    # random-access table RMW) + the records read + the vertex records written
+    alg_bytes = n_kmers * 64 + n_records * 4 * b.rec_words + stats["distinct"] * 56
     peak, peak_kind = _peaks()
     achieved = alg_bytes / (hash_ms * 1e-3) / 1e9
     traffic = None
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            traffic = json.load(f).get(rs.name, {}).get("hash_build_dram_bytes")
+            traffic = json.load(f).get(rs.name, {}).get("dram_bytes_per_launch")
     except Exception:
         pass
     cpu = None
@@ -279,22 +261,23 @@ def run_ours(args):
         rate, sub, dt = _oracle_rate(rs, args.cpu_seconds, threads)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
+    launches_per_step = 3 + (2 if args.mode == "fused" else 2 * len(b.batches)) + 1
     line = {
         "metric": METRIC, "value": n_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": _config_json(rs, args, {"batches": len(batches)}),
+        "config": _config_json(rs, args, {"mode": args.mode, "batches": len(b.batches)}),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "kernel": "hash_build_kernel",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "kernel": "subgraph_kernel" if args.mode == "fused" else "hash_build_kernel",
                      "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
-                     "hash_kmers_per_s": n_kmers / (hash_ms * 1e-3)},
+                     "kernel_ms": hash_ms, "kernel_kmers_per_s": n_kmers / (hash_ms * 1e-3)},
         "cpu_baseline": cpu,
         "e2e": {"value": n_kmers / (statistics.mean(e2e_ms) * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": d2h, "ms": statistics.mean(e2e_ms)},
-        "gpu_launches": args.steps * (4 + len(batches) * (2 if len(batches) > 1 else 1)),
+        "gpu_launches": args.steps * launches_per_step,
         "clocks": clk.summary(),
-        "breakdown_ms": {"msp": statistics.mean(msp_ms), "hash_build": hash_ms,
-                         "plan_fill_other": ms - statistics.mean(msp_ms) - hash_ms, "extract": extract_ms},
+        "breakdown_ms": phases,
         "stats": stats, "invariants_ok": bool(inv_ok), "gen_s": gen_s,
     }
     print(json.dumps(line), flush=True)
@@ -313,6 +296,7 @@ def main():
     ap.add_argument("--lam", type=float, default=2.0)
     ap.add_argument("--alpha", type=float, default=0.5)
     ap.add_argument("--table-budget", type=int, default=None)
+    ap.add_argument("--mode", choices=["fused", "resident"], default="fused")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

@@ -83,13 +83,18 @@ typedef struct {
  *   words 1..: the bases S[s-has_left .. e+K-1+has_right], 2-bit, 16 per word,
  *              first base in the most significant bits (Sec. III-B).
  * A superkmer longer than the record holds is stored as consecutive pieces,
- * each with its own adjacency bases (the graph is unchanged). */
+ * each with its own adjacency bases (the graph is unchanged).  Records are
+ * first written in read order to d_staging (capacity staging_cap records),
+ * then scattered into partition order. */
 typedef struct {
-  uint64_t* d_n_records;     /* [NP]   records per partition (count pass) */
-  uint64_t* d_n_kmers;       /* [NP]   N^i_kmer, K-mers per partition (count pass; sizes tables) */
-  uint64_t* d_record_offset; /* [NP+1] exclusive prefix sum of d_n_records (count pass) */
-  uint64_t* d_fill;          /* [NP]   emission cursors (emit pass; zeroed by the call) */
-  uint32_t* d_records;       /* record buffer, d_record_offset[NP] records; NULL => count pass */
+  uint64_t* d_n_records;     /* [NP]   records per partition (pass 1) */
+  uint64_t* d_n_kmers;       /* [NP]   N^i_kmer, K-mers per partition (pass 1; sizes tables) */
+  uint64_t* d_record_offset; /* [NP+1] exclusive prefix sum of d_n_records (pass 1) */
+  uint64_t* d_fill;          /* [NP]   scatter cursors (pass 2; zeroed by the call) */
+  uint64_t* d_staged;        /* [1]    records reserved in d_staging (pass 1) */
+  uint32_t* d_staging;       /* staging_cap records, read order (pass 1 output, pass 2 input) */
+  uint64_t staging_cap;      /* capacity of d_staging in records */
+  uint32_t* d_records;       /* d_record_offset[NP] records in partition order; NULL => pass 1 */
 } dbg_partition_set;
 
 /* ---- sizes ------------------------------------------------------------ */
@@ -98,8 +103,10 @@ DBG_API int dbg_abi_version(void);
 DBG_API uint32_t dbg_record_words(const dbg_params* prm);
 /* K-mers a record holds at most. */
 DBG_API uint32_t dbg_record_max_kmers(const dbg_params* prm);
-/* Bytes per hash-table slot (64). */
+/* Bytes per hash-table slot: a key entry (dbg_key_bytes: 16 for K <= 31, 32
+ * otherwise) plus a 32-byte counter record. */
 DBG_API uint32_t dbg_slot_bytes(const dbg_params* prm);
+DBG_API uint32_t dbg_key_bytes(const dbg_params* prm);
 /* Table capacity for a partition with n_kmers K-mers: ceil(lambda/(4 alpha) * n_kmers)
  * (Sec. IV-A), at least 1 when n_kmers > 0 (Property 1 sizing). */
 DBG_API uint64_t dbg_table_capacity(const dbg_params* prm, uint64_t n_kmers);
@@ -115,44 +122,62 @@ DBG_API dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64_t*
 /* ---- a2-a4: Step 1, MSP (Sec. III-B; Defs. 1-2) ------------
  * d_bases: packed stream (dbg_packed_words(total) words), d_offsets: [n_reads+1]
  * base offsets of the reads in the stream.
- * part->d_records == NULL: count pass -- zeroes and fills d_n_records, d_n_kmers
- *   and d_record_offset (size query; the caller reads d_record_offset[NP],
- *   allocates and calls again).
- * part->d_records != NULL: emit pass -- requires d_record_offset from a count
- *   pass over the same reads; zeroes d_fill and writes every record. */
+ * part->d_records == NULL: pass 1 -- zeroes and fills d_n_records, d_n_kmers,
+ *   d_record_offset and *d_staged, and writes the records (read order) into
+ *   d_staging while they fit.  The caller reads d_record_offset[NP] (or the
+ *   sizes); if it exceeds staging_cap, it grows d_staging and repeats pass 1.
+ * part->d_records != NULL: pass 2 -- scatters the staged records into
+ *   partition order (d_record_offset[NP] records). */
 DBG_API dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
                              const uint64_t* d_offsets, uint64_t n_reads,
                              const dbg_partition_set* part, cudaStream_t stream);
 
 /* ---- a5: sizing (Property 1; Sec. IV-A) ----------------------
  * d_table_offset[NP+1] = exclusive prefix sum of dbg_table_capacity(N^i_kmer)
- * (in slots).  Tables of partitions [b, e) need d_table_offset[e]-d_table_offset[b]
- * slots of dbg_slot_bytes each, zero-filled before dbg_hash_build (EMPTY = 0). */
+ * (in slots). */
 DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers,
                           uint64_t* d_table_offset, cudaStream_t stream);
 
-/* ---- a6: Step 2, hash build (Sec. III-C; Sec. III-D)
+/* ---- a5-a7 fused: Step 2 through an L2-resident ring (the hot path) ------
+ * For partitions [pid_begin, pid_end): zero-fill the key entries of the
+ * partition's table, build it (one insertion per distinct vertex, multiple
+ * updates, Sec. III-C), and compact it into d_out -- one
+ * persistent kernel in which each partition's table lives in one of 4 ring
+ * regions of d_ring (ring_bytes >= dbg_subgraph_ring_bytes(max capacity);
+ * a smaller ring sets status bit 2 -> DBG_ENOSPACE).  d_workspace holds
+ * dbg_subgraph_workspace_bytes(pid_end - pid_begin) bytes of scheduling
+ * state.  Output appends to d_out[*d_n_out ...] and accumulates *d_stats as in
+ * dbg_extract_graph. */
+DBG_API uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t max_capacity);
+DBG_API uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions);
+DBG_API dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                               int32_t pid_end, const uint64_t* d_table_offset, void* d_ring,
+                               uint64_t ring_bytes, void* d_workspace, uint64_t workspace_bytes,
+                               dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
+                               dbg_stats* d_stats, uint32_t* d_status, cudaStream_t stream);
+
+/* ---- a6: Step 2 with resident tables (Sec. III-C) ------------
  * Inserts every K-mer occurrence of partitions [pid_begin, pid_end) into that
- * partition's table: one insertion per distinct vertex (a 64- or 128-bit
- * CAS claims an EMPTY slot), multiple updates (atomic adds on the edge
- * counters).  Partition i's table starts at
- *   (char*)d_slots + (d_table_offset[i] - slot_base) * dbg_slot_bytes().
+ * partition's table.  d_table holds the tables of all these partitions,
+ * n = d_table_offset[pid_end] - d_table_offset[pid_begin] slots: first the n
+ * key entries (dbg_key_bytes each, zero-filled by the caller = EMPTY), then
+ * n 32-byte counter records (no initialisation needed); partition i owns
+ * slots [d_table_offset[i] - d_table_offset[pid_begin], ...) of both arrays.
  * Overflow sets bit 0 of *d_status (reported by dbg_sync_status). */
 DBG_API dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
-                          int32_t pid_end, void* d_slots, const uint64_t* d_table_offset,
-                          uint64_t slot_base, uint32_t* d_status, cudaStream_t stream);
+                          int32_t pid_end, void* d_table, const uint64_t* d_table_offset,
+                          uint32_t* d_status, cudaStream_t stream);
 
 /* ---- a7: output (Def. 3) -------------------------------------
- * Compacts the occupied slots of partitions [pid_begin, pid_end) into
- * d_out[*d_n_out ...] (appends; the caller zeroes *d_n_out and *d_stats
+ * Compacts the occupied slots of resident tables (layout of dbg_hash_build)
+ * into d_out[*d_n_out ...] (appends; the caller zeroes *d_n_out and *d_stats
  * once) and accumulates *d_stats.  Records beyond out_cap are dropped and
  * set bit 1 of *d_status (DBG_ENOSPACE; *d_n_out still counts them).
  * Record order is unspecified (reading S): use dbg_sort_vertices. */
-DBG_API dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_slots,
-                             const uint64_t* d_table_offset, uint64_t slot_base,
-                             int32_t pid_begin, int32_t pid_end, dbg_vertex* d_out,
-                             uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
-                             uint32_t* d_status, cudaStream_t stream);
+DBG_API dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_table,
+                             const uint64_t* d_table_offset, int32_t pid_begin, int32_t pid_end,
+                             dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
+                             dbg_stats* d_stats, uint32_t* d_status, cudaStream_t stream);
 
 /* Sorts n vertices ascending by (kmer_hi, kmer_lo) (reading Q) from d_in to
  * d_out (distinct buffers) using a caller workspace of
@@ -163,7 +188,7 @@ DBG_API dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_
                              cudaStream_t stream);
 
 /* Synchronizes the stream, then decodes *d_status: bit 0 -> DBG_ETABLEFULL,
- * bit 1 -> DBG_ENOSPACE; also returns DBG_ECUDA on a sticky CUDA error. */
+ * bit 1 or 2 -> DBG_ENOSPACE; also returns DBG_ECUDA on a sticky CUDA error. */
 DBG_API dbg_status dbg_sync_status(const uint32_t* d_status, cudaStream_t stream);
 
 DBG_API const char* dbg_status_string(dbg_status s);

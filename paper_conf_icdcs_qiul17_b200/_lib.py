@@ -33,7 +33,8 @@ class dbg_params(ctypes.Structure):
 class dbg_partition_set(ctypes.Structure):
     _fields_ = [("d_n_records", ctypes.c_void_p), ("d_n_kmers", ctypes.c_void_p),
                 ("d_record_offset", ctypes.c_void_p), ("d_fill", ctypes.c_void_p),
-                ("d_records", ctypes.c_void_p)]
+                ("d_staged", ctypes.c_void_p), ("d_staging", ctypes.c_void_p),
+                ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p)]
 
 
 # dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
@@ -54,13 +55,18 @@ SIGNATURES = {
     "dbg_record_words": (ctypes.c_uint32, [_PRM]),
     "dbg_record_max_kmers": (ctypes.c_uint32, [_PRM]),
     "dbg_slot_bytes": (ctypes.c_uint32, [_PRM]),
+    "dbg_key_bytes": (ctypes.c_uint32, [_PRM]),
     "dbg_table_capacity": (_U64, [_PRM, _U64]),
     "dbg_packed_words": (_U64, [_U64]),
     "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
     "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P]),
-    "dbg_hash_build": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _U64, _P, _P]),
-    "dbg_extract_graph": (ctypes.c_int, [_PRM, _P, _P, _U64, _I32, _I32, _P, _U64, _P, _P, _P, _P]),
+    "dbg_subgraph_ring_bytes": (_U64, [_PRM, _U64]),
+    "dbg_subgraph_workspace_bytes": (_U64, [_PRM, _I32]),
+    "dbg_build_subgraphs": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _U64, _P, _U64, _P, _U64, _P, _P,
+                                           _P, _P]),
+    "dbg_hash_build": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _P, _P]),
+    "dbg_extract_graph": (ctypes.c_int, [_PRM, _P, _P, _I32, _I32, _P, _U64, _P, _P, _P, _P]),
     "dbg_sort_workspace_bytes": (_U64, [_PRM, _U64]),
     "dbg_sort_vertices": (ctypes.c_int, [_PRM, _P, _P, _U64, _P, _U64, _P]),
     "dbg_sync_status": (ctypes.c_int, [_P, _P]),
@@ -117,8 +123,10 @@ def params(k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float =
     return dbg_params(k, p, num_partitions, lam, alpha)
 
 
-def partition_set(n_records, n_kmers, record_offset, fill, records=None) -> dbg_partition_set:
-    return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(records))
+def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
+                  records=None) -> dbg_partition_set:
+    return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(staged),
+                             _ptr(staging), staging_cap, _ptr(records))
 
 
 # --------------------------------------------------------------------------- entry points
@@ -138,6 +146,10 @@ def dbg_record_max_kmers(prm: dbg_params) -> int:
 
 def dbg_slot_bytes(prm: dbg_params) -> int:
     return load().dbg_slot_bytes(ctypes.byref(prm))
+
+
+def dbg_key_bytes(prm: dbg_params) -> int:
+    return load().dbg_key_bytes(ctypes.byref(prm))
 
 
 def dbg_table_capacity(prm: dbg_params, n_kmers: int) -> int:
@@ -167,18 +179,35 @@ def dbg_table_plan(prm, d_n_kmers, d_table_offset, stream=None) -> None:
                                                    _ptr(d_table_offset), _stream(stream)))
 
 
-def dbg_hash_build(prm, part, pid_begin: int, pid_end: int, d_slots, d_table_offset, slot_base: int,
-                   d_status, stream=None) -> None:
+def dbg_subgraph_ring_bytes(prm, max_capacity: int) -> int:
+    return load().dbg_subgraph_ring_bytes(ctypes.byref(prm), max_capacity)
+
+
+def dbg_subgraph_workspace_bytes(prm, n_partitions: int) -> int:
+    return load().dbg_subgraph_workspace_bytes(ctypes.byref(prm), n_partitions)
+
+
+def dbg_build_subgraphs(prm, part, pid_begin: int, pid_end: int, d_table_offset, d_ring, ring_bytes: int,
+                        d_workspace, workspace_bytes: int, d_out, out_cap: int, d_n_out, d_stats, d_status,
+                        stream=None) -> None:
+    _check("dbg_build_subgraphs", load().dbg_build_subgraphs(
+        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_table_offset), _ptr(d_ring), ring_bytes,
+        _ptr(d_workspace), workspace_bytes, _ptr(d_out), out_cap, _ptr(d_n_out), _ptr(d_stats), _ptr(d_status),
+        _stream(stream)))
+
+
+def dbg_hash_build(prm, part, pid_begin: int, pid_end: int, d_table, d_table_offset, d_status,
+                   stream=None) -> None:
     _check("dbg_hash_build", load().dbg_hash_build(
-        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_slots), _ptr(d_table_offset),
-        slot_base, _ptr(d_status), _stream(stream)))
+        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_table), _ptr(d_table_offset),
+        _ptr(d_status), _stream(stream)))
 
 
-def dbg_extract_graph(prm, d_slots, d_table_offset, slot_base: int, pid_begin: int, pid_end: int,
-                      d_out, out_cap: int, d_n_out, d_stats, d_status, stream=None) -> None:
+def dbg_extract_graph(prm, d_table, d_table_offset, pid_begin: int, pid_end: int, d_out, out_cap: int, d_n_out,
+                      d_stats, d_status, stream=None) -> None:
     _check("dbg_extract_graph", load().dbg_extract_graph(
-        ctypes.byref(prm), _ptr(d_slots), _ptr(d_table_offset), slot_base, pid_begin, pid_end,
-        _ptr(d_out), out_cap, _ptr(d_n_out), _ptr(d_stats), _ptr(d_status), _stream(stream)))
+        ctypes.byref(prm), _ptr(d_table), _ptr(d_table_offset), pid_begin, pid_end, _ptr(d_out), out_cap,
+        _ptr(d_n_out), _ptr(d_stats), _ptr(d_status), _stream(stream)))
 
 
 def dbg_sort_workspace_bytes(prm, n: int) -> int:

@@ -17,11 +17,6 @@ extern "C" uint32_t dbg_record_max_kmers(const dbg_params* prm) {
   return prm ? record_max_kmers(prm->k) : 0u;
 }
 
-extern "C" uint32_t dbg_slot_bytes(const dbg_params* prm) {
-  (void)prm;
-  return kSlotBytes;
-}
-
 // Sec. IV-A: "we use [N^i_kmer] with a load ratio alpha to set the
 // hash table size as lambda/(4 alpha) N^i_kmer"; lambda = 2, alpha = 0.5 by
 // default, which makes the capacity N^i_kmer (Table II).
@@ -71,7 +66,7 @@ extern "C" dbg_status dbg_sync_status(const uint32_t* d_status, cudaStream_t str
     return DBG_ECUDA;
   if (cudaStreamSynchronize(stream) != cudaSuccess) return DBG_ECUDA;
   if (h & kStatusTableFull) return DBG_ETABLEFULL;
-  if (h & kStatusNoSpace) return DBG_ENOSPACE;
+  if (h & (kStatusNoSpace | 4u)) return DBG_ENOSPACE;
   return DBG_OK;
 }
 

@@ -10,7 +10,6 @@ namespace dbg {
 
 constexpr int kWarp = 32;
 constexpr uint32_t kFull = 0xffffffffu;
-constexpr uint32_t kSlotBytes = 64;     // one 64-B aligned slot = 2 sectors, 1/2 line
 constexpr uint32_t kMaxPid = (1u << 22) - 1;
 constexpr uint64_t kOccupied = 1ull << 63;
 

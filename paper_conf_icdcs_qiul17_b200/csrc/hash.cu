@@ -2,60 +2,167 @@
 // (Sec. III-C; Sec. III-D), kernel (b) of the north
 // star, plus extraction of the vertex records (Def. 3).
 //
-// Table: open addressing, linear probing, 64-B slots (two 32-B sectors):
-//   K <= 31: u64 key | u32 out[4] | u32 in[4] | u32 t_out | pad
-//   K <= 63: u64 key_hi | u64 key_lo | u32 out[4] | u32 in[4] | u32 t_out | pad
-// Key words carry bit 63 = occupied, so a zero-filled table is EMPTY and one
-// memset initialises keys and counters together.  For two-word keys the
-// 2K-bit code is split 63/63 bits, so each word of a claimed key is non-zero
-// and a torn 16-B read (one word still zero) is recognisable.
-//
-// One insertion, multiple updates: the first
-// occurrence of a vertex claims an EMPTY slot with a single 64-bit (K <= 31)
-// or 128-bit (K <= 63) atomicCAS -- the whole key is published atomically, so
-// the paper's {empty, locked, occupied} state word and its "locked" spin
-// are unnecessary; every later occurrence finds the key with a
-// plain load and only issues red.global.add on its counters.
+// Table of one partition with capacity n (open addressing, linear probing):
+//   key entries  n x KE bytes  (zero-filled = EMPTY)
+//     K <= 31: KE = 16  { u64 key; u32 t_out; u32 pad }
+//     K <= 63: KE = 32  { u64 key_hi; u64 key_lo; u32 t_out; u32 pad[3] }
+//   counters     n x 32 bytes  { u32 out[4]; u32 in[4] }  (never zero-filled)
+// The key word (hi word for K > 31) carries the paper's occupancy state
+// (Sec. III-C3, Fig. 4) in its two top bits:
+//   0                 empty
+//   OCC | code        locked   (claimed; counters being initialised)
+//   OCC | READY | code occupied (never modified again, read concurrently)
+// One insertion: a thread that sees EMPTY claims the slot with a
+// single 64-bit (K <= 31) or 128-bit (K <= 63) atomicCAS that publishes the
+// whole key at once, initialises the vertex's counters with its own
+// occurrence, and sets READY with a release.  Multiple updates:
+// every other occurrence compares keys and issues red.global.add on two
+// counters; only a thread that finds its own key still "locked" waits (the
+// paper's blocked readers).  So only the 16/32-B key entries need
+// zero-filling, not the 32-B counter records.
 //
 // Counter economy: each occurrence increments exactly one "out-side" counter
 // (out[c] if it has a successor in the vertex orientation, else t_out) and at
 // most one in-side counter, so count = sum(out) + t_out is derived at
-// extraction and the per-occurrence count atomic of the paper's entry
-// disappears: two reds per K-mer instead of three.
+// extraction: two reds per K-mer instead of the paper's three.
+//
+// Kernels:
+//  hash_build_kernel    tables of partitions [b, e) resident (dbg_hash_build)
+//  extract_kernel       compaction of resident tables (dbg_extract_graph)
+//  subgraph_kernel      fused Step 2 (dbg_build_subgraphs): a persistent
+//                       kernel streams partitions through a ring of RING
+//                       L2-sized table regions; work items (zero a key chunk,
+//                       hash a record chunk, extract a slot chunk) are claimed
+//                       in a fixed global order from one atomic counter and
+//                       chained by per-partition completion counters, so a
+//                       partition's table lives in L2 from zero-fill to
+//                       extraction (the B200 form of "localize memory access
+//                       by configuring the hash table size").
+#include <cub/block/block_reduce.cuh>
+#include <cub/block/block_scan.cuh>
 #include <cub/device/device_radix_sort.cuh>
 
 #include "dbg_device.cuh"
+
+int dbg_sm_count();
+bool dbg_params_ok(const dbg_params* prm);
 
 namespace dbg {
 
 typedef unsigned __int128 u128;
 
-constexpr int kHashThreads = 256;
+constexpr int kThreads = 256;
+constexpr uint64_t kReady = 1ull << 62;
+constexpr uint64_t kCodeMask = kReady - 1;
 constexpr uint64_t kSlotSeed = 0x9e3779b97f4a7c15ull;
+constexpr int kRing = 4;
+constexpr uint32_t kZeroSlots = 4096;          // key entries per zero item
+constexpr uint32_t kHashRecs = kThreads;       // records per hash item
+constexpr int kXPer = 8;
+constexpr uint32_t kExtractSlots = kThreads * kXPer;
+constexpr uint32_t kStatusRing = 4u;
 
-template <int KW>
-struct SlotLayout;
-template <>
-struct SlotLayout<1> {
-  typedef uint64_t Code;
-  static constexpr int kOut = 2, kIn = 6, kTerm = 10;  // u32 indices within the slot
-};
-template <>
-struct SlotLayout<2> {
-  typedef u128 Code;
-  static constexpr int kOut = 4, kIn = 8, kTerm = 12;
+__host__ __device__ inline uint32_t key_bytes(int k) { return k <= 31 ? 16u : 32u; }
+constexpr uint32_t kCtrBytes = 32;
+
+struct Table {
+  char* keys;      // key entries
+  uint32_t* ctr;   // counter records (8 u32 each)
+  uint64_t cap;
 };
 
-struct HashArgs {
-  const uint32_t* records;
-  const uint64_t* rec_off;
-  const uint64_t* tab_off;
-  uint64_t slot_base;
-  char* slots;
-  uint32_t* status;
-  int pid_begin, pid_end;
-  int k;
-};
+__device__ __forceinline__ uint64_t slot_hash(uint64_t code) { return fmix64(code ^ kSlotSeed); }
+__device__ __forceinline__ uint64_t slot_hash(u128 code) {
+  return fmix64((uint64_t)code ^ fmix64((uint64_t)(code >> 64) ^ kSlotSeed));
+}
+
+__device__ __forceinline__ void red_add(uint32_t* p) {
+  asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(p) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Claimer: counters start at this occurrence's increments; then READY.
+__device__ __forceinline__ void init_vertex(uint32_t* ctr, uint32_t* t_out, uint64_t* state, int o, int i) {
+  uint4* cp = reinterpret_cast<uint4*>(ctr);
+  __stcg(cp, make_uint4(o == 0, o == 1, o == 2, o == 3));
+  __stcg(cp + 1, make_uint4(i == 0, i == 1, i == 2, i == 3));
+  __stcg(t_out, (uint32_t)(o == 4));
+  __threadfence();
+  atomicOr(reinterpret_cast<unsigned long long*>(state), (unsigned long long)kReady);
+}
+
+__device__ __forceinline__ void update_vertex(uint32_t* ctr, uint32_t* t_out, const uint64_t* state,
+                                              uint64_t seen, int o, int i) {
+  if (!(seen & kReady))  // locked: blocked until the claimer publishes
+    while (!(ld_acquire(state) & kReady)) __nanosleep(20);
+  red_add(o < 4 ? ctr + o : t_out);
+  if (i >= 0) red_add(ctr + 4 + i);
+}
+
+// Insert-or-update of one occurrence; o in 0..4 (4 = no out-side neighbour),
+// i in -1..3.  Returns false if the probe sequence wrapped (table full).
+__device__ __forceinline__ bool upsert(const Table& t, uint64_t code, int o, int i) {
+  const uint64_t want = code | kOccupied;
+  uint64_t idx = __umul64hi(slot_hash(code), t.cap);
+  for (uint64_t pr = 0; pr < t.cap; ++pr) {
+    uint64_t* kp = reinterpret_cast<uint64_t*>(t.keys + idx * 16);
+    uint64_t cur = __ldcg(kp);
+    if (cur == 0) {
+      cur = atomicCAS(reinterpret_cast<unsigned long long*>(kp), 0ull, (unsigned long long)want);
+      if (cur == 0) {
+        init_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), kp, o, i);
+        return true;
+      }
+    }
+    if ((cur & ~kReady) == want) {
+      update_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), kp, cur, o, i);
+      return true;
+    }
+    idx = idx + 1 == t.cap ? 0 : idx + 1;
+  }
+  return false;
+}
+
+__device__ __forceinline__ bool upsert(const Table& t, u128 code, int o, int i) {
+  const uint64_t want_hi = (uint64_t)(code >> 64) | kOccupied, want_lo = (uint64_t)code;
+  uint64_t idx = __umul64hi(slot_hash(code), t.cap);
+  for (uint64_t pr = 0; pr < t.cap; ++pr) {
+    ulonglong2* kp = reinterpret_cast<ulonglong2*>(t.keys + idx * 32);
+    ulonglong2 cur = __ldcg(kp);
+    if (cur.x == 0) {  // empty -- or a torn read of a key being published: the CAS decides
+      ulonglong2 want;
+      want.x = want_hi;
+      want.y = want_lo;
+      cur = atomicCAS(kp, make_ulonglong2(0ull, 0ull), want);
+      if (cur.x == 0 && cur.y == 0) {
+        init_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), reinterpret_cast<uint64_t*>(kp),
+                    o, i);
+        return true;
+      }
+    } else if (cur.y == 0) {
+      // a 16-B load is not single-copy atomic: a claimed hi word next to a zero low
+      // word may be a torn read of a key being published -- the no-op CAS returns
+      // the entry atomically
+      cur = atomicCAS(kp, cur, cur);
+    }
+    if ((cur.x & ~kReady) == want_hi && cur.y == want_lo) {
+      update_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), reinterpret_cast<uint64_t*>(kp),
+                    cur.x, o, i);
+      return true;
+    }
+    idx = idx + 1 == t.cap ? 0 : idx + 1;
+  }
+  return false;
+}
 
 template <int R>
 __device__ __forceinline__ uint32_t base_at(const uint32_t (&w)[R], int i) {
@@ -66,133 +173,58 @@ __device__ __forceinline__ uint32_t base_at(const uint32_t (&w)[R], int i) {
   return (v >> (30 - 2 * (i & 15))) & 3u;
 }
 
-__device__ __forceinline__ uint64_t slot_hash(uint64_t code) { return fmix64(code ^ kSlotSeed); }
-__device__ __forceinline__ uint64_t slot_hash(u128 code) {
-  return fmix64((uint64_t)code ^ fmix64((uint64_t)(code >> 64) ^ kSlotSeed));
-}
-
-// Finds the slot of `code` in the table [tbase, cap), inserting it if absent.
-// Returns nullptr if the probe sequence wrapped (table full, reading O).
-__device__ __forceinline__ uint32_t* find_or_insert(char* tbase, uint64_t cap, uint64_t code) {
-  const unsigned long long key = code | kOccupied;
-  uint64_t idx = __umul64hi(slot_hash(code), cap);
-  for (uint64_t pr = 0; pr < cap; ++pr) {
-    unsigned long long* kp = reinterpret_cast<unsigned long long*>(tbase + idx * kSlotBytes);
-    unsigned long long cur = __ldcg(kp);
-    if (cur == key) return reinterpret_cast<uint32_t*>(kp);
-    if (cur == 0) {
-      cur = atomicCAS(kp, 0ull, key);  // one insertion per distinct vertex
-      if (cur == 0 || cur == key) return reinterpret_cast<uint32_t*>(kp);
-    }
-    idx = idx + 1 == cap ? 0 : idx + 1;
-  }
-  return nullptr;
-}
-
-__device__ __forceinline__ uint32_t* find_or_insert(char* tbase, uint64_t cap, u128 code) {
-  const unsigned long long khi = (unsigned long long)(code >> 63) | kOccupied;
-  const unsigned long long klo = ((unsigned long long)code & ~kOccupied) | kOccupied;
-  uint64_t idx = __umul64hi(slot_hash(code), cap);
-  for (uint64_t pr = 0; pr < cap; ++pr) {
-    ulonglong2* kp = reinterpret_cast<ulonglong2*>(tbase + idx * kSlotBytes);
-    ulonglong2 cur = __ldcg(kp);
-    if (cur.x == khi && cur.y == klo) return reinterpret_cast<uint32_t*>(kp);
-    if (cur.x == 0 || cur.y == 0) {  // empty, or a torn read of a key being published
-      ulonglong2 want;
-      want.x = khi;
-      want.y = klo;
-      cur = atomicCAS(kp, make_ulonglong2(0ull, 0ull), want);
-      if ((cur.x == 0 && cur.y == 0) || (cur.x == khi && cur.y == klo))
-        return reinterpret_cast<uint32_t*>(kp);
-    }
-    idx = idx + 1 == cap ? 0 : idx + 1;
-  }
-  return nullptr;
-}
-
-__device__ __forceinline__ void red_add(uint32_t* p) {
-  asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(p) : "memory");
-}
-
-// Binary search: the partition i in [lo, hi) with off[i] <= x < off[i+1].
-__device__ __forceinline__ int find_part(const uint64_t* __restrict__ off, int lo, int hi, uint64_t x) {
-  while (hi - lo > 1) {
-    int mid = (lo + hi) >> 1;
-    if (__ldg(off + mid) <= x) lo = mid;
-    else hi = mid;
-  }
-  return lo;
-}
-
-// One thread per record (a superkmer piece): roll the forward and reverse
-// codes over its K-mers (<kmer, edge> pair generation), then
-// insert/update each canonical K-mer.
-template <int KW, int R>
-__global__ void __launch_bounds__(kHashThreads) hash_build_kernel(HashArgs a) {
-  typedef typename SlotLayout<KW>::Code Code;
-  const uint64_t r_begin = a.rec_off[a.pid_begin], r_end = a.rec_off[a.pid_end];
-  const int K = a.k;
-  const Code mask = (K == 32 * KW) ? ~(Code)0 : (((Code)1 << (2 * K)) - 1);
-  const int top = 2 * K - 2;
-  for (uint64_t rec = r_begin + (uint64_t)blockIdx.x * kHashThreads + threadIdx.x; rec < r_end;
-       rec += (uint64_t)gridDim.x * kHashThreads) {
-    uint32_t w[R];
-    const uint4* src = reinterpret_cast<const uint4*>(a.records + rec * R);
+// <kmer, edge> pair generation from one record and the
+// insert/update of every K-mer.  Returns false on overflow.
+template <typename Code, int R>
+__device__ __forceinline__ bool hash_record(const uint32_t* rp, int K, const Table& t) {
+  uint32_t w[R];
+  const uint4* src = reinterpret_cast<const uint4*>(rp);
 #pragma unroll
-    for (int v = 0; v < R / 4; ++v) {
-      uint4 x = __ldcs(src + v);  // streamed once
-      w[4 * v] = x.x;
-      w[4 * v + 1] = x.y;
-      w[4 * v + 2] = x.z;
-      w[4 * v + 3] = x.w;
+  for (int v = 0; v < R / 4; ++v) {
+    const uint4 x = __ldcs(src + v);  // streamed once
+    w[4 * v] = x.x;
+    w[4 * v + 1] = x.y;
+    w[4 * v + 2] = x.z;
+    w[4 * v + 3] = x.w;
+  }
+  const uint32_t hdr = w[0];
+  const int n = hdr & 255u;
+  const int hl = (hdr >> 8) & 1u, hr = (hdr >> 9) & 1u;
+  const Code mask = ((Code)1 << (2 * K)) - 1;
+  const int top = 2 * K - 2;
+  Code fwd = 0, rc = 0;
+  for (int j = 0; j < K; ++j) {
+    const uint32_t b = base_at<R>(w, hl + j);
+    fwd = (fwd << 2) | (Code)b;
+    rc |= (Code)(3u - b) << (2 * j);
+  }
+  int pred = hl ? (int)base_at<R>(w, 0) : -1;
+  bool ok = true;
+  for (int s = 0; s < n; ++s) {
+    const bool has_succ = s < n - 1 || hr;
+    const int succ = has_succ ? (int)base_at<R>(w, hl + s + K) : -1;
+    const bool is_fwd = fwd < rc;  // odd K: never equal (reading C)
+    int o, i;
+    if (is_fwd) {  // reading J
+      o = succ >= 0 ? succ : 4;
+      i = pred;
+    } else {
+      o = pred >= 0 ? 3 - pred : 4;
+      i = succ >= 0 ? 3 - succ : -1;
     }
-    const uint32_t hdr = w[0];
-    const int n = hdr & 255u;
-    const int hl = (hdr >> 8) & 1u, hr = (hdr >> 9) & 1u;
-    const uint32_t pid = hdr >> 10;
-    const uint64_t t0 = __ldg(a.tab_off + pid);
-    const uint64_t cap = __ldg(a.tab_off + pid + 1) - t0;
-    char* tbase = a.slots + (t0 - a.slot_base) * kSlotBytes;
-    Code fwd = 0, rc = 0;
-    for (int j = 0; j < K; ++j) {
-      const uint32_t b = base_at<R>(w, hl + j);
-      fwd = (fwd << 2) | (Code)b;
-      rc |= (Code)(3u - b) << (2 * j);
-    }
-    int pred = hl ? (int)base_at<R>(w, 0) : -1;
-    for (int t = 0; t < n; ++t) {
-      const bool has_succ = t < n - 1 || hr;
-      const int succ = has_succ ? (int)base_at<R>(w, hl + t + K) : -1;
-      const bool is_fwd = fwd < rc;  // odd K: never equal (reading C)
-      int o_idx, i_idx;
-      if (is_fwd) {  // reading J
-        o_idx = succ >= 0 ? SlotLayout<KW>::kOut + succ : SlotLayout<KW>::kTerm;
-        i_idx = pred >= 0 ? SlotLayout<KW>::kIn + pred : -1;
-      } else {
-        o_idx = pred >= 0 ? SlotLayout<KW>::kOut + 3 - pred : SlotLayout<KW>::kTerm;
-        i_idx = succ >= 0 ? SlotLayout<KW>::kIn + 3 - succ : -1;
-      }
-      uint32_t* slot = find_or_insert(tbase, cap, is_fwd ? fwd : rc);
-      if (slot) {
-        red_add(slot + o_idx);
-        if (i_idx >= 0) red_add(slot + i_idx);
-      } else {
-        atomicOr(a.status, kStatusTableFull);
-      }
-      if (t + 1 < n) {
-        pred = (int)(uint32_t)(fwd >> top) & 3;
-        fwd = ((fwd << 2) | (Code)succ) & mask;
-        rc = (rc >> 2) | ((Code)(3 - succ) << top);
-      }
+    ok &= upsert(t, is_fwd ? fwd : rc, o, i);
+    if (s + 1 < n) {
+      pred = (int)(uint32_t)(fwd >> top) & 3;
+      fwd = ((fwd << 2) | (Code)succ) & mask;
+      rc = (rc >> 2) | ((Code)(3 - succ) << top);
     }
   }
+  return ok;
 }
 
-struct ExtractArgs {
-  const char* slots;
-  const uint64_t* tab_off;
-  uint64_t slot_base;
-  int pid_begin, pid_end;
+// --------------------------------------------------------------- extraction
+
+struct OutArgs {
   dbg_vertex* out;
   uint64_t out_cap;
   unsigned long long* n_out;
@@ -200,96 +232,295 @@ struct ExtractArgs {
   uint32_t* status;
 };
 
-__device__ __forceinline__ unsigned long long warp_sum(unsigned long long v) {
+struct XShared {
+  typename cub::BlockScan<uint32_t, kThreads>::TempStorage scan;
+  typename cub::BlockReduce<unsigned long long, kThreads>::TempStorage red;
+  unsigned long long base;
+};
+
+// Block-wide: compact the occupied entries among slots [0, n) of a contiguous
+// key/counter range into records; pid_of(local slot) gives the partition.
+// Two passes keep registers low: occupancy bits + block scan, then re-read
+// (L1/L2 hits) and write each occupied entry.
+template <int KW, typename PidFn>
+__device__ __forceinline__ void extract_tile(const char* keys, const uint32_t* ctr, uint64_t n, PidFn pid_of,
+                                             const OutArgs& oa, XShared& sh) {
+  constexpr uint32_t KE = KW == 1 ? 16 : 32;
+  uint32_t bits = 0;
 #pragma unroll
-  for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(kFull, v, d);
-  return v;
+  for (int q = 0; q < kXPer; ++q) {
+    const uint64_t s = (uint64_t)q * kThreads + threadIdx.x;
+    if (s < n && (__ldcg(reinterpret_cast<const uint64_t*>(keys + s * KE)) & kOccupied)) bits |= 1u << q;
+  }
+  const uint32_t cnt = __popc(bits);
+  uint32_t excl, total;
+  cub::BlockScan<uint32_t, kThreads>(sh.scan).ExclusiveSum(cnt, excl, total);
+  if (threadIdx.x == 0) sh.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
+  __syncthreads();
+  uint64_t pos = sh.base + excl;
+  unsigned long long st_count = 0, st_edges = 0, st_sum = 0;
+  while (bits) {
+    const int q = __ffs(bits) - 1;
+    bits &= bits - 1;
+    const uint64_t s = (uint64_t)q * kThreads + threadIdx.x;
+    const uint64_t* kp = reinterpret_cast<const uint64_t*>(keys + s * KE);
+    const uint64_t k0 = __ldcg(kp);
+    dbg_vertex v;
+    uint32_t tout;
+    if (KW == 1) {
+      v.kmer_hi = 0;
+      v.kmer_lo = k0 & kCodeMask;
+      tout = __ldcg(reinterpret_cast<const uint32_t*>(kp + 1));
+    } else {
+      v.kmer_hi = k0 & kCodeMask;
+      v.kmer_lo = __ldcg(kp + 1);
+      tout = __ldcg(reinterpret_cast<const uint32_t*>(kp + 2));
+    }
+    const uint4* cp = reinterpret_cast<const uint4*>(ctr + s * 8);
+    const uint4 a = __ldcg(cp), b = __ldcg(cp + 1);
+    v.out[0] = a.x; v.out[1] = a.y; v.out[2] = a.z; v.out[3] = a.w;
+    v.in[0] = b.x; v.in[1] = b.y; v.in[2] = b.z; v.in[3] = b.w;
+    v.count = a.x + a.y + a.z + a.w + tout;  // count = sum(out) + t_out
+    v.pid = pid_of(s);
+    if (pos < oa.out_cap) oa.out[pos] = v;
+    else atomicOr(oa.status, kStatusNoSpace);
+    ++pos;
+    const uint64_t f[11] = {v.kmer_hi, v.kmer_lo, v.count, a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    uint64_t h = 0;
+#pragma unroll
+    for (int t = 0; t < 11; ++t) h = fmix64(h ^ f[t]);
+    st_sum += h;
+    st_count += v.count;
+    st_edges += (uint64_t)a.x + a.y + a.z + a.w + b.x + b.y + b.z + b.w;
+  }
+  if (total) {  // block-uniform
+    typedef cub::BlockReduce<unsigned long long, kThreads> Red;
+    const unsigned long long c = Red(sh.red).Sum(st_count);
+    __syncthreads();
+    const unsigned long long e = Red(sh.red).Sum(st_edges);
+    __syncthreads();
+    const unsigned long long h = Red(sh.red).Sum(st_sum);
+    if (threadIdx.x == 0) {
+      atomicAdd(oa.stats + 0, (unsigned long long)total);
+      atomicAdd(oa.stats + 1, c);
+      atomicAdd(oa.stats + 2, e);
+      atomicAdd(oa.stats + 3, h);
+    }
+  }
+  __syncthreads();
 }
 
-// Compaction of occupied slots into dbg_vertex records + totals + checksum.
+// Binary search: the partition i in [lo, hi) with off[i] <= x < off[i+1].
+__device__ __forceinline__ int find_part(const uint64_t* __restrict__ off, int lo, int hi, uint64_t x) {
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (__ldg(off + mid) <= x) lo = mid;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// --------------------------------------------------------------- resident tables
+
+struct ResidentArgs {
+  const uint32_t* records;
+  const uint64_t* rec_off;
+  const uint64_t* tab_off;
+  char* table;  // [keys of all slots of [b,e)] [counters of all slots]
+  int pid_begin, pid_end, k;
+  uint32_t* status;
+};
+
+template <typename Code, int R>
+__global__ void __launch_bounds__(kThreads) hash_build_kernel(ResidentArgs a) {
+  constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
+  const uint64_t r_begin = a.rec_off[a.pid_begin], r_end = a.rec_off[a.pid_end];
+  const uint64_t s0 = a.tab_off[a.pid_begin], n_slots = a.tab_off[a.pid_end] - s0;
+  uint32_t* ctr_base = reinterpret_cast<uint32_t*>(a.table + n_slots * KE);
+  for (uint64_t rec = r_begin + (uint64_t)blockIdx.x * kThreads + threadIdx.x; rec < r_end;
+       rec += (uint64_t)gridDim.x * kThreads) {
+    const uint32_t* rp = a.records + rec * R;
+    const uint32_t pid = __ldg(rp) >> 10;
+    const uint64_t t0 = __ldg(a.tab_off + pid) - s0;
+    Table t;
+    t.keys = a.table + t0 * KE;
+    t.ctr = ctr_base + t0 * 8;
+    t.cap = __ldg(a.tab_off + pid + 1) - __ldg(a.tab_off + pid);
+    if (!hash_record<Code, R>(rp, a.k, t)) atomicOr(a.status, kStatusTableFull);
+  }
+}
+
 template <int KW>
-__global__ void __launch_bounds__(256) extract_kernel(ExtractArgs a) {
-  const uint64_t s_begin = a.tab_off[a.pid_begin], s_end = a.tab_off[a.pid_end];
-  const int lane = threadIdx.x & 31;
-  const uint64_t n_iter = (s_end - s_begin + 31) / 32 * 32;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_iter;
-       i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t s = s_begin + i;
-    bool occ = false;
-    dbg_vertex v;
-    if (s < s_end) {
-      const char* sp = a.slots + (s - a.slot_base) * kSlotBytes;
-      const uint4* q = reinterpret_cast<const uint4*>(sp);
-      uint4 x0 = __ldcs(q), x1 = __ldcs(q + 1), x2 = __ldcs(q + 2), x3 = __ldcs(q + 3);
-      uint32_t u[16] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w,
-                        x2.x, x2.y, x2.z, x2.w, x3.x, x3.y, x3.z, x3.w};
-      const uint64_t k0 = ((uint64_t)u[1] << 32) | u[0];
-      if (k0 & kOccupied) {
-        occ = true;
-        int c0;
-        if (KW == 1) {
-          v.kmer_hi = 0;
-          v.kmer_lo = k0 & ~kOccupied;
-          c0 = 2;
-        } else {
-          const uint64_t k1 = ((uint64_t)u[3] << 32) | u[2];
-          const u128 code = ((u128)(k0 & ~kOccupied) << 63) | (u128)(k1 & ~kOccupied);
-          v.kmer_hi = (uint64_t)(code >> 64);
-          v.kmer_lo = (uint64_t)code;
-          c0 = 4;
-        }
-        uint32_t cnt = u[c0 + 8];  // t_out
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          v.out[c] = u[c0 + c];
-          v.in[c] = u[c0 + 4 + c];
-          cnt += v.out[c];
-        }
-        v.count = cnt;  // count = sum(out) + t_out
-        v.pid = (uint32_t)find_part(a.tab_off, a.pid_begin, a.pid_end, s);
+__global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, OutArgs oa) {
+  constexpr uint32_t KE = KW == 1 ? 16 : 32;
+  __shared__ XShared sh;
+  const uint64_t s0 = a.tab_off[a.pid_begin], n_slots = a.tab_off[a.pid_end] - s0;
+  const uint32_t* ctr_base = reinterpret_cast<const uint32_t*>(a.table + n_slots * KE);
+  for (uint64_t t0 = (uint64_t)blockIdx.x * kExtractSlots; t0 < n_slots; t0 += (uint64_t)gridDim.x * kExtractSlots) {
+    const uint64_t n = min((uint64_t)kExtractSlots, n_slots - t0);
+    const int lo = a.pid_begin, hi = a.pid_end;
+    const uint64_t* off = a.tab_off;
+    extract_tile<KW>(a.table + t0 * KE, ctr_base + t0 * 8, n,
+                     [=](uint64_t s) { return (uint32_t)find_part(off, lo, hi, s0 + t0 + s); }, oa, sh);
+  }
+}
+
+// --------------------------------------------------------------- fused Step 2
+
+struct SubgraphArgs {
+  const uint32_t* records;
+  const uint64_t* rec_off;
+  const uint64_t* tab_off;
+  int pid_begin, n_part, k;
+  char* ring;
+  uint64_t region_slots, region_bytes;
+  const unsigned long long* stage_off;  // [n_part + 3]
+  unsigned long long* work;             // claimed-item counter
+  uint32_t* done;                       // [3][n_part]: zero, hash, extract items done
+};
+
+__device__ __forceinline__ uint64_t div_up(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+struct PartGeom {
+  uint64_t cap, rec0, nrec;
+};
+__device__ __forceinline__ PartGeom geom(const SubgraphArgs& a, int p) {
+  PartGeom g;
+  const int pid = a.pid_begin + p;
+  g.cap = a.tab_off[pid + 1] - a.tab_off[pid];
+  g.rec0 = a.rec_off[pid];
+  g.nrec = a.rec_off[pid + 1] - g.rec0;
+  return g;
+}
+
+// Single CTA: stage offsets of the work list and zeroed completion counters.
+// Stage s holds: zero items of partition s, hash items of s-1, extract items of s-2.
+__global__ void __launch_bounds__(kThreads) subgraph_plan_kernel(SubgraphArgs a, uint32_t* status) {
+  typedef cub::BlockScan<unsigned long long, kThreads> Scan;
+  __shared__ typename Scan::TempStorage tmp;
+  __shared__ unsigned long long carry;
+  for (int i = threadIdx.x; i < 3 * a.n_part; i += kThreads) a.done[i] = 0;
+  if (threadIdx.x == 0) {
+    carry = 0;
+    *a.work = 0;
+  }
+  __syncthreads();
+  const int n_stage = a.n_part + 2;
+  unsigned long long* so = const_cast<unsigned long long*>(a.stage_off);
+  for (int base = 0; base < n_stage; base += kThreads) {
+    const int s = base + threadIdx.x;
+    unsigned long long items = 0;
+    if (s < n_stage) {
+      if (s < a.n_part) {
+        const PartGeom g = geom(a, s);
+        if (g.cap > a.region_slots) atomicOr(status, kStatusRing);
+        items += div_up(g.cap, kZeroSlots);
       }
+      if (s >= 1 && s - 1 < a.n_part) items += div_up(geom(a, s - 1).nrec, kHashRecs);
+      if (s >= 2) items += div_up(geom(a, s - 2).cap, kExtractSlots);
     }
-    const uint32_t ballot = __ballot_sync(kFull, occ);
-    unsigned long long base = 0;
-    if (ballot) {
-      if (lane == 0) base = atomicAdd(a.n_out, (unsigned long long)__popc(ballot));
-      base = __shfl_sync(kFull, base, 0);
+    unsigned long long excl, total;
+    Scan(tmp).ExclusiveSum(items, excl, total);
+    if (s < n_stage) so[s] = carry + excl;
+    __syncthreads();
+    if (threadIdx.x == 0) carry += total;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) so[n_stage] = carry;
+}
+
+__device__ __forceinline__ void wait_count(const uint32_t* p, uint32_t need) {
+  if (need == 0) return;
+  while (ld_acquire32(p) < need) __nanosleep(64);
+}
+
+template <typename Code, int R>
+__global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, OutArgs oa) {
+  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
+  constexpr uint32_t KE = KW == 1 ? 16 : 32;
+  __shared__ XShared sh;
+  __shared__ unsigned long long s_item;
+  const int n_stage = a.n_part + 2;
+  const unsigned long long total = a.stage_off[n_stage];
+  uint32_t* done_z = a.done;
+  uint32_t* done_h = a.done + a.n_part;
+  uint32_t* done_x = a.done + 2 * a.n_part;
+  for (;;) {
+    if (threadIdx.x == 0) s_item = atomicAdd(a.work, 1ull);
+    __syncthreads();
+    const unsigned long long item = s_item;
+    __syncthreads();
+    if (item >= total) break;
+    // locate the stage (binary search over n_stage + 1 offsets)
+    int lo = 0, hi = n_stage;
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (a.stage_off[mid] <= item) lo = mid;
+      else hi = mid;
     }
-    unsigned long long st_count = 0, st_edges = 0, st_sum = 0;
-    if (occ) {
-      const uint64_t pos = base + __popc(ballot & ((1u << lane) - 1u));
-      if (pos < a.out_cap) a.out[pos] = v;
-      else atomicOr(a.status, kStatusNoSpace);
-      st_count = v.count;
-      uint64_t f[11] = {v.kmer_hi, v.kmer_lo, v.count, v.out[0], v.out[1], v.out[2], v.out[3],
-                        v.in[0], v.in[1], v.in[2], v.in[3]};
-      uint64_t h = 0;
-#pragma unroll
-      for (int t = 0; t < 11; ++t) {
-        h = fmix64(h ^ f[t]);
-        if (t >= 3) st_edges += f[t];
+    const int s = lo;
+    uint64_t j = item - a.stage_off[s];
+    int kind = -1, p = -1;
+    PartGeom g;
+    if (s < a.n_part) {
+      g = geom(a, s);
+      const uint64_t nz = div_up(g.cap, kZeroSlots);
+      if (j < nz) kind = 0, p = s;
+      else j -= nz;
+    }
+    if (kind < 0 && s >= 1 && s - 1 < a.n_part) {
+      g = geom(a, s - 1);
+      const uint64_t nh = div_up(g.nrec, kHashRecs);
+      if (j < nh) kind = 1, p = s - 1;
+      else j -= nh;
+    }
+    if (kind < 0) {
+      kind = 2;
+      p = s - 2;
+      g = geom(a, p);
+    }
+    char* keys = a.ring + (uint64_t)(p % kRing) * a.region_bytes;
+    uint32_t* ctr = reinterpret_cast<uint32_t*>(keys + a.region_slots * KE);
+    // dependencies: region reuse, zero-before-hash, hash-before-extract
+    if (threadIdx.x == 0) {
+      if (kind == 0 && p >= kRing) wait_count(done_x + p - kRing, (uint32_t)div_up(geom(a, p - kRing).cap, kExtractSlots));
+      if (kind == 1) wait_count(done_z + p, (uint32_t)div_up(g.cap, kZeroSlots));
+      if (kind == 2) wait_count(done_h + p, (uint32_t)div_up(g.nrec, kHashRecs));
+    }
+    __syncthreads();
+    if (kind == 0) {
+      const uint64_t s0 = j * kZeroSlots, s1 = min(g.cap, s0 + kZeroSlots);
+      uint4* z = reinterpret_cast<uint4*>(keys + s0 * KE);
+      const uint64_t n16 = (s1 - s0) * (KE / 16);
+      for (uint64_t q = threadIdx.x; q < n16; q += kThreads) __stcg(z + q, make_uint4(0, 0, 0, 0));
+    } else if (kind == 1) {
+      const uint64_t r = j * kHashRecs + threadIdx.x;
+      if (r < g.nrec) {
+        Table t;
+        t.keys = keys;
+        t.ctr = ctr;
+        t.cap = g.cap;
+        if (!hash_record<Code, R>(a.records + (g.rec0 + r) * R, a.k, t)) atomicOr(oa.status, kStatusTableFull);
       }
-      st_sum = h;
+    } else {
+      const uint64_t s0 = j * kExtractSlots;
+      const uint64_t n = min((uint64_t)kExtractSlots, g.cap - s0);
+      const uint32_t pid = (uint32_t)(a.pid_begin + p);
+      extract_tile<KW>(keys + s0 * KE, ctr + s0 * 8, n, [=](uint64_t) { return pid; }, oa, sh);
     }
-    if (ballot) {
-      st_count = warp_sum(st_count);
-      st_edges = warp_sum(st_edges);
-      st_sum = warp_sum(st_sum);
-      if (lane == 0) {
-        atomicAdd(a.stats + 0, (unsigned long long)__popc(ballot));
-        atomicAdd(a.stats + 1, st_count);
-        atomicAdd(a.stats + 2, st_edges);
-        atomicAdd(a.stats + 3, st_sum);
-      }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atomicAdd(kind == 0 ? done_z + p : kind == 1 ? done_h + p : done_x + p, 1u);
     }
   }
 }
 
+// --------------------------------------------------------------- sort
+
 __global__ void sort_prepare_kernel(const dbg_vertex* __restrict__ in, uint64_t n,
-                                    unsigned long long* __restrict__ key,
-                                    unsigned long long* __restrict__ idx) {
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (uint64_t)gridDim.x * blockDim.x) {
+                                    unsigned long long* __restrict__ key, unsigned long long* __restrict__ idx) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     key[i] = in[i].kmer_lo;
     idx[i] = i;
   }
@@ -298,16 +529,13 @@ __global__ void sort_prepare_kernel(const dbg_vertex* __restrict__ in, uint64_t 
 __global__ void sort_gather_hi_kernel(const dbg_vertex* __restrict__ in, uint64_t n,
                                       const unsigned long long* __restrict__ idx,
                                       unsigned long long* __restrict__ key) {
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (uint64_t)gridDim.x * blockDim.x)
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     key[i] = in[idx[i]].kmer_hi;
 }
 
 __global__ void sort_gather_kernel(const dbg_vertex* __restrict__ in, uint64_t n,
-                                   const unsigned long long* __restrict__ idx,
-                                   dbg_vertex* __restrict__ out) {
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (uint64_t)gridDim.x * blockDim.x)
+                                   const unsigned long long* __restrict__ idx, dbg_vertex* __restrict__ out) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     out[i] = in[idx[i]];
 }
 
@@ -315,75 +543,122 @@ __global__ void sort_gather_kernel(const dbg_vertex* __restrict__ in, uint64_t n
 
 using namespace dbg;
 
-static int sm_count_h() {
-  int dev = 0, n = 148;
-  if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-  return n;
-}
+extern "C" uint32_t dbg_key_bytes(const dbg_params* prm) { return prm ? key_bytes(prm->k) : 0u; }
 
-static bool hash_params_ok(const dbg_params* prm) {
-  return prm && prm->k >= 1 && prm->k <= 63 && (prm->k & 1) && prm->p >= 1 && prm->p <= prm->k &&
-         prm->p <= 31 && prm->num_partitions >= 1 && (uint32_t)prm->num_partitions <= kMaxPid;
-}
+extern "C" uint32_t dbg_slot_bytes(const dbg_params* prm) { return prm ? key_bytes(prm->k) + kCtrBytes : 0u; }
 
-extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set* part,
-                                     int32_t pid_begin, int32_t pid_end, void* d_slots,
-                                     const uint64_t* d_table_offset, uint64_t slot_base,
+extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                                     int32_t pid_end, void* d_table, const uint64_t* d_table_offset,
                                      uint32_t* d_status, cudaStream_t stream) {
-  if (!hash_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_slots ||
+  if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table ||
       !d_table_offset || !d_status)
     return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
-  HashArgs a;
+  ResidentArgs a;
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
   a.tab_off = d_table_offset;
-  a.slot_base = slot_base;
-  a.slots = static_cast<char*>(d_slots);
-  a.status = d_status;
+  a.table = static_cast<char*>(d_table);
   a.pid_begin = pid_begin;
   a.pid_end = pid_end;
   a.k = prm->k;
-  const int grid = sm_count_h() * 8;  // 8 CTAs x 256 threads = 64 warps per SM
-  if (prm->k <= 31) hash_build_kernel<1, 4><<<grid, kHashThreads, 0, stream>>>(a);
-  else if (prm->k <= 39) hash_build_kernel<2, 4><<<grid, kHashThreads, 0, stream>>>(a);
-  else hash_build_kernel<2, 8><<<grid, kHashThreads, 0, stream>>>(a);
+  a.status = d_status;
+  const int grid = dbg_sm_count() * 8;
+  if (prm->k <= 31) hash_build_kernel<uint64_t, 4><<<grid, kThreads, 0, stream>>>(a);
+  else if (prm->k <= 39) hash_build_kernel<u128, 4><<<grid, kThreads, 0, stream>>>(a);
+  else hash_build_kernel<u128, 8><<<grid, kThreads, 0, stream>>>(a);
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_slots,
-                                        const uint64_t* d_table_offset, uint64_t slot_base,
-                                        int32_t pid_begin, int32_t pid_end, dbg_vertex* d_out,
-                                        uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
-                                        uint32_t* d_status, cudaStream_t stream) {
-  if (!hash_params_ok(prm) || !d_slots || !d_table_offset || !d_n_out || !d_stats || !d_status ||
+extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_table, const uint64_t* d_table_offset,
+                                        int32_t pid_begin, int32_t pid_end, dbg_vertex* d_out, uint64_t out_cap,
+                                        uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
+                                        cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !d_table || !d_table_offset || !d_n_out || !d_stats || !d_status ||
       (out_cap && !d_out))
     return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
-  ExtractArgs a;
-  a.slots = static_cast<const char*>(d_slots);
+  ResidentArgs a;
+  a.records = nullptr;
+  a.rec_off = nullptr;
   a.tab_off = d_table_offset;
-  a.slot_base = slot_base;
+  a.table = static_cast<char*>(const_cast<void*>(d_table));
   a.pid_begin = pid_begin;
   a.pid_end = pid_end;
-  a.out = d_out;
-  a.out_cap = out_cap;
-  a.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
-  a.stats = reinterpret_cast<unsigned long long*>(d_stats);
+  a.k = prm->k;
   a.status = d_status;
-  const int grid = sm_count_h() * 8;
-  if (prm->k <= 31) extract_kernel<1><<<grid, 256, 0, stream>>>(a);
-  else extract_kernel<2><<<grid, 256, 0, stream>>>(a);
+  OutArgs oa;
+  oa.out = d_out;
+  oa.out_cap = out_cap;
+  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
+  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
+  oa.status = d_status;
+  const int grid = dbg_sm_count() * 4;
+  if (prm->k <= 31) extract_kernel<1><<<grid, kThreads, 0, stream>>>(a, oa);
+  else extract_kernel<2><<<grid, kThreads, 0, stream>>>(a, oa);
+  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+}
+
+extern "C" uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions) {
+  (void)prm;
+  const uint64_t n = n_partitions > 0 ? (uint64_t)n_partitions : 1;
+  return 8 * (n + 3) + 8 + 4 * 3 * n + 64;
+}
+
+extern "C" uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t max_capacity) {
+  if (!prm) return 0;
+  return (uint64_t)kRing * max_capacity * (key_bytes(prm->k) + kCtrBytes);
+}
+
+extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                                          int32_t pid_end, const uint64_t* d_table_offset, void* d_ring,
+                                          uint64_t ring_bytes, void* d_workspace, uint64_t workspace_bytes,
+                                          dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
+                                          dbg_stats* d_stats, uint32_t* d_status, cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table_offset ||
+      !d_ring || !d_workspace || !d_n_out || !d_stats || !d_status || (out_cap && !d_out))
+    return DBG_EINVAL;
+  if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
+  const int n_part = pid_end - pid_begin;
+  if (n_part == 0) return DBG_OK;
+  if (workspace_bytes < dbg_subgraph_workspace_bytes(prm, n_part)) return DBG_EINVAL;
+  const uint64_t slot = key_bytes(prm->k) + kCtrBytes;
+  SubgraphArgs a;
+  a.records = part->d_records;
+  a.rec_off = part->d_record_offset;
+  a.tab_off = d_table_offset;
+  a.pid_begin = pid_begin;
+  a.n_part = n_part;
+  a.k = prm->k;
+  a.ring = static_cast<char*>(d_ring);
+  a.region_slots = ring_bytes / kRing / slot;
+  a.region_slots &= ~(uint64_t)63;  // keep regions 64 B x 64 aligned
+  a.region_bytes = a.region_slots * slot;
+  if (a.region_slots == 0) return DBG_EINVAL;
+  char* ws = static_cast<char*>(d_workspace);
+  a.stage_off = reinterpret_cast<unsigned long long*>(ws);
+  a.work = reinterpret_cast<unsigned long long*>(ws + 8 * (n_part + 3));
+  a.done = reinterpret_cast<uint32_t*>(ws + 8 * (n_part + 3) + 8);
+  OutArgs oa;
+  oa.out = d_out;
+  oa.out_cap = out_cap;
+  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
+  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
+  oa.status = d_status;
+  subgraph_plan_kernel<<<1, kThreads, 0, stream>>>(a, d_status);
+  const int grid = dbg_sm_count() * 4;
+  if (prm->k <= 31) subgraph_kernel<uint64_t, 4><<<grid, kThreads, 0, stream>>>(a, oa);
+  else if (prm->k <= 39) subgraph_kernel<u128, 4><<<grid, kThreads, 0, stream>>>(a, oa);
+  else subgraph_kernel<u128, 8><<<grid, kThreads, 0, stream>>>(a, oa);
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
 static size_t cub_sort_bytes(uint64_t n) {
   size_t bytes = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, bytes, (unsigned long long*)nullptr,
-                                  (unsigned long long*)nullptr, (unsigned long long*)nullptr,
-                                  (unsigned long long*)nullptr, (int64_t)n, 0, 64);
+  cub::DeviceRadixSort::SortPairs(nullptr, bytes, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
+                                  (unsigned long long*)nullptr, (unsigned long long*)nullptr, (int64_t)n, 0, 64);
   return bytes;
 }
 
@@ -394,11 +669,9 @@ extern "C" uint64_t dbg_sort_workspace_bytes(const dbg_params* prm, uint64_t n) 
   return 4 * align256(8 * (n ? n : 1)) + align256(cub_sort_bytes(n ? n : 1));
 }
 
-extern "C" dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_in,
-                                        dbg_vertex* d_out, uint64_t n, void* d_workspace,
-                                        uint64_t workspace_bytes, cudaStream_t stream) {
-  if (!hash_params_ok(prm) || (n && (!d_in || !d_out || !d_workspace)) || d_in == d_out)
-    return DBG_EINVAL;
+extern "C" dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_in, dbg_vertex* d_out, uint64_t n,
+                                        void* d_workspace, uint64_t workspace_bytes, cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || (n && (!d_in || !d_out || !d_workspace)) || d_in == d_out) return DBG_EINVAL;
   if (n == 0) return DBG_OK;
   if (workspace_bytes < dbg_sort_workspace_bytes(prm, n)) return DBG_EINVAL;
   char* ws = static_cast<char*>(d_workspace);
@@ -409,18 +682,17 @@ extern "C" dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex*
   unsigned long long* i1 = reinterpret_cast<unsigned long long*>(ws + 3 * arr);
   void* tmp = ws + 4 * arr;
   size_t tmp_bytes = workspace_bytes - 4 * arr;
-  const int grid = sm_count_h() * 4;
+  const int grid = dbg_sm_count() * 4;
   sort_prepare_kernel<<<grid, 256, 0, stream>>>(d_in, n, k0, i0);
   const int k = prm->k;
   const int lo_bits = k <= 31 ? 2 * k : 64;
-  if (cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k0, k1, i0, i1, (int64_t)n, 0, lo_bits,
-                                      stream) != cudaSuccess)
+  if (cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k0, k1, i0, i1, (int64_t)n, 0, lo_bits, stream) != cudaSuccess)
     return DBG_ECUDA;
   unsigned long long* idx = i1;
   if (k > 31) {  // LSD: then a stable sort by the high word
     sort_gather_hi_kernel<<<grid, 256, 0, stream>>>(d_in, n, i1, k0);
-    if (cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k0, k1, i1, i0, (int64_t)n, 0,
-                                        2 * k - 64, stream) != cudaSuccess)
+    if (cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k0, k1, i1, i0, (int64_t)n, 0, 2 * k - 64, stream) !=
+        cudaSuccess)
       return DBG_ECUDA;
     idx = i0;
   }

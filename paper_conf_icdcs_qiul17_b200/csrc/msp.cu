@@ -1,163 +1,266 @@
 // msp.cu -- Step 1 of ParaHash on sm_100a: MSP graph partitioning
 // (Sec. III-B; Defs. 1-2), kernel (a) of the north star.
 //
-// One warp scans one read at a time in chunks of 32 K-mers (lane t <-> K-mer
-// i0+t).  For the chunk, the canonical value of every P-mer it needs
-// (c_j = min(code(s_j), code(rc(s_j))), readings A/D/E) is computed by the
-// lanes from the 2-bit stream (two u64 loads + funnel shift + bit-reverse)
-// into a per-warp shared-memory row; each lane then takes the minimum over
-// its window of w = K-P+1 values (Def. 1).  Superkmer boundaries (Def. 2,
-// reading G: maximal runs of equal minimizer) come from a warp ballot; the
-// lane that sees a boundary emits the superkmer that closes there.  The
-// partition id is fmix64(m) mod NP (reading I).
+// Pass 1, msp_kernel: one thread scans one read (32 consecutive reads per
+// warp, so the 2-bit words a warp loads are contiguous).  Per base it rolls
+// the forward and reverse-complement codes of the current P-mer, takes the
+// canonical value c_q = min(code, rc code) (readings A, D, E) and feeds it to
+// a sliding-window minimum over w = K-P+1 P-mers (Definition 1: the
+// P-minimum-substring of K-mer i is min c_q over q in [i, i+K-P]).  The window
+// minimum is van Herk / Gil-Werman: blocks of w values, a running prefix
+// minimum of the current block and the suffix minima of the previous block,
+// kept in place in one per-thread shared-memory row -- O(1) per base and no
+// divergence across the lanes of a warp.  A superkmer (Def. 2, reading G) is
+// a maximal run of K-mers with equal minimizer; each is appended as a
+// descriptor (start, end, minimizer) to a per-thread shared-memory list.
+// When any list fills (or the reads end) the warp flushes: pid = fmix64(m)
+// mod NP (reading I) via a precomputed 64-bit reciprocal, a warp scan sizes
+// the records, one atomicAdd reserves a contiguous staging range, and each
+// lane writes its fixed-width records (dbg.h) with the two adjacency bases
+// (Sec. III-B).  Per-partition record/K-mer histograms are kept in
+// shared memory and flushed once per CTA (N^i_kmer).
 //
-// The paper left superkmer generation ("memory movement of irregular
-// lengths") to the CPU; here the same kernel emits fixed-width
-// records (dbg.h) straight into the per-partition HBM buffers: a count pass
-// sizes them (per-partition histograms in shared memory, P:L972-975's
-// prefix sum of superkmer lengths gives N^i_kmer), a scan turns sizes into
-// offsets, and an emit pass writes the records.
+// The paper computed only "superkmer ids and offsets" on the GPU and left
+// the irregular copy to the CPU; here both run in this kernel.
+//
+// Pass 2, scan_kernel: record offsets per partition (exclusive prefix sum).
+// Pass 3, scatter_kernel: counting-sort scatter of the staged records into
+// their partitions' contiguous ranges (CTA histogram -> one global
+// reservation per partition per tile).
 #include <cub/block/block_scan.cuh>
 
 #include "dbg_device.cuh"
 
 namespace dbg {
 
-constexpr int kMspWarps = 8;
-constexpr int kMspThreads = kMspWarps * kWarp;
-constexpr int kCbuf = 96;  // >= 32 + w - 1 for w <= 63, padded
-constexpr int kSmemHistMaxNp = 4096;
+constexpr int kMspThreads = 128;
+constexpr int kMaxDesc = 12;             // descriptors per thread between flushes
+constexpr int kSmemHistMaxNp = 8192;
+
+// Unsigned 64-bit division by an invariant integer (Granlund & Montgomery
+// 1994, Fig. 4.1): exact x mod d for every 64-bit x, d >= 1.
+struct FastMod {
+  uint64_t d, m;
+  int sh1, sh2;
+};
+
+static FastMod make_fastmod(uint64_t d) {
+  int l = 0;
+  while (l < 64 && (1ull << l) < d) ++l;  // l = ceil(log2 d)
+  FastMod f;
+  f.d = d;
+  const unsigned __int128 two_l = (unsigned __int128)1 << l;
+  f.m = (uint64_t)((((unsigned __int128)1 << 64) * (two_l - d)) / d + 1);
+  f.sh1 = l < 1 ? l : 1;
+  f.sh2 = l - 1 > 0 ? l - 1 : 0;
+  return f;
+}
+
+__device__ __forceinline__ uint32_t fast_mod(const FastMod& f, uint64_t x) {
+  const uint64_t t1 = __umul64hi(f.m, x);
+  const uint64_t q = (t1 + ((x - t1) >> f.sh1)) >> f.sh2;
+  return (uint32_t)(x - q * f.d);
+}
 
 struct MspArgs {
   const uint64_t* words;
   uint64_t n_words;
   const uint64_t* offsets;
   uint64_t n_reads;
-  int k, p, np;
+  int k, p, np, w;
   uint32_t rec_words, max_kmers;
-  unsigned long long* n_records;  // [np] (count mode)
-  unsigned long long* n_kmers;    // [np] (count mode)
-  const uint64_t* rec_off;        // [np+1] (emit mode)
-  unsigned long long* fill;       // [np]   (emit mode)
-  uint32_t* records;              // (emit mode)
+  FastMod mod;
+  unsigned long long* n_records;  // [np]
+  unsigned long long* n_kmers;    // [np]
+  uint32_t* staging;              // records in read order
+  uint64_t staging_cap;           // records
+  unsigned long long* staged;     // cursor (records reserved)
 };
 
-// Canonical P-mer value at stream position pos (Def. 1 with readings A/D).
-__device__ __forceinline__ uint64_t canon_pmer(const MspArgs& a, uint64_t pos) {
-  uint64_t f = window64(a.words, a.n_words, pos) >> (64 - 2 * a.p);
-  uint64_t r = revcomp64(f, a.p);
-  return f < r ? f : r;
+template <typename CT>
+struct MspSmem {
+  // row[t * kMspThreads + tid], t < w: the van Herk block (in place)
+  // desc_se[d * kMspThreads + tid] = start | end << 32; desc_m = minimizer
+  CT* row;
+  unsigned long long* desc_se;
+  unsigned long long* desc_m;
+  uint32_t* hist_rec;
+  uint32_t* hist_kmer;
+};
+
+// Writes one record (dbg.h layout) for K-mers [ps, pe] of the read at stream
+// offset o, length L.
+__device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, uint64_t o, int64_t L,
+                                             int64_t ps, int64_t pe, uint32_t pid) {
+  const uint32_t hl = ps > 0 ? 1u : 0u;  // reading H
+  const uint32_t hr = pe + a.k < L ? 1u : 0u;
+  const int64_t bs = ps - hl;
+  const int64_t nb = (int64_t)hl + (pe - ps + 1) + a.k - 1 + hr;
+  uint32_t w[8];
+  w[0] = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
+#pragma unroll
+  for (int q = 0; q < 7; q += 2) {  // two 16-base words per 64-bit window
+    uint64_t v = 0;
+    const int64_t left = nb - 16 * q;
+    if (q + 1 < (int)a.rec_words && left > 0) {
+      v = window64(a.words, a.n_words, o + bs + 16 * q);
+      if (left < 32) v &= ~(~0ull >> (2 * left));  // zero the bases past the record
+    }
+    w[q + 1] = (uint32_t)(v >> 32);
+    if (q + 2 < 8) w[q + 2] = (uint32_t)v;
+  }
+  uint4* d4 = reinterpret_cast<uint4*>(dst);
+  d4[0] = make_uint4(w[0], w[1], w[2], w[3]);
+  if (a.rec_words == 8) d4[1] = make_uint4(w[4], w[5], w[6], w[7]);
 }
 
-// Writes the pieces of superkmer [s, e] (K-mer start positions within the
-// read at stream offset o of length L) into partition pid (emit mode), or
-// counts them (count mode).
-template <bool kEmit>
-__device__ __forceinline__ void emit_superkmer(const MspArgs& a, uint64_t o, int64_t L, int64_t s,
-                                               int64_t e, uint32_t pid, unsigned long long* sh_rec,
-                                               unsigned long long* sh_kmer) {
-  const int64_t n = e - s + 1;
+// Warp-collective flush of the per-thread descriptor lists.
+template <typename CT>
+__device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
+                                                  uint64_t o, int64_t L) {
+  const int tid = threadIdx.x, lane = tid & 31;
   const int64_t nmax = a.max_kmers;
-  const uint64_t pieces = (uint64_t)((n + nmax - 1) / nmax);
-  if (!kEmit) {
-    if (sh_rec) {
-      atomicAdd(sh_rec + pid, (unsigned long long)pieces);
-      atomicAdd(sh_kmer + pid, (unsigned long long)n);
+  uint32_t my_records = 0;
+  for (int d = 0; d < ndesc; ++d) {
+    const unsigned long long se = sm.desc_se[d * kMspThreads + tid];
+    const int64_t n = (int64_t)(se >> 32) - (int64_t)(se & 0xffffffffu) + 1;
+    my_records += (uint32_t)((n + nmax - 1) / nmax);
+  }
+  uint32_t incl = my_records;
+#pragma unroll
+  for (int dlt = 1; dlt < 32; dlt <<= 1) {
+    const uint32_t v = __shfl_up_sync(kFull, incl, dlt);
+    if (lane >= dlt) incl += v;
+  }
+  const uint32_t total = __shfl_sync(kFull, incl, 31);
+  unsigned long long base = 0;
+  if (total) {
+    if (lane == 0) base = atomicAdd(a.staged, (unsigned long long)total);
+    base = __shfl_sync(kFull, base, 0);
+  }
+  uint64_t slot = base + incl - my_records;
+  for (int d = 0; d < ndesc; ++d) {
+    const unsigned long long se = sm.desc_se[d * kMspThreads + tid];
+    const int64_t s = (int64_t)(se & 0xffffffffu), e = (int64_t)(se >> 32);
+    const uint64_t m = (uint64_t)sm.desc_m[d * kMspThreads + tid];
+    const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
+    const int64_t n = e - s + 1;
+    const uint32_t pieces = (uint32_t)((n + nmax - 1) / nmax);
+    if (sm.hist_rec) {
+      atomicAdd(sm.hist_rec + pid, pieces);
+      atomicAdd(sm.hist_kmer + pid, (uint32_t)n);
     } else {
       atomicAdd(a.n_records + pid, (unsigned long long)pieces);
       atomicAdd(a.n_kmers + pid, (unsigned long long)n);
     }
-    return;
-  }
-  uint64_t slot = a.rec_off[pid] + atomicAdd(a.fill + pid, (unsigned long long)pieces);
-  for (int64_t ps = s; ps <= e; ps += nmax, ++slot) {
-    const int64_t pe = min(e, ps + nmax - 1);
-    const uint32_t hl = ps > 0 ? 1u : 0u;                 // reading H
-    const uint32_t hr = pe + a.k < L ? 1u : 0u;
-    const int64_t bs = ps - hl;
-    const int64_t nb = (int64_t)hl + (pe - ps + 1) + a.k - 1 + hr;
-    uint32_t w[8];
-    w[0] = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
-#pragma unroll
-    for (int q = 0; q < 7; ++q) {
-      if (q + 1 < (int)a.rec_words) {
-        int64_t left = nb - 16 * q;  // bases still to place
-        uint32_t v = 0;
-        if (left > 0) {
-          v = (uint32_t)(window64(a.words, a.n_words, o + bs + 16 * q) >> 32);
-          if (left < 16) v &= ~(0xffffffffu >> (2 * left));  // zero the bases past the record
-        }
-        w[q + 1] = v;
-      }
+    for (int64_t ps = s; ps <= e; ps += nmax, ++slot) {
+      if (slot < a.staging_cap)
+        write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
     }
-    uint4* dst = reinterpret_cast<uint4*>(a.records + slot * a.rec_words);
-    dst[0] = make_uint4(w[0], w[1], w[2], w[3]);
-    if (a.rec_words == 8) dst[1] = make_uint4(w[4], w[5], w[6], w[7]);
   }
+  ndesc = 0;
 }
 
-template <bool kEmit>
+template <typename CT>
 __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
-  extern __shared__ unsigned long long smem[];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint64_t* cbuf = reinterpret_cast<uint64_t*>(smem) + warp * kCbuf;
-  unsigned long long* sh_rec = nullptr;
-  unsigned long long* sh_kmer = nullptr;
-  const bool smem_hist = !kEmit && a.np <= kSmemHistMaxNp;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int tid = threadIdx.x, lane = tid & 31;
+  MspSmem<CT> sm;
+  unsigned char* sp = smem_raw;
+  sm.desc_se = reinterpret_cast<unsigned long long*>(sp);
+  sp += sizeof(unsigned long long) * kMaxDesc * kMspThreads;
+  sm.desc_m = reinterpret_cast<unsigned long long*>(sp);
+  sp += sizeof(unsigned long long) * kMaxDesc * kMspThreads;
+  sm.row = reinterpret_cast<CT*>(sp);
+  sp += sizeof(CT) * a.w * kMspThreads;
+  sp = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sp) + 15) & ~uintptr_t(15));
+  const bool smem_hist = a.np <= kSmemHistMaxNp;
+  sm.hist_rec = smem_hist ? reinterpret_cast<uint32_t*>(sp) : nullptr;
+  sm.hist_kmer = smem_hist ? sm.hist_rec + a.np : nullptr;
   if (smem_hist) {
-    sh_rec = smem + kMspWarps * kCbuf;
-    sh_kmer = sh_rec + a.np;
-    for (int i = threadIdx.x; i < 2 * a.np; i += blockDim.x) sh_rec[i] = 0;
-    __syncthreads();
+    for (int i = tid; i < 2 * a.np; i += kMspThreads) sm.hist_rec[i] = 0;
   }
-  const int K = a.k;
-  const int w = a.k - a.p + 1;  // P-mers per K-mer window (Def. 1: j in [i, i+K-P])
-  const uint64_t n_warps = (uint64_t)gridDim.x * kMspWarps;
-  for (uint64_t r = (uint64_t)blockIdx.x * kMspWarps + warp; r < a.n_reads; r += n_warps) {
-    const uint64_t o = a.offsets[r];
-    const int64_t L = (int64_t)(a.offsets[r + 1] - o);
-    if (L < K) continue;  // reading N
-    const int64_t nk = L - K + 1;
-    const int64_t npm = L - a.p + 1;  // P-mers in the read
-    int64_t s_open = 0;               // start of the superkmer still open
-    uint64_t m_carry = 0;             // minimizer of K-mer i0-1
-    for (int64_t i0 = 0; i0 < nk; i0 += 32) {
-      const int jn = (int)(npm - i0 < (int64_t)(32 + w - 1) ? npm - i0 : (int64_t)(32 + w - 1));
-      for (int t = lane; t < jn; t += 32) cbuf[t] = canon_pmer(a, o + i0 + t);
-      __syncwarp();
-      const int64_t i = i0 + lane;
-      const bool valid = i < nk;
-      uint64_t m = ~0ull;
-      if (valid)
-        for (int d = 0; d < w; ++d) m = min(m, cbuf[lane + d]);
-      __syncwarp();
-      uint64_t mp = __shfl_up_sync(kFull, m, 1);
-      if (lane == 0) mp = m_carry;
-      const bool is_start = valid && (i == 0 || m != mp);
-      const uint32_t starts = __ballot_sync(kFull, is_start);
-      // (1) the superkmer that closes at K-mer i-1, emitted by the lane starting the next one
-      if (is_start && i > 0) {
-        const uint32_t below = starts & ((1u << lane) - 1u);
-        const int64_t s = below ? i0 + 31 - __clz(below) : s_open;
-        emit_superkmer<kEmit>(a, o, L, s, i - 1, (uint32_t)(fmix64(mp) % (uint64_t)a.np), sh_rec,
-                              sh_kmer);
-      }
-      // (2) the read's last superkmer, emitted by the lane holding the last K-mer
-      if (valid && i == nk - 1) {
-        const uint32_t upto = starts & (lane == 31 ? kFull : ((2u << lane) - 1u));
-        const int64_t s = upto ? i0 + 31 - __clz(upto) : s_open;
-        emit_superkmer<kEmit>(a, o, L, s, i, (uint32_t)(fmix64(m) % (uint64_t)a.np), sh_rec,
-                              sh_kmer);
-      }
-      if (starts) s_open = i0 + 31 - __clz(starts);
-      m_carry = __shfl_sync(kFull, m, 31);
+  __syncthreads();
+
+  const int K = a.k, P = a.p, w = a.w;
+  const CT maskP = (CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1));
+  const int topP = 2 * P - 2;
+  const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
+  CT* row = sm.row + tid;
+  // all lanes of a warp iterate together; a warp covers 32 consecutive reads
+  for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
+    const uint64_t r = r0 + lane;
+    uint64_t o = 0;
+    int64_t L = 0;
+    if (r < a.n_reads) {
+      o = a.offsets[r];
+      L = (int64_t)(a.offsets[r + 1] - o);
     }
+    const int64_t nk = L - K + 1;
+    int64_t Lmax = L;
+#pragma unroll
+    for (int dlt = 16; dlt; dlt >>= 1) Lmax = max(Lmax, (int64_t)__shfl_xor_sync(kFull, (long long)Lmax, dlt));
+    int ndesc = 0;
+    CT f = 0, rc = 0, pre = 0;
+    uint64_t m_cur = 0;
+    int64_t s_start = 0;
+    int u = 0;  // position within the current van Herk block
+    uint64_t wbuf = 0;
+    for (int64_t j = 0; j < Lmax; ++j) {
+      if (j < L && nk > 0) {
+        if ((j & 31) == 0) wbuf = window64(a.words, a.n_words, o + j);
+        const uint32_t b = (uint32_t)(wbuf >> 62);
+        wbuf <<= 2;
+        f = ((f << 2) | (CT)b) & maskP;
+        rc = (rc >> 2) | ((CT)(3u - b) << topP);
+        if (j >= P - 1) {
+          const int64_t q = j - P + 1;  // P-mer index
+          const CT c = f < rc ? f : rc;
+          const CT snext = (u + 1 < w) ? row[(u + 1) * kMspThreads] : (CT)0;
+          row[u * kMspThreads] = c;
+          pre = (u == 0) ? c : (c < pre ? c : pre);
+          if (q >= w - 1) {  // K-mer i = q-w+1 is complete
+            const int64_t i = q - w + 1;
+            const CT mm = (u == w - 1) ? pre : (snext < pre ? snext : pre);
+            const uint64_t m = (uint64_t)mm;
+            if (i == 0) {
+              m_cur = m;
+              s_start = 0;
+            } else if (m != m_cur) {
+              sm.desc_se[ndesc * kMspThreads + tid] =
+                  (unsigned long long)s_start | ((unsigned long long)(i - 1) << 32);
+              sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
+              ++ndesc;
+              s_start = i;
+              m_cur = m;
+            }
+            if (i == nk - 1) {  // the read's last superkmer
+              sm.desc_se[ndesc * kMspThreads + tid] =
+                  (unsigned long long)s_start | ((unsigned long long)i << 32);
+              sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
+              ++ndesc;
+            }
+          }
+          if (u == w - 1) {  // block complete: suffix minima in place
+            for (int t = w - 2; t >= 0; --t) {
+              const CT x = row[t * kMspThreads], y = row[(t + 1) * kMspThreads];
+              if (y < x) row[t * kMspThreads] = y;
+            }
+            u = 0;
+          } else {
+            ++u;
+          }
+        }
+      }
+      if (__any_sync(kFull, ndesc >= kMaxDesc - 1)) flush_descriptors<CT>(a, sm, ndesc, o, L);
+    }
+    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, o, L);
   }
   if (smem_hist) {
     __syncthreads();
-    for (int i = threadIdx.x; i < a.np; i += blockDim.x) {
-      if (sh_rec[i]) atomicAdd(a.n_records + i, sh_rec[i]);
-      if (sh_kmer[i]) atomicAdd(a.n_kmers + i, sh_kmer[i]);
+    for (int i = tid; i < a.np; i += kMspThreads) {
+      if (sm.hist_rec[i]) atomicAdd(a.n_records + i, (unsigned long long)sm.hist_rec[i]);
+      if (sm.hist_kmer[i]) atomicAdd(a.n_kmers + i, (unsigned long long)sm.hist_kmer[i]);
     }
   }
 }
@@ -195,73 +298,154 @@ __global__ void __launch_bounds__(kScanThreads) scan_kernel(const uint64_t* __re
   if (threadIdx.x == 0) out[n] = carry;
 }
 
+// Pass 3: scatter staged records into partition order.
+constexpr int kScatterThreads = 256;
+constexpr int kScatterPer = 8;  // records per thread per tile
+template <int R>
+__global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t* __restrict__ staging,
+                                                                  const unsigned long long* staged,
+                                                                  uint64_t staging_cap,
+                                                                  const uint64_t* __restrict__ rec_off,
+                                                                  unsigned long long* fill,
+                                                                  uint32_t* __restrict__ records, int np) {
+  extern __shared__ unsigned long long sh_base[];  // [np] global bases (per tile), then [np] counts
+  uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_base + np);
+  const uint64_t n = min((uint64_t)*staged, staging_cap);
+  const bool smem = np <= kSmemHistMaxNp;
+  constexpr int kTile = kScatterThreads * kScatterPer;
+  for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile) {
+    if (smem) {
+      for (int i = threadIdx.x; i < np; i += kScatterThreads) sh_cnt[i] = 0;
+      __syncthreads();
+    }
+    uint4 rec[kScatterPer][R / 4];
+    uint32_t rank[kScatterPer];
+#pragma unroll
+    for (int v = 0; v < kScatterPer; ++v) {
+      const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
+      rank[v] = 0;
+      if (idx < n) {
+        const uint4* src = reinterpret_cast<const uint4*>(staging + idx * R);
+#pragma unroll
+        for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(src + c);
+        const uint32_t pid = rec[v][0].x >> 10;
+        if (smem) rank[v] = atomicAdd(sh_cnt + pid, 1u);
+        else rank[v] = (uint32_t)atomicAdd(fill + pid, 1ull);
+      }
+    }
+    if (smem) {
+      __syncthreads();
+      for (int i = threadIdx.x; i < np; i += kScatterThreads)
+        if (sh_cnt[i]) sh_base[i] = atomicAdd(fill + i, (unsigned long long)sh_cnt[i]);
+      __syncthreads();
+    }
+#pragma unroll
+    for (int v = 0; v < kScatterPer; ++v) {
+      const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
+      if (idx < n) {
+        const uint32_t pid = rec[v][0].x >> 10;
+        const uint64_t pos = rec_off[pid] + (smem ? sh_base[pid] + rank[v] : rank[v]);
+        uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
+#pragma unroll
+        for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];
+      }
+    }
+    if (smem) __syncthreads();
+  }
+}
+
 }  // namespace dbg
 
 using namespace dbg;
 
-static int sm_count() {
+int dbg_sm_count() {
   int dev = 0, n = 148;
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
   return n;
 }
 
-static bool params_ok(const dbg_params* prm) {
+bool dbg_params_ok(const dbg_params* prm) {
   return prm && prm->k >= 1 && prm->k <= 63 && (prm->k & 1) && prm->p >= 1 && prm->p <= prm->k &&
          prm->p <= 31 && prm->num_partitions >= 1 && (uint32_t)prm->num_partitions <= kMaxPid;
+}
+
+template <typename CT>
+static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
+  size_t smem = sizeof(unsigned long long) * 2 * kMaxDesc * kMspThreads + sizeof(CT) * a.w * kMspThreads + 16;
+  if (a.np <= kSmemHistMaxNp) smem += sizeof(uint32_t) * 2 * a.np;
+  cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  msp_kernel<CT><<<grid, kMspThreads, smem, stream>>>(a);
+  return cudaGetLastError();
 }
 
 extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_bases,
                                         uint64_t n_words, const uint64_t* d_offsets,
                                         uint64_t n_reads, const dbg_partition_set* part,
                                         cudaStream_t stream) {
-  if (!params_ok(prm) || !part || !d_offsets || !part->d_record_offset) return DBG_EINVAL;
+  if (!dbg_params_ok(prm) || !part || !d_offsets || !part->d_record_offset || !part->d_n_records ||
+      !part->d_n_kmers || !part->d_staged)
+    return DBG_EINVAL;
   if (n_reads && (!d_bases || !n_words)) return DBG_EINVAL;
-  const bool emit = part->d_records != nullptr;
-  if (!emit && (!part->d_n_records || !part->d_n_kmers)) return DBG_EINVAL;
-  if (emit && !part->d_fill) return DBG_EINVAL;
   const int np = prm->num_partitions;
-  MspArgs a;
-  a.words = d_bases;
-  a.n_words = n_words;
-  a.offsets = d_offsets;
-  a.n_reads = n_reads;
-  a.k = prm->k;
-  a.p = prm->p;
-  a.np = np;
-  a.rec_words = record_words(prm->k);
-  a.max_kmers = record_max_kmers(prm->k);
-  a.n_records = reinterpret_cast<unsigned long long*>(part->d_n_records);
-  a.n_kmers = reinterpret_cast<unsigned long long*>(part->d_n_kmers);
-  a.rec_off = part->d_record_offset;
-  a.fill = reinterpret_cast<unsigned long long*>(part->d_fill);
-  a.records = part->d_records;
-  const uint64_t want = (n_reads + kMspWarps - 1) / kMspWarps;
-  const uint64_t cap = (uint64_t)sm_count() * 8;
-  const int grid = (int)(want < cap ? (want ? want : 1) : cap);
-  size_t smem = sizeof(unsigned long long) * kMspWarps * kCbuf;
-  if (!emit) {
+  const uint32_t R = record_words(prm->k);
+  if (part->d_records == nullptr) {
+    // passes 1 + 2: minimizers, superkmers, staging, sizes, offsets
+    if (part->staging_cap && !part->d_staging) return DBG_EINVAL;
+    MspArgs a;
+    a.words = d_bases;
+    a.n_words = n_words;
+    a.offsets = d_offsets;
+    a.n_reads = n_reads;
+    a.k = prm->k;
+    a.p = prm->p;
+    a.np = np;
+    a.w = prm->k - prm->p + 1;
+    a.rec_words = R;
+    a.max_kmers = record_max_kmers(prm->k);
+    a.mod = make_fastmod((uint64_t)np);
+    a.n_records = reinterpret_cast<unsigned long long*>(part->d_n_records);
+    a.n_kmers = reinterpret_cast<unsigned long long*>(part->d_n_kmers);
+    a.staging = part->d_staging;
+    a.staging_cap = part->staging_cap;
+    a.staged = reinterpret_cast<unsigned long long*>(part->d_staged);
     if (cudaMemsetAsync(part->d_n_records, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
-        cudaMemsetAsync(part->d_n_kmers, 0, sizeof(uint64_t) * np, stream) != cudaSuccess)
+        cudaMemsetAsync(part->d_n_kmers, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
+        cudaMemsetAsync(part->d_staged, 0, sizeof(uint64_t), stream) != cudaSuccess)
       return DBG_ECUDA;
-    if (np <= kSmemHistMaxNp) smem += sizeof(unsigned long long) * 2 * np;
-    static bool attr_set = false;
-    if (!attr_set) {
-      cudaFuncSetAttribute(msp_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)(sizeof(unsigned long long) * (kMspWarps * kCbuf + 2 * kSmemHistMaxNp)));
-      attr_set = true;
+    if (n_reads) {
+      const uint64_t want = (n_reads + kMspThreads - 1) / kMspThreads;
+      const uint64_t cap = (uint64_t)dbg_sm_count() * 8;
+      const int grid = (int)(want < cap ? want : cap);
+      const cudaError_t e = prm->p <= 16 ? launch_msp<uint32_t>(a, grid, stream)
+                                         : launch_msp<uint64_t>(a, grid, stream);
+      if (e != cudaSuccess) return DBG_ECUDA;
     }
-    if (n_reads) msp_kernel<false><<<grid, kMspThreads, smem, stream>>>(a);
     scan_kernel<false><<<1, kScanThreads, 0, stream>>>(part->d_n_records, part->d_record_offset, np, 0.0);
   } else {
+    // pass 3: scatter (requires staged <= staging_cap; the caller checks sum(n_records))
+    if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
     if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * np, stream) != cudaSuccess) return DBG_ECUDA;
-    if (n_reads) msp_kernel<true><<<grid, kMspThreads, smem, stream>>>(a);
+    const size_t smem = np <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * np : 0;
+    const int grid = dbg_sm_count() * 4;
+    if (R == 4) {
+      cudaFuncSetAttribute(scatter_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      scatter_kernel<4><<<grid, kScatterThreads, smem, stream>>>(
+          part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
+          part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
+    } else {
+      cudaFuncSetAttribute(scatter_kernel<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      scatter_kernel<8><<<grid, kScatterThreads, smem, stream>>>(
+          part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
+          part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
+    }
   }
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
 extern "C" dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers,
                                      uint64_t* d_table_offset, cudaStream_t stream) {
-  if (!params_ok(prm) || !d_n_kmers || !d_table_offset) return DBG_EINVAL;
+  if (!dbg_params_ok(prm) || !d_n_kmers || !d_table_offset) return DBG_EINVAL;
   if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
   const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   scan_kernel<true><<<1, kScanThreads, 0, stream>>>(d_n_kmers, d_table_offset, prm->num_partitions, ratio);

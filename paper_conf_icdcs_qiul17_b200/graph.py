@@ -3,17 +3,20 @@
 PyTorch provides device memory and the stream; every step of the path runs in
 libdbg.so kernels:
 
-    a0  encode_reads         dbg_encode_ascii (host C)
-    a1  DbgBuilder.upload    H2D copy of the packed reads
-    a2-a4 DbgBuilder.msp     dbg_msp_partition (count pass -> sizes -> emit pass)
-    a5  DbgBuilder.plan      dbg_table_plan (lambda/(4 alpha) N^i_kmer)
-    a5-a6 DbgBuilder.hash    zero-fill + dbg_hash_build, batch by batch
-    a7  DbgBuilder.extract   dbg_extract_graph (+ dbg_sort_vertices)
+    a0     encode_reads          dbg_encode_ascii (host C)
+    a1     DbgBuilder.upload     H2D copy of the packed reads
+    a2-a4  DbgBuilder.msp        dbg_msp_partition pass 1 (minimizers, superkmers,
+                                 staging, sizes) -> size readback -> pass 2 (scatter)
+    a5     DbgBuilder.plan       dbg_table_plan (lambda/(4 alpha) N^i_kmer)
+    a5-a7  DbgBuilder.step2      dbg_build_subgraphs: zero + hash + extract of every
+                                 partition in one persistent kernel through an
+                                 L2-resident ring of tables ("fused", the default), or
+                                 dbg_hash_build + dbg_extract_graph over batches of
+                                 partitions with resident tables ("resident")
+    a7     DbgBuilder.vertices   dbg_sort_vertices + D2H
 
-Partitions are processed in batches of consecutive partition ids whose tables
-fit ``table_budget_bytes`` (the paper's "one partition at a time", P:L359-367,
-generalised to as many partitions as HBM holds); each batch is extracted before
-its table memory is reused.
+The paper builds "one partition at a time"; the fused
+mode keeps up to 4 partition tables in flight, each sized by Property 1.
 """
 from __future__ import annotations
 
@@ -46,45 +49,83 @@ class GraphResult:
     batches: list = field(default_factory=list)
 
 
+class _null:
+    def __enter__(self):
+        return None
+
+    def __exit__(self, *a):
+        return False
+
+
+def _grow(t: torch.Tensor, n: int, dtype, device, slack: float = 1.0) -> torch.Tensor:
+    if t.numel() >= n:
+        return t
+    del t
+    return torch.empty(max(int(n * slack), 16), dtype=dtype, device=device)
+
+
 class DbgBuilder:
     """Reusable buffers + the call sequence of the path for one (K, P, NP) setting."""
 
     def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
-                 device: str | torch.device = "cuda", table_budget_bytes: int | None = None):
+                 device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
+                 mode: str = "fused"):
         if k % 2 == 0 or not 1 <= k <= 63:
             raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
         if not 1 <= p <= min(k, 31):
             raise ValueError("P must be in 1..min(K, 31)")
-        self.k, self.p, self.np = k, p, num_partitions
+        if mode not in ("fused", "resident"):
+            raise ValueError(mode)
+        self.k, self.p, self.np, self.mode = k, p, num_partitions, mode
         self.prm = _lib.params(k, p, num_partitions, lam, alpha)
         self.device = torch.device(device)
         _lib.load()
         self.rec_words = _lib.dbg_record_words(self.prm)
         self.slot_bytes = _lib.dbg_slot_bytes(self.prm)
+        self.key_bytes = _lib.dbg_key_bytes(self.prm)
         dev = self.device
         NP = num_partitions
-        self.d_n_records = torch.zeros(NP, dtype=torch.int64, device=dev)
-        self.d_n_kmers = torch.zeros(NP, dtype=torch.int64, device=dev)
-        self.d_rec_off = torch.zeros(NP + 1, dtype=torch.int64, device=dev)
-        self.d_fill = torch.zeros(NP, dtype=torch.int64, device=dev)
-        self.d_tab_off = torch.zeros(NP + 1, dtype=torch.int64, device=dev)
+        i64 = dict(dtype=torch.int64, device=dev)
+        self.d_n_records = torch.zeros(NP, **i64)
+        self.d_n_kmers = torch.zeros(NP, **i64)
+        self.d_rec_off = torch.zeros(NP + 1, **i64)
+        self.d_fill = torch.zeros(NP, **i64)
+        self.d_staged = torch.zeros(1, **i64)
+        self.d_tab_off = torch.zeros(NP + 1, **i64)
         self.d_status = torch.zeros(1, dtype=torch.int32, device=dev)
-        self.d_n_out = torch.zeros(1, dtype=torch.int64, device=dev)
-        self.d_stats = torch.zeros(4, dtype=torch.int64, device=dev)
+        self.d_n_out = torch.zeros(1, **i64)
+        self.d_stats = torch.zeros(4, **i64)
+        self.staging = torch.empty(0, dtype=torch.int32, device=dev)
         self.records = torch.empty(0, dtype=torch.int32, device=dev)
-        self.slots = torch.empty(0, dtype=torch.uint8, device=dev)
+        self.table = torch.empty(0, dtype=torch.uint8, device=dev)
+        self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
+        self.work = torch.empty(0, dtype=torch.uint8, device=dev)
         self.out = torch.empty(0, dtype=torch.uint8, device=dev)
         self.table_budget_bytes = table_budget_bytes
         self.part_kmers = np.zeros(NP, dtype=np.int64)
         self.part_records = np.zeros(NP, dtype=np.int64)
+        self.caps = np.zeros(NP, dtype=np.int64)
         self.tab_host = np.zeros(NP + 1, dtype=np.int64)
         self.batches: list[tuple[int, int]] = []
         self._caps_key = None
-        self._caps = None
-        self.hash_timer: list | None = None  # if a list: (start, end) CUDA events per hash launch
+        self.timer: dict | None = None  # name -> list of (start, end) CUDA events, when set
+
+    # ------------------------------------------------------------------ timing helper
+    def _mark(self, name: str, stream):
+        if self.timer is None:
+            return None
+        ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+        ev[0].record(stream)
+        self.timer.setdefault(name, []).append(ev)
+        return ev
+
+    @staticmethod
+    def _done(ev, stream):
+        if ev is not None:
+            ev[1].record(stream)
 
     # ------------------------------------------------------------------ a1
-    def upload(self, packed: torch.Tensor, offsets: np.ndarray | torch.Tensor, stream=None):
+    def upload(self, packed: torch.Tensor, offsets, stream=None):
         """H2D of the packed reads and base offsets (row a1)."""
         if not isinstance(offsets, torch.Tensor):
             offsets = torch.from_numpy(np.ascontiguousarray(offsets, dtype=np.uint64).view(np.int64))
@@ -95,24 +136,37 @@ class DbgBuilder:
 
     # ------------------------------------------------------------------ a2-a4
     def part_set(self, with_records: bool) -> _lib.dbg_partition_set:
-        return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill,
+        return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill, self.d_staged,
+                                  self.staging, self.staging.numel() // self.rec_words,
                                   self.records if with_records else None)
 
-    def msp(self, d_bases: torch.Tensor, d_offsets: torch.Tensor, stream=None) -> None:
+    def _staging_estimate(self, n_kmers_upper: int, n_reads: int) -> int:
+        w = self.k - self.p + 1
+        return int(min(n_kmers_upper, 2.6 * n_kmers_upper / (w + 1) + 2 * n_reads)) + 4096
+
+    def msp(self, d_bases: torch.Tensor, d_offsets: torch.Tensor, stream=None):
         stream = stream or torch.cuda.current_stream(self.device)
         n_reads = d_offsets.numel() - 1
         n_words = d_bases.numel()
+        if self.staging.numel() == 0:
+            self.staging = _grow(self.staging, self._staging_estimate(n_words * 32, n_reads) * self.rec_words,
+                                 torch.int32, self.device)
+        ev = self._mark("msp_pass1", stream)
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(False), stream)
+        self._done(ev, stream)
         with torch.cuda.stream(stream):
             sizes = torch.cat([self.d_n_records, self.d_n_kmers]).cpu()  # the one size readback
         sizes = sizes.numpy()
         self.part_records = sizes[:self.np].copy()
         self.part_kmers = sizes[self.np:].copy()
         total = int(self.part_records.sum())
-        need = total * self.rec_words
-        if self.records.numel() < max(need, 16):
-            self.records = torch.empty(int(need * 1.05) + 16, dtype=torch.int32, device=self.device)
+        if total > self.staging.numel() // self.rec_words:  # staging too small: exact size, redo pass 1
+            self.staging = _grow(self.staging, total * self.rec_words, torch.int32, self.device, 1.05)
+            _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(False), stream)
+        self.records = _grow(self.records, total * self.rec_words, torch.int32, self.device, 1.05)
+        ev = self._mark("msp_scatter", stream)
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
+        self._done(ev, stream)
 
     # ------------------------------------------------------------------ a5
     def plan(self, stream=None) -> list[tuple[int, int]]:
@@ -120,17 +174,23 @@ class DbgBuilder:
         _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, stream)
         key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha)
         if self._caps_key != key:  # host copy of the same C sizing function (dbg_table_capacity)
-            self._caps = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in self.part_kmers],
-                                  dtype=np.int64)
+            self.caps = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in self.part_kmers],
+                                 dtype=np.int64)
             self._caps_key = key
-        caps = self._caps
         self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
-        self.tab_host[1:] = np.cumsum(caps)
+        self.tab_host[1:] = np.cumsum(self.caps)
+        if self.mode == "fused":
+            self.batches = [(0, self.np)]
+            ring = _lib.dbg_subgraph_ring_bytes(self.prm, int(self.caps.max(initial=1)) + 64)
+            self.ring = _grow(self.ring, ring, torch.uint8, self.device)
+            self.work = _grow(self.work, _lib.dbg_subgraph_workspace_bytes(self.prm, self.np), torch.uint8,
+                              self.device)
+            return self.batches
         budget = self.table_budget_bytes
         if budget is None:
             free, _ = torch.cuda.mem_get_info(self.device)
             budget = max(int(free * 0.6), 1 << 26)
-        max_slots = max(budget // self.slot_bytes, int(caps.max(initial=0)))
+        max_slots = max(budget // self.slot_bytes, int(self.caps.max(initial=0)))
         batches, b = [], 0
         while b < self.np:
             e = b + 1
@@ -140,40 +200,42 @@ class DbgBuilder:
             b = e
         self.batches = batches
         need = max((self.tab_host[e] - self.tab_host[b] for b, e in batches), default=0) * self.slot_bytes
-        if self.slots.numel() < need:
-            self.slots = torch.empty(0, dtype=torch.uint8, device=self.device)
-            self.slots = torch.empty(int(need), dtype=torch.uint8, device=self.device)
+        self.table = _grow(self.table, int(need), torch.uint8, self.device)
         return batches
 
-    # ------------------------------------------------------------------ a5-a6
-    def hash_batch(self, b: int, e: int, stream=None) -> None:
-        stream = stream or torch.cuda.current_stream(self.device)
-        n_slots = int(self.tab_host[e] - self.tab_host[b])
-        with torch.cuda.stream(stream):
-            self.slots[: n_slots * self.slot_bytes].zero_()  # EMPTY = 0 (hash.cu slot layout)
-        if self.hash_timer is not None:
-            ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-            ev[0].record(stream)
-        _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.slots, self.d_tab_off,
-                            int(self.tab_host[b]), self.d_status, stream)
-        if self.hash_timer is not None:
-            ev[1].record(stream)
-            self.hash_timer.append(ev)
-
-    # ------------------------------------------------------------------ a7
+    # ------------------------------------------------------------------ a5-a7
     def reset_output(self, cap: int, stream=None) -> None:
         with torch.cuda.stream(stream or torch.cuda.current_stream(self.device)):
             self.d_n_out.zero_()
             self.d_stats.zero_()
             self.d_status.zero_()
-        if self.out.numel() < cap * VERTEX_DTYPE.itemsize:
-            self.out = torch.empty(cap * VERTEX_DTYPE.itemsize, dtype=torch.uint8, device=self.device)
+        self.out = _grow(self.out, cap * VERTEX_DTYPE.itemsize, torch.uint8, self.device)
 
-    def extract_batch(self, b: int, e: int, stream=None) -> None:
+    def out_cap(self) -> int:
+        return self.out.numel() // VERTEX_DTYPE.itemsize
+
+    def step2(self, stream=None) -> None:
+        """Zero-fill + hash + extract of every partition (output appended to self.out)."""
         stream = stream or torch.cuda.current_stream(self.device)
-        cap = self.out.numel() // VERTEX_DTYPE.itemsize
-        _lib.dbg_extract_graph(self.prm, self.slots, self.d_tab_off, int(self.tab_host[b]), b, e, self.out,
-                               cap, self.d_n_out, self.d_stats, self.d_status, stream)
+        if self.mode == "fused":
+            ev = self._mark("step2", stream)
+            _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.ring,
+                                     self.ring.numel(), self.work, self.work.numel(), self.out, self.out_cap(),
+                                     self.d_n_out, self.d_stats, self.d_status, stream)
+            self._done(ev, stream)
+            return
+        for (b, e) in self.batches:
+            n_slots = int(self.tab_host[e] - self.tab_host[b])
+            with torch.cuda.stream(stream):
+                self.table[: n_slots * self.key_bytes].zero_()  # EMPTY key entries (hash.cu)
+            ev = self._mark("hash_build", stream)
+            _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.table, self.d_tab_off, self.d_status,
+                                stream)
+            self._done(ev, stream)
+            ev = self._mark("extract", stream)
+            _lib.dbg_extract_graph(self.prm, self.table, self.d_tab_off, b, e, self.out, self.out_cap(),
+                                   self.d_n_out, self.d_stats, self.d_status, stream)
+            self._done(ev, stream)
 
     def stats(self) -> dict:
         s = self.d_stats.cpu().numpy().view(np.uint64)
@@ -198,46 +260,35 @@ class DbgBuilder:
               want_vertices: bool = True, sort: bool = True) -> GraphResult:
         stream = stream or torch.cuda.current_stream(self.device)
         self.msp(d_bases, d_offsets, stream)
-        batches = self.plan(stream)
+        self.plan(stream)
         n_kmers = int(self.part_kmers.sum())
-        cap = out_cap if out_cap is not None else n_kmers
+        cap = out_cap if out_cap is not None else max(self.out_cap(), n_kmers // 2 + 1024)
         while True:
             self.reset_output(cap, stream)
-            cap = self.out.numel() // VERTEX_DTYPE.itemsize
-            for b, e in batches:
-                self.hash_batch(b, e, stream)
-                self.extract_batch(b, e, stream)
+            self.step2(stream)
             st = _lib.dbg_sync_status(self.d_status, stream)
-            if st == _lib.DBG_ENOSPACE:
+            if st == _lib.DBG_ENOSPACE and int(self.d_n_out.item()) > self.out_cap():
                 cap = int(self.d_n_out.item())
                 continue
             if st == _lib.DBG_ETABLEFULL:  # reading O: rebuild at capacity N^i_kmer
                 if self.prm.lambda_ / (4 * self.prm.alpha) >= 1.0:
                     raise _lib.DbgError("dbg_hash_build", st, "table full at capacity >= N^i_kmer")
                 self.prm = _lib.params(self.k, self.p, self.np, 2.0, 0.5)
-                batches = self.plan(stream)
+                self.plan(stream)
                 continue
             if st != _lib.DBG_OK:
                 raise _lib.DbgError("dbg_sync_status", st, _lib.dbg_status_string(st))
             break
         verts = self.vertices(sort=sort, stream=stream) if want_vertices else None
         return GraphResult(verts, int(self.d_n_out.item()), self.stats(), n_kmers, self.part_kmers.copy(),
-                           self.part_records.copy(), list(batches))
-
-
-class _null:
-    def __enter__(self):
-        return None
-
-    def __exit__(self, *a):
-        return False
+                           self.part_records.copy(), list(self.batches))
 
 
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
                 lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
-                table_budget_bytes: int | None = None) -> GraphResult:
+                table_budget_bytes: int | None = None, mode: str = "fused") -> GraphResult:
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
-    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes)
+    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode)
     packed = encode_reads(seq)
     d_bases, d_offsets = builder.upload(packed, offsets)
     return builder.build(d_bases, d_offsets, sort=sort)

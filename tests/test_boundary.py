@@ -28,7 +28,7 @@ def _declared():
 
 def test_exports_every_declared_symbol(lib):
     names = _declared()
-    assert len(names) == 15
+    assert len(names) == 19
     raw = lib.load()
     for n in names:
         assert hasattr(raw, n), n
@@ -41,7 +41,9 @@ def test_abi_and_sizes(lib):
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
     assert lib.dbg_record_words(p63) == 8 and lib.dbg_record_max_kmers(p63) == 48
-    assert lib.dbg_slot_bytes(p31) == 64
+    assert lib.dbg_slot_bytes(p31) == 48 and lib.dbg_key_bytes(p31) == 16
+    assert lib.dbg_slot_bytes(p63) == 64 and lib.dbg_key_bytes(p63) == 32
+    assert lib.dbg_subgraph_ring_bytes(p31, 1000) == 4 * 1000 * 48
     assert lib.dbg_packed_words(0) == 1 and lib.dbg_packed_words(32) == 2 and lib.dbg_packed_words(33) == 3
 
 
@@ -93,14 +95,14 @@ def test_encoder_fig4_and_rules(lib):
 def test_invalid_arguments_return_before_launch(lib):
     from paper_conf_icdcs_qiul17_b200._lib import DbgError, partition_set
 
-    part = partition_set(1, 1, 1, 1, None)
+    part = partition_set(1, 1, 1, 1, 1, None, 0, None)
     for prm in (lib.params(30, 11, 16), lib.params(31, 0, 16), lib.params(31, 32, 16), lib.params(31, 11, 0),
                 lib.params(65, 11, 16)):
         with pytest.raises(DbgError) as e:
             lib.dbg_msp_partition(prm, 1, 1, 1, 1, part, None)
         assert e.value.status == lib.DBG_EINVAL
     with pytest.raises(DbgError):
-        lib.dbg_hash_build(lib.params(31, 11, 16), part, 5, 2, 1, 1, 0, 1, None)
+        lib.dbg_hash_build(lib.params(31, 11, 16), partition_set(1, 1, 1, 1, 1, None, 0, 1), 5, 2, 1, 1, 1, None)
     assert lib.dbg_status_string(lib.DBG_ETABLEFULL).startswith("hash table full")
 
 

@@ -116,29 +116,43 @@ def test_msp_records_vs_oracle_superkmers():
         assert occurrences_from_records(recs, k) == occurrences_from_oracle_msp(sk, rs.reads(), k)
 
 
-def test_table_overflow_detected_and_rebuilt():
+@pytest.mark.parametrize("mode", ["fused", "resident"])
+def test_table_overflow_detected_and_rebuilt(mode):
     """Reading O: an undersized table (lambda/(4 alpha) << distinct/N) overflows; the status word
     reports DBG_ETABLEFULL and the builder rebuilds at capacity N^i_kmer with the same result."""
     g = genome(20_000, seed=5)
     seq, offs = make_reads(g, 3000, 100, 0.01, seed=6)
     rs = ReadSet(seq, offs)
-    b = DbgBuilder(31, 11, 4, lam=0.04, alpha=0.5)
+    b = DbgBuilder(31, 11, 4, lam=0.04, alpha=0.5, mode=mode)
     d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
     b.msp(d_bases, d_off)
-    for (lo, hi) in b.plan():
-        b.reset_output(1 << 20)
-        b.hash_batch(lo, hi)
+    b.plan()
+    b.reset_output(1 << 20)
+    b.step2()
     assert _lib.dbg_sync_status(b.d_status) == _lib.DBG_ETABLEFULL
-    _check(rs, 31, 11, 4, lam=0.04, alpha=0.5)
+    _check(rs, 31, 11, 4, lam=0.04, alpha=0.5, mode=mode)
 
 
-def test_batches_give_same_graph():
+def test_resident_batches_give_same_graph():
     rs = make_config("tiny", scale=0.5)
     a = build_graph(rs.seq, rs.offsets, 31, 11, 16)
-    b = build_graph(rs.seq, rs.offsets, 31, 11, 16, table_budget_bytes=64 * 2000)
+    b = build_graph(rs.seq, rs.offsets, 31, 11, 16, table_budget_bytes=48 * 2000, mode="resident")
     assert len(b.batches) > 4
     assert a.vertices.tobytes() == b.vertices.tobytes()
     assert a.stats == b.stats
+
+
+@pytest.mark.parametrize("k,p,np_", [(31, 11, 16), (63, 19, 8), (41, 17, 5), (7, 3, 3)])
+def test_resident_mode_parity(k, p, np_):
+    rs = random_reads(300, 1, 2 * k + 100, seed=k + np_, n_rate=0.01)
+    _check(rs, k, p, np_, mode="resident")
+
+
+def test_ring_with_many_small_partitions():
+    """More partitions than ring regions, many empty: the fused kernel's region reuse chain."""
+    rs = random_reads(500, 40, 160, seed=77)
+    _check(rs, 31, 11, 1000)
+    _check(rs, 15, 7, 37)
 
 
 def test_repeat_runs_deterministic():
