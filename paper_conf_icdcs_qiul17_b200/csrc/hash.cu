@@ -380,6 +380,10 @@ struct SubgraphArgs {
 };
 
 __device__ __forceinline__ uint64_t div_up(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+// Every partition has at least one zero item (a no-op when it is empty), so
+// "zero items of p-RING done" transitively implies every earlier user of the
+// ring region is done, even through empty partitions.
+__device__ __forceinline__ uint64_t n_zero_items(uint64_t cap) { return cap ? div_up(cap, kZeroSlots) : 1; }
 
 struct PartGeom {
   uint64_t cap, rec0, nrec;
@@ -414,7 +418,7 @@ __global__ void __launch_bounds__(kThreads) subgraph_plan_kernel(SubgraphArgs a,
       if (s < a.n_part) {
         const PartGeom g = geom(a, s);
         if (g.cap > a.region_slots) atomicOr(status, kStatusRing);
-        items += div_up(g.cap, kZeroSlots);
+        items += n_zero_items(g.cap);
       }
       if (s >= 1 && s - 1 < a.n_part) items += div_up(geom(a, s - 1).nrec, kHashRecs);
       if (s >= 2) items += div_up(geom(a, s - 2).cap, kExtractSlots);
@@ -464,7 +468,7 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
     PartGeom g;
     if (s < a.n_part) {
       g = geom(a, s);
-      const uint64_t nz = div_up(g.cap, kZeroSlots);
+      const uint64_t nz = n_zero_items(g.cap);
       if (j < nz) kind = 0, p = s;
       else j -= nz;
     }
@@ -483,8 +487,12 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
     uint32_t* ctr = reinterpret_cast<uint32_t*>(keys + a.region_slots * KE);
     // dependencies: region reuse, zero-before-hash, hash-before-extract
     if (threadIdx.x == 0) {
-      if (kind == 0 && p >= kRing) wait_count(done_x + p - kRing, (uint32_t)div_up(geom(a, p - kRing).cap, kExtractSlots));
-      if (kind == 1) wait_count(done_z + p, (uint32_t)div_up(g.cap, kZeroSlots));
+      if (kind == 0 && p >= kRing) {  // region reuse: the previous user is fully extracted
+        const uint64_t cq = geom(a, p - kRing).cap;
+        wait_count(done_z + p - kRing, (uint32_t)n_zero_items(cq));
+        wait_count(done_x + p - kRing, (uint32_t)div_up(cq, kExtractSlots));
+      }
+      if (kind == 1) wait_count(done_z + p, (uint32_t)n_zero_items(g.cap));
       if (kind == 2) wait_count(done_h + p, (uint32_t)div_up(g.nrec, kHashRecs));
     }
     __syncthreads();
