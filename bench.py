@@ -184,7 +184,8 @@ def run_ours(args):
     offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
     n_kmers = rs.n_kmers()
     stream = torch.cuda.current_stream(dev)
-    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode)
+    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode,
+                   args.group_slots)
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
@@ -266,7 +267,8 @@ def run_ours(args):
         "metric": METRIC, "value": n_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": _config_json(rs, args, {"mode": args.mode, "batches": len(b.batches)}),
+        "config": _config_json(rs, args, {"mode": args.mode, "batches": len(b.batches),
+                                          "group_slots": args.group_slots}),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "kernel": "subgraph_kernel" if args.mode == "fused" else "hash_build_kernel",
@@ -297,6 +299,7 @@ def main():
     ap.add_argument("--alpha", type=float, default=0.5)
     ap.add_argument("--table-budget", type=int, default=None)
     ap.add_argument("--mode", choices=["fused", "resident"], default="fused")
+    ap.add_argument("--group-slots", type=int, default=1 << 19)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

@@ -139,22 +139,28 @@ DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kme
                           uint64_t* d_table_offset, cudaStream_t stream);
 
 /* ---- a5-a7 fused: Step 2 through an L2-resident ring (the hot path) ------
- * For partitions [pid_begin, pid_end): zero-fill the key entries of the
+ * For partitions [pid_begin, pid_end): zero-fill the key entries of each
  * partition's table, build it (one insertion per distinct vertex, multiple
- * updates, Sec. III-C), and compact it into d_out -- one
- * persistent kernel in which each partition's table lives in one of 4 ring
- * regions of d_ring (ring_bytes >= dbg_subgraph_ring_bytes(max capacity);
- * a smaller ring sets status bit 2 -> DBG_ENOSPACE).  d_workspace holds
- * dbg_subgraph_workspace_bytes(pid_end - pid_begin) bytes of scheduling
- * state.  Output appends to d_out[*d_n_out ...] and accumulates *d_stats as in
- * dbg_extract_graph. */
-DBG_API uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t max_capacity);
-DBG_API uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions);
+ * updates, Sec. III-C), and compact it into d_out -- all in one
+ * persistent kernel.  Partitions are taken in groups of consecutive
+ * partitions spanning about group_slots table slots (the caller picks it so
+ * a few groups fit in L2: the B200 form of sizing tables for locality,
+ * P:L665-675); each group's tables live in one of the ring regions of d_ring
+ * (ring_bytes >= dbg_subgraph_ring_bytes(group_slots, max capacity); a
+ * smaller ring sets status bit 2 -> DBG_ENOSPACE).  total_slots =
+ * d_table_offset[pid_end] - d_table_offset[pid_begin] (host copy, sizes the
+ * workspace: dbg_subgraph_workspace_bytes bytes of scheduling state).
+ * Output appends to d_out[*d_n_out ...] and accumulates *d_stats as
+ * dbg_extract_graph does. */
+DBG_API uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t group_slots, uint64_t max_capacity);
+DBG_API uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions, uint64_t total_slots,
+                                      uint64_t group_slots);
 DBG_API dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
-                               int32_t pid_end, const uint64_t* d_table_offset, void* d_ring,
-                               uint64_t ring_bytes, void* d_workspace, uint64_t workspace_bytes,
-                               dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
-                               dbg_stats* d_stats, uint32_t* d_status, cudaStream_t stream);
+                               int32_t pid_end, const uint64_t* d_table_offset, uint64_t total_slots,
+                               uint64_t group_slots, void* d_ring, uint64_t ring_bytes, void* d_workspace,
+                               uint64_t workspace_bytes, dbg_vertex* d_out, uint64_t out_cap,
+                               uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
+                               cudaStream_t stream);
 
 /* ---- a6: Step 2 with resident tables (Sec. III-C) ------------
  * Inserts every K-mer occurrence of partitions [pid_begin, pid_end) into that

@@ -55,7 +55,6 @@ constexpr int kThreads = 256;
 constexpr uint64_t kReady = 1ull << 62;
 constexpr uint64_t kCodeMask = kReady - 1;
 constexpr uint64_t kSlotSeed = 0x9e3779b97f4a7c15ull;
-constexpr int kRing = 4;
 constexpr uint32_t kZeroSlots = 4096;          // key entries per zero item
 constexpr uint32_t kHashRecs = kThreads;       // records per hash item
 constexpr int kXPer = 8;
@@ -366,71 +365,114 @@ __global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, Ou
 }
 
 // --------------------------------------------------------------- fused Step 2
+//
+// Partitions [b, e) are cut into groups of consecutive partitions: partition
+// p belongs to group floor((tab_off[p] - tab_off[b]) / group_slots), so a
+// group spans at most group_slots + max capacity slots.  Group g uses ring
+// region g % kRing: key entries of the group's partitions back to back, then
+// their counter records.  The work list is a sequence of stages; stage s holds
+//   Z(s)          zero-fill the key entries of group s,
+//   H(s-1)        hash the records of group s-1,
+//   X(s-1-kLagX)  extract group s-1-kLagX,
+// and CTAs claim items in list order.  Dependencies (per-group completion
+// counters): H(g) after Z(g); X(g) after H(g); Z(g) after Z(g-kRing) and
+// X(g-kRing) (ring reuse; every group has >= 1 zero item so the chain is
+// transitive through empty groups).  Every dependency of an item lies in an
+// earlier stage, so the schedule cannot deadlock, and the lag of extraction
+// behind hashing keeps CTAs from stalling on a group's last hash items.
+
+constexpr int kLagX = 2;
+constexpr int kRingGroups = kLagX + 4;
 
 struct SubgraphArgs {
   const uint32_t* records;
   const uint64_t* rec_off;
   const uint64_t* tab_off;
-  int pid_begin, n_part, k;
+  int pid_begin, pid_end, k;
+  uint64_t group_slots, n_groups_max;
   char* ring;
   uint64_t region_slots, region_bytes;
-  const unsigned long long* stage_off;  // [n_part + 3]
-  unsigned long long* work;             // claimed-item counter
-  uint32_t* done;                       // [3][n_part]: zero, hash, extract items done
+  uint32_t* gfirst;               // [n_groups_max + 1] first partition of each group
+  unsigned long long* stage_off;  // [n_groups_max + kLagX + 3]
+  unsigned long long* work;       // [0] claimed-item counter, [1] n_groups
+  uint32_t* done;                 // [3][n_groups_max]: zero, hash, extract items done
 };
 
 __device__ __forceinline__ uint64_t div_up(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
-// Every partition has at least one zero item (a no-op when it is empty), so
-// "zero items of p-RING done" transitively implies every earlier user of the
-// ring region is done, even through empty partitions.
-__device__ __forceinline__ uint64_t n_zero_items(uint64_t cap) { return cap ? div_up(cap, kZeroSlots) : 1; }
 
-struct PartGeom {
-  uint64_t cap, rec0, nrec;
+struct GroupGeom {
+  int p0, p1;              // partitions [p0, p1)
+  uint64_t slot0, span;    // first slot (tab_off coordinates), slots
+  uint64_t rec0, nrec;     // records
 };
-__device__ __forceinline__ PartGeom geom(const SubgraphArgs& a, int p) {
-  PartGeom g;
-  const int pid = a.pid_begin + p;
-  g.cap = a.tab_off[pid + 1] - a.tab_off[pid];
-  g.rec0 = a.rec_off[pid];
-  g.nrec = a.rec_off[pid + 1] - g.rec0;
-  return g;
+__device__ __forceinline__ GroupGeom ggeom(const SubgraphArgs& a, int g) {
+  GroupGeom G;
+  G.p0 = (int)a.gfirst[g];
+  G.p1 = (int)a.gfirst[g + 1];
+  G.slot0 = a.tab_off[G.p0];
+  G.span = a.tab_off[G.p1] - G.slot0;
+  G.rec0 = a.rec_off[G.p0];
+  G.nrec = a.rec_off[G.p1] - G.rec0;
+  return G;
 }
+__device__ __forceinline__ uint64_t nz_items(const GroupGeom& G) { return G.span ? div_up(G.span, kZeroSlots) : 1; }
+__device__ __forceinline__ uint64_t nh_items(const GroupGeom& G) { return div_up(G.nrec, kHashRecs); }
+__device__ __forceinline__ uint64_t nx_items(const GroupGeom& G) { return div_up(G.span, kExtractSlots); }
 
-// Single CTA: stage offsets of the work list and zeroed completion counters.
-// Stage s holds: zero items of partition s, hash items of s-1, extract items of s-2.
+// Single CTA: groups, stage offsets of the work list, zeroed completion counters.
 __global__ void __launch_bounds__(kThreads) subgraph_plan_kernel(SubgraphArgs a, uint32_t* status) {
   typedef cub::BlockScan<unsigned long long, kThreads> Scan;
   __shared__ typename Scan::TempStorage tmp;
   __shared__ unsigned long long carry;
-  for (int i = threadIdx.x; i < 3 * a.n_part; i += kThreads) a.done[i] = 0;
+  const uint64_t base = a.tab_off[a.pid_begin];
+  const uint64_t total = a.tab_off[a.pid_end] - base;
+  uint64_t n_g = total ? div_up(total, a.group_slots) : 1;
+  if (n_g > a.n_groups_max) {
+    if (threadIdx.x == 0) atomicOr(status, kStatusRing);
+    n_g = a.n_groups_max;
+  }
+  // first partition of group g: lower bound of (tab_off[p] - base) / group_slots >= g
+  for (uint64_t g = threadIdx.x; g <= n_g; g += kThreads) {
+    int lo = a.pid_begin, hi = a.pid_end;
+    if (g == n_g) {
+      lo = a.pid_end;
+    } else {
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if ((a.tab_off[mid] - base) / a.group_slots < g) lo = mid + 1;
+        else hi = mid;
+      }
+    }
+    a.gfirst[g] = (uint32_t)lo;
+  }
+  for (uint64_t i = threadIdx.x; i < 3 * n_g; i += kThreads) a.done[i] = 0;
   if (threadIdx.x == 0) {
     carry = 0;
-    *a.work = 0;
+    a.work[0] = 0;
+    a.work[1] = n_g;
   }
   __syncthreads();
-  const int n_stage = a.n_part + 2;
-  unsigned long long* so = const_cast<unsigned long long*>(a.stage_off);
-  for (int base = 0; base < n_stage; base += kThreads) {
-    const int s = base + threadIdx.x;
+  const int n_stage = (int)n_g + 1 + kLagX;
+  for (int s0 = 0; s0 < n_stage; s0 += kThreads) {
+    const int s = s0 + threadIdx.x;
     unsigned long long items = 0;
     if (s < n_stage) {
-      if (s < a.n_part) {
-        const PartGeom g = geom(a, s);
-        if (g.cap > a.region_slots) atomicOr(status, kStatusRing);
-        items += n_zero_items(g.cap);
+      if (s < (int)n_g) {
+        const GroupGeom G = ggeom(a, s);
+        if (G.span > a.region_slots) atomicOr(status, kStatusRing);
+        items += nz_items(G);
       }
-      if (s >= 1 && s - 1 < a.n_part) items += div_up(geom(a, s - 1).nrec, kHashRecs);
-      if (s >= 2) items += div_up(geom(a, s - 2).cap, kExtractSlots);
+      if (s >= 1 && s - 1 < (int)n_g) items += nh_items(ggeom(a, s - 1));
+      if (s >= 1 + kLagX) items += nx_items(ggeom(a, s - 1 - kLagX));
     }
-    unsigned long long excl, total;
-    Scan(tmp).ExclusiveSum(items, excl, total);
-    if (s < n_stage) so[s] = carry + excl;
+    unsigned long long excl, tot;
+    Scan(tmp).ExclusiveSum(items, excl, tot);
+    if (s < n_stage) a.stage_off[s] = carry + excl;
     __syncthreads();
-    if (threadIdx.x == 0) carry += total;
+    if (threadIdx.x == 0) carry += tot;
     __syncthreads();
   }
-  if (threadIdx.x == 0) so[n_stage] = carry;
+  if (threadIdx.x == 0) a.stage_off[n_stage] = carry;
 }
 
 __device__ __forceinline__ void wait_count(const uint32_t* p, uint32_t need) {
@@ -444,19 +486,19 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
   constexpr uint32_t KE = KW == 1 ? 16 : 32;
   __shared__ XShared sh;
   __shared__ unsigned long long s_item;
-  const int n_stage = a.n_part + 2;
+  const int n_g = (int)a.work[1];
+  const int n_stage = n_g + 1 + kLagX;
   const unsigned long long total = a.stage_off[n_stage];
   uint32_t* done_z = a.done;
-  uint32_t* done_h = a.done + a.n_part;
-  uint32_t* done_x = a.done + 2 * a.n_part;
+  uint32_t* done_h = a.done + n_g;
+  uint32_t* done_x = a.done + 2 * n_g;
   for (;;) {
     if (threadIdx.x == 0) s_item = atomicAdd(a.work, 1ull);
     __syncthreads();
     const unsigned long long item = s_item;
     __syncthreads();
     if (item >= total) break;
-    // locate the stage (binary search over n_stage + 1 offsets)
-    int lo = 0, hi = n_stage;
+    int lo = 0, hi = n_stage;  // stage: last s with stage_off[s] <= item
     while (hi - lo > 1) {
       const int mid = (lo + hi) >> 1;
       if (a.stage_off[mid] <= item) lo = mid;
@@ -464,62 +506,67 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
     }
     const int s = lo;
     uint64_t j = item - a.stage_off[s];
-    int kind = -1, p = -1;
-    PartGeom g;
-    if (s < a.n_part) {
-      g = geom(a, s);
-      const uint64_t nz = n_zero_items(g.cap);
-      if (j < nz) kind = 0, p = s;
-      else j -= nz;
+    int kind = -1, g = -1;
+    GroupGeom G;
+    if (s < n_g) {
+      G = ggeom(a, s);
+      const uint64_t n = nz_items(G);
+      if (j < n) kind = 0, g = s;
+      else j -= n;
     }
-    if (kind < 0 && s >= 1 && s - 1 < a.n_part) {
-      g = geom(a, s - 1);
-      const uint64_t nh = div_up(g.nrec, kHashRecs);
-      if (j < nh) kind = 1, p = s - 1;
-      else j -= nh;
+    if (kind < 0 && s >= 1 && s - 1 < n_g) {
+      G = ggeom(a, s - 1);
+      const uint64_t n = nh_items(G);
+      if (j < n) kind = 1, g = s - 1;
+      else j -= n;
     }
     if (kind < 0) {
       kind = 2;
-      p = s - 2;
-      g = geom(a, p);
+      g = s - 1 - kLagX;
+      G = ggeom(a, g);
     }
-    char* keys = a.ring + (uint64_t)(p % kRing) * a.region_bytes;
+    char* keys = a.ring + (uint64_t)(g % kRingGroups) * a.region_bytes;
     uint32_t* ctr = reinterpret_cast<uint32_t*>(keys + a.region_slots * KE);
-    // dependencies: region reuse, zero-before-hash, hash-before-extract
     if (threadIdx.x == 0) {
-      if (kind == 0 && p >= kRing) {  // region reuse: the previous user is fully extracted
-        const uint64_t cq = geom(a, p - kRing).cap;
-        wait_count(done_z + p - kRing, (uint32_t)n_zero_items(cq));
-        wait_count(done_x + p - kRing, (uint32_t)div_up(cq, kExtractSlots));
+      if (kind == 0 && g >= kRingGroups) {  // ring reuse: the previous user is fully extracted
+        const GroupGeom Q = ggeom(a, g - kRingGroups);
+        wait_count(done_z + g - kRingGroups, (uint32_t)nz_items(Q));
+        wait_count(done_x + g - kRingGroups, (uint32_t)nx_items(Q));
       }
-      if (kind == 1) wait_count(done_z + p, (uint32_t)n_zero_items(g.cap));
-      if (kind == 2) wait_count(done_h + p, (uint32_t)div_up(g.nrec, kHashRecs));
+      if (kind == 1) wait_count(done_z + g, (uint32_t)nz_items(G));
+      if (kind == 2) wait_count(done_h + g, (uint32_t)nh_items(G));
     }
     __syncthreads();
     if (kind == 0) {
-      const uint64_t s0 = j * kZeroSlots, s1 = min(g.cap, s0 + kZeroSlots);
+      const uint64_t s0 = j * kZeroSlots, s1 = min(G.span, s0 + kZeroSlots);
       uint4* z = reinterpret_cast<uint4*>(keys + s0 * KE);
-      const uint64_t n16 = (s1 - s0) * (KE / 16);
+      const uint64_t n16 = s1 > s0 ? (s1 - s0) * (KE / 16) : 0;
       for (uint64_t q = threadIdx.x; q < n16; q += kThreads) __stcg(z + q, make_uint4(0, 0, 0, 0));
     } else if (kind == 1) {
       const uint64_t r = j * kHashRecs + threadIdx.x;
-      if (r < g.nrec) {
+      if (r < G.nrec) {
+        const uint32_t* rp = a.records + (G.rec0 + r) * R;
+        const uint32_t pid = __ldg(rp) >> 10;
+        const uint64_t t0 = a.tab_off[pid] - G.slot0;
         Table t;
-        t.keys = keys;
-        t.ctr = ctr;
-        t.cap = g.cap;
-        if (!hash_record<Code, R>(a.records + (g.rec0 + r) * R, a.k, t)) atomicOr(oa.status, kStatusTableFull);
+        t.keys = keys + t0 * KE;
+        t.ctr = ctr + t0 * 8;
+        t.cap = a.tab_off[pid + 1] - a.tab_off[pid];
+        if (!hash_record<Code, R>(rp, a.k, t)) atomicOr(oa.status, kStatusTableFull);
       }
     } else {
       const uint64_t s0 = j * kExtractSlots;
-      const uint64_t n = min((uint64_t)kExtractSlots, g.cap - s0);
-      const uint32_t pid = (uint32_t)(a.pid_begin + p);
-      extract_tile<KW>(keys + s0 * KE, ctr + s0 * 8, n, [=](uint64_t) { return pid; }, oa, sh);
+      const uint64_t n = min((uint64_t)kExtractSlots, G.span - s0);
+      const uint64_t* off = a.tab_off;
+      const uint64_t gs0 = G.slot0;
+      const int p0 = G.p0, p1 = G.p1;
+      extract_tile<KW>(keys + s0 * KE, ctr + s0 * 8, n,
+                       [=](uint64_t sl) { return (uint32_t)find_part(off, p0, p1, gs0 + s0 + sl); }, oa, sh);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
-      atomicAdd(kind == 0 ? done_z + p : kind == 1 ? done_h + p : done_x + p, 1u);
+      atomicAdd(kind == 0 ? done_z + g : kind == 1 ? done_h + g : done_x + g, 1u);
     }
   }
 }
@@ -609,46 +656,57 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_tab
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-extern "C" uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions) {
-  (void)prm;
-  const uint64_t n = n_partitions > 0 ? (uint64_t)n_partitions : 1;
-  return 8 * (n + 3) + 8 + 4 * 3 * n + 64;
+static uint64_t n_groups_max(uint64_t total_slots, uint64_t group_slots) {
+  return (group_slots ? total_slots / group_slots : 0) + 2;
 }
 
-extern "C" uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t max_capacity) {
+extern "C" uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions, uint64_t total_slots,
+                                                 uint64_t group_slots) {
+  (void)prm;
+  (void)n_partitions;
+  const uint64_t g = n_groups_max(total_slots, group_slots);
+  return 4 * (g + 1) + 8 * (g + kLagX + 3) + 16 + 4 * 3 * g + 64;
+}
+
+extern "C" uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t group_slots, uint64_t max_capacity) {
   if (!prm) return 0;
-  return (uint64_t)kRing * max_capacity * (key_bytes(prm->k) + kCtrBytes);
+  const uint64_t region = (group_slots + max_capacity + 63) & ~(uint64_t)63;
+  return (uint64_t)kRingGroups * region * (key_bytes(prm->k) + kCtrBytes);
 }
 
 extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
-                                          int32_t pid_end, const uint64_t* d_table_offset, void* d_ring,
-                                          uint64_t ring_bytes, void* d_workspace, uint64_t workspace_bytes,
-                                          dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
-                                          dbg_stats* d_stats, uint32_t* d_status, cudaStream_t stream) {
+                                          int32_t pid_end, const uint64_t* d_table_offset, uint64_t total_slots,
+                                          uint64_t group_slots, void* d_ring, uint64_t ring_bytes,
+                                          void* d_workspace, uint64_t workspace_bytes, dbg_vertex* d_out,
+                                          uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
+                                          uint32_t* d_status, cudaStream_t stream) {
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table_offset ||
-      !d_ring || !d_workspace || !d_n_out || !d_stats || !d_status || (out_cap && !d_out))
+      !d_ring || !d_workspace || !d_n_out || !d_stats || !d_status || (out_cap && !d_out) || group_slots == 0)
     return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
-  const int n_part = pid_end - pid_begin;
-  if (n_part == 0) return DBG_OK;
-  if (workspace_bytes < dbg_subgraph_workspace_bytes(prm, n_part)) return DBG_EINVAL;
+  if (pid_begin == pid_end) return DBG_OK;
+  if (workspace_bytes < dbg_subgraph_workspace_bytes(prm, pid_end - pid_begin, total_slots, group_slots))
+    return DBG_EINVAL;
   const uint64_t slot = key_bytes(prm->k) + kCtrBytes;
   SubgraphArgs a;
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
   a.tab_off = d_table_offset;
   a.pid_begin = pid_begin;
-  a.n_part = n_part;
+  a.pid_end = pid_end;
   a.k = prm->k;
+  a.group_slots = group_slots;
+  a.n_groups_max = n_groups_max(total_slots, group_slots);
   a.ring = static_cast<char*>(d_ring);
-  a.region_slots = ring_bytes / kRing / slot;
-  a.region_slots &= ~(uint64_t)63;  // keep regions 64 B x 64 aligned
+  a.region_slots = (ring_bytes / kRingGroups / slot) & ~(uint64_t)63;
   a.region_bytes = a.region_slots * slot;
   if (a.region_slots == 0) return DBG_EINVAL;
   char* ws = static_cast<char*>(d_workspace);
+  const uint64_t g = a.n_groups_max;
   a.stage_off = reinterpret_cast<unsigned long long*>(ws);
-  a.work = reinterpret_cast<unsigned long long*>(ws + 8 * (n_part + 3));
-  a.done = reinterpret_cast<uint32_t*>(ws + 8 * (n_part + 3) + 8);
+  a.work = reinterpret_cast<unsigned long long*>(ws + 8 * (g + kLagX + 3));
+  a.done = reinterpret_cast<uint32_t*>(ws + 8 * (g + kLagX + 3) + 16);
+  a.gfirst = a.done + 3 * g;
   OutArgs oa;
   oa.out = d_out;
   oa.out_cap = out_cap;

@@ -16,7 +16,8 @@ libdbg.so kernels:
     a7     DbgBuilder.vertices   dbg_sort_vertices + D2H
 
 The paper builds "one partition at a time"; the fused
-mode keeps up to 4 partition tables in flight, each sized by Property 1.
+mode streams groups of consecutive partitions (~group_slots table slots each)
+through a ring of L2-sized regions, each table sized by Property 1.
 """
 from __future__ import annotations
 
@@ -58,7 +59,7 @@ class _null:
 
 
 def _grow(t: torch.Tensor, n: int, dtype, device, slack: float = 1.0) -> torch.Tensor:
-    if t.numel() >= n:
+    if t.numel() >= n and t.numel() > 0:
         return t
     del t
     return torch.empty(max(int(n * slack), 16), dtype=dtype, device=device)
@@ -69,7 +70,7 @@ class DbgBuilder:
 
     def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
                  device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
-                 mode: str = "fused"):
+                 mode: str = "fused", group_slots: int = 1 << 19):
         if k % 2 == 0 or not 1 <= k <= 63:
             raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
         if not 1 <= p <= min(k, 31):
@@ -77,6 +78,8 @@ class DbgBuilder:
         if mode not in ("fused", "resident"):
             raise ValueError(mode)
         self.k, self.p, self.np, self.mode = k, p, num_partitions, mode
+        self.group_slots = int(group_slots)  # fused mode: table slots per ring group (L2 sizing)
+        self.total_slots = 0
         self.prm = _lib.params(k, p, num_partitions, lam, alpha)
         self.device = torch.device(device)
         _lib.load()
@@ -181,10 +184,11 @@ class DbgBuilder:
         self.tab_host[1:] = np.cumsum(self.caps)
         if self.mode == "fused":
             self.batches = [(0, self.np)]
-            ring = _lib.dbg_subgraph_ring_bytes(self.prm, int(self.caps.max(initial=1)) + 64)
+            self.total_slots = int(self.tab_host[-1])
+            ring = _lib.dbg_subgraph_ring_bytes(self.prm, self.group_slots, int(self.caps.max(initial=1)))
             self.ring = _grow(self.ring, ring, torch.uint8, self.device)
-            self.work = _grow(self.work, _lib.dbg_subgraph_workspace_bytes(self.prm, self.np), torch.uint8,
-                              self.device)
+            wsb = _lib.dbg_subgraph_workspace_bytes(self.prm, self.np, self.total_slots, self.group_slots)
+            self.work = _grow(self.work, wsb, torch.uint8, self.device)
             return self.batches
         budget = self.table_budget_bytes
         if budget is None:
@@ -219,9 +223,9 @@ class DbgBuilder:
         stream = stream or torch.cuda.current_stream(self.device)
         if self.mode == "fused":
             ev = self._mark("step2", stream)
-            _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.ring,
-                                     self.ring.numel(), self.work, self.work.numel(), self.out, self.out_cap(),
-                                     self.d_n_out, self.d_stats, self.d_status, stream)
+            _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.total_slots,
+                                     self.group_slots, self.ring, self.ring.numel(), self.work, self.work.numel(),
+                                     self.out, self.out_cap(), self.d_n_out, self.d_stats, self.d_status, stream)
             self._done(ev, stream)
             return
         for (b, e) in self.batches:
@@ -286,9 +290,10 @@ class DbgBuilder:
 
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
                 lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
-                table_budget_bytes: int | None = None, mode: str = "fused") -> GraphResult:
+                table_budget_bytes: int | None = None, mode: str = "fused",
+                group_slots: int = 1 << 19) -> GraphResult:
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
-    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode)
+    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots)
     packed = encode_reads(seq)
     d_bases, d_offsets = builder.upload(packed, offsets)
     return builder.build(d_bases, d_offsets, sort=sort)
