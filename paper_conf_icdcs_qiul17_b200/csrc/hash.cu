@@ -109,12 +109,12 @@ __device__ __forceinline__ void update_vertex(uint32_t* ctr, uint32_t* t_out, co
 
 // Insert-or-update of one occurrence; o in 0..4 (4 = no out-side neighbour),
 // i in -1..3.  Returns false if the probe sequence wrapped (table full).
-__device__ __forceinline__ bool upsert(const Table& t, uint64_t code, int o, int i) {
+__device__ __forceinline__ bool upsert(const Table& t, uint64_t code, int o, int i, uint64_t idx,
+                                       uint64_t first) {
   const uint64_t want = code | kOccupied;
-  uint64_t idx = __umul64hi(slot_hash(code), t.cap);
   for (uint64_t pr = 0; pr < t.cap; ++pr) {
     uint64_t* kp = reinterpret_cast<uint64_t*>(t.keys + idx * 16);
-    uint64_t cur = __ldcg(kp);
+    uint64_t cur = pr ? __ldcg(kp) : first;
     if (cur == 0) {
       cur = atomicCAS(reinterpret_cast<unsigned long long*>(kp), 0ull, (unsigned long long)want);
       if (cur == 0) {
@@ -131,9 +131,9 @@ __device__ __forceinline__ bool upsert(const Table& t, uint64_t code, int o, int
   return false;
 }
 
-__device__ __forceinline__ bool upsert(const Table& t, u128 code, int o, int i) {
+__device__ __forceinline__ bool upsert(const Table& t, u128 code, int o, int i, uint64_t idx, uint64_t first) {
   const uint64_t want_hi = (uint64_t)(code >> 64) | kOccupied, want_lo = (uint64_t)code;
-  uint64_t idx = __umul64hi(slot_hash(code), t.cap);
+  (void)first;  // the 16-byte entry is re-read whole
   for (uint64_t pr = 0; pr < t.cap; ++pr) {
     ulonglong2* kp = reinterpret_cast<ulonglong2*>(t.keys + idx * 32);
     ulonglong2 cur = __ldcg(kp);
@@ -163,61 +163,154 @@ __device__ __forceinline__ bool upsert(const Table& t, u128 code, int o, int i) 
   return false;
 }
 
-template <int R>
-__device__ __forceinline__ uint32_t base_at(const uint32_t (&w)[R], int i) {
-  const int q = i >> 4;
-  uint32_t v = w[1];
-#pragma unroll
-  for (int t = 1; t < R - 1; ++t) v = (q == t) ? w[1 + t] : v;
-  return (v >> (30 - 2 * (i & 15))) & 3u;
+// ----- K-mer decoding from a record held in shared memory (dbg.h layout)
+
+__device__ __forceinline__ uint32_t rec_word(const uint32_t* w, int q, int R) { return q < R ? w[q] : 0u; }
+
+__device__ __forceinline__ uint32_t rec_base(const uint32_t* w, int i) {
+  return (w[1 + (i >> 4)] >> (30 - 2 * (i & 15))) & 3u;
 }
 
-// <kmer, edge> pair generation from one record and the
-// insert/update of every K-mer.  Returns false on overflow.
+// The 64 bits of the record's base string that start at base b.
+__device__ __forceinline__ uint64_t rec_bits64(const uint32_t* w, int b, int R) {
+  const int q = 1 + (b >> 4), off = 2 * (b & 15);
+  const uint64_t hi = ((uint64_t)rec_word(w, q, R) << 32) | rec_word(w, q + 1, R);
+  if (off == 0) return hi;
+  return (hi << off) | (rec_word(w, q + 2, R) >> (32 - off));
+}
+
+__device__ __forceinline__ void kmer_at(const uint32_t* w, int b, int K, int R, uint64_t& fwd, uint64_t& rc) {
+  fwd = rec_bits64(w, b, R) >> (64 - 2 * K);
+  rc = revcomp64(fwd, K);
+}
+
+__device__ __forceinline__ u128 revcomp128(u128 x, int k) {
+  const uint64_t lo = (uint64_t)x, hi = (uint64_t)(x >> 64);
+  uint64_t a = __brevll(~lo), b = __brevll(~hi);  // reversed: the old low half becomes the high half
+  a = ((a >> 1) & 0x5555555555555555ull) | ((a & 0x5555555555555555ull) << 1);
+  b = ((b >> 1) & 0x5555555555555555ull) | ((b & 0x5555555555555555ull) << 1);
+  return (((u128)a << 64) | (u128)b) >> (128 - 2 * k);
+}
+
+__device__ __forceinline__ void kmer_at(const uint32_t* w, int b, int K, int R, u128& fwd, u128& rc) {
+  const uint64_t hi = rec_bits64(w, b, R), lo = rec_bits64(w, b + 32, R);
+  fwd = (((u128)hi << 64) | (u128)lo) >> (128 - 2 * K);
+  rc = revcomp128(fwd, K);
+}
+
+// Per-warp staging of up to 32 records: words, table placement, K-mer prefix.
+template <int R>
+struct WarpRecs {
+  uint32_t w[32][R];
+  unsigned long long t0[32];   // first slot of the record's table (table-block coordinates)
+  unsigned long long cap[32];  // capacity of that table
+  uint32_t pre[33];            // exclusive prefix of the records' K-mer counts
+};
+
+// One occurrence to insert/update: canonical code, out-side counter o (0..3,
+// 4 = t_out), in-side counter i (-1..3), its table and first probe slot.
+template <typename Code>
+struct Job {
+  Code code;
+  int o, i;
+  uint64_t t0, cap, idx;
+  bool valid;
+};
+
+// Decodes K-mer number kid of the warp's records (the cursor r only moves
+// forward): <kmer, edge> pair generation, in the canonical
+// orientation of reading J.
 template <typename Code, int R>
-__device__ __forceinline__ bool hash_record(const uint32_t* rp, int K, const Table& t) {
-  uint32_t w[R];
-  const uint4* src = reinterpret_cast<const uint4*>(rp);
-#pragma unroll
-  for (int v = 0; v < R / 4; ++v) {
-    const uint4 x = __ldcs(src + v);  // streamed once
-    w[4 * v] = x.x;
-    w[4 * v + 1] = x.y;
-    w[4 * v + 2] = x.z;
-    w[4 * v + 3] = x.w;
-  }
+__device__ __forceinline__ Job<Code> make_job(const WarpRecs<R>& sm, uint32_t kid, uint32_t total, int& r, int K) {
+  Job<Code> jb;
+  jb.valid = kid < total;
+  if (!jb.valid) return jb;
+  while (sm.pre[r + 1] <= kid) ++r;
+  const uint32_t* w = sm.w[r];
   const uint32_t hdr = w[0];
-  const int n = hdr & 255u;
-  const int hl = (hdr >> 8) & 1u, hr = (hdr >> 9) & 1u;
-  const Code mask = ((Code)1 << (2 * K)) - 1;
-  const int top = 2 * K - 2;
-  Code fwd = 0, rc = 0;
-  for (int j = 0; j < K; ++j) {
-    const uint32_t b = base_at<R>(w, hl + j);
-    fwd = (fwd << 2) | (Code)b;
-    rc |= (Code)(3u - b) << (2 * j);
+  const int n = hdr & 255u, hl = (hdr >> 8) & 1u, hr = (hdr >> 9) & 1u;
+  const int t = (int)(kid - sm.pre[r]);
+  const int b = hl + t;  // first base of the K-mer in the record
+  Code fwd, rc;
+  kmer_at(w, b, K, R, fwd, rc);
+  const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1) : -1;
+  const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K) : -1;
+  if (fwd < rc) {  // odd K: never equal (reading C)
+    jb.code = fwd;
+    jb.o = succ >= 0 ? succ : 4;
+    jb.i = pred;
+  } else {
+    jb.code = rc;
+    jb.o = pred >= 0 ? 3 - pred : 4;
+    jb.i = succ >= 0 ? 3 - succ : -1;
   }
-  int pred = hl ? (int)base_at<R>(w, 0) : -1;
+  jb.t0 = sm.t0[r];
+  jb.cap = sm.cap[r];
+  jb.idx = __umul64hi(slot_hash(jb.code), jb.cap);
+  return jb;
+}
+
+template <typename Code>
+__device__ __forceinline__ bool resolve(const Job<Code>& jb, char* keys, uint32_t* ctr, uint64_t first) {
+  constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
+  Table t;
+  t.keys = keys + jb.t0 * KE;
+  t.ctr = ctr + jb.t0 * 8;
+  t.cap = jb.cap;
+  return upsert(t, jb.code, jb.o, jb.i, jb.idx, first);
+}
+
+// Insert/update of every K-mer of up to 32 records per warp.
+// The warp's K-mers are dealt round-robin to its lanes (no lane idles behind
+// a long record), two per lane at a time with both first probes in flight.
+// table_of(pid, t0, cap) places a partition's table in the block [keys, ctr).
+// Returns false if a table overflowed.
+template <typename Code, int R, typename TableOf>
+__device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, int K, char* keys, uint32_t* ctr,
+                                          TableOf table_of, WarpRecs<R>& sm) {
+  constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
+  const int lane = threadIdx.x & 31;
+  uint32_t n = 0;
+  if (lane < n_recs) {
+    const uint4* src = reinterpret_cast<const uint4*>(recs + (uint64_t)lane * R);
+#pragma unroll
+    for (int v = 0; v < R / 4; ++v) {
+      const uint4 x = __ldcs(src + v);  // streamed once
+      sm.w[lane][4 * v] = x.x;
+      sm.w[lane][4 * v + 1] = x.y;
+      sm.w[lane][4 * v + 2] = x.z;
+      sm.w[lane][4 * v + 3] = x.w;
+    }
+    const uint32_t hdr = sm.w[lane][0];
+    n = hdr & 255u;
+    uint64_t t0, cap;
+    table_of(hdr >> 10, t0, cap);
+    sm.t0[lane] = t0;
+    sm.cap[lane] = cap;
+  }
+  uint32_t incl = n;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t v = __shfl_up_sync(kFull, incl, d);
+    if (lane >= d) incl += v;
+  }
+  sm.pre[lane + 1] = incl;
+  if (lane == 0) sm.pre[0] = 0;
+  const uint32_t total = __shfl_sync(kFull, incl, 31);
+  __syncwarp();
   bool ok = true;
-  for (int s = 0; s < n; ++s) {
-    const bool has_succ = s < n - 1 || hr;
-    const int succ = has_succ ? (int)base_at<R>(w, hl + s + K) : -1;
-    const bool is_fwd = fwd < rc;  // odd K: never equal (reading C)
-    int o, i;
-    if (is_fwd) {  // reading J
-      o = succ >= 0 ? succ : 4;
-      i = pred;
-    } else {
-      o = pred >= 0 ? 3 - pred : 4;
-      i = succ >= 0 ? 3 - succ : -1;
-    }
-    ok &= upsert(t, is_fwd ? fwd : rc, o, i);
-    if (s + 1 < n) {
-      pred = (int)(uint32_t)(fwd >> top) & 3;
-      fwd = ((fwd << 2) | (Code)succ) & mask;
-      rc = (rc >> 2) | ((Code)(3 - succ) << top);
-    }
+  int ra = 0, rb = 0;
+  for (uint32_t kid = lane; kid < total; kid += 64) {
+    const Job<Code> A = make_job<Code, R>(sm, kid, total, ra, K);
+    if (rb < ra) rb = ra;
+    const Job<Code> B = make_job<Code, R>(sm, kid + 32, total, rb, K);
+    const uint64_t fa = __ldcg(reinterpret_cast<const unsigned long long*>(keys + (A.t0 + A.idx) * KE));
+    const uint64_t fb = B.valid ? __ldcg(reinterpret_cast<const unsigned long long*>(keys + (B.t0 + B.idx) * KE))
+                                : 0ull;
+    ok &= resolve(A, keys, ctr, fa);
+    if (B.valid) ok &= resolve(B, keys, ctr, fb);
   }
+  __syncwarp();
   return ok;
 }
 
@@ -333,19 +426,23 @@ struct ResidentArgs {
 template <typename Code, int R>
 __global__ void __launch_bounds__(kThreads) hash_build_kernel(ResidentArgs a) {
   constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
+  __shared__ WarpRecs<R> sh[kThreads / 32];
   const uint64_t r_begin = a.rec_off[a.pid_begin], r_end = a.rec_off[a.pid_end];
   const uint64_t s0 = a.tab_off[a.pid_begin], n_slots = a.tab_off[a.pid_end] - s0;
   uint32_t* ctr_base = reinterpret_cast<uint32_t*>(a.table + n_slots * KE);
-  for (uint64_t rec = r_begin + (uint64_t)blockIdx.x * kThreads + threadIdx.x; rec < r_end;
-       rec += (uint64_t)gridDim.x * kThreads) {
-    const uint32_t* rp = a.records + rec * R;
-    const uint32_t pid = __ldg(rp) >> 10;
-    const uint64_t t0 = __ldg(a.tab_off + pid) - s0;
-    Table t;
-    t.keys = a.table + t0 * KE;
-    t.ctr = ctr_base + t0 * 8;
-    t.cap = __ldg(a.tab_off + pid + 1) - __ldg(a.tab_off + pid);
-    if (!hash_record<Code, R>(rp, a.k, t)) atomicOr(a.status, kStatusTableFull);
+  const uint64_t* off = a.tab_off;
+  auto table_of = [=](uint32_t pid, uint64_t& t0, uint64_t& cap) {
+    t0 = __ldg(off + pid) - s0;
+    cap = __ldg(off + pid + 1) - __ldg(off + pid);
+  };
+  const int warp = threadIdx.x >> 5;
+  const uint64_t n_chunks = (r_end - r_begin + 31) / 32;
+  for (uint64_t c = (uint64_t)blockIdx.x * (kThreads / 32) + warp; c < n_chunks;
+       c += (uint64_t)gridDim.x * (kThreads / 32)) {
+    const uint64_t r0 = r_begin + 32 * c;
+    const int64_t n = (int64_t)min((uint64_t)32, r_end - r0);
+    if (!hash_warp<Code, R>(a.records + r0 * R, n, a.k, a.table, ctr_base, table_of, sh[warp]))
+      atomicOr(a.status, kStatusTableFull);
   }
 }
 
@@ -381,8 +478,8 @@ __global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, Ou
 // earlier stage, so the schedule cannot deadlock, and the lag of extraction
 // behind hashing keeps CTAs from stalling on a group's last hash items.
 
-constexpr int kLagX = 2;
-constexpr int kRingGroups = kLagX + 4;
+constexpr int kLagX = 1;
+constexpr int kRingGroups = kLagX + 3;
 
 struct SubgraphArgs {
   const uint32_t* records;
@@ -485,6 +582,7 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   constexpr uint32_t KE = KW == 1 ? 16 : 32;
   __shared__ XShared sh;
+  __shared__ WarpRecs<R> shw[kThreads / 32];
   __shared__ unsigned long long s_item;
   const int n_g = (int)a.work[1];
   const int n_stage = n_g + 1 + kLagX;
@@ -543,16 +641,18 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
       const uint64_t n16 = s1 > s0 ? (s1 - s0) * (KE / 16) : 0;
       for (uint64_t q = threadIdx.x; q < n16; q += kThreads) __stcg(z + q, make_uint4(0, 0, 0, 0));
     } else if (kind == 1) {
-      const uint64_t r = j * kHashRecs + threadIdx.x;
-      if (r < G.nrec) {
-        const uint32_t* rp = a.records + (G.rec0 + r) * R;
-        const uint32_t pid = __ldg(rp) >> 10;
-        const uint64_t t0 = a.tab_off[pid] - G.slot0;
-        Table t;
-        t.keys = keys + t0 * KE;
-        t.ctr = ctr + t0 * 8;
-        t.cap = a.tab_off[pid + 1] - a.tab_off[pid];
-        if (!hash_record<Code, R>(rp, a.k, t)) atomicOr(oa.status, kStatusTableFull);
+      const int warp = threadIdx.x >> 5;
+      const uint64_t r = j * kHashRecs + 32 * warp;
+      const int64_t n = r < G.nrec ? (int64_t)min((uint64_t)32, G.nrec - r) : 0;
+      if (n > 0) {
+        const uint64_t* off = a.tab_off;
+        const uint64_t gs0 = G.slot0;
+        auto table_of = [=](uint32_t pid, uint64_t& t0, uint64_t& cap) {
+          t0 = off[pid] - gs0;
+          cap = off[pid + 1] - off[pid];
+        };
+        if (!hash_warp<Code, R>(a.records + (G.rec0 + r) * R, n, a.k, keys, ctr, table_of, shw[warp]))
+          atomicOr(oa.status, kStatusTableFull);
       }
     } else {
       const uint64_t s0 = j * kExtractSlots;
