@@ -139,10 +139,10 @@ DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kme
                           uint64_t* d_table_offset, cudaStream_t stream);
 
 /* ---- a5-a7 fused: Step 2 through an L2-resident ring (the hot path) ------
- * For partitions [pid_begin, pid_end): zero-fill the key entries of each
- * partition's table, build it (one insertion per distinct vertex, multiple
- * updates, Sec. III-C), and compact it into d_out -- all in one
- * persistent kernel.  Partitions are taken in groups of consecutive
+ * For partitions [pid_begin, pid_end): build each partition's table (one
+ * insertion per distinct vertex, multiple updates, Sec. III-C)
+ * and compact it into d_out -- all in one persistent kernel.  d_ring must be
+ * all-zero when first used (extraction leaves it clean again).  Partitions are taken in groups of consecutive
  * partitions spanning about group_slots table slots (the caller picks it so
  * a few groups fit in L2: the B200 form of sizing tables for locality,
  * P:L665-675); each group's tables live in one of the ring regions of d_ring
@@ -166,10 +166,11 @@ DBG_API dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partitio
  * Inserts every K-mer occurrence of partitions [pid_begin, pid_end) into that
  * partition's table.  d_table holds the tables of all these partitions,
  * n = d_table_offset[pid_end] - d_table_offset[pid_begin] slots: first the n
- * key entries (dbg_key_bytes each, zero-filled by the caller = EMPTY), then
- * n 32-byte counter records (no initialisation needed); partition i owns
- * slots [d_table_offset[i] - d_table_offset[pid_begin], ...) of both arrays.
- * Overflow sets bit 0 of *d_status (reported by dbg_sync_status). */
+ * key entries (dbg_key_bytes each), then n 32-byte counter records; partition
+ * i owns slots [d_table_offset[i] - d_table_offset[pid_begin], ...) of both
+ * arrays.  The table must be all-zero (memset once when allocated:
+ * dbg_extract_graph zeroes every slot it reads, so an extracted table is
+ * clean again).  Overflow sets bit 0 of *d_status (dbg_sync_status). */
 DBG_API dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
                           int32_t pid_end, void* d_table, const uint64_t* d_table_offset,
                           uint32_t* d_status, cudaStream_t stream);
@@ -177,10 +178,11 @@ DBG_API dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set
 /* ---- a7: output (Def. 3) -------------------------------------
  * Compacts the occupied slots of resident tables (layout of dbg_hash_build)
  * into d_out[*d_n_out ...] (appends; the caller zeroes *d_n_out and *d_stats
- * once) and accumulates *d_stats.  Records beyond out_cap are dropped and
+ * once), accumulates *d_stats, and zeroes every slot it read (the table is
+ * clean for the next dbg_hash_build).  Records beyond out_cap are dropped and
  * set bit 1 of *d_status (DBG_ENOSPACE; *d_n_out still counts them).
  * Record order is unspecified (reading S): use dbg_sort_vertices. */
-DBG_API dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_table,
+DBG_API dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table,
                              const uint64_t* d_table_offset, int32_t pid_begin, int32_t pid_end,
                              dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
                              dbg_stats* d_stats, uint32_t* d_status, cudaStream_t stream);

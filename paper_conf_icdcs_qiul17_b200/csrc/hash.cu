@@ -3,23 +3,27 @@
 // star, plus extraction of the vertex records (Def. 3).
 //
 // Table of one partition with capacity n (open addressing, linear probing):
-//   key entries  n x KE bytes  (zero-filled = EMPTY)
+//   key entries  n x KE bytes
 //     K <= 31: KE = 16  { u64 key; u32 t_out; u32 pad }
 //     K <= 63: KE = 32  { u64 key_hi; u64 key_lo; u32 t_out; u32 pad[3] }
-//   counters     n x 32 bytes  { u32 out[4]; u32 in[4] }  (never zero-filled)
-// The key word (hi word for K > 31) carries the paper's occupancy state
-// (Sec. III-C3, Fig. 4) in its two top bits:
-//   0                 empty
-//   OCC | code        locked   (claimed; counters being initialised)
-//   OCC | READY | code occupied (never modified again, read concurrently)
-// One insertion: a thread that sees EMPTY claims the slot with a
-// single 64-bit (K <= 31) or 128-bit (K <= 63) atomicCAS that publishes the
-// whole key at once, initialises the vertex's counters with its own
-// occurrence, and sets READY with a release.  Multiple updates:
-// every other occurrence compares keys and issues red.global.add on two
-// counters; only a thread that finds its own key still "locked" waits (the
-// paper's blocked readers).  So only the 16/32-B key entries need
-// zero-filling, not the 32-B counter records.
+//   counters     n x 32 bytes  { u32 out[4]; u32 in[4] }
+// A key word is 0 (empty) or OCC | code (bit 63 of the hi word = occupied).
+//
+// One insertion, multiple updates: every probe is an
+// atomicCAS(slot, EMPTY, key) -- 64-bit for K <= 31, 128-bit for K <= 63 --
+// whose return value decides in one round trip: EMPTY means this occurrence
+// inserted the vertex (the single insertion), the own key means the vertex is
+// already there, anything else means probe on.  The whole key is published by
+// that one CAS, so the paper's {empty, locked, occupied} protocol for
+// multi-word keys (Fig. 4) collapses to {empty, occupied}: there
+// is no partially written key to wait for.  Then red.global.add on two
+// counters (the multiple updates).
+//
+// Clean-on-extract: tables are all-zero before hashing (one memset when the
+// buffer is allocated), and extraction writes zeros back over every occupied
+// slot it reads.  So no per-partition zero-fill is needed, counters never
+// need initialising by the inserting thread, and no memory fence is needed
+// between the key CAS and the counter updates.
 //
 // Counter economy: each occurrence increments exactly one "out-side" counter
 // (out[c] if it has a successor in the vertex orientation, else t_out) and at
@@ -27,17 +31,12 @@
 // extraction: two reds per K-mer instead of the paper's three.
 //
 // Kernels:
-//  hash_build_kernel    tables of partitions [b, e) resident (dbg_hash_build)
-//  extract_kernel       compaction of resident tables (dbg_extract_graph)
+//  hash_build_kernel    resident tables of partitions [b, e) (dbg_hash_build)
+//  extract_kernel       compaction + clean of resident tables (dbg_extract_graph)
 //  subgraph_kernel      fused Step 2 (dbg_build_subgraphs): a persistent
-//                       kernel streams partitions through a ring of RING
-//                       L2-sized table regions; work items (zero a key chunk,
-//                       hash a record chunk, extract a slot chunk) are claimed
-//                       in a fixed global order from one atomic counter and
-//                       chained by per-partition completion counters, so a
-//                       partition's table lives in L2 from zero-fill to
-//                       extraction (the B200 form of "localize memory access
-//                       by configuring the hash table size").
+//                       kernel streams groups of partitions through a ring of
+//                       L2-sized table regions (hash a record chunk / extract
+//                       a slot chunk, claimed in a fixed global order)
 #include <cub/block/block_reduce.cuh>
 #include <cub/block/block_scan.cuh>
 #include <cub/device/device_radix_sort.cuh>
@@ -52,23 +51,16 @@ namespace dbg {
 typedef unsigned __int128 u128;
 
 constexpr int kThreads = 256;
-constexpr uint64_t kReady = 1ull << 62;
-constexpr uint64_t kCodeMask = kReady - 1;
+constexpr uint64_t kCodeMask = (1ull << 62) - 1;
 constexpr uint64_t kSlotSeed = 0x9e3779b97f4a7c15ull;
-constexpr uint32_t kZeroSlots = 4096;          // key entries per zero item
-constexpr uint32_t kHashRecs = kThreads;       // records per hash item
+constexpr uint32_t kHashRecs = kThreads;  // records per hash item (32 per warp)
 constexpr int kXPer = 8;
 constexpr uint32_t kExtractSlots = kThreads * kXPer;
 constexpr uint32_t kStatusRing = 4u;
+constexpr int kJobs = 4;  // occurrences in flight per lane
 
 __host__ __device__ inline uint32_t key_bytes(int k) { return k <= 31 ? 16u : 32u; }
 constexpr uint32_t kCtrBytes = 32;
-
-struct Table {
-  char* keys;      // key entries
-  uint32_t* ctr;   // counter records (8 u32 each)
-  uint64_t cap;
-};
 
 __device__ __forceinline__ uint64_t slot_hash(uint64_t code) { return fmix64(code ^ kSlotSeed); }
 __device__ __forceinline__ uint64_t slot_hash(u128 code) {
@@ -78,90 +70,41 @@ __device__ __forceinline__ uint64_t slot_hash(u128 code) {
 __device__ __forceinline__ void red_add(uint32_t* p) {
   asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(p) : "memory");
 }
-__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
 __device__ __forceinline__ uint32_t ld_acquire32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
 
-// Claimer: counters start at this occurrence's increments; then READY.
-__device__ __forceinline__ void init_vertex(uint32_t* ctr, uint32_t* t_out, uint64_t* state, int o, int i) {
-  uint4* cp = reinterpret_cast<uint4*>(ctr);
-  __stcg(cp, make_uint4(o == 0, o == 1, o == 2, o == 3));
-  __stcg(cp + 1, make_uint4(i == 0, i == 1, i == 2, i == 3));
-  __stcg(t_out, (uint32_t)(o == 4));
-  __threadfence();
-  atomicOr(reinterpret_cast<unsigned long long*>(state), (unsigned long long)kReady);
-}
+// ----- key words and the probe CAS
 
-__device__ __forceinline__ void update_vertex(uint32_t* ctr, uint32_t* t_out, const uint64_t* state,
-                                              uint64_t seen, int o, int i) {
-  if (!(seen & kReady))  // locked: blocked until the claimer publishes
-    while (!(ld_acquire(state) & kReady)) __nanosleep(20);
-  red_add(o < 4 ? ctr + o : t_out);
-  if (i >= 0) red_add(ctr + 4 + i);
-}
-
-// Insert-or-update of one occurrence; o in 0..4 (4 = no out-side neighbour),
-// i in -1..3.  Returns false if the probe sequence wrapped (table full).
-__device__ __forceinline__ bool upsert(const Table& t, uint64_t code, int o, int i, uint64_t idx,
-                                       uint64_t first) {
-  const uint64_t want = code | kOccupied;
-  for (uint64_t pr = 0; pr < t.cap; ++pr) {
-    uint64_t* kp = reinterpret_cast<uint64_t*>(t.keys + idx * 16);
-    uint64_t cur = pr ? __ldcg(kp) : first;
-    if (cur == 0) {
-      cur = atomicCAS(reinterpret_cast<unsigned long long*>(kp), 0ull, (unsigned long long)want);
-      if (cur == 0) {
-        init_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), kp, o, i);
-        return true;
-      }
-    }
-    if ((cur & ~kReady) == want) {
-      update_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), kp, cur, o, i);
-      return true;
-    }
-    idx = idx + 1 == t.cap ? 0 : idx + 1;
+template <typename Code>
+struct KeyOf;
+template <>
+struct KeyOf<uint64_t> {
+  typedef unsigned long long T;
+  static __device__ __forceinline__ T make(uint64_t code) { return code | kOccupied; }
+  static __device__ __forceinline__ bool empty(T v) { return v == 0; }
+  static __device__ __forceinline__ bool same(T a, T b) { return a == b; }
+  static __device__ __forceinline__ T cas(char* kp, T want) {
+    return atomicCAS(reinterpret_cast<unsigned long long*>(kp), 0ull, want);
   }
-  return false;
-}
-
-__device__ __forceinline__ bool upsert(const Table& t, u128 code, int o, int i, uint64_t idx, uint64_t first) {
-  const uint64_t want_hi = (uint64_t)(code >> 64) | kOccupied, want_lo = (uint64_t)code;
-  (void)first;  // the 16-byte entry is re-read whole
-  for (uint64_t pr = 0; pr < t.cap; ++pr) {
-    ulonglong2* kp = reinterpret_cast<ulonglong2*>(t.keys + idx * 32);
-    ulonglong2 cur = __ldcg(kp);
-    if (cur.x == 0) {  // empty -- or a torn read of a key being published: the CAS decides
-      ulonglong2 want;
-      want.x = want_hi;
-      want.y = want_lo;
-      cur = atomicCAS(kp, make_ulonglong2(0ull, 0ull), want);
-      if (cur.x == 0 && cur.y == 0) {
-        init_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), reinterpret_cast<uint64_t*>(kp),
-                    o, i);
-        return true;
-      }
-    } else if (cur.y == 0) {
-      // a 16-B load is not single-copy atomic: a claimed hi word next to a zero low
-      // word may be a torn read of a key being published -- the no-op CAS returns
-      // the entry atomically
-      cur = atomicCAS(kp, cur, cur);
-    }
-    if ((cur.x & ~kReady) == want_hi && cur.y == want_lo) {
-      update_vertex(t.ctr + idx * 8, reinterpret_cast<uint32_t*>(kp + 1), reinterpret_cast<uint64_t*>(kp),
-                    cur.x, o, i);
-      return true;
-    }
-    idx = idx + 1 == t.cap ? 0 : idx + 1;
+};
+template <>
+struct KeyOf<u128> {
+  typedef ulonglong2 T;
+  static __device__ __forceinline__ T make(u128 code) {
+    T t;
+    t.x = (uint64_t)(code >> 64) | kOccupied;  // hi word: <= 62 code bits + OCC
+    t.y = (uint64_t)code;
+    return t;
   }
-  return false;
-}
+  static __device__ __forceinline__ bool empty(T v) { return v.x == 0 && v.y == 0; }
+  static __device__ __forceinline__ bool same(T a, T b) { return a.x == b.x && a.y == b.y; }
+  static __device__ __forceinline__ T cas(char* kp, T want) {
+    return atomicCAS(reinterpret_cast<ulonglong2*>(kp), make_ulonglong2(0ull, 0ull), want);
+  }
+};
 
 // ----- K-mer decoding from a record held in shared memory (dbg.h layout)
 
@@ -207,24 +150,21 @@ struct WarpRecs {
   uint32_t pre[33];            // exclusive prefix of the records' K-mer counts
 };
 
-// One occurrence to insert/update: canonical code, out-side counter o (0..3,
-// 4 = t_out), in-side counter i (-1..3), its table and first probe slot.
+// One occurrence: canonical key, out-side counter o (0..3, 4 = t_out), in-side
+// counter i (-1..3), its table and current probe slot.
 template <typename Code>
 struct Job {
-  Code code;
-  int o, i;
+  typename KeyOf<Code>::T want;
   uint64_t t0, cap, idx;
-  bool valid;
+  int o, i;
 };
 
 // Decodes K-mer number kid of the warp's records (the cursor r only moves
 // forward): <kmer, edge> pair generation, in the canonical
 // orientation of reading J.
 template <typename Code, int R>
-__device__ __forceinline__ Job<Code> make_job(const WarpRecs<R>& sm, uint32_t kid, uint32_t total, int& r, int K) {
+__device__ __forceinline__ Job<Code> make_job(const WarpRecs<R>& sm, uint32_t kid, int& r, int K) {
   Job<Code> jb;
-  jb.valid = kid < total;
-  if (!jb.valid) return jb;
   while (sm.pre[r + 1] <= kid) ++r;
   const uint32_t* w = sm.w[r];
   const uint32_t hdr = w[0];
@@ -235,39 +175,33 @@ __device__ __forceinline__ Job<Code> make_job(const WarpRecs<R>& sm, uint32_t ki
   kmer_at(w, b, K, R, fwd, rc);
   const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1) : -1;
   const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K) : -1;
+  Code code;
   if (fwd < rc) {  // odd K: never equal (reading C)
-    jb.code = fwd;
+    code = fwd;
     jb.o = succ >= 0 ? succ : 4;
     jb.i = pred;
   } else {
-    jb.code = rc;
+    code = rc;
     jb.o = pred >= 0 ? 3 - pred : 4;
     jb.i = succ >= 0 ? 3 - succ : -1;
   }
+  jb.want = KeyOf<Code>::make(code);
   jb.t0 = sm.t0[r];
   jb.cap = sm.cap[r];
-  jb.idx = __umul64hi(slot_hash(jb.code), jb.cap);
+  jb.idx = __umul64hi(slot_hash(code), jb.cap);
   return jb;
 }
 
-template <typename Code>
-__device__ __forceinline__ bool resolve(const Job<Code>& jb, char* keys, uint32_t* ctr, uint64_t first) {
-  constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
-  Table t;
-  t.keys = keys + jb.t0 * KE;
-  t.ctr = ctr + jb.t0 * 8;
-  t.cap = jb.cap;
-  return upsert(t, jb.code, jb.o, jb.i, jb.idx, first);
-}
-
 // Insert/update of every K-mer of up to 32 records per warp.
-// The warp's K-mers are dealt round-robin to its lanes (no lane idles behind
-// a long record), two per lane at a time with both first probes in flight.
+// Lane l takes a contiguous share of the warp's K-mers (balanced whatever the
+// record lengths) and keeps kJobs occurrences in flight: their probe CASes
+// are issued together, collisions are resolved, then the counter reds.
 // table_of(pid, t0, cap) places a partition's table in the block [keys, ctr).
 // Returns false if a table overflowed.
 template <typename Code, int R, typename TableOf>
 __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, int K, char* keys, uint32_t* ctr,
                                           TableOf table_of, WarpRecs<R>& sm) {
+  typedef KeyOf<Code> KO;
   constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
   const int lane = threadIdx.x & 31;
   uint32_t n = 0;
@@ -298,17 +232,40 @@ __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, 
   if (lane == 0) sm.pre[0] = 0;
   const uint32_t total = __shfl_sync(kFull, incl, 31);
   __syncwarp();
+  const uint32_t share = (total + 31) / 32;
+  const uint32_t k0 = min(total, lane * share), k1 = min(total, k0 + share);
   bool ok = true;
-  int ra = 0, rb = 0;
-  for (uint32_t kid = lane; kid < total; kid += 64) {
-    const Job<Code> A = make_job<Code, R>(sm, kid, total, ra, K);
-    if (rb < ra) rb = ra;
-    const Job<Code> B = make_job<Code, R>(sm, kid + 32, total, rb, K);
-    const uint64_t fa = __ldcg(reinterpret_cast<const unsigned long long*>(keys + (A.t0 + A.idx) * KE));
-    const uint64_t fb = B.valid ? __ldcg(reinterpret_cast<const unsigned long long*>(keys + (B.t0 + B.idx) * KE))
-                                : 0ull;
-    ok &= resolve(A, keys, ctr, fa);
-    if (B.valid) ok &= resolve(B, keys, ctr, fb);
+  int r = 0;
+  for (uint32_t kid = k0; kid < k1; kid += kJobs) {
+    Job<Code> jb[kJobs];
+    typename KO::T cur[kJobs];
+    bool live[kJobs];
+#pragma unroll
+    for (int q = 0; q < kJobs; ++q) {
+      live[q] = kid + q < k1;
+      if (live[q]) {
+        jb[q] = make_job<Code, R>(sm, kid + q, r, K);
+        cur[q] = KO::cas(keys + (jb[q].t0 + jb[q].idx) * KE, jb[q].want);  // probe = insert attempt
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < kJobs; ++q) {
+      if (!live[q]) continue;
+      uint64_t probes = 1;
+      while (!KO::empty(cur[q]) && !KO::same(cur[q], jb[q].want)) {  // occupied by another vertex
+        if (probes++ == jb[q].cap) break;
+        jb[q].idx = jb[q].idx + 1 == jb[q].cap ? 0 : jb[q].idx + 1;
+        cur[q] = KO::cas(keys + (jb[q].t0 + jb[q].idx) * KE, jb[q].want);
+      }
+      if (!KO::empty(cur[q]) && !KO::same(cur[q], jb[q].want)) {
+        ok = false;  // wrapped: table full (reading O)
+        continue;
+      }
+      const uint64_t s = jb[q].t0 + jb[q].idx;
+      uint32_t* c = ctr + s * 8;
+      red_add(jb[q].o < 4 ? c + jb[q].o : reinterpret_cast<uint32_t*>(keys + s * KE + KE / 2));
+      if (jb[q].i >= 0) red_add(c + 4 + jb[q].i);
+    }
   }
   __syncwarp();
   return ok;
@@ -331,11 +288,11 @@ struct XShared {
 };
 
 // Block-wide: compact the occupied entries among slots [0, n) of a contiguous
-// key/counter range into records; pid_of(local slot) gives the partition.
-// Two passes keep registers low: occupancy bits + block scan, then re-read
-// (L1/L2 hits) and write each occupied entry.
+// key/counter range into records and zero them again (clean-on-extract);
+// pid_of(local slot) gives the partition.  Two passes keep registers low:
+// occupancy bits + block scan, then re-read (L1/L2 hits), write, clean.
 template <int KW, typename PidFn>
-__device__ __forceinline__ void extract_tile(const char* keys, const uint32_t* ctr, uint64_t n, PidFn pid_of,
+__device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t n, PidFn pid_of,
                                              const OutArgs& oa, XShared& sh) {
   constexpr uint32_t KE = KW == 1 ? 16 : 32;
   uint32_t bits = 0;
@@ -355,21 +312,26 @@ __device__ __forceinline__ void extract_tile(const char* keys, const uint32_t* c
     const int q = __ffs(bits) - 1;
     bits &= bits - 1;
     const uint64_t s = (uint64_t)q * kThreads + threadIdx.x;
-    const uint64_t* kp = reinterpret_cast<const uint64_t*>(keys + s * KE);
-    const uint64_t k0 = __ldcg(kp);
+    uint4* kp4 = reinterpret_cast<uint4*>(keys + s * KE);
+    const uint4 e0 = __ldcg(kp4);
     dbg_vertex v;
     uint32_t tout;
     if (KW == 1) {
       v.kmer_hi = 0;
-      v.kmer_lo = k0 & kCodeMask;
-      tout = __ldcg(reinterpret_cast<const uint32_t*>(kp + 1));
+      v.kmer_lo = (((uint64_t)e0.y << 32) | e0.x) & kCodeMask;
+      tout = e0.z;
     } else {
-      v.kmer_hi = k0 & kCodeMask;
-      v.kmer_lo = __ldcg(kp + 1);
-      tout = __ldcg(reinterpret_cast<const uint32_t*>(kp + 2));
+      v.kmer_hi = (((uint64_t)e0.y << 32) | e0.x) & kCodeMask;
+      v.kmer_lo = ((uint64_t)e0.w << 32) | e0.z;
+      tout = __ldcg(reinterpret_cast<const uint32_t*>(kp4 + 1));
     }
-    const uint4* cp = reinterpret_cast<const uint4*>(ctr + s * 8);
+    uint4* cp = reinterpret_cast<uint4*>(ctr + s * 8);
     const uint4 a = __ldcg(cp), b = __ldcg(cp + 1);
+    const uint4 z = make_uint4(0, 0, 0, 0);
+    __stcg(kp4, z);  // clean-on-extract
+    if (KW == 2) __stcg(kp4 + 1, z);
+    __stcg(cp, z);
+    __stcg(cp + 1, z);
     v.out[0] = a.x; v.out[1] = a.y; v.out[2] = a.z; v.out[3] = a.w;
     v.in[0] = b.x; v.in[1] = b.y; v.in[2] = b.z; v.in[3] = b.w;
     v.count = a.x + a.y + a.z + a.w + tout;  // count = sum(out) + t_out
@@ -451,7 +413,7 @@ __global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, Ou
   constexpr uint32_t KE = KW == 1 ? 16 : 32;
   __shared__ XShared sh;
   const uint64_t s0 = a.tab_off[a.pid_begin], n_slots = a.tab_off[a.pid_end] - s0;
-  const uint32_t* ctr_base = reinterpret_cast<const uint32_t*>(a.table + n_slots * KE);
+  uint32_t* ctr_base = reinterpret_cast<uint32_t*>(a.table + n_slots * KE);
   for (uint64_t t0 = (uint64_t)blockIdx.x * kExtractSlots; t0 < n_slots; t0 += (uint64_t)gridDim.x * kExtractSlots) {
     const uint64_t n = min((uint64_t)kExtractSlots, n_slots - t0);
     const int lo = a.pid_begin, hi = a.pid_end;
@@ -466,17 +428,15 @@ __global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, Ou
 // Partitions [b, e) are cut into groups of consecutive partitions: partition
 // p belongs to group floor((tab_off[p] - tab_off[b]) / group_slots), so a
 // group spans at most group_slots + max capacity slots.  Group g uses ring
-// region g % kRing: key entries of the group's partitions back to back, then
-// their counter records.  The work list is a sequence of stages; stage s holds
-//   Z(s)          zero-fill the key entries of group s,
-//   H(s-1)        hash the records of group s-1,
-//   X(s-1-kLagX)  extract group s-1-kLagX,
-// and CTAs claim items in list order.  Dependencies (per-group completion
-// counters): H(g) after Z(g); X(g) after H(g); Z(g) after Z(g-kRing) and
-// X(g-kRing) (ring reuse; every group has >= 1 zero item so the chain is
-// transitive through empty groups).  Every dependency of an item lies in an
-// earlier stage, so the schedule cannot deadlock, and the lag of extraction
-// behind hashing keeps CTAs from stalling on a group's last hash items.
+// region g % kRingGroups: key entries of the group's partitions back to back,
+// then their counter records.  The work list is a sequence of stages; stage s
+// holds H(s) (hash the records of group s) and X(s-1-kLagX) (extract group
+// s-1-kLagX), and CTAs claim items in list order.  Dependencies (per-group
+// completion counters): X(g) after H(g); H(g) after H(g-kRingGroups) and
+// X(g-kRingGroups) (ring reuse: the region is clean again; every group has
+// >= 1 hash item so the chain is transitive through empty groups).  Every
+// dependency of an item lies in an earlier stage, so the schedule cannot
+// deadlock; the lag keeps CTAs from stalling on a group's last hash items.
 
 constexpr int kLagX = 1;
 constexpr int kRingGroups = kLagX + 3;
@@ -492,15 +452,15 @@ struct SubgraphArgs {
   uint32_t* gfirst;               // [n_groups_max + 1] first partition of each group
   unsigned long long* stage_off;  // [n_groups_max + kLagX + 3]
   unsigned long long* work;       // [0] claimed-item counter, [1] n_groups
-  uint32_t* done;                 // [3][n_groups_max]: zero, hash, extract items done
+  uint32_t* done;                 // [2][n_groups_max]: hash, extract items done
 };
 
 __device__ __forceinline__ uint64_t div_up(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
 struct GroupGeom {
-  int p0, p1;              // partitions [p0, p1)
-  uint64_t slot0, span;    // first slot (tab_off coordinates), slots
-  uint64_t rec0, nrec;     // records
+  int p0, p1;            // partitions [p0, p1)
+  uint64_t slot0, span;  // first slot (tab_off coordinates), slots
+  uint64_t rec0, nrec;   // records
 };
 __device__ __forceinline__ GroupGeom ggeom(const SubgraphArgs& a, int g) {
   GroupGeom G;
@@ -512,8 +472,7 @@ __device__ __forceinline__ GroupGeom ggeom(const SubgraphArgs& a, int g) {
   G.nrec = a.rec_off[G.p1] - G.rec0;
   return G;
 }
-__device__ __forceinline__ uint64_t nz_items(const GroupGeom& G) { return G.span ? div_up(G.span, kZeroSlots) : 1; }
-__device__ __forceinline__ uint64_t nh_items(const GroupGeom& G) { return div_up(G.nrec, kHashRecs); }
+__device__ __forceinline__ uint64_t nh_items(const GroupGeom& G) { return G.nrec ? div_up(G.nrec, kHashRecs) : 1; }
 __device__ __forceinline__ uint64_t nx_items(const GroupGeom& G) { return div_up(G.span, kExtractSlots); }
 
 // Single CTA: groups, stage offsets of the work list, zeroed completion counters.
@@ -542,7 +501,7 @@ __global__ void __launch_bounds__(kThreads) subgraph_plan_kernel(SubgraphArgs a,
     }
     a.gfirst[g] = (uint32_t)lo;
   }
-  for (uint64_t i = threadIdx.x; i < 3 * n_g; i += kThreads) a.done[i] = 0;
+  for (uint64_t i = threadIdx.x; i < 2 * n_g; i += kThreads) a.done[i] = 0;
   if (threadIdx.x == 0) {
     carry = 0;
     a.work[0] = 0;
@@ -557,9 +516,8 @@ __global__ void __launch_bounds__(kThreads) subgraph_plan_kernel(SubgraphArgs a,
       if (s < (int)n_g) {
         const GroupGeom G = ggeom(a, s);
         if (G.span > a.region_slots) atomicOr(status, kStatusRing);
-        items += nz_items(G);
+        items += nh_items(G);
       }
-      if (s >= 1 && s - 1 < (int)n_g) items += nh_items(ggeom(a, s - 1));
       if (s >= 1 + kLagX) items += nx_items(ggeom(a, s - 1 - kLagX));
     }
     unsigned long long excl, tot;
@@ -587,9 +545,8 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
   const int n_g = (int)a.work[1];
   const int n_stage = n_g + 1 + kLagX;
   const unsigned long long total = a.stage_off[n_stage];
-  uint32_t* done_z = a.done;
-  uint32_t* done_h = a.done + n_g;
-  uint32_t* done_x = a.done + 2 * n_g;
+  uint32_t* done_h = a.done;
+  uint32_t* done_x = a.done + n_g;
   for (;;) {
     if (threadIdx.x == 0) s_item = atomicAdd(a.work, 1ull);
     __syncthreads();
@@ -608,14 +565,8 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
     GroupGeom G;
     if (s < n_g) {
       G = ggeom(a, s);
-      const uint64_t n = nz_items(G);
-      if (j < n) kind = 0, g = s;
-      else j -= n;
-    }
-    if (kind < 0 && s >= 1 && s - 1 < n_g) {
-      G = ggeom(a, s - 1);
       const uint64_t n = nh_items(G);
-      if (j < n) kind = 1, g = s - 1;
+      if (j < n) kind = 1, g = s;
       else j -= n;
     }
     if (kind < 0) {
@@ -626,21 +577,15 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
     char* keys = a.ring + (uint64_t)(g % kRingGroups) * a.region_bytes;
     uint32_t* ctr = reinterpret_cast<uint32_t*>(keys + a.region_slots * KE);
     if (threadIdx.x == 0) {
-      if (kind == 0 && g >= kRingGroups) {  // ring reuse: the previous user is fully extracted
+      if (kind == 1 && g >= kRingGroups) {  // ring reuse: the previous user is extracted (and clean)
         const GroupGeom Q = ggeom(a, g - kRingGroups);
-        wait_count(done_z + g - kRingGroups, (uint32_t)nz_items(Q));
+        wait_count(done_h + g - kRingGroups, (uint32_t)nh_items(Q));
         wait_count(done_x + g - kRingGroups, (uint32_t)nx_items(Q));
       }
-      if (kind == 1) wait_count(done_z + g, (uint32_t)nz_items(G));
       if (kind == 2) wait_count(done_h + g, (uint32_t)nh_items(G));
     }
     __syncthreads();
-    if (kind == 0) {
-      const uint64_t s0 = j * kZeroSlots, s1 = min(G.span, s0 + kZeroSlots);
-      uint4* z = reinterpret_cast<uint4*>(keys + s0 * KE);
-      const uint64_t n16 = s1 > s0 ? (s1 - s0) * (KE / 16) : 0;
-      for (uint64_t q = threadIdx.x; q < n16; q += kThreads) __stcg(z + q, make_uint4(0, 0, 0, 0));
-    } else if (kind == 1) {
+    if (kind == 1) {
       const int warp = threadIdx.x >> 5;
       const uint64_t r = j * kHashRecs + 32 * warp;
       const int64_t n = r < G.nrec ? (int64_t)min((uint64_t)32, G.nrec - r) : 0;
@@ -666,7 +611,7 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
-      atomicAdd(kind == 0 ? done_z + g : kind == 1 ? done_h + g : done_x + g, 1u);
+      atomicAdd(kind == 1 ? done_h + g : done_x + g, 1u);
     }
   }
 }
@@ -726,7 +671,7 @@ extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_table, const uint64_t* d_table_offset,
+extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, const uint64_t* d_table_offset,
                                         int32_t pid_begin, int32_t pid_end, dbg_vertex* d_out, uint64_t out_cap,
                                         uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
                                         cudaStream_t stream) {
@@ -739,7 +684,7 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, const void* d_tab
   a.records = nullptr;
   a.rec_off = nullptr;
   a.tab_off = d_table_offset;
-  a.table = static_cast<char*>(const_cast<void*>(d_table));
+  a.table = static_cast<char*>(d_table);
   a.pid_begin = pid_begin;
   a.pid_end = pid_end;
   a.k = prm->k;

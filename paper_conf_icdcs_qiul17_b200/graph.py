@@ -111,6 +111,7 @@ class DbgBuilder:
         self.tab_host = np.zeros(NP + 1, dtype=np.int64)
         self.batches: list[tuple[int, int]] = []
         self._caps_key = None
+        self._dirty = False
         self.timer: dict | None = None  # name -> list of (start, end) CUDA events, when set
 
     # ------------------------------------------------------------------ timing helper
@@ -186,7 +187,7 @@ class DbgBuilder:
             self.batches = [(0, self.np)]
             self.total_slots = int(self.tab_host[-1])
             ring = _lib.dbg_subgraph_ring_bytes(self.prm, self.group_slots, int(self.caps.max(initial=1)))
-            self.ring = _grow(self.ring, ring, torch.uint8, self.device)
+            self.ring = self._clean_buffer(self.ring, ring, stream)
             wsb = _lib.dbg_subgraph_workspace_bytes(self.prm, self.np, self.total_slots, self.group_slots)
             self.work = _grow(self.work, wsb, torch.uint8, self.device)
             return self.batches
@@ -204,8 +205,19 @@ class DbgBuilder:
             b = e
         self.batches = batches
         need = max((self.tab_host[e] - self.tab_host[b] for b, e in batches), default=0) * self.slot_bytes
-        self.table = _grow(self.table, int(need), torch.uint8, self.device)
+        self.table = self._clean_buffer(self.table, int(need), stream)
         return batches
+
+    def _clean_buffer(self, t: torch.Tensor, nbytes: int, stream) -> torch.Tensor:
+        """Tables must be all-zero before hashing; extraction leaves them clean again
+        (clean-on-extract, hash.cu), so a buffer is zeroed only when (re)allocated or
+        after an interrupted build."""
+        grown = _grow(t, nbytes, torch.uint8, self.device)
+        if grown is not t or self._dirty:
+            with torch.cuda.stream(stream):
+                grown.zero_()
+            self._dirty = False
+        return grown
 
     # ------------------------------------------------------------------ a5-a7
     def reset_output(self, cap: int, stream=None) -> None:
@@ -219,8 +231,13 @@ class DbgBuilder:
         return self.out.numel() // VERTEX_DTYPE.itemsize
 
     def step2(self, stream=None) -> None:
-        """Zero-fill + hash + extract of every partition (output appended to self.out)."""
+        """Hash + extract of every partition (output appended to self.out)."""
         stream = stream or torch.cuda.current_stream(self.device)
+        self._dirty = True  # until every hashed table has been extracted
+        self._step2(stream)
+        self._dirty = False
+
+    def _step2(self, stream) -> None:
         if self.mode == "fused":
             ev = self._mark("step2", stream)
             _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.total_slots,
@@ -229,9 +246,6 @@ class DbgBuilder:
             self._done(ev, stream)
             return
         for (b, e) in self.batches:
-            n_slots = int(self.tab_host[e] - self.tab_host[b])
-            with torch.cuda.stream(stream):
-                self.table[: n_slots * self.key_bytes].zero_()  # EMPTY key entries (hash.cu)
             ev = self._mark("hash_build", stream)
             _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.table, self.d_tab_off, self.d_status,
                                 stream)
@@ -274,7 +288,7 @@ class DbgBuilder:
             if st == _lib.DBG_ENOSPACE and int(self.d_n_out.item()) > self.out_cap():
                 cap = int(self.d_n_out.item())
                 continue
-            if st == _lib.DBG_ETABLEFULL:  # reading O: rebuild at capacity N^i_kmer
+            if st == _lib.DBG_ETABLEFULL:  # reading O: rebuild at capacity N^i_kmer (tables are clean again)
                 if self.prm.lambda_ / (4 * self.prm.alpha) >= 1.0:
                     raise _lib.DbgError("dbg_hash_build", st, "table full at capacity >= N^i_kmer")
                 self.prm = _lib.params(self.k, self.p, self.np, 2.0, 0.5)
