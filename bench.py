@@ -298,7 +298,7 @@ def main():
     ap.add_argument("--lam", type=float, default=2.0)
     ap.add_argument("--alpha", type=float, default=0.5)
     ap.add_argument("--table-budget", type=int, default=None)
-    ap.add_argument("--mode", choices=["fused", "resident"], default="fused")
+    ap.add_argument("--mode", choices=["fused", "resident"], default="resident")
     ap.add_argument("--group-slots", type=int, default=1 << 19)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -9,15 +9,16 @@
 //   counters     n x 32 bytes  { u32 out[4]; u32 in[4] }
 // A key word is 0 (empty) or OCC | code (bit 63 of the hi word = occupied).
 //
-// One insertion, multiple updates: every probe is an
-// atomicCAS(slot, EMPTY, key) -- 64-bit for K <= 31, 128-bit for K <= 63 --
-// whose return value decides in one round trip: EMPTY means this occurrence
-// inserted the vertex (the single insertion), the own key means the vertex is
-// already there, anything else means probe on.  The whole key is published by
-// that one CAS, so the paper's {empty, locked, occupied} protocol for
-// multi-word keys (Fig. 4) collapses to {empty, occupied}: there
-// is no partially written key to wait for.  Then red.global.add on two
-// counters (the multiple updates).
+// One insertion, multiple updates: a probe loads the
+// key entry; an EMPTY slot is claimed with atomicCAS(slot, EMPTY, key) --
+// 64-bit for K <= 31, 128-bit for K <= 63 -- whose return value decides:
+// EMPTY means this occurrence inserted the vertex (the single insertion), the
+// own key means another thread just did, anything else means probe on.  The
+// whole key is published by that one CAS, so the paper's {empty, locked,
+// occupied} protocol for multi-word keys (Fig. 4) collapses to
+// {empty, occupied}: there is no partially written key to wait for.  Then
+// red.global.add on two counters (the multiple updates).  (Probing with the
+// CAS itself was measured slower: every probe then costs an L2 atomic.)
 //
 // Clean-on-extract: tables are all-zero before hashing (one memset when the
 // buffer is allocated), and extraction writes zeros back over every occupied
@@ -89,6 +90,9 @@ struct KeyOf<uint64_t> {
   static __device__ __forceinline__ T cas(char* kp, T want) {
     return atomicCAS(reinterpret_cast<unsigned long long*>(kp), 0ull, want);
   }
+  static __device__ __forceinline__ T load(const char* kp) {
+    return __ldcg(reinterpret_cast<const unsigned long long*>(kp));
+  }
 };
 template <>
 struct KeyOf<u128> {
@@ -103,6 +107,16 @@ struct KeyOf<u128> {
   static __device__ __forceinline__ bool same(T a, T b) { return a.x == b.x && a.y == b.y; }
   static __device__ __forceinline__ T cas(char* kp, T want) {
     return atomicCAS(reinterpret_cast<ulonglong2*>(kp), make_ulonglong2(0ull, 0ull), want);
+  }
+  // A 16-B load is not single-copy atomic: a torn read of a key being
+  // published shows one word of it and one zero word.  Such a value is
+  // neither EMPTY nor a key (every claimed hi word has OCC set and claimed
+  // entries never change), except the ambiguous (hi, 0) pair, which is
+  // treated as EMPTY so the CAS returns the entry atomically.
+  static __device__ __forceinline__ T load(const char* kp) {
+    T v = __ldcg(reinterpret_cast<const ulonglong2*>(kp));
+    if (v.x == 0 || v.y == 0) v = make_ulonglong2(0ull, 0ull);
+    return v;
   }
 };
 
@@ -245,17 +259,21 @@ __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, 
       live[q] = kid + q < k1;
       if (live[q]) {
         jb[q] = make_job<Code, R>(sm, kid + q, r, K);
-        cur[q] = KO::cas(keys + (jb[q].t0 + jb[q].idx) * KE, jb[q].want);  // probe = insert attempt
+        cur[q] = KO::load(keys + (jb[q].t0 + jb[q].idx) * KE);  // all first probes in flight
       }
     }
 #pragma unroll
     for (int q = 0; q < kJobs; ++q) {
       if (!live[q]) continue;
       uint64_t probes = 1;
-      while (!KO::empty(cur[q]) && !KO::same(cur[q], jb[q].want)) {  // occupied by another vertex
+      for (;;) {
+        // a plain load finds the vertex (the common case: duplicates outnumber
+        // distinct vertices ~4:1); only an EMPTY slot costs a CAS
+        if (KO::empty(cur[q])) cur[q] = KO::cas(keys + (jb[q].t0 + jb[q].idx) * KE, jb[q].want);
+        if (KO::empty(cur[q]) || KO::same(cur[q], jb[q].want)) break;
         if (probes++ == jb[q].cap) break;
         jb[q].idx = jb[q].idx + 1 == jb[q].cap ? 0 : jb[q].idx + 1;
-        cur[q] = KO::cas(keys + (jb[q].t0 + jb[q].idx) * KE, jb[q].want);
+        cur[q] = KO::load(keys + (jb[q].t0 + jb[q].idx) * KE);
       }
       if (!KO::empty(cur[q]) && !KO::same(cur[q], jb[q].want)) {
         ok = false;  // wrapped: table full (reading O)

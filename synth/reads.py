@@ -136,7 +136,7 @@ CONFIGS = {
                  gseed=1, rseed=101,
                  desc="tiny synthetic genome 50 kbp, 100 bp error-free reads at 10x, K=31, p=11, "
                       "16 MSP partitions"),
-    "ecoli": dict(genome=4_600_000, reads=2_760_000, read_len=100, error=0.01, k=31, p=11, np=64,
+    "ecoli": dict(genome=4_600_000, reads=2_760_000, read_len=100, error=0.01, k=31, p=11, np=2048,
                   gseed=2, rseed=102,
                   desc="E. coli-shaped synthetic: 4.6 Mbp genome, 100 bp reads at 60x with 1% "
                        "substitution errors, K=31"),
