@@ -177,15 +177,18 @@ def run_ours(args):
         return multi.bench_main(args, METRIC, UNIT)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    from paper_conf_icdcs_qiul17_b200 import DbgBuilder, encode_reads, _lib
+    from paper_conf_icdcs_qiul17_b200 import DbgBuilder, auto_refine, encode_reads, _lib
 
     rs, gen_s = _workload(args)
     packed = encode_reads(rs.seq, pin=True)
     offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
     n_kmers = rs.n_kmers()
     stream = torch.cuda.current_stream(dev)
+    refine = args.refine
+    if refine is None:
+        refine = auto_refine(n_kmers, rs.k, rs.p, rs.num_partitions, args.lam, args.alpha) if args.mode == "smem" else 1
     b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode,
-                   args.group_slots)
+                   args.group_slots, refine)
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
@@ -242,8 +245,9 @@ def run_ours(args):
     d2h = 32 + 16 * rs.num_partitions
 
     ms = statistics.mean(step_ms)
-    key = "step2" if args.mode == "fused" else "hash_build"
-    hash_ms = phases.get(key, float("nan"))
+    key = {"fused": "step2", "resident": "hash_build", "smem": "step2_smem"}[args.mode]
+    hash_ms = phases.get(key, float("nan")) + (phases.get("hash_build", 0.0) + phases.get("extract", 0.0)
+                                               if args.mode == "smem" else 0.0)
     n_records = int(b.part_records.sum())
     # one 32-B sector read + write-back per K-mer occurrence (the paper's
     # random-access table RMW) + the records read + the vertex records written
@@ -262,16 +266,20 @@ def run_ours(args):
         rate, sub, dt = _oracle_rate(rs, args.cpu_seconds, threads)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
-    launches_per_step = 3 + (2 if args.mode == "fused" else 2 * len(b.batches)) + 1
+    launches_per_step = 3 + {"fused": 2, "resident": 2 * len(b.batches),
+                             "smem": 1 + 2 * len(b.batches)}[args.mode] + 1
     line = {
         "metric": METRIC, "value": n_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": _config_json(rs, args, {"mode": args.mode, "batches": len(b.batches),
-                                          "group_slots": args.group_slots}),
+                                          "group_slots": args.group_slots, "refine": refine,
+                                          "fine_partitions": b.np,
+                                          "smem_slots": _lib.dbg_smem_table_slots(b.prm)}),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
-                     "kernel": "subgraph_kernel" if args.mode == "fused" else "hash_build_kernel",
+                     "kernel": {"fused": "subgraph_kernel", "resident": "hash_build_kernel",
+                                "smem": "smem_subgraph_kernel"}[args.mode],
                      "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
                      "kernel_ms": hash_ms, "kernel_kmers_per_s": n_kmers / (hash_ms * 1e-3)},
         "cpu_baseline": cpu,
@@ -298,7 +306,8 @@ def main():
     ap.add_argument("--lam", type=float, default=2.0)
     ap.add_argument("--alpha", type=float, default=0.5)
     ap.add_argument("--table-budget", type=int, default=None)
-    ap.add_argument("--mode", choices=["fused", "resident"], default="resident")
+    ap.add_argument("--mode", choices=["smem", "fused", "resident"], default="smem")
+    ap.add_argument("--refine", type=int, default=None, help="fine partitions per partition (default: auto)")
     ap.add_argument("--group-slots", type=int, default=1 << 19)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

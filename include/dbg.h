@@ -16,7 +16,9 @@
  *    reported by dbg_sync_status, the only call that synchronizes.
  *  - Thread-safe across distinct buffers; one host thread per device.
  *  - K must be odd (reading C), 1 <= K <= 63; 1 <= P <= min(K, 31);
- *    1 <= num_partitions <= 4,194,303.  Reads shorter than K contribute
+ *    1 <= num_partitions * refine <= 4,194,303.  Every per-partition array
+ *    and pid range below is in FINE partitions (NP * refine of them); only
+ *    dbg_vertex.pid reports the paper's partition (fine pid mod NP).  Reads shorter than K contribute
  *    nothing and are not an error (reading N).
  */
 #ifndef PARAHASH_DBG_H
@@ -29,7 +31,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 1
+#define DBG_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -52,6 +54,9 @@ typedef struct {
   int32_t num_partitions; /* NP, number of superkmer partitions (Sec. III-B) */
   float lambda;           /* average errors per read (Property 1); default 2 */
   float alpha;            /* load ratio; default 0.5 => capacity = N^i_kmer */
+  int32_t refine;         /* F >= 1: the device works on NP*F fine partitions, fine pid =
+                             fmix64(m) mod (NP*F), so a fine partition's table fits one SM;
+                             the paper's partition of a vertex is fine pid mod NP (0 = 1) */
 } dbg_params;
 
 /* One vertex of Definition 3: the canonical K-mer (the
@@ -138,7 +143,27 @@ DBG_API dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_ba
 DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers,
                           uint64_t* d_table_offset, cudaStream_t stream);
 
-/* ---- a5-a7 fused: Step 2 through an L2-resident ring (the hot path) ------
+/* ---- a5-a7 on-chip: Step 2 in shared memory (the hot path) ---------------
+ * Every fine partition whose table (capacity from Property 1) fits one CTA's
+ * shared memory -- at most dbg_smem_table_slots() slots -- is built and
+ * extracted by one CTA: shared-memory 64/128-bit CAS claims the key, shared-
+ * memory atomics count the edges (u16 fields: no count can exceed the
+ * partition's N^i_kmer < 65536), and the occupied slots are compacted
+ * straight into d_out.  Larger partitions are skipped here and left to the
+ * global-table path (dbg_table_plan_split + dbg_hash_build +
+ * dbg_extract_graph).  d_work: one caller-owned uint64 (scheduling cursor).
+ * Output appends to d_out[*d_n_out ...] and accumulates *d_stats. */
+DBG_API uint64_t dbg_smem_table_slots(const dbg_params* prm);
+DBG_API dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
+                                    uint64_t* d_work, dbg_vertex* d_out, uint64_t out_cap,
+                                    uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
+                                    cudaStream_t stream);
+/* As dbg_table_plan, but partitions whose capacity is <= smem_slots get
+ * capacity 0 (they are built on chip), so resident tables cover only the rest. */
+DBG_API dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t smem_slots,
+                                uint64_t* d_table_offset, cudaStream_t stream);
+
+/* ---- a5-a7 fused: Step 2 through an L2-resident ring -----------------------
  * For partitions [pid_begin, pid_end): build each partition's table (one
  * insertion per distinct vertex, multiple updates, Sec. III-C)
  * and compact it into d_out -- all in one persistent kernel.  d_ring must be

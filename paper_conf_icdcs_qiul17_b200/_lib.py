@@ -27,7 +27,7 @@ class DbgError(RuntimeError):
 
 class dbg_params(ctypes.Structure):
     _fields_ = [("k", ctypes.c_int32), ("p", ctypes.c_int32), ("num_partitions", ctypes.c_int32),
-                ("lambda_", ctypes.c_float), ("alpha", ctypes.c_float)]
+                ("lambda_", ctypes.c_float), ("alpha", ctypes.c_float), ("refine", ctypes.c_int32)]
 
 
 class dbg_partition_set(ctypes.Structure):
@@ -61,6 +61,9 @@ SIGNATURES = {
     "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
     "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P]),
+    "dbg_smem_table_slots": (_U64, [_PRM]),
+    "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _P, _P, _U64, _P, _P, _P, _P]),
+    "dbg_table_plan_split": (ctypes.c_int, [_PRM, _P, _U64, _P, _P]),
     "dbg_subgraph_ring_bytes": (_U64, [_PRM, _U64, _U64]),
     "dbg_subgraph_workspace_bytes": (_U64, [_PRM, _I32, _U64, _U64]),
     "dbg_build_subgraphs": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _U64, _P, _U64, _P, _U64, _P, _U64,
@@ -88,7 +91,7 @@ def load():
             f = getattr(lib, name)
             f.restype = res
             f.argtypes = args
-        if lib.dbg_abi_version() != 1:
+        if lib.dbg_abi_version() != 2:
             raise ImportError("libdbg.so ABI version mismatch")
         _lib = lib
     return _lib
@@ -119,8 +122,13 @@ def _stream(stream) -> int | None:
     return stream.cuda_stream
 
 
-def params(k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5) -> dbg_params:
-    return dbg_params(k, p, num_partitions, lam, alpha)
+def params(k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
+           refine: int = 1) -> dbg_params:
+    return dbg_params(k, p, num_partitions, lam, alpha, refine)
+
+
+def fine_partitions(prm: dbg_params) -> int:
+    return prm.num_partitions * max(1, prm.refine)
 
 
 def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
@@ -177,6 +185,22 @@ def dbg_msp_partition(prm, d_bases, n_words: int, d_offsets, n_reads: int, part:
 def dbg_table_plan(prm, d_n_kmers, d_table_offset, stream=None) -> None:
     _check("dbg_table_plan", load().dbg_table_plan(ctypes.byref(prm), _ptr(d_n_kmers),
                                                    _ptr(d_table_offset), _stream(stream)))
+
+
+def dbg_smem_table_slots(prm) -> int:
+    return load().dbg_smem_table_slots(ctypes.byref(prm))
+
+
+def dbg_build_subgraphs_smem(prm, part, d_work, d_out, out_cap: int, d_n_out, d_stats, d_status,
+                             stream=None) -> None:
+    _check("dbg_build_subgraphs_smem", load().dbg_build_subgraphs_smem(
+        ctypes.byref(prm), ctypes.byref(part), _ptr(d_work), _ptr(d_out), out_cap, _ptr(d_n_out), _ptr(d_stats),
+        _ptr(d_status), _stream(stream)))
+
+
+def dbg_table_plan_split(prm, d_n_kmers, smem_slots: int, d_table_offset, stream=None) -> None:
+    _check("dbg_table_plan_split", load().dbg_table_plan_split(ctypes.byref(prm), _ptr(d_n_kmers), smem_slots,
+                                                               _ptr(d_table_offset), _stream(stream)))
 
 
 def dbg_subgraph_ring_bytes(prm, group_slots: int, max_capacity: int) -> int:

@@ -24,6 +24,11 @@ __host__ __device__ inline uint32_t record_max_kmers(int k) {
   return 16u * (record_words(k) - 1u) - (uint32_t)k - 1u;
 }
 
+// Number of fine partitions the device works on (dbg.h: num_partitions * refine).
+__host__ __device__ inline int fine_partitions(const dbg_params* prm) {
+  return prm->num_partitions * (prm->refine > 1 ? prm->refine : 1);
+}
+
 // MurmurHash3 64-bit finaliser: the partition function of reading I
 // ("superkmer ID ... from the minimizer's hash bit value with a modulo",
 // P:L455-459), and the slot hash of the tables.

@@ -230,9 +230,9 @@ __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, 
       sm.w[lane][4 * v + 3] = x.w;
     }
     const uint32_t hdr = sm.w[lane][0];
-    n = hdr & 255u;
     uint64_t t0, cap;
     table_of(hdr >> 10, t0, cap);
+    n = cap ? hdr & 255u : 0u;  // capacity 0: the partition is built elsewhere (on chip)
     sm.t0[lane] = t0;
     sm.cap[lane] = cap;
   }
@@ -292,6 +292,7 @@ __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, 
 // --------------------------------------------------------------- extraction
 
 struct OutArgs {
+  uint32_t np_out;  // the paper's NP: dbg_vertex.pid = fine pid mod NP
   dbg_vertex* out;
   uint64_t out_cap;
   unsigned long long* n_out;
@@ -353,7 +354,7 @@ __device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t
     v.out[0] = a.x; v.out[1] = a.y; v.out[2] = a.z; v.out[3] = a.w;
     v.in[0] = b.x; v.in[1] = b.y; v.in[2] = b.z; v.in[3] = b.w;
     v.count = a.x + a.y + a.z + a.w + tout;  // count = sum(out) + t_out
-    v.pid = pid_of(s);
+    v.pid = pid_of(s) % oa.np_out;
     if (pos < oa.out_cap) oa.out[pos] = v;
     else atomicOr(oa.status, kStatusNoSpace);
     ++pos;
@@ -634,6 +635,217 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
   }
 }
 
+// --------------------------------------------------------------- on-chip Step 2
+//
+// One CTA builds one fine partition at a time entirely in shared memory
+// (dbg_build_subgraphs_smem): zero the partition's slots, hash its records
+// (16 warps, K-mers spread over lanes as in hash_warp), then compact the
+// occupied slots straight into the output.  Slot = key (8 B; 16 B for
+// K > 31) + 16-bit counter fields out[0..3], in[0..3], t_out packed two per
+// 32-bit word: a field never exceeds the partition's K-mer count, and the
+// on-chip path takes only partitions with capacity (>= N^i_kmer) below
+// 65536, so the 32-bit shared-memory atomicAdd of (1 << 16*half) never
+// carries across fields.
+
+constexpr int kSmemThreads = 512;
+constexpr int kSmemWarps = kSmemThreads / 32;
+constexpr int kSmemXPer = 4;
+constexpr uint32_t kSmemXTile = kSmemThreads * kSmemXPer;
+constexpr uint64_t kSmemMaxSlots = 65535;
+
+template <int KW>
+struct SmemSlot {
+  static constexpr uint32_t kBytes = KW == 1 ? 32 : 48;  // key + 6 or 8 field words
+  static constexpr uint32_t kFieldOff = KW == 1 ? 8 : 16;
+};
+
+struct SmemShared512 {
+  typename cub::BlockScan<uint32_t, kSmemThreads>::TempStorage scan;
+  typename cub::BlockReduce<unsigned long long, kSmemThreads>::TempStorage red;
+  unsigned long long base;
+  unsigned long long part;
+};
+
+template <int R>
+__host__ __device__ constexpr uint32_t smem_fixed_bytes() {
+  return (uint32_t)((sizeof(WarpRecs<R>) * kSmemWarps + sizeof(SmemShared512) + 127) & ~size_t(127));
+}
+
+struct SmemArgs {
+  const uint32_t* records;
+  const uint64_t* rec_off;
+  const uint64_t* n_kmers;
+  int n_fine, k;
+  double ratio;       // lambda / (4 alpha)
+  uint64_t slots;     // table slots that fit
+  unsigned long long* work;
+};
+
+__device__ __forceinline__ void smem_count(uint32_t* fields, int f) {
+  atomicAdd(fields + (f >> 1), 1u << (16 * (f & 1)));
+}
+
+// Insert/update of one occurrence in a shared-memory table.
+template <typename Code>
+__device__ __forceinline__ bool smem_upsert(char* table, uint64_t cap, const Job<Code>& jb) {
+  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
+  typedef KeyOf<Code> KO;
+  uint64_t idx = jb.idx;
+  for (uint64_t pr = 0; pr < cap; ++pr) {
+    char* kp = table + idx * SmemSlot<KW>::kBytes;
+    typename KO::T cur;
+    if constexpr (KW == 1) {
+      cur = *reinterpret_cast<volatile unsigned long long*>(kp);
+      if (cur == 0) cur = KO::cas(kp, jb.want);
+    } else {
+      cur = KO::cas(kp, jb.want);  // 16-B shared-memory CAS: atomic read-or-claim
+    }
+    if (KO::empty(cur) || KO::same(cur, jb.want)) {
+      uint32_t* fields = reinterpret_cast<uint32_t*>(kp + SmemSlot<KW>::kFieldOff);
+      smem_count(fields, jb.o < 4 ? jb.o : 8);
+      if (jb.i >= 0) smem_count(fields, 4 + jb.i);
+      return true;
+    }
+    idx = idx + 1 == cap ? 0 : idx + 1;
+  }
+  return false;
+}
+
+template <typename Code, int R>
+__device__ __forceinline__ bool hash_warp_smem(const uint32_t* recs, int64_t n_recs, int K, char* table,
+                                               uint64_t cap, WarpRecs<R>& sm) {
+  const int lane = threadIdx.x & 31;
+  uint32_t n = 0;
+  if (lane < n_recs) {
+    const uint4* src = reinterpret_cast<const uint4*>(recs + (uint64_t)lane * R);
+#pragma unroll
+    for (int v = 0; v < R / 4; ++v) {
+      const uint4 x = __ldcs(src + v);  // streamed once
+      sm.w[lane][4 * v] = x.x;
+      sm.w[lane][4 * v + 1] = x.y;
+      sm.w[lane][4 * v + 2] = x.z;
+      sm.w[lane][4 * v + 3] = x.w;
+    }
+    n = sm.w[lane][0] & 255u;
+    sm.t0[lane] = 0;
+    sm.cap[lane] = cap;
+  }
+  uint32_t incl = n;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t v = __shfl_up_sync(kFull, incl, d);
+    if (lane >= d) incl += v;
+  }
+  sm.pre[lane + 1] = incl;
+  if (lane == 0) sm.pre[0] = 0;
+  const uint32_t total = __shfl_sync(kFull, incl, 31);
+  __syncwarp();
+  const uint32_t share = (total + 31) / 32;
+  const uint32_t k0 = min(total, lane * share), k1 = min(total, k0 + share);
+  bool ok = true;
+  int r = 0;
+  for (uint32_t kid = k0; kid < k1; ++kid) ok &= smem_upsert(table, cap, make_job<Code, R>(sm, kid, r, K));
+  __syncwarp();
+  return ok;
+}
+
+template <typename Code, int R>
+__global__ void __launch_bounds__(kSmemThreads, 1) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
+  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
+  constexpr uint32_t SB = SmemSlot<KW>::kBytes;
+  extern __shared__ __align__(128) unsigned char smem[];
+  WarpRecs<R>* shw = reinterpret_cast<WarpRecs<R>*>(smem);
+  SmemShared512& sh = *reinterpret_cast<SmemShared512*>(smem + sizeof(WarpRecs<R>) * kSmemWarps);
+  char* table = reinterpret_cast<char*>(smem + smem_fixed_bytes<R>());
+  const int warp = threadIdx.x >> 5;
+  for (;;) {
+    if (threadIdx.x == 0) sh.part = atomicAdd(a.work, 1ull);
+    __syncthreads();
+    const uint64_t p = sh.part;
+    __syncthreads();
+    if (p >= (uint64_t)a.n_fine) break;
+    const uint64_t nk = a.n_kmers[p];
+    if (nk == 0) continue;
+    const double c = ceil(a.ratio * (double)nk);  // capacity, Sec. IV-A
+    const uint64_t cap = c < 1.0 ? 1ull : (uint64_t)c;
+    if (cap > a.slots) continue;  // left to the global-table path (dbg_table_plan_split)
+    uint4* z = reinterpret_cast<uint4*>(table);
+    for (uint32_t q = threadIdx.x; q < cap * (SB / 16); q += kSmemThreads) z[q] = make_uint4(0, 0, 0, 0);
+    __syncthreads();
+    const uint64_t r0 = a.rec_off[p], nrec = a.rec_off[p + 1] - r0;
+    bool ok = true;
+    for (uint64_t ch = warp; ch * 32 < nrec; ch += kSmemWarps) {
+      const int64_t n = (int64_t)min((uint64_t)32, nrec - ch * 32);
+      ok &= hash_warp_smem<Code, R>(a.records + (r0 + ch * 32) * R, n, a.k, table, cap, shw[warp]);
+    }
+    if (!ok) atomicOr(oa.status, kStatusTableFull);
+    __syncthreads();
+    // extraction: block-wide compaction of the occupied slots into the output
+    for (uint64_t t0 = 0; t0 < cap; t0 += kSmemXTile) {
+      uint32_t bits = 0;
+#pragma unroll
+      for (int q = 0; q < kSmemXPer; ++q) {
+        const uint64_t s = t0 + (uint64_t)q * kSmemThreads + threadIdx.x;
+        if (s < cap && (*reinterpret_cast<const unsigned long long*>(table + s * SB) & kOccupied)) bits |= 1u << q;
+      }
+      const uint32_t cnt = __popc(bits);
+      uint32_t excl, total;
+      cub::BlockScan<uint32_t, kSmemThreads>(sh.scan).ExclusiveSum(cnt, excl, total);
+      if (threadIdx.x == 0) sh.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
+      __syncthreads();
+      uint64_t pos = sh.base + excl;
+      unsigned long long st_count = 0, st_edges = 0, st_sum = 0;
+      while (bits) {
+        const int q = __ffs(bits) - 1;
+        bits &= bits - 1;
+        const uint64_t s = t0 + (uint64_t)q * kSmemThreads + threadIdx.x;
+        const char* sp = table + s * SB;
+        const uint64_t k0 = *reinterpret_cast<const unsigned long long*>(sp);
+        const uint32_t* f = reinterpret_cast<const uint32_t*>(sp + SmemSlot<KW>::kFieldOff);
+        dbg_vertex v;
+        if (KW == 1) {
+          v.kmer_hi = 0;
+          v.kmer_lo = k0 & kCodeMask;
+        } else {
+          v.kmer_hi = k0 & kCodeMask;
+          v.kmer_lo = *reinterpret_cast<const unsigned long long*>(sp + 8);
+        }
+        v.out[0] = f[0] & 0xffffu; v.out[1] = f[0] >> 16; v.out[2] = f[1] & 0xffffu; v.out[3] = f[1] >> 16;
+        v.in[0] = f[2] & 0xffffu; v.in[1] = f[2] >> 16; v.in[2] = f[3] & 0xffffu; v.in[3] = f[3] >> 16;
+        const uint32_t tout = f[4] & 0xffffu;
+        v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + tout;  // count = sum(out) + t_out
+        v.pid = (uint32_t)(p % oa.np_out);
+        if (pos < oa.out_cap) oa.out[pos] = v;
+        else atomicOr(oa.status, kStatusNoSpace);
+        ++pos;
+        const uint64_t fl[11] = {v.kmer_hi, v.kmer_lo, v.count, v.out[0], v.out[1], v.out[2], v.out[3],
+                                 v.in[0], v.in[1], v.in[2], v.in[3]};
+        uint64_t h = 0;
+#pragma unroll
+        for (int t = 0; t < 11; ++t) h = fmix64(h ^ fl[t]);
+        st_sum += h;
+        st_count += v.count;
+        st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
+      }
+      if (total) {  // block-uniform
+        typedef cub::BlockReduce<unsigned long long, kSmemThreads> Red;
+        const unsigned long long cc = Red(sh.red).Sum(st_count);
+        __syncthreads();
+        const unsigned long long e = Red(sh.red).Sum(st_edges);
+        __syncthreads();
+        const unsigned long long hh = Red(sh.red).Sum(st_sum);
+        if (threadIdx.x == 0) {
+          atomicAdd(oa.stats + 0, (unsigned long long)total);
+          atomicAdd(oa.stats + 1, cc);
+          atomicAdd(oa.stats + 2, e);
+          atomicAdd(oa.stats + 3, hh);
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
 // --------------------------------------------------------------- sort
 
 __global__ void sort_prepare_kernel(const dbg_vertex* __restrict__ in, uint64_t n,
@@ -671,7 +883,7 @@ extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table ||
       !d_table_offset || !d_status)
     return DBG_EINVAL;
-  if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
+  if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
   ResidentArgs a;
   a.records = part->d_records;
@@ -696,7 +908,7 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   if (!dbg_params_ok(prm) || !d_table || !d_table_offset || !d_n_out || !d_stats || !d_status ||
       (out_cap && !d_out))
     return DBG_EINVAL;
-  if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
+  if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
   ResidentArgs a;
   a.records = nullptr;
@@ -708,6 +920,7 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   a.k = prm->k;
   a.status = d_status;
   OutArgs oa;
+  oa.np_out = (uint32_t)prm->num_partitions;
   oa.out = d_out;
   oa.out_cap = out_cap;
   oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
@@ -717,6 +930,62 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   if (prm->k <= 31) extract_kernel<1><<<grid, kThreads, 0, stream>>>(a, oa);
   else extract_kernel<2><<<grid, kThreads, 0, stream>>>(a, oa);
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+}
+
+template <int R>
+static uint64_t smem_slots_for(int k) {
+  const uint64_t avail = 227u * 1024u - smem_fixed_bytes<R>();
+  const uint32_t sb = k <= 31 ? SmemSlot<1>::kBytes : SmemSlot<2>::kBytes;
+  const uint64_t n = (avail / sb) & ~(uint64_t)63;
+  return n < kSmemMaxSlots ? n : kSmemMaxSlots;
+}
+
+extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
+  if (!prm) return 0;
+  return record_words(prm->k) == 4 ? smem_slots_for<4>(prm->k) : smem_slots_for<8>(prm->k);
+}
+
+template <typename Code, int R>
+static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
+  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
+  const size_t bytes = smem_fixed_bytes<R>() + a.slots * SmemSlot<KW>::kBytes;
+  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)bytes);
+  if (e != cudaSuccess) return e;
+  smem_subgraph_kernel<Code, R><<<dbg_sm_count(), kSmemThreads, bytes, stream>>>(a, oa);
+  return cudaGetLastError();
+}
+
+extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
+                                               uint64_t* d_work, dbg_vertex* d_out, uint64_t out_cap,
+                                               uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
+                                               cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !part->d_n_kmers || !d_work ||
+      !d_n_out || !d_stats || !d_status || (out_cap && !d_out))
+    return DBG_EINVAL;
+  if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
+  SmemArgs a;
+  a.records = part->d_records;
+  a.rec_off = part->d_record_offset;
+  a.n_kmers = part->d_n_kmers;
+  a.n_fine = fine_partitions(prm);
+  a.k = prm->k;
+  a.ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
+  a.slots = dbg_smem_table_slots(prm);
+  a.work = reinterpret_cast<unsigned long long*>(d_work);
+  OutArgs oa;
+  oa.np_out = (uint32_t)prm->num_partitions;
+  oa.out = d_out;
+  oa.out_cap = out_cap;
+  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
+  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
+  oa.status = d_status;
+  if (cudaMemsetAsync(d_work, 0, sizeof(uint64_t), stream) != cudaSuccess) return DBG_ECUDA;
+  cudaError_t e;
+  if (prm->k <= 31) e = launch_smem<uint64_t, 4>(a, oa, stream);
+  else if (prm->k <= 39) e = launch_smem<u128, 4>(a, oa, stream);
+  else e = launch_smem<u128, 8>(a, oa, stream);
+  return e == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
 static uint64_t n_groups_max(uint64_t total_slots, uint64_t group_slots) {
@@ -746,7 +1015,7 @@ extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_parti
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table_offset ||
       !d_ring || !d_workspace || !d_n_out || !d_stats || !d_status || (out_cap && !d_out) || group_slots == 0)
     return DBG_EINVAL;
-  if (pid_begin < 0 || pid_end > prm->num_partitions || pid_begin > pid_end) return DBG_EINVAL;
+  if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
   if (workspace_bytes < dbg_subgraph_workspace_bytes(prm, pid_end - pid_begin, total_slots, group_slots))
     return DBG_EINVAL;
@@ -771,6 +1040,7 @@ extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_parti
   a.done = reinterpret_cast<uint32_t*>(ws + 8 * (g + kLagX + 3) + 16);
   a.gfirst = a.done + 3 * g;
   OutArgs oa;
+  oa.np_out = (uint32_t)prm->num_partitions;
   oa.out = d_out;
   oa.out_cap = out_cap;
   oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);

@@ -271,7 +271,7 @@ constexpr int kScanThreads = 256;
 template <bool kCapacity>
 __global__ void __launch_bounds__(kScanThreads) scan_kernel(const uint64_t* __restrict__ in,
                                                             uint64_t* __restrict__ out, int n,
-                                                            double ratio) {
+                                                            double ratio, uint64_t skip_upto) {
   using Scan = cub::BlockScan<unsigned long long, kScanThreads>;
   __shared__ typename Scan::TempStorage tmp;
   __shared__ unsigned long long carry;
@@ -286,6 +286,7 @@ __global__ void __launch_bounds__(kScanThreads) scan_kernel(const uint64_t* __re
         // capacity_i = ceil(lambda / (4 alpha) * N^i_kmer), at least 1
         double c = ceil(ratio * (double)v);
         v = c < 1.0 ? 1ull : (unsigned long long)c;
+        if (v <= skip_upto) v = 0;  // built on chip (dbg_table_plan_split)
       }
     }
     unsigned long long excl, total;
@@ -366,7 +367,8 @@ int dbg_sm_count() {
 
 bool dbg_params_ok(const dbg_params* prm) {
   return prm && prm->k >= 1 && prm->k <= 63 && (prm->k & 1) && prm->p >= 1 && prm->p <= prm->k &&
-         prm->p <= 31 && prm->num_partitions >= 1 && (uint32_t)prm->num_partitions <= kMaxPid;
+         prm->p <= 31 && prm->num_partitions >= 1 && prm->refine >= 0 &&
+         (uint64_t)prm->num_partitions * (uint64_t)(prm->refine > 1 ? prm->refine : 1) <= kMaxPid;
 }
 
 template <typename CT>
@@ -387,7 +389,7 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
       !part->d_n_kmers || !part->d_staged)
     return DBG_EINVAL;
   if (n_reads && (!d_bases || !n_words)) return DBG_EINVAL;
-  const int np = prm->num_partitions;
+  const int np = fine_partitions(prm);
   const uint32_t R = record_words(prm->k);
   if (part->d_records == nullptr) {
     // passes 1 + 2: minimizers, superkmers, staging, sizes, offsets
@@ -421,7 +423,7 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
                                          : launch_msp<uint64_t>(a, grid, stream);
       if (e != cudaSuccess) return DBG_ECUDA;
     }
-    scan_kernel<false><<<1, kScanThreads, 0, stream>>>(part->d_n_records, part->d_record_offset, np, 0.0);
+    scan_kernel<false><<<1, kScanThreads, 0, stream>>>(part->d_n_records, part->d_record_offset, np, 0.0, 0);
   } else {
     // pass 3: scatter (requires staged <= staging_cap; the caller checks sum(n_records))
     if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
@@ -448,6 +450,16 @@ extern "C" dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_
   if (!dbg_params_ok(prm) || !d_n_kmers || !d_table_offset) return DBG_EINVAL;
   if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
   const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
-  scan_kernel<true><<<1, kScanThreads, 0, stream>>>(d_n_kmers, d_table_offset, prm->num_partitions, ratio);
+  scan_kernel<true><<<1, kScanThreads, 0, stream>>>(d_n_kmers, d_table_offset, fine_partitions(prm), ratio, 0);
+  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+}
+
+extern "C" dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t smem_slots,
+                                           uint64_t* d_table_offset, cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !d_n_kmers || !d_table_offset) return DBG_EINVAL;
+  if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
+  const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
+  scan_kernel<true><<<1, kScanThreads, 0, stream>>>(d_n_kmers, d_table_offset, fine_partitions(prm), ratio,
+                                                    smem_slots);
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }

@@ -70,17 +70,20 @@ class DbgBuilder:
 
     def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
                  device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
-                 mode: str = "fused", group_slots: int = 1 << 19):
+                 mode: str = "smem", group_slots: int = 1 << 19, refine: int = 1):
         if k % 2 == 0 or not 1 <= k <= 63:
             raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
         if not 1 <= p <= min(k, 31):
             raise ValueError("P must be in 1..min(K, 31)")
-        if mode not in ("fused", "resident"):
+        if mode not in ("smem", "fused", "resident"):
             raise ValueError(mode)
-        self.k, self.p, self.np, self.mode = k, p, num_partitions, mode
+        self.k, self.p, self.mode = k, p, mode
+        self.np_out = num_partitions                 # the paper's NP (dbg_vertex.pid)
+        self.refine = max(1, int(refine))
+        self.np = num_partitions * self.refine       # fine partitions the device works on
         self.group_slots = int(group_slots)  # fused mode: table slots per ring group (L2 sizing)
         self.total_slots = 0
-        self.prm = _lib.params(k, p, num_partitions, lam, alpha)
+        self.prm = _lib.params(k, p, num_partitions, lam, alpha, self.refine)
         self.device = torch.device(device)
         _lib.load()
         self.rec_words = _lib.dbg_record_words(self.prm)
@@ -96,6 +99,7 @@ class DbgBuilder:
         self.d_staged = torch.zeros(1, **i64)
         self.d_tab_off = torch.zeros(NP + 1, **i64)
         self.d_status = torch.zeros(1, dtype=torch.int32, device=dev)
+        self.d_work = torch.zeros(1, **i64)
         self.d_n_out = torch.zeros(1, **i64)
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
@@ -176,11 +180,16 @@ class DbgBuilder:
     def plan(self, stream=None) -> list[tuple[int, int]]:
         stream = stream or torch.cuda.current_stream(self.device)
         _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, stream)
-        key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha)
+        key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha, self.mode)
         if self._caps_key != key:  # host copy of the same C sizing function (dbg_table_capacity)
             self.caps = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in self.part_kmers],
                                  dtype=np.int64)
+            if self.mode == "smem":  # on-chip partitions need no global table (dbg_table_plan_split)
+                self.caps[self.caps <= _lib.dbg_smem_table_slots(self.prm)] = 0
             self._caps_key = key
+        if self.mode == "smem":
+            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, _lib.dbg_smem_table_slots(self.prm),
+                                      self.d_tab_off, stream)
         self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
         self.tab_host[1:] = np.cumsum(self.caps)
         if self.mode == "fused":
@@ -190,6 +199,9 @@ class DbgBuilder:
             self.ring = self._clean_buffer(self.ring, ring, stream)
             wsb = _lib.dbg_subgraph_workspace_bytes(self.prm, self.np, self.total_slots, self.group_slots)
             self.work = _grow(self.work, wsb, torch.uint8, self.device)
+            return self.batches
+        if self.mode == "smem" and not self.caps.any():
+            self.batches = []
             return self.batches
         budget = self.table_budget_bytes
         if budget is None:
@@ -201,7 +213,8 @@ class DbgBuilder:
             e = b + 1
             while e < self.np and self.tab_host[e + 1] - self.tab_host[b] <= max_slots:
                 e += 1
-            batches.append((b, e))
+            if self.tab_host[e] > self.tab_host[b]:
+                batches.append((b, e))
             b = e
         self.batches = batches
         need = max((self.tab_host[e] - self.tab_host[b] for b, e in batches), default=0) * self.slot_bytes
@@ -238,6 +251,11 @@ class DbgBuilder:
         self._dirty = False
 
     def _step2(self, stream) -> None:
+        if self.mode == "smem":
+            ev = self._mark("step2_smem", stream)
+            _lib.dbg_build_subgraphs_smem(self.prm, self.part_set(True), self.d_work, self.out, self.out_cap(),
+                                          self.d_n_out, self.d_stats, self.d_status, stream)
+            self._done(ev, stream)
         if self.mode == "fused":
             ev = self._mark("step2", stream)
             _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.total_slots,
@@ -291,7 +309,7 @@ class DbgBuilder:
             if st == _lib.DBG_ETABLEFULL:  # reading O: rebuild at capacity N^i_kmer (tables are clean again)
                 if self.prm.lambda_ / (4 * self.prm.alpha) >= 1.0:
                     raise _lib.DbgError("dbg_hash_build", st, "table full at capacity >= N^i_kmer")
-                self.prm = _lib.params(self.k, self.p, self.np, 2.0, 0.5)
+                self.prm = _lib.params(self.k, self.p, self.np_out, 2.0, 0.5, self.refine)
                 self.plan(stream)
                 continue
             if st != _lib.DBG_OK:
@@ -302,12 +320,30 @@ class DbgBuilder:
                            self.part_records.copy(), list(self.batches))
 
 
+def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
+                fill: float = 0.4) -> int:
+    """Refinement F so that an average fine partition's table (Property-1 capacity) fills
+    about `fill` of one SM's shared-memory table (dbg_smem_table_slots)."""
+    prm = _lib.params(k, p, num_partitions, lam, alpha)
+    slots = _lib.dbg_smem_table_slots(prm)
+    per_part = max(1.0, fill * slots / max(lam / (4 * alpha), 1e-9))
+    f = max(1, int(np.ceil(n_kmers / (num_partitions * per_part))))
+    f = 1 << int(np.ceil(np.log2(f)))
+    while num_partitions * f > 4_194_303 and f > 1:
+        f //= 2
+    return f
+
+
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
                 lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
-                table_budget_bytes: int | None = None, mode: str = "fused",
-                group_slots: int = 1 << 19) -> GraphResult:
+                table_budget_bytes: int | None = None, mode: str = "smem",
+                group_slots: int = 1 << 19, refine: int | str = "auto") -> GraphResult:
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
-    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots)
+    if refine == "auto":
+        lens = np.diff(np.asarray(offsets, dtype=np.int64))
+        refine = auto_refine(int(np.maximum(lens - k + 1, 0).sum()), k, p, num_partitions, lam, alpha) \
+            if mode == "smem" else 1
+    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots, refine)
     packed = encode_reads(seq)
     d_bases, d_offsets = builder.upload(packed, offsets)
     return builder.build(d_bases, d_offsets, sort=sort)

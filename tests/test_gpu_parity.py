@@ -116,7 +116,7 @@ def test_msp_records_vs_oracle_superkmers():
         assert occurrences_from_records(recs, k) == occurrences_from_oracle_msp(sk, rs.reads(), k)
 
 
-@pytest.mark.parametrize("mode", ["fused", "resident"])
+@pytest.mark.parametrize("mode", ["smem", "fused", "resident"])
 def test_table_overflow_detected_and_rebuilt(mode):
     """Reading O: an undersized table (lambda/(4 alpha) << distinct/N) overflows; the status word
     reports DBG_ETABLEFULL and the builder rebuilds at capacity N^i_kmer with the same result."""
@@ -151,8 +151,31 @@ def test_resident_mode_parity(k, p, np_):
 def test_ring_with_many_small_partitions():
     """More partitions than ring regions, many empty: the fused kernel's region reuse chain."""
     rs = random_reads(500, 40, 160, seed=77)
-    _check(rs, 31, 11, 1000)
-    _check(rs, 15, 7, 37)
+    _check(rs, 31, 11, 1000, mode="fused")
+    _check(rs, 15, 7, 37, mode="fused")
+
+
+@pytest.mark.parametrize("k,p,np_,refine", [(31, 11, 1, 1), (31, 11, 3, 1), (63, 19, 2, 1), (31, 11, 4, 8),
+                                             (41, 13, 3, 16), (21, 7, 5, 64)])
+def test_smem_with_global_tier(k, p, np_, refine):
+    """On-chip tables for partitions that fit one SM, the global-table path for the rest (here NP is
+    small, so some partitions exceed dbg_smem_table_slots), and refined partitions whose pid is
+    reported modulo NP -- all equal to the oracle."""
+    g = genome(60_000, seed=k + np_)
+    seq, offs = make_reads(g, 4000, 100, 0.01, seed=refine + 3)
+    rs = ReadSet(seq, offs)
+    res, _ = _check(rs, k, p, np_, refine=refine)
+    if refine == 1 and np_ <= 3:
+        assert res.batches, "expected some partitions on the global-table path"
+
+
+def test_auto_refine_small_partitions():
+    from paper_conf_icdcs_qiul17_b200 import auto_refine
+    rs = make_config("tiny")
+    f = auto_refine(rs.n_kmers(), 31, 11, 16)
+    assert f >= 2 and (f & (f - 1)) == 0
+    res, _ = _check(rs, 31, 11, 16, refine=f)
+    assert not res.batches  # every fine partition built on chip
 
 
 def test_repeat_runs_deterministic():
