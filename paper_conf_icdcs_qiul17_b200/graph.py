@@ -90,7 +90,7 @@ class DbgBuilder:
         self.slot_bytes = _lib.dbg_slot_bytes(self.prm)
         self.key_bytes = _lib.dbg_key_bytes(self.prm)
         dev = self.device
-        NP = num_partitions
+        NP = self.np
         i64 = dict(dtype=torch.int64, device=dev)
         self.d_n_records = torch.zeros(NP, **i64)
         self.d_n_kmers = torch.zeros(NP, **i64)
