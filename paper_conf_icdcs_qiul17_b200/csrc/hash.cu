@@ -638,14 +638,16 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
 // --------------------------------------------------------------- on-chip Step 2
 //
 // One CTA builds one fine partition at a time entirely in shared memory
-// (dbg_build_subgraphs_smem): zero the partition's slots, hash its records
-// (16 warps, K-mers spread over lanes as in hash_warp), then compact the
-// occupied slots straight into the output.  Slot = key (8 B; 16 B for
-// K > 31) + 16-bit counter fields out[0..3], in[0..3], t_out packed two per
-// 32-bit word: a field never exceeds the partition's K-mer count, and the
-// on-chip path takes only partitions with capacity (>= N^i_kmer) below
-// 65536, so the 32-bit shared-memory atomicAdd of (1 << 16*half) never
-// carries across fields.
+// (dbg_build_subgraphs_smem): its warps hash the partition's records (K-mers
+// spread over lanes as in hash_warp), then the CTA compacts the occupied
+// slots straight into the output and zeroes them again (clean-on-extract, so
+// no zero pass between partitions).  Slot = key (8 B; 16 B for K > 31) +
+// 16-bit counter fields out[0..3], in[0..3], t_out packed two per 32-bit
+// word: a field never exceeds the partition's K-mer count, and the on-chip
+// path takes only partitions with capacity (>= N^i_kmer) below 65536, so the
+// 32-bit shared-memory atomicAdd of (1 << 16*half) never carries across
+// fields.  Per partition: one block scan, one global atomicAdd (output
+// reservation) and two barriers; totals are reduced once per CTA.
 
 constexpr int kSmemThreads = 512;
 constexpr int kSmemWarps = kSmemThreads / 32;
@@ -663,7 +665,6 @@ struct SmemShared512 {
   typename cub::BlockScan<uint32_t, kSmemThreads>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, kSmemThreads>::TempStorage red;
   unsigned long long base;
-  unsigned long long part;
 };
 
 template <int R>
@@ -678,7 +679,6 @@ struct SmemArgs {
   int n_fine, k;
   double ratio;       // lambda / (4 alpha)
   uint64_t slots;     // table slots that fit
-  unsigned long long* work;
 };
 
 __device__ __forceinline__ void smem_count(uint32_t* fields, int f) {
@@ -758,91 +758,88 @@ __global__ void __launch_bounds__(kSmemThreads, 1) smem_subgraph_kernel(SmemArgs
   SmemShared512& sh = *reinterpret_cast<SmemShared512*>(smem + sizeof(WarpRecs<R>) * kSmemWarps);
   char* table = reinterpret_cast<char*>(smem + smem_fixed_bytes<R>());
   const int warp = threadIdx.x >> 5;
-  for (;;) {
-    if (threadIdx.x == 0) sh.part = atomicAdd(a.work, 1ull);
-    __syncthreads();
-    const uint64_t p = sh.part;
-    __syncthreads();
-    if (p >= (uint64_t)a.n_fine) break;
+  {  // the table starts clean; extraction keeps it clean
+    uint4* z = reinterpret_cast<uint4*>(table);
+    for (uint64_t q = threadIdx.x; q < a.slots * (SB / 16); q += kSmemThreads) z[q] = make_uint4(0, 0, 0, 0);
+  }
+  unsigned long long st_n = 0, st_count = 0, st_edges = 0, st_sum = 0;
+  bool ok = true;
+  for (uint64_t p = blockIdx.x; p < (uint64_t)a.n_fine; p += gridDim.x) {
     const uint64_t nk = a.n_kmers[p];
     if (nk == 0) continue;
     const double c = ceil(a.ratio * (double)nk);  // capacity, Sec. IV-A
     const uint64_t cap = c < 1.0 ? 1ull : (uint64_t)c;
     if (cap > a.slots) continue;  // left to the global-table path (dbg_table_plan_split)
-    uint4* z = reinterpret_cast<uint4*>(table);
-    for (uint32_t q = threadIdx.x; q < cap * (SB / 16); q += kSmemThreads) z[q] = make_uint4(0, 0, 0, 0);
-    __syncthreads();
     const uint64_t r0 = a.rec_off[p], nrec = a.rec_off[p + 1] - r0;
-    bool ok = true;
-    for (uint64_t ch = warp; ch * 32 < nrec; ch += kSmemWarps) {
-      const int64_t n = (int64_t)min((uint64_t)32, nrec - ch * 32);
-      ok &= hash_warp_smem<Code, R>(a.records + (r0 + ch * 32) * R, n, a.k, table, cap, shw[warp]);
+    // spread the records over all warps (chunks of <= 32 records)
+    const uint64_t cs = min((uint64_t)32, (nrec + kSmemWarps - 1) / kSmemWarps);
+    __syncthreads();  // previous partition's extraction (and the initial zero fill) complete
+    for (uint64_t ch = warp; ch * cs < nrec; ch += kSmemWarps) {
+      const int64_t n = (int64_t)min(cs, nrec - ch * cs);
+      ok &= hash_warp_smem<Code, R>(a.records + (r0 + ch * cs) * R, n, a.k, table, cap, shw[warp]);
     }
-    if (!ok) atomicOr(oa.status, kStatusTableFull);
     __syncthreads();
-    // extraction: block-wide compaction of the occupied slots into the output
-    for (uint64_t t0 = 0; t0 < cap; t0 += kSmemXTile) {
-      uint32_t bits = 0;
+    // extraction: each thread owns slots s = q * kSmemThreads + tid; one block
+    // scan sizes the partition's output, one global atomic reserves it
+    uint32_t cnt = 0;
+    for (uint64_t s = threadIdx.x; s < cap; s += kSmemThreads)
+      cnt += (*reinterpret_cast<const unsigned long long*>(table + s * SB) & kOccupied) ? 1u : 0u;
+    uint32_t excl, total;
+    cub::BlockScan<uint32_t, kSmemThreads>(sh.scan).ExclusiveSum(cnt, excl, total);
+    if (threadIdx.x == 0) sh.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
+    __syncthreads();
+    uint64_t pos = sh.base + excl;
+    const uint32_t pid = (uint32_t)(p % oa.np_out);
+    for (uint64_t s = threadIdx.x; s < cap; s += kSmemThreads) {
+      char* sp = table + s * SB;
+      const uint64_t k0 = *reinterpret_cast<const unsigned long long*>(sp);
+      if (!(k0 & kOccupied)) continue;
+      uint32_t* f = reinterpret_cast<uint32_t*>(sp + SmemSlot<KW>::kFieldOff);
+      dbg_vertex v;
+      if (KW == 1) {
+        v.kmer_hi = 0;
+        v.kmer_lo = k0 & kCodeMask;
+      } else {
+        v.kmer_hi = k0 & kCodeMask;
+        v.kmer_lo = *reinterpret_cast<const unsigned long long*>(sp + 8);
+      }
+      const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
+      v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
+      v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
+      v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
+      v.pid = pid;
+      uint4* z = reinterpret_cast<uint4*>(sp);  // clean-on-extract
 #pragma unroll
-      for (int q = 0; q < kSmemXPer; ++q) {
-        const uint64_t s = t0 + (uint64_t)q * kSmemThreads + threadIdx.x;
-        if (s < cap && (*reinterpret_cast<const unsigned long long*>(table + s * SB) & kOccupied)) bits |= 1u << q;
-      }
-      const uint32_t cnt = __popc(bits);
-      uint32_t excl, total;
-      cub::BlockScan<uint32_t, kSmemThreads>(sh.scan).ExclusiveSum(cnt, excl, total);
-      if (threadIdx.x == 0) sh.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
-      __syncthreads();
-      uint64_t pos = sh.base + excl;
-      unsigned long long st_count = 0, st_edges = 0, st_sum = 0;
-      while (bits) {
-        const int q = __ffs(bits) - 1;
-        bits &= bits - 1;
-        const uint64_t s = t0 + (uint64_t)q * kSmemThreads + threadIdx.x;
-        const char* sp = table + s * SB;
-        const uint64_t k0 = *reinterpret_cast<const unsigned long long*>(sp);
-        const uint32_t* f = reinterpret_cast<const uint32_t*>(sp + SmemSlot<KW>::kFieldOff);
-        dbg_vertex v;
-        if (KW == 1) {
-          v.kmer_hi = 0;
-          v.kmer_lo = k0 & kCodeMask;
-        } else {
-          v.kmer_hi = k0 & kCodeMask;
-          v.kmer_lo = *reinterpret_cast<const unsigned long long*>(sp + 8);
-        }
-        v.out[0] = f[0] & 0xffffu; v.out[1] = f[0] >> 16; v.out[2] = f[1] & 0xffffu; v.out[3] = f[1] >> 16;
-        v.in[0] = f[2] & 0xffffu; v.in[1] = f[2] >> 16; v.in[2] = f[3] & 0xffffu; v.in[3] = f[3] >> 16;
-        const uint32_t tout = f[4] & 0xffffu;
-        v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + tout;  // count = sum(out) + t_out
-        v.pid = (uint32_t)(p % oa.np_out);
-        if (pos < oa.out_cap) oa.out[pos] = v;
-        else atomicOr(oa.status, kStatusNoSpace);
-        ++pos;
-        const uint64_t fl[11] = {v.kmer_hi, v.kmer_lo, v.count, v.out[0], v.out[1], v.out[2], v.out[3],
-                                 v.in[0], v.in[1], v.in[2], v.in[3]};
-        uint64_t h = 0;
+      for (uint32_t q = 0; q < SB / 16; ++q) z[q] = make_uint4(0, 0, 0, 0);
+      if (pos < oa.out_cap) oa.out[pos] = v;
+      else atomicOr(oa.status, kStatusNoSpace);
+      ++pos;
+      const uint64_t fl[11] = {v.kmer_hi, v.kmer_lo, v.count, v.out[0], v.out[1], v.out[2], v.out[3],
+                               v.in[0], v.in[1], v.in[2], v.in[3]};
+      uint64_t h = 0;
 #pragma unroll
-        for (int t = 0; t < 11; ++t) h = fmix64(h ^ fl[t]);
-        st_sum += h;
-        st_count += v.count;
-        st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
-      }
-      if (total) {  // block-uniform
-        typedef cub::BlockReduce<unsigned long long, kSmemThreads> Red;
-        const unsigned long long cc = Red(sh.red).Sum(st_count);
-        __syncthreads();
-        const unsigned long long e = Red(sh.red).Sum(st_edges);
-        __syncthreads();
-        const unsigned long long hh = Red(sh.red).Sum(st_sum);
-        if (threadIdx.x == 0) {
-          atomicAdd(oa.stats + 0, (unsigned long long)total);
-          atomicAdd(oa.stats + 1, cc);
-          atomicAdd(oa.stats + 2, e);
-          atomicAdd(oa.stats + 3, hh);
-        }
-      }
-      __syncthreads();
+      for (int t = 0; t < 11; ++t) h = fmix64(h ^ fl[t]);
+      st_n += 1;
+      st_sum += h;
+      st_count += v.count;
+      st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
     }
+  }
+  if (!ok) atomicOr(oa.status, kStatusTableFull);
+  __syncthreads();
+  typedef cub::BlockReduce<unsigned long long, kSmemThreads> Red;
+  const unsigned long long n = Red(sh.red).Sum(st_n);
+  __syncthreads();
+  const unsigned long long cc = Red(sh.red).Sum(st_count);
+  __syncthreads();
+  const unsigned long long e = Red(sh.red).Sum(st_edges);
+  __syncthreads();
+  const unsigned long long hh = Red(sh.red).Sum(st_sum);
+  if (threadIdx.x == 0 && n) {
+    atomicAdd(oa.stats + 0, n);
+    atomicAdd(oa.stats + 1, cc);
+    atomicAdd(oa.stats + 2, e);
+    atomicAdd(oa.stats + 3, hh);
   }
 }
 
@@ -972,7 +969,7 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   a.k = prm->k;
   a.ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   a.slots = dbg_smem_table_slots(prm);
-  a.work = reinterpret_cast<unsigned long long*>(d_work);
+  (void)d_work;  // reserved (static partition schedule)
   OutArgs oa;
   oa.np_out = (uint32_t)prm->num_partitions;
   oa.out = d_out;
@@ -980,7 +977,6 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
   oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
   oa.status = d_status;
-  if (cudaMemsetAsync(d_work, 0, sizeof(uint64_t), stream) != cudaSuccess) return DBG_ECUDA;
   cudaError_t e;
   if (prm->k <= 31) e = launch_smem<uint64_t, 4>(a, oa, stream);
   else if (prm->k <= 39) e = launch_smem<u128, 4>(a, oa, stream);

@@ -115,6 +115,8 @@ class DbgBuilder:
         self.tab_host = np.zeros(NP + 1, dtype=np.int64)
         self.batches: list[tuple[int, int]] = []
         self._caps_key = None
+        self._batch_key = None
+        self._batches_cache: list[tuple[int, int]] = []
         self._dirty = False
         self.timer: dict | None = None  # name -> list of (start, end) CUDA events, when set
 
@@ -182,8 +184,11 @@ class DbgBuilder:
         _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, stream)
         key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha, self.mode)
         if self._caps_key != key:  # host copy of the same C sizing function (dbg_table_capacity)
-            self.caps = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in self.part_kmers],
-                                 dtype=np.int64)
+            nz = np.nonzero(self.part_kmers)[0]
+            self.caps = np.zeros(self.np, dtype=np.int64)
+            uniq, inv = np.unique(self.part_kmers[nz], return_inverse=True)
+            self.caps[nz] = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in uniq],
+                                     dtype=np.int64)[inv]
             if self.mode == "smem":  # on-chip partitions need no global table (dbg_table_plan_split)
                 self.caps[self.caps <= _lib.dbg_smem_table_slots(self.prm)] = 0
             self._caps_key = key
@@ -208,14 +213,18 @@ class DbgBuilder:
             free, _ = torch.cuda.mem_get_info(self.device)
             budget = max(int(free * 0.6), 1 << 26)
         max_slots = max(budget // self.slot_bytes, int(self.caps.max(initial=0)))
-        batches, b = [], 0
-        while b < self.np:
-            e = b + 1
-            while e < self.np and self.tab_host[e + 1] - self.tab_host[b] <= max_slots:
-                e += 1
-            if self.tab_host[e] > self.tab_host[b]:
-                batches.append((b, e))
-            b = e
+        bkey = (self._caps_key, max_slots)
+        if self._batch_key != bkey:  # greedy batches of consecutive partitions (vectorised)
+            batches, b, th = [], 0, self.tab_host
+            while b < self.np:
+                e = int(np.searchsorted(th, th[b] + max_slots, side="right")) - 1
+                e = min(max(e, b + 1), self.np)
+                if th[e] > th[b]:
+                    batches.append((b, e))
+                b = e
+            self._batches_cache = batches
+            self._batch_key = bkey
+        batches = self._batches_cache
         self.batches = batches
         need = max((self.tab_host[e] - self.tab_host[b] for b, e in batches), default=0) * self.slot_bytes
         self.table = self._clean_buffer(self.table, int(need), stream)
