@@ -74,8 +74,9 @@ typedef struct {
   uint32_t pid;
 } dbg_vertex;
 
-/* Totals; checksum = sum over vertices of h, h = fmix64 chained over
- * (kmer_hi, kmer_lo, count, out[0..3], in[0..3]). */
+/* Totals (filled by the extraction calls); checksum = sum over vertices of
+ * h, h = fmix64 chained over (kmer_hi, kmer_lo, count, out[0..3], in[0..3])
+ * (SURVEY.md 8(d)), filled by dbg_checksum_vertices. */
 typedef struct {
   uint64_t distinct, sum_count, sum_edges, checksum;
 } dbg_stats;
@@ -219,6 +220,14 @@ DBG_API uint64_t dbg_sort_workspace_bytes(const dbg_params* prm, uint64_t n);
 DBG_API dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_in, dbg_vertex* d_out,
                              uint64_t n, void* d_workspace, uint64_t workspace_bytes,
                              cudaStream_t stream);
+
+/* Adds the order-independent checksum of n vertex records (SURVEY.md 8(d):
+ * per record h = fmix64 chained over kmer_hi, kmer_lo, count, out[0..3],
+ * in[0..3]; the sum of h mod 2^64) to d_stats->checksum.  The extraction
+ * calls fill distinct / sum_count / sum_edges only; this validation
+ * statistic is computed apart from the path. */
+DBG_API dbg_status dbg_checksum_vertices(const dbg_params* prm, const dbg_vertex* d_vertices, uint64_t n,
+                                 dbg_stats* d_stats, cudaStream_t stream);
 
 /* Synchronizes the stream, then decodes *d_status: bit 0 -> DBG_ETABLEFULL,
  * bit 1 or 2 -> DBG_ENOSPACE; also returns DBG_ECUDA on a sticky CUDA error. */

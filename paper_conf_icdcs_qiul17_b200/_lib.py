@@ -72,6 +72,7 @@ SIGNATURES = {
     "dbg_extract_graph": (ctypes.c_int, [_PRM, _P, _P, _I32, _I32, _P, _U64, _P, _P, _P, _P]),
     "dbg_sort_workspace_bytes": (_U64, [_PRM, _U64]),
     "dbg_sort_vertices": (ctypes.c_int, [_PRM, _P, _P, _U64, _P, _U64, _P]),
+    "dbg_checksum_vertices": (ctypes.c_int, [_PRM, _P, _U64, _P, _P]),
     "dbg_sync_status": (ctypes.c_int, [_P, _P]),
     "dbg_status_string": (ctypes.c_char_p, [ctypes.c_int]),
 }
@@ -242,6 +243,11 @@ def dbg_sort_vertices(prm, d_in, d_out, n: int, d_workspace, workspace_bytes: in
     _check("dbg_sort_vertices", load().dbg_sort_vertices(
         ctypes.byref(prm), _ptr(d_in), _ptr(d_out), n, _ptr(d_workspace), workspace_bytes,
         _stream(stream)))
+
+
+def dbg_checksum_vertices(prm, d_vertices, n: int, d_stats, stream=None) -> None:
+    _check("dbg_checksum_vertices", load().dbg_checksum_vertices(ctypes.byref(prm), _ptr(d_vertices), n,
+                                                                 _ptr(d_stats), _stream(stream)))
 
 
 def dbg_sync_status(d_status, stream=None) -> int:

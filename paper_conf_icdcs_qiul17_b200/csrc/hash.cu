@@ -326,7 +326,7 @@ __device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t
   if (threadIdx.x == 0) sh.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
   __syncthreads();
   uint64_t pos = sh.base + excl;
-  unsigned long long st_count = 0, st_edges = 0, st_sum = 0;
+  unsigned long long st_count = 0, st_edges = 0;
   while (bits) {
     const int q = __ffs(bits) - 1;
     bits &= bits - 1;
@@ -358,11 +358,6 @@ __device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t
     if (pos < oa.out_cap) oa.out[pos] = v;
     else atomicOr(oa.status, kStatusNoSpace);
     ++pos;
-    const uint64_t f[11] = {v.kmer_hi, v.kmer_lo, v.count, a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
-    uint64_t h = 0;
-#pragma unroll
-    for (int t = 0; t < 11; ++t) h = fmix64(h ^ f[t]);
-    st_sum += h;
     st_count += v.count;
     st_edges += (uint64_t)a.x + a.y + a.z + a.w + b.x + b.y + b.z + b.w;
   }
@@ -371,13 +366,10 @@ __device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t
     const unsigned long long c = Red(sh.red).Sum(st_count);
     __syncthreads();
     const unsigned long long e = Red(sh.red).Sum(st_edges);
-    __syncthreads();
-    const unsigned long long h = Red(sh.red).Sum(st_sum);
     if (threadIdx.x == 0) {
       atomicAdd(oa.stats + 0, (unsigned long long)total);
       atomicAdd(oa.stats + 1, c);
       atomicAdd(oa.stats + 2, e);
-      atomicAdd(oa.stats + 3, h);
     }
   }
   __syncthreads();
@@ -638,21 +630,25 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
 // --------------------------------------------------------------- on-chip Step 2
 //
 // One CTA builds one fine partition at a time entirely in shared memory
-// (dbg_build_subgraphs_smem): its warps hash the partition's records (K-mers
-// spread over lanes as in hash_warp), then the CTA compacts the occupied
-// slots straight into the output and zeroes them again (clean-on-extract, so
-// no zero pass between partitions).  Slot = key (8 B; 16 B for K > 31) +
-// 16-bit counter fields out[0..3], in[0..3], t_out packed two per 32-bit
-// word: a field never exceeds the partition's K-mer count, and the on-chip
-// path takes only partitions with capacity (>= N^i_kmer) below 65536, so the
-// 32-bit shared-memory atomicAdd of (1 << 16*half) never carries across
-// fields.  Per partition: one block scan, one global atomicAdd (output
-// reservation) and two barriers; totals are reduced once per CTA.
+// (dbg_build_subgraphs_smem).  The partition's records are loaded in batches
+// into shared memory, a block scan of their K-mer counts flattens the batch,
+// and each thread takes an equal contiguous run of K-mers, rolling the
+// forward/reverse codes from one K-mer to the next inside a record
+// (<kmer, edge> pair generation).  Each occurrence is inserted or
+// updated in the shared-memory table (one insertion, multiple updates,
+// P:L504-511): a 64/128-bit shared-memory CAS claims an empty slot, shared-
+// memory atomics count the edges.  The CTA then compacts the occupied slots
+// straight into the output and zeroes them again (clean-on-extract, so no
+// zero pass between partitions).
+//
+// Slot = key (8 B; 16 B for K > 31) + 16-bit counter fields out[0..3],
+// in[0..3], t_out packed two per 32-bit word: a field never exceeds the
+// partition's K-mer count, and the on-chip path takes only partitions whose
+// capacity (>= N^i_kmer) is below 65536, so the 32-bit shared-memory
+// atomicAdd of (1 << 16*half) never carries across fields.
 
 constexpr int kSmemThreads = 512;
-constexpr int kSmemWarps = kSmemThreads / 32;
-constexpr int kSmemXPer = 4;
-constexpr uint32_t kSmemXTile = kSmemThreads * kSmemXPer;
+constexpr int kRecBatch = 1024;  // records staged per batch (2 per thread)
 constexpr uint64_t kSmemMaxSlots = 65535;
 
 template <int KW>
@@ -661,7 +657,10 @@ struct SmemSlot {
   static constexpr uint32_t kFieldOff = KW == 1 ? 8 : 16;
 };
 
-struct SmemShared512 {
+template <int R>
+struct SmemStage {
+  uint32_t w[kRecBatch][R];
+  uint32_t pre[kRecBatch + 1];
   typename cub::BlockScan<uint32_t, kSmemThreads>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, kSmemThreads>::TempStorage red;
   unsigned long long base;
@@ -669,7 +668,7 @@ struct SmemShared512 {
 
 template <int R>
 __host__ __device__ constexpr uint32_t smem_fixed_bytes() {
-  return (uint32_t)((sizeof(WarpRecs<R>) * kSmemWarps + sizeof(SmemShared512) + 127) & ~size_t(127));
+  return (uint32_t)((sizeof(SmemStage<R>) + 127) & ~size_t(127));
 }
 
 struct SmemArgs {
@@ -677,33 +676,43 @@ struct SmemArgs {
   const uint64_t* rec_off;
   const uint64_t* n_kmers;
   int n_fine, k;
-  double ratio;       // lambda / (4 alpha)
-  uint64_t slots;     // table slots that fit
+  double ratio;    // lambda / (4 alpha)
+  uint64_t slots;  // table slots that fit
 };
 
 __device__ __forceinline__ void smem_count(uint32_t* fields, int f) {
   atomicAdd(fields + (f >> 1), 1u << (16 * (f & 1)));
 }
 
-// Insert/update of one occurrence in a shared-memory table.
+// 32-bit table hash of a code (the probe sequence is free, reading P).
+__device__ __forceinline__ uint32_t smem_hash(uint64_t code) {
+  return (uint32_t)(((code ^ (code >> 29)) * 0x9e3779b97f4a7c15ull) >> 32);
+}
+__device__ __forceinline__ uint32_t smem_hash(unsigned long long code) { return smem_hash((uint64_t)code); }
+__device__ __forceinline__ uint32_t smem_hash(u128 code) {
+  return smem_hash((uint64_t)((uint64_t)code ^ ((uint64_t)(code >> 64) * 0xc2b2ae3d27d4eb4full)));
+}
+
+// Insert/update of one occurrence in a shared-memory table of cap slots.
 template <typename Code>
-__device__ __forceinline__ bool smem_upsert(char* table, uint64_t cap, const Job<Code>& jb) {
+__device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code, int o, int i) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   typedef KeyOf<Code> KO;
-  uint64_t idx = jb.idx;
-  for (uint64_t pr = 0; pr < cap; ++pr) {
+  const typename KO::T want = KO::make(code);
+  uint32_t idx = __umulhi(smem_hash(code), cap);
+  for (uint32_t pr = 0; pr < cap; ++pr) {
     char* kp = table + idx * SmemSlot<KW>::kBytes;
     typename KO::T cur;
     if constexpr (KW == 1) {
       cur = *reinterpret_cast<volatile unsigned long long*>(kp);
-      if (cur == 0) cur = KO::cas(kp, jb.want);
+      if (cur == 0) cur = KO::cas(kp, want);
     } else {
-      cur = KO::cas(kp, jb.want);  // 16-B shared-memory CAS: atomic read-or-claim
+      cur = KO::cas(kp, want);  // 16-B shared-memory CAS: atomic read-or-claim
     }
-    if (KO::empty(cur) || KO::same(cur, jb.want)) {
+    if (KO::empty(cur) || KO::same(cur, want)) {
       uint32_t* fields = reinterpret_cast<uint32_t*>(kp + SmemSlot<KW>::kFieldOff);
-      smem_count(fields, jb.o < 4 ? jb.o : 8);
-      if (jb.i >= 0) smem_count(fields, 4 + jb.i);
+      smem_count(fields, o < 4 ? o : 8);
+      if (i >= 0) smem_count(fields, 4 + i);
       return true;
     }
     idx = idx + 1 == cap ? 0 : idx + 1;
@@ -712,89 +721,115 @@ __device__ __forceinline__ bool smem_upsert(char* table, uint64_t cap, const Job
 }
 
 template <typename Code, int R>
-__device__ __forceinline__ bool hash_warp_smem(const uint32_t* recs, int64_t n_recs, int K, char* table,
-                                               uint64_t cap, WarpRecs<R>& sm) {
-  const int lane = threadIdx.x & 31;
-  uint32_t n = 0;
-  if (lane < n_recs) {
-    const uint4* src = reinterpret_cast<const uint4*>(recs + (uint64_t)lane * R);
-#pragma unroll
-    for (int v = 0; v < R / 4; ++v) {
-      const uint4 x = __ldcs(src + v);  // streamed once
-      sm.w[lane][4 * v] = x.x;
-      sm.w[lane][4 * v + 1] = x.y;
-      sm.w[lane][4 * v + 2] = x.z;
-      sm.w[lane][4 * v + 3] = x.w;
-    }
-    n = sm.w[lane][0] & 255u;
-    sm.t0[lane] = 0;
-    sm.cap[lane] = cap;
-  }
-  uint32_t incl = n;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const uint32_t v = __shfl_up_sync(kFull, incl, d);
-    if (lane >= d) incl += v;
-  }
-  sm.pre[lane + 1] = incl;
-  if (lane == 0) sm.pre[0] = 0;
-  const uint32_t total = __shfl_sync(kFull, incl, 31);
-  __syncwarp();
-  const uint32_t share = (total + 31) / 32;
-  const uint32_t k0 = min(total, lane * share), k1 = min(total, k0 + share);
-  bool ok = true;
-  int r = 0;
-  for (uint32_t kid = k0; kid < k1; ++kid) ok &= smem_upsert(table, cap, make_job<Code, R>(sm, kid, r, K));
-  __syncwarp();
-  return ok;
-}
-
-template <typename Code, int R>
 __global__ void __launch_bounds__(kSmemThreads, 1) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   constexpr uint32_t SB = SmemSlot<KW>::kBytes;
+  typedef cub::BlockScan<uint32_t, kSmemThreads> Scan;
   extern __shared__ __align__(128) unsigned char smem[];
-  WarpRecs<R>* shw = reinterpret_cast<WarpRecs<R>*>(smem);
-  SmemShared512& sh = *reinterpret_cast<SmemShared512*>(smem + sizeof(WarpRecs<R>) * kSmemWarps);
+  SmemStage<R>& st = *reinterpret_cast<SmemStage<R>*>(smem);
   char* table = reinterpret_cast<char*>(smem + smem_fixed_bytes<R>());
-  const int warp = threadIdx.x >> 5;
+  const int K = a.k;
+  const int top = 2 * K - 2;
+  const Code mask = ((Code)1 << (2 * K)) - 1;
   {  // the table starts clean; extraction keeps it clean
     uint4* z = reinterpret_cast<uint4*>(table);
     for (uint64_t q = threadIdx.x; q < a.slots * (SB / 16); q += kSmemThreads) z[q] = make_uint4(0, 0, 0, 0);
   }
-  unsigned long long st_n = 0, st_count = 0, st_edges = 0, st_sum = 0;
+  unsigned long long st_n = 0, st_count = 0, st_edges = 0;
   bool ok = true;
   for (uint64_t p = blockIdx.x; p < (uint64_t)a.n_fine; p += gridDim.x) {
     const uint64_t nk = a.n_kmers[p];
     if (nk == 0) continue;
     const double c = ceil(a.ratio * (double)nk);  // capacity, Sec. IV-A
-    const uint64_t cap = c < 1.0 ? 1ull : (uint64_t)c;
-    if (cap > a.slots) continue;  // left to the global-table path (dbg_table_plan_split)
+    const uint64_t cap64 = c < 1.0 ? 1ull : (uint64_t)c;
+    if (cap64 > a.slots) continue;  // left to the global-table path (dbg_table_plan_split)
+    const uint32_t cap = (uint32_t)cap64;
     const uint64_t r0 = a.rec_off[p], nrec = a.rec_off[p + 1] - r0;
-    // spread the records over all warps (chunks of <= 32 records)
-    const uint64_t cs = min((uint64_t)32, (nrec + kSmemWarps - 1) / kSmemWarps);
-    __syncthreads();  // previous partition's extraction (and the initial zero fill) complete
-    for (uint64_t ch = warp; ch * cs < nrec; ch += kSmemWarps) {
-      const int64_t n = (int64_t)min(cs, nrec - ch * cs);
-      ok &= hash_warp_smem<Code, R>(a.records + (r0 + ch * cs) * R, n, a.k, table, cap, shw[warp]);
+    for (uint64_t rb = 0; rb < nrec; rb += kRecBatch) {
+      const int nb = (int)min((uint64_t)kRecBatch, nrec - rb);
+      __syncthreads();  // staging free; previous extraction (table clean) complete
+      uint32_t cnt[2];
+#pragma unroll
+      for (int v = 0; v < 2; ++v) {
+        const int j = 2 * threadIdx.x + v;
+        cnt[v] = 0;
+        if (j < nb) {
+          const uint4* src = reinterpret_cast<const uint4*>(a.records + (r0 + rb + j) * R);
+#pragma unroll
+          for (int q = 0; q < R / 4; ++q) {
+            const uint4 x = __ldcs(src + q);  // streamed once
+            st.w[j][4 * q] = x.x;
+            st.w[j][4 * q + 1] = x.y;
+            st.w[j][4 * q + 2] = x.z;
+            st.w[j][4 * q + 3] = x.w;
+            if (q == 0) cnt[v] = x.x & 255u;
+          }
+        }
+      }
+      uint32_t excl[2], total;
+      Scan(st.scan).ExclusiveSum(cnt, excl, total);
+      st.pre[2 * threadIdx.x] = excl[0];
+      st.pre[2 * threadIdx.x + 1] = excl[1];
+      if (threadIdx.x == 0) st.pre[kRecBatch] = total;
+      __syncthreads();
+      // this thread's contiguous run of K-mers [k0, k1)
+      const uint32_t share = (total + kSmemThreads - 1) / kSmemThreads;
+      const uint32_t k0 = min(total, threadIdx.x * share), k1 = min(total, k0 + share);
+      if (k0 < k1) {
+        int lo = 0, hi = nb;  // record holding K-mer k0: last r with pre[r] <= k0
+        while (hi - lo > 1) {
+          const int mid = (lo + hi) >> 1;
+          if (st.pre[mid] <= k0) lo = mid;
+          else hi = mid;
+        }
+        int r = lo;
+        int t = (int)(k0 - st.pre[r]);
+        const uint32_t* w = st.w[r];
+        int n = w[0] & 255u, hl = (w[0] >> 8) & 1u, hr = (w[0] >> 9) & 1u;
+        Code fwd, rc;
+        kmer_at(w, hl + t, K, R, fwd, rc);
+        for (uint32_t kid = k0;;) {
+          const int b = hl + t;
+          const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1) : -1;
+          const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K) : -1;
+          if (fwd < rc) {  // odd K: never equal (reading C); edges in the canonical orientation (reading J)
+            ok &= smem_upsert<Code>(table, cap, fwd, succ >= 0 ? succ : 4, pred);
+          } else {
+            ok &= smem_upsert<Code>(table, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1);
+          }
+          if (++kid >= k1) break;
+          if (++t < n) {  // next K-mer of the same record: roll one base
+            fwd = ((fwd << 2) | (Code)succ) & mask;
+            rc = (rc >> 2) | ((Code)(3 - succ) << top);
+          } else {  // next record
+            ++r;
+            t = 0;
+            w = st.w[r];
+            n = w[0] & 255u;
+            hl = (w[0] >> 8) & 1u;
+            hr = (w[0] >> 9) & 1u;
+            kmer_at(w, hl, K, R, fwd, rc);
+          }
+        }
+      }
     }
     __syncthreads();
     // extraction: each thread owns slots s = q * kSmemThreads + tid; one block
     // scan sizes the partition's output, one global atomic reserves it
     uint32_t cnt = 0;
-    for (uint64_t s = threadIdx.x; s < cap; s += kSmemThreads)
+    for (uint32_t s = threadIdx.x; s < cap; s += kSmemThreads)
       cnt += (*reinterpret_cast<const unsigned long long*>(table + s * SB) & kOccupied) ? 1u : 0u;
     uint32_t excl, total;
-    cub::BlockScan<uint32_t, kSmemThreads>(sh.scan).ExclusiveSum(cnt, excl, total);
-    if (threadIdx.x == 0) sh.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
+    Scan(st.scan).ExclusiveSum(cnt, excl, total);
+    if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
     __syncthreads();
-    uint64_t pos = sh.base + excl;
+    uint64_t pos = st.base + excl;
     const uint32_t pid = (uint32_t)(p % oa.np_out);
-    for (uint64_t s = threadIdx.x; s < cap; s += kSmemThreads) {
+    for (uint32_t s = threadIdx.x; s < cap; s += kSmemThreads) {
       char* sp = table + s * SB;
       const uint64_t k0 = *reinterpret_cast<const unsigned long long*>(sp);
       if (!(k0 & kOccupied)) continue;
-      uint32_t* f = reinterpret_cast<uint32_t*>(sp + SmemSlot<KW>::kFieldOff);
+      const uint32_t* f = reinterpret_cast<const uint32_t*>(sp + SmemSlot<KW>::kFieldOff);
       dbg_vertex v;
       if (KW == 1) {
         v.kmer_hi = 0;
@@ -814,13 +849,7 @@ __global__ void __launch_bounds__(kSmemThreads, 1) smem_subgraph_kernel(SmemArgs
       if (pos < oa.out_cap) oa.out[pos] = v;
       else atomicOr(oa.status, kStatusNoSpace);
       ++pos;
-      const uint64_t fl[11] = {v.kmer_hi, v.kmer_lo, v.count, v.out[0], v.out[1], v.out[2], v.out[3],
-                               v.in[0], v.in[1], v.in[2], v.in[3]};
-      uint64_t h = 0;
-#pragma unroll
-      for (int t = 0; t < 11; ++t) h = fmix64(h ^ fl[t]);
       st_n += 1;
-      st_sum += h;
       st_count += v.count;
       st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
     }
@@ -828,19 +857,39 @@ __global__ void __launch_bounds__(kSmemThreads, 1) smem_subgraph_kernel(SmemArgs
   if (!ok) atomicOr(oa.status, kStatusTableFull);
   __syncthreads();
   typedef cub::BlockReduce<unsigned long long, kSmemThreads> Red;
-  const unsigned long long n = Red(sh.red).Sum(st_n);
+  const unsigned long long n = Red(st.red).Sum(st_n);
   __syncthreads();
-  const unsigned long long cc = Red(sh.red).Sum(st_count);
+  const unsigned long long cc = Red(st.red).Sum(st_count);
   __syncthreads();
-  const unsigned long long e = Red(sh.red).Sum(st_edges);
-  __syncthreads();
-  const unsigned long long hh = Red(sh.red).Sum(st_sum);
+  const unsigned long long e = Red(st.red).Sum(st_edges);
   if (threadIdx.x == 0 && n) {
     atomicAdd(oa.stats + 0, n);
     atomicAdd(oa.stats + 1, cc);
     atomicAdd(oa.stats + 2, e);
-    atomicAdd(oa.stats + 3, hh);
   }
+}
+
+// --------------------------------------------------------------- checksum
+
+// Order-independent checksum of vertex records: per record
+// h = fmix64 chained over its 11 fields; the sum of h (mod 2^64) is added to
+// *sum.  A validation statistic, computed apart from the path.
+__global__ void __launch_bounds__(256) checksum_kernel(const dbg_vertex* __restrict__ v, uint64_t n,
+                                                      unsigned long long* sum) {
+  typedef cub::BlockReduce<unsigned long long, 256> Red;
+  __shared__ typename Red::TempStorage tmp;
+  unsigned long long acc = 0;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const dbg_vertex x = v[i];
+    const uint64_t f[11] = {x.kmer_hi, x.kmer_lo, x.count, x.out[0], x.out[1], x.out[2], x.out[3],
+                            x.in[0], x.in[1], x.in[2], x.in[3]};
+    uint64_t h = 0;
+#pragma unroll
+    for (int t = 0; t < 11; ++t) h = fmix64(h ^ f[t]);
+    acc += h;
+  }
+  const unsigned long long s = Red(tmp).Sum(acc);
+  if (threadIdx.x == 0 && s) atomicAdd(sum, s);
 }
 
 // --------------------------------------------------------------- sort
@@ -982,6 +1031,16 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   else if (prm->k <= 39) e = launch_smem<u128, 4>(a, oa, stream);
   else e = launch_smem<u128, 8>(a, oa, stream);
   return e == cudaSuccess ? DBG_OK : DBG_ECUDA;
+}
+
+extern "C" dbg_status dbg_checksum_vertices(const dbg_params* prm, const dbg_vertex* d_vertices, uint64_t n,
+                                            dbg_stats* d_stats, cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !d_stats || (n && !d_vertices)) return DBG_EINVAL;
+  if (n == 0) return DBG_OK;
+  const uint64_t want = (n + 255) / 256, cap = (uint64_t)dbg_sm_count() * 8;
+  checksum_kernel<<<(int)(want < cap ? want : cap), 256, 0, stream>>>(
+      d_vertices, n, reinterpret_cast<unsigned long long*>(d_stats) + 3);
+  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
 static uint64_t n_groups_max(uint64_t total_slots, uint64_t group_slots) {

@@ -282,7 +282,14 @@ class DbgBuilder:
                                    self.d_n_out, self.d_stats, self.d_status, stream)
             self._done(ev, stream)
 
-    def stats(self) -> dict:
+    def stats(self, checksum: bool = True, stream=None) -> dict:
+        """Totals of the last extraction; the checksum is computed here (dbg_checksum_vertices)."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        if checksum:
+            n = min(int(self.d_n_out.item()), self.out_cap())
+            with torch.cuda.stream(stream):
+                self.d_stats[3].zero_()
+            _lib.dbg_checksum_vertices(self.prm, self.out, n, self.d_stats, stream)
         s = self.d_stats.cpu().numpy().view(np.uint64)
         return {f: int(v) for f, v in zip(STATS_FIELDS, s)}
 
