@@ -42,6 +42,8 @@
 #include <cub/block/block_scan.cuh>
 #include <cub/device/device_radix_sort.cuh>
 
+#include <cstdlib>
+
 #include "dbg_device.cuh"
 
 int dbg_sm_count();
@@ -647,8 +649,6 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
 // capacity (>= N^i_kmer) is below 65536, so the 32-bit shared-memory
 // atomicAdd of (1 << 16*half) never carries across fields.
 
-constexpr int kSmemThreads = 512;
-constexpr int kRecBatch = 1024;  // records staged per batch (2 per thread)
 constexpr uint64_t kSmemMaxSlots = 65535;
 
 template <int KW>
@@ -657,18 +657,19 @@ struct SmemSlot {
   static constexpr uint32_t kFieldOff = KW == 1 ? 8 : 16;
 };
 
-template <int R>
+// T threads per CTA stage 2T records per batch.
+template <int R, int T>
 struct SmemStage {
-  uint32_t w[kRecBatch][R];
-  uint32_t pre[kRecBatch + 1];
-  typename cub::BlockScan<uint32_t, kSmemThreads>::TempStorage scan;
-  typename cub::BlockReduce<unsigned long long, kSmemThreads>::TempStorage red;
+  uint32_t w[2 * T][R];
+  uint32_t pre[2 * T + 1];
+  typename cub::BlockScan<uint32_t, T>::TempStorage scan;
+  typename cub::BlockReduce<unsigned long long, T>::TempStorage red;
   unsigned long long base;
 };
 
-template <int R>
+template <int R, int T>
 __host__ __device__ constexpr uint32_t smem_fixed_bytes() {
-  return (uint32_t)((sizeof(SmemStage<R>) + 127) & ~size_t(127));
+  return (uint32_t)((sizeof(SmemStage<R, T>) + 127) & ~size_t(127));
 }
 
 struct SmemArgs {
@@ -720,14 +721,15 @@ __device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code
   return false;
 }
 
-template <typename Code, int R>
-__global__ void __launch_bounds__(kSmemThreads, 1) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
+template <typename Code, int R, int kSmemThreads, int kMinCtas>
+__global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   constexpr uint32_t SB = SmemSlot<KW>::kBytes;
+  constexpr int kRecBatch = 2 * kSmemThreads;
   typedef cub::BlockScan<uint32_t, kSmemThreads> Scan;
   extern __shared__ __align__(128) unsigned char smem[];
-  SmemStage<R>& st = *reinterpret_cast<SmemStage<R>*>(smem);
-  char* table = reinterpret_cast<char*>(smem + smem_fixed_bytes<R>());
+  SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
+  char* table = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
   const int K = a.k;
   const int top = 2 * K - 2;
   const Code mask = ((Code)1 << (2 * K)) - 1;
@@ -978,28 +980,58 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-template <int R>
-static uint64_t smem_slots_for(int k) {
-  const uint64_t avail = 227u * 1024u - smem_fixed_bytes<R>();
+// CTAs per SM of the on-chip kernel (1, 2 or 4; env DBG_SMEM_CTAS, default 4):
+// several CTAs overlap one partition's load/scan/extract latencies with
+// another's hashing; the table per CTA shrinks accordingly.
+static int smem_ctas() {
+  static int v = [] {
+    const char* e = getenv("DBG_SMEM_CTAS");
+    const int x = e ? atoi(e) : 4;
+    return (x == 1 || x == 2 || x == 4) ? x : 4;
+  }();
+  return v;
+}
+
+template <int R, int T>
+static uint64_t smem_slots_for(int k, int ctas) {
+  const uint64_t avail = (227u * 1024u) / ctas - smem_fixed_bytes<R, T>() - 1024u;
   const uint32_t sb = k <= 31 ? SmemSlot<1>::kBytes : SmemSlot<2>::kBytes;
   const uint64_t n = (avail / sb) & ~(uint64_t)63;
   return n < kSmemMaxSlots ? n : kSmemMaxSlots;
 }
 
+static uint64_t smem_slots(int k, int ctas) {
+  const bool r4 = record_words(k) == 4;
+  switch (ctas) {
+    case 1: return r4 ? smem_slots_for<4, 512>(k, 1) : smem_slots_for<8, 512>(k, 1);
+    case 2: return r4 ? smem_slots_for<4, 256>(k, 2) : smem_slots_for<8, 256>(k, 2);
+    default: return r4 ? smem_slots_for<4, 128>(k, 4) : smem_slots_for<8, 128>(k, 4);
+  }
+}
+
 extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
   if (!prm) return 0;
-  return record_words(prm->k) == 4 ? smem_slots_for<4>(prm->k) : smem_slots_for<8>(prm->k);
+  return smem_slots(prm->k, smem_ctas());
+}
+
+template <typename Code, int R, int T, int C>
+static cudaError_t launch_smem_t(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
+  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
+  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes;
+  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e != cudaSuccess) return e;
+  smem_subgraph_kernel<Code, R, T, C><<<dbg_sm_count() * C, T, bytes, stream>>>(a, oa);
+  return cudaGetLastError();
 }
 
 template <typename Code, int R>
 static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
-  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  const size_t bytes = smem_fixed_bytes<R>() + a.slots * SmemSlot<KW>::kBytes;
-  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)bytes);
-  if (e != cudaSuccess) return e;
-  smem_subgraph_kernel<Code, R><<<dbg_sm_count(), kSmemThreads, bytes, stream>>>(a, oa);
-  return cudaGetLastError();
+  switch (smem_ctas()) {
+    case 1: return launch_smem_t<Code, R, 512, 1>(a, oa, stream);
+    case 2: return launch_smem_t<Code, R, 256, 2>(a, oa, stream);
+    default: return launch_smem_t<Code, R, 128, 4>(a, oa, stream);
+  }
 }
 
 extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,

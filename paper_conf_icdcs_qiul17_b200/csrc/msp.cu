@@ -265,9 +265,11 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   }
 }
 
-// Exclusive prefix sum out[0..n] of f(in[0..n-1]) in one CTA (n = NP is small);
-// f = identity (record offsets) or the table capacity of Sec. IV-A.
-constexpr int kScanThreads = 256;
+// Exclusive prefix sum out[0..n] of f(in[0..n-1]) in one CTA (n = number of
+// fine partitions: up to a few 10^5); f = identity (record offsets) or the
+// table capacity of Sec. IV-A.  512 threads x 8 consecutive items per pass.
+constexpr int kScanThreads = 512;
+constexpr int kScanItems = 8;
 template <bool kCapacity>
 __global__ void __launch_bounds__(kScanThreads) scan_kernel(const uint64_t* __restrict__ in,
                                                             uint64_t* __restrict__ out, int n,
@@ -277,21 +279,30 @@ __global__ void __launch_bounds__(kScanThreads) scan_kernel(const uint64_t* __re
   __shared__ unsigned long long carry;
   if (threadIdx.x == 0) carry = 0;
   __syncthreads();
-  for (int base = 0; base < n; base += kScanThreads) {
-    const int i = base + threadIdx.x;
-    unsigned long long v = 0;
-    if (i < n) {
-      v = in[i];
-      if (kCapacity && v) {
-        // capacity_i = ceil(lambda / (4 alpha) * N^i_kmer), at least 1
-        double c = ceil(ratio * (double)v);
-        v = c < 1.0 ? 1ull : (unsigned long long)c;
-        if (v <= skip_upto) v = 0;  // built on chip (dbg_table_plan_split)
+  constexpr int kTile = kScanThreads * kScanItems;
+  for (int base = 0; base < n; base += kTile) {
+    unsigned long long v[kScanItems];
+#pragma unroll
+    for (int q = 0; q < kScanItems; ++q) {
+      const int i = base + threadIdx.x * kScanItems + q;
+      v[q] = 0;
+      if (i < n) {
+        v[q] = in[i];
+        if (kCapacity && v[q]) {
+          // capacity_i = ceil(lambda / (4 alpha) * N^i_kmer), at least 1
+          const double c = ceil(ratio * (double)v[q]);
+          v[q] = c < 1.0 ? 1ull : (unsigned long long)c;
+          if (v[q] <= skip_upto) v[q] = 0;  // built on chip (dbg_table_plan_split)
+        }
       }
     }
-    unsigned long long excl, total;
-    Scan(tmp).ExclusiveSum(v, excl, total);
-    if (i < n) out[i] = carry + excl;
+    unsigned long long total;
+    Scan(tmp).ExclusiveSum(v, v, total);
+#pragma unroll
+    for (int q = 0; q < kScanItems; ++q) {
+      const int i = base + threadIdx.x * kScanItems + q;
+      if (i < n) out[i] = carry + v[q];
+    }
     __syncthreads();
     if (threadIdx.x == 0) carry += total;
     __syncthreads();

@@ -344,10 +344,7 @@ def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 
     slots = _lib.dbg_smem_table_slots(prm)
     per_part = max(1.0, fill * slots / max(lam / (4 * alpha), 1e-9))
     f = max(1, int(np.ceil(n_kmers / (num_partitions * per_part))))
-    f = 1 << int(np.ceil(np.log2(f)))
-    while num_partitions * f > 4_194_303 and f > 1:
-        f //= 2
-    return f
+    return max(1, min(f, 4_194_303 // num_partitions))
 
 
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
