@@ -62,7 +62,8 @@ SIGNATURES = {
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
     "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P]),
     "dbg_smem_table_slots": (_U64, [_PRM]),
-    "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _P, _P, _U64, _P, _P, _P, _P]),
+    "dbg_smem_workspace_bytes": (_U64, [_PRM]),
+    "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _P, _U64, _P, _U64, _P, _P, _P, _P]),
     "dbg_table_plan_split": (ctypes.c_int, [_PRM, _P, _U64, _P, _P]),
     "dbg_subgraph_ring_bytes": (_U64, [_PRM, _U64, _U64]),
     "dbg_subgraph_workspace_bytes": (_U64, [_PRM, _I32, _U64, _U64]),
@@ -192,11 +193,15 @@ def dbg_smem_table_slots(prm) -> int:
     return load().dbg_smem_table_slots(ctypes.byref(prm))
 
 
-def dbg_build_subgraphs_smem(prm, part, d_work, d_out, out_cap: int, d_n_out, d_stats, d_status,
+def dbg_smem_workspace_bytes(prm) -> int:
+    return load().dbg_smem_workspace_bytes(ctypes.byref(prm))
+
+
+def dbg_build_subgraphs_smem(prm, part, d_work, work_bytes: int, d_out, out_cap: int, d_n_out, d_stats, d_status,
                              stream=None) -> None:
     _check("dbg_build_subgraphs_smem", load().dbg_build_subgraphs_smem(
-        ctypes.byref(prm), ctypes.byref(part), _ptr(d_work), _ptr(d_out), out_cap, _ptr(d_n_out), _ptr(d_stats),
-        _ptr(d_status), _stream(stream)))
+        ctypes.byref(prm), ctypes.byref(part), _ptr(d_work), work_bytes, _ptr(d_out), out_cap, _ptr(d_n_out),
+        _ptr(d_stats), _ptr(d_status), _stream(stream)))
 
 
 def dbg_table_plan_split(prm, d_n_kmers, smem_slots: int, d_table_offset, stream=None) -> None:

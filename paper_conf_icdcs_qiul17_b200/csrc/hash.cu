@@ -661,6 +661,8 @@ struct SmemSlot {
 template <int R, int T>
 struct SmemStage {
   uint32_t w[2 * T][R];
+  uint32_t t0[2 * T];   // first slot of the record's partition table in the CTA table
+  uint32_t cap[2 * T];  // its capacity (0: partition off chip)
   uint32_t pre[2 * T + 1];
   typename cub::BlockScan<uint32_t, T>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, T>::TempStorage red;
@@ -671,15 +673,6 @@ template <int R, int T>
 __host__ __device__ constexpr uint32_t smem_fixed_bytes() {
   return (uint32_t)((sizeof(SmemStage<R, T>) + 127) & ~size_t(127));
 }
-
-struct SmemArgs {
-  const uint32_t* records;
-  const uint64_t* rec_off;
-  const uint64_t* n_kmers;
-  int n_fine, k;
-  double ratio;    // lambda / (4 alpha)
-  uint64_t slots;  // table slots that fit
-};
 
 __device__ __forceinline__ void smem_count(uint32_t* fields, int f) {
   atomicAdd(fields + (f >> 1), 1u << (16 * (f & 1)));
@@ -721,6 +714,130 @@ __device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code
   return false;
 }
 
+struct SmemArgs {
+  const uint32_t* records;
+  const uint64_t* rec_off;
+  const uint64_t* n_kmers;
+  int n_fine, k;
+  double ratio;      // lambda / (4 alpha)
+  uint64_t slots;    // table slots that fit one CTA
+  uint64_t* P;       // [n_fine + 1] prefix of on-chip capacities (0 for partitions off chip)
+  uint32_t* gfirst;  // [n_fine + 2] first partition of each group
+  unsigned long long* n_groups;
+};
+
+// Capacity of partition p on chip (Sec. IV-A), or 0 if it is
+// empty or does not fit (then it goes to the global-table path).
+__device__ __forceinline__ uint64_t smem_cap(const SmemArgs& a, uint64_t nk) {
+  if (nk == 0) return 0;
+  const double c = ceil(a.ratio * (double)nk);
+  const uint64_t cap = c < 1.0 ? 1ull : (uint64_t)c;
+  return cap <= a.slots ? cap : 0;
+}
+
+// Single CTA: P = prefix of on-chip capacities, then groups of consecutive
+// partitions that share one CTA table.  With H = slots/2 and w(p) =
+// floor(P[p]/H), partition p starts a group iff p == 0, w(p) != w(p-1), or p
+// or p-1 has capacity > H.  A group of small partitions then lies in one
+// H-window and spans < H + H = slots; a large one is alone (<= slots).
+constexpr int kPlanThreads = 512, kPlanItems = 8;
+__global__ void __launch_bounds__(kPlanThreads) smem_plan_kernel(SmemArgs a) {
+  typedef cub::BlockScan<unsigned long long, kPlanThreads> Scan;
+  __shared__ typename Scan::TempStorage tmp;
+  __shared__ unsigned long long carry_p, carry_g, last_cap, last_w;
+  const uint64_t H = a.slots / 2;
+  if (threadIdx.x == 0) {
+    carry_p = 0;
+    carry_g = 0;
+    last_cap = 0;
+    last_w = ~0ull;
+  }
+  __syncthreads();
+  constexpr int kTile = kPlanThreads * kPlanItems;
+  for (int base = 0; base < a.n_fine; base += kTile) {
+    unsigned long long cap[kPlanItems], pre[kPlanItems];
+#pragma unroll
+    for (int q = 0; q < kPlanItems; ++q) {
+      const int p = base + threadIdx.x * kPlanItems + q;
+      cap[q] = p < a.n_fine ? smem_cap(a, a.n_kmers[p]) : 0;
+    }
+    unsigned long long tot;
+    Scan(tmp).ExclusiveSum(cap, pre, tot);
+    __syncthreads();
+    // start flags need the previous partition's capacity and window
+    unsigned long long flag[kPlanItems], gpre[kPlanItems];
+    const unsigned long long cp = carry_p;
+#pragma unroll
+    for (int q = 0; q < kPlanItems; ++q) {
+      const int p = base + threadIdx.x * kPlanItems + q;
+      const unsigned long long P = cp + pre[q];
+      unsigned long long pcap, pw;
+      if (q > 0) {
+        pcap = cap[q - 1];
+        pw = (cp + pre[q - 1]) / H;
+      } else {
+        // neighbour item lives in the previous thread (or tile)
+        pcap = 0;
+        pw = 0;
+      }
+      flag[q] = 0;
+      if (p < a.n_fine) {
+        a.P[p] = P;
+        flag[q] = (P / H != pw) || cap[q] > H || pcap > H;
+      }
+      (void)pw;
+    }
+    // fix item 0 with the previous thread's last item (shuffle within warps, smem across)
+    {
+      const unsigned long long my_last_cap = cap[kPlanItems - 1];
+      const unsigned long long my_last_w = (cp + pre[kPlanItems - 1]) / H;
+      __shared__ unsigned long long sh_cap[kPlanThreads], sh_w[kPlanThreads];
+      sh_cap[threadIdx.x] = my_last_cap;
+      sh_w[threadIdx.x] = my_last_w;
+      __syncthreads();
+      const int p0 = base + threadIdx.x * kPlanItems;
+      if (p0 < a.n_fine) {
+        unsigned long long pcap, pw;
+        if (threadIdx.x > 0) {
+          pcap = sh_cap[threadIdx.x - 1];
+          pw = sh_w[threadIdx.x - 1];
+        } else {
+          pcap = last_cap;
+          pw = last_w;
+        }
+        const unsigned long long P = cp + pre[0];
+        flag[0] = p0 == 0 || (P / H != pw) || cap[0] > H || pcap > H;
+      }
+      __syncthreads();
+      if (threadIdx.x == kPlanThreads - 1) {
+        last_cap = my_last_cap;
+        last_w = my_last_w;
+      }
+    }
+    unsigned long long gtot;
+    Scan(tmp).ExclusiveSum(flag, gpre, gtot);
+    const unsigned long long cg = carry_g;
+#pragma unroll
+    for (int q = 0; q < kPlanItems; ++q) {
+      const int p = base + threadIdx.x * kPlanItems + q;
+      if (p < a.n_fine && flag[q]) a.gfirst[cg + gpre[q]] = (uint32_t)p;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      carry_p += tot;
+      carry_g += gtot;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    a.P[a.n_fine] = carry_p;
+    a.gfirst[carry_g] = (uint32_t)a.n_fine;
+    *a.n_groups = carry_g;
+  }
+}
+
+// A group of consecutive fine partitions shares one CTA table: each partition
+// p owns slots [P[p] - P[first], P[p+1] - P[first]).
 template <typename Code, int R, int kSmemThreads, int kMinCtas>
 __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
@@ -739,14 +856,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   }
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
   bool ok = true;
-  for (uint64_t p = blockIdx.x; p < (uint64_t)a.n_fine; p += gridDim.x) {
-    const uint64_t nk = a.n_kmers[p];
-    if (nk == 0) continue;
-    const double c = ceil(a.ratio * (double)nk);  // capacity, Sec. IV-A
-    const uint64_t cap64 = c < 1.0 ? 1ull : (uint64_t)c;
-    if (cap64 > a.slots) continue;  // left to the global-table path (dbg_table_plan_split)
-    const uint32_t cap = (uint32_t)cap64;
-    const uint64_t r0 = a.rec_off[p], nrec = a.rec_off[p + 1] - r0;
+  const uint64_t n_groups = *a.n_groups;
+  for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
+    const int first = (int)a.gfirst[g], last = (int)a.gfirst[g + 1];
+    const uint64_t P0 = a.P[first], span = a.P[last] - P0;
+    if (span == 0) continue;  // nothing on chip in this group
+    const uint64_t r0 = a.rec_off[first], nrec = a.rec_off[last] - r0;
     for (uint64_t rb = 0; rb < nrec; rb += kRecBatch) {
       const int nb = (int)min((uint64_t)kRecBatch, nrec - rb);
       __syncthreads();  // staging free; previous extraction (table clean) complete
@@ -764,8 +879,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             st.w[j][4 * q + 1] = x.y;
             st.w[j][4 * q + 2] = x.z;
             st.w[j][4 * q + 3] = x.w;
-            if (q == 0) cnt[v] = x.x & 255u;
           }
+          const uint32_t pid = st.w[j][0] >> 10;
+          const uint64_t pp = a.P[pid], pc = a.P[pid + 1] - pp;
+          st.t0[j] = (uint32_t)(pp - P0);
+          st.cap[j] = (uint32_t)pc;
+          cnt[v] = pc ? st.w[j][0] & 255u : 0u;  // off-chip partition: skipped here
         }
       }
       uint32_t excl[2], total;
@@ -785,9 +904,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           else hi = mid;
         }
         int r = lo;
+        while (st.pre[r + 1] == st.pre[r]) ++r;  // skip records that contribute nothing
         int t = (int)(k0 - st.pre[r]);
         const uint32_t* w = st.w[r];
         int n = w[0] & 255u, hl = (w[0] >> 8) & 1u, hr = (w[0] >> 9) & 1u;
+        char* tab = table + (uint64_t)st.t0[r] * SB;
+        uint32_t cap = st.cap[r];
         Code fwd, rc;
         kmer_at(w, hl + t, K, R, fwd, rc);
         for (uint32_t kid = k0;;) {
@@ -795,21 +917,24 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1) : -1;
           const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K) : -1;
           if (fwd < rc) {  // odd K: never equal (reading C); edges in the canonical orientation (reading J)
-            ok &= smem_upsert<Code>(table, cap, fwd, succ >= 0 ? succ : 4, pred);
+            ok &= smem_upsert<Code>(tab, cap, fwd, succ >= 0 ? succ : 4, pred);
           } else {
-            ok &= smem_upsert<Code>(table, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1);
+            ok &= smem_upsert<Code>(tab, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1);
           }
           if (++kid >= k1) break;
           if (++t < n) {  // next K-mer of the same record: roll one base
             fwd = ((fwd << 2) | (Code)succ) & mask;
             rc = (rc >> 2) | ((Code)(3 - succ) << top);
-          } else {  // next record
-            ++r;
+          } else {  // next record that contributes K-mers
+            do ++r;
+            while (st.pre[r + 1] == st.pre[r]);
             t = 0;
             w = st.w[r];
             n = w[0] & 255u;
             hl = (w[0] >> 8) & 1u;
             hr = (w[0] >> 9) & 1u;
+            tab = table + (uint64_t)st.t0[r] * SB;
+            cap = st.cap[r];
             kmer_at(w, hl, K, R, fwd, rc);
           }
         }
@@ -817,17 +942,16 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
     }
     __syncthreads();
     // extraction: each thread owns slots s = q * kSmemThreads + tid; one block
-    // scan sizes the partition's output, one global atomic reserves it
+    // scan sizes the group's output, one global atomic reserves it
     uint32_t cnt = 0;
-    for (uint32_t s = threadIdx.x; s < cap; s += kSmemThreads)
+    for (uint32_t s = threadIdx.x; s < span; s += kSmemThreads)
       cnt += (*reinterpret_cast<const unsigned long long*>(table + s * SB) & kOccupied) ? 1u : 0u;
     uint32_t excl, total;
     Scan(st.scan).ExclusiveSum(cnt, excl, total);
     if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
     __syncthreads();
     uint64_t pos = st.base + excl;
-    const uint32_t pid = (uint32_t)(p % oa.np_out);
-    for (uint32_t s = threadIdx.x; s < cap; s += kSmemThreads) {
+    for (uint32_t s = threadIdx.x; s < span; s += kSmemThreads) {
       char* sp = table + s * SB;
       const uint64_t k0 = *reinterpret_cast<const unsigned long long*>(sp);
       if (!(k0 & kOccupied)) continue;
@@ -844,7 +968,14 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
       v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
       v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
-      v.pid = pid;
+      // the slot's partition: last p in [first, last) with P[p] - P0 <= s
+      int lo = first, hi = last;
+      while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (__ldg(a.P + mid) - P0 <= s) lo = mid;
+        else hi = mid;
+      }
+      v.pid = (uint32_t)(lo % oa.np_out);
       uint4* z = reinterpret_cast<uint4*>(sp);  // clean-on-extract
 #pragma unroll
       for (uint32_t q = 0; q < SB / 16; ++q) z[q] = make_uint4(0, 0, 0, 0);
@@ -980,14 +1111,14 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-// CTAs per SM of the on-chip kernel (1, 2 or 4; env DBG_SMEM_CTAS, default 4):
+// CTAs per SM of the on-chip kernel (1, 2 or 4; env DBG_SMEM_CTAS, default 1):
 // several CTAs overlap one partition's load/scan/extract latencies with
 // another's hashing; the table per CTA shrinks accordingly.
 static int smem_ctas() {
   static int v = [] {
     const char* e = getenv("DBG_SMEM_CTAS");
-    const int x = e ? atoi(e) : 4;
-    return (x == 1 || x == 2 || x == 4) ? x : 4;
+    const int x = e ? atoi(e) : 1;
+    return (x == 1 || x == 2 || x == 4) ? x : 1;
   }();
   return v;
 }
@@ -1034,14 +1165,21 @@ static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_
   }
 }
 
+extern "C" uint64_t dbg_smem_workspace_bytes(const dbg_params* prm) {
+  if (!prm) return 0;
+  const uint64_t n = (uint64_t)fine_partitions(prm);
+  return 8 * (n + 1) + 4 * (n + 2) + 16 + 64;
+}
+
 extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
-                                               uint64_t* d_work, dbg_vertex* d_out, uint64_t out_cap,
-                                               uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
-                                               cudaStream_t stream) {
+                                               void* d_work, uint64_t work_bytes, dbg_vertex* d_out,
+                                               uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
+                                               uint32_t* d_status, cudaStream_t stream) {
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !part->d_n_kmers || !d_work ||
       !d_n_out || !d_stats || !d_status || (out_cap && !d_out))
     return DBG_EINVAL;
   if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
+  if (work_bytes < dbg_smem_workspace_bytes(prm)) return DBG_EINVAL;
   SmemArgs a;
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
@@ -1050,7 +1188,11 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   a.k = prm->k;
   a.ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   a.slots = dbg_smem_table_slots(prm);
-  (void)d_work;  // reserved (static partition schedule)
+  char* ws = static_cast<char*>(d_work);
+  a.P = reinterpret_cast<uint64_t*>(ws);
+  a.n_groups = reinterpret_cast<unsigned long long*>(ws + 8 * ((uint64_t)a.n_fine + 1));
+  a.gfirst = reinterpret_cast<uint32_t*>(ws + 8 * ((uint64_t)a.n_fine + 1) + 16);
+  smem_plan_kernel<<<1, kPlanThreads, 0, stream>>>(a);
   OutArgs oa;
   oa.np_out = (uint32_t)prm->num_partitions;
   oa.out = d_out;

@@ -99,7 +99,6 @@ class DbgBuilder:
         self.d_staged = torch.zeros(1, **i64)
         self.d_tab_off = torch.zeros(NP + 1, **i64)
         self.d_status = torch.zeros(1, dtype=torch.int32, device=dev)
-        self.d_work = torch.zeros(1, **i64)
         self.d_n_out = torch.zeros(1, **i64)
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
@@ -262,8 +261,10 @@ class DbgBuilder:
     def _step2(self, stream) -> None:
         if self.mode == "smem":
             ev = self._mark("step2_smem", stream)
-            _lib.dbg_build_subgraphs_smem(self.prm, self.part_set(True), self.d_work, self.out, self.out_cap(),
-                                          self.d_n_out, self.d_stats, self.d_status, stream)
+            wsb = _lib.dbg_smem_workspace_bytes(self.prm)
+            self.work = _grow(self.work, wsb, torch.uint8, self.device)
+            _lib.dbg_build_subgraphs_smem(self.prm, self.part_set(True), self.work, self.work.numel(), self.out,
+                                          self.out_cap(), self.d_n_out, self.d_stats, self.d_status, stream)
             self._done(ev, stream)
         if self.mode == "fused":
             ev = self._mark("step2", stream)
@@ -337,9 +338,11 @@ class DbgBuilder:
 
 
 def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
-                fill: float = 0.4) -> int:
-    """Refinement F so that an average fine partition's table (Property-1 capacity) fills
-    about `fill` of one SM's shared-memory table (dbg_smem_table_slots)."""
+                fill: float = 1.0 / 16) -> int:
+    """Refinement F so that an average fine partition's table (Property-1 capacity) is about
+    `fill` of one CTA's shared-memory table (dbg_smem_table_slots): minimizer skew (PAPER.md
+    Fig. 6) makes the largest partitions ~20x the mean, and small partitions are
+    packed into groups on chip anyway."""
     prm = _lib.params(k, p, num_partitions, lam, alpha)
     slots = _lib.dbg_smem_table_slots(prm)
     per_part = max(1.0, fill * slots / max(lam / (4 * alpha), 1e-9))

@@ -7,7 +7,7 @@ from paper_conf_icdcs_qiul17_b200 import DbgBuilder, encode_reads
 
 name = sys.argv[1] if len(sys.argv) > 1 else "ecoli"
 rs = make_config(name)
-for refine in (1, 32, 256, 2048):
+for refine in (1, 32, 256, 1024):
     b = DbgBuilder(rs.k, rs.p, rs.num_partitions, refine=refine)
     d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
     b.msp(d_bases, d_off)
