@@ -687,9 +687,11 @@ __device__ __forceinline__ uint32_t smem_hash(u128 code) {
   return smem_hash((uint64_t)((uint64_t)code ^ ((uint64_t)(code >> 64) * 0xc2b2ae3d27d4eb4full)));
 }
 
-// Insert/update of one occurrence in a shared-memory table of cap slots.
+// Insert/update of one occurrence in a shared-memory table of cap slots; the
+// inserting thread also records the (fine) partition id in the slot's spare
+// field word 5, read back at extraction.
 template <typename Code>
-__device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code, int o, int i) {
+__device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code, int o, int i, uint32_t pid) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   typedef KeyOf<Code> KO;
   const typename KO::T want = KO::make(code);
@@ -705,6 +707,7 @@ __device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code
     }
     if (KO::empty(cur) || KO::same(cur, want)) {
       uint32_t* fields = reinterpret_cast<uint32_t*>(kp + SmemSlot<KW>::kFieldOff);
+      if (KO::empty(cur)) fields[5] = pid;
       smem_count(fields, o < 4 ? o : 8);
       if (i >= 0) smem_count(fields, 4 + i);
       return true;
@@ -910,6 +913,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         int n = w[0] & 255u, hl = (w[0] >> 8) & 1u, hr = (w[0] >> 9) & 1u;
         char* tab = table + (uint64_t)st.t0[r] * SB;
         uint32_t cap = st.cap[r];
+        uint32_t pid = w[0] >> 10;
         Code fwd, rc;
         kmer_at(w, hl + t, K, R, fwd, rc);
         for (uint32_t kid = k0;;) {
@@ -917,9 +921,9 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1) : -1;
           const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K) : -1;
           if (fwd < rc) {  // odd K: never equal (reading C); edges in the canonical orientation (reading J)
-            ok &= smem_upsert<Code>(tab, cap, fwd, succ >= 0 ? succ : 4, pred);
+            ok &= smem_upsert<Code>(tab, cap, fwd, succ >= 0 ? succ : 4, pred, pid);
           } else {
-            ok &= smem_upsert<Code>(tab, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1);
+            ok &= smem_upsert<Code>(tab, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1, pid);
           }
           if (++kid >= k1) break;
           if (++t < n) {  // next K-mer of the same record: roll one base
@@ -935,6 +939,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             hr = (w[0] >> 9) & 1u;
             tab = table + (uint64_t)st.t0[r] * SB;
             cap = st.cap[r];
+            pid = w[0] >> 10;
             kmer_at(w, hl, K, R, fwd, rc);
           }
         }
@@ -968,14 +973,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
       v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
       v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
-      // the slot's partition: last p in [first, last) with P[p] - P0 <= s
-      int lo = first, hi = last;
-      while (hi - lo > 1) {
-        const int mid = (lo + hi) >> 1;
-        if (__ldg(a.P + mid) - P0 <= s) lo = mid;
-        else hi = mid;
-      }
-      v.pid = (uint32_t)(lo % oa.np_out);
+      v.pid = f[5] % oa.np_out;  // fine pid recorded by the inserting thread
       uint4* z = reinterpret_cast<uint4*>(sp);  // clean-on-extract
 #pragma unroll
       for (uint32_t q = 0; q < SB / 16; ++q) z[q] = make_uint4(0, 0, 0, 0);

@@ -192,8 +192,10 @@ class DbgBuilder:
                 self.caps[self.caps <= _lib.dbg_smem_table_slots(self.prm)] = 0
             self._caps_key = key
         if self.mode == "smem":
+            ev = self._mark("plan", stream)
             _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, _lib.dbg_smem_table_slots(self.prm),
                                       self.d_tab_off, stream)
+            self._done(ev, stream)
         self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
         self.tab_host[1:] = np.cumsum(self.caps)
         if self.mode == "fused":
