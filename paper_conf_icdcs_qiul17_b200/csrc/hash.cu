@@ -124,22 +124,26 @@ struct KeyOf<u128> {
 
 // ----- K-mer decoding from a record held in shared memory (dbg.h layout)
 
-__device__ __forceinline__ uint32_t rec_word(const uint32_t* w, int q, int R) { return q < R ? w[q] : 0u; }
+// Record words may be staged with a stride (word q at w[q * stride]).
+__device__ __forceinline__ uint32_t rec_word(const uint32_t* w, int q, int R, int stride = 1) {
+  return q < R ? w[q * stride] : 0u;
+}
 
-__device__ __forceinline__ uint32_t rec_base(const uint32_t* w, int i) {
-  return (w[1 + (i >> 4)] >> (30 - 2 * (i & 15))) & 3u;
+__device__ __forceinline__ uint32_t rec_base(const uint32_t* w, int i, int stride = 1) {
+  return (w[(1 + (i >> 4)) * stride] >> (30 - 2 * (i & 15))) & 3u;
 }
 
 // The 64 bits of the record's base string that start at base b.
-__device__ __forceinline__ uint64_t rec_bits64(const uint32_t* w, int b, int R) {
+__device__ __forceinline__ uint64_t rec_bits64(const uint32_t* w, int b, int R, int stride = 1) {
   const int q = 1 + (b >> 4), off = 2 * (b & 15);
-  const uint64_t hi = ((uint64_t)rec_word(w, q, R) << 32) | rec_word(w, q + 1, R);
+  const uint64_t hi = ((uint64_t)rec_word(w, q, R, stride) << 32) | rec_word(w, q + 1, R, stride);
   if (off == 0) return hi;
-  return (hi << off) | (rec_word(w, q + 2, R) >> (32 - off));
+  return (hi << off) | (rec_word(w, q + 2, R, stride) >> (32 - off));
 }
 
-__device__ __forceinline__ void kmer_at(const uint32_t* w, int b, int K, int R, uint64_t& fwd, uint64_t& rc) {
-  fwd = rec_bits64(w, b, R) >> (64 - 2 * K);
+__device__ __forceinline__ void kmer_at(const uint32_t* w, int b, int K, int R, uint64_t& fwd, uint64_t& rc,
+                                        int stride = 1) {
+  fwd = rec_bits64(w, b, R, stride) >> (64 - 2 * K);
   rc = revcomp64(fwd, K);
 }
 
@@ -151,8 +155,9 @@ __device__ __forceinline__ u128 revcomp128(u128 x, int k) {
   return (((u128)a << 64) | (u128)b) >> (128 - 2 * k);
 }
 
-__device__ __forceinline__ void kmer_at(const uint32_t* w, int b, int K, int R, u128& fwd, u128& rc) {
-  const uint64_t hi = rec_bits64(w, b, R), lo = rec_bits64(w, b + 32, R);
+__device__ __forceinline__ void kmer_at(const uint32_t* w, int b, int K, int R, u128& fwd, u128& rc,
+                                        int stride = 1) {
+  const uint64_t hi = rec_bits64(w, b, R, stride), lo = rec_bits64(w, b + 32, R, stride);
   fwd = (((u128)hi << 64) | (u128)lo) >> (128 - 2 * K);
   rc = revcomp128(fwd, K);
 }
@@ -651,16 +656,20 @@ __global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, O
 
 constexpr uint64_t kSmemMaxSlots = 65535;
 
+// Shared-memory table, structure of arrays (dense keys keep random probes
+// spread over the banks): keys[cap] (8 B, or 16 B for K > 31), then
+// fields[cap][6] u32: out0|out1, out2|out3, in0|in1, in2|in3, t_out, fine pid.
 template <int KW>
 struct SmemSlot {
-  static constexpr uint32_t kBytes = KW == 1 ? 32 : 48;  // key + 6 or 8 field words
-  static constexpr uint32_t kFieldOff = KW == 1 ? 8 : 16;
+  static constexpr uint32_t kKeyBytes = KW == 1 ? 8 : 16;
+  static constexpr uint32_t kFieldWords = 6;
+  static constexpr uint32_t kBytes = kKeyBytes + 4 * kFieldWords;
 };
 
 // T threads per CTA stage 2T records per batch.
 template <int R, int T>
 struct SmemStage {
-  uint32_t w[2 * T][R];
+  uint32_t w[R][2 * T];  // transposed: record j's word q at w[q][j] (bank-conflict-free staging)
   uint32_t t0[2 * T];   // first slot of the record's partition table in the CTA table
   uint32_t cap[2 * T];  // its capacity (0: partition off chip)
   uint32_t pre[2 * T + 1];
@@ -688,16 +697,17 @@ __device__ __forceinline__ uint32_t smem_hash(u128 code) {
 }
 
 // Insert/update of one occurrence in a shared-memory table of cap slots; the
-// inserting thread also records the (fine) partition id in the slot's spare
-// field word 5, read back at extraction.
+// inserting thread also records the (fine) partition id in field word 5,
+// read back at extraction.
 template <typename Code>
-__device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code, int o, int i, uint32_t pid) {
+__device__ __forceinline__ bool smem_upsert(char* keys, uint32_t* fld, uint32_t cap, Code code, int o, int i,
+                                            uint32_t pid) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   typedef KeyOf<Code> KO;
   const typename KO::T want = KO::make(code);
   uint32_t idx = __umulhi(smem_hash(code), cap);
   for (uint32_t pr = 0; pr < cap; ++pr) {
-    char* kp = table + idx * SmemSlot<KW>::kBytes;
+    char* kp = keys + idx * SmemSlot<KW>::kKeyBytes;
     typename KO::T cur;
     if constexpr (KW == 1) {
       cur = *reinterpret_cast<volatile unsigned long long*>(kp);
@@ -706,10 +716,10 @@ __device__ __forceinline__ bool smem_upsert(char* table, uint32_t cap, Code code
       cur = KO::cas(kp, want);  // 16-B shared-memory CAS: atomic read-or-claim
     }
     if (KO::empty(cur) || KO::same(cur, want)) {
-      uint32_t* fields = reinterpret_cast<uint32_t*>(kp + SmemSlot<KW>::kFieldOff);
-      if (KO::empty(cur)) fields[5] = pid;
-      smem_count(fields, o < 4 ? o : 8);
-      if (i >= 0) smem_count(fields, 4 + i);
+      uint32_t* f = fld + idx * SmemSlot<KW>::kFieldWords;
+      if (KO::empty(cur)) f[5] = pid;
+      smem_count(f, o < 4 ? o : 8);
+      if (i >= 0) smem_count(f, 4 + i);
       return true;
     }
     idx = idx + 1 == cap ? 0 : idx + 1;
@@ -844,18 +854,22 @@ __global__ void __launch_bounds__(kPlanThreads) smem_plan_kernel(SmemArgs a) {
 template <typename Code, int R, int kSmemThreads, int kMinCtas>
 __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  constexpr uint32_t SB = SmemSlot<KW>::kBytes;
+  constexpr uint32_t KB = SmemSlot<KW>::kKeyBytes, FW = SmemSlot<KW>::kFieldWords;
   constexpr int kRecBatch = 2 * kSmemThreads;
   typedef cub::BlockScan<uint32_t, kSmemThreads> Scan;
   extern __shared__ __align__(128) unsigned char smem[];
   SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
-  char* table = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
+  char* keys = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
+  uint32_t* fld = reinterpret_cast<uint32_t*>(keys + a.slots * KB);
   const int K = a.k;
   const int top = 2 * K - 2;
   const Code mask = ((Code)1 << (2 * K)) - 1;
   {  // the table starts clean; extraction keeps it clean
-    uint4* z = reinterpret_cast<uint4*>(table);
-    for (uint64_t q = threadIdx.x; q < a.slots * (SB / 16); q += kSmemThreads) z[q] = make_uint4(0, 0, 0, 0);
+    uint4* z = reinterpret_cast<uint4*>(keys);
+    for (uint64_t q = threadIdx.x; q < a.slots * (SmemSlot<KW>::kBytes / 16); q += kSmemThreads)
+      z[q] = make_uint4(0, 0, 0, 0);
+    uint32_t* zt = reinterpret_cast<uint32_t*>(z + a.slots * (SmemSlot<KW>::kBytes / 16));
+    for (uint64_t q = threadIdx.x; q < (a.slots * SmemSlot<KW>::kBytes % 16) / 4; q += kSmemThreads) zt[q] = 0;
   }
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
   bool ok = true;
@@ -878,16 +892,16 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
 #pragma unroll
           for (int q = 0; q < R / 4; ++q) {
             const uint4 x = __ldcs(src + q);  // streamed once
-            st.w[j][4 * q] = x.x;
-            st.w[j][4 * q + 1] = x.y;
-            st.w[j][4 * q + 2] = x.z;
-            st.w[j][4 * q + 3] = x.w;
+            st.w[4 * q][j] = x.x;
+            st.w[4 * q + 1][j] = x.y;
+            st.w[4 * q + 2][j] = x.z;
+            st.w[4 * q + 3][j] = x.w;
           }
-          const uint32_t pid = st.w[j][0] >> 10;
+          const uint32_t pid = st.w[0][j] >> 10;
           const uint64_t pp = a.P[pid], pc = a.P[pid + 1] - pp;
           st.t0[j] = (uint32_t)(pp - P0);
           st.cap[j] = (uint32_t)pc;
-          cnt[v] = pc ? st.w[j][0] & 255u : 0u;  // off-chip partition: skipped here
+          cnt[v] = pc ? st.w[0][j] & 255u : 0u;  // off-chip partition: skipped here
         }
       }
       uint32_t excl[2], total;
@@ -908,22 +922,24 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         }
         int r = lo;
         while (st.pre[r + 1] == st.pre[r]) ++r;  // skip records that contribute nothing
+        constexpr int S = kRecBatch;  // staging stride
         int t = (int)(k0 - st.pre[r]);
-        const uint32_t* w = st.w[r];
+        const uint32_t* w = &st.w[0][r];
         int n = w[0] & 255u, hl = (w[0] >> 8) & 1u, hr = (w[0] >> 9) & 1u;
-        char* tab = table + (uint64_t)st.t0[r] * SB;
+        char* tk = keys + (uint64_t)st.t0[r] * KB;
+        uint32_t* tf = fld + (uint64_t)st.t0[r] * FW;
         uint32_t cap = st.cap[r];
         uint32_t pid = w[0] >> 10;
         Code fwd, rc;
-        kmer_at(w, hl + t, K, R, fwd, rc);
+        kmer_at(w, hl + t, K, R, fwd, rc, S);
         for (uint32_t kid = k0;;) {
           const int b = hl + t;
-          const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1) : -1;
-          const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K) : -1;
+          const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1, S) : -1;
+          const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K, S) : -1;
           if (fwd < rc) {  // odd K: never equal (reading C); edges in the canonical orientation (reading J)
-            ok &= smem_upsert<Code>(tab, cap, fwd, succ >= 0 ? succ : 4, pred, pid);
+            ok &= smem_upsert<Code>(tk, tf, cap, fwd, succ >= 0 ? succ : 4, pred, pid);
           } else {
-            ok &= smem_upsert<Code>(tab, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1, pid);
+            ok &= smem_upsert<Code>(tk, tf, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1, pid);
           }
           if (++kid >= k1) break;
           if (++t < n) {  // next K-mer of the same record: roll one base
@@ -933,14 +949,15 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             do ++r;
             while (st.pre[r + 1] == st.pre[r]);
             t = 0;
-            w = st.w[r];
+            w = &st.w[0][r];
             n = w[0] & 255u;
             hl = (w[0] >> 8) & 1u;
             hr = (w[0] >> 9) & 1u;
-            tab = table + (uint64_t)st.t0[r] * SB;
+            tk = keys + (uint64_t)st.t0[r] * KB;
+            tf = fld + (uint64_t)st.t0[r] * FW;
             cap = st.cap[r];
             pid = w[0] >> 10;
-            kmer_at(w, hl, K, R, fwd, rc);
+            kmer_at(w, hl, K, R, fwd, rc, S);
           }
         }
       }
@@ -950,33 +967,34 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
     // scan sizes the group's output, one global atomic reserves it
     uint32_t cnt = 0;
     for (uint32_t s = threadIdx.x; s < span; s += kSmemThreads)
-      cnt += (*reinterpret_cast<const unsigned long long*>(table + s * SB) & kOccupied) ? 1u : 0u;
+      cnt += (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied) ? 1u : 0u;
     uint32_t excl, total;
     Scan(st.scan).ExclusiveSum(cnt, excl, total);
     if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
     __syncthreads();
     uint64_t pos = st.base + excl;
     for (uint32_t s = threadIdx.x; s < span; s += kSmemThreads) {
-      char* sp = table + s * SB;
-      const uint64_t k0 = *reinterpret_cast<const unsigned long long*>(sp);
+      unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+      const uint64_t k0 = kp[0];
       if (!(k0 & kOccupied)) continue;
-      const uint32_t* f = reinterpret_cast<const uint32_t*>(sp + SmemSlot<KW>::kFieldOff);
+      uint32_t* f = fld + s * FW;
       dbg_vertex v;
       if (KW == 1) {
         v.kmer_hi = 0;
         v.kmer_lo = k0 & kCodeMask;
       } else {
         v.kmer_hi = k0 & kCodeMask;
-        v.kmer_lo = *reinterpret_cast<const unsigned long long*>(sp + 8);
+        v.kmer_lo = kp[1];
       }
       const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
       v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
       v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
       v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
       v.pid = f[5] % oa.np_out;  // fine pid recorded by the inserting thread
-      uint4* z = reinterpret_cast<uint4*>(sp);  // clean-on-extract
+      kp[0] = 0;  // clean-on-extract
+      if (KW == 2) kp[1] = 0;
 #pragma unroll
-      for (uint32_t q = 0; q < SB / 16; ++q) z[q] = make_uint4(0, 0, 0, 0);
+      for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
       if (pos < oa.out_cap) oa.out[pos] = v;
       else atomicOr(oa.status, kStatusNoSpace);
       ++pos;
