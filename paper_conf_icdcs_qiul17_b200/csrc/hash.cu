@@ -864,12 +864,10 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   const int K = a.k;
   const int top = 2 * K - 2;
   const Code mask = ((Code)1 << (2 * K)) - 1;
-  {  // the table starts clean; extraction keeps it clean
+  {  // the table starts clean; extraction keeps it clean (slots is a multiple of 64)
     uint4* z = reinterpret_cast<uint4*>(keys);
-    for (uint64_t q = threadIdx.x; q < a.slots * (SmemSlot<KW>::kBytes / 16); q += kSmemThreads)
+    for (uint64_t q = threadIdx.x; q < a.slots * SmemSlot<KW>::kBytes / 16; q += kSmemThreads)
       z[q] = make_uint4(0, 0, 0, 0);
-    uint32_t* zt = reinterpret_cast<uint32_t*>(z + a.slots * (SmemSlot<KW>::kBytes / 16));
-    for (uint64_t q = threadIdx.x; q < (a.slots * SmemSlot<KW>::kBytes % 16) / 4; q += kSmemThreads) zt[q] = 0;
   }
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
   bool ok = true;
