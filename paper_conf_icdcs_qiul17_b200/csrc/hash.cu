@@ -666,13 +666,14 @@ struct SmemSlot {
   static constexpr uint32_t kBytes = kKeyBytes + 4 * kFieldWords;
 };
 
-// T threads per CTA stage 2T records per batch.
+// T threads per CTA stage RB(T) records per batch.
+__host__ __device__ constexpr int smem_rec_batch(int T) { return T >= 1024 ? T : 2 * T; }
 template <int R, int T>
 struct SmemStage {
-  uint32_t w[R][2 * T];  // transposed: record j's word q at w[q][j] (bank-conflict-free staging)
-  uint32_t t0[2 * T];   // first slot of the record's partition table in the CTA table
-  uint32_t cap[2 * T];  // its capacity (0: partition off chip)
-  uint32_t pre[2 * T + 1];
+  uint32_t w[R][smem_rec_batch(T)];  // transposed: record j's word q at w[q][j] (bank-conflict-free)
+  uint32_t t0[smem_rec_batch(T)];    // first slot of the record's partition table in the CTA table
+  uint32_t cap[smem_rec_batch(T)];   // its capacity (0: partition off chip)
+  uint32_t pre[smem_rec_batch(T) + 1];
   typename cub::BlockScan<uint32_t, T>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, T>::TempStorage red;
   unsigned long long base;
@@ -855,7 +856,8 @@ template <typename Code, int R, int kSmemThreads, int kMinCtas>
 __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   constexpr uint32_t KB = SmemSlot<KW>::kKeyBytes, FW = SmemSlot<KW>::kFieldWords;
-  constexpr int kRecBatch = 2 * kSmemThreads;
+  constexpr int kRecBatch = smem_rec_batch(kSmemThreads);
+  constexpr int kRPT = kRecBatch / kSmemThreads;  // records per thread per batch
   typedef cub::BlockScan<uint32_t, kSmemThreads> Scan;
   extern __shared__ __align__(128) unsigned char smem[];
   SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
@@ -880,10 +882,10 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
     for (uint64_t rb = 0; rb < nrec; rb += kRecBatch) {
       const int nb = (int)min((uint64_t)kRecBatch, nrec - rb);
       __syncthreads();  // staging free; previous extraction (table clean) complete
-      uint32_t cnt[2];
+      uint32_t cnt[kRPT];
 #pragma unroll
-      for (int v = 0; v < 2; ++v) {
-        const int j = 2 * threadIdx.x + v;
+      for (int v = 0; v < kRPT; ++v) {
+        const int j = kRPT * threadIdx.x + v;
         cnt[v] = 0;
         if (j < nb) {
           const uint4* src = reinterpret_cast<const uint4*>(a.records + (r0 + rb + j) * R);
@@ -902,10 +904,10 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           cnt[v] = pc ? st.w[0][j] & 255u : 0u;  // off-chip partition: skipped here
         }
       }
-      uint32_t excl[2], total;
+      uint32_t excl[kRPT], total;
       Scan(st.scan).ExclusiveSum(cnt, excl, total);
-      st.pre[2 * threadIdx.x] = excl[0];
-      st.pre[2 * threadIdx.x + 1] = excl[1];
+#pragma unroll
+      for (int v = 0; v < kRPT; ++v) st.pre[kRPT * threadIdx.x + v] = excl[v];
       if (threadIdx.x == 0) st.pre[kRecBatch] = total;
       __syncthreads();
       // this thread's contiguous run of K-mers [k0, k1)
@@ -1125,14 +1127,16 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-// CTAs per SM of the on-chip kernel (1, 2 or 4; env DBG_SMEM_CTAS, default 1):
+// CTAs per SM of the on-chip kernel (env DBG_SMEM_CTAS):
 // several CTAs overlap one partition's load/scan/extract latencies with
 // another's hashing; the table per CTA shrinks accordingly.
+// 0 = one CTA of 1024 threads per SM (the default), 1/2/4 = that many CTAs of
+// 512/256/128 threads.
 static int smem_ctas() {
   static int v = [] {
     const char* e = getenv("DBG_SMEM_CTAS");
-    const int x = e ? atoi(e) : 1;
-    return (x == 1 || x == 2 || x == 4) ? x : 1;
+    const int x = e ? atoi(e) : 0;
+    return (x == 0 || x == 1 || x == 2 || x == 4) ? x : 0;
   }();
   return v;
 }
@@ -1148,6 +1152,7 @@ static uint64_t smem_slots_for(int k, int ctas) {
 static uint64_t smem_slots(int k, int ctas) {
   const bool r4 = record_words(k) == 4;
   switch (ctas) {
+    case 0: return r4 ? smem_slots_for<4, 1024>(k, 1) : smem_slots_for<8, 1024>(k, 1);
     case 1: return r4 ? smem_slots_for<4, 512>(k, 1) : smem_slots_for<8, 512>(k, 1);
     case 2: return r4 ? smem_slots_for<4, 256>(k, 2) : smem_slots_for<8, 256>(k, 2);
     default: return r4 ? smem_slots_for<4, 128>(k, 4) : smem_slots_for<8, 128>(k, 4);
@@ -1173,6 +1178,7 @@ static cudaError_t launch_smem_t(const SmemArgs& a, const OutArgs& oa, cudaStrea
 template <typename Code, int R>
 static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
   switch (smem_ctas()) {
+    case 0: return launch_smem_t<Code, R, 1024, 1>(a, oa, stream);
     case 1: return launch_smem_t<Code, R, 512, 1>(a, oa, stream);
     case 2: return launch_smem_t<Code, R, 256, 2>(a, oa, stream);
     default: return launch_smem_t<Code, R, 128, 4>(a, oa, stream);
