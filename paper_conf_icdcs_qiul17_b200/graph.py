@@ -340,7 +340,7 @@ class DbgBuilder:
 
 
 def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
-                fill: float = 1.0 / 16) -> int:
+                fill: float = 0.25) -> int:
     """Refinement F so that an average fine partition's table (Property-1 capacity) is about
     `fill` of one CTA's shared-memory table (dbg_smem_table_slots): minimizer skew (PAPER.md
     Fig. 6) makes the largest partitions ~20x the mean, and small partitions are
