@@ -145,7 +145,7 @@ DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kme
                           uint64_t* d_table_offset, cudaStream_t stream);
 
 /* ---- a5-a7 on-chip: Step 2 in shared memory (the hot path) ---------------
- * Every fine partition whose table (capacity from Property 1, Sec. IV-A
+ * Every fine partition in [pid_begin, pid_end) whose table (capacity from Property 1, Sec. IV-A
  * P:L783-788) fits one CTA's shared memory -- at most dbg_smem_table_slots()
  * slots -- is built and extracted on chip: consecutive such partitions are
  * grouped so that a group's tables fill one CTA's table space; the CTA hashes
@@ -159,9 +159,10 @@ DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kme
 DBG_API uint64_t dbg_smem_table_slots(const dbg_params* prm);
 DBG_API uint64_t dbg_smem_workspace_bytes(const dbg_params* prm);
 DBG_API dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
-                                    void* d_work, uint64_t work_bytes, dbg_vertex* d_out,
-                                    uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
-                                    uint32_t* d_status, cudaStream_t stream);
+                                    int32_t pid_begin, int32_t pid_end, void* d_work,
+                                    uint64_t work_bytes, dbg_vertex* d_out, uint64_t out_cap,
+                                    uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
+                                    cudaStream_t stream);
 /* As dbg_table_plan, but partitions whose capacity is <= smem_slots get
  * capacity 0 (they are built on chip), so resident tables cover only the rest. */
 DBG_API dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t smem_slots,

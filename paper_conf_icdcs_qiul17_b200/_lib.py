@@ -63,7 +63,7 @@ SIGNATURES = {
     "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P]),
     "dbg_smem_table_slots": (_U64, [_PRM]),
     "dbg_smem_workspace_bytes": (_U64, [_PRM]),
-    "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _P, _U64, _P, _U64, _P, _P, _P, _P]),
+    "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _P, _U64, _P, _P, _P, _P]),
     "dbg_table_plan_split": (ctypes.c_int, [_PRM, _P, _U64, _P, _P]),
     "dbg_subgraph_ring_bytes": (_U64, [_PRM, _U64, _U64]),
     "dbg_subgraph_workspace_bytes": (_U64, [_PRM, _I32, _U64, _U64]),
@@ -197,11 +197,11 @@ def dbg_smem_workspace_bytes(prm) -> int:
     return load().dbg_smem_workspace_bytes(ctypes.byref(prm))
 
 
-def dbg_build_subgraphs_smem(prm, part, d_work, work_bytes: int, d_out, out_cap: int, d_n_out, d_stats, d_status,
-                             stream=None) -> None:
+def dbg_build_subgraphs_smem(prm, part, pid_begin: int, pid_end: int, d_work, work_bytes: int, d_out, out_cap: int,
+                             d_n_out, d_stats, d_status, stream=None) -> None:
     _check("dbg_build_subgraphs_smem", load().dbg_build_subgraphs_smem(
-        ctypes.byref(prm), ctypes.byref(part), _ptr(d_work), work_bytes, _ptr(d_out), out_cap, _ptr(d_n_out),
-        _ptr(d_stats), _ptr(d_status), _stream(stream)))
+        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_work), work_bytes, _ptr(d_out), out_cap,
+        _ptr(d_n_out), _ptr(d_stats), _ptr(d_status), _stream(stream)))
 
 
 def dbg_table_plan_split(prm, d_n_kmers, smem_slots: int, d_table_offset, stream=None) -> None:

@@ -732,11 +732,11 @@ struct SmemArgs {
   const uint32_t* records;
   const uint64_t* rec_off;
   const uint64_t* n_kmers;
-  int n_fine, k;
+  int pid0, n_fine, k;  // fine partitions [pid0, pid0 + n_fine)
   double ratio;      // lambda / (4 alpha)
   uint64_t slots;    // table slots that fit one CTA
-  uint64_t* P;       // [n_fine + 1] prefix of on-chip capacities (0 for partitions off chip)
-  uint32_t* gfirst;  // [n_fine + 2] first partition of each group
+  uint64_t* P;       // [n_fine + 1] prefix of on-chip capacities (0 for partitions off chip), local index
+  uint32_t* gfirst;  // [n_fine + 2] first (absolute) partition of each group
   unsigned long long* n_groups;
 };
 
@@ -773,7 +773,7 @@ __global__ void __launch_bounds__(kPlanThreads) smem_plan_kernel(SmemArgs a) {
 #pragma unroll
     for (int q = 0; q < kPlanItems; ++q) {
       const int p = base + threadIdx.x * kPlanItems + q;
-      cap[q] = p < a.n_fine ? smem_cap(a, a.n_kmers[p]) : 0;
+      cap[q] = p < a.n_fine ? smem_cap(a, a.n_kmers[a.pid0 + p]) : 0;
     }
     unsigned long long tot;
     Scan(tmp).ExclusiveSum(cap, pre, tot);
@@ -834,7 +834,7 @@ __global__ void __launch_bounds__(kPlanThreads) smem_plan_kernel(SmemArgs a) {
 #pragma unroll
     for (int q = 0; q < kPlanItems; ++q) {
       const int p = base + threadIdx.x * kPlanItems + q;
-      if (p < a.n_fine && flag[q]) a.gfirst[cg + gpre[q]] = (uint32_t)p;
+      if (p < a.n_fine && flag[q]) a.gfirst[cg + gpre[q]] = (uint32_t)(a.pid0 + p);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -845,7 +845,7 @@ __global__ void __launch_bounds__(kPlanThreads) smem_plan_kernel(SmemArgs a) {
   }
   if (threadIdx.x == 0) {
     a.P[a.n_fine] = carry_p;
-    a.gfirst[carry_g] = (uint32_t)a.n_fine;
+    a.gfirst[carry_g] = (uint32_t)(a.pid0 + a.n_fine);
     *a.n_groups = carry_g;
   }
 }
@@ -876,7 +876,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   const uint64_t n_groups = *a.n_groups;
   for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
     const int first = (int)a.gfirst[g], last = (int)a.gfirst[g + 1];
-    const uint64_t P0 = a.P[first], span = a.P[last] - P0;
+    const uint64_t P0 = a.P[first - a.pid0], span = a.P[last - a.pid0] - P0;
     if (span == 0) continue;  // nothing on chip in this group
     const uint64_t r0 = a.rec_off[first], nrec = a.rec_off[last] - r0;
     for (uint64_t rb = 0; rb < nrec; rb += kRecBatch) {
@@ -897,7 +897,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             st.w[4 * q + 2][j] = x.z;
             st.w[4 * q + 3][j] = x.w;
           }
-          const uint32_t pid = st.w[0][j] >> 10;
+          const uint32_t pid = (st.w[0][j] >> 10) - a.pid0;
           const uint64_t pp = a.P[pid], pc = a.P[pid + 1] - pp;
           st.t0[j] = (uint32_t)(pp - P0);
           st.cap[j] = (uint32_t)pc;
@@ -1192,19 +1192,23 @@ extern "C" uint64_t dbg_smem_workspace_bytes(const dbg_params* prm) {
 }
 
 extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
-                                               void* d_work, uint64_t work_bytes, dbg_vertex* d_out,
-                                               uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
-                                               uint32_t* d_status, cudaStream_t stream) {
+                                               int32_t pid_begin, int32_t pid_end, void* d_work,
+                                               uint64_t work_bytes, dbg_vertex* d_out, uint64_t out_cap,
+                                               uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
+                                               cudaStream_t stream) {
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !part->d_n_kmers || !d_work ||
       !d_n_out || !d_stats || !d_status || (out_cap && !d_out))
     return DBG_EINVAL;
   if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
+  if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
+  if (pid_begin == pid_end) return DBG_OK;
   if (work_bytes < dbg_smem_workspace_bytes(prm)) return DBG_EINVAL;
   SmemArgs a;
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
   a.n_kmers = part->d_n_kmers;
-  a.n_fine = fine_partitions(prm);
+  a.pid0 = pid_begin;
+  a.n_fine = pid_end - pid_begin;
   a.k = prm->k;
   a.ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   a.slots = dbg_smem_table_slots(prm);

@@ -83,6 +83,7 @@ class DbgBuilder:
         self.np = num_partitions * self.refine       # fine partitions the device works on
         self.group_slots = int(group_slots)  # fused mode: table slots per ring group (L2 sizing)
         self.total_slots = 0
+        self.owned = (0, self.np)  # fine partitions this builder hashes (multi-GPU: a shard)
         self.prm = _lib.params(k, p, num_partitions, lam, alpha, self.refine)
         self.device = torch.device(device)
         _lib.load()
@@ -177,11 +178,36 @@ class DbgBuilder:
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
         self._done(ev, stream)
 
+    def load_exchanged(self, received: torch.Tensor, n_received: int, global_records: np.ndarray,
+                       global_kmers: np.ndarray, owned: tuple[int, int], stream=None) -> None:
+        """Multi-GPU: after the record exchange, make this builder's partition set describe only
+        the owned fine partitions [lo, hi) (records received from every rank, scattered into
+        partition order by dbg_msp_partition pass 2; sizes summed over ranks)."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        lo, hi = owned
+        self.owned = (lo, hi)
+        rec = np.zeros(self.np, dtype=np.int64)
+        kmr = np.zeros(self.np, dtype=np.int64)
+        rec[lo:hi] = global_records[lo:hi]
+        kmr[lo:hi] = global_kmers[lo:hi]
+        off = np.zeros(self.np + 1, dtype=np.int64)
+        off[1:] = np.cumsum(rec)
+        assert int(off[-1]) == n_received, (int(off[-1]), n_received)
+        self.part_records, self.part_kmers = rec, kmr
+        with torch.cuda.stream(stream):
+            self.d_n_records.copy_(torch.from_numpy(rec), non_blocking=True)
+            self.d_n_kmers.copy_(torch.from_numpy(kmr), non_blocking=True)
+            self.d_rec_off.copy_(torch.from_numpy(off), non_blocking=True)
+            self.d_staged.fill_(n_received)
+        self.staging = received
+        self.records = _grow(self.records, n_received * self.rec_words, torch.int32, self.device, 1.05)
+        _lib.dbg_msp_partition(self.prm, 1, 1, self.d_rec_off, 0, self.part_set(True), stream)
+
     # ------------------------------------------------------------------ a5
     def plan(self, stream=None) -> list[tuple[int, int]]:
         stream = stream or torch.cuda.current_stream(self.device)
         _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, stream)
-        key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha, self.mode)
+        key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha, self.mode, self.owned)
         if self._caps_key != key:  # host copy of the same C sizing function (dbg_table_capacity)
             nz = np.nonzero(self.part_kmers)[0]
             self.caps = np.zeros(self.np, dtype=np.int64)
@@ -190,6 +216,9 @@ class DbgBuilder:
                                      dtype=np.int64)[inv]
             if self.mode == "smem":  # on-chip partitions need no global table (dbg_table_plan_split)
                 self.caps[self.caps <= _lib.dbg_smem_table_slots(self.prm)] = 0
+            lo, hi = self.owned
+            self.caps[:lo] = 0
+            self.caps[hi:] = 0
             self._caps_key = key
         if self.mode == "smem":
             ev = self._mark("plan", stream)
@@ -216,10 +245,10 @@ class DbgBuilder:
         max_slots = max(budget // self.slot_bytes, int(self.caps.max(initial=0)))
         bkey = (self._caps_key, max_slots)
         if self._batch_key != bkey:  # greedy batches of consecutive partitions (vectorised)
-            batches, b, th = [], 0, self.tab_host
-            while b < self.np:
+            batches, b, th = [], self.owned[0], self.tab_host
+            while b < self.owned[1]:
                 e = int(np.searchsorted(th, th[b] + max_slots, side="right")) - 1
-                e = min(max(e, b + 1), self.np)
+                e = min(max(e, b + 1), self.owned[1])
                 if th[e] > th[b]:
                     batches.append((b, e))
                 b = e
@@ -241,6 +270,31 @@ class DbgBuilder:
                 grown.zero_()
             self._dirty = False
         return grown
+
+    def load_exchanged(self, received: torch.Tensor, n_received: int, global_records: np.ndarray,
+                       global_kmers: np.ndarray, owned: tuple[int, int], stream=None) -> None:
+        """Multi-GPU: after the record exchange, make this builder's partition set describe only
+        the owned fine partitions [lo, hi) (records received from every rank, scattered into
+        partition order by dbg_msp_partition pass 2; sizes summed over ranks)."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        lo, hi = owned
+        self.owned = (lo, hi)
+        rec = np.zeros(self.np, dtype=np.int64)
+        kmr = np.zeros(self.np, dtype=np.int64)
+        rec[lo:hi] = global_records[lo:hi]
+        kmr[lo:hi] = global_kmers[lo:hi]
+        off = np.zeros(self.np + 1, dtype=np.int64)
+        off[1:] = np.cumsum(rec)
+        assert int(off[-1]) == n_received, (int(off[-1]), n_received)
+        self.part_records, self.part_kmers = rec, kmr
+        with torch.cuda.stream(stream):
+            self.d_n_records.copy_(torch.from_numpy(rec), non_blocking=True)
+            self.d_n_kmers.copy_(torch.from_numpy(kmr), non_blocking=True)
+            self.d_rec_off.copy_(torch.from_numpy(off), non_blocking=True)
+            self.d_staged.fill_(n_received)
+        self.staging = received
+        self.records = _grow(self.records, n_received * self.rec_words, torch.int32, self.device, 1.05)
+        _lib.dbg_msp_partition(self.prm, 1, 1, self.d_rec_off, 0, self.part_set(True), stream)
 
     # ------------------------------------------------------------------ a5-a7
     def reset_output(self, cap: int, stream=None) -> None:
@@ -265,8 +319,9 @@ class DbgBuilder:
             ev = self._mark("step2_smem", stream)
             wsb = _lib.dbg_smem_workspace_bytes(self.prm)
             self.work = _grow(self.work, wsb, torch.uint8, self.device)
-            _lib.dbg_build_subgraphs_smem(self.prm, self.part_set(True), self.work, self.work.numel(), self.out,
-                                          self.out_cap(), self.d_n_out, self.d_stats, self.d_status, stream)
+            _lib.dbg_build_subgraphs_smem(self.prm, self.part_set(True), self.owned[0], self.owned[1], self.work,
+                                          self.work.numel(), self.out, self.out_cap(), self.d_n_out, self.d_stats,
+                                          self.d_status, stream)
             self._done(ev, stream)
         if self.mode == "fused":
             ev = self._mark("step2", stream)

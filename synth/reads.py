@@ -154,14 +154,16 @@ CONFIGS = {
 }
 
 
-def make_config(name: str, scale: float = 1.0, num_partitions: int | None = None) -> ReadSet:
+def make_config(name: str, scale: float = 1.0, num_partitions: int | None = None,
+                read_seed_offset: int = 0) -> ReadSet:
     """The named configuration; ``scale`` < 1 shrinks genome and read count together
-    (same coverage, error rate and read length) for quick runs."""
+    (same coverage, error rate and read length) for quick runs; ``read_seed_offset`` draws a
+    different read set from the same genome (multi-GPU weak scaling)."""
     c = CONFIGS[name]
     G = max(int(c["genome"] * scale), c["read_len"] * 4)
     n = max(int(c["reads"] * scale), 1)
     g = genome(G, c["gseed"])
-    seq, offsets = make_reads(g, n, c["read_len"], c["error"], c["rseed"])
+    seq, offsets = make_reads(g, n, c["read_len"], c["error"], c["rseed"] + read_seed_offset)
     return ReadSet(seq, offsets, name=name, k=c["k"], p=c["p"],
                    num_partitions=num_partitions or c["np"],
                    meta=dict(genome=G, reads=n, read_len=c["read_len"], error=c["error"],

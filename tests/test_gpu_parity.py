@@ -243,3 +243,46 @@ def test_full_size_config_sampled(name):
     orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT,
                        keys=np.stack([sel["kmer_hi"], sel["kmer_lo"]], 1))
     compare_vertices(sel, orc)
+
+
+def test_sharded_path_two_logical_ranks_one_gpu():
+    """Row e on one GPU: two 'ranks' each run MSP on half of the reads, records are routed to the
+    owners of their fine partitions exactly as multi.exchange_records does (slices in partition
+    order), each owner builds its partitions -- the union equals the oracle on all reads."""
+    from paper_conf_icdcs_qiul17_b200.multi import owner_bounds, send_counts
+
+    g = genome(40_000, seed=9)
+    seq, offs = make_reads(g, 6000, 100, 0.01, seed=10)
+    rs = ReadSet(seq, offs)
+    k, p, np_, refine = 31, 11, 8, 8
+    halves = [rs.subset(0, 3000), rs.subset(3000, 6000)]
+    bs = []
+    for h in halves:
+        b = DbgBuilder(k, p, np_, refine=refine)
+        d_bases, d_off = b.upload(encode_reads(h.seq), h.offsets)
+        b.msp(d_bases, d_off)
+        bs.append(b)
+    n_fine = bs[0].np
+    bounds = owner_bounds(n_fine, 2)
+    g_rec = bs[0].part_records + bs[1].part_records
+    g_kmr = bs[0].part_kmers + bs[1].part_kmers
+    R = bs[0].rec_words
+    outs = []
+    for owner in range(2):
+        parts = []
+        for b in bs:
+            sc = np.concatenate([[0], np.cumsum(send_counts(b.part_records, bounds))])
+            parts.append(b.records[sc[owner] * R: sc[owner + 1] * R])
+        recv = torch.cat(parts)
+        n = recv.numel() // R
+        ob = DbgBuilder(k, p, np_, refine=refine)
+        ob.load_exchanged(recv, n, g_rec, g_kmr, (int(bounds[owner]), int(bounds[owner + 1])))
+        ob.plan()
+        ob.reset_output(max(n * 16, 1024))
+        ob.step2()
+        assert _lib.dbg_sync_status(ob.d_status) == 0
+        outs.append(ob.vertices(sort=False))
+    allv = np.concatenate(outs)
+    allv = allv[np.lexsort((allv["kmer_lo"], allv["kmer_hi"]))]
+    orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT)
+    compare_vertices(allv, orc)
