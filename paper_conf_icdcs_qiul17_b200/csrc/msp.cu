@@ -34,7 +34,7 @@
 namespace dbg {
 
 constexpr int kMspThreads = 128;
-constexpr int kMaxDesc = 12;             // descriptors per thread between flushes
+constexpr int kMaxDesc = 40;             // descriptors per thread between flushes (>= 34)
 constexpr int kSmemHistMaxNp = 8192;
 
 // Unsigned 64-bit division by an invariant integer (Granlund & Montgomery
@@ -80,28 +80,27 @@ struct MspArgs {
 template <typename CT>
 struct MspSmem {
   // row[t * kMspThreads + tid], t < w: the van Herk block (in place)
-  // desc_se[d * kMspThreads + tid] = start | end << 32; desc_m = minimizer
+  // desc_e[d * kMspThreads + tid]: last K-mer of descriptor d (its first is the previous
+  // descriptor's last + 1, or the carried start); desc_m: its minimizer
   CT* row;
-  unsigned long long* desc_se;
-  unsigned long long* desc_m;
-  uint32_t* hist_rec;
-  uint32_t* hist_kmer;
+  uint32_t* desc_e;
+  CT* desc_m;
 };
 
 // Writes one record (dbg.h layout) for K-mers [ps, pe] of the read at stream
 // offset o, length L.
-__device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, uint64_t o, int64_t L,
-                                             int64_t ps, int64_t pe, uint32_t pid) {
+__device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, uint64_t o, int L, int ps, int pe,
+                                             uint32_t pid) {
   const uint32_t hl = ps > 0 ? 1u : 0u;  // reading H
   const uint32_t hr = pe + a.k < L ? 1u : 0u;
-  const int64_t bs = ps - hl;
-  const int64_t nb = (int64_t)hl + (pe - ps + 1) + a.k - 1 + hr;
+  const int bs = ps - (int)hl;
+  const int nb = (int)hl + (pe - ps + 1) + a.k - 1 + (int)hr;
   uint32_t w[8];
   w[0] = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
 #pragma unroll
   for (int q = 0; q < 7; q += 2) {  // two 16-base words per 64-bit window
     uint64_t v = 0;
-    const int64_t left = nb - 16 * q;
+    const int left = nb - 16 * q;
     if (q + 1 < (int)a.rec_words && left > 0) {
       v = window64(a.words, a.n_words, o + bs + 16 * q);
       if (left < 32) v &= ~(~0ull >> (2 * left));  // zero the bases past the record
@@ -114,17 +113,21 @@ __device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, ui
   if (a.rec_words == 8) d4[1] = make_uint4(w[4], w[5], w[6], w[7]);
 }
 
-// Warp-collective flush of the per-thread descriptor lists.
+// Warp-collective flush of the per-thread descriptor lists: partition ids,
+// size histograms, one staging reservation per warp, record writes.
 template <typename CT>
 __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
-                                                  uint64_t o, int64_t L) {
+                                                  int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
-  const int64_t nmax = a.max_kmers;
+  const int nmax = (int)a.max_kmers;
   uint32_t my_records = 0;
-  for (int d = 0; d < ndesc; ++d) {
-    const unsigned long long se = sm.desc_se[d * kMspThreads + tid];
-    const int64_t n = (int64_t)(se >> 32) - (int64_t)(se & 0xffffffffu) + 1;
-    my_records += (uint32_t)((n + nmax - 1) / nmax);
+  {
+    int s = s_next;
+    for (int d = 0; d < ndesc; ++d) {
+      const int e = (int)sm.desc_e[d * kMspThreads + tid];
+      my_records += (uint32_t)((e - s + nmax) / nmax);
+      s = e + 1;
+    }
   }
   uint32_t incl = my_records;
 #pragma unroll
@@ -139,48 +142,38 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     base = __shfl_sync(kFull, base, 0);
   }
   uint64_t slot = base + incl - my_records;
+  int s = s_next;
   for (int d = 0; d < ndesc; ++d) {
-    const unsigned long long se = sm.desc_se[d * kMspThreads + tid];
-    const int64_t s = (int64_t)(se & 0xffffffffu), e = (int64_t)(se >> 32);
+    const int e = (int)sm.desc_e[d * kMspThreads + tid];
     const uint64_t m = (uint64_t)sm.desc_m[d * kMspThreads + tid];
     const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
-    const int64_t n = e - s + 1;
+    const int n = e - s + 1;
     const uint32_t pieces = (uint32_t)((n + nmax - 1) / nmax);
-    if (sm.hist_rec) {
-      atomicAdd(sm.hist_rec + pid, pieces);
-      atomicAdd(sm.hist_kmer + pid, (uint32_t)n);
-    } else {
-      atomicAdd(a.n_records + pid, (unsigned long long)pieces);
-      atomicAdd(a.n_kmers + pid, (unsigned long long)n);
-    }
-    for (int64_t ps = s; ps <= e; ps += nmax, ++slot) {
+    atomicAdd(a.n_records + pid, (unsigned long long)pieces);
+    atomicAdd(a.n_kmers + pid, (unsigned long long)n);
+    for (int ps = s; ps <= e; ps += nmax, ++slot) {
       if (slot < a.staging_cap)
         write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
     }
+    s = e + 1;
   }
+  s_next = s;
   ndesc = 0;
 }
 
+// kMaxDesc >= 32 + 2: a 32-base chunk closes at most one superkmer per K-mer
+// plus the read's last one, so the flush vote is needed once per chunk.
 template <typename CT>
 __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int tid = threadIdx.x, lane = tid & 31;
   MspSmem<CT> sm;
   unsigned char* sp = smem_raw;
-  sm.desc_se = reinterpret_cast<unsigned long long*>(sp);
-  sp += sizeof(unsigned long long) * kMaxDesc * kMspThreads;
-  sm.desc_m = reinterpret_cast<unsigned long long*>(sp);
-  sp += sizeof(unsigned long long) * kMaxDesc * kMspThreads;
+  sm.desc_m = reinterpret_cast<CT*>(sp);
+  sp += sizeof(CT) * kMaxDesc * kMspThreads;
+  sm.desc_e = reinterpret_cast<uint32_t*>(sp);
+  sp += sizeof(uint32_t) * kMaxDesc * kMspThreads;
   sm.row = reinterpret_cast<CT*>(sp);
-  sp += sizeof(CT) * a.w * kMspThreads;
-  sp = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sp) + 15) & ~uintptr_t(15));
-  const bool smem_hist = a.np <= kSmemHistMaxNp;
-  sm.hist_rec = smem_hist ? reinterpret_cast<uint32_t*>(sp) : nullptr;
-  sm.hist_kmer = smem_hist ? sm.hist_rec + a.np : nullptr;
-  if (smem_hist) {
-    for (int i = tid; i < 2 * a.np; i += kMspThreads) sm.hist_rec[i] = 0;
-  }
-  __syncthreads();
 
   const int K = a.k, P = a.p, w = a.w;
   const CT maskP = (CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1));
@@ -191,77 +184,62 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
     const uint64_t r = r0 + lane;
     uint64_t o = 0;
-    int64_t L = 0;
+    int L = 0;
     if (r < a.n_reads) {
       o = a.offsets[r];
-      L = (int64_t)(a.offsets[r + 1] - o);
+      L = (int)(a.offsets[r + 1] - o);
     }
-    const int64_t nk = L - K + 1;
-    int64_t Lmax = L;
+    const int nk = L - K + 1;
+    if (nk <= 0) L = 0;  // reading N: no K-mers
+    int Lmax = L;
 #pragma unroll
-    for (int dlt = 16; dlt; dlt >>= 1) Lmax = max(Lmax, (int64_t)__shfl_xor_sync(kFull, (long long)Lmax, dlt));
-    int ndesc = 0;
-    CT f = 0, rc = 0, pre = 0;
-    uint64_t m_cur = 0;
-    int64_t s_start = 0;
+    for (int dlt = 16; dlt; dlt >>= 1) Lmax = max(Lmax, __shfl_xor_sync(kFull, Lmax, dlt));
+    int ndesc = 0, s_next = 0;
+    CT f = 0, rc = 0, pre = 0, m_cur = 0;
     int u = 0;  // position within the current van Herk block
-    uint64_t wbuf = 0;
-    for (int64_t j = 0; j < Lmax; ++j) {
-      if (j < L && nk > 0) {
-        if ((j & 31) == 0) wbuf = window64(a.words, a.n_words, o + j);
+    for (int c0 = 0; c0 < Lmax; c0 += 32) {
+      uint64_t wbuf = c0 < L ? window64(a.words, a.n_words, o + c0) : 0;
+      const int jn = min(32, L - c0);  // bases of this read in the chunk (<= 0: none)
+      for (int jj = 0; jj < jn; ++jj) {
+        const int j = c0 + jj;
         const uint32_t b = (uint32_t)(wbuf >> 62);
         wbuf <<= 2;
         f = ((f << 2) | (CT)b) & maskP;
         rc = (rc >> 2) | ((CT)(3u - b) << topP);
-        if (j >= P - 1) {
-          const int64_t q = j - P + 1;  // P-mer index
-          const CT c = f < rc ? f : rc;
-          const CT snext = (u + 1 < w) ? row[(u + 1) * kMspThreads] : (CT)0;
-          row[u * kMspThreads] = c;
-          pre = (u == 0) ? c : (c < pre ? c : pre);
-          if (q >= w - 1) {  // K-mer i = q-w+1 is complete
-            const int64_t i = q - w + 1;
-            const CT mm = (u == w - 1) ? pre : (snext < pre ? snext : pre);
-            const uint64_t m = (uint64_t)mm;
-            if (i == 0) {
-              m_cur = m;
-              s_start = 0;
-            } else if (m != m_cur) {
-              sm.desc_se[ndesc * kMspThreads + tid] =
-                  (unsigned long long)s_start | ((unsigned long long)(i - 1) << 32);
-              sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
-              ++ndesc;
-              s_start = i;
-              m_cur = m;
-            }
-            if (i == nk - 1) {  // the read's last superkmer
-              sm.desc_se[ndesc * kMspThreads + tid] =
-                  (unsigned long long)s_start | ((unsigned long long)i << 32);
-              sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
-              ++ndesc;
-            }
+        if (j < P - 1) continue;
+        const int q = j - P + 1;  // P-mer index
+        const CT c = f < rc ? f : rc;
+        const CT snext = (u + 1 < w) ? row[(u + 1) * kMspThreads] : (CT)0;
+        row[u * kMspThreads] = c;
+        pre = (u == 0 || c < pre) ? c : pre;
+        if (q >= w - 1) {  // K-mer i = q-w+1 is complete
+          const int i = q - w + 1;
+          const CT m = (u == w - 1 || pre < snext) ? pre : snext;
+          if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
+            sm.desc_e[ndesc * kMspThreads + tid] = (uint32_t)(i - 1);
+            sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
+            ++ndesc;
           }
-          if (u == w - 1) {  // block complete: suffix minima in place
-            for (int t = w - 2; t >= 0; --t) {
-              const CT x = row[t * kMspThreads], y = row[(t + 1) * kMspThreads];
-              if (y < x) row[t * kMspThreads] = y;
-            }
-            u = 0;
-          } else {
-            ++u;
+          m_cur = m;
+          if (i == nk - 1) {  // the read's last superkmer
+            sm.desc_e[ndesc * kMspThreads + tid] = (uint32_t)i;
+            sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
+            ++ndesc;
           }
         }
+        if (u == w - 1) {  // block complete: suffix minima in place
+          for (int t = w - 2; t >= 0; --t) {
+            const CT x = row[t * kMspThreads], y = row[(t + 1) * kMspThreads];
+            if (y < x) row[t * kMspThreads] = y;
+          }
+          u = 0;
+        } else {
+          ++u;
+        }
       }
-      if (__any_sync(kFull, ndesc >= kMaxDesc - 1)) flush_descriptors<CT>(a, sm, ndesc, o, L);
+      if (__any_sync(kFull, ndesc > kMaxDesc - 34)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
     }
-    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, o, L);
-  }
-  if (smem_hist) {
-    __syncthreads();
-    for (int i = tid; i < a.np; i += kMspThreads) {
-      if (sm.hist_rec[i]) atomicAdd(a.n_records + i, (unsigned long long)sm.hist_rec[i]);
-      if (sm.hist_kmer[i]) atomicAdd(a.n_kmers + i, (unsigned long long)sm.hist_kmer[i]);
-    }
+    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
   }
 }
 
@@ -384,8 +362,7 @@ bool dbg_params_ok(const dbg_params* prm) {
 
 template <typename CT>
 static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
-  size_t smem = sizeof(unsigned long long) * 2 * kMaxDesc * kMspThreads + sizeof(CT) * a.w * kMspThreads + 16;
-  if (a.np <= kSmemHistMaxNp) smem += sizeof(uint32_t) * 2 * a.np;
+  const size_t smem = (sizeof(CT) + sizeof(uint32_t)) * kMaxDesc * kMspThreads + sizeof(CT) * a.w * kMspThreads;
   cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   msp_kernel<CT><<<grid, kMspThreads, smem, stream>>>(a);
