@@ -735,6 +735,7 @@ struct SmemArgs {
   int pid0, n_fine, k;  // fine partitions [pid0, pid0 + n_fine)
   double ratio;      // lambda / (4 alpha)
   uint64_t slots;    // table slots that fit one CTA
+  FastMod np_mod;    // reported pid = fine pid mod NP
   uint64_t* P;       // [n_fine + 1] prefix of on-chip capacities (0 for partitions off chip), local index
   uint32_t* gfirst;  // [n_fine + 2] first (absolute) partition of each group
   unsigned long long* n_groups;
@@ -936,11 +937,13 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           const int b = hl + t;
           const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1, S) : -1;
           const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K, S) : -1;
-          if (fwd < rc) {  // odd K: never equal (reading C); edges in the canonical orientation (reading J)
-            ok &= smem_upsert<Code>(tk, tf, cap, fwd, succ >= 0 ? succ : 4, pred, pid);
-          } else {
-            ok &= smem_upsert<Code>(tk, tf, cap, rc, pred >= 0 ? 3 - pred : 4, succ >= 0 ? 3 - succ : -1, pid);
-          }
+          // canonical orientation and edge indices (readings C, J), selected branch-free so
+          // that one upsert serves both orientations (no divergent duplicate of it)
+          const bool is_fwd = fwd < rc;
+          const Code code = is_fwd ? fwd : rc;
+          const int o = is_fwd ? (succ >= 0 ? succ : 4) : (pred >= 0 ? 3 - pred : 4);
+          const int i = is_fwd ? pred : (succ >= 0 ? 3 - succ : -1);
+          ok &= smem_upsert<Code>(tk, tf, cap, code, o, i, pid);
           if (++kid >= k1) break;
           if (++t < n) {  // next K-mer of the same record: roll one base
             fwd = ((fwd << 2) | (Code)succ) & mask;
@@ -963,44 +966,67 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       }
     }
     __syncthreads();
-    // extraction: each thread owns slots s = q * kSmemThreads + tid; one block
-    // scan sizes the group's output, one global atomic reserves it
+    // extraction: each warp owns a contiguous run of slots; one block scan of the
+    // warps' occupied counts sizes the group's output, one global atomic reserves it.
+    // Occupied slot indices are then queued per warp (the idle record staging is the
+    // queue, 128 entries per warp) and emitted with every lane busy.
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    constexpr int kWarps = kSmemThreads / 32;
+    const uint32_t wspan = ((uint32_t)span + kWarps * 32 - 1) / (kWarps * 32) * 32;  // slots per warp
+    const uint32_t ws0 = min((uint32_t)span, warp * wspan), ws1 = min((uint32_t)span, ws0 + wspan);
     uint32_t cnt = 0;
-    for (uint32_t s = threadIdx.x; s < span; s += kSmemThreads)
-      cnt += (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied) ? 1u : 0u;
+    for (uint32_t c = ws0; c < ws1; c += 32) {
+      const uint32_t s = c + lane;
+      cnt += __popc(__ballot_sync(kFull, s < ws1 &&
+                                            (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied)));
+    }
     uint32_t excl, total;
-    Scan(st.scan).ExclusiveSum(cnt, excl, total);
+    Scan(st.scan).ExclusiveSum(lane == 0 ? cnt : 0u, excl, total);
     if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
     __syncthreads();
-    uint64_t pos = st.base + excl;
-    for (uint32_t s = threadIdx.x; s < span; s += kSmemThreads) {
-      unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
-      const uint64_t k0 = kp[0];
-      if (!(k0 & kOccupied)) continue;
-      uint32_t* f = fld + s * FW;
-      dbg_vertex v;
-      if (KW == 1) {
-        v.kmer_hi = 0;
-        v.kmer_lo = k0 & kCodeMask;
-      } else {
-        v.kmer_hi = k0 & kCodeMask;
-        v.kmer_lo = kp[1];
+    uint64_t pos = st.base + __shfl_sync(kFull, excl, 0);
+    uint32_t* queue = &st.w[0][0] + warp * 128;
+    for (uint32_t sub = ws0; sub < ws1; sub += 128) {
+      uint32_t qn = 0;
+      for (uint32_t c = sub; c < min(ws1, sub + 128); c += 32) {
+        const uint32_t s = c + lane;
+        const bool occ = s < ws1 && (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied);
+        const uint32_t bal = __ballot_sync(kFull, occ);
+        if (occ) queue[qn + __popc(bal & ((1u << lane) - 1u))] = s;
+        qn += __popc(bal);
       }
-      const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
-      v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
-      v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
-      v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
-      v.pid = f[5] % oa.np_out;  // fine pid recorded by the inserting thread
-      kp[0] = 0;  // clean-on-extract
-      if (KW == 2) kp[1] = 0;
+      __syncwarp();
+      for (uint32_t e = lane; e < qn; e += 32) {
+        const uint32_t s = queue[e];
+        unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+        const uint64_t k0 = kp[0];
+        uint32_t* f = fld + s * FW;
+        dbg_vertex v;
+        if (KW == 1) {
+          v.kmer_hi = 0;
+          v.kmer_lo = k0 & kCodeMask;
+        } else {
+          v.kmer_hi = k0 & kCodeMask;
+          v.kmer_lo = kp[1];
+        }
+        const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
+        v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
+        v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
+        v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
+        v.pid = fast_mod(a.np_mod, f[5]);  // fine pid recorded by the inserting thread, mod NP
+        kp[0] = 0;  // clean-on-extract
+        if (KW == 2) kp[1] = 0;
 #pragma unroll
-      for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
-      if (pos < oa.out_cap) oa.out[pos] = v;
-      else atomicOr(oa.status, kStatusNoSpace);
-      ++pos;
-      st_n += 1;
-      st_count += v.count;
-      st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
+        for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
+        const uint64_t my = pos + e;
+        if (my < oa.out_cap) oa.out[my] = v;
+        else atomicOr(oa.status, kStatusNoSpace);
+        st_n += 1;
+        st_count += v.count;
+        st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
+      }
+      pos += qn;
+      __syncwarp();
     }
   }
   if (!ok) atomicOr(oa.status, kStatusTableFull);
@@ -1209,6 +1235,7 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   a.n_kmers = part->d_n_kmers;
   a.pid0 = pid_begin;
   a.n_fine = pid_end - pid_begin;
+  a.np_mod = make_fastmod((uint64_t)prm->num_partitions);
   a.k = prm->k;
   a.ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   a.slots = dbg_smem_table_slots(prm);

@@ -37,31 +37,6 @@ constexpr int kMspThreads = 128;
 constexpr int kMaxDesc = 40;             // descriptors per thread between flushes (>= 34)
 constexpr int kSmemHistMaxNp = 8192;
 
-// Unsigned 64-bit division by an invariant integer (Granlund & Montgomery
-// 1994, Fig. 4.1): exact x mod d for every 64-bit x, d >= 1.
-struct FastMod {
-  uint64_t d, m;
-  int sh1, sh2;
-};
-
-static FastMod make_fastmod(uint64_t d) {
-  int l = 0;
-  while (l < 64 && (1ull << l) < d) ++l;  // l = ceil(log2 d)
-  FastMod f;
-  f.d = d;
-  const unsigned __int128 two_l = (unsigned __int128)1 << l;
-  f.m = (uint64_t)((((unsigned __int128)1 << 64) * (two_l - d)) / d + 1);
-  f.sh1 = l < 1 ? l : 1;
-  f.sh2 = l - 1 > 0 ? l - 1 : 0;
-  return f;
-}
-
-__device__ __forceinline__ uint32_t fast_mod(const FastMod& f, uint64_t x) {
-  const uint64_t t1 = __umul64hi(f.m, x);
-  const uint64_t q = (t1 + ((x - t1) >> f.sh1)) >> f.sh2;
-  return (uint32_t)(x - q * f.d);
-}
-
 struct MspArgs {
   const uint64_t* words;
   uint64_t n_words;
