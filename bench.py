@@ -208,12 +208,21 @@ def run_ours(args):
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
 
+    host_ms = {"msp": [], "plan": [], "reset": [], "step2": []}
+
     def step():
-        """One pass of rows a2-a7 (MSP, sizing, fused zero/hash/extract)."""
+        """One pass of rows a2-a7 (MSP, sizing, on-chip / global Step 2)."""
+        t = time.perf_counter()
         b.msp(d_bases, d_off, stream)
+        t1 = time.perf_counter()
         b.plan(stream)
+        t2 = time.perf_counter()
         b.reset_output(n_kmers // 2 + 1024, stream)
+        t3 = time.perf_counter()
         b.step2(stream)
+        t4 = time.perf_counter()
+        for k, v in zip(("msp", "plan", "reset", "step2"), (t1 - t, t2 - t1, t3 - t2, t4 - t3)):
+            host_ms[k].append(1e3 * v)
 
     for _ in range(args.warmup):
         step()
@@ -303,6 +312,7 @@ def run_ours(args):
         "gpu_launches": args.steps * launches_per_step,
         "clocks": clk.summary(),
         "breakdown_ms": phases,
+        "host_ms": {k: round(statistics.mean(v[-args.steps:]), 3) for k, v in host_ms.items() if v},
         "stats": stats, "invariants_ok": bool(inv_ok), "gen_s": gen_s,
     }
     print(json.dumps(line), flush=True)
