@@ -239,9 +239,9 @@ class DbgBuilder:
             self.batches = []
             return self.batches
         budget = self.table_budget_bytes
-        if budget is None:
+        if budget is None:  # once per builder: cudaMemGetInfo costs milliseconds
             free, _ = torch.cuda.mem_get_info(self.device)
-            budget = max(int(free * 0.6), 1 << 26)
+            budget = self.table_budget_bytes = max(int(free * 0.6), 1 << 26)
         max_slots = max(budget // self.slot_bytes, int(self.caps.max(initial=0)))
         bkey = (self._caps_key, max_slots)
         if self._batch_key != bkey:  # greedy batches of consecutive partitions (vectorised)
