@@ -426,6 +426,39 @@ __global__ void __launch_bounds__(kThreads) hash_build_kernel(ResidentArgs a) {
   }
 }
 
+// Same as hash_build_kernel for an explicit list of partitions (the oversize
+// ones of the on-chip path): warp-chunks of 32 records are numbered across the
+// listed partitions by chunk_prefix (exclusive prefix of ceil(records/32)).
+template <typename Code, int R>
+__global__ void __launch_bounds__(kThreads) hash_build_list_kernel(ResidentArgs a, const uint32_t* pids,
+                                                                  const uint64_t* chunk_prefix, int n_pids) {
+  constexpr uint32_t KE = sizeof(Code) == 8 ? 16 : 32;
+  __shared__ WarpRecs<R> sh[kThreads / 32];
+  const uint64_t s0 = a.tab_off[a.pid_begin], n_slots = a.tab_off[a.pid_end] - s0;
+  uint32_t* ctr_base = reinterpret_cast<uint32_t*>(a.table + n_slots * KE);
+  const uint64_t* off = a.tab_off;
+  auto table_of = [=](uint32_t pid, uint64_t& t0, uint64_t& cap) {
+    t0 = __ldg(off + pid) - s0;
+    cap = __ldg(off + pid + 1) - __ldg(off + pid);
+  };
+  const int warp = threadIdx.x >> 5;
+  const uint64_t n_chunks = chunk_prefix[n_pids];
+  for (uint64_t c = (uint64_t)blockIdx.x * (kThreads / 32) + warp; c < n_chunks;
+       c += (uint64_t)gridDim.x * (kThreads / 32)) {
+    int lo = 0, hi = n_pids;  // listed partition holding chunk c
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (chunk_prefix[mid] <= c) lo = mid;
+      else hi = mid;
+    }
+    const uint32_t pid = pids[lo];
+    const uint64_t r0 = a.rec_off[pid] + 32 * (c - chunk_prefix[lo]);
+    const int64_t n = (int64_t)min((uint64_t)32, a.rec_off[pid + 1] - r0);
+    if (!hash_warp<Code, R>(a.records + r0 * R, n, a.k, a.table, ctr_base, table_of, sh[warp]))
+      atomicOr(a.status, kStatusTableFull);
+  }
+}
+
 template <int KW>
 __global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, OutArgs oa) {
   constexpr uint32_t KE = KW == 1 ? 16 : 32;
@@ -1119,6 +1152,30 @@ extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_
   if (prm->k <= 31) hash_build_kernel<uint64_t, 4><<<grid, kThreads, 0, stream>>>(a);
   else if (prm->k <= 39) hash_build_kernel<u128, 4><<<grid, kThreads, 0, stream>>>(a);
   else hash_build_kernel<u128, 8><<<grid, kThreads, 0, stream>>>(a);
+  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+}
+
+extern "C" dbg_status dbg_hash_build_list(const dbg_params* prm, const dbg_partition_set* part,
+                                          const uint32_t* d_pids, const uint64_t* d_chunk_prefix, int32_t n_pids,
+                                          void* d_table, const uint64_t* d_table_offset, uint32_t* d_status,
+                                          cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table ||
+      !d_table_offset || !d_status || n_pids < 0 || (n_pids && (!d_pids || !d_chunk_prefix)))
+    return DBG_EINVAL;
+  if (n_pids == 0) return DBG_OK;
+  ResidentArgs a;
+  a.records = part->d_records;
+  a.rec_off = part->d_record_offset;
+  a.tab_off = d_table_offset;
+  a.table = static_cast<char*>(d_table);
+  a.pid_begin = 0;
+  a.pid_end = fine_partitions(prm);
+  a.k = prm->k;
+  a.status = d_status;
+  const int grid = dbg_sm_count() * 8;
+  if (prm->k <= 31) hash_build_list_kernel<uint64_t, 4><<<grid, kThreads, 0, stream>>>(a, d_pids, d_chunk_prefix, n_pids);
+  else if (prm->k <= 39) hash_build_list_kernel<u128, 4><<<grid, kThreads, 0, stream>>>(a, d_pids, d_chunk_prefix, n_pids);
+  else hash_build_list_kernel<u128, 8><<<grid, kThreads, 0, stream>>>(a, d_pids, d_chunk_prefix, n_pids);
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 

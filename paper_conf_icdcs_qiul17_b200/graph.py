@@ -116,6 +116,7 @@ class DbgBuilder:
         self.batches: list[tuple[int, int]] = []
         self._caps_key = None
         self._batch_key = None
+        self._big_key = None
         self._batches_cache: list[tuple[int, int]] = []
         self._dirty = False
         self.timer: dict | None = None  # name -> list of (start, end) CUDA events, when set
@@ -332,13 +333,32 @@ class DbgBuilder:
             return
         for (b, e) in self.batches:
             ev = self._mark("hash_build", stream)
-            _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.table, self.d_tab_off, self.d_status,
-                                stream)
+            if self.mode == "smem":  # only the oversize partitions have records to hash here
+                pids, prefix = self._big_list(b, e)
+                _lib.dbg_hash_build_list(self.prm, self.part_set(True), pids, prefix, pids.numel(), self.table,
+                                         self.d_tab_off, self.d_status, stream)
+            else:
+                _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.table, self.d_tab_off,
+                                    self.d_status, stream)
             self._done(ev, stream)
             ev = self._mark("extract", stream)
             _lib.dbg_extract_graph(self.prm, self.table, self.d_tab_off, b, e, self.out, self.out_cap(),
                                    self.d_n_out, self.d_stats, self.d_status, stream)
             self._done(ev, stream)
+
+    def _big_list(self, b: int, e: int):
+        """Device list of the partitions in [b, e) with a global table (capacity > 0) and the prefix
+        of their 32-record chunk counts (cached per plan)."""
+        key = (self._caps_key, b, e)
+        if self._big_key != key:
+            pids = np.nonzero(self.caps[b:e])[0].astype(np.int64) + b
+            chunks = (self.part_records[pids] + 31) // 32
+            prefix = np.zeros(len(pids) + 1, dtype=np.int64)
+            prefix[1:] = np.cumsum(chunks)
+            self._big = (torch.from_numpy(pids.astype(np.int32)).to(self.device),
+                         torch.from_numpy(prefix).to(self.device))
+            self._big_key = key
+        return self._big
 
     def stats(self, checksum: bool = True, stream=None) -> dict:
         """Totals of the last extraction; the checksum is computed here (dbg_checksum_vertices)."""
