@@ -207,6 +207,9 @@ def run_ours(args):
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    # output capacity: distinct vertices <= K-mers; 0.4 x covers the configs' error rates (a build
+    # that overflows it reports DBG_ENOSPACE and the invariant check fails loudly)
+    out_cap = int(args.out_frac * n_kmers) + 1024
 
     host_ms = {"msp": [], "plan": [], "reset": [], "step2": []}
 
@@ -217,7 +220,7 @@ def run_ours(args):
         t1 = time.perf_counter()
         b.plan(stream)
         t2 = time.perf_counter()
-        b.reset_output(n_kmers // 2 + 1024, stream)
+        b.reset_output(out_cap, stream)
         t3 = time.perf_counter()
         b.step2(stream)
         t4 = time.perf_counter()
@@ -264,7 +267,7 @@ def run_ours(args):
         eh.record(stream)
         b.msp(db, do, stream)
         b.plan(stream)
-        b.reset_output(n_kmers // 2 + 1024, stream)
+        b.reset_output(out_cap, stream)
         b.step2(stream)
         host_stats.copy_(b.d_stats, non_blocking=True)  # D2H of the step's result
         e1.record(stream)
@@ -342,6 +345,7 @@ def main():
     ap.add_argument("--refine", type=int, default=None, help="fine partitions per partition (default: auto)")
     ap.add_argument("--group-slots", type=int, default=1 << 19)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--out-frac", type=float, default=0.4, help="output capacity / K-mers")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.impl == "reference":
