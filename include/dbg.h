@@ -205,15 +205,15 @@ DBG_API dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_set
                           int32_t pid_end, void* d_table, const uint64_t* d_table_offset,
                           uint32_t* d_status, cudaStream_t stream);
 
-/* As dbg_hash_build over the whole table block of partitions [0, NP*refine)
+/* As dbg_hash_build for the table block of partitions [pid_begin, pid_end)
  * (d_table_offset from dbg_table_plan_split), but only for the n_pids listed
- * partitions: d_pids[n_pids] fine partition ids, d_chunk_prefix[n_pids+1] the
- * exclusive prefix sum of ceil(records of d_pids[j] / 32).  Used for the
- * partitions too large for the on-chip path. */
-DBG_API dbg_status dbg_hash_build_list(const dbg_params* prm, const dbg_partition_set* part,
-                               const uint32_t* d_pids, const uint64_t* d_chunk_prefix, int32_t n_pids,
-                               void* d_table, const uint64_t* d_table_offset, uint32_t* d_status,
-                               cudaStream_t stream);
+ * partitions (all inside the range): d_pids[n_pids] fine partition ids,
+ * d_chunk_prefix[n_pids+1] the exclusive prefix sum of ceil(records of
+ * d_pids[j] / 32).  Used for the partitions too large for the on-chip path. */
+DBG_API dbg_status dbg_hash_build_list(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                               int32_t pid_end, const uint32_t* d_pids, const uint64_t* d_chunk_prefix,
+                               int32_t n_pids, void* d_table, const uint64_t* d_table_offset,
+                               uint32_t* d_status, cudaStream_t stream);
 
 /* ---- a7: output (Def. 3) -------------------------------------
  * Compacts the occupied slots of resident tables (layout of dbg_hash_build)

@@ -70,7 +70,7 @@ SIGNATURES = {
     "dbg_build_subgraphs": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _U64, _P, _U64, _P, _U64, _P, _U64,
                                            _P, _P, _P, _P]),
     "dbg_hash_build": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _P, _P]),
-    "dbg_hash_build_list": (ctypes.c_int, [_PRM, _PART, _P, _P, _I32, _P, _P, _P, _P]),
+    "dbg_hash_build_list": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _I32, _P, _P, _P, _P]),
     "dbg_extract_graph": (ctypes.c_int, [_PRM, _P, _P, _I32, _I32, _P, _U64, _P, _P, _P, _P]),
     "dbg_sort_workspace_bytes": (_U64, [_PRM, _U64]),
     "dbg_sort_vertices": (ctypes.c_int, [_PRM, _P, _P, _U64, _P, _U64, _P]),
@@ -234,11 +234,11 @@ def dbg_hash_build(prm, part, pid_begin: int, pid_end: int, d_table, d_table_off
         _ptr(d_status), _stream(stream)))
 
 
-def dbg_hash_build_list(prm, part, d_pids, d_chunk_prefix, n_pids: int, d_table, d_table_offset, d_status,
-                        stream=None) -> None:
+def dbg_hash_build_list(prm, part, pid_begin: int, pid_end: int, d_pids, d_chunk_prefix, n_pids: int, d_table,
+                        d_table_offset, d_status, stream=None) -> None:
     _check("dbg_hash_build_list", load().dbg_hash_build_list(
-        ctypes.byref(prm), ctypes.byref(part), _ptr(d_pids), _ptr(d_chunk_prefix), n_pids, _ptr(d_table),
-        _ptr(d_table_offset), _ptr(d_status), _stream(stream)))
+        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_pids), _ptr(d_chunk_prefix), n_pids,
+        _ptr(d_table), _ptr(d_table_offset), _ptr(d_status), _stream(stream)))
 
 
 def dbg_extract_graph(prm, d_table, d_table_offset, pid_begin: int, pid_end: int, d_out, out_cap: int, d_n_out,

@@ -1155,21 +1155,22 @@ extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-extern "C" dbg_status dbg_hash_build_list(const dbg_params* prm, const dbg_partition_set* part,
-                                          const uint32_t* d_pids, const uint64_t* d_chunk_prefix, int32_t n_pids,
-                                          void* d_table, const uint64_t* d_table_offset, uint32_t* d_status,
-                                          cudaStream_t stream) {
+extern "C" dbg_status dbg_hash_build_list(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                                          int32_t pid_end, const uint32_t* d_pids, const uint64_t* d_chunk_prefix,
+                                          int32_t n_pids, void* d_table, const uint64_t* d_table_offset,
+                                          uint32_t* d_status, cudaStream_t stream) {
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table ||
       !d_table_offset || !d_status || n_pids < 0 || (n_pids && (!d_pids || !d_chunk_prefix)))
     return DBG_EINVAL;
+  if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (n_pids == 0) return DBG_OK;
   ResidentArgs a;
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
   a.tab_off = d_table_offset;
   a.table = static_cast<char*>(d_table);
-  a.pid_begin = 0;
-  a.pid_end = fine_partitions(prm);
+  a.pid_begin = pid_begin;
+  a.pid_end = pid_end;
   a.k = prm->k;
   a.status = d_status;
   const int grid = dbg_sm_count() * 8;

@@ -335,8 +335,8 @@ class DbgBuilder:
             ev = self._mark("hash_build", stream)
             if self.mode == "smem":  # only the oversize partitions have records to hash here
                 pids, prefix = self._big_list(b, e)
-                _lib.dbg_hash_build_list(self.prm, self.part_set(True), pids, prefix, pids.numel(), self.table,
-                                         self.d_tab_off, self.d_status, stream)
+                _lib.dbg_hash_build_list(self.prm, self.part_set(True), b, e, pids, prefix, pids.numel(),
+                                         self.table, self.d_tab_off, self.d_status, stream)
             else:
                 _lib.dbg_hash_build(self.prm, self.part_set(True), b, e, self.table, self.d_tab_off,
                                     self.d_status, stream)

@@ -286,3 +286,13 @@ def test_sharded_path_two_logical_ranks_one_gpu():
     allv = allv[np.lexsort((allv["kmer_lo"], allv["kmer_hi"]))]
     orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT)
     compare_vertices(allv, orc)
+
+
+def test_smem_global_tier_in_several_batches():
+    """Oversize partitions whose global tables do not fit the table budget at once are built in
+    several batches (each batch's table block starts at its first partition)."""
+    g = genome(60_000, seed=12)
+    seq, offs = make_reads(g, 4000, 100, 0.01, seed=13)
+    rs = ReadSet(seq, offs)
+    res, _ = _check(rs, 31, 11, 3, refine=1, table_budget_bytes=48 * 20_000)
+    assert len(res.batches) >= 2
