@@ -114,6 +114,8 @@ def _workload(args):
 
     t = time.time()
     rs = make_config(args.config, scale=args.scale, num_partitions=args.np)
+    if args.p is not None:
+        rs.p = args.p
     return rs, time.time() - t
 
 
@@ -182,6 +184,19 @@ def run_reference(args):
 
 
 # ------------------------------------------------------------------------------- our arm
+def _placement(b) -> dict:
+    """Share of the K-mers whose partition is grouped on chip, split over several CTA tables, or
+    built in the global tables (dbg_smem_onchip)."""
+    from paper_conf_icdcs_qiul17_b200 import _lib
+
+    pk = b.part_kmers
+    uniq, inv = np.unique(pk, return_inverse=True)
+    place = np.array([_lib.dbg_smem_onchip(b.prm, int(n)) for n in uniq])[inv]
+    tot = max(int(pk.sum()), 1)
+    return {"grouped": float(pk[place == 1].sum()) / tot, "split": float(pk[place >= 2].sum()) / tot,
+            "global": float(pk[place == 0].sum()) / tot, "split_ctas": int(place[place >= 2].sum())}
+
+
 def run_ours(args):
     import torch
 
@@ -192,7 +207,7 @@ def run_ours(args):
         return multi.bench_main(args, METRIC, UNIT)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    from paper_conf_icdcs_qiul17_b200 import DbgBuilder, auto_refine, encode_reads, _lib
+    from paper_conf_icdcs_qiul17_b200 import DbgBuilder, auto_fine_p, auto_refine, encode_reads, _lib
 
     rs, gen_s = _workload(args)
     packed = encode_reads(rs.seq, pin=True)
@@ -202,8 +217,11 @@ def run_ours(args):
     refine = args.refine
     if refine is None:
         refine = auto_refine(n_kmers, rs.k, rs.p, rs.num_partitions, args.lam, args.alpha) if args.mode == "smem" else 1
+    fine_p = args.fine_p
+    if fine_p is None:
+        fine_p = auto_fine_p(n_kmers, rs.k, rs.p, args.lam, args.alpha) if args.mode == "smem" else 0
     b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode,
-                   args.group_slots, refine)
+                   args.group_slots, refine, args.smem_split, fine_p)
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
@@ -299,16 +317,20 @@ def run_ours(args):
         rate, sub, dt = _oracle_rate(rs, args.cpu_seconds, threads)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
-    launches_per_step = 3 + {"fused": 2, "resident": 2 * len(b.batches),
-                             "smem": 1 + 2 * len(b.batches)}[args.mode] + 1
+    scan = 1 if b.np <= 16384 else 3  # scan.cuh: one CTA, or tile sums + tile scan + apply
+    launches_per_step = 1 + scan + 1 + scan + {"fused": 2, "resident": 2 * len(b.batches),
+                                              "smem": 6 + 2 * len(b.batches)}[args.mode]
+    placement = _placement(b) if args.mode == "smem" else None
     line = {
         "metric": METRIC, "value": n_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": _config_json(rs, args, {"mode": args.mode, "batches": len(b.batches),
                                           "group_slots": args.group_slots, "refine": refine,
-                                          "fine_partitions": b.np,
-                                          "smem_slots": _lib.dbg_smem_table_slots(b.prm)}),
+                                          "fine_partitions": b.np, "smem_split": args.smem_split,
+                                          "fine_p": fine_p or rs.p,
+                                          "smem_slots": _lib.dbg_smem_table_slots(b.prm),
+                                          "kmer_placement": placement}),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "kernel": {"fused": "subgraph_kernel", "resident": "hash_build_kernel",
@@ -338,12 +360,17 @@ def main():
     ap.add_argument("--config", default="ecoli")
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--np", type=int, default=None, help="override the number of partitions")
+    ap.add_argument("--p", type=int, default=None, help="override the minimizer length P")
     ap.add_argument("--lam", type=float, default=2.0)
     ap.add_argument("--alpha", type=float, default=0.5)
     ap.add_argument("--table-budget", type=int, default=None)
     ap.add_argument("--mode", choices=["smem", "fused", "resident"], default="smem")
     ap.add_argument("--refine", type=int, default=None, help="fine partitions per partition (default: auto)")
     ap.add_argument("--group-slots", type=int, default=1 << 19)
+    ap.add_argument("--fine-p", type=int, default=None,
+                    help="minimizer length of the fine partitioning (default: auto; dbg_params.fine_p)")
+    ap.add_argument("--smem-split", type=int, default=0,
+                    help="most CTAs an oversize partition is split over on chip (0: default, 1: none)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--out-frac", type=float, default=0.4, help="output capacity / K-mers")
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 2
+#define DBG_ABI_VERSION 3
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -57,6 +57,15 @@ typedef struct {
   int32_t refine;         /* F >= 1: the device works on NP*F fine partitions, fine pid =
                              fmix64(m) mod (NP*F), so a fine partition's table fits one SM;
                              the paper's partition of a vertex is fine pid mod NP (0 = 1) */
+  int32_t smem_split;     /* on-chip path only: most CTAs (sub-tables) one partition too large
+                             for a CTA table may be split over, 1..64; 1 = no splitting,
+                             0 = default (32).  Larger partitions take the global tables. */
+  int32_t fine_p;         /* minimizer length of the device's fine partitioning, 1..min(k,31);
+                             0 = p.  Step 1 then cuts superkmers at changes of this minimizer
+                             and fine pid = fmix64(its minimizer) mod (NP*F), which spreads the
+                             K-mers of large genomes (few distinct P-mers per base) evenly;
+                             dbg_vertex.pid stays the paper's partition, computed from the
+                             vertex's canonical P-minimizer (reading V). */
 } dbg_params;
 
 /* One vertex of Definition 3: the canonical K-mer (the
@@ -140,9 +149,11 @@ DBG_API dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_ba
 
 /* ---- a5: sizing (Property 1; Sec. IV-A) ----------------------
  * d_table_offset[NP+1] = exclusive prefix sum of dbg_table_capacity(N^i_kmer)
- * (in slots). */
+ * (in slots).  d_scratch: NP uint64 of caller memory for the multi-CTA scan
+ * (e.g. the idle d_fill of the partition set), or NULL (one CTA: slow for
+ * large NP). */
 DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers,
-                          uint64_t* d_table_offset, cudaStream_t stream);
+                          uint64_t* d_table_offset, uint64_t* d_scratch, cudaStream_t stream);
 
 /* ---- a5-a7 on-chip: Step 2 in shared memory (the hot path) ---------------
  * Every fine partition in [pid_begin, pid_end) whose table (capacity from Property 1, Sec. IV-A
@@ -150,23 +161,32 @@ DBG_API dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kme
  * slots -- is built and extracted on chip: consecutive such partitions are
  * grouped so that a group's tables fill one CTA's table space; the CTA hashes
  * the group's records (shared-memory 64/128-bit CAS claims a key, shared-
- * memory atomics count the edges in 16-bit fields: no count can exceed the
- * partition's N^i_kmer < 65536) and compacts the occupied slots straight into
- * d_out.  Larger partitions are skipped here and left to the global-table
- * path (dbg_table_plan_split + dbg_hash_build + dbg_extract_graph).
- * d_work: dbg_smem_workspace_bytes() bytes of caller memory (group plan).
+ * memory atomics count the edges in 16-bit fields) and compacts the occupied
+ * slots straight into d_out.  A partition with capacity c above the slots is
+ * split over ns = ceil(1.25 c / slots) <= prm->smem_split CTAs
+ * (dbg_smem_onchip): each reads all of its records and keeps the K-mers whose key hash
+ * selects its sub-table (one vertex, one sub-table), so each CTA table holds
+ * an expected <= 80% of its slots.  Counters on chip are 16-bit, so only
+ * partitions with N^i_kmer <= 65535 (a bound on any of their vertex counts)
+ * go on chip.  The other partitions are skipped here and left to the global-table path
+ * (dbg_table_plan_split + dbg_hash_build_list + dbg_extract_graph).
+ * d_work: dbg_smem_workspace_bytes() bytes of caller memory (the plan).
  * Output appends to d_out[*d_n_out ...] and accumulates *d_stats. */
 DBG_API uint64_t dbg_smem_table_slots(const dbg_params* prm);
+/* Where a partition with n_kmers K-mers is built: 1 = grouped on chip, ns >= 2
+ * = split over ns CTAs, 0 = global tables (N^i_kmer > 65535, or ns > smem_split);
+ * -1 for invalid params. */
+DBG_API int32_t dbg_smem_onchip(const dbg_params* prm, uint64_t n_kmers);
 DBG_API uint64_t dbg_smem_workspace_bytes(const dbg_params* prm);
 DBG_API dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
                                     int32_t pid_begin, int32_t pid_end, void* d_work,
                                     uint64_t work_bytes, dbg_vertex* d_out, uint64_t out_cap,
                                     uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
                                     cudaStream_t stream);
-/* As dbg_table_plan, but partitions whose capacity is <= smem_slots get
- * capacity 0 (they are built on chip), so resident tables cover only the rest. */
-DBG_API dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t smem_slots,
-                                uint64_t* d_table_offset, cudaStream_t stream);
+/* As dbg_table_plan, but partitions built on chip (dbg_smem_onchip > 0) get
+ * capacity 0, so resident tables cover only the rest. */
+DBG_API dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers,
+                                uint64_t* d_table_offset, uint64_t* d_scratch, cudaStream_t stream);
 
 /* ---- a5-a7 fused: Step 2 through an L2-resident ring -----------------------
  * For partitions [pid_begin, pid_end): build each partition's table (one

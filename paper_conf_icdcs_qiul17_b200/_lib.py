@@ -27,7 +27,8 @@ class DbgError(RuntimeError):
 
 class dbg_params(ctypes.Structure):
     _fields_ = [("k", ctypes.c_int32), ("p", ctypes.c_int32), ("num_partitions", ctypes.c_int32),
-                ("lambda_", ctypes.c_float), ("alpha", ctypes.c_float), ("refine", ctypes.c_int32)]
+                ("lambda_", ctypes.c_float), ("alpha", ctypes.c_float), ("refine", ctypes.c_int32),
+                ("smem_split", ctypes.c_int32), ("fine_p", ctypes.c_int32)]
 
 
 class dbg_partition_set(ctypes.Structure):
@@ -60,11 +61,12 @@ SIGNATURES = {
     "dbg_packed_words": (_U64, [_U64]),
     "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
-    "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P]),
+    "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P, _P]),
     "dbg_smem_table_slots": (_U64, [_PRM]),
+    "dbg_smem_onchip": (ctypes.c_int32, [_PRM, _U64]),
     "dbg_smem_workspace_bytes": (_U64, [_PRM]),
     "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _P, _U64, _P, _P, _P, _P]),
-    "dbg_table_plan_split": (ctypes.c_int, [_PRM, _P, _U64, _P, _P]),
+    "dbg_table_plan_split": (ctypes.c_int, [_PRM, _P, _P, _P, _P]),
     "dbg_subgraph_ring_bytes": (_U64, [_PRM, _U64, _U64]),
     "dbg_subgraph_workspace_bytes": (_U64, [_PRM, _I32, _U64, _U64]),
     "dbg_build_subgraphs": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _U64, _P, _U64, _P, _U64, _P, _U64,
@@ -80,6 +82,7 @@ SIGNATURES = {
 }
 
 _lib = None
+ABI_VERSION = 3
 
 
 def load():
@@ -94,7 +97,7 @@ def load():
             f = getattr(lib, name)
             f.restype = res
             f.argtypes = args
-        if lib.dbg_abi_version() != 2:
+        if lib.dbg_abi_version() != ABI_VERSION:
             raise ImportError("libdbg.so ABI version mismatch")
         _lib = lib
     return _lib
@@ -126,8 +129,8 @@ def _stream(stream) -> int | None:
 
 
 def params(k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
-           refine: int = 1) -> dbg_params:
-    return dbg_params(k, p, num_partitions, lam, alpha, refine)
+           refine: int = 1, smem_split: int = 0, fine_p: int = 0) -> dbg_params:
+    return dbg_params(k, p, num_partitions, lam, alpha, refine, smem_split, fine_p)
 
 
 def fine_partitions(prm: dbg_params) -> int:
@@ -185,13 +188,17 @@ def dbg_msp_partition(prm, d_bases, n_words: int, d_offsets, n_reads: int, part:
         _stream(stream)))
 
 
-def dbg_table_plan(prm, d_n_kmers, d_table_offset, stream=None) -> None:
+def dbg_table_plan(prm, d_n_kmers, d_table_offset, d_scratch=None, stream=None) -> None:
     _check("dbg_table_plan", load().dbg_table_plan(ctypes.byref(prm), _ptr(d_n_kmers),
-                                                   _ptr(d_table_offset), _stream(stream)))
+                                                   _ptr(d_table_offset), _ptr(d_scratch), _stream(stream)))
 
 
 def dbg_smem_table_slots(prm) -> int:
     return load().dbg_smem_table_slots(ctypes.byref(prm))
+
+
+def dbg_smem_onchip(prm, n_kmers: int) -> int:
+    return load().dbg_smem_onchip(ctypes.byref(prm), n_kmers)
 
 
 def dbg_smem_workspace_bytes(prm) -> int:
@@ -205,9 +212,10 @@ def dbg_build_subgraphs_smem(prm, part, pid_begin: int, pid_end: int, d_work, wo
         _ptr(d_n_out), _ptr(d_stats), _ptr(d_status), _stream(stream)))
 
 
-def dbg_table_plan_split(prm, d_n_kmers, smem_slots: int, d_table_offset, stream=None) -> None:
-    _check("dbg_table_plan_split", load().dbg_table_plan_split(ctypes.byref(prm), _ptr(d_n_kmers), smem_slots,
-                                                               _ptr(d_table_offset), _stream(stream)))
+def dbg_table_plan_split(prm, d_n_kmers, d_table_offset, d_scratch=None, stream=None) -> None:
+    _check("dbg_table_plan_split", load().dbg_table_plan_split(ctypes.byref(prm), _ptr(d_n_kmers),
+                                                               _ptr(d_table_offset), _ptr(d_scratch),
+                                                               _stream(stream)))
 
 
 def dbg_subgraph_ring_bytes(prm, group_slots: int, max_capacity: int) -> int:

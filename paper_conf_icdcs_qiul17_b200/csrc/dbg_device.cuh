@@ -29,6 +29,37 @@ __host__ __device__ inline int fine_partitions(const dbg_params* prm) {
   return prm->num_partitions * (prm->refine > 1 ? prm->refine : 1);
 }
 
+// Minimizer length of the device's fine partitioning (dbg.h fine_p; 0 = P).
+__host__ __device__ inline int partition_p(const dbg_params* prm) { return prm->fine_p ? prm->fine_p : prm->p; }
+
+// Table capacity of a partition (Sec. IV-A): ceil(lambda/(4 alpha)
+// * N^i_kmer), at least 1 when the partition is not empty.
+__host__ __device__ inline uint64_t table_capacity(double ratio, uint64_t nk) {
+  if (nk == 0) return 0;
+  const double c = ceil(ratio * (double)nk);
+  return c < 1.0 ? 1ull : (uint64_t)c;
+}
+
+// On-chip path (hash.cu): a partition's table lives in one CTA's shared memory
+// ("grouped", 1) when its capacity fits the CTA table, or is split over ns >= 2
+// CTA tables, ns = ceil(1.25 cap / slots) <= max_split; otherwise (0) it takes
+// the global tables.  On-chip counters are 16 bits wide and a vertex's count
+// never exceeds its partition's N^i_kmer, so only partitions with
+// N^i_kmer <= 65535 go on chip.
+constexpr uint64_t kSmemMaxKmers = 65535;
+constexpr int32_t kDefaultSmemSplit = 32, kMaxSmemSplit = 64;
+__host__ __device__ inline uint32_t smem_max_split(const dbg_params* prm) {
+  const int32_t m = prm->smem_split == 0 ? kDefaultSmemSplit : prm->smem_split;
+  return (uint32_t)(m < 1 ? 1 : (m > kMaxSmemSplit ? kMaxSmemSplit : m));
+}
+__host__ __device__ inline uint32_t onchip_tables(uint64_t nk, uint64_t cap, uint64_t slots, uint32_t max_split) {
+  if (nk == 0 || nk > kSmemMaxKmers) return 0;
+  if (cap <= slots) return 1;
+  if (max_split < 2) return 0;
+  const uint64_t ns = (5 * cap + 4 * slots - 1) / (4 * slots);
+  return ns <= max_split ? (uint32_t)ns : 0u;
+}
+
 // MurmurHash3 64-bit finaliser: the partition function of reading I
 // ("superkmer ID ... from the minimizer's hash bit value with a modulo",
 // P:L455-459), and the slot hash of the tables.

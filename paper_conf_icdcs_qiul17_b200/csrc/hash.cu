@@ -45,6 +45,7 @@
 #include <cstdlib>
 
 #include "dbg_device.cuh"
+#include "scan.cuh"
 
 int dbg_sm_count();
 bool dbg_params_ok(const dbg_params* prm);
@@ -299,13 +300,74 @@ __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, 
 // --------------------------------------------------------------- extraction
 
 struct OutArgs {
-  uint32_t np_out;  // the paper's NP: dbg_vertex.pid = fine pid mod NP
+  uint32_t np_out;  // the paper's NP: dbg_vertex.pid = fine pid mod NP ...
+  bool kmer_pid;    // ... or, when fine_p != P, the partition of the vertex's P-minimizer
+  int k, p;
+  FastMod np_mod;
   dbg_vertex* out;
   uint64_t out_cap;
   unsigned long long* n_out;
   unsigned long long* stats;  // distinct, sum_count, sum_edges, checksum
   uint32_t* status;
 };
+
+static OutArgs make_out_args(const dbg_params* prm, dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
+                             dbg_stats* d_stats, uint32_t* d_status) {
+  OutArgs oa;
+  oa.np_out = (uint32_t)prm->num_partitions;
+  oa.kmer_pid = partition_p(prm) != prm->p;
+  oa.k = prm->k;
+  oa.p = prm->p;
+  oa.np_mod = make_fastmod((uint64_t)prm->num_partitions);
+  oa.out = d_out;
+  oa.out_cap = out_cap;
+  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
+  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
+  oa.status = d_status;
+  return oa;
+}
+
+// The paper's partition of a vertex (readings D, E, I, V): fmix64 of the
+// canonical P-minimizer of its canonical K-mer (code = hi:lo, 2K bits, first
+// base most significant) mod NP -- the minimizer of every superkmer that holds
+// the K-mer, on either strand.  With rc the K-mer's reverse complement, the
+// canonical P-mer at offset q is min(code >> 2(K-P-q), rc >> 2q) & mask: two
+// funnel shifts per window, no dependence chain across windows.
+template <typename PT>
+__device__ __forceinline__ uint64_t kmer_minimizer64(uint64_t code, int K, int P) {
+  const uint64_t rc = revcomp64(code, K);
+  const PT mask = (PT)((2ull << (2 * P - 1)) - 1);
+  PT m = (PT)~(PT)0;
+  for (int q = 0, s = 2 * (K - P); q <= K - P; ++q, s -= 2) {
+    const PT f = (PT)(code >> s) & mask, r = (PT)(rc >> (2 * q)) & mask;
+    const PT c = f < r ? f : r;
+    m = c < m ? c : m;
+  }
+  return (uint64_t)m;
+}
+
+template <typename PT>
+__device__ __forceinline__ uint64_t kmer_minimizer128(u128 code, int K, int P) {
+  const u128 rc = revcomp128(code, K);
+  const PT mask = (PT)((2ull << (2 * P - 1)) - 1);
+  PT m = (PT)~(PT)0;
+  for (int q = 0, s = 2 * (K - P); q <= K - P; ++q, s -= 2) {
+    const PT f = (PT)(uint64_t)(code >> s) & mask, r = (PT)(uint64_t)(rc >> (2 * q)) & mask;
+    const PT c = f < r ? f : r;
+    m = c < m ? c : m;
+  }
+  return (uint64_t)m;
+}
+
+__device__ __forceinline__ uint32_t kmer_partition(uint64_t hi, uint64_t lo, const OutArgs& oa) {
+  uint64_t m;
+  if (oa.k <= 31) m = oa.p <= 16 ? kmer_minimizer64<uint32_t>(lo, oa.k, oa.p) : kmer_minimizer64<uint64_t>(lo, oa.k, oa.p);
+  else {
+    const u128 code = ((u128)hi << 64) | lo;
+    m = oa.p <= 16 ? kmer_minimizer128<uint32_t>(code, oa.k, oa.p) : kmer_minimizer128<uint64_t>(code, oa.k, oa.p);
+  }
+  return fast_mod(oa.np_mod, fmix64(m));
+}
 
 struct XShared {
   typename cub::BlockScan<uint32_t, kThreads>::TempStorage scan;
@@ -361,7 +423,7 @@ __device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t
     v.out[0] = a.x; v.out[1] = a.y; v.out[2] = a.z; v.out[3] = a.w;
     v.in[0] = b.x; v.in[1] = b.y; v.in[2] = b.z; v.in[3] = b.w;
     v.count = a.x + a.y + a.z + a.w + tout;  // count = sum(out) + t_out
-    v.pid = pid_of(s) % oa.np_out;
+    v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : pid_of(s) % oa.np_out;
     if (pos < oa.out_cap) oa.out[pos] = v;
     else atomicOr(oa.status, kStatusNoSpace);
     ++pos;
@@ -710,6 +772,7 @@ struct SmemStage {
   typename cub::BlockScan<uint32_t, T>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, T>::TempStorage red;
   unsigned long long base;
+  uint32_t item[4];  // current work item: first, last partition, sub-table j, sub-tables (0: done)
 };
 
 template <int R, int T>
@@ -766,122 +829,163 @@ struct SmemArgs {
   const uint64_t* rec_off;
   const uint64_t* n_kmers;
   int pid0, n_fine, k;  // fine partitions [pid0, pid0 + n_fine)
-  double ratio;      // lambda / (4 alpha)
-  uint64_t slots;    // table slots that fit one CTA
-  FastMod np_mod;    // reported pid = fine pid mod NP
-  uint64_t* P;       // [n_fine + 1] prefix of on-chip capacities (0 for partitions off chip), local index
-  uint32_t* gfirst;  // [n_fine + 2] first (absolute) partition of each group
-  unsigned long long* n_groups;
+  double ratio;         // lambda / (4 alpha)
+  uint64_t slots;       // table slots that fit one CTA
+  uint32_t max_split;   // CTAs (sub-tables) an oversize partition may be split over; < 2: none
+  FastMod np_mod;       // reported pid = fine pid mod NP
+  uint64_t* P;          // [n_fine + 1] prefix of grouped on-chip capacities (0 for the others), local index
+  uint32_t* gfirst;     // [n_fine + 2] first (absolute) partition of each group
+  uint32_t* sp;         // [n_fine] split partitions (absolute ids), ascending
+  uint32_t* ss;         // [n_fine + 1] exclusive prefix of their sub-table counts
+  uint8_t* flag;        // [n_fine] group-start flags
+  unsigned long long *t_gc, *t_sp, *t_fl;  // per-tile sums (scan.cuh), tiles + 1 each
+  unsigned long long* ctr;  // [0] groups, [1] split partitions, [2] split items, [3] work counter
 };
 
-// Capacity of partition p on chip (Sec. IV-A), or 0 if it is
-// empty or does not fit (then it goes to the global-table path).
-__device__ __forceinline__ uint64_t smem_cap(const SmemArgs& a, uint64_t nk) {
-  if (nk == 0) return 0;
-  const double c = ceil(a.ratio * (double)nk);
-  const uint64_t cap = c < 1.0 ? 1ull : (uint64_t)c;
-  return cap <= a.slots ? cap : 0;
+// A partition's table capacity (Sec. IV-A), its grouped on-chip
+// capacity (0 unless onchip_tables == 1) and its sub-table count when split
+// (0 unless onchip_tables >= 2; dbg_device.cuh).
+struct OnChip {
+  uint64_t cap, gc;
+  uint32_t ns;
+};
+__device__ __forceinline__ OnChip on_chip(const SmemArgs& a, uint64_t nk) {
+  OnChip o;
+  o.cap = table_capacity(a.ratio, nk);
+  const uint32_t t = onchip_tables(nk, o.cap, a.slots, a.max_split);
+  o.gc = t == 1 ? o.cap : 0;
+  o.ns = t >= 2 ? t : 0;
+  return o;
 }
 
-// Single CTA: P = prefix of on-chip capacities, then groups of consecutive
-// partitions that share one CTA table.  With H = slots/2 and w(p) =
-// floor(P[p]/H), partition p starts a group iff p == 0, w(p) != w(p-1), or p
-// or p-1 has capacity > H.  A group of small partitions then lies in one
-// H-window and spans < H + H = slots; a large one is alone (<= slots).
-constexpr int kPlanThreads = 512, kPlanItems = 8;
-__global__ void __launch_bounds__(kPlanThreads) smem_plan_kernel(SmemArgs a) {
-  typedef cub::BlockScan<unsigned long long, kPlanThreads> Scan;
-  __shared__ typename Scan::TempStorage tmp;
-  __shared__ unsigned long long carry_p, carry_g, last_cap, last_w;
-  const uint64_t H = a.slots / 2;
-  if (threadIdx.x == 0) {
-    carry_p = 0;
-    carry_g = 0;
-    last_cap = 0;
-    last_w = ~0ull;
-  }
-  __syncthreads();
-  constexpr int kTile = kPlanThreads * kPlanItems;
-  for (int base = 0; base < a.n_fine; base += kTile) {
-    unsigned long long cap[kPlanItems], pre[kPlanItems];
+// The plan (5 launches, scan.cuh tiles): A per-tile sums of the grouped
+// capacities and of the split counts; B scans of those; C writes P, the split
+// list and the group-start flags; D scans the flag counts; E writes gfirst.
+// Groups: with H = slots/2 and w(p) = floor(P[p]/H), partition p starts a
+// group iff p == 0, w(p) != w(p-1), or p or p-1 has capacity > H.  A group of
+// small partitions lies in one H-window and spans < H + H = slots; a larger
+// one is alone; a split or global partition is alone with span 0 (skipped).
+constexpr unsigned long long kSplitOne = 1ull << 32;  // packed (split partitions << 32) | sub-tables
+
+__global__ void __launch_bounds__(kTileThreads) smem_plan_reduce_kernel(SmemArgs a) {
+  typedef cub::BlockReduce<unsigned long long, kTileThreads> Red;
+  __shared__ typename Red::TempStorage tmp;
+  const int base = blockIdx.x * kTileSize;
+  unsigned long long gc = 0, sp = 0;
 #pragma unroll
-    for (int q = 0; q < kPlanItems; ++q) {
-      const int p = base + threadIdx.x * kPlanItems + q;
-      cap[q] = p < a.n_fine ? smem_cap(a, a.n_kmers[a.pid0 + p]) : 0;
+  for (int q = 0; q < kTileItems; ++q) {
+    const int p = base + q * kTileThreads + threadIdx.x;
+    if (p < a.n_fine) {
+      const OnChip o = on_chip(a, a.n_kmers[a.pid0 + p]);
+      gc += o.gc;
+      sp += o.ns ? kSplitOne | o.ns : 0ull;
     }
-    unsigned long long tot;
-    Scan(tmp).ExclusiveSum(cap, pre, tot);
-    __syncthreads();
-    // start flags need the previous partition's capacity and window
-    unsigned long long flag[kPlanItems], gpre[kPlanItems];
-    const unsigned long long cp = carry_p;
+  }
+  gc = Red(tmp).Sum(gc);
+  __syncthreads();
+  sp = Red(tmp).Sum(sp);
+  if (threadIdx.x == 0) {
+    a.t_gc[blockIdx.x] = gc;
+    a.t_sp[blockIdx.x] = sp;
+  }
+}
+
+__global__ void __launch_bounds__(kTileThreads) smem_plan_apply_kernel(SmemArgs a) {
+  typedef cub::BlockScan<unsigned long long, kTileThreads> Scan;
+  typedef cub::BlockReduce<unsigned int, kTileThreads> Red;
+  __shared__ union {
+    typename Scan::TempStorage scan;
+    typename Red::TempStorage red;
+  } tmp;
+  const uint64_t H = a.slots / 2;
+  const int base = blockIdx.x * kTileSize + threadIdx.x * kTileItems;
+  unsigned long long cap[kTileItems], P[kTileItems], sp[kTileItems];
+  uint32_t is_split = 0;
 #pragma unroll
-    for (int q = 0; q < kPlanItems; ++q) {
-      const int p = base + threadIdx.x * kPlanItems + q;
-      const unsigned long long P = cp + pre[q];
-      unsigned long long pcap, pw;
+  for (int q = 0; q < kTileItems; ++q) {
+    const int p = base + q;
+    const OnChip o = on_chip(a, p < a.n_fine ? a.n_kmers[a.pid0 + p] : 0ull);
+    cap[q] = o.cap;
+    P[q] = o.gc;
+    sp[q] = o.ns ? kSplitOne | o.ns : 0ull;
+    is_split |= (o.ns ? 1u : 0u) << q;
+  }
+  unsigned long long tot_gc, tot_sp;
+  Scan(tmp.scan).ExclusiveSum(P, P, tot_gc);
+  __syncthreads();
+  Scan(tmp.scan).ExclusiveSum(sp, sp, tot_sp);
+  __syncthreads();
+  const unsigned long long o_gc = a.t_gc[blockIdx.x], o_sp = a.t_sp[blockIdx.x];
+  unsigned int nflag = 0;
+#pragma unroll
+  for (int q = 0; q < kTileItems; ++q) {
+    const int p = base + q;
+    if (p >= a.n_fine) break;
+    const unsigned long long Pp = o_gc + P[q];
+    a.P[p] = Pp;
+    if (is_split >> q & 1u) {
+      const unsigned long long x = o_sp + sp[q];
+      a.sp[x >> 32] = (uint32_t)(a.pid0 + p);
+      a.ss[x >> 32] = (uint32_t)x;
+    }
+    bool f = p == 0;
+    if (!f) {
+      unsigned long long pcap, pP;
       if (q > 0) {
         pcap = cap[q - 1];
-        pw = (cp + pre[q - 1]) / H;
-      } else {
-        // neighbour item lives in the previous thread (or tile)
-        pcap = 0;
-        pw = 0;
+        pP = o_gc + P[q - 1];
+      } else {  // the neighbour belongs to another thread or tile: recompute it
+        const OnChip o = on_chip(a, a.n_kmers[a.pid0 + p - 1]);
+        pcap = o.cap;
+        pP = Pp - o.gc;
       }
-      flag[q] = 0;
-      if (p < a.n_fine) {
-        a.P[p] = P;
-        flag[q] = (P / H != pw) || cap[q] > H || pcap > H;
-      }
-      (void)pw;
+      f = Pp / H != pP / H || cap[q] > H || pcap > H;
     }
-    // fix item 0 with the previous thread's last item (shuffle within warps, smem across)
-    {
-      const unsigned long long my_last_cap = cap[kPlanItems - 1];
-      const unsigned long long my_last_w = (cp + pre[kPlanItems - 1]) / H;
-      __shared__ unsigned long long sh_cap[kPlanThreads], sh_w[kPlanThreads];
-      sh_cap[threadIdx.x] = my_last_cap;
-      sh_w[threadIdx.x] = my_last_w;
-      __syncthreads();
-      const int p0 = base + threadIdx.x * kPlanItems;
-      if (p0 < a.n_fine) {
-        unsigned long long pcap, pw;
-        if (threadIdx.x > 0) {
-          pcap = sh_cap[threadIdx.x - 1];
-          pw = sh_w[threadIdx.x - 1];
-        } else {
-          pcap = last_cap;
-          pw = last_w;
-        }
-        const unsigned long long P = cp + pre[0];
-        flag[0] = p0 == 0 || (P / H != pw) || cap[0] > H || pcap > H;
-      }
-      __syncthreads();
-      if (threadIdx.x == kPlanThreads - 1) {
-        last_cap = my_last_cap;
-        last_w = my_last_w;
-      }
-    }
-    unsigned long long gtot;
-    Scan(tmp).ExclusiveSum(flag, gpre, gtot);
-    const unsigned long long cg = carry_g;
-#pragma unroll
-    for (int q = 0; q < kPlanItems; ++q) {
-      const int p = base + threadIdx.x * kPlanItems + q;
-      if (p < a.n_fine && flag[q]) a.gfirst[cg + gpre[q]] = (uint32_t)(a.pid0 + p);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      carry_p += tot;
-      carry_g += gtot;
-    }
-    __syncthreads();
+    a.flag[p] = f;
+    nflag += f;
   }
+  nflag = Red(tmp.red).Sum(nflag);
   if (threadIdx.x == 0) {
-    a.P[a.n_fine] = carry_p;
-    a.gfirst[carry_g] = (uint32_t)(a.pid0 + a.n_fine);
-    *a.n_groups = carry_g;
+    a.t_fl[blockIdx.x] = nflag;
+    if (blockIdx.x == gridDim.x - 1) {
+      const unsigned long long s = o_sp + tot_sp;
+      a.P[a.n_fine] = o_gc + tot_gc;
+      a.ss[s >> 32] = (uint32_t)s;
+      a.ctr[1] = s >> 32;
+      a.ctr[2] = (uint32_t)s;
+    }
   }
+}
+
+__global__ void __launch_bounds__(kTileThreads) smem_plan_groups_kernel(SmemArgs a) {
+  typedef cub::BlockScan<unsigned int, kTileThreads> Scan;
+  __shared__ typename Scan::TempStorage tmp;
+  const int base = blockIdx.x * kTileSize + threadIdx.x * kTileItems;
+  unsigned int f[kTileItems];
+#pragma unroll
+  for (int q = 0; q < kTileItems; ++q) f[q] = base + q < a.n_fine ? a.flag[base + q] : 0u;
+  unsigned int tot;
+  Scan(tmp).ExclusiveSum(f, f, tot);
+  const unsigned long long o = a.t_fl[blockIdx.x];
+#pragma unroll
+  for (int q = 0; q < kTileItems; ++q) {
+    const int p = base + q;
+    if (p < a.n_fine && a.flag[p]) a.gfirst[o + f[q]] = (uint32_t)(a.pid0 + p);
+  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
+    a.gfirst[o + tot] = (uint32_t)(a.pid0 + a.n_fine);
+    a.ctr[0] = o + tot;
+    a.ctr[3] = 0;  // work counter of smem_subgraph_kernel
+  }
+}
+
+// Sub-table of a K-mer in a split partition: a hash independent of the slot hash.
+template <typename Code>
+__device__ __forceinline__ uint32_t sub_table(Code code, uint32_t n) {
+  uint64_t x;
+  if constexpr (sizeof(Code) == 8) x = (uint64_t)code;
+  else x = (uint64_t)code ^ ((uint64_t)(code >> 64) * 0x9e3779b97f4a7c15ull);
+  return __umulhi((uint32_t)(fmix64(x) >> 32), n);
 }
 
 // A group of consecutive fine partitions shares one CTA table: each partition
@@ -907,10 +1011,43 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   }
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
   bool ok = true;
-  const uint64_t n_groups = *a.n_groups;
-  for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-    const int first = (int)a.gfirst[g], last = (int)a.gfirst[g + 1];
-    const uint64_t P0 = a.P[first - a.pid0], span = a.P[last - a.pid0] - P0;
+  const uint64_t n_split = a.ctr[2], n_items = n_split + a.ctr[0];
+  // Work items, taken from a global counter: first the sub-tables of the split
+  // partitions (the longest items), then the groups.
+  for (;;) {
+    __syncthreads();  // the previous item (staging, st.item) is finished
+    if (threadIdx.x == 0) {
+      const uint64_t g = atomicAdd(a.ctr + 3, 1ull);
+      uint32_t first = 0, last = 0, j = 0, ns = 1;
+      if (g < n_split) {  // split partition i with ss[i] <= g < ss[i+1]
+        uint32_t lo = 0, hi = (uint32_t)a.ctr[1];
+        while (hi - lo > 1) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (a.ss[mid] <= g) lo = mid;
+          else hi = mid;
+        }
+        first = a.sp[lo];
+        last = first + 1;
+        j = (uint32_t)g - a.ss[lo];
+        ns = a.ss[lo + 1] - a.ss[lo];
+      } else if (g < n_items) {
+        first = a.gfirst[g - n_split];
+        last = a.gfirst[g - n_split + 1];
+      } else {
+        ns = 0;  // done
+      }
+      st.item[0] = first;
+      st.item[1] = last;
+      st.item[2] = j;
+      st.item[3] = ns;
+    }
+    __syncthreads();
+    const uint32_t sub_n = st.item[3], sub_j = st.item[2];
+    if (sub_n == 0) break;
+    const bool split = sub_n > 1;
+    const int first = (int)st.item[0], last = (int)st.item[1];
+    const uint64_t P0 = split ? 0 : a.P[first - a.pid0];
+    const uint64_t span = split ? a.slots : a.P[last - a.pid0] - P0;
     if (span == 0) continue;  // nothing on chip in this group
     const uint64_t r0 = a.rec_off[first], nrec = a.rec_off[last] - r0;
     for (uint64_t rb = 0; rb < nrec; rb += kRecBatch) {
@@ -931,11 +1068,17 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             st.w[4 * q + 2][j] = x.z;
             st.w[4 * q + 3][j] = x.w;
           }
-          const uint32_t pid = (st.w[0][j] >> 10) - a.pid0;
-          const uint64_t pp = a.P[pid], pc = a.P[pid + 1] - pp;
-          st.t0[j] = (uint32_t)(pp - P0);
-          st.cap[j] = (uint32_t)pc;
-          cnt[v] = pc ? st.w[0][j] & 255u : 0u;  // off-chip partition: skipped here
+          if (split) {  // one partition, the whole CTA table
+            st.t0[j] = 0;
+            st.cap[j] = (uint32_t)a.slots;
+            cnt[v] = st.w[0][j] & 255u;
+          } else {
+            const uint32_t pid = (st.w[0][j] >> 10) - a.pid0;
+            const uint64_t pp = a.P[pid], pc = a.P[pid + 1] - pp;
+            st.t0[j] = (uint32_t)(pp - P0);
+            st.cap[j] = (uint32_t)pc;
+            cnt[v] = pc ? st.w[0][j] & 255u : 0u;  // off-chip partition: skipped here
+          }
         }
       }
       uint32_t excl[kRPT], total;
@@ -976,7 +1119,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           const Code code = is_fwd ? fwd : rc;
           const int o = is_fwd ? (succ >= 0 ? succ : 4) : (pred >= 0 ? 3 - pred : 4);
           const int i = is_fwd ? pred : (succ >= 0 ? 3 - succ : -1);
-          ok &= smem_upsert<Code>(tk, tf, cap, code, o, i, pid);
+          if (sub_n == 1 || sub_table(code, sub_n) == sub_j) ok &= smem_upsert<Code>(tk, tf, cap, code, o, i, pid);
           if (++kid >= k1) break;
           if (++t < n) {  // next K-mer of the same record: roll one base
             fwd = ((fwd << 2) | (Code)succ) & mask;
@@ -1046,7 +1189,8 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
         v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
         v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
-        v.pid = fast_mod(a.np_mod, f[5]);  // fine pid recorded by the inserting thread, mod NP
+        // fine pid recorded by the inserting thread, mod NP (or from the P-minimizer, reading V)
+        v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, f[5]);
         kp[0] = 0;  // clean-on-extract
         if (KW == 2) kp[1] = 0;
 #pragma unroll
@@ -1198,13 +1342,7 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   a.pid_end = pid_end;
   a.k = prm->k;
   a.status = d_status;
-  OutArgs oa;
-  oa.np_out = (uint32_t)prm->num_partitions;
-  oa.out = d_out;
-  oa.out_cap = out_cap;
-  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
-  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
-  oa.status = d_status;
+  const OutArgs oa = make_out_args(prm, d_out, out_cap, d_n_out, d_stats, d_status);
   const int grid = dbg_sm_count() * 4;
   if (prm->k <= 31) extract_kernel<1><<<grid, kThreads, 0, stream>>>(a, oa);
   else extract_kernel<2><<<grid, kThreads, 0, stream>>>(a, oa);
@@ -1269,10 +1407,46 @@ static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_
   }
 }
 
+extern "C" int32_t dbg_smem_onchip(const dbg_params* prm, uint64_t n_kmers) {
+  if (!dbg_params_ok(prm) || !(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return -1;
+  const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
+  return (int32_t)onchip_tables(n_kmers, table_capacity(ratio, n_kmers), dbg_smem_table_slots(prm),
+                                smem_max_split(prm));
+}
+
+static uint64_t al16(uint64_t x) { return (x + 15) & ~(uint64_t)15; }
+
+// Workspace: P | 3 tile-sum arrays | counters | gfirst | sp | ss | flags.
+static uint64_t smem_workspace(uint64_t n, SmemArgs* a, char* ws) {
+  const uint64_t tiles = (uint64_t)scan_tiles((int)n) + 1;
+  uint64_t o = 0;
+  auto take = [&](uint64_t bytes) { const uint64_t at = o; o += al16(bytes); return ws + at; };
+  char* P = take(8 * (n + 1));
+  char* t_gc = take(8 * tiles);
+  char* t_sp = take(8 * tiles);
+  char* t_fl = take(8 * tiles);
+  char* ctr = take(64);
+  char* gfirst = take(4 * (n + 2));
+  char* sp = take(4 * n + 4);
+  char* ss = take(4 * (n + 1));
+  char* flag = take(n + 1);
+  if (a) {
+    a->P = reinterpret_cast<uint64_t*>(P);
+    a->t_gc = reinterpret_cast<unsigned long long*>(t_gc);
+    a->t_sp = reinterpret_cast<unsigned long long*>(t_sp);
+    a->t_fl = reinterpret_cast<unsigned long long*>(t_fl);
+    a->ctr = reinterpret_cast<unsigned long long*>(ctr);
+    a->gfirst = reinterpret_cast<uint32_t*>(gfirst);
+    a->sp = reinterpret_cast<uint32_t*>(sp);
+    a->ss = reinterpret_cast<uint32_t*>(ss);
+    a->flag = reinterpret_cast<uint8_t*>(flag);
+  }
+  return o;
+}
+
 extern "C" uint64_t dbg_smem_workspace_bytes(const dbg_params* prm) {
   if (!prm) return 0;
-  const uint64_t n = (uint64_t)fine_partitions(prm);
-  return 8 * (n + 1) + 4 * (n + 2) + 16 + 64;
+  return smem_workspace((uint64_t)fine_partitions(prm), nullptr, nullptr);
 }
 
 extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_partition_set* part,
@@ -1297,18 +1471,16 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   a.k = prm->k;
   a.ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   a.slots = dbg_smem_table_slots(prm);
-  char* ws = static_cast<char*>(d_work);
-  a.P = reinterpret_cast<uint64_t*>(ws);
-  a.n_groups = reinterpret_cast<unsigned long long*>(ws + 8 * ((uint64_t)a.n_fine + 1));
-  a.gfirst = reinterpret_cast<uint32_t*>(ws + 8 * ((uint64_t)a.n_fine + 1) + 16);
-  smem_plan_kernel<<<1, kPlanThreads, 0, stream>>>(a);
-  OutArgs oa;
-  oa.np_out = (uint32_t)prm->num_partitions;
-  oa.out = d_out;
-  oa.out_cap = out_cap;
-  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
-  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
-  oa.status = d_status;
+  a.max_split = smem_max_split(prm);
+  smem_workspace((uint64_t)a.n_fine, &a, static_cast<char*>(d_work));
+  const int tiles = scan_tiles(a.n_fine);
+  smem_plan_reduce_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
+  tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_gc, tiles);
+  tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_sp, tiles);
+  smem_plan_apply_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
+  tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_fl, tiles);
+  smem_plan_groups_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
+  const OutArgs oa = make_out_args(prm, d_out, out_cap, d_n_out, d_stats, d_status);
   cudaError_t e;
   if (prm->k <= 31) e = launch_smem<uint64_t, 4>(a, oa, stream);
   else if (prm->k <= 39) e = launch_smem<u128, 4>(a, oa, stream);
@@ -1377,13 +1549,7 @@ extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_parti
   a.work = reinterpret_cast<unsigned long long*>(ws + 8 * (g + kLagX + 3));
   a.done = reinterpret_cast<uint32_t*>(ws + 8 * (g + kLagX + 3) + 16);
   a.gfirst = a.done + 3 * g;
-  OutArgs oa;
-  oa.np_out = (uint32_t)prm->num_partitions;
-  oa.out = d_out;
-  oa.out_cap = out_cap;
-  oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
-  oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
-  oa.status = d_status;
+  const OutArgs oa = make_out_args(prm, d_out, out_cap, d_n_out, d_stats, d_status);
   subgraph_plan_kernel<<<1, kThreads, 0, stream>>>(a, d_status);
   const int grid = dbg_sm_count() * 4;
   if (prm->k <= 31) subgraph_kernel<uint64_t, 4><<<grid, kThreads, 0, stream>>>(a, oa);

@@ -23,13 +23,14 @@
 // The paper computed only "superkmer ids and offsets" on the GPU and left
 // the irregular copy to the CPU; here both run in this kernel.
 //
-// Pass 2, scan_kernel: record offsets per partition (exclusive prefix sum).
+// Pass 2, exclusive_scan (scan.cuh): record offsets per partition.
 // Pass 3, scatter_kernel: counting-sort scatter of the staged records into
 // their partitions' contiguous ranges (CTA histogram -> one global
 // reservation per partition per tile).
 #include <cub/block/block_scan.cuh>
 
 #include "dbg_device.cuh"
+#include "scan.cuh"
 
 namespace dbg {
 
@@ -218,51 +219,6 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   }
 }
 
-// Exclusive prefix sum out[0..n] of f(in[0..n-1]) in one CTA (n = number of
-// fine partitions: up to a few 10^5); f = identity (record offsets) or the
-// table capacity of Sec. IV-A.  512 threads x 8 consecutive items per pass.
-constexpr int kScanThreads = 512;
-constexpr int kScanItems = 8;
-template <bool kCapacity>
-__global__ void __launch_bounds__(kScanThreads) scan_kernel(const uint64_t* __restrict__ in,
-                                                            uint64_t* __restrict__ out, int n,
-                                                            double ratio, uint64_t skip_upto) {
-  using Scan = cub::BlockScan<unsigned long long, kScanThreads>;
-  __shared__ typename Scan::TempStorage tmp;
-  __shared__ unsigned long long carry;
-  if (threadIdx.x == 0) carry = 0;
-  __syncthreads();
-  constexpr int kTile = kScanThreads * kScanItems;
-  for (int base = 0; base < n; base += kTile) {
-    unsigned long long v[kScanItems];
-#pragma unroll
-    for (int q = 0; q < kScanItems; ++q) {
-      const int i = base + threadIdx.x * kScanItems + q;
-      v[q] = 0;
-      if (i < n) {
-        v[q] = in[i];
-        if (kCapacity && v[q]) {
-          // capacity_i = ceil(lambda / (4 alpha) * N^i_kmer), at least 1
-          const double c = ceil(ratio * (double)v[q]);
-          v[q] = c < 1.0 ? 1ull : (unsigned long long)c;
-          if (v[q] <= skip_upto) v[q] = 0;  // built on chip (dbg_table_plan_split)
-        }
-      }
-    }
-    unsigned long long total;
-    Scan(tmp).ExclusiveSum(v, v, total);
-#pragma unroll
-    for (int q = 0; q < kScanItems; ++q) {
-      const int i = base + threadIdx.x * kScanItems + q;
-      if (i < n) out[i] = carry + v[q];
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) carry += total;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) out[n] = carry;
-}
-
 // Pass 3: scatter staged records into partition order.
 constexpr int kScatterThreads = 256;
 constexpr int kScatterPer = 8;  // records per thread per tile
@@ -331,7 +287,8 @@ int dbg_sm_count() {
 
 bool dbg_params_ok(const dbg_params* prm) {
   return prm && prm->k >= 1 && prm->k <= 63 && (prm->k & 1) && prm->p >= 1 && prm->p <= prm->k &&
-         prm->p <= 31 && prm->num_partitions >= 1 && prm->refine >= 0 &&
+         prm->p <= 31 && prm->fine_p >= 0 && prm->fine_p <= prm->k && prm->fine_p <= 31 &&
+         prm->num_partitions >= 1 && prm->refine >= 0 &&
          (uint64_t)prm->num_partitions * (uint64_t)(prm->refine > 1 ? prm->refine : 1) <= kMaxPid;
 }
 
@@ -363,9 +320,9 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
     a.offsets = d_offsets;
     a.n_reads = n_reads;
     a.k = prm->k;
-    a.p = prm->p;
+    a.p = partition_p(prm);  // the fine partitioning's minimizer (dbg.h fine_p)
     a.np = np;
-    a.w = prm->k - prm->p + 1;
+    a.w = prm->k - a.p + 1;
     a.rec_words = R;
     a.max_kmers = record_max_kmers(prm->k);
     a.mod = make_fastmod((uint64_t)np);
@@ -382,11 +339,14 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
       const uint64_t want = (n_reads + kMspThreads - 1) / kMspThreads;
       const uint64_t cap = (uint64_t)dbg_sm_count() * 8;
       const int grid = (int)(want < cap ? want : cap);
-      const cudaError_t e = prm->p <= 16 ? launch_msp<uint32_t>(a, grid, stream)
+      const cudaError_t e = a.p <= 16 ? launch_msp<uint32_t>(a, grid, stream)
                                          : launch_msp<uint64_t>(a, grid, stream);
       if (e != cudaSuccess) return DBG_ECUDA;
     }
-    scan_kernel<false><<<1, kScanThreads, 0, stream>>>(part->d_n_records, part->d_record_offset, np, 0.0, 0);
+    // d_fill is idle until pass 2 (which zeroes it): scratch for the tile sums
+    if (exclusive_scan(IdentityOp{part->d_n_records}, np, part->d_record_offset,
+                       reinterpret_cast<unsigned long long*>(part->d_fill), stream) != cudaSuccess)
+      return DBG_ECUDA;
   } else {
     // pass 3: scatter (requires staged <= staging_cap; the caller checks sum(n_records))
     if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
@@ -408,21 +368,24 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-extern "C" dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers,
-                                     uint64_t* d_table_offset, cudaStream_t stream) {
+static dbg_status table_plan(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t slots,
+                             uint64_t* d_table_offset, uint64_t* d_scratch, cudaStream_t stream) {
   if (!dbg_params_ok(prm) || !d_n_kmers || !d_table_offset) return DBG_EINVAL;
   if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
   const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
-  scan_kernel<true><<<1, kScanThreads, 0, stream>>>(d_n_kmers, d_table_offset, fine_partitions(prm), ratio, 0);
-  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+  const cudaError_t e = exclusive_scan(CapacityOp{d_n_kmers, ratio, slots, smem_max_split(prm)},
+                                       fine_partitions(prm), d_table_offset,
+                                       reinterpret_cast<unsigned long long*>(d_scratch), stream);
+  return e == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-extern "C" dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t smem_slots,
-                                           uint64_t* d_table_offset, cudaStream_t stream) {
-  if (!dbg_params_ok(prm) || !d_n_kmers || !d_table_offset) return DBG_EINVAL;
-  if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
-  const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
-  scan_kernel<true><<<1, kScanThreads, 0, stream>>>(d_n_kmers, d_table_offset, fine_partitions(prm), ratio,
-                                                    smem_slots);
-  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+extern "C" dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t* d_table_offset,
+                                     uint64_t* d_scratch, cudaStream_t stream) {
+  return table_plan(prm, d_n_kmers, 0, d_table_offset, d_scratch, stream);
+}
+
+extern "C" dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t* d_table_offset,
+                                           uint64_t* d_scratch, cudaStream_t stream) {
+  if (!prm) return DBG_EINVAL;
+  return table_plan(prm, d_n_kmers, dbg_smem_table_slots(prm), d_table_offset, d_scratch, stream);
 }

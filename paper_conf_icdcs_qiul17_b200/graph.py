@@ -7,17 +7,18 @@ libdbg.so kernels:
     a1     DbgBuilder.upload     H2D copy of the packed reads
     a2-a4  DbgBuilder.msp        dbg_msp_partition pass 1 (minimizers, superkmers,
                                  staging, sizes) -> size readback -> pass 2 (scatter)
-    a5     DbgBuilder.plan       dbg_table_plan (lambda/(4 alpha) N^i_kmer)
-    a5-a7  DbgBuilder.step2      dbg_build_subgraphs: zero + hash + extract of every
-                                 partition in one persistent kernel through an
-                                 L2-resident ring of tables ("fused", the default), or
-                                 dbg_hash_build + dbg_extract_graph over batches of
-                                 partitions with resident tables ("resident")
+    a5     DbgBuilder.plan       dbg_table_plan[_split] (lambda/(4 alpha) N^i_kmer)
+    a5-a7  DbgBuilder.step2      mode "smem" (the default): dbg_build_subgraphs_smem builds
+                                 every partition whose table fits on chip (grouped, or split
+                                 over several CTAs) in shared memory, then
+                                 dbg_hash_build_list + dbg_extract_graph build the remaining
+                                 (oversize) partitions in global tables, in batches;
+                                 mode "resident": dbg_hash_build + dbg_extract_graph for all;
+                                 mode "fused": dbg_build_subgraphs (L2 ring of tables)
     a7     DbgBuilder.vertices   dbg_sort_vertices + D2H
 
-The paper builds "one partition at a time"; the fused
-mode streams groups of consecutive partitions (~group_slots table slots each)
-through a ring of L2-sized regions, each table sized by Property 1.
+The paper builds "one partition at a time"; here the
+device works on NP*refine fine partitions (dbg.h), many at once.
 """
 from __future__ import annotations
 
@@ -70,7 +71,8 @@ class DbgBuilder:
 
     def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
                  device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
-                 mode: str = "smem", group_slots: int = 1 << 19, refine: int = 1):
+                 mode: str = "smem", group_slots: int = 1 << 19, refine: int = 1, smem_split: int = 0,
+                 fine_p: int = 0):
         if k % 2 == 0 or not 1 <= k <= 63:
             raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
         if not 1 <= p <= min(k, 31):
@@ -84,7 +86,9 @@ class DbgBuilder:
         self.group_slots = int(group_slots)  # fused mode: table slots per ring group (L2 sizing)
         self.total_slots = 0
         self.owned = (0, self.np)  # fine partitions this builder hashes (multi-GPU: a shard)
-        self.prm = _lib.params(k, p, num_partitions, lam, alpha, self.refine)
+        self.smem_split = int(smem_split)  # 0: library default (dbg_params.smem_split)
+        self.fine_p = int(fine_p)          # 0: P (dbg_params.fine_p)
+        self.prm = _lib.params(k, p, num_partitions, lam, alpha, self.refine, self.smem_split, self.fine_p)
         self.device = torch.device(device)
         _lib.load()
         self.rec_words = _lib.dbg_record_words(self.prm)
@@ -207,25 +211,26 @@ class DbgBuilder:
     # ------------------------------------------------------------------ a5
     def plan(self, stream=None) -> list[tuple[int, int]]:
         stream = stream or torch.cuda.current_stream(self.device)
-        _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, stream)
+        ev = self._mark("plan", stream)
+        # d_fill is idle after the scatter: scratch of the multi-CTA scan
+        if self.mode == "smem":  # on-chip partitions need no global table
+            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
+        else:
+            _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
+        self._done(ev, stream)
         key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha, self.mode, self.owned)
-        if self._caps_key != key:  # host copy of the same C sizing function (dbg_table_capacity)
+        if self._caps_key != key:  # host copy of the same C sizing functions (per distinct size)
             nz = np.nonzero(self.part_kmers)[0]
             self.caps = np.zeros(self.np, dtype=np.int64)
             uniq, inv = np.unique(self.part_kmers[nz], return_inverse=True)
-            self.caps[nz] = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in uniq],
-                                     dtype=np.int64)[inv]
-            if self.mode == "smem":  # on-chip partitions need no global table (dbg_table_plan_split)
-                self.caps[self.caps <= _lib.dbg_smem_table_slots(self.prm)] = 0
+            cap_u = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in uniq], dtype=np.int64)
+            if self.mode == "smem":
+                cap_u[np.array([_lib.dbg_smem_onchip(self.prm, int(n)) > 0 for n in uniq], dtype=bool)] = 0
+            self.caps[nz] = cap_u[inv]
             lo, hi = self.owned
             self.caps[:lo] = 0
             self.caps[hi:] = 0
             self._caps_key = key
-        if self.mode == "smem":
-            ev = self._mark("plan", stream)
-            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, _lib.dbg_smem_table_slots(self.prm),
-                                      self.d_tab_off, stream)
-            self._done(ev, stream)
         self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
         self.tab_host[1:] = np.cumsum(self.caps)
         if self.mode == "fused":
@@ -271,31 +276,6 @@ class DbgBuilder:
                 grown.zero_()
             self._dirty = False
         return grown
-
-    def load_exchanged(self, received: torch.Tensor, n_received: int, global_records: np.ndarray,
-                       global_kmers: np.ndarray, owned: tuple[int, int], stream=None) -> None:
-        """Multi-GPU: after the record exchange, make this builder's partition set describe only
-        the owned fine partitions [lo, hi) (records received from every rank, scattered into
-        partition order by dbg_msp_partition pass 2; sizes summed over ranks)."""
-        stream = stream or torch.cuda.current_stream(self.device)
-        lo, hi = owned
-        self.owned = (lo, hi)
-        rec = np.zeros(self.np, dtype=np.int64)
-        kmr = np.zeros(self.np, dtype=np.int64)
-        rec[lo:hi] = global_records[lo:hi]
-        kmr[lo:hi] = global_kmers[lo:hi]
-        off = np.zeros(self.np + 1, dtype=np.int64)
-        off[1:] = np.cumsum(rec)
-        assert int(off[-1]) == n_received, (int(off[-1]), n_received)
-        self.part_records, self.part_kmers = rec, kmr
-        with torch.cuda.stream(stream):
-            self.d_n_records.copy_(torch.from_numpy(rec), non_blocking=True)
-            self.d_n_kmers.copy_(torch.from_numpy(kmr), non_blocking=True)
-            self.d_rec_off.copy_(torch.from_numpy(off), non_blocking=True)
-            self.d_staged.fill_(n_received)
-        self.staging = received
-        self.records = _grow(self.records, n_received * self.rec_words, torch.int32, self.device, 1.05)
-        _lib.dbg_msp_partition(self.prm, 1, 1, self.d_rec_off, 0, self.part_set(True), stream)
 
     # ------------------------------------------------------------------ a5-a7
     def reset_output(self, cap: int, stream=None) -> None:
@@ -403,7 +383,8 @@ class DbgBuilder:
             if st == _lib.DBG_ETABLEFULL:  # reading O: rebuild at capacity N^i_kmer (tables are clean again)
                 if self.prm.lambda_ / (4 * self.prm.alpha) >= 1.0:
                     raise _lib.DbgError("dbg_hash_build", st, "table full at capacity >= N^i_kmer")
-                self.prm = _lib.params(self.k, self.p, self.np_out, 2.0, 0.5, self.refine)
+                self.prm = _lib.params(self.k, self.p, self.np_out, 2.0, 0.5, self.refine, self.smem_split,
+                                       self.fine_p)
                 self.plan(stream)
                 continue
             if st != _lib.DBG_OK:
@@ -427,16 +408,34 @@ def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 
     return max(1, min(f, 4_194_303 // num_partitions))
 
 
+def auto_fine_p(n_kmers: int, k: int, p: int, lam: float = 2.0, alpha: float = 0.5) -> int:
+    """Minimizer length of the device's fine partitioning (dbg_params.fine_p): the smallest P' >= P
+    with 4^P' >= 4 (K - P' + 1) N / slots.  A P'-mer occurs about 2G / 4^P' times in a genome of G
+    bases and a lexicographically small one is the minimizer of about K - P' + 1 K-mers per
+    occurrence, so at coverage N / G its partition holds about 2 (K - P' + 1) N / 4^P' K-mers; the
+    rule keeps that below half a CTA table even for the most frequent minimizers."""
+    slots = _lib.dbg_smem_table_slots(_lib.params(k, p, 1, lam, alpha))
+    ratio = max(lam / (4 * alpha), 1e-9)
+    for q in range(p, min(k, 31) + 1):
+        if 4.0 ** q >= 4.0 * (k - q + 1) * n_kmers * ratio / slots:
+            return q
+    return min(k, 31)
+
+
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
                 lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
                 table_budget_bytes: int | None = None, mode: str = "smem",
-                group_slots: int = 1 << 19, refine: int | str = "auto") -> GraphResult:
+                group_slots: int = 1 << 19, refine: int | str = "auto", smem_split: int = 0,
+                fine_p: int | str = "auto") -> GraphResult:
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
+    lens = np.diff(np.asarray(offsets, dtype=np.int64))
+    n_kmers = int(np.maximum(lens - k + 1, 0).sum())
     if refine == "auto":
-        lens = np.diff(np.asarray(offsets, dtype=np.int64))
-        refine = auto_refine(int(np.maximum(lens - k + 1, 0).sum()), k, p, num_partitions, lam, alpha) \
-            if mode == "smem" else 1
-    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots, refine)
+        refine = auto_refine(n_kmers, k, p, num_partitions, lam, alpha) if mode == "smem" else 1
+    if fine_p == "auto":
+        fine_p = auto_fine_p(n_kmers, k, p, lam, alpha) if mode == "smem" else 0
+    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots, refine,
+                         smem_split, fine_p)
     packed = encode_reads(seq)
     d_bases, d_offsets = builder.upload(packed, offsets)
     return builder.build(d_bases, d_offsets, sort=sort)

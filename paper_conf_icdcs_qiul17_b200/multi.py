@@ -86,7 +86,7 @@ def bench_main(args, metric: str, unit: str) -> int:
     """`bench.py` under torchrun (WORLD_SIZE > 1): weak scaling -- every rank owns a read set of the
     configuration's size (same genome, its own reads), so the job builds the graph of world x reads."""
     from synth import make_config
-    from . import DbgBuilder, auto_refine, encode_reads, _lib
+    from . import DbgBuilder, auto_fine_p, auto_refine, encode_reads, _lib
 
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
@@ -99,8 +99,9 @@ def bench_main(args, metric: str, unit: str) -> int:
     n_kmers = rs.n_kmers()
     refine = args.refine if args.refine is not None else auto_refine(n_kmers, rs.k, rs.p, rs.num_partitions,
                                                                       args.lam, args.alpha)
+    fine_p = args.fine_p if args.fine_p is not None else auto_fine_p(n_kmers, rs.k, rs.p, args.lam, args.alpha)
     b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, "smem",
-                   args.group_slots, refine)
+                   args.group_slots, refine, args.smem_split, fine_p)
     stream = torch.cuda.current_stream(dev)
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)

@@ -28,7 +28,7 @@ def _declared():
 
 def test_exports_every_declared_symbol(lib):
     names = _declared()
-    assert len(names) == 25
+    assert len(names) == 26
     raw = lib.load()
     for n in names:
         assert hasattr(raw, n), n
@@ -36,7 +36,7 @@ def test_exports_every_declared_symbol(lib):
 
 
 def test_abi_and_sizes(lib):
-    assert lib.dbg_abi_version() == 2
+    assert lib.dbg_abi_version() == 3
     p31 = lib.params(31, 11, 16)
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
@@ -65,6 +65,40 @@ def test_table2_sizing_pin(lib):
     assert lib.dbg_table_capacity(lib.params(31, 11, 16, 1.0, 0.5), 1001) == 501
     assert lib.dbg_table_capacity(prm, 0) == 0
     assert lib.dbg_table_capacity(lib.params(31, 11, 16, 0.001, 0.5), 10) == 1
+
+
+def test_onchip_placement_rule(lib):
+    """dbg.h dbg_smem_onchip: grouped (1) while the Property-1 capacity fits a CTA table, split over
+    ceil(1.25 c / slots) <= smem_split CTAs above that, global (0) past the split limit or when
+    N^i_kmer > 65535 (16-bit on-chip counters)."""
+    prm = lib.params(31, 11, 16)              # capacity = N^i_kmer
+    S = lib.dbg_smem_table_slots(prm)
+    assert S >= 1024 and S % 64 == 0
+    on = lambda prm, n: lib.dbg_smem_onchip(prm, n)
+    assert on(prm, 0) == 0 and on(prm, 1) == 1 and on(prm, S) == 1
+    assert on(prm, S + 1) == 2                 # ceil(1.25 (S+1) / S)
+    assert on(prm, 2 * S) == 3 and on(prm, (8 * S) // 5) == 2 and on(prm, (8 * S) // 5 + 1) == 3
+    assert on(prm, 65535) == -(-5 * 65535 // (4 * S)) and on(prm, 65536) == 0
+    assert on(lib.params(31, 11, 16, smem_split=1), S + 1) == 0
+    two = lib.params(31, 11, 16, smem_split=2)
+    assert on(two, (8 * S) // 5) == 2 and on(two, (8 * S) // 5 + 1) == 0
+    half = lib.params(31, 11, 16, 1.0, 0.5)   # capacity = ceil(N / 2)
+    assert on(half, 2 * S) == 1 and on(half, 2 * S + 1) == 2
+    assert on(lib.params(30, 11, 16), 10) == -1
+
+
+def test_auto_fine_p_rule(lib):
+    """graph.auto_fine_p: the smallest P' >= P with 4^P' >= 4 (K-P'+1) N lambda/(4 alpha) / slots."""
+    from paper_conf_icdcs_qiul17_b200 import auto_fine_p
+
+    S = lib.dbg_smem_table_slots(lib.params(31, 11, 1))
+    assert auto_fine_p(1000, 31, 11) == 11
+    for n in (276_000_000, 2_627_000_000, 28_000_000_000, 10 ** 15):
+        q = auto_fine_p(n, 31, 11)
+        assert 4.0 ** q >= 4 * (31 - q + 1) * n / S
+        assert q == 11 or 4.0 ** (q - 1) < 4 * (31 - q + 2) * n / S
+    assert auto_fine_p(2_627_000_000, 31, 11) > 11          # chr14-sized input: longer minimizer
+    assert auto_fine_p(10 ** 9, 63, 19) == 19
 
 
 def test_encoder_fig4_and_rules(lib):
@@ -97,7 +131,8 @@ def test_invalid_arguments_return_before_launch(lib):
 
     part = partition_set(1, 1, 1, 1, 1, None, 0, None)
     for prm in (lib.params(30, 11, 16), lib.params(31, 0, 16), lib.params(31, 32, 16), lib.params(31, 11, 0),
-                lib.params(65, 11, 16)):
+                lib.params(65, 11, 16), lib.params(31, 11, 16, fine_p=32), lib.params(21, 11, 16, fine_p=23),
+                lib.params(31, 11, 16, fine_p=-1)):
         with pytest.raises(DbgError) as e:
             lib.dbg_msp_partition(prm, 1, 1, 1, 1, part, None)
         assert e.value.status == lib.DBG_EINVAL

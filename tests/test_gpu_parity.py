@@ -165,9 +165,62 @@ def test_smem_with_global_tier(k, p, np_, refine):
     g = genome(60_000, seed=k + np_)
     seq, offs = make_reads(g, 4000, 100, 0.01, seed=refine + 3)
     rs = ReadSet(seq, offs)
-    res, _ = _check(rs, k, p, np_, refine=refine)
+    res, _ = _check(rs, k, p, np_, refine=refine, smem_split=1)
     if refine == 1 and np_ <= 3:
         assert res.batches, "expected some partitions on the global-table path"
+
+
+@pytest.mark.parametrize("k,p,np_,refine,split", [(31, 11, 3, 1, 0), (31, 11, 1, 2, 0), (63, 19, 2, 1, 0),
+                                                   (41, 13, 12, 1, 3), (21, 7, 4, 2, 64), (31, 11, 12, 1, 2)])
+def test_smem_split_partitions(k, p, np_, refine, split):
+    """Partitions larger than one CTA table built on chip over several sub-tables (dbg.h
+    dbg_smem_onchip), next to grouped ones and (with a small split limit) global ones.  1500 reads
+    of 100 bp: partitions of ~10^4 K-mers, above one CTA table and below the 65535 bound."""
+    g = genome(60_000, seed=k + np_ + 1)
+    seq, offs = make_reads(g, 1500, 100, 0.01, seed=refine + 5)
+    rs = ReadSet(seq, offs)
+    res, _ = _check(rs, k, p, np_, refine=refine, smem_split=split)
+    prm = _lib.params(k, p, np_, refine=refine, smem_split=split)
+    place = np.array([_lib.dbg_smem_onchip(prm, int(n)) for n in res.part_kmers])
+    assert (place >= 2).any(), "expected split partitions"
+    assert bool(res.batches) == bool((place[res.part_kmers > 0] == 0).any())
+
+
+@pytest.mark.parametrize("k,p,np_,fine_p,refine", [(31, 11, 16, 13, 1), (31, 11, 7, 19, 4), (63, 19, 8, 25, 2),
+                                                   (41, 13, 5, 31, 1), (31, 11, 9, 7, 3), (21, 9, 3, 21, 1)])
+def test_fine_minimizer_partitioning(k, p, np_, fine_p, refine):
+    """dbg_params.fine_p (reading V): the device partitions by a P'-minimizer; the graph and every
+    vertex's pid (the partition of its P-minimizer) still equal the oracle's at P."""
+    g = genome(30_000, seed=k + fine_p)
+    seq, offs = make_reads(g, 2000, 100, 0.01, seed=fine_p)
+    rs = ReadSet(seq, offs)
+    _check(rs, k, p, np_, refine=refine, fine_p=fine_p)
+    rr = random_reads(300, 1, 2 * k + 80, seed=fine_p, n_rate=0.01)
+    _check(rr, k, p, np_, refine=refine, fine_p=fine_p)
+
+
+def test_fine_minimizer_records_vs_oracle_msp():
+    """Kernel (a) with fine_p: the records are the oracle's MSP superkmers at P' (Defs. 1-2)."""
+    for (k, p, q, np_, seed) in [(31, 11, 15, 16, 1), (63, 19, 27, 8, 2), (15, 5, 9, 3, 3)]:
+        rs = random_reads(200, 1, 300, seed=seed, n_rate=0.01)
+        b = DbgBuilder(k, p, np_, fine_p=q)
+        d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+        b.msp(d_bases, d_off)
+        torch.cuda.synchronize()
+        nrec = int(b.part_records.sum())
+        recs = decode_records(b.records[: nrec * b.rec_words].cpu().numpy().view(np.uint32), b.rec_words, k)
+        sk = oracle.msp(rs.seq, rs.offsets, k, q, np_)
+        assert np.array_equal(b.part_kmers, np.bincount(sk["pid"], weights=sk["n_kmers"],
+                                                         minlength=np_).astype(np.int64))
+        assert occurrences_from_records(recs, k) == occurrences_from_oracle_msp(sk, rs.reads(), k)
+
+
+def test_split_partition_hot_key_over_16_bits():
+    """A vertex seen more than 65535 times sits in a partition with N^i_kmer > 65535: it must take
+    the global tables (32-bit counters), not a 16-bit on-chip table."""
+    reads = ["A" * 1200] * 60 + ["ACGT" * 300] * 5
+    res, orc = _check(_readset(reads), 31, 11, 4)
+    assert res.vertices["count"].max() == 60 * (1200 - 31 + 1) > 65535
 
 
 def test_auto_refine_small_partitions():
@@ -294,5 +347,5 @@ def test_smem_global_tier_in_several_batches():
     g = genome(60_000, seed=12)
     seq, offs = make_reads(g, 4000, 100, 0.01, seed=13)
     rs = ReadSet(seq, offs)
-    res, _ = _check(rs, 31, 11, 3, refine=1, table_budget_bytes=48 * 20_000)
+    res, _ = _check(rs, 31, 11, 3, refine=1, table_budget_bytes=48 * 20_000, smem_split=1)
     assert len(res.batches) >= 2
