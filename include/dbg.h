@@ -142,7 +142,11 @@ DBG_API dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64_t*
  *   d_staging while they fit.  The caller reads d_record_offset[NP] (or the
  *   sizes); if it exceeds staging_cap, it grows d_staging and repeats pass 1.
  * part->d_records != NULL: pass 2 -- scatters the staged records into
- *   partition order (d_record_offset[NP] records). */
+ *   partition order (d_record_offset[NP] records).
+ * A caller may enqueue pass 2 and Step 2 before reading the sizes back: after a
+ * staging overflow (*d_staged > staging_cap) pass 2 and
+ * dbg_build_subgraphs_smem do nothing, and the caller grows d_staging and
+ * repeats the step.  d_records then needs room for staging_cap records. */
 DBG_API dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
                              const uint64_t* d_offsets, uint64_t n_reads,
                              const dbg_partition_set* part, cudaStream_t stream);

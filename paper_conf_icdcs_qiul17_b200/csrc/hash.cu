@@ -761,19 +761,51 @@ struct SmemSlot {
   static constexpr uint32_t kBytes = kKeyBytes + 4 * kFieldWords;
 };
 
-// T threads per CTA stage RB(T) records per batch.
-__host__ __device__ constexpr int smem_rec_batch(int T) { return T >= 1024 ? T : 2 * T; }
+// Decoded work item (32 B): records [r0, r0 + nrec) of partitions [first, last);
+// P0 = the group's first slot in the plan's prefix P; meta = span (16 bits) |
+// sub-table j << 16 | sub-table count ns << 24 (ns = 1: a group; 0: no more work).
+struct __align__(16) ItemDesc {
+  uint64_t r0, P0;
+  uint32_t nrec, first, last, meta;
+};
+__host__ __device__ constexpr uint32_t item_meta(uint32_t span, uint32_t j, uint32_t ns) {
+  return span | j << 16 | ns << 24;
+}
+
+constexpr int kGroupParts = 256;  // partitions per group at most (plan rule)
+
+// Records per batch: 1024 four-word or 512 eight-word records (16 KB) from 512
+// threads up; fewer for smaller CTAs.
+template <int R, int T>
+__host__ __device__ constexpr int smem_rec_batch() { return (T >= 512 ? 1024 : 2 * T) * 4 / R; }
+
 template <int R, int T>
 struct SmemStage {
-  uint32_t w[R][smem_rec_batch(T)];  // transposed: record j's word q at w[q][j] (bank-conflict-free)
-  uint32_t t0[smem_rec_batch(T)];    // first slot of the record's partition table in the CTA table
-  uint32_t cap[smem_rec_batch(T)];   // its capacity (0: partition off chip)
-  uint32_t pre[smem_rec_batch(T) + 1];
+  static constexpr int RB = smem_rec_batch<R, T>();
+  uint32_t w[2][R][RB];                       // records of two batches, transposed: word q of record j at w[b][q][j]
+  unsigned long long Pq[2][kGroupParts + 2];  // P[first .. last] of the current and the next item
+  uint32_t pre[RB + 1];
+  ItemDesc it[4];                             // items i .. i+3 (ring)
   typename cub::BlockScan<uint32_t, T>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, T>::TempStorage red;
   unsigned long long base;
-  uint32_t item[4];  // current work item: first, last partition, sub-table j, sub-tables (0: done)
 };
+
+// cp.async (sm_80+ asynchronous global -> shared copies; completion per thread).
+__device__ __forceinline__ void cp_async4(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+               "l"(src));
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+               "l"(src));
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+               "l"(src));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
 template <int R, int T>
 __host__ __device__ constexpr uint32_t smem_fixed_bytes() {
@@ -828,6 +860,8 @@ struct SmemArgs {
   const uint32_t* records;
   const uint64_t* rec_off;
   const uint64_t* n_kmers;
+  const unsigned long long* staged;  // pass-1 records; > staging_cap: overflow, nothing to build
+  uint64_t staging_cap;
   int pid0, n_fine, k;  // fine partitions [pid0, pid0 + n_fine)
   double ratio;         // lambda / (4 alpha)
   uint64_t slots;       // table slots that fit one CTA
@@ -840,6 +874,7 @@ struct SmemArgs {
   uint8_t* flag;        // [n_fine] group-start flags
   unsigned long long *t_gc, *t_sp, *t_fl;  // per-tile sums (scan.cuh), tiles + 1 each
   unsigned long long* ctr;  // [0] groups, [1] split partitions, [2] split items, [3] work counter
+  ItemDesc* gdesc;          // [n_fine] decoded groups
 };
 
 // A partition's table capacity (Sec. IV-A), its grouped on-chip
@@ -862,7 +897,8 @@ __device__ __forceinline__ OnChip on_chip(const SmemArgs& a, uint64_t nk) {
 // capacities and of the split counts; B scans of those; C writes P, the split
 // list and the group-start flags; D scans the flag counts; E writes gfirst.
 // Groups: with H = slots/2 and w(p) = floor(P[p]/H), partition p starts a
-// group iff p == 0, w(p) != w(p-1), or p or p-1 has capacity > H.  A group of
+// group iff p == 0, w(p) != w(p-1), p or p-1 has capacity > H, or p is a
+// multiple of kGroupParts (a group's partition offsets fit shared memory).  A group of
 // small partitions lies in one H-window and spans < H + H = slots; a larger
 // one is alone; a split or global partition is alone with span 0 (skipped).
 constexpr unsigned long long kSplitOne = 1ull << 32;  // packed (split partitions << 32) | sub-tables
@@ -939,7 +975,7 @@ __global__ void __launch_bounds__(kTileThreads) smem_plan_apply_kernel(SmemArgs 
         pcap = o.cap;
         pP = Pp - o.gc;
       }
-      f = Pp / H != pP / H || cap[q] > H || pcap > H;
+      f = Pp / H != pP / H || cap[q] > H || pcap > H || p % kGroupParts == 0;
     }
     a.flag[p] = f;
     nflag += f;
@@ -979,6 +1015,60 @@ __global__ void __launch_bounds__(kTileThreads) smem_plan_groups_kernel(SmemArgs
   }
 }
 
+// F: one descriptor per group (records, plan offsets); groups with nothing on
+// chip get no records.
+__global__ void __launch_bounds__(256) smem_plan_desc_kernel(SmemArgs a) {
+  const uint64_t ng = a.ctr[0];
+  for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < ng; g += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t first = a.gfirst[g], last = a.gfirst[g + 1];
+    const uint64_t P0 = a.P[first - a.pid0], span = a.P[last - a.pid0] - P0;
+    ItemDesc d;
+    d.r0 = a.rec_off[first];
+    d.P0 = P0;
+    d.nrec = span ? (uint32_t)(a.rec_off[last] - d.r0) : 0u;
+    d.first = first;
+    d.last = last;
+    d.meta = item_meta((uint32_t)span, 0, 1);
+    a.gdesc[g] = d;
+  }
+}
+
+// Warp-wide: claim result g -> descriptor of item g in *out (visible after the
+// caller's next cp_async_wait_all + barrier).  Groups: one 32-B cp.async of
+// the plan's descriptor; split sub-tables: a 32-ary search of the split list.
+__device__ __forceinline__ void fetch_item(const SmemArgs& a, uint64_t g, uint64_t n_split, uint64_t n_items,
+                                           ItemDesc* out, int lane) {
+  if (g >= n_items) {
+    if (lane == 0) out->meta = 0;
+    return;
+  }
+  if (g >= n_split) {
+    if (lane == 0) {
+      const char* src = reinterpret_cast<const char*>(a.gdesc + (g - n_split));
+      cp_async16(out, src);
+      cp_async16(reinterpret_cast<char*>(out) + 16, src + 16);
+    }
+    return;
+  }
+  uint32_t lo = 0, n = (uint32_t)a.ctr[1];  // last i in [lo, lo + n) with ss[i] <= g; ss[lo] <= g
+  while (n > 1) {
+    const uint32_t step = (n + 31) / 32;
+    const bool le = (uint32_t)lane * step < n && a.ss[lo + lane * step] <= g;
+    const int L = 31 - __clz(__ballot_sync(kFull, le));
+    lo += L * step;
+    n = min(step, n - L * step);
+  }
+  if (lane == 0) {
+    const uint32_t p = a.sp[lo], j = (uint32_t)g - a.ss[lo], ns = a.ss[lo + 1] - a.ss[lo];
+    out->r0 = a.rec_off[p];
+    out->P0 = 0;
+    out->nrec = (uint32_t)(a.rec_off[p + 1] - out->r0);
+    out->first = p;
+    out->last = p + 1;
+    out->meta = item_meta((uint32_t)a.slots, j, ns);
+  }
+}
+
 // Sub-table of a K-mer in a split partition: a hash independent of the slot hash.
 template <typename Code>
 __device__ __forceinline__ uint32_t sub_table(Code code, uint32_t n) {
@@ -994,217 +1084,231 @@ template <typename Code, int R, int kSmemThreads, int kMinCtas>
 __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   constexpr uint32_t KB = SmemSlot<KW>::kKeyBytes, FW = SmemSlot<KW>::kFieldWords;
-  constexpr int kRecBatch = smem_rec_batch(kSmemThreads);
-  constexpr int kRPT = kRecBatch / kSmemThreads;  // records per thread per batch
+  constexpr int RB = SmemStage<R, kSmemThreads>::RB;
+  constexpr int kRPT = RB >= kSmemThreads ? RB / kSmemThreads : 1;  // records per thread per batch
   typedef cub::BlockScan<uint32_t, kSmemThreads> Scan;
   extern __shared__ __align__(128) unsigned char smem[];
   SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
   char* keys = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
   uint32_t* fld = reinterpret_cast<uint32_t*>(keys + a.slots * KB);
   const int K = a.k;
-  const int top = 2 * K - 2;
-  const Code mask = ((Code)1 << (2 * K)) - 1;
   {  // the table starts clean; extraction keeps it clean (slots is a multiple of 64)
     uint4* z = reinterpret_cast<uint4*>(keys);
     for (uint64_t q = threadIdx.x; q < a.slots * SmemSlot<KW>::kBytes / 16; q += kSmemThreads)
       z[q] = make_uint4(0, 0, 0, 0);
   }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
   bool ok = true;
+  if (a.staged && *a.staged > a.staging_cap) return;  // staging overflow: the records are incomplete
   const uint64_t n_split = a.ctr[2], n_items = n_split + a.ctr[0];
-  // Work items, taken from a global counter: first the sub-tables of the split
-  // partitions (the longest items), then the groups.
+  // Work items are claimed from a global counter, first the sub-tables of the
+  // split partitions (the longest items), then the groups, and decoded three
+  // items ahead (ring st.it).  The CTA consumes a stream of record batches;
+  // the next batch -- of the same item, or the next item's first with its plan
+  // offsets -- is copied in with cp.async while the current one is hashed.
+  uint64_t g_next = 0;  // warp 0 lane 0: the claim for the next item to decode
+  if (warp == 0) {
+    uint64_t g[4] = {0, 0, 0, 0};
+    if (lane == 0)
+      for (int q = 0; q < 4; ++q) g[q] = atomicAdd(a.ctr + 3, 1ull);
+    for (int q = 0; q < 3; ++q) fetch_item(a, __shfl_sync(kFull, g[q], 0), n_split, n_items, st.it + q, lane);
+    g_next = g[3];
+    cp_async_wait_all();
+  }
+  __syncthreads();
+  auto prefetch = [&](const ItemDesc& I, uint32_t rb, int bb, int ip, bool with_p) {
+    const uint32_t n = min((uint32_t)RB, I.nrec - rb);
+    const uint32_t* src = a.records + (I.r0 + rb) * R;
+    for (uint32_t j = threadIdx.x; j < n; j += kSmemThreads)
+#pragma unroll
+      for (int q = 0; q < R; ++q) cp_async4(&st.w[bb][q][j], src + (uint64_t)j * R + q);
+    if (with_p)
+      for (uint32_t t = threadIdx.x; t <= I.last - I.first; t += kSmemThreads)
+        cp_async8(&st.Pq[ip][t], a.P + (I.first - a.pid0) + t);
+  };
+  if (st.it[0].meta >> 24) prefetch(st.it[0], 0, 0, 0, (st.it[0].meta >> 24) == 1);
+  cp_async_commit();
+  int ci = 0, ip = 0, bb = 0;
+  uint32_t rb = 0;
   for (;;) {
-    __syncthreads();  // the previous item (staging, st.item) is finished
-    if (threadIdx.x == 0) {
-      const uint64_t g = atomicAdd(a.ctr + 3, 1ull);
-      uint32_t first = 0, last = 0, j = 0, ns = 1;
-      if (g < n_split) {  // split partition i with ss[i] <= g < ss[i+1]
-        uint32_t lo = 0, hi = (uint32_t)a.ctr[1];
-        while (hi - lo > 1) {
-          const uint32_t mid = (lo + hi) >> 1;
-          if (a.ss[mid] <= g) lo = mid;
-          else hi = mid;
-        }
-        first = a.sp[lo];
-        last = first + 1;
-        j = (uint32_t)g - a.ss[lo];
-        ns = a.ss[lo + 1] - a.ss[lo];
-      } else if (g < n_items) {
-        first = a.gfirst[g - n_split];
-        last = a.gfirst[g - n_split + 1];
-      } else {
-        ns = 0;  // done
-      }
-      st.item[0] = first;
-      st.item[1] = last;
-      st.item[2] = j;
-      st.item[3] = ns;
-    }
-    __syncthreads();
-    const uint32_t sub_n = st.item[3], sub_j = st.item[2];
+    cp_async_wait_all();
+    __syncthreads();  // this batch is in st.w[bb]; the other buffer and the previous item are done
+    const ItemDesc I = st.it[ci];
+    const uint32_t sub_n = I.meta >> 24;
     if (sub_n == 0) break;
+    const uint32_t sub_j = (I.meta >> 16) & 255u, span = I.meta & 0xffffu;
     const bool split = sub_n > 1;
-    const int first = (int)st.item[0], last = (int)st.item[1];
-    const uint64_t P0 = split ? 0 : a.P[first - a.pid0];
-    const uint64_t span = split ? a.slots : a.P[last - a.pid0] - P0;
-    if (span == 0) continue;  // nothing on chip in this group
-    const uint64_t r0 = a.rec_off[first], nrec = a.rec_off[last] - r0;
-    for (uint64_t rb = 0; rb < nrec; rb += kRecBatch) {
-      const int nb = (int)min((uint64_t)kRecBatch, nrec - rb);
-      __syncthreads();  // staging free; previous extraction (table clean) complete
-      uint32_t cnt[kRPT];
-#pragma unroll
-      for (int v = 0; v < kRPT; ++v) {
-        const int j = kRPT * threadIdx.x + v;
-        cnt[v] = 0;
-        if (j < nb) {
-          const uint4* src = reinterpret_cast<const uint4*>(a.records + (r0 + rb + j) * R);
-#pragma unroll
-          for (int q = 0; q < R / 4; ++q) {
-            const uint4 x = __ldcs(src + q);  // streamed once
-            st.w[4 * q][j] = x.x;
-            st.w[4 * q + 1][j] = x.y;
-            st.w[4 * q + 2][j] = x.z;
-            st.w[4 * q + 3][j] = x.w;
-          }
-          if (split) {  // one partition, the whole CTA table
-            st.t0[j] = 0;
-            st.cap[j] = (uint32_t)a.slots;
-            cnt[v] = st.w[0][j] & 255u;
-          } else {
-            const uint32_t pid = (st.w[0][j] >> 10) - a.pid0;
-            const uint64_t pp = a.P[pid], pc = a.P[pid + 1] - pp;
-            st.t0[j] = (uint32_t)(pp - P0);
-            st.cap[j] = (uint32_t)pc;
-            cnt[v] = pc ? st.w[0][j] & 255u : 0u;  // off-chip partition: skipped here
-          }
-        }
-      }
-      uint32_t excl[kRPT], total;
-      Scan(st.scan).ExclusiveSum(cnt, excl, total);
-#pragma unroll
-      for (int v = 0; v < kRPT; ++v) st.pre[kRPT * threadIdx.x + v] = excl[v];
-      if (threadIdx.x == 0) st.pre[kRecBatch] = total;
-      __syncthreads();
-      // this thread's contiguous run of K-mers [k0, k1)
-      const uint32_t share = (total + kSmemThreads - 1) / kSmemThreads;
-      const uint32_t k0 = min(total, threadIdx.x * share), k1 = min(total, k0 + share);
-      if (k0 < k1) {
-        int lo = 0, hi = nb;  // record holding K-mer k0: last r with pre[r] <= k0
-        while (hi - lo > 1) {
-          const int mid = (lo + hi) >> 1;
-          if (st.pre[mid] <= k0) lo = mid;
-          else hi = mid;
-        }
-        int r = lo;
-        while (st.pre[r + 1] == st.pre[r]) ++r;  // skip records that contribute nothing
-        constexpr int S = kRecBatch;  // staging stride
-        int t = (int)(k0 - st.pre[r]);
-        const uint32_t* w = &st.w[0][r];
-        int n = w[0] & 255u, hl = (w[0] >> 8) & 1u, hr = (w[0] >> 9) & 1u;
-        char* tk = keys + (uint64_t)st.t0[r] * KB;
-        uint32_t* tf = fld + (uint64_t)st.t0[r] * FW;
-        uint32_t cap = st.cap[r];
-        uint32_t pid = w[0] >> 10;
-        Code fwd, rc;
-        kmer_at(w, hl + t, K, R, fwd, rc, S);
-        for (uint32_t kid = k0;;) {
-          const int b = hl + t;
-          const int pred = (t > 0 || hl) ? (int)rec_base(w, b - 1, S) : -1;
-          const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K, S) : -1;
-          // canonical orientation and edge indices (readings C, J), selected branch-free so
-          // that one upsert serves both orientations (no divergent duplicate of it)
-          const bool is_fwd = fwd < rc;
-          const Code code = is_fwd ? fwd : rc;
-          const int o = is_fwd ? (succ >= 0 ? succ : 4) : (pred >= 0 ? 3 - pred : 4);
-          const int i = is_fwd ? pred : (succ >= 0 ? 3 - succ : -1);
-          if (sub_n == 1 || sub_table(code, sub_n) == sub_j) ok &= smem_upsert<Code>(tk, tf, cap, code, o, i, pid);
-          if (++kid >= k1) break;
-          if (++t < n) {  // next K-mer of the same record: roll one base
-            fwd = ((fwd << 2) | (Code)succ) & mask;
-            rc = (rc >> 2) | ((Code)(3 - succ) << top);
-          } else {  // next record that contributes K-mers
-            do ++r;
-            while (st.pre[r + 1] == st.pre[r]);
-            t = 0;
-            w = &st.w[0][r];
-            n = w[0] & 255u;
-            hl = (w[0] >> 8) & 1u;
-            hr = (w[0] >> 9) & 1u;
-            tk = keys + (uint64_t)st.t0[r] * KB;
-            tf = fld + (uint64_t)st.t0[r] * FW;
-            cap = st.cap[r];
-            pid = w[0] >> 10;
-            kmer_at(w, hl, K, R, fwd, rc, S);
-          }
-        }
-      }
+    const int nb = (int)min((uint32_t)RB, I.nrec - rb);
+    const bool last_batch = rb + RB >= I.nrec;
+    if (rb == 0 && warp == 0) {  // item start: claim the next one and decode item i+3
+      const uint64_t g = __shfl_sync(kFull, g_next, 0);
+      if (lane == 0) g_next = atomicAdd(a.ctr + 3, 1ull);
+      fetch_item(a, g, n_split, n_items, st.it + ((ci + 3) & 3), lane);
     }
-    __syncthreads();
-    // extraction: each warp owns a contiguous run of slots; one block scan of the
-    // warps' occupied counts sizes the group's output, one global atomic reserves it.
-    // Occupied slot indices are then queued per warp (the idle record staging is the
-    // queue, 128 entries per warp) and emitted with every lane busy.
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    constexpr int kWarps = kSmemThreads / 32;
-    const uint32_t wspan = ((uint32_t)span + kWarps * 32 - 1) / (kWarps * 32) * 32;  // slots per warp
-    const uint32_t ws0 = min((uint32_t)span, warp * wspan), ws1 = min((uint32_t)span, ws0 + wspan);
-    uint32_t cnt = 0;
-    for (uint32_t c = ws0; c < ws1; c += 32) {
-      const uint32_t s = c + lane;
-      cnt += __popc(__ballot_sync(kFull, s < ws1 &&
-                                            (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied)));
+    if (!last_batch) {
+      prefetch(I, rb + RB, bb ^ 1, ip, false);
+    } else {
+      const ItemDesc& N = st.it[(ci + 1) & 3];
+      if (N.meta >> 24) prefetch(N, 0, bb ^ 1, ip ^ 1, (N.meta >> 24) == 1);
     }
-    uint32_t excl, total;
-    Scan(st.scan).ExclusiveSum(lane == 0 ? cnt : 0u, excl, total);
-    if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
-    __syncthreads();
-    uint64_t pos = st.base + __shfl_sync(kFull, excl, 0);
-    uint32_t* queue = &st.w[0][0] + warp * 128;
-    for (uint32_t sub = ws0; sub < ws1; sub += 128) {
-      uint32_t qn = 0;
-      for (uint32_t c = sub; c < min(ws1, sub + 128); c += 32) {
-        const uint32_t s = c + lane;
-        const bool occ = s < ws1 && (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied);
-        const uint32_t bal = __ballot_sync(kFull, occ);
-        if (occ) queue[qn + __popc(bal & ((1u << lane) - 1u))] = s;
-        qn += __popc(bal);
-      }
-      __syncwarp();
-      for (uint32_t e = lane; e < qn; e += 32) {
-        const uint32_t s = queue[e];
-        unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
-        const uint64_t k0 = kp[0];
-        uint32_t* f = fld + s * FW;
-        dbg_vertex v;
-        if (KW == 1) {
-          v.kmer_hi = 0;
-          v.kmer_lo = k0 & kCodeMask;
+    cp_async_commit();
+    const unsigned long long* Pq = st.Pq[ip];
+    uint32_t cnt[kRPT];
+#pragma unroll
+    for (int v = 0; v < kRPT; ++v) {
+      const int j = kRPT * threadIdx.x + v;
+      cnt[v] = 0;
+      if (j < nb) {
+        const uint32_t w0 = st.w[bb][0][j];
+        if (split) {
+          cnt[v] = w0 & 255u;
         } else {
-          v.kmer_hi = k0 & kCodeMask;
-          v.kmer_lo = kp[1];
+          const uint32_t x = (w0 >> 10) - I.first;
+          cnt[v] = Pq[x + 1] != Pq[x] ? w0 & 255u : 0u;  // off-chip partition: skipped here
         }
-        const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
-        v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
-        v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
-        v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
-        // fine pid recorded by the inserting thread, mod NP (or from the P-minimizer, reading V)
-        v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, f[5]);
-        kp[0] = 0;  // clean-on-extract
-        if (KW == 2) kp[1] = 0;
-#pragma unroll
-        for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
-        const uint64_t my = pos + e;
-        if (my < oa.out_cap) oa.out[my] = v;
-        else atomicOr(oa.status, kStatusNoSpace);
-        st_n += 1;
-        st_count += v.count;
-        st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
       }
-      pos += qn;
-      __syncwarp();
     }
+    uint32_t excl[kRPT], total;
+    Scan(st.scan).ExclusiveSum(cnt, excl, total);
+#pragma unroll
+    for (int v = 0; v < kRPT; ++v)
+      if (kRPT * threadIdx.x + v < RB) st.pre[kRPT * threadIdx.x + v] = excl[v];
+    if (threadIdx.x == 0) st.pre[RB] = total;
+    __syncthreads();
+    // this thread's contiguous run of K-mers [k0, k1)
+    const uint32_t share = (total + kSmemThreads - 1) / kSmemThreads;
+    const uint32_t k0 = min(total, threadIdx.x * share), k1 = min(total, k0 + share);
+    if (k0 < k1) {
+      int lo = 0, hi = nb;  // record holding K-mer k0: last r with pre[r] <= k0
+      while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (st.pre[mid] <= k0) lo = mid;
+        else hi = mid;
+      }
+      int r = lo;
+      while (st.pre[r + 1] == st.pre[r]) ++r;  // skip records that contribute nothing
+      constexpr int S = RB;                      // staging stride
+      const uint32_t* w;
+      int t = (int)(k0 - st.pre[r]), n, hl, hr;
+      char* tk;
+      uint32_t* tf;
+      uint32_t cap, pid;
+      auto header = [&](int rr) {  // record rr of the batch: its bases and its partition's table
+        w = &st.w[bb][0][rr];
+        const uint32_t w0 = w[0];
+        n = w0 & 255u;
+        hl = (w0 >> 8) & 1u;
+        hr = (w0 >> 9) & 1u;
+        pid = w0 >> 10;
+        uint64_t t0;
+        if (split) {
+          t0 = 0;
+          cap = (uint32_t)a.slots;
+        } else {
+          const uint32_t x = pid - I.first;
+          t0 = Pq[x] - I.P0;
+          cap = (uint32_t)(Pq[x + 1] - Pq[x]);
+        }
+        tk = keys + t0 * KB;
+        tf = fld + t0 * FW;
+      };
+      header(r);
+      // Every K-mer is decoded from the staged words (no rolling): the lanes of a
+      // warp stay converged; only the small header reload at a record change diverges.
+      for (uint32_t kid = k0;;) {
+        const int b = hl + t;
+        Code fwd, rc;
+        kmer_at(w, b, K, R, fwd, rc, S);
+        const int pred = b > 0 ? (int)rec_base(w, b - 1, S) : -1;
+        const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K, S) : -1;
+        // canonical orientation and edge indices (readings C, J), selected branch-free so
+        // that one upsert serves both orientations (no divergent duplicate of it)
+        const bool is_fwd = fwd < rc;
+        const Code code = is_fwd ? fwd : rc;
+        const int o = is_fwd ? (succ >= 0 ? succ : 4) : (pred >= 0 ? 3 - pred : 4);
+        const int i = is_fwd ? pred : (succ >= 0 ? 3 - succ : -1);
+        if (sub_n == 1 || sub_table(code, sub_n) == sub_j) ok &= smem_upsert<Code>(tk, tf, cap, code, o, i, pid);
+        if (++kid >= k1) break;
+        if (++t == n) {  // next record that contributes K-mers
+          do ++r;
+          while (st.pre[r + 1] == st.pre[r]);
+          t = 0;
+          header(r);
+        }
+      }
+    }
+    if (last_batch) {
+      __syncthreads();
+      // extraction: each warp owns a contiguous run of slots; one block scan of the
+      // warps' occupied counts sizes the item's output, one global atomic reserves it.
+      // Occupied slot indices are then queued per warp (in the batch's finished record
+      // buffer, 128 entries per warp) and emitted with every lane busy.
+      constexpr int kWarps = kSmemThreads / 32;
+      const uint32_t wspan = (span + kWarps * 32 - 1) / (kWarps * 32) * 32;  // slots per warp
+      const uint32_t ws0 = min(span, warp * wspan), ws1 = min(span, ws0 + wspan);
+      uint32_t cnt = 0;
+      for (uint32_t c = ws0; c < ws1; c += 32) {
+        const uint32_t s = c + lane;
+        cnt += __popc(__ballot_sync(kFull, s < ws1 &&
+                                              (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied)));
+      }
+      uint32_t excl, total;
+      Scan(st.scan).ExclusiveSum(lane == 0 ? cnt : 0u, excl, total);
+      if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
+      __syncthreads();
+      uint64_t pos = st.base + __shfl_sync(kFull, excl, 0);
+      uint32_t* queue = &st.w[bb][0][0] + warp * 128;
+      for (uint32_t sub = ws0; sub < ws1; sub += 128) {
+        uint32_t qn = 0;
+        for (uint32_t c = sub; c < min(ws1, sub + 128); c += 32) {
+          const uint32_t s = c + lane;
+          const bool occ = s < ws1 && (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied);
+          const uint32_t bal = __ballot_sync(kFull, occ);
+          if (occ) queue[qn + __popc(bal & ((1u << lane) - 1u))] = s;
+          qn += __popc(bal);
+        }
+        __syncwarp();
+        for (uint32_t e = lane; e < qn; e += 32) {
+          const uint32_t s = queue[e];
+          unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+          const uint64_t kw0 = kp[0];
+          uint32_t* f = fld + s * FW;
+          dbg_vertex v;
+          if (KW == 1) {
+            v.kmer_hi = 0;
+            v.kmer_lo = kw0 & kCodeMask;
+          } else {
+            v.kmer_hi = kw0 & kCodeMask;
+            v.kmer_lo = kp[1];
+          }
+          const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
+          v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
+          v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
+          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
+          // fine pid recorded by the inserting thread, mod NP (or from the P-minimizer, reading V)
+          v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, f[5]);
+          kp[0] = 0;  // clean-on-extract
+          if (KW == 2) kp[1] = 0;
+#pragma unroll
+          for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
+          const uint64_t my = pos + e;
+          if (my < oa.out_cap) oa.out[my] = v;
+          else atomicOr(oa.status, kStatusNoSpace);
+          st_n += 1;
+          st_count += v.count;
+          st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
+        }
+        pos += qn;
+        __syncwarp();
+      }
+      ci = (ci + 1) & 3;
+      ip ^= 1;
+      rb = 0;
+    } else {
+      rb += RB;
+    }
+    bb ^= 1;
   }
   if (!ok) atomicOr(oa.status, kStatusTableFull);
   __syncthreads();
@@ -1430,7 +1534,9 @@ static uint64_t smem_workspace(uint64_t n, SmemArgs* a, char* ws) {
   char* sp = take(4 * n + 4);
   char* ss = take(4 * (n + 1));
   char* flag = take(n + 1);
+  char* gdesc = take(sizeof(ItemDesc) * (n + 1));
   if (a) {
+    a->gdesc = reinterpret_cast<ItemDesc*>(gdesc);
     a->P = reinterpret_cast<uint64_t*>(P);
     a->t_gc = reinterpret_cast<unsigned long long*>(t_gc);
     a->t_sp = reinterpret_cast<unsigned long long*>(t_sp);
@@ -1465,6 +1571,8 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
   a.n_kmers = part->d_n_kmers;
+  a.staged = reinterpret_cast<const unsigned long long*>(part->d_staged);
+  a.staging_cap = part->staging_cap;
   a.pid0 = pid_begin;
   a.n_fine = pid_end - pid_begin;
   a.np_mod = make_fastmod((uint64_t)prm->num_partitions);
@@ -1480,6 +1588,8 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   smem_plan_apply_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_fl, tiles);
   smem_plan_groups_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
+  smem_plan_desc_kernel<<<(a.n_fine + 255) / 256 < dbg_sm_count() * 8 ? (a.n_fine + 255) / 256 : dbg_sm_count() * 8,
+                          256, 0, stream>>>(a);
   const OutArgs oa = make_out_args(prm, d_out, out_cap, d_n_out, d_stats, d_status);
   cudaError_t e;
   if (prm->k <= 31) e = launch_smem<uint64_t, 4>(a, oa, stream);

@@ -231,7 +231,8 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
                                                                   uint32_t* __restrict__ records, int np) {
   extern __shared__ unsigned long long sh_base[];  // [np] global bases (per tile), then [np] counts
   uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_base + np);
-  const uint64_t n = min((uint64_t)*staged, staging_cap);
+  const uint64_t n = *staged;
+  if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
   const bool smem = np <= kSmemHistMaxNp;
   constexpr int kTile = kScatterThreads * kScatterPer;
   for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile) {
@@ -348,7 +349,7 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
                        reinterpret_cast<unsigned long long*>(part->d_fill), stream) != cudaSuccess)
       return DBG_ECUDA;
   } else {
-    // pass 3: scatter (requires staged <= staging_cap; the caller checks sum(n_records))
+    // pass 3: scatter (a no-op after a staging overflow, *d_staged > staging_cap)
     if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
     if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * np, stream) != cudaSuccess) return DBG_ECUDA;
     const size_t smem = np <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * np : 0;

@@ -123,6 +123,12 @@ class DbgBuilder:
         self._big_key = None
         self._batches_cache: list[tuple[int, int]] = []
         self._dirty = False
+        self._tab_key = None
+        self._any_global = False
+        self._h_sizes = torch.empty(0, dtype=torch.int64)
+        self._sizes_ev = torch.cuda.Event() if self.device.type == "cuda" else None
+        self._sizes_pending = False
+        self.overflowed = False
         self.timer: dict | None = None  # name -> list of (start, end) CUDA events, when set
 
     # ------------------------------------------------------------------ timing helper
@@ -160,28 +166,47 @@ class DbgBuilder:
         return int(min(n_kmers_upper, 2.6 * n_kmers_upper / (w + 1) + 2 * n_reads)) + 4096
 
     def msp(self, d_bases: torch.Tensor, d_offsets: torch.Tensor, stream=None):
+        """Step 1: pass 1 (minimizers, superkmers, sizes, staging), the sizes copied back
+        asynchronously, pass 2 (scatter).  Nothing here waits for the device: sync_sizes() reads
+        the sizes when the host needs them, after the device work behind them is enqueued."""
         stream = stream or torch.cuda.current_stream(self.device)
         n_reads = d_offsets.numel() - 1
         n_words = d_bases.numel()
         if self.staging.numel() == 0:
             self.staging = _grow(self.staging, self._staging_estimate(n_words * 32, n_reads) * self.rec_words,
                                  torch.int32, self.device)
+        self.overflowed = False
         ev = self._mark("msp_pass1", stream)
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(False), stream)
         self._done(ev, stream)
+        if self._h_sizes.numel() != 2 * self.np:
+            self._h_sizes = torch.empty(2 * self.np, dtype=torch.int64, pin_memory=True)
         with torch.cuda.stream(stream):
-            sizes = torch.cat([self.d_n_records, self.d_n_kmers]).cpu()  # the one size readback
-        sizes = sizes.numpy()
-        self.part_records = sizes[:self.np].copy()
-        self.part_kmers = sizes[self.np:].copy()
-        total = int(self.part_records.sum())
-        if total > self.staging.numel() // self.rec_words:  # staging too small: exact size, redo pass 1
-            self.staging = _grow(self.staging, total * self.rec_words, torch.int32, self.device, 1.05)
-            _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(False), stream)
-        self.records = _grow(self.records, total * self.rec_words, torch.int32, self.device, 1.05)
+            self._h_sizes[:self.np].copy_(self.d_n_records, non_blocking=True)
+            self._h_sizes[self.np:].copy_(self.d_n_kmers, non_blocking=True)
+        self._sizes_ev.record(stream)
+        self._sizes_pending = True
+        # room for every staged record: after an overflow pass 2 and Step 2 do nothing (dbg.h)
+        self.records = _grow(self.records, self.staging.numel(), torch.int32, self.device)
         ev = self._mark("msp_scatter", stream)
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
         self._done(ev, stream)
+
+    def sync_sizes(self) -> bool:
+        """Waits for the pass-1 sizes (part_records, part_kmers).  False after a staging overflow:
+        the staging has been grown and the step must be repeated (self.overflowed)."""
+        if not self._sizes_pending:
+            return not self.overflowed
+        self._sizes_ev.synchronize()
+        sizes = self._h_sizes.numpy()
+        self.part_records = sizes[:self.np].copy()
+        self.part_kmers = sizes[self.np:].copy()
+        self._sizes_pending = False
+        total = int(self.part_records.sum())
+        if total > self.staging.numel() // self.rec_words:
+            self.staging = _grow(self.staging, total * self.rec_words, torch.int32, self.device, 1.05)
+            self.overflowed = True
+        return not self.overflowed
 
     def load_exchanged(self, received: torch.Tensor, n_received: int, global_records: np.ndarray,
                        global_kmers: np.ndarray, owned: tuple[int, int], stream=None) -> None:
@@ -199,6 +224,8 @@ class DbgBuilder:
         off[1:] = np.cumsum(rec)
         assert int(off[-1]) == n_received, (int(off[-1]), n_received)
         self.part_records, self.part_kmers = rec, kmr
+        self._sizes_pending = False
+        self.overflowed = False
         with torch.cuda.stream(stream):
             self.d_n_records.copy_(torch.from_numpy(rec), non_blocking=True)
             self.d_n_kmers.copy_(torch.from_numpy(kmr), non_blocking=True)
@@ -210,29 +237,53 @@ class DbgBuilder:
 
     # ------------------------------------------------------------------ a5
     def plan(self, stream=None) -> list[tuple[int, int]]:
+        """Sizing (row a5).  Mode "smem": the on-chip plan runs on the device inside
+        dbg_build_subgraphs_smem, and the global tables of oversize partitions are planned in
+        step2 once the sizes are back -- nothing to do here.  Other modes: tables for all."""
         stream = stream or torch.cuda.current_stream(self.device)
-        ev = self._mark("plan", stream)
-        # d_fill is idle after the scatter: scratch of the multi-CTA scan
-        if self.mode == "smem":  # on-chip partitions need no global table
-            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
-        else:
-            _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
-        self._done(ev, stream)
+        if self.mode == "smem":
+            return self.batches
+        if not self.sync_sizes():
+            self.batches = []
+            return self.batches
+        return self._plan_tables(stream)
+
+    def _plan_tables(self, stream) -> list[tuple[int, int]]:
+        """Global tables: capacities (host copy of the C sizing functions, cached per size
+        vector), batches that fit the table budget, and d_table_offset on the device."""
         key = (self.part_kmers.tobytes(), self.prm.lambda_, self.prm.alpha, self.mode, self.owned)
-        if self._caps_key != key:  # host copy of the same C sizing functions (per distinct size)
+        if self._caps_key != key:
             nz = np.nonzero(self.part_kmers)[0]
             self.caps = np.zeros(self.np, dtype=np.int64)
             uniq, inv = np.unique(self.part_kmers[nz], return_inverse=True)
             cap_u = np.array([_lib.dbg_table_capacity(self.prm, int(n)) for n in uniq], dtype=np.int64)
-            if self.mode == "smem":
+            if self.mode == "smem":  # on-chip partitions need no global table
                 cap_u[np.array([_lib.dbg_smem_onchip(self.prm, int(n)) > 0 for n in uniq], dtype=bool)] = 0
             self.caps[nz] = cap_u[inv]
             lo, hi = self.owned
             self.caps[:lo] = 0
             self.caps[hi:] = 0
             self._caps_key = key
-        self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
-        self.tab_host[1:] = np.cumsum(self.caps)
+            self._any_global = bool(self.caps.any())
+        if self.mode == "smem" and not self._any_global:
+            self.batches = []
+            return self.batches
+        ev = self._mark("plan", stream)
+        # d_fill is idle after the scatter: scratch of the multi-CTA scan
+        if self.mode == "smem":
+            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
+        else:
+            _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
+        self._done(ev, stream)
+        # d_fill is idle after the scatter: scratch of the multi-CTA scan
+        if self.mode == "smem":  # on-chip partitions need no global table
+            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
+        else:
+            _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
+        if self._tab_key != self._caps_key:
+            self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
+            self.tab_host[1:] = np.cumsum(self.caps)
+            self._tab_key = self._caps_key
         if self.mode == "fused":
             self.batches = [(0, self.np)]
             self.total_slots = int(self.tab_host[-1])
@@ -240,9 +291,6 @@ class DbgBuilder:
             self.ring = self._clean_buffer(self.ring, ring, stream)
             wsb = _lib.dbg_subgraph_workspace_bytes(self.prm, self.np, self.total_slots, self.group_slots)
             self.work = _grow(self.work, wsb, torch.uint8, self.device)
-            return self.batches
-        if self.mode == "smem" and not self.caps.any():
-            self.batches = []
             return self.batches
         budget = self.table_budget_bytes
         if budget is None:  # once per builder: cudaMemGetInfo costs milliseconds
@@ -296,6 +344,8 @@ class DbgBuilder:
         self._dirty = False
 
     def _step2(self, stream) -> None:
+        if self.overflowed:  # pass 2 did nothing; the caller repeats the step
+            return
         if self.mode == "smem":
             ev = self._mark("step2_smem", stream)
             wsb = _lib.dbg_smem_workspace_bytes(self.prm)
@@ -304,6 +354,10 @@ class DbgBuilder:
                                           self.work.numel(), self.out, self.out_cap(), self.d_n_out, self.d_stats,
                                           self.d_status, stream)
             self._done(ev, stream)
+            # the sizes are read back while the on-chip kernel runs; then the global tier
+            if not self.sync_sizes():
+                return
+            self._plan_tables(stream)
         if self.mode == "fused":
             ev = self._mark("step2", stream)
             _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.total_slots,
@@ -370,6 +424,8 @@ class DbgBuilder:
               want_vertices: bool = True, sort: bool = True) -> GraphResult:
         stream = stream or torch.cuda.current_stream(self.device)
         self.msp(d_bases, d_offsets, stream)
+        while not self.sync_sizes():  # staging overflow: grown, repeat Step 1
+            self.msp(d_bases, d_offsets, stream)
         self.plan(stream)
         n_kmers = int(self.part_kmers.sum())
         cap = out_cap if out_cap is not None else max(self.out_cap(), n_kmers // 2 + 1024)

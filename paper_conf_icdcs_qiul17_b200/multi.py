@@ -72,6 +72,8 @@ def distributed_step(builder, d_bases, d_offsets, stream, out_cap: int, group=No
     world, rank = dist.get_world_size(group), dist.get_rank(group)
     builder.owned = (0, builder.np)
     builder.msp(d_bases, d_offsets, stream)                      # Step 1 on local reads
+    while not builder.sync_sizes():                               # staging overflow: grown, repeat
+        builder.msp(d_bases, d_offsets, stream)
     bounds = owner_bounds(builder.np, world)
     g_rec, g_kmr = global_sizes(builder.part_records, builder.part_kmers, builder.device, group)
     recv, n_recv, _ = exchange_records(builder.records, builder.part_records, bounds, builder.rec_words, group)

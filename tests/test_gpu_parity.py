@@ -97,6 +97,7 @@ def test_msp_records_vs_oracle_superkmers():
         b = DbgBuilder(k, p, np_)
         d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
         b.msp(d_bases, d_off)
+        assert b.sync_sizes()
         torch.cuda.synchronize()
         nrec = int(b.part_records.sum())
         words = b.records[: nrec * b.rec_words].cpu().numpy().view(np.uint32)
@@ -127,6 +128,7 @@ def test_table_overflow_detected_and_rebuilt(mode):
     b = DbgBuilder(31, 11, 4, lam=0.04, alpha=0.5, mode=mode)
     d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
     b.msp(d_bases, d_off)
+    assert b.sync_sizes()
     b.plan()
     b.reset_output(1 << 20)
     b.step2()
@@ -206,6 +208,7 @@ def test_fine_minimizer_records_vs_oracle_msp():
         b = DbgBuilder(k, p, np_, fine_p=q)
         d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
         b.msp(d_bases, d_off)
+        assert b.sync_sizes()
         torch.cuda.synchronize()
         nrec = int(b.part_records.sum())
         recs = decode_records(b.records[: nrec * b.rec_words].cpu().numpy().view(np.uint32), b.rec_words, k)
@@ -314,6 +317,7 @@ def test_sharded_path_two_logical_ranks_one_gpu():
         b = DbgBuilder(k, p, np_, refine=refine)
         d_bases, d_off = b.upload(encode_reads(h.seq), h.offsets)
         b.msp(d_bases, d_off)
+        assert b.sync_sizes()
         bs.append(b)
     n_fine = bs[0].np
     bounds = owner_bounds(n_fine, 2)
@@ -349,3 +353,21 @@ def test_smem_global_tier_in_several_batches():
     rs = ReadSet(seq, offs)
     res, _ = _check(rs, 31, 11, 3, refine=1, table_budget_bytes=48 * 20_000, smem_split=1)
     assert len(res.batches) >= 2
+
+
+def test_staging_overflow_repeats_the_step():
+    """dbg.h pass 2: after a staging overflow, pass 2 and the on-chip kernel do nothing (no write
+    past the buffers); the builder grows the staging and the repeated step is exact."""
+    rs = random_reads(3000, 60, 200, seed=31)
+    b = DbgBuilder(31, 11, 16, refine=4)
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    b.staging = torch.empty(64 * b.rec_words, dtype=torch.int32, device=b.device)  # far too small
+    b.msp(d_bases, d_off)
+    b.plan()
+    b.reset_output(1 << 20)
+    b.step2()
+    assert b.overflowed and int(b.d_n_out.item()) == 0
+    assert b.staging.numel() // b.rec_words >= int(b.part_records.sum())
+    res = b.build(d_bases, d_off)
+    orc = oracle.graph(rs.seq, rs.offsets, 31, 11, 16, n_threads=NT)
+    compare_vertices(res.vertices, orc)
