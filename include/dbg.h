@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 3
+#define DBG_ABI_VERSION 4
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -66,6 +66,12 @@ typedef struct {
                              K-mers of large genomes (few distinct P-mers per base) evenly;
                              dbg_vertex.pid stays the paper's partition, computed from the
                              vertex's canonical P-minimizer (reading V). */
+  uint32_t min_count;     /* row f4: vertices with count < min_count are dropped at extraction
+                             ("erroneous vertices can only be filtered by the number of their
+                             occurrences after the graph is constructed"; reading R).
+                             Their slots are still cleaned; dbg_stats and *d_n_out count only
+                             the vertices written; edge counters of kept vertices are unchanged.
+                             0 or 1 = keep every vertex (the unfiltered graph of Def. 3). */
 } dbg_params;
 
 /* One vertex of Definition 3: the canonical K-mer (the
@@ -266,6 +272,22 @@ DBG_API dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_
  * statistic is computed apart from the path. */
 DBG_API dbg_status dbg_checksum_vertices(const dbg_params* prm, const dbg_vertex* d_vertices, uint64_t n,
                                  dbg_stats* d_stats, cudaStream_t stream);
+
+/* ---- f4: graph writer ---------------------------
+ * Writes n host records (any order; sorted records from dbg_sort_vertices
+ * give a sorted file) to the file at path: a 64-byte dbg_graph_header, then
+ * the records.  append != 0 and an existing file with the same magic and K:
+ * the records are appended and header.n_vertices updated (one call per
+ * batch of partitions); otherwise the file is created or truncated.
+ * DBG_EINVAL on a bad argument, an I/O error or a header mismatch. */
+typedef struct {
+  char magic[8];           /* "PHDBG\0\0\1" (format version 1) */
+  uint32_t k, p, num_partitions, min_count;
+  uint64_t n_vertices;
+  uint64_t reserved[4];
+} dbg_graph_header;
+DBG_API dbg_status dbg_write_graph(const char* path, const dbg_params* prm, const dbg_vertex* h_vertices,
+                           uint64_t n, int append);
 
 /* Synchronizes the stream, then decodes *d_status: bit 0 -> DBG_ETABLEFULL,
  * bit 1 or 2 -> DBG_ENOSPACE; also returns DBG_ECUDA on a sticky CUDA error. */

@@ -184,3 +184,14 @@ def canonical(kmer: str):
 
 def kmer_minimizer(kmer: str, p: int) -> int:
     return int(_load().oracle_kmer_minimizer(kmer.encode(), len(kmer), p))
+
+
+def filter_low_count(records, min_count: int):
+    """Row f4 (Sec. III-C1: "these erroneous vertices can only be filtered by
+    the number of their occurrences after the graph is constructed"): the records whose vertex
+    count is at least ``min_count``, unchanged and in the same order (reading R: the
+    edge multiplicities of a kept vertex are not edited).  ``min_count`` <= 1 keeps every record."""
+    rec = np.asarray(records, dtype=VERTEX_DTYPE)
+    if min_count <= 1:
+        return rec.copy()
+    return rec[rec["count"] >= min_count].copy()

@@ -28,7 +28,7 @@ class DbgError(RuntimeError):
 class dbg_params(ctypes.Structure):
     _fields_ = [("k", ctypes.c_int32), ("p", ctypes.c_int32), ("num_partitions", ctypes.c_int32),
                 ("lambda_", ctypes.c_float), ("alpha", ctypes.c_float), ("refine", ctypes.c_int32),
-                ("smem_split", ctypes.c_int32), ("fine_p", ctypes.c_int32)]
+                ("smem_split", ctypes.c_int32), ("fine_p", ctypes.c_int32), ("min_count", ctypes.c_uint32)]
 
 
 class dbg_partition_set(ctypes.Structure):
@@ -77,12 +77,13 @@ SIGNATURES = {
     "dbg_sort_workspace_bytes": (_U64, [_PRM, _U64]),
     "dbg_sort_vertices": (ctypes.c_int, [_PRM, _P, _P, _U64, _P, _U64, _P]),
     "dbg_checksum_vertices": (ctypes.c_int, [_PRM, _P, _U64, _P, _P]),
+    "dbg_write_graph": (ctypes.c_int, [ctypes.c_char_p, _PRM, _P, _U64, ctypes.c_int]),
     "dbg_sync_status": (ctypes.c_int, [_P, _P]),
     "dbg_status_string": (ctypes.c_char_p, [ctypes.c_int]),
 }
 
 _lib = None
-ABI_VERSION = 3
+ABI_VERSION = 4
 
 
 def load():
@@ -129,8 +130,8 @@ def _stream(stream) -> int | None:
 
 
 def params(k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
-           refine: int = 1, smem_split: int = 0, fine_p: int = 0) -> dbg_params:
-    return dbg_params(k, p, num_partitions, lam, alpha, refine, smem_split, fine_p)
+           refine: int = 1, smem_split: int = 0, fine_p: int = 0, min_count: int = 0) -> dbg_params:
+    return dbg_params(k, p, num_partitions, lam, alpha, refine, smem_split, fine_p, min_count)
 
 
 def fine_partitions(prm: dbg_params) -> int:
@@ -269,6 +270,11 @@ def dbg_sort_vertices(prm, d_in, d_out, n: int, d_workspace, workspace_bytes: in
 def dbg_checksum_vertices(prm, d_vertices, n: int, d_stats, stream=None) -> None:
     _check("dbg_checksum_vertices", load().dbg_checksum_vertices(ctypes.byref(prm), _ptr(d_vertices), n,
                                                                  _ptr(d_stats), _stream(stream)))
+
+
+def dbg_write_graph(path: str, prm, h_vertices, n: int, append: bool = False) -> None:
+    _check("dbg_write_graph", load().dbg_write_graph(os.fsencode(path), ctypes.byref(prm), _ptr(h_vertices), n,
+                                                     int(bool(append))))
 
 
 def dbg_sync_status(d_status, stream=None) -> int:

@@ -1,11 +1,15 @@
 // api.cu -- host side of libdbg.so: sizes, the host 2-bit encoder (row a0) and
 // status handling.  See include/dbg.h for the contract of every entry point.
 #include <cmath>
+#include <cstdio>
 #include <cstring>
 
 #include "dbg_device.cuh"
 
 using namespace dbg;
+
+static_assert(sizeof(dbg_graph_header) == 64, "graph file header is 64 bytes");
+static const char kGraphMagic[8] = {'P', 'H', 'D', 'B', 'G', 0, 0, 1};
 
 extern "C" int dbg_abi_version(void) { return DBG_ABI_VERSION; }
 
@@ -57,6 +61,47 @@ extern "C" dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64
     h_words[w] = v;
   }
   return DBG_OK;
+}
+
+// Row f4 graph writer: the paper writes the constructed subgraphs to an output
+// graph file.  Format (little endian): a 64-byte
+// header {char magic[8] = "PHDBG\0\0\1"; u32 k, p, num_partitions, min_count;
+// u64 n_vertices; u64 reserved[4]} followed by n_vertices dbg_vertex records.
+// append != 0 adds records to an existing file and updates its count.
+extern "C" dbg_status dbg_write_graph(const char* path, const dbg_params* prm, const dbg_vertex* h_vertices,
+                                      uint64_t n, int append) {
+  if (!path || !prm || (n && !h_vertices)) return DBG_EINVAL;
+  dbg_graph_header h;
+  memset(&h, 0, sizeof(h));
+  FILE* f = nullptr;
+  if (append) f = fopen(path, "r+b");
+  if (f) {
+    if (fread(&h, sizeof(h), 1, f) != 1 || memcmp(h.magic, kGraphMagic, 8) != 0 || h.k != (uint32_t)prm->k) {
+      fclose(f);
+      return DBG_EINVAL;
+    }
+    if (fseek(f, 0, SEEK_END) != 0) {
+      fclose(f);
+      return DBG_EINVAL;
+    }
+  } else {
+    f = fopen(path, "wb");
+    if (!f) return DBG_EINVAL;
+    memcpy(h.magic, kGraphMagic, 8);
+    h.k = (uint32_t)prm->k;
+    h.p = (uint32_t)prm->p;
+    h.num_partitions = (uint32_t)prm->num_partitions;
+    h.min_count = prm->min_count;
+    if (fwrite(&h, sizeof(h), 1, f) != 1) {
+      fclose(f);
+      return DBG_EINVAL;
+    }
+  }
+  bool ok = n == 0 || fwrite(h_vertices, sizeof(dbg_vertex), n, f) == n;
+  h.n_vertices += n;
+  ok = ok && fseek(f, 0, SEEK_SET) == 0 && fwrite(&h, sizeof(h), 1, f) == 1;
+  ok = (fclose(f) == 0) && ok;
+  return ok ? DBG_OK : DBG_EINVAL;
 }
 
 extern "C" dbg_status dbg_sync_status(const uint32_t* d_status, cudaStream_t stream) {

@@ -309,6 +309,7 @@ struct OutArgs {
   unsigned long long* n_out;
   unsigned long long* stats;  // distinct, sum_count, sum_edges, checksum
   uint32_t* status;
+  uint32_t min_count;  // row f4: vertices with count < min_count are dropped (0, 1: keep all)
 };
 
 static OutArgs make_out_args(const dbg_params* prm, dbg_vertex* d_out, uint64_t out_cap, uint64_t* d_n_out,
@@ -324,6 +325,7 @@ static OutArgs make_out_args(const dbg_params* prm, dbg_vertex* d_out, uint64_t 
   oa.n_out = reinterpret_cast<unsigned long long*>(d_n_out);
   oa.stats = reinterpret_cast<unsigned long long*>(d_stats);
   oa.status = d_status;
+  oa.min_count = prm->min_count;
   return oa;
 }
 
@@ -388,6 +390,26 @@ __device__ __forceinline__ void extract_tile(char* keys, uint32_t* ctr, uint64_t
   for (int q = 0; q < kXPer; ++q) {
     const uint64_t s = (uint64_t)q * kThreads + threadIdx.x;
     if (s < n && (__ldcg(reinterpret_cast<const uint64_t*>(keys + s * KE)) & kOccupied)) bits |= 1u << q;
+  }
+  if (oa.min_count > 1) {  // row f4: drop (and clean) the vertices with count < min_count
+    uint32_t b = bits;
+    while (b) {
+      const int q = __ffs(b) - 1;
+      b &= b - 1;
+      const uint64_t s = (uint64_t)q * kThreads + threadIdx.x;
+      uint4* kp4 = reinterpret_cast<uint4*>(keys + s * KE);
+      uint4* cp = reinterpret_cast<uint4*>(ctr + s * 8);
+      const uint32_t tout = __ldcg(reinterpret_cast<const uint32_t*>(keys + s * KE + (KW == 1 ? 8 : 16)));
+      const uint4 a = __ldcg(cp);
+      if (a.x + a.y + a.z + a.w + tout < oa.min_count) {
+        const uint4 z = make_uint4(0, 0, 0, 0);
+        __stcg(kp4, z);
+        if (KW == 2) __stcg(kp4 + 1, z);
+        __stcg(cp, z);
+        __stcg(cp + 1, z);
+        bits &= ~(1u << q);
+      }
+    }
   }
   const uint32_t cnt = __popc(bits);
   uint32_t excl, total;
@@ -1247,12 +1269,22 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       constexpr int kWarps = kSmemThreads / 32;
       const uint32_t wspan = (span + kWarps * 32 - 1) / (kWarps * 32) * 32;  // slots per warp
       const uint32_t ws0 = min(span, warp * wspan), ws1 = min(span, ws0 + wspan);
+      // row f4: a vertex with count < min_count is cleaned here and never emitted
+      auto keep = [&](uint32_t s) -> bool {
+        if (s >= ws1 || !(*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied)) return false;
+        if (oa.min_count <= 1) return true;
+        uint32_t* f = fld + s * FW;
+        const uint32_t f0 = f[0], f1 = f[1];
+        if ((f0 & 0xffffu) + (f0 >> 16) + (f1 & 0xffffu) + (f1 >> 16) + (f[4] & 0xffffu) >= oa.min_count) return true;
+        unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+        kp[0] = 0;
+        if (KW == 2) kp[1] = 0;
+#pragma unroll
+        for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
+        return false;
+      };
       uint32_t cnt = 0;
-      for (uint32_t c = ws0; c < ws1; c += 32) {
-        const uint32_t s = c + lane;
-        cnt += __popc(__ballot_sync(kFull, s < ws1 &&
-                                              (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied)));
-      }
+      for (uint32_t c = ws0; c < ws1; c += 32) cnt += __popc(__ballot_sync(kFull, keep(c + lane)));
       uint32_t excl, total;
       Scan(st.scan).ExclusiveSum(lane == 0 ? cnt : 0u, excl, total);
       if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
@@ -1264,7 +1296,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         for (uint32_t c = sub; c < min(ws1, sub + 128); c += 32) {
           const uint32_t s = c + lane;
           const bool occ = s < ws1 && (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied);
-          const uint32_t bal = __ballot_sync(kFull, occ);
+          const uint32_t bal = __ballot_sync(kFull, occ);  // filtered slots were cleaned by keep()
           if (occ) queue[qn + __popc(bal & ((1u << lane) - 1u))] = s;
           qn += __popc(bal);
         }

@@ -72,7 +72,7 @@ class DbgBuilder:
     def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
                  device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
                  mode: str = "smem", group_slots: int = 1 << 19, refine: int = 1, smem_split: int = 0,
-                 fine_p: int = 0):
+                 fine_p: int = 0, min_count: int = 0):
         if k % 2 == 0 or not 1 <= k <= 63:
             raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
         if not 1 <= p <= min(k, 31):
@@ -88,7 +88,9 @@ class DbgBuilder:
         self.owned = (0, self.np)  # fine partitions this builder hashes (multi-GPU: a shard)
         self.smem_split = int(smem_split)  # 0: library default (dbg_params.smem_split)
         self.fine_p = int(fine_p)          # 0: P (dbg_params.fine_p)
-        self.prm = _lib.params(k, p, num_partitions, lam, alpha, self.refine, self.smem_split, self.fine_p)
+        self.min_count = int(min_count)    # row f4: drop vertices with count < min_count (0, 1: none)
+        self.prm = _lib.params(k, p, num_partitions, lam, alpha, self.refine, self.smem_split, self.fine_p,
+                               self.min_count)
         self.device = torch.device(device)
         _lib.load()
         self.rec_words = _lib.dbg_record_words(self.prm)
@@ -275,11 +277,6 @@ class DbgBuilder:
         else:
             _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
         self._done(ev, stream)
-        # d_fill is idle after the scatter: scratch of the multi-CTA scan
-        if self.mode == "smem":  # on-chip partitions need no global table
-            _lib.dbg_table_plan_split(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
-        else:
-            _lib.dbg_table_plan(self.prm, self.d_n_kmers, self.d_tab_off, self.d_fill, stream)
         if self._tab_key != self._caps_key:
             self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
             self.tab_host[1:] = np.cumsum(self.caps)
@@ -440,7 +437,7 @@ class DbgBuilder:
                 if self.prm.lambda_ / (4 * self.prm.alpha) >= 1.0:
                     raise _lib.DbgError("dbg_hash_build", st, "table full at capacity >= N^i_kmer")
                 self.prm = _lib.params(self.k, self.p, self.np_out, 2.0, 0.5, self.refine, self.smem_split,
-                                       self.fine_p)
+                                       self.fine_p, self.min_count)
                 self.plan(stream)
                 continue
             if st != _lib.DBG_OK:
@@ -449,6 +446,30 @@ class DbgBuilder:
         verts = self.vertices(sort=sort, stream=stream) if want_vertices else None
         return GraphResult(verts, int(self.d_n_out.item()), self.stats(), n_kmers, self.part_kmers.copy(),
                            self.part_records.copy(), list(self.batches))
+
+
+GRAPH_HEADER_DTYPE = np.dtype([("magic", "S8"), ("k", "<u4"), ("p", "<u4"), ("num_partitions", "<u4"),
+                               ("min_count", "<u4"), ("n_vertices", "<u8"), ("reserved", "<u8", (4,))])
+assert GRAPH_HEADER_DTYPE.itemsize == 64
+
+
+def write_graph(path: str, prm: _lib.dbg_params, vertices: np.ndarray, append: bool = False) -> None:
+    """Row f4 graph writer (dbg_write_graph): host records -> graph file (64-B header + records)."""
+    v = np.ascontiguousarray(vertices, dtype=VERTEX_DTYPE)
+    _lib.dbg_write_graph(path, prm, v if len(v) else None, len(v), append)
+
+
+def read_graph(path: str) -> tuple[dict, np.ndarray]:
+    """Reads a file written by dbg_write_graph: (header fields, records)."""
+    raw = np.fromfile(path, dtype=np.uint8)
+    h = raw[:64].view(GRAPH_HEADER_DTYPE)[0]
+    if bytes(h["magic"]).ljust(8, b"\0") != b"PHDBG\0\0\x01":
+        raise ValueError(f"{path}: not a graph file")
+    n = int(h["n_vertices"])
+    recs = raw[64:64 + n * VERTEX_DTYPE.itemsize].view(VERTEX_DTYPE)
+    if len(recs) != n:
+        raise ValueError(f"{path}: truncated ({len(recs)} of {n} records)")
+    return {f: int(h[f]) for f in ("k", "p", "num_partitions", "min_count", "n_vertices")}, recs.copy()
 
 
 def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
@@ -482,7 +503,7 @@ def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partit
                 lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
                 table_budget_bytes: int | None = None, mode: str = "smem",
                 group_slots: int = 1 << 19, refine: int | str = "auto", smem_split: int = 0,
-                fine_p: int | str = "auto") -> GraphResult:
+                fine_p: int | str = "auto", min_count: int = 0) -> GraphResult:
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
     lens = np.diff(np.asarray(offsets, dtype=np.int64))
     n_kmers = int(np.maximum(lens - k + 1, 0).sum())
@@ -491,7 +512,7 @@ def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partit
     if fine_p == "auto":
         fine_p = auto_fine_p(n_kmers, k, p, lam, alpha) if mode == "smem" else 0
     builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots, refine,
-                         smem_split, fine_p)
+                         smem_split, fine_p, min_count)
     packed = encode_reads(seq)
     d_bases, d_offsets = builder.upload(packed, offsets)
     return builder.build(d_bases, d_offsets, sort=sort)

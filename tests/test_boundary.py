@@ -28,7 +28,7 @@ def _declared():
 
 def test_exports_every_declared_symbol(lib):
     names = _declared()
-    assert len(names) == 26
+    assert len(names) == 27
     raw = lib.load()
     for n in names:
         assert hasattr(raw, n), n
@@ -36,7 +36,7 @@ def test_exports_every_declared_symbol(lib):
 
 
 def test_abi_and_sizes(lib):
-    assert lib.dbg_abi_version() == 3
+    assert lib.dbg_abi_version() == 4
     p31 = lib.params(31, 11, 16)
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
@@ -150,3 +150,28 @@ def test_product_has_no_oracle_dependency():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert not bad.search(src), f
+
+
+def test_graph_writer_roundtrip(lib, tmp_path):
+    """Row f4 graph writer (host-only entry point): header + records, append updates the count."""
+    from paper_conf_icdcs_qiul17_b200 import read_graph, write_graph
+
+    rng = np.random.default_rng(3)
+    v = np.zeros(1000, dtype=lib.VERTEX_DTYPE)
+    v["kmer_lo"] = rng.integers(0, 1 << 62, 1000, dtype=np.uint64)
+    v["count"] = rng.integers(1, 50, 1000)
+    v["out"] = rng.integers(0, 9, (1000, 4))
+    v["pid"] = rng.integers(0, 16, 1000)
+    prm = lib.params(31, 11, 16, min_count=2)
+    path = str(tmp_path / "g.dbg")
+    write_graph(path, prm, v[:600])
+    write_graph(path, prm, v[600:], append=True)
+    write_graph(path, prm, v[:0], append=True)
+    h, got = read_graph(path)
+    assert h == {"k": 31, "p": 11, "num_partitions": 16, "min_count": 2, "n_vertices": 1000}
+    assert got.tobytes() == v.tobytes()
+    assert os.path.getsize(path) == 64 + 56 * 1000
+    with pytest.raises(lib.DbgError):  # append with another K: header mismatch
+        write_graph(path, lib.params(33, 11, 16), v[:1], append=True)
+    write_graph(path, prm, v[:5])  # no append: truncates
+    assert read_graph(path)[0]["n_vertices"] == 5

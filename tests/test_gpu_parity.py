@@ -371,3 +371,29 @@ def test_staging_overflow_repeats_the_step():
     res = b.build(d_bases, d_off)
     orc = oracle.graph(rs.seq, rs.offsets, 31, 11, 16, n_threads=NT)
     compare_vertices(res.vertices, orc)
+
+
+@pytest.mark.parametrize("mode,k,p,np_,refine,split", [("smem", 31, 11, 4, 8, 0), ("smem", 31, 11, 2, 1, 1),
+                                                       ("smem", 63, 19, 3, 2, 0), ("fused", 31, 11, 16, 1, 0),
+                                                       ("resident", 63, 19, 8, 1, 0)])
+@pytest.mark.parametrize("min_count", [2, 3])
+def test_low_count_filter(mode, k, p, np_, refine, split, min_count):
+    """Row f4: extraction drops vertices with count < min_count, in every Step-2 tier
+    (grouped and split on-chip tables, global tables), and equals oracle.filter_low_count."""
+    g = genome(30_000, seed=21)
+    seq, offs = make_reads(g, 6000, 100, 0.01, seed=22)
+    rs = ReadSet(seq, offs)
+    b = DbgBuilder(k, p, np_, mode=mode, refine=refine, smem_split=split, min_count=min_count)
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    res = b.build(d_bases, d_off)
+    full = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT)
+    orc = oracle.filter_low_count(full, min_count)
+    assert 0 < len(orc) < len(full)
+    compare_vertices(res.vertices, orc)
+    assert res.stats["distinct"] == len(orc)
+    assert res.stats["sum_count"] == int(orc["count"].sum())
+    assert res.stats["checksum"] == oracle.checksum(orc)
+    # the resident tables were cleaned, filtered slots included: an unfiltered rebuild with the same
+    # builder (same table buffers) is exact
+    b.prm.min_count = b.min_count = 0
+    compare_vertices(b.build(d_bases, d_off).vertices, full)

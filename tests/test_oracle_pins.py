@@ -295,3 +295,43 @@ def test_checksum_order_independent(oracle_lib):
     for x in (0, 1, 2, 0xDEADBEEF, (1 << 64) - 1):
         assert oracle_lib.fmix64(x) == brute.fmix64(x)
     assert brute.fmix64(0) == 0
+
+
+# ---------------------------------------------------------------- row f4: low-count filtering
+
+
+def test_filter_low_count_keeps_genome_kmers(oracle_lib):
+    """Row f4: "a single error ... generates ... K erroneous kmers ... these
+    erroneous vertices can only be filtered by the number of their occurrences".  Error-free reads
+    tile a random genome (every interior K-mer covered >= 3 times) and 40 reads carry one distinct
+    substitution each.  Filtering at 2 must keep exactly the K-mers occurring >= 2 times by a
+    string count (collections.Counter over canonical strings), which are genome K-mers only, with
+    their records unchanged; every erroneous K-mer (not in the genome on either strand) is gone."""
+    import collections
+
+    rng = np.random.default_rng(11)
+    K, P, NP, L = 21, 7, 8, 80
+    g = "".join("ACGT"[x] for x in rng.integers(0, 4, 2000))
+    reads = [g[s:s + L] for s in range(0, len(g) - L + 1, 20)]
+    errs = []
+    for j in range(40):
+        s = 25 * j + 3
+        r = list(g[s:s + L])
+        q = 40 + (j % 7)
+        r[q] = "ACGT"[("ACGT".index(r[q]) + 1 + j % 3) % 4]
+        errs.append("".join(r))
+    rs = _readset(reads + errs)
+    recs = oracle_lib.graph(rs.seq, rs.offsets, K, P, NP)
+    kept = oracle_lib.filter_low_count(recs, 2)
+    cnt = collections.Counter(brute.canonical_string(r[i:i + K]) for r in reads + errs for i in range(len(r) - K + 1))
+    want = {v for v, c in cnt.items() if c >= 2}
+    got = _as_dict(kept, K)
+    assert set(got) == want
+    genome_kmers = {brute.canonical_string(g[i:i + K]) for i in range(len(g) - K + 1)}
+    assert want <= genome_kmers
+    erroneous = set(cnt) - genome_kmers
+    assert len(erroneous) > 40 * (K - 5) and not (erroneous & set(got))
+    full = _as_dict(recs, K)
+    assert all(full[v] == e for v, e in got.items())  # kept records are not edited
+    assert len(oracle_lib.filter_low_count(recs, 1)) == len(recs)
+    assert len(oracle_lib.filter_low_count(recs, 0)) == len(recs)
