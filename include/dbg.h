@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 4
+#define DBG_ABI_VERSION 5
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -116,6 +116,13 @@ typedef struct {
   uint32_t* d_staging;       /* staging_cap records, read order (pass 1 output, pass 2 input) */
   uint64_t staging_cap;      /* capacity of d_staging in records */
   uint32_t* d_records;       /* d_record_offset[NP] records in partition order; NULL => pass 1 */
+  uint32_t* d_rank;          /* [staging_cap] or NULL.  Pass 1 writes each staged record's rank
+                                within its partition (the per-partition count it reserved), and
+                                pass 2 then places record i at d_record_offset[pid] + d_rank[i]
+                                without atomics.  NULL: pass 2 ranks with atomics on d_fill (the
+                                form for records that did not come from pass 1, e.g. received
+                                from other GPUs).  Pass 2 must see the pass-1 ranks of the same
+                                staging. */
 } dbg_partition_set;
 
 /* ---- sizes ------------------------------------------------------------ */

@@ -806,7 +806,10 @@ struct SmemStage {
   static constexpr int RB = smem_rec_batch<R, T>();
   uint32_t w[2][R][RB];                       // records of two batches, transposed: word q of record j at w[b][q][j]
   unsigned long long Pq[2][kGroupParts + 2];  // P[first .. last] of the current and the next item
-  uint32_t pre[RB + 1];
+  uint32_t pre[RB + 1];                       // K-mer offsets of the records with on-chip K-mers
+  uint2 desc[RB];                             // their descriptors: x = batch position | n << 10 |
+                                              // hl << 18 | hr << 19, y = table offset | capacity << 16
+  uint16_t rwin[(RB * (16 * (R - 1) - 1) + 31) / 32 + 1];  // record of the first K-mer of each warp window
   ItemDesc it[4];                             // items i .. i+3 (ring)
   typename cub::BlockScan<uint32_t, T>::TempStorage scan;
   typename cub::BlockReduce<unsigned long long, T>::TempStorage red;
@@ -834,6 +837,25 @@ __host__ __device__ constexpr uint32_t smem_fixed_bytes() {
   return (uint32_t)((sizeof(SmemStage<R, T>) + 127) & ~size_t(127));
 }
 
+// 32-bit shared-window addresses (no generic-pointer arithmetic in the probe loop).
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint64_t lds64(uint32_t a) {
+  uint64_t v;
+  asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t cas_shared64(uint32_t a, uint64_t want) {
+  uint64_t old;
+  asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(a), "l"(0ull), "l"(want) : "memory");
+  return old;
+}
+__device__ __forceinline__ void red_shared_add(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+
 __device__ __forceinline__ void smem_count(uint32_t* fields, int f) {
   atomicAdd(fields + (f >> 1), 1u << (16 * (f & 1)));
 }
@@ -845,37 +867,6 @@ __device__ __forceinline__ uint32_t smem_hash(uint64_t code) {
 __device__ __forceinline__ uint32_t smem_hash(unsigned long long code) { return smem_hash((uint64_t)code); }
 __device__ __forceinline__ uint32_t smem_hash(u128 code) {
   return smem_hash((uint64_t)((uint64_t)code ^ ((uint64_t)(code >> 64) * 0xc2b2ae3d27d4eb4full)));
-}
-
-// Insert/update of one occurrence in a shared-memory table of cap slots; the
-// inserting thread also records the (fine) partition id in field word 5,
-// read back at extraction.
-template <typename Code>
-__device__ __forceinline__ bool smem_upsert(char* keys, uint32_t* fld, uint32_t cap, Code code, int o, int i,
-                                            uint32_t pid) {
-  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  typedef KeyOf<Code> KO;
-  const typename KO::T want = KO::make(code);
-  uint32_t idx = __umulhi(smem_hash(code), cap);
-  for (uint32_t pr = 0; pr < cap; ++pr) {
-    char* kp = keys + idx * SmemSlot<KW>::kKeyBytes;
-    typename KO::T cur;
-    if constexpr (KW == 1) {
-      cur = *reinterpret_cast<volatile unsigned long long*>(kp);
-      if (cur == 0) cur = KO::cas(kp, want);
-    } else {
-      cur = KO::cas(kp, want);  // 16-B shared-memory CAS: atomic read-or-claim
-    }
-    if (KO::empty(cur) || KO::same(cur, want)) {
-      uint32_t* f = fld + idx * SmemSlot<KW>::kFieldWords;
-      if (KO::empty(cur)) f[5] = pid;
-      smem_count(f, o < 4 ? o : 8);
-      if (i >= 0) smem_count(f, 4 + i);
-      return true;
-    }
-    idx = idx + 1 == cap ? 0 : idx + 1;
-  }
-  return false;
 }
 
 struct SmemArgs {
@@ -1113,6 +1104,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
   char* keys = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
   uint32_t* fld = reinterpret_cast<uint32_t*>(keys + a.slots * KB);
+  const uint32_t keys_s = smem_addr(keys), fld_s = smem_addr(fld);
   const int K = a.k;
   {  // the table starts clean; extraction keeps it clean (slots is a multiple of 64)
     uint4* z = reinterpret_cast<uint4*>(keys);
@@ -1176,6 +1168,8 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
     }
     cp_async_commit();
     const unsigned long long* Pq = st.Pq[ip];
+    // Flatten the batch: one packed scan gives every record with on-chip K-mers its
+    // K-mer offset (low 16 bits) and its index among those records (high 16 bits).
     uint32_t cnt[kRPT];
 #pragma unroll
     for (int v = 0; v < kRPT; ++v) {
@@ -1183,123 +1177,172 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       cnt[v] = 0;
       if (j < nb) {
         const uint32_t w0 = st.w[bb][0][j];
+        uint32_t c;
         if (split) {
-          cnt[v] = w0 & 255u;
+          c = w0 & 255u;
         } else {
           const uint32_t x = (w0 >> 10) - I.first;
-          cnt[v] = Pq[x + 1] != Pq[x] ? w0 & 255u : 0u;  // off-chip partition: skipped here
+          c = Pq[x + 1] != Pq[x] ? w0 & 255u : 0u;  // off-chip partition: skipped here
         }
+        cnt[v] = c ? c | 1u << 16 : 0u;
       }
     }
-    uint32_t excl[kRPT], total;
-    Scan(st.scan).ExclusiveSum(cnt, excl, total);
+    uint32_t excl[kRPT], packed_total;
+    Scan(st.scan).ExclusiveSum(cnt, excl, packed_total);
+    const uint32_t total = packed_total & 0xffffu, nc = packed_total >> 16;
+    // Record c (compacted) holds K-mers [cpre[c], cpre[c+1]); rwin[m] = the record holding
+    // K-mer 32m, the first of warp window m.
 #pragma unroll
-    for (int v = 0; v < kRPT; ++v)
-      if (kRPT * threadIdx.x + v < RB) st.pre[kRPT * threadIdx.x + v] = excl[v];
-    if (threadIdx.x == 0) st.pre[RB] = total;
-    __syncthreads();
-    // this thread's contiguous run of K-mers [k0, k1)
-    const uint32_t share = (total + kSmemThreads - 1) / kSmemThreads;
-    const uint32_t k0 = min(total, threadIdx.x * share), k1 = min(total, k0 + share);
-    if (k0 < k1) {
-      int lo = 0, hi = nb;  // record holding K-mer k0: last r with pre[r] <= k0
-      while (hi - lo > 1) {
-        const int mid = (lo + hi) >> 1;
-        if (st.pre[mid] <= k0) lo = mid;
-        else hi = mid;
-      }
-      int r = lo;
-      while (st.pre[r + 1] == st.pre[r]) ++r;  // skip records that contribute nothing
-      constexpr int S = RB;                      // staging stride
-      const uint32_t* w;
-      int t = (int)(k0 - st.pre[r]), n, hl, hr;
-      char* tk;
-      uint32_t* tf;
-      uint32_t cap, pid;
-      auto header = [&](int rr) {  // record rr of the batch: its bases and its partition's table
-        w = &st.w[bb][0][rr];
-        const uint32_t w0 = w[0];
-        n = w0 & 255u;
-        hl = (w0 >> 8) & 1u;
-        hr = (w0 >> 9) & 1u;
-        pid = w0 >> 10;
-        uint64_t t0;
-        if (split) {
-          t0 = 0;
-          cap = (uint32_t)a.slots;
-        } else {
-          const uint32_t x = pid - I.first;
-          t0 = Pq[x] - I.P0;
-          cap = (uint32_t)(Pq[x + 1] - Pq[x]);
+    for (int v = 0; v < kRPT; ++v) {
+      if (cnt[v]) {
+        const uint32_t c = excl[v] >> 16, e = excl[v] & 0xffffu, n = cnt[v] & 0xffffu;
+        const int jj = kRPT * threadIdx.x + v;
+        const uint32_t w0 = st.w[bb][0][jj];
+        uint32_t t0 = 0, cp = (uint32_t)a.slots;
+        if (!split) {
+          const uint32_t x = (w0 >> 10) - I.first;
+          t0 = (uint32_t)(Pq[x] - I.P0);
+          cp = (uint32_t)(Pq[x + 1] - Pq[x]);
         }
-        tk = keys + t0 * KB;
-        tf = fld + t0 * FW;
-      };
-      header(r);
-      // Every K-mer is decoded from the staged words (no rolling): the lanes of a
-      // warp stay converged; only the small header reload at a record change diverges.
-      for (uint32_t kid = k0;;) {
+        st.pre[c] = e;
+        st.desc[c] = make_uint2((uint32_t)jj | (w0 & 1023u) << 10, t0 | cp << 16);
+        for (uint32_t m = (e + 31) >> 5; 32 * m < e + n; ++m) st.rwin[m] = (uint16_t)c;
+      }
+    }
+    if (threadIdx.x == 0) st.pre[nc] = total;
+    __syncthreads();
+    {
+      // Warp windows: window m = K-mers [32m, 32m + 32), lane l takes K-mer 32m + l;
+      // window m goes to warp m mod (warps), so the warps' loads differ by at most one
+      // window and no thread waits on a long record.  All lanes run every step, so the
+      // probe vote is warp-wide and the counter updates run reconverged.
+      constexpr int S = RB;  // staging stride
+      constexpr uint32_t kWarps = kSmemThreads / 32;
+      typedef KeyOf<Code> KO;
+      for (uint32_t m = warp; 32 * m < total; m += kWarps) {
+        const uint32_t kb = 32 * m, kid = kb + lane;
+        const bool act = kid < total;
+        const uint32_t rb = st.rwin[m];
+        // records starting inside the window: one bit each at their first K-mer
+        const uint32_t nxt = rb + 1 + lane;
+        const uint32_t x0 = nxt < nc ? st.pre[nxt] : total;
+        const uint32_t starts = __reduce_or_sync(kFull, x0 < kb + 32 ? 1u << (x0 - kb) : 0u);
+        const uint32_t c = rb + __popc(starts & ((2u << lane) - 1u));
+        const uint32_t cc = act ? c : rb;
+        const uint2 d = st.desc[cc];
+        const int t = (int)(kid - st.pre[cc]);
+        const int j = d.x & 1023u, n = (d.x >> 10) & 255u, hl = (d.x >> 18) & 1u, hr = (d.x >> 19) & 1u;
+        const uint32_t t0 = d.y & 0xffffu, cap = d.y >> 16;
+        const uint32_t* w = &st.w[bb][0][j];
         const int b = hl + t;
         Code fwd, rc;
-        kmer_at(w, b, K, R, fwd, rc, S);
-        const int pred = b > 0 ? (int)rec_base(w, b - 1, S) : -1;
-        const int succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K, S) : -1;
+        int pred, succ;
+        if constexpr (R == 4) {
+          const int q = b >> 4;  // the words holding bases b .. b + 47 - 16q
+          const uint32_t a1 = w[(1 + q) * S], a2 = q < 2 ? w[(2 + q) * S] : 0u, a3 = q == 0 ? w[3 * S] : 0u;
+          const int pb = b - 1;  // the predecessor base
+          pred = b > 0 ? (int)((w[(1 + (pb >> 4)) * S] >> (30 - 2 * (pb & 15))) & 3u) : -1;
+          if constexpr (sizeof(Code) == 8) {
+            // 64 bits of the record from base b: two 32-bit funnel shifts
+            const uint32_t sh = 2 * (b & 15);
+            const uint64_t win = ((uint64_t)__funnelshift_l(a2, a1, sh) << 32) | __funnelshift_l(a3, a2, sh);
+            fwd = win >> (64 - 2 * K);
+            succ = (t < n - 1 || hr) ? (int)((win >> (62 - 2 * K)) & 3u) : -1;
+            rc = revcomp64(fwd, K);
+          } else {
+            const u128 X = ((u128)(((uint64_t)a1 << 32) | a2) << 64) | ((u128)a3 << 32);
+            const u128 Y = X << (2 * (b & 15));
+            fwd = (Code)(Y >> (128 - 2 * K));
+            succ = (t < n - 1 || hr) ? (int)((uint32_t)(uint64_t)(Y >> (126 - 2 * K)) & 3u) : -1;
+            rc = revcomp128(fwd, K);
+          }
+        } else {
+          kmer_at(w, b, K, R, fwd, rc, S);
+          pred = b > 0 ? (int)rec_base(w, b - 1, S) : -1;
+          succ = (t < n - 1 || hr) ? (int)rec_base(w, b + K, S) : -1;
+        }
         // canonical orientation and edge indices (readings C, J), selected branch-free so
-        // that one upsert serves both orientations (no divergent duplicate of it)
+        // that one probe serves both orientations
         const bool is_fwd = fwd < rc;
         const Code code = is_fwd ? fwd : rc;
         const int o = is_fwd ? (succ >= 0 ? succ : 4) : (pred >= 0 ? 3 - pred : 4);
         const int i = is_fwd ? pred : (succ >= 0 ? 3 - succ : -1);
-        if (sub_n == 1 || sub_table(code, sub_n) == sub_j) ok &= smem_upsert<Code>(tk, tf, cap, code, o, i, pid);
-        if (++kid >= k1) break;
-        if (++t == n) {  // next record that contributes K-mers
-          do ++r;
-          while (st.pre[r + 1] == st.pre[r]);
-          t = 0;
-          header(r);
+        const bool want = act && (sub_n == 1 || sub_table(code, sub_n) == sub_j);
+        // one insertion, multiple updates: probe rounds until every lane has
+        // found or claimed its slot, then the counter updates, warp-converged
+        const typename KO::T key = KO::make(code);
+        uint32_t idx = __umulhi(smem_hash(code), cap), probes = 0;
+        uint32_t pend = want, inserted = 0;
+        const uint32_t kaddr = keys_s + t0 * KB;
+        while (__any_sync(kFull, pend)) {
+          if (pend) {
+            typename KO::T cur;
+            if constexpr (KW == 1) {
+              const uint32_t ka = kaddr + idx * KB;
+              cur = lds64(ka);
+              if (cur == 0) cur = cas_shared64(ka, key);
+            } else {
+              cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);  // 16-B shared-memory CAS: read-or-claim
+            }
+            inserted = KO::empty(cur);
+            if (inserted | KO::same(cur, key)) {
+              pend = 0;
+            } else {
+              idx = idx + 1 == cap ? 0 : idx + 1;
+              if (++probes == cap) {  // wrapped: table full (reading O)
+                pend = 0;
+                ok = false;
+                idx = ~0u;
+              }
+            }
+          }
+        }
+        if (want && idx != ~0u) {  // the multiple updates: 16-bit fields, two per word
+          const uint32_t fa = fld_s + (t0 + idx) * (FW * 4);
+          if (inserted) sts32(fa + 20, w[0] >> 10);
+          const int fo = o < 4 ? o : 8;
+          red_shared_add(fa + 4 * (fo >> 1), 1u << (16 * (fo & 1)));
+          if (i >= 0) red_shared_add(fa + 4 * ((4 + i) >> 1), 1u << (16 * (i & 1)));
         }
       }
     }
     if (last_batch) {
       __syncthreads();
-      // extraction: each warp owns a contiguous run of slots; one block scan of the
-      // warps' occupied counts sizes the item's output, one global atomic reserves it.
-      // Occupied slot indices are then queued per warp (in the batch's finished record
-      // buffer, 128 entries per warp) and emitted with every lane busy.
+      // extraction: each warp owns a contiguous run of slots and works alone: it queues
+      // the kept occupied slots of a chunk (16-bit indices, in the finished record buffer
+      // of this batch), reserves their output with one global atomic and emits them with
+      // every lane busy -- no block-wide scan or barrier.
       constexpr int kWarps = kSmemThreads / 32;
+      constexpr uint32_t kQ = (uint32_t)(sizeof(st.w[0]) / 2 / kWarps) / 32 * 32;  // queue entries per warp
       const uint32_t wspan = (span + kWarps * 32 - 1) / (kWarps * 32) * 32;  // slots per warp
       const uint32_t ws0 = min(span, warp * wspan), ws1 = min(span, ws0 + wspan);
-      // row f4: a vertex with count < min_count is cleaned here and never emitted
-      auto keep = [&](uint32_t s) -> bool {
-        if (s >= ws1 || !(*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied)) return false;
-        if (oa.min_count <= 1) return true;
-        uint32_t* f = fld + s * FW;
-        const uint32_t f0 = f[0], f1 = f[1];
-        if ((f0 & 0xffffu) + (f0 >> 16) + (f1 & 0xffffu) + (f1 >> 16) + (f[4] & 0xffffu) >= oa.min_count) return true;
-        unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
-        kp[0] = 0;
-        if (KW == 2) kp[1] = 0;
-#pragma unroll
-        for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
-        return false;
-      };
-      uint32_t cnt = 0;
-      for (uint32_t c = ws0; c < ws1; c += 32) cnt += __popc(__ballot_sync(kFull, keep(c + lane)));
-      uint32_t excl, total;
-      Scan(st.scan).ExclusiveSum(lane == 0 ? cnt : 0u, excl, total);
-      if (threadIdx.x == 0) st.base = total ? atomicAdd(oa.n_out, (unsigned long long)total) : 0ull;
-      __syncthreads();
-      uint64_t pos = st.base + __shfl_sync(kFull, excl, 0);
-      uint32_t* queue = &st.w[bb][0][0] + warp * 128;
-      for (uint32_t sub = ws0; sub < ws1; sub += 128) {
+      uint16_t* queue = reinterpret_cast<uint16_t*>(&st.w[bb][0][0]) + warp * kQ;
+      for (uint32_t sub = ws0; sub < ws1; sub += kQ) {
+        const uint32_t se = min(ws1, sub + kQ);
         uint32_t qn = 0;
-        for (uint32_t c = sub; c < min(ws1, sub + 128); c += 32) {
+        for (uint32_t c = sub; c < se; c += 32) {
           const uint32_t s = c + lane;
-          const bool occ = s < ws1 && (*reinterpret_cast<const unsigned long long*>(keys + s * KB) & kOccupied);
-          const uint32_t bal = __ballot_sync(kFull, occ);  // filtered slots were cleaned by keep()
-          if (occ) queue[qn + __popc(bal & ((1u << lane) - 1u))] = s;
+          bool keep = s < se && (lds64(keys_s + s * KB) & kOccupied);
+          if (keep && oa.min_count > 1) {  // row f4: a low-count vertex is cleaned, never emitted
+            const uint32_t* f = fld + s * FW;
+            const uint32_t f0 = f[0], f1 = f[1];
+            if ((f0 & 0xffffu) + (f0 >> 16) + (f1 & 0xffffu) + (f1 >> 16) + (f[4] & 0xffffu) < oa.min_count) {
+              keep = false;
+              unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+              kp[0] = 0;
+              if (KW == 2) kp[1] = 0;
+              uint32_t* fz = fld + s * FW;
+#pragma unroll
+              for (uint32_t q = 0; q < FW; ++q) fz[q] = 0;
+            }
+          }
+          const uint32_t bal = __ballot_sync(kFull, keep);
+          if (keep) queue[qn + __popc(bal & ((1u << lane) - 1u))] = (uint16_t)s;
           qn += __popc(bal);
         }
+        unsigned long long pos = 0;
+        if (lane == 0 && qn) pos = atomicAdd(oa.n_out, (unsigned long long)qn);
+        pos = __shfl_sync(kFull, pos, 0);
         __syncwarp();
         for (uint32_t e = lane; e < qn; e += 32) {
           const uint32_t s = queue[e];
@@ -1331,7 +1374,6 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           st_count += v.count;
           st_edges += (uint64_t)v.out[0] + v.out[1] + v.out[2] + v.out[3] + v.in[0] + v.in[1] + v.in[2] + v.in[3];
         }
-        pos += qn;
         __syncwarp();
       }
       ci = (ci + 1) & 3;

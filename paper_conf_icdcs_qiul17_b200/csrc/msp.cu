@@ -51,6 +51,7 @@ struct MspArgs {
   uint32_t* staging;              // records in read order
   uint64_t staging_cap;           // records
   unsigned long long* staged;     // cursor (records reserved)
+  uint32_t* rank;                 // [staging_cap] rank of each staged record in its partition, or null
 };
 
 template <typename CT>
@@ -125,11 +126,16 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
     const int n = e - s + 1;
     const uint32_t pieces = (uint32_t)((n + nmax - 1) / nmax);
-    atomicAdd(a.n_records + pid, (unsigned long long)pieces);
+    // the per-partition record count doubles as the records' ranks in their partition
+    uint32_t rk = 0;
+    if (a.rank) rk = (uint32_t)atomicAdd(a.n_records + pid, (unsigned long long)pieces);
+    else atomicAdd(a.n_records + pid, (unsigned long long)pieces);
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
-    for (int ps = s; ps <= e; ps += nmax, ++slot) {
-      if (slot < a.staging_cap)
+    for (int ps = s; ps <= e; ps += nmax, ++slot, ++rk) {
+      if (slot < a.staging_cap) {
         write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
+        if (a.rank) a.rank[slot] = rk;
+      }
     }
     s = e + 1;
   }
@@ -216,6 +222,28 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
       if (__any_sync(kFull, ndesc > kMaxDesc - 34)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
     }
     if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+  }
+}
+
+// Pass 3 with the ranks of pass 1: record i goes to rec_off[pid] + rank[i]
+// (no atomics; a coalesced read, one random 16/32-byte write per record).
+template <int R>
+__global__ void __launch_bounds__(256) scatter_ranked_kernel(const uint32_t* __restrict__ staging,
+                                                            const uint32_t* __restrict__ rank,
+                                                            const unsigned long long* staged, uint64_t staging_cap,
+                                                            const uint64_t* __restrict__ rec_off,
+                                                            uint32_t* __restrict__ records) {
+  const uint64_t n = *staged;
+  if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint4* src = reinterpret_cast<const uint4*>(staging + i * R);
+    uint4 rec[R / 4];
+#pragma unroll
+    for (int c = 0; c < R / 4; ++c) rec[c] = __ldcs(src + c);
+    const uint64_t pos = __ldg(rec_off + (rec[0].x >> 10)) + __ldcs(rank + i);
+    uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
+#pragma unroll
+    for (int c = 0; c < R / 4; ++c) dst[c] = rec[c];
   }
 }
 
@@ -332,6 +360,7 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
     a.staging = part->d_staging;
     a.staging_cap = part->staging_cap;
     a.staged = reinterpret_cast<unsigned long long*>(part->d_staged);
+    a.rank = part->d_rank;
     if (cudaMemsetAsync(part->d_n_records, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
         cudaMemsetAsync(part->d_n_kmers, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
         cudaMemsetAsync(part->d_staged, 0, sizeof(uint64_t), stream) != cudaSuccess)
@@ -350,7 +379,20 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
       return DBG_ECUDA;
   } else {
     // pass 3: scatter (a no-op after a staging overflow, *d_staged > staging_cap)
-    if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
+    if (!part->d_staging) return DBG_EINVAL;
+    if (part->d_rank) {  // ranks from pass 1: no atomics
+      const int grid = dbg_sm_count() * 8;
+      if (R == 4)
+        scatter_ranked_kernel<4><<<grid, 256, 0, stream>>>(
+            part->d_staging, part->d_rank, reinterpret_cast<const unsigned long long*>(part->d_staged),
+            part->staging_cap, part->d_record_offset, part->d_records);
+      else
+        scatter_ranked_kernel<8><<<grid, 256, 0, stream>>>(
+            part->d_staging, part->d_rank, reinterpret_cast<const unsigned long long*>(part->d_staged),
+            part->staging_cap, part->d_record_offset, part->d_records);
+      return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+    }
+    if (!part->d_fill) return DBG_EINVAL;
     if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * np, stream) != cudaSuccess) return DBG_ECUDA;
     const size_t smem = np <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * np : 0;
     const int grid = dbg_sm_count() * 4;
