@@ -28,6 +28,9 @@ sys.path.insert(0, ROOT)
 
 METRIC = "K-mers hashed/sec (graph build, device-timed) at 1/2/4/8 B200; HBM roofline %"
 UNIT = "kmers/s"
+# version tag of the on-chip kernel: profiles/traffic.json (ncu --set full) is quoted only when it
+# was captured on this version
+KERNEL_VERSION = "smem-v6"
 
 
 def _peaks():
@@ -198,18 +201,30 @@ def _placement(b) -> dict:
 
 
 def run_ours(args):
+    """Our arm.  N = 1: the whole path on one GPU.  N > 1 (torchrun): one process per GPU, weak
+    scaling -- every rank owns a read set of the configuration's size (same genome, its own reads);
+    a step is multi.distributed_step (local MSP, one record exchange to the partition owners,
+    owned-partition Step 2, NCCL reduces), timed on each rank's stream, max over ranks."""
     import torch
 
     ws, rank, local = _dist()
-    if ws > 1:
-        from paper_conf_icdcs_qiul17_b200 import multi
-
-        return multi.bench_main(args, METRIC, UNIT)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     from paper_conf_icdcs_qiul17_b200 import DbgBuilder, auto_fine_p, auto_refine, encode_reads, _lib
 
-    rs, gen_s = _workload(args)
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+        from paper_conf_icdcs_qiul17_b200 import multi
+
+        dist.init_process_group("nccl", device_id=dev)
+    t = time.time()
+    from synth import make_config
+
+    rs = make_config(args.config, scale=args.scale, num_partitions=args.np, read_seed_offset=7919 * rank)
+    if args.p is not None:
+        rs.p = args.p
+    gen_s = time.time() - t
     packed = encode_reads(rs.seq, pin=True)
     offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
     n_kmers = rs.n_kmers()
@@ -220,8 +235,10 @@ def run_ours(args):
     fine_p = args.fine_p
     if fine_p is None:
         fine_p = auto_fine_p(n_kmers, rs.k, rs.p, args.lam, args.alpha) if args.mode == "smem" else 0
+    if ws > 1 and args.mode != "smem":
+        raise SystemExit("multi-GPU runs use mode smem")
     b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode,
-                   args.group_slots, refine, args.smem_split, fine_p)
+                   args.group_slots, refine, args.smem_split, fine_p, args.min_count)
     d_bases, d_off = b.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
@@ -231,10 +248,13 @@ def run_ours(args):
 
     host_ms = {"msp": [], "plan": [], "reset": [], "step2": []}
 
-    def step():
-        """One pass of rows a2-a7 (MSP, sizing, on-chip / global Step 2)."""
+    def step(db, do):
+        """One pass of rows a2-a7 (MSP, sizing, on-chip / global Step 2) on this rank."""
+        if ws > 1:
+            multi.distributed_step(b, db, do, stream, out_cap)
+            return
         t = time.perf_counter()
-        b.msp(d_bases, d_off, stream)
+        b.msp(db, do, stream)
         t1 = time.perf_counter()
         b.plan(stream)
         t2 = time.perf_counter()
@@ -245,8 +265,20 @@ def run_ours(args):
         for k, v in zip(("msp", "plan", "reset", "step2"), (t1 - t, t2 - t1, t3 - t2, t4 - t3)):
             host_ms[k].append(1e3 * v)
 
+    def barrier():
+        torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
     for _ in range(args.warmup):
-        step()
+        step(d_bases, d_off)
     st = _lib.dbg_sync_status(b.d_status, stream)
     assert st == 0, _lib.dbg_status_string(st)
 
@@ -255,20 +287,24 @@ def run_ours(args):
     with ClockSampler(local) as clk:
         for _ in range(args.steps):
             flush.zero_()
+            barrier()
             e0, e1 = E(), E()
-            torch.cuda.synchronize()
             e0.record(stream)
-            step()
+            step(d_bases, d_off)
             e1.record(stream)
-            torch.cuda.synchronize()
+            barrier()
             step_ms.append(e0.elapsed_time(e1))
     phases = {k: statistics.mean(a.elapsed_time(c) for a, c in v) for k, v in b.timer.items()}
     b.timer = None
     st = _lib.dbg_sync_status(b.d_status, stream)
     stats = b.stats()
     L = rs.lengths()
-    inv_ok = (st == 0 and stats["sum_count"] == n_kmers
-              and stats["sum_edges"] == 2 * int(np.maximum(L - rs.k, 0).sum()))
+    tot = torch.tensor([n_kmers, stats["sum_count"], stats["sum_edges"], stats["distinct"],
+                        2 * int(np.maximum(L - rs.k, 0).sum()), int(st == 0)], dtype=torch.int64, device=dev)
+    if dist is not None:
+        dist.all_reduce(tot)
+    total_kmers, sum_count, sum_edges, distinct, want_edges, ok_ranks = (int(x) for x in tot.cpu())
+    inv_ok = ok_ranks == ws and sum_count == total_kmers and sum_edges == want_edges
 
     # e2e through the public API: H2D of the packed reads (pinned) + path + D2H of the stats
     e2e_ms, h2d_ms = [], []
@@ -277,77 +313,96 @@ def run_ours(args):
     host_stats = torch.empty(4, dtype=torch.int64, pin_memory=True)
     for _ in range(max(3, min(args.steps, 5))):
         flush.zero_()
-        torch.cuda.synchronize()
+        barrier()
         e0, e1, eh = E(), E(), E()
         e0.record(stream)
         db.copy_(packed, non_blocking=True)   # H2D of the step's input from pinned memory
         do.copy_(offsets, non_blocking=True)
         eh.record(stream)
-        b.msp(db, do, stream)
-        b.plan(stream)
-        b.reset_output(out_cap, stream)
-        b.step2(stream)
+        step(db, do)
         host_stats.copy_(b.d_stats, non_blocking=True)  # D2H of the step's result
         e1.record(stream)
-        torch.cuda.synchronize()
-        e2e_ms.append(e0.elapsed_time(e1))
+        barrier()
+        e2e_ms.append(max_over_ranks(e0.elapsed_time(e1)))
         h2d_ms.append(e0.elapsed_time(eh))
     h2d = packed.numel() * 8 + offsets.numel() * 8
-    d2h = 32 + 16 * rs.num_partitions
+    d2h = 32
 
-    ms = statistics.mean(step_ms)
+    ms = max_over_ranks(statistics.mean(step_ms))
     key = {"fused": "step2", "resident": "hash_build", "smem": "step2_smem"}[args.mode]
     hash_ms = phases.get(key, float("nan")) + (phases.get("hash_build", 0.0) + phases.get("extract", 0.0)
                                                if args.mode == "smem" else 0.0)
+    # this rank's Step-2 work (after the exchange: the K-mers of its own partitions)
+    my_kmers = int(b.part_kmers.sum())
     n_records = int(b.part_records.sum())
     # one 32-B sector read + write-back per K-mer occurrence (the paper's
     # random-access table RMW) + the records read + the vertex records written
-    alg_bytes = n_kmers * 64 + n_records * 4 * b.rec_words + stats["distinct"] * 56
+    alg_bytes = my_kmers * 64 + n_records * 4 * b.rec_words + stats["distinct"] * 56
     peak, peak_kind = _peaks()
     achieved = alg_bytes / (hash_ms * 1e-3) / 1e9
     traffic = None
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            traffic = json.load(f).get(rs.name, {}).get("dram_bytes_per_launch")
+            tr = json.load(f).get(rs.name, {})
+            if ws == 1 and tr.get("kernel_version") == KERNEL_VERSION:
+                traffic = tr.get("dram_bytes_per_launch")
     except Exception:
         pass
     cpu = None
-    if not args.no_cpu_baseline:
+    if not args.no_cpu_baseline and ws == 1:
         threads = os.cpu_count() or 1
         rate, sub, dt = _oracle_rate(rs, args.cpu_seconds, threads)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
     scan = 1 if b.np <= 16384 else 3  # scan.cuh: one CTA, or tile sums + tile scan + apply
-    launches_per_step = 1 + scan + 1 + scan + {"fused": 2, "resident": 2 * len(b.batches),
-                                              "smem": 6 + 2 * len(b.batches)}[args.mode]
+    # msp_kernel + its scan + scatter_kernel, then Step 2: the on-chip plan (7 kernels) + the on-chip
+    # kernel (+ per global-tier batch: its plan scan once, hash_build_list + extract_kernel)
+    nb = len(b.batches)
+    launches_per_step = 2 + scan + {"fused": scan + 2, "resident": scan + 2 * nb,
+                                    "smem": 8 + 2 * nb + (scan if nb else 0)}[args.mode]
     placement = _placement(b) if args.mode == "smem" else None
+    if rank != 0:
+        dist.barrier()
+        dist.destroy_process_group()
+        return 0
+    cfg_extra = {"mode": args.mode, "batches": len(b.batches), "group_slots": args.group_slots, "refine": refine,
+                 "fine_partitions": b.np, "smem_split": args.smem_split, "fine_p": fine_p or rs.p,
+                 "smem_slots": _lib.dbg_smem_table_slots(b.prm), "kmer_placement": placement,
+                 "kernel_version": KERNEL_VERSION}
+    if ws > 1:
+        cfg_extra.update({"reads_per_rank": rs.n_reads, "kmers_total": total_kmers,
+                          "parallelism": f"reads sharded; fine partitions owned by rank (one all_to_all of "
+                                         f"records over NCCL); {ws} GPUs"})
+    if args.min_count > 1:
+        cfg_extra["min_count"] = args.min_count
     line = {
-        "metric": METRIC, "value": n_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+        "metric": METRIC, "value": total_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": _config_json(rs, args, {"mode": args.mode, "batches": len(b.batches),
-                                          "group_slots": args.group_slots, "refine": refine,
-                                          "fine_partitions": b.np, "smem_split": args.smem_split,
-                                          "fine_p": fine_p or rs.p,
-                                          "smem_slots": _lib.dbg_smem_table_slots(b.prm),
-                                          "kmer_placement": placement}),
+        "config": _config_json(rs, args, cfg_extra),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "kernel": {"fused": "subgraph_kernel", "resident": "hash_build_kernel",
                                 "smem": "smem_subgraph_kernel"}[args.mode],
                      "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
-                     "kernel_ms": hash_ms, "kernel_kmers_per_s": n_kmers / (hash_ms * 1e-3)},
+                     "kernel_ms": hash_ms, "kernel_kmers_per_s": my_kmers / (hash_ms * 1e-3),
+                     "rank": 0},
         "cpu_baseline": cpu,
-        "e2e": {"value": n_kmers / (statistics.median(e2e_ms) * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
-                "d2h_bytes_per_step": d2h, "ms": statistics.median(e2e_ms), "h2d_ms": statistics.median(h2d_ms),
-                "all_ms": [round(x, 3) for x in e2e_ms]},
+        "e2e": {"value": total_kmers / (statistics.median(e2e_ms) * 1e-3), "unit": UNIT,
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "ms": statistics.median(e2e_ms),
+                "h2d_ms": statistics.median(h2d_ms), "all_ms": [round(x, 3) for x in e2e_ms]},
         "gpu_launches": args.steps * launches_per_step,
         "clocks": clk.summary(),
         "breakdown_ms": phases,
         "host_ms": {k: round(statistics.mean(v[-args.steps:]), 3) for k, v in host_ms.items() if v},
-        "stats": stats, "invariants_ok": bool(inv_ok), "gen_s": gen_s,
+        "stats": {"distinct": distinct, "sum_count": sum_count, "sum_edges": sum_edges,
+                  "checksum": stats["checksum"] if ws == 1 else None},
+        "invariants_ok": bool(inv_ok), "gen_s": gen_s,
     }
     print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
     return 0
 
 
@@ -374,6 +429,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--out-frac", type=float, default=0.4, help="output capacity / K-mers")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--min-count", type=int, default=0, help="row f4 low-count filter (0: the full graph)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 5
+#define DBG_ABI_VERSION 7
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -116,13 +116,6 @@ typedef struct {
   uint32_t* d_staging;       /* staging_cap records, read order (pass 1 output, pass 2 input) */
   uint64_t staging_cap;      /* capacity of d_staging in records */
   uint32_t* d_records;       /* d_record_offset[NP] records in partition order; NULL => pass 1 */
-  uint32_t* d_rank;          /* [staging_cap] or NULL.  Pass 1 writes each staged record's rank
-                                within its partition (the per-partition count it reserved), and
-                                pass 2 then places record i at d_record_offset[pid] + d_rank[i]
-                                without atomics.  NULL: pass 2 ranks with atomics on d_fill (the
-                                form for records that did not come from pass 1, e.g. received
-                                from other GPUs).  Pass 2 must see the pass-1 ranks of the same
-                                staging. */
 } dbg_partition_set;
 
 /* ---- sizes ------------------------------------------------------------ */
@@ -163,6 +156,22 @@ DBG_API dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64_t*
 DBG_API dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
                              const uint64_t* d_offsets, uint64_t n_reads,
                              const dbg_partition_set* part, cudaStream_t stream);
+
+/* ---- f2: pass 1 over read batches and partition ranges (Sec. III-E)
+ * As dbg_msp_partition pass 1 (part->d_records must be NULL), but only the
+ * superkmers of fine partitions [pid_lo, pid_hi) are counted (d_n_records,
+ * d_n_kmers) and staged; the others are dropped.  append != 0 keeps the
+ * counters and *d_staged of the previous calls (the reads of this call are
+ * another batch of the same input: its records go after the staged ones);
+ * append == 0 zeroes them first.  d_record_offset is recomputed by every call
+ * (it is final after the last batch).  Staging overflow behaves as in
+ * dbg_msp_partition.  Pass 2 is dbg_msp_partition with d_records set.
+ * With staging_cap = 0 the call only counts (a sizing pass over all batches
+ * that chooses the partition ranges of the passes). */
+DBG_API dbg_status dbg_msp_partition_range(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
+                                   const uint64_t* d_offsets, uint64_t n_reads,
+                                   const dbg_partition_set* part, int32_t pid_lo, int32_t pid_hi,
+                                   int append, cudaStream_t stream);
 
 /* ---- a5: sizing (Property 1; Sec. IV-A) ----------------------
  * d_table_offset[NP+1] = exclusive prefix sum of dbg_table_capacity(N^i_kmer)

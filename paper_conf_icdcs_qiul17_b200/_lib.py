@@ -35,7 +35,7 @@ class dbg_partition_set(ctypes.Structure):
     _fields_ = [("d_n_records", ctypes.c_void_p), ("d_n_kmers", ctypes.c_void_p),
                 ("d_record_offset", ctypes.c_void_p), ("d_fill", ctypes.c_void_p),
                 ("d_staged", ctypes.c_void_p), ("d_staging", ctypes.c_void_p),
-                ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p), ("d_rank", ctypes.c_void_p)]
+                ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p)]
 
 
 # dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
@@ -61,6 +61,7 @@ SIGNATURES = {
     "dbg_packed_words": (_U64, [_U64]),
     "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
+    "dbg_msp_partition_range": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _I32, _I32, ctypes.c_int, _P]),
     "dbg_table_plan": (ctypes.c_int, [_PRM, _P, _P, _P, _P]),
     "dbg_smem_table_slots": (_U64, [_PRM]),
     "dbg_smem_onchip": (ctypes.c_int32, [_PRM, _U64]),
@@ -83,7 +84,7 @@ SIGNATURES = {
 }
 
 _lib = None
-ABI_VERSION = 5
+ABI_VERSION = 7
 
 
 def load():
@@ -139,9 +140,9 @@ def fine_partitions(prm: dbg_params) -> int:
 
 
 def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
-                  records=None, rank=None) -> dbg_partition_set:
+                  records=None) -> dbg_partition_set:
     return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(staged),
-                             _ptr(staging), staging_cap, _ptr(records), _ptr(rank))
+                             _ptr(staging), staging_cap, _ptr(records))
 
 
 # --------------------------------------------------------------------------- entry points
@@ -187,6 +188,13 @@ def dbg_msp_partition(prm, d_bases, n_words: int, d_offsets, n_reads: int, part:
     _check("dbg_msp_partition", load().dbg_msp_partition(
         ctypes.byref(prm), _ptr(d_bases), n_words, _ptr(d_offsets), n_reads, ctypes.byref(part),
         _stream(stream)))
+
+
+def dbg_msp_partition_range(prm, d_bases, n_words: int, d_offsets, n_reads: int, part: dbg_partition_set,
+                            pid_lo: int, pid_hi: int, append: bool, stream=None) -> None:
+    _check("dbg_msp_partition_range", load().dbg_msp_partition_range(
+        ctypes.byref(prm), _ptr(d_bases), n_words, _ptr(d_offsets), n_reads, ctypes.byref(part), pid_lo, pid_hi,
+        int(bool(append)), _stream(stream)))
 
 
 def dbg_table_plan(prm, d_n_kmers, d_table_offset, d_scratch=None, stream=None) -> None:

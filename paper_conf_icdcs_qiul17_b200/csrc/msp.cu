@@ -51,7 +51,8 @@ struct MspArgs {
   uint32_t* staging;              // records in read order
   uint64_t staging_cap;           // records
   unsigned long long* staged;     // cursor (records reserved)
-  uint32_t* rank;                 // [staging_cap] rank of each staged record in its partition, or null
+  uint32_t pid_lo, pid_hi;        // only superkmers of fine partitions [pid_lo, pid_hi) are counted and staged
+  bool ranged;                    // pid_lo > 0 or pid_hi < np
 };
 
 template <typename CT>
@@ -97,12 +98,16 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
                                                   int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
   const int nmax = (int)a.max_kmers;
+  auto pid_of = [&](int d) -> uint32_t {
+    const uint64_t m = (uint64_t)sm.desc_m[d * kMspThreads + tid];
+    return a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
+  };
   uint32_t my_records = 0;
   {
     int s = s_next;
     for (int d = 0; d < ndesc; ++d) {
       const int e = (int)sm.desc_e[d * kMspThreads + tid];
-      my_records += (uint32_t)((e - s + nmax) / nmax);
+      if (!a.ranged || (pid_of(d) - a.pid_lo < a.pid_hi - a.pid_lo)) my_records += (uint32_t)((e - s + nmax) / nmax);
       s = e + 1;
     }
   }
@@ -122,20 +127,18 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
   int s = s_next;
   for (int d = 0; d < ndesc; ++d) {
     const int e = (int)sm.desc_e[d * kMspThreads + tid];
-    const uint64_t m = (uint64_t)sm.desc_m[d * kMspThreads + tid];
-    const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
+    const uint32_t pid = pid_of(d);
+    if (a.ranged && pid - a.pid_lo >= a.pid_hi - a.pid_lo) {  // another pass's partition (row f2)
+      s = e + 1;
+      continue;
+    }
     const int n = e - s + 1;
     const uint32_t pieces = (uint32_t)((n + nmax - 1) / nmax);
-    // the per-partition record count doubles as the records' ranks in their partition
-    uint32_t rk = 0;
-    if (a.rank) rk = (uint32_t)atomicAdd(a.n_records + pid, (unsigned long long)pieces);
-    else atomicAdd(a.n_records + pid, (unsigned long long)pieces);
+    atomicAdd(a.n_records + pid, (unsigned long long)pieces);
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
-    for (int ps = s; ps <= e; ps += nmax, ++slot, ++rk) {
-      if (slot < a.staging_cap) {
+    for (int ps = s; ps <= e; ps += nmax, ++slot) {
+      if (slot < a.staging_cap)
         write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
-        if (a.rank) a.rank[slot] = rk;
-      }
     }
     s = e + 1;
   }
@@ -225,28 +228,6 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   }
 }
 
-// Pass 3 with the ranks of pass 1: record i goes to rec_off[pid] + rank[i]
-// (no atomics; a coalesced read, one random 16/32-byte write per record).
-template <int R>
-__global__ void __launch_bounds__(256) scatter_ranked_kernel(const uint32_t* __restrict__ staging,
-                                                            const uint32_t* __restrict__ rank,
-                                                            const unsigned long long* staged, uint64_t staging_cap,
-                                                            const uint64_t* __restrict__ rec_off,
-                                                            uint32_t* __restrict__ records) {
-  const uint64_t n = *staged;
-  if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint4* src = reinterpret_cast<const uint4*>(staging + i * R);
-    uint4 rec[R / 4];
-#pragma unroll
-    for (int c = 0; c < R / 4; ++c) rec[c] = __ldcs(src + c);
-    const uint64_t pos = __ldg(rec_off + (rec[0].x >> 10)) + __ldcs(rank + i);
-    uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
-#pragma unroll
-    for (int c = 0; c < R / 4; ++c) dst[c] = rec[c];
-  }
-}
-
 // Pass 3: scatter staged records into partition order.
 constexpr int kScatterThreads = 256;
 constexpr int kScatterPer = 8;  // records per thread per tile
@@ -330,16 +311,36 @@ static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
   return cudaGetLastError();
 }
 
+static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
+                                const uint64_t* d_offsets, uint64_t n_reads, const dbg_partition_set* part,
+                                int32_t pid_lo, int32_t pid_hi, int append, cudaStream_t stream);
+
 extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d_bases,
                                         uint64_t n_words, const uint64_t* d_offsets,
                                         uint64_t n_reads, const dbg_partition_set* part,
                                         cudaStream_t stream) {
+  if (!dbg_params_ok(prm)) return DBG_EINVAL;
+  return msp_partition(prm, d_bases, n_words, d_offsets, n_reads, part, 0, fine_partitions(prm), 0, stream);
+}
+
+extern "C" dbg_status dbg_msp_partition_range(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
+                                              const uint64_t* d_offsets, uint64_t n_reads,
+                                              const dbg_partition_set* part, int32_t pid_lo, int32_t pid_hi,
+                                              int append, cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !part || part->d_records) return DBG_EINVAL;
+  return msp_partition(prm, d_bases, n_words, d_offsets, n_reads, part, pid_lo, pid_hi, append, stream);
+}
+
+static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
+                                const uint64_t* d_offsets, uint64_t n_reads, const dbg_partition_set* part,
+                                int32_t pid_lo, int32_t pid_hi, int append, cudaStream_t stream) {
   if (!dbg_params_ok(prm) || !part || !d_offsets || !part->d_record_offset || !part->d_n_records ||
       !part->d_n_kmers || !part->d_staged)
     return DBG_EINVAL;
   if (n_reads && (!d_bases || !n_words)) return DBG_EINVAL;
   const int np = fine_partitions(prm);
   const uint32_t R = record_words(prm->k);
+  if (pid_lo < 0 || pid_hi > np || pid_lo >= pid_hi) return DBG_EINVAL;
   if (part->d_records == nullptr) {
     // passes 1 + 2: minimizers, superkmers, staging, sizes, offsets
     if (part->staging_cap && !part->d_staging) return DBG_EINVAL;
@@ -360,10 +361,12 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
     a.staging = part->d_staging;
     a.staging_cap = part->staging_cap;
     a.staged = reinterpret_cast<unsigned long long*>(part->d_staged);
-    a.rank = part->d_rank;
-    if (cudaMemsetAsync(part->d_n_records, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
-        cudaMemsetAsync(part->d_n_kmers, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
-        cudaMemsetAsync(part->d_staged, 0, sizeof(uint64_t), stream) != cudaSuccess)
+    a.pid_lo = (uint32_t)pid_lo;
+    a.pid_hi = (uint32_t)pid_hi;
+    a.ranged = pid_lo > 0 || pid_hi < np;
+    if (!append && (cudaMemsetAsync(part->d_n_records, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
+                    cudaMemsetAsync(part->d_n_kmers, 0, sizeof(uint64_t) * np, stream) != cudaSuccess ||
+                    cudaMemsetAsync(part->d_staged, 0, sizeof(uint64_t), stream) != cudaSuccess))
       return DBG_ECUDA;
     if (n_reads) {
       const uint64_t want = (n_reads + kMspThreads - 1) / kMspThreads;
@@ -379,20 +382,7 @@ extern "C" dbg_status dbg_msp_partition(const dbg_params* prm, const uint64_t* d
       return DBG_ECUDA;
   } else {
     // pass 3: scatter (a no-op after a staging overflow, *d_staged > staging_cap)
-    if (!part->d_staging) return DBG_EINVAL;
-    if (part->d_rank) {  // ranks from pass 1: no atomics
-      const int grid = dbg_sm_count() * 8;
-      if (R == 4)
-        scatter_ranked_kernel<4><<<grid, 256, 0, stream>>>(
-            part->d_staging, part->d_rank, reinterpret_cast<const unsigned long long*>(part->d_staged),
-            part->staging_cap, part->d_record_offset, part->d_records);
-      else
-        scatter_ranked_kernel<8><<<grid, 256, 0, stream>>>(
-            part->d_staging, part->d_rank, reinterpret_cast<const unsigned long long*>(part->d_staged),
-            part->staging_cap, part->d_record_offset, part->d_records);
-      return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
-    }
-    if (!part->d_fill) return DBG_EINVAL;
+    if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
     if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * np, stream) != cudaSuccess) return DBG_ECUDA;
     const size_t smem = np <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * np : 0;
     const int grid = dbg_sm_count() * 4;

@@ -109,8 +109,6 @@ class DbgBuilder:
         self.d_n_out = torch.zeros(1, **i64)
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
-        self.rank = torch.empty(0, dtype=torch.int32, device=dev)
-        self.ranked = True  # records staged by pass 1 (False: received from other ranks)
         self.records = torch.empty(0, dtype=torch.int32, device=dev)
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
         self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
@@ -161,14 +159,9 @@ class DbgBuilder:
 
     # ------------------------------------------------------------------ a2-a4
     def part_set(self, with_records: bool) -> _lib.dbg_partition_set:
-        cap = self.staging.numel() // self.rec_words
-        rank = None
-        if self.ranked:  # pass-1 ranks: pass 2 scatters without atomics (dbg.h d_rank)
-            if self.rank.numel() < cap:
-                self.rank = torch.empty(cap, dtype=torch.int32, device=self.device)
-            rank = self.rank
         return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill, self.d_staged,
-                                  self.staging, cap, self.records if with_records else None, rank)
+                                  self.staging, self.staging.numel() // self.rec_words,
+                                  self.records if with_records else None)
 
     def _staging_estimate(self, n_kmers_upper: int, n_reads: int) -> int:
         w = self.k - self.p + 1
@@ -185,7 +178,6 @@ class DbgBuilder:
             self.staging = _grow(self.staging, self._staging_estimate(n_words * 32, n_reads) * self.rec_words,
                                  torch.int32, self.device)
         self.overflowed = False
-        self.ranked = True
         ev = self._mark("msp_pass1", stream)
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(False), stream)
         self._done(ev, stream)
@@ -242,7 +234,6 @@ class DbgBuilder:
             self.d_rec_off.copy_(torch.from_numpy(off), non_blocking=True)
             self.d_staged.fill_(n_received)
         self.staging = received
-        self.ranked = False  # received records carry no pass-1 ranks: pass 2 ranks with atomics
         self.records = _grow(self.records, n_received * self.rec_words, torch.int32, self.device, 1.05)
         _lib.dbg_msp_partition(self.prm, 1, 1, self.d_rec_off, 0, self.part_set(True), stream)
 

@@ -17,11 +17,6 @@ gloo on CPU tensors (tests/test_multi.py).
 """
 from __future__ import annotations
 
-import json
-import os
-import statistics
-import time
-
 import numpy as np
 import torch
 import torch.distributed as dist
@@ -82,70 +77,3 @@ def distributed_step(builder, d_bases, d_offsets, stream, out_cap: int, group=No
     builder.plan(stream)
     builder.reset_output(out_cap, stream)
     builder.step2(stream)                                         # Step 2 on owned partitions
-
-
-def bench_main(args, metric: str, unit: str) -> int:
-    """`bench.py` under torchrun (WORLD_SIZE > 1): weak scaling -- every rank owns a read set of the
-    configuration's size (same genome, its own reads), so the job builds the graph of world x reads."""
-    from synth import make_config
-    from . import DbgBuilder, auto_fine_p, auto_refine, encode_reads, _lib
-
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
-    dist.init_process_group("nccl", device_id=dev)
-    world, rank = dist.get_world_size(), dist.get_rank()
-    rs = make_config(args.config, scale=args.scale, num_partitions=args.np, read_seed_offset=7919 * rank)
-    packed = encode_reads(rs.seq, pin=True)
-    offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
-    n_kmers = rs.n_kmers()
-    refine = args.refine if args.refine is not None else auto_refine(n_kmers, rs.k, rs.p, rs.num_partitions,
-                                                                      args.lam, args.alpha)
-    fine_p = args.fine_p if args.fine_p is not None else auto_fine_p(n_kmers, rs.k, rs.p, args.lam, args.alpha)
-    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, "smem",
-                   args.group_slots, refine, args.smem_split, fine_p)
-    stream = torch.cuda.current_stream(dev)
-    d_bases, d_off = b.upload(packed, offsets, stream)
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-    out_cap = n_kmers // 2 + 1024
-    for _ in range(args.warmup):
-        distributed_step(b, d_bases, d_off, stream, out_cap)
-    torch.cuda.synchronize()
-    times = []
-    for _ in range(args.steps):
-        flush.zero_()
-        torch.cuda.synchronize()
-        dist.barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        distributed_step(b, d_bases, d_off, stream, out_cap)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        dist.barrier()
-        times.append(e0.elapsed_time(e1))
-    ms = torch.tensor([statistics.mean(times)], device=dev)
-    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
-    tot = torch.tensor([n_kmers], dtype=torch.int64, device=dev)
-    dist.all_reduce(tot)
-    st = b.d_stats[:3].clone()
-    dist.all_reduce(st)
-    status = _lib.dbg_sync_status(b.d_status, stream)
-    ok = torch.tensor([int(status == 0)], device=dev)
-    dist.all_reduce(ok, op=dist.ReduceOp.MIN)
-    if rank == 0:
-        total = int(tot.item())
-        line = {
-            "metric": metric, "value": total / (float(ms.item()) * 1e-3), "unit": unit, "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(ms.item()), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-            "config": {"workload": rs.name, "reads_per_rank": rs.n_reads, "k": rs.k, "p": rs.p,
-                       "num_partitions": rs.num_partitions, "refine": refine, "kmers_total": total,
-                       "parallelism": f"reads sharded, fine partitions owned by rank, 1 exchange ({world} GPUs)",
-                       "l2": "flushed between timed steps (512 MiB write)"},
-            "stats": {"distinct": int(st[0].item()), "sum_count": int(st[1].item()), "sum_edges": int(st[2].item())},
-            "status_ok": bool(ok.item()), "gpu_launches": args.steps * 7,
-        }
-        print(json.dumps(line), flush=True)
-    dist.barrier()
-    dist.destroy_process_group()
-    return 0

@@ -77,3 +77,20 @@ def test_exchange_records_gloo_world2(n_fine, R):
     for p in procs:
         p.join(timeout=60)
     assert all(ok for _, ok, _, _ in res), res
+
+
+def test_stream_plan_ranges():
+    """Row f2 host logic: consecutive ranges covering every fine partition, each within the staging
+    budget unless a single partition exceeds it."""
+    sys.path.insert(0, ROOT)
+    from paper_conf_icdcs_qiul17_b200.stream import plan_ranges
+
+    rng = np.random.default_rng(5)
+    for budget in (1, 7, 50, 10 ** 9):
+        rec = rng.integers(0, 20, 300)
+        rr = plan_ranges(rec, budget)
+        assert rr[0][0] == 0 and rr[-1][1] == len(rec)
+        assert all(a[1] == b[0] for a, b in zip(rr, rr[1:]))
+        for lo, hi in rr:
+            assert hi > lo
+            assert rec[lo:hi].sum() <= budget or (rec[lo:hi] > 0).sum() == 1
