@@ -38,6 +38,11 @@ VERTEX_DTYPE = np.dtype(
 )
 assert VERTEX_DTYPE.itemsize == 56
 
+# Row f3 (K <= 127): four key words, most significant first
+VERTEX_WIDE_DTYPE = np.dtype([("key", "<u8", (4,)), ("count", "<u4"), ("out", "<u4", (4,)), ("in", "<u4", (4,)),
+                              ("pid", "<u4")])
+assert VERTEX_WIDE_DTYPE.itemsize == 72
+
 SUPERKMER_DTYPE = np.dtype(
     [
         ("read", "<u8"),
@@ -96,6 +101,9 @@ def _load():
         lib.oracle_canonical.restype = None
         lib.oracle_kmer_minimizer.argtypes = [ctypes.c_char_p, ctypes.c_int, ctypes.c_int]
         lib.oracle_kmer_minimizer.restype = ctypes.c_uint64
+        lib.oracle_graph_wide.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int,
+                                          ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_void_p), u64p]
+        lib.oracle_graph_wide.restype = ctypes.c_int
         lib.oracle_free.argtypes = [ctypes.c_void_p]
         lib.oracle_free.restype = None
         _lib = lib
@@ -195,3 +203,22 @@ def filter_low_count(records, min_count: int):
     if min_count <= 1:
         return rec.copy()
     return rec[rec["count"] >= min_count].copy()
+
+
+def graph_wide(seq, offsets, k: int, p: int, num_partitions: int):
+    """Row f3: sorted vertex records (VERTEX_WIDE_DTYPE) for K up to 127 -- the definition with the
+    canonical K-mer held as a string (oracle_graph_wide), single-threaded."""
+    lib = _load()
+    seq, offsets = _as_inputs(seq, offsets)
+    out = ctypes.c_void_p()
+    n = ctypes.c_uint64()
+    rc = lib.oracle_graph_wide(seq.ctypes.data if seq.size else None, offsets.ctypes.data, len(offsets) - 1, k, p,
+                               num_partitions, ctypes.byref(out), ctypes.byref(n))
+    if rc != 0:
+        raise RuntimeError(f"oracle_graph_wide failed with code {rc}")
+    try:
+        buf = (ctypes.c_char * (n.value * VERTEX_WIDE_DTYPE.itemsize)).from_address(out.value)
+        arr = np.frombuffer(buf, dtype=VERTEX_WIDE_DTYPE).copy()
+    finally:
+        lib.oracle_free(out)
+    return arr

@@ -361,6 +361,73 @@ uint64_t oracle_checksum(const oracle_vertex* v, uint64_t n) {
   return sum;
 }
 
+// Row f3 (K up to 127, keys of up to four 64-bit words): the same definition,
+// with the vertex held as its canonical string (std::map<std::string, Rec> per
+// partition; string order = lexicographic order = numeric order of the codes,
+// reading A).  The code of a vertex is sum_i code(v_i) 4^(K-1-i) as a 256-bit
+// integer, written as four 64-bit words, most significant first.
+typedef struct {
+  uint64_t key[4];
+  uint32_t count;
+  uint32_t out[4];
+  uint32_t in[4];
+  uint32_t pid;
+} oracle_vertex_wide;
+
+int oracle_graph_wide(const char* seq, const uint64_t* offs, uint64_t n_reads, int K, int P, int NP,
+                      oracle_vertex_wide** out, uint64_t* n_out) {
+  *out = nullptr;
+  *n_out = 0;
+  if (K < 1 || K > 127 || P < 1 || P > K || P > 31 || NP < 1) return 1;
+  std::vector<std::map<std::string, Rec>> maps(NP);
+  for (uint64_t r = 0; r < n_reads; ++r) {
+    std::string S = read_string(seq, offs, r);
+    if (S.size() < (size_t)K) continue;  // reading N
+    for (size_t i = 0; i + K <= S.size(); ++i) {
+      const uint32_t pid = partition_of(canonical_minimizer(S, i, K, P), NP);
+      const std::string x = S.substr(i, K), y = reverse_complement(x);
+      const bool fwd = x <= y;
+      Rec& rec = maps[pid][fwd ? x : y];
+      rec.count += 1;
+      const bool has_pred = i > 0, has_succ = i + K < S.size();
+      if (fwd) {
+        if (has_succ) rec.out[code_of(S[i + K])] += 1;
+        if (has_pred) rec.in[code_of(S[i - 1])] += 1;
+      } else {
+        if (has_succ) rec.in[3 - code_of(S[i + K])] += 1;
+        if (has_pred) rec.out[3 - code_of(S[i - 1])] += 1;
+      }
+    }
+  }
+  std::map<std::string, std::pair<Rec, uint32_t>> all;  // sorted by the canonical string
+  for (int p = 0; p < NP; ++p)
+    for (auto& kv : maps[p]) {
+      if (all.count(kv.first)) return 2;  // a vertex in two partitions
+      all[kv.first] = std::make_pair(kv.second, (uint32_t)p);
+    }
+  oracle_vertex_wide* v = (oracle_vertex_wide*)malloc(sizeof(oracle_vertex_wide) * (all.size() ? all.size() : 1));
+  if (!v) return 3;
+  uint64_t w = 0;
+  for (auto& kv : all) {
+    oracle_vertex_wide& o = v[w++];
+    memset(o.key, 0, sizeof(o.key));
+    const std::string& t = kv.first;
+    for (int i = 0; i < K; ++i) {  // base i is bit pair 2(K-1-i) of the 256-bit code
+      const int bit = 2 * (K - 1 - i);
+      o.key[3 - bit / 64] |= (uint64_t)code_of(t[i]) << (bit % 64);
+    }
+    o.count = kv.second.first.count;
+    for (int c = 0; c < 4; ++c) {
+      o.out[c] = kv.second.first.out[c];
+      o.in[c] = kv.second.first.in[c];
+    }
+    o.pid = kv.second.second;
+  }
+  *out = v;
+  *n_out = all.size();
+  return 0;
+}
+
 void oracle_free(void* p) { free(p); }
 
 }  // extern "C"

@@ -335,3 +335,57 @@ def test_filter_low_count_keeps_genome_kmers(oracle_lib):
     assert all(full[v] == e for v, e in got.items())  # kept records are not edited
     assert len(oracle_lib.filter_low_count(recs, 1)) == len(recs)
     assert len(oracle_lib.filter_low_count(recs, 0)) == len(recs)
+
+
+# ---------------------------------------------------------------- row f3: K up to 127
+
+
+def _wide_as_dict(recs, k):
+    d = {}
+    for r in recs:
+        code = 0
+        for w in r["key"]:
+            code = (code << 64) | int(w)
+        s = "".join("ACGT"[(code >> (2 * (k - 1 - t))) & 3] for t in range(k))
+        d[s] = [int(r["count"]), [int(x) for x in r["out"]], [int(x) for x in r["in"]], int(r["pid"])]
+    return d
+
+
+@pytest.mark.parametrize("k,p,np_,seed", [(65, 21, 7, 1), (71, 13, 3, 2), (99, 31, 16, 3), (127, 19, 5, 4),
+                                           (101, 1, 2, 5)])
+def test_wide_oracle_vs_string_brute_force(oracle_lib, k, p, np_, seed):
+    """Row f3 (Sec. III-C3 L569-615 needs K > 63 keys): the string-keyed oracle equals the pure-Python
+    string brute force (oracle/brute.py) on ragged reads with N bases and repeats, codes included."""
+    rng = np.random.default_rng(seed)
+    base = "".join("ACGT"[x] for x in rng.integers(0, 4, 400))
+    reads = []
+    for _ in range(40):
+        L = int(rng.integers(k - 3, k + 90))
+        s0 = int(rng.integers(0, 400 - min(L, 399)))
+        r = base[s0:s0 + L]
+        if rng.random() < 0.5:
+            r = brute.rc(r)
+        r = "".join(c if rng.random() > 0.01 else "N" for c in r)
+        reads.append(r)
+    reads.append(base[:k])  # L = K: one K-mer, no edges (reading N)
+    rs = _readset(reads)
+    got = _wide_as_dict(oracle_lib.graph_wide(rs.seq, rs.offsets, k, p, np_), k)
+    want = brute.graph(reads, k, p, np_)
+    assert got == want
+    recs = oracle_lib.graph_wide(rs.seq, rs.offsets, k, p, np_)
+    keys = [tuple(int(x) for x in r["key"]) for r in recs]
+    assert keys == sorted(keys)  # reading Q: ascending canonical code
+
+
+def test_wide_oracle_equals_two_word_oracle(oracle_lib):
+    """For K <= 63 the string-keyed oracle and the 128-bit-keyed oracle are the same graph."""
+    rs = random_reads(300, 1, 200, seed=12, n_rate=0.01)
+    for k, p, np_ in [(31, 11, 16), (63, 19, 8), (5, 3, 3)]:
+        a = oracle_lib.graph(rs.seq, rs.offsets, k, p, np_)
+        b = oracle_lib.graph_wide(rs.seq, rs.offsets, k, p, np_)
+        assert len(a) == len(b)
+        assert np.array_equal(b["key"][:, 0], np.zeros(len(b), dtype=np.uint64))
+        assert np.array_equal(b["key"][:, 1], np.zeros(len(b), dtype=np.uint64))
+        assert np.array_equal(b["key"][:, 2], a["key_hi"]) and np.array_equal(b["key"][:, 3], a["key_lo"])
+        for f in ("count", "out", "in", "pid"):
+            assert np.array_equal(a[f], b[f])
