@@ -15,7 +15,12 @@
  *    output overflow) are recorded in a caller-owned uint32 status word and
  *    reported by dbg_sync_status, the only call that synchronizes.
  *  - Thread-safe across distinct buffers; one host thread per device.
- *  - K must be odd (reading C), 1 <= K <= 63; 1 <= P <= min(K, 31);
+ *  - K must be odd (reading C), 1 <= K <= 127; 1 <= P <= min(K, 31).  K > 63
+ *    (row f3: four-word keys, the paper's empty/locked/occupied protocol) runs
+ *    only through the resident tables: dbg_msp_partition[_range],
+ *    dbg_table_plan, dbg_hash_build, dbg_extract_graph (dbg_vertex_wide
+ *    output); fine_p must be 0 or P; the on-chip, fused, sort and checksum
+ *    calls return DBG_EINVAL;
  *    1 <= num_partitions * refine <= 4,194,303.  Every per-partition array
  *    and pid range below is in FINE partitions (NP * refine of them); only
  *    dbg_vertex.pid reports the paper's partition (fine pid mod NP).  Reads shorter than K contribute
@@ -31,7 +36,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 7
+#define DBG_ABI_VERSION 8
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -49,7 +54,7 @@ typedef enum {
 
 /* Parameters of Sec. IV-A and Sec. V-A. */
 typedef struct {
-  int32_t k;              /* K-mer length, odd, 1..63 (reading C, T) */
+  int32_t k;              /* K-mer length, odd, 1..127 (readings C, T; > 63: row f3) */
   int32_t p;              /* minimizer length P, 1..min(k,31) (Def. 1) */
   int32_t num_partitions; /* NP, number of superkmer partitions (Sec. III-B) */
   float lambda;           /* average errors per read (Property 1); default 2 */
@@ -89,6 +94,19 @@ typedef struct {
   uint32_t pid;
 } dbg_vertex;
 
+/* Row f3 (K > 63, up to 127; Sec. III-C3): the same vertex with a
+ * 2K-bit code of up to 254 bits in four 64-bit words, kmer[0] most
+ * significant (the code is sum_i code(v_i) 4^(K-1-i)).  72 bytes.  Written by
+ * dbg_extract_graph when K > 63 (d_out then points to dbg_vertex_wide
+ * records and out_cap counts them). */
+typedef struct {
+  uint64_t kmer[4];
+  uint32_t count;
+  uint32_t out[4];
+  uint32_t in[4];
+  uint32_t pid;
+} dbg_vertex_wide;
+
 /* Totals (filled by the extraction calls); checksum = sum over vertices of
  * h, h = fmix64 chained over (kmer_hi, kmer_lo, count, out[0..3], in[0..3])
  * (SURVEY.md 8(d)), filled by dbg_checksum_vertices. */
@@ -120,12 +138,13 @@ typedef struct {
 
 /* ---- sizes ------------------------------------------------------------ */
 DBG_API int dbg_abi_version(void);
-/* uint32 words per superkmer record for these params (4 for K <= 39, else 8). */
+/* uint32 words per superkmer record for these params (4 for K <= 39, 8 for
+ * K <= 63, 16 for K <= 127). */
 DBG_API uint32_t dbg_record_words(const dbg_params* prm);
 /* K-mers a record holds at most. */
 DBG_API uint32_t dbg_record_max_kmers(const dbg_params* prm);
 /* Bytes per hash-table slot: a key entry (dbg_key_bytes: 16 for K <= 31, 32
- * otherwise) plus a 32-byte counter record. */
+ * for K <= 63, 48 for K <= 127) plus a 32-byte counter record. */
 DBG_API uint32_t dbg_slot_bytes(const dbg_params* prm);
 DBG_API uint32_t dbg_key_bytes(const dbg_params* prm);
 /* Table capacity for a partition with n_kmers K-mers: ceil(lambda/(4 alpha) * n_kmers)

@@ -41,6 +41,10 @@ class dbg_partition_set(ctypes.Structure):
 # dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
 VERTEX_DTYPE = np.dtype([("kmer_hi", "<u8"), ("kmer_lo", "<u8"), ("count", "<u4"),
                          ("out", "<u4", (4,)), ("in", "<u4", (4,)), ("pid", "<u4")])
+# row f3 (K > 63): dbg_vertex_wide, four key words most significant first (72 B)
+VERTEX_WIDE_DTYPE = np.dtype([("kmer", "<u8", (4,)), ("count", "<u4"), ("out", "<u4", (4,)), ("in", "<u4", (4,)),
+                              ("pid", "<u4")])
+assert VERTEX_WIDE_DTYPE.itemsize == 72
 STATS_FIELDS = ("distinct", "sum_count", "sum_edges", "checksum")
 assert VERTEX_DTYPE.itemsize == 56
 
@@ -84,7 +88,7 @@ SIGNATURES = {
 }
 
 _lib = None
-ABI_VERSION = 7
+ABI_VERSION = 8
 
 
 def load():

@@ -16,7 +16,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIBDIR = os.path.join(PKG, "lib")
 LIB = os.path.join(LIBDIR, "libdbg.so")
-SOURCES = ["api.cu", "msp.cu", "hash.cu"]
+SOURCES = ["api.cu", "msp.cu", "hash.cu", "wide.cu"]
 HEADERS = ["dbg_device.cuh", os.path.join("..", "..", "include", "dbg.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -17,8 +17,9 @@ constexpr uint64_t kOccupied = 1ull << 63;
 constexpr uint32_t kStatusTableFull = 1u;
 constexpr uint32_t kStatusNoSpace = 2u;
 
-// Record geometry (dbg.h): 4 words (48 bases) for K <= 39, else 8 (112 bases).
-__host__ __device__ inline uint32_t record_words(int k) { return k <= 39 ? 4u : 8u; }
+// Record geometry (dbg.h): 4 words (48 bases) for K <= 39, 8 (112 bases) for
+// K <= 63, 16 (240 bases) for K <= 127 (row f3).
+__host__ __device__ inline uint32_t record_words(int k) { return k <= 39 ? 4u : (k <= 63 ? 8u : 16u); }
 __host__ __device__ inline uint32_t record_max_kmers(int k) {
   // bases = 16 * (R - 1) >= has_left + n + K - 1 + has_right
   return 16u * (record_words(k) - 1u) - (uint32_t)k - 1u;

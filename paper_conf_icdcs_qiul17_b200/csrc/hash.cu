@@ -49,6 +49,13 @@
 
 int dbg_sm_count();
 bool dbg_params_ok(const dbg_params* prm);
+// row f3 (wide.cu): K > 63 in the resident tables, with the locked-state protocol
+dbg_status dbg_wide_hash_build(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
+                               int32_t pid_end, void* d_table, const uint64_t* d_table_offset, uint32_t* d_status,
+                               cudaStream_t stream);
+dbg_status dbg_wide_extract(const dbg_params* prm, void* d_table, const uint64_t* d_table_offset, int32_t pid_begin,
+                            int32_t pid_end, void* d_out, uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
+                            uint32_t* d_status, cudaStream_t stream);
 
 namespace dbg {
 
@@ -63,7 +70,7 @@ constexpr uint32_t kExtractSlots = kThreads * kXPer;
 constexpr uint32_t kStatusRing = 4u;
 constexpr int kJobs = 4;  // occurrences in flight per lane
 
-__host__ __device__ inline uint32_t key_bytes(int k) { return k <= 31 ? 16u : 32u; }
+__host__ __device__ inline uint32_t key_bytes(int k) { return k <= 31 ? 16u : (k <= 63 ? 32u : 48u); }
 constexpr uint32_t kCtrBytes = 32;
 
 __device__ __forceinline__ uint64_t slot_hash(uint64_t code) { return fmix64(code ^ kSlotSeed); }
@@ -1461,6 +1468,7 @@ extern "C" dbg_status dbg_hash_build(const dbg_params* prm, const dbg_partition_
     return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
+  if (prm->k > 63) return dbg_wide_hash_build(prm, part, pid_begin, pid_end, d_table, d_table_offset, d_status, stream);
   ResidentArgs a;
   a.records = part->d_records;
   a.rec_off = part->d_record_offset;
@@ -1485,6 +1493,7 @@ extern "C" dbg_status dbg_hash_build_list(const dbg_params* prm, const dbg_parti
       !d_table_offset || !d_status || n_pids < 0 || (n_pids && (!d_pids || !d_chunk_prefix)))
     return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
+  if (prm->k > 63) return DBG_EINVAL;  // K > 63: dbg_hash_build (resident tables only)
   if (n_pids == 0) return DBG_OK;
   ResidentArgs a;
   a.records = part->d_records;
@@ -1511,6 +1520,9 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
     return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
+  if (prm->k > 63)  // d_out holds dbg_vertex_wide records (dbg.h)
+    return dbg_wide_extract(prm, d_table, d_table_offset, pid_begin, pid_end, d_out, out_cap, d_n_out, d_stats,
+                            d_status, stream);
   ResidentArgs a;
   a.records = nullptr;
   a.rec_off = nullptr;
@@ -1560,7 +1572,7 @@ static uint64_t smem_slots(int k, int ctas) {
 }
 
 extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
-  if (!prm) return 0;
+  if (!prm || prm->k > 63) return 0;
   return smem_slots(prm->k, smem_ctas());
 }
 
@@ -1587,6 +1599,7 @@ static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_
 
 extern "C" int32_t dbg_smem_onchip(const dbg_params* prm, uint64_t n_kmers) {
   if (!dbg_params_ok(prm) || !(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return -1;
+  if (prm->k > 63) return 0;  // row f3: resident (global) tables only
   const double ratio = (double)prm->lambda / (4.0 * (double)prm->alpha);
   return (int32_t)onchip_tables(n_kmers, table_capacity(ratio, n_kmers), dbg_smem_table_slots(prm),
                                 smem_max_split(prm));
@@ -1637,6 +1650,7 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !part->d_n_kmers || !d_work ||
       !d_n_out || !d_stats || !d_status || (out_cap && !d_out))
     return DBG_EINVAL;
+  if (prm->k > 63) return DBG_EINVAL;  // row f3: resident tables only
   if (!(prm->lambda > 0.f) || !(prm->alpha > 0.f)) return DBG_EINVAL;
   if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
@@ -1674,7 +1688,7 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
 
 extern "C" dbg_status dbg_checksum_vertices(const dbg_params* prm, const dbg_vertex* d_vertices, uint64_t n,
                                             dbg_stats* d_stats, cudaStream_t stream) {
-  if (!dbg_params_ok(prm) || !d_stats || (n && !d_vertices)) return DBG_EINVAL;
+  if (!dbg_params_ok(prm) || prm->k > 63 || !d_stats || (n && !d_vertices)) return DBG_EINVAL;
   if (n == 0) return DBG_OK;
   const uint64_t want = (n + 255) / 256, cap = (uint64_t)dbg_sm_count() * 8;
   checksum_kernel<<<(int)(want < cap ? want : cap), 256, 0, stream>>>(
@@ -1709,6 +1723,7 @@ extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_parti
   if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table_offset ||
       !d_ring || !d_workspace || !d_n_out || !d_stats || !d_status || (out_cap && !d_out) || group_slots == 0)
     return DBG_EINVAL;
+  if (prm->k > 63) return DBG_EINVAL;  // row f3: resident tables only
   if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
   if (pid_begin == pid_end) return DBG_OK;
   if (workspace_bytes < dbg_subgraph_workspace_bytes(prm, pid_end - pid_begin, total_slots, group_slots))
@@ -1758,7 +1773,8 @@ extern "C" uint64_t dbg_sort_workspace_bytes(const dbg_params* prm, uint64_t n) 
 
 extern "C" dbg_status dbg_sort_vertices(const dbg_params* prm, const dbg_vertex* d_in, dbg_vertex* d_out, uint64_t n,
                                         void* d_workspace, uint64_t workspace_bytes, cudaStream_t stream) {
-  if (!dbg_params_ok(prm) || (n && (!d_in || !d_out || !d_workspace)) || d_in == d_out) return DBG_EINVAL;
+  if (!dbg_params_ok(prm) || prm->k > 63 || (n && (!d_in || !d_out || !d_workspace)) || d_in == d_out)
+    return DBG_EINVAL;
   if (n == 0) return DBG_OK;
   if (workspace_bytes < dbg_sort_workspace_bytes(prm, n)) return DBG_EINVAL;
   char* ws = static_cast<char*>(d_workspace);

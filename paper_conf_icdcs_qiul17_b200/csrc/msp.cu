@@ -73,22 +73,37 @@ __device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, ui
   const uint32_t hr = pe + a.k < L ? 1u : 0u;
   const int bs = ps - (int)hl;
   const int nb = (int)hl + (pe - ps + 1) + a.k - 1 + (int)hr;
-  uint32_t w[8];
-  w[0] = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
-#pragma unroll
-  for (int q = 0; q < 7; q += 2) {  // two 16-base words per 64-bit window
-    uint64_t v = 0;
-    const int left = nb - 16 * q;
-    if (q + 1 < (int)a.rec_words && left > 0) {
-      v = window64(a.words, a.n_words, o + bs + 16 * q);
-      if (left < 32) v &= ~(~0ull >> (2 * left));  // zero the bases past the record
-    }
-    w[q + 1] = (uint32_t)(v >> 32);
-    if (q + 2 < 8) w[q + 2] = (uint32_t)v;
-  }
   uint4* d4 = reinterpret_cast<uint4*>(dst);
-  d4[0] = make_uint4(w[0], w[1], w[2], w[3]);
-  if (a.rec_words == 8) d4[1] = make_uint4(w[4], w[5], w[6], w[7]);
+  // 16-byte chunks of the record: word 0 = header, then 16 bases per word, two words per
+  // 64-bit window of the stream (rec_words = 4, 8 or 16)
+  for (int c = 0; c < (int)a.rec_words / 4; ++c) {
+    uint32_t w[4];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int q = 4 * c + 2 * h;  // record word q and q+1 hold data words q-1 and q ...
+      // ... i.e. bases 16(q-1) .. 16(q+1)-1; word 0 is the header
+      uint64_t v = 0;
+      const int first = 16 * (q - 1);
+      if (q == 0) {
+        const int left = nb;
+        if (left > 0) {
+          v = window64(a.words, a.n_words, o + bs);
+          if (left < 32) v &= ~(~0ull >> (2 * left));
+        }
+        w[0] = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
+        w[1] = (uint32_t)(v >> 32);  // bases 0..15
+        continue;
+      }
+      const int left = nb - first;
+      if (left > 0) {
+        v = window64(a.words, a.n_words, o + bs + first);
+        if (left < 32) v &= ~(~0ull >> (2 * left));  // zero the bases past the record
+      }
+      w[2 * h] = (uint32_t)(v >> 32);
+      w[2 * h + 1] = (uint32_t)v;
+    }
+    d4[c] = make_uint4(w[0], w[1], w[2], w[3]);
+  }
 }
 
 // Warp-collective flush of the per-thread descriptor lists: partition ids,
@@ -243,16 +258,17 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
   const uint64_t n = *staged;
   if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
   const bool smem = np <= kSmemHistMaxNp;
-  constexpr int kTile = kScatterThreads * kScatterPer;
+  constexpr int kPer = R >= 16 ? 2 : kScatterPer;
+  constexpr int kTile = kScatterThreads * kPer;
   for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile) {
     if (smem) {
       for (int i = threadIdx.x; i < np; i += kScatterThreads) sh_cnt[i] = 0;
       __syncthreads();
     }
-    uint4 rec[kScatterPer][R / 4];
-    uint32_t rank[kScatterPer];
+    uint4 rec[kPer][R / 4];
+    uint32_t rank[kPer];
 #pragma unroll
-    for (int v = 0; v < kScatterPer; ++v) {
+    for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       rank[v] = 0;
       if (idx < n) {
@@ -271,7 +287,7 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
       __syncthreads();
     }
 #pragma unroll
-    for (int v = 0; v < kScatterPer; ++v) {
+    for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       if (idx < n) {
         const uint32_t pid = rec[v][0].x >> 10;
@@ -296,7 +312,9 @@ int dbg_sm_count() {
 }
 
 bool dbg_params_ok(const dbg_params* prm) {
-  return prm && prm->k >= 1 && prm->k <= 63 && (prm->k & 1) && prm->p >= 1 && prm->p <= prm->k &&
+  // K <= 127 (row f3); K > 63 keeps the device partitioning on P (no fine_p, reading V)
+  if (prm && prm->k > 63 && prm->fine_p != 0 && prm->fine_p != prm->p) return false;
+  return prm && prm->k >= 1 && prm->k <= 127 && (prm->k & 1) && prm->p >= 1 && prm->p <= prm->k &&
          prm->p <= 31 && prm->fine_p >= 0 && prm->fine_p <= prm->k && prm->fine_p <= 31 &&
          prm->num_partitions >= 1 && prm->refine >= 0 &&
          (uint64_t)prm->num_partitions * (uint64_t)(prm->refine > 1 ? prm->refine : 1) <= kMaxPid;
@@ -391,9 +409,14 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       scatter_kernel<4><<<grid, kScatterThreads, smem, stream>>>(
           part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
           part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
-    } else {
+    } else if (R == 8) {
       cudaFuncSetAttribute(scatter_kernel<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       scatter_kernel<8><<<grid, kScatterThreads, smem, stream>>>(
+          part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
+          part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
+    } else {
+      cudaFuncSetAttribute(scatter_kernel<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      scatter_kernel<16><<<grid, kScatterThreads, smem, stream>>>(
           part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
           part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
     }
@@ -419,6 +442,6 @@ extern "C" dbg_status dbg_table_plan(const dbg_params* prm, const uint64_t* d_n_
 
 extern "C" dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers, uint64_t* d_table_offset,
                                            uint64_t* d_scratch, cudaStream_t stream) {
-  if (!prm) return DBG_EINVAL;
+  if (!prm || prm->k > 63) return DBG_EINVAL;
   return table_plan(prm, d_n_kmers, dbg_smem_table_slots(prm), d_table_offset, d_scratch, stream);
 }

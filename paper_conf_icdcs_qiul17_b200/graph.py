@@ -28,7 +28,7 @@ import numpy as np
 import torch
 
 from . import _lib
-from ._lib import VERTEX_DTYPE, STATS_FIELDS
+from ._lib import VERTEX_DTYPE, VERTEX_WIDE_DTYPE, STATS_FIELDS
 
 
 def encode_reads(seq: np.ndarray, pin: bool = False) -> torch.Tensor:
@@ -73,13 +73,16 @@ class DbgBuilder:
                  device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
                  mode: str = "smem", group_slots: int = 1 << 19, refine: int = 1, smem_split: int = 0,
                  fine_p: int = 0, min_count: int = 0):
-        if k % 2 == 0 or not 1 <= k <= 63:
-            raise ValueError("K must be odd and 1..63 (DESIGN.md reading C)")
+        if k % 2 == 0 or not 1 <= k <= 127:
+            raise ValueError("K must be odd and 1..127 (DESIGN.md reading C)")
+        if k > 63 and mode != "resident":
+            raise ValueError("K > 63 (row f3) runs through the resident tables: mode='resident'")
         if not 1 <= p <= min(k, 31):
             raise ValueError("P must be in 1..min(K, 31)")
         if mode not in ("smem", "fused", "resident"):
             raise ValueError(mode)
         self.k, self.p, self.mode = k, p, mode
+        self.vdtype = VERTEX_WIDE_DTYPE if k > 63 else VERTEX_DTYPE  # dbg_vertex_wide for K > 63
         self.np_out = num_partitions                 # the paper's NP (dbg_vertex.pid)
         self.refine = max(1, int(refine))
         self.np = num_partitions * self.refine       # fine partitions the device works on
@@ -328,10 +331,10 @@ class DbgBuilder:
             self.d_n_out.zero_()
             self.d_stats.zero_()
             self.d_status.zero_()
-        self.out = _grow(self.out, cap * VERTEX_DTYPE.itemsize, torch.uint8, self.device)
+        self.out = _grow(self.out, cap * self.vdtype.itemsize, torch.uint8, self.device)
 
     def out_cap(self) -> int:
-        return self.out.numel() // VERTEX_DTYPE.itemsize
+        return self.out.numel() // self.vdtype.itemsize
 
     def step2(self, stream=None) -> None:
         """Hash + extract of every partition (output appended to self.out)."""
@@ -394,7 +397,7 @@ class DbgBuilder:
     def stats(self, checksum: bool = True, stream=None) -> dict:
         """Totals of the last extraction; the checksum is computed here (dbg_checksum_vertices)."""
         stream = stream or torch.cuda.current_stream(self.device)
-        if checksum:
+        if checksum and self.k <= 63:
             n = min(int(self.d_n_out.item()), self.out_cap())
             with torch.cuda.stream(stream):
                 self.d_stats[3].zero_()
@@ -406,8 +409,14 @@ class DbgBuilder:
         """D2H of the compacted records (sorted on the device by dbg_sort_vertices)."""
         stream = stream or torch.cuda.current_stream(self.device)
         n = int(self.d_n_out.item())
-        nbytes = n * VERTEX_DTYPE.itemsize
+        nbytes = n * self.vdtype.itemsize
         src = self.out[:nbytes]
+        if self.k > 63:  # dbg_vertex_wide: sorted on the host (dbg_sort_vertices takes K <= 63)
+            v = src.cpu().numpy().view(self.vdtype)
+            if sort and n:
+                k = v["kmer"]
+                v = v[np.lexsort((k[:, 3], k[:, 2], k[:, 1], k[:, 0]))]
+            return v
         if sort and n:
             dst = torch.empty(nbytes, dtype=torch.uint8, device=self.device)
             wsb = _lib.dbg_sort_workspace_bytes(self.prm, n)
@@ -507,6 +516,8 @@ def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partit
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
     lens = np.diff(np.asarray(offsets, dtype=np.int64))
     n_kmers = int(np.maximum(lens - k + 1, 0).sum())
+    if k > 63:  # row f3: resident tables, partitions on P
+        mode, refine, fine_p = "resident", 1 if refine == "auto" else refine, 0
     if refine == "auto":
         refine = auto_refine(n_kmers, k, p, num_partitions, lam, alpha) if mode == "smem" else 1
     if fine_p == "auto":

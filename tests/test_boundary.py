@@ -36,7 +36,7 @@ def test_exports_every_declared_symbol(lib):
 
 
 def test_abi_and_sizes(lib):
-    assert lib.dbg_abi_version() == 7
+    assert lib.dbg_abi_version() == 8
     p31 = lib.params(31, 11, 16)
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
@@ -131,7 +131,8 @@ def test_invalid_arguments_return_before_launch(lib):
 
     part = partition_set(1, 1, 1, 1, 1, None, 0, None)
     for prm in (lib.params(30, 11, 16), lib.params(31, 0, 16), lib.params(31, 32, 16), lib.params(31, 11, 0),
-                lib.params(65, 11, 16), lib.params(31, 11, 16, fine_p=32), lib.params(21, 11, 16, fine_p=23),
+                lib.params(129, 11, 16), lib.params(64, 11, 16), lib.params(65, 11, 16, fine_p=13),
+                lib.params(31, 11, 16, fine_p=32), lib.params(21, 11, 16, fine_p=23),
                 lib.params(31, 11, 16, fine_p=-1)):
         with pytest.raises(DbgError) as e:
             lib.dbg_msp_partition(prm, 1, 1, 1, 1, part, None)
@@ -139,6 +140,14 @@ def test_invalid_arguments_return_before_launch(lib):
     with pytest.raises(DbgError):
         lib.dbg_hash_build(lib.params(31, 11, 16), partition_set(1, 1, 1, 1, 1, None, 0, 1), 5, 2, 1, 1, 1, None)
     assert lib.dbg_status_string(lib.DBG_ETABLEFULL).startswith("hash table full")
+    # row f3: K > 63 runs through the resident tables only
+    p65 = lib.params(65, 21, 4)
+    assert lib.dbg_record_words(p65) == 16 and lib.dbg_record_max_kmers(p65) == 240 - 65 - 1
+    assert lib.dbg_key_bytes(p65) == 48 and lib.dbg_slot_bytes(p65) == 80
+    assert lib.dbg_smem_onchip(p65, 100) == 0 and lib.dbg_smem_table_slots(p65) == 0
+    with pytest.raises(DbgError) as e:
+        lib.dbg_table_plan_split(p65, 1, 1, None, None)
+    assert e.value.status == lib.DBG_EINVAL
 
 
 def test_product_has_no_oracle_dependency():
