@@ -361,6 +361,14 @@ def run_ours(args):
     launches_per_step = 2 + scan + {"fused": scan + 2, "resident": scan + 2 * nb,
                                     "smem": 8 + 2 * nb + (scan if nb else 0)}[args.mode]
     placement = _placement(b) if args.mode == "smem" else None
+    # Fig. 6 / Table II analogue (row f1): the paper's partitions (fine pid mod NP) -- skew and the
+    # table size lambda/(4 alpha) N^i_kmer x slot bytes of the largest one
+    paper_parts = np.bincount(np.arange(b.np) % rs.num_partitions, weights=b.part_kmers,
+                              minlength=rs.num_partitions)
+    psizes = {"max_over_mean": float(paper_parts.max() / max(paper_parts.mean(), 1e-9)),
+              "max_kmers": int(paper_parts.max()), "mean_kmers": float(paper_parts.mean()),
+              "max_table_mb": _lib.dbg_table_capacity(b.prm, int(paper_parts.max())) * b.slot_bytes / 1e6,
+              "fine_max_over_mean": float(b.part_kmers.max() / max(b.part_kmers.mean(), 1e-9))}
     if rank != 0:
         dist.barrier()
         dist.destroy_process_group()
@@ -368,7 +376,7 @@ def run_ours(args):
     cfg_extra = {"mode": args.mode, "batches": len(b.batches), "group_slots": args.group_slots, "refine": refine,
                  "fine_partitions": b.np, "smem_split": args.smem_split, "fine_p": fine_p or rs.p,
                  "smem_slots": _lib.dbg_smem_table_slots(b.prm), "kmer_placement": placement,
-                 "kernel_version": KERNEL_VERSION}
+                 "kernel_version": KERNEL_VERSION, "partition_sizes": psizes}
     if ws > 1:
         cfg_extra.update({"reads_per_rank": rs.n_reads, "kmers_total": total_kmers,
                           "parallelism": f"reads sharded; fine partitions owned by rank (one all_to_all of "
