@@ -106,6 +106,40 @@ __device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, ui
   }
 }
 
+// 32-bit shared-window accesses for the per-base loop (keeps generic-pointer
+// arithmetic and the shared-window base out of it).
+__device__ __forceinline__ uint32_t sh_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint32_t sh_ld(uint32_t a, uint32_t) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t sh_ld(uint32_t a, uint64_t) {
+  uint64_t v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sh_st(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sh_st(uint32_t a, uint64_t v) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+// Pins a value in a register (the compiler may not re-derive it from the
+// constant bank inside the per-base loop).
+template <typename T>
+__device__ __forceinline__ T in_reg(T v) {
+  if constexpr (sizeof(T) == 8) {
+    uint64_t x = (uint64_t)v;
+    asm volatile("" : "+l"(x));
+    return (T)x;
+  } else {
+    uint32_t x = (uint32_t)v;
+    asm volatile("" : "+r"(x));
+    return (T)x;
+  }
+}
+
 // Warp-collective flush of the per-thread descriptor lists: partition ids,
 // size histograms, one staging reservation per warp, record writes.
 template <typename CT>
@@ -175,11 +209,16 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   sp += sizeof(uint32_t) * kMaxDesc * kMspThreads;
   sm.row = reinterpret_cast<CT*>(sp);
 
-  const int K = a.k, P = a.p, w = a.w;
-  const CT maskP = (CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1));
-  const int topP = 2 * P - 2;
+  const int K = a.k, P = in_reg(a.p), w = in_reg(a.w);
+  const CT maskP = in_reg((CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1)));
+  const int topP = in_reg(2 * P - 2);
   const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
   CT* row = sm.row + tid;
+  // shared-window addresses of this thread's column of the van Herk block and descriptors
+  const uint32_t row_a = in_reg(sh_addr(row)), de_a = in_reg(sh_addr(sm.desc_e + tid)),
+                 dm_a = in_reg(sh_addr(sm.desc_m + tid));
+  constexpr uint32_t kRowStep = kMspThreads * sizeof(CT), kDescStepE = kMspThreads * 4,
+                     kDescStepM = kMspThreads * sizeof(CT);
   // all lanes of a warp iterate together; a warp covers 32 consecutive reads
   for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
     const uint64_t r = r0 + lane;
@@ -209,28 +248,32 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
         if (j < P - 1) continue;
         const int q = j - P + 1;  // P-mer index
         const CT c = f < rc ? f : rc;
-        const CT snext = (u + 1 < w) ? row[(u + 1) * kMspThreads] : (CT)0;
-        row[u * kMspThreads] = c;
+        const uint32_t ua = row_a + (uint32_t)u * kRowStep;
+        const CT snext = (u + 1 < w) ? sh_ld(ua + kRowStep, (CT)0) : (CT)0;
+        sh_st(ua, c);
         pre = (u == 0 || c < pre) ? c : pre;
         if (q >= w - 1) {  // K-mer i = q-w+1 is complete
           const int i = q - w + 1;
           const CT m = (u == w - 1 || pre < snext) ? pre : snext;
           if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
-            sm.desc_e[ndesc * kMspThreads + tid] = (uint32_t)(i - 1);
-            sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
+            sh_st(de_a + (uint32_t)ndesc * kDescStepE, (uint32_t)(i - 1));
+            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, m_cur);
             ++ndesc;
           }
           m_cur = m;
           if (i == nk - 1) {  // the read's last superkmer
-            sm.desc_e[ndesc * kMspThreads + tid] = (uint32_t)i;
-            sm.desc_m[ndesc * kMspThreads + tid] = m_cur;
+            sh_st(de_a + (uint32_t)ndesc * kDescStepE, (uint32_t)i);
+            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, m_cur);
             ++ndesc;
           }
         }
         if (u == w - 1) {  // block complete: suffix minima in place
+          CT y = sh_ld(row_a + (uint32_t)(w - 1) * kRowStep, (CT)0);
           for (int t = w - 2; t >= 0; --t) {
-            const CT x = row[t * kMspThreads], y = row[(t + 1) * kMspThreads];
-            if (y < x) row[t * kMspThreads] = y;
+            const uint32_t ta = row_a + (uint32_t)t * kRowStep;
+            const CT x = sh_ld(ta, (CT)0);
+            if (y < x) sh_st(ta, y);
+            else y = x;
           }
           u = 0;
         } else {
@@ -267,18 +310,32 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
     }
     uint4 rec[kPer][R / 4];
     uint32_t rank[kPer];
+    // all loads of the tile first, then all rank atomics, then all stores: kPer records of
+    // each thread in flight at every stage (the kernel is latency-bound)
+#pragma unroll
+    for (int v = 0; v < kPer; ++v) {
+      const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
+      if (idx < n) {
+        const uint4* src = reinterpret_cast<const uint4*>(staging + idx * R);
+#pragma unroll
+        for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(src + c);
+      }
+    }
 #pragma unroll
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       rank[v] = 0;
       if (idx < n) {
-        const uint4* src = reinterpret_cast<const uint4*>(staging + idx * R);
-#pragma unroll
-        for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(src + c);
         const uint32_t pid = rec[v][0].x >> 10;
         if (smem) rank[v] = atomicAdd(sh_cnt + pid, 1u);
         else rank[v] = (uint32_t)atomicAdd(fill + pid, 1ull);
       }
+    }
+    uint64_t base[kPer];
+#pragma unroll
+    for (int v = 0; v < kPer; ++v) {
+      const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
+      base[v] = idx < n ? __ldg(rec_off + (rec[v][0].x >> 10)) : 0;
     }
     if (smem) {
       __syncthreads();
@@ -291,7 +348,7 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       if (idx < n) {
         const uint32_t pid = rec[v][0].x >> 10;
-        const uint64_t pos = rec_off[pid] + (smem ? sh_base[pid] + rank[v] : rank[v]);
+        const uint64_t pos = base[v] + (smem ? sh_base[pid] + rank[v] : rank[v]);
         uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
 #pragma unroll
         for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];

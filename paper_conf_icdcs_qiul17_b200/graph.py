@@ -197,6 +197,52 @@ class DbgBuilder:
         _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
         self._done(ev, stream)
 
+    def msp_overlapped(self, h_packed: torch.Tensor, h_offsets: torch.Tensor, d_bases: torch.Tensor,
+                       d_offsets: torch.Tensor, n_batches: int = 8, stream=None, copy_stream=None):
+        """Rows a1-a4 with the upload overlapped (Sec. III-E): the pinned host reads go
+        H2D in n_batches read ranges on copy_stream, and pass 1 of range b (dbg_msp_partition_range
+        over all partitions, appending) runs on `stream` as soon as its words have arrived, while
+        range b+1 is still in flight; then the sizes copy and pass 2 as in msp()."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        copy_stream = copy_stream or torch.cuda.Stream(self.device)
+        n_reads = h_offsets.numel() - 1
+        n_words = h_packed.numel()
+        if self.staging.numel() == 0:
+            self.staging = _grow(self.staging, self._staging_estimate(n_words * 32, n_reads) * self.rec_words,
+                                 torch.int32, self.device)
+        self.overflowed = False
+        offs = h_offsets.numpy()
+        bounds = [n_reads * i // n_batches for i in range(n_batches + 1)]
+        copy_stream.wait_stream(stream)  # d_bases / d_offsets are free (the previous step is done with them)
+        w_done = 0
+        ev = self._mark("msp_pass1", stream)
+        for i in range(n_batches):
+            r0, r1 = bounds[i], bounds[i + 1]
+            w1 = min(n_words, int(offs[r1]) // 32 + 2)  # the words of reads < r1 (+ the pad word)
+            with torch.cuda.stream(copy_stream):
+                if w1 > w_done:
+                    d_bases[w_done:w1].copy_(h_packed[w_done:w1], non_blocking=True)
+                d_offsets[r0:r1 + 1].copy_(h_offsets[r0:r1 + 1], non_blocking=True)
+            w_done = max(w_done, w1)
+            arrived = torch.cuda.Event()
+            arrived.record(copy_stream)
+            stream.wait_event(arrived)
+            if r1 > r0 or i == 0:
+                _lib.dbg_msp_partition_range(self.prm, d_bases, n_words, d_offsets[r0:], r1 - r0,
+                                             self.part_set(False), 0, self.np, i > 0, stream)
+        self._done(ev, stream)
+        if self._h_sizes.numel() != 2 * self.np:
+            self._h_sizes = torch.empty(2 * self.np, dtype=torch.int64, pin_memory=True)
+        with torch.cuda.stream(stream):
+            self._h_sizes[:self.np].copy_(self.d_n_records, non_blocking=True)
+            self._h_sizes[self.np:].copy_(self.d_n_kmers, non_blocking=True)
+        self._sizes_ev.record(stream)
+        self._sizes_pending = True
+        self.records = _grow(self.records, self.staging.numel(), torch.int32, self.device)
+        ev = self._mark("msp_scatter", stream)
+        _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
+        self._done(ev, stream)
+
     def sync_sizes(self) -> bool:
         """Waits for the pass-1 sizes (part_records, part_kmers).  False after a staging overflow:
         the staging has been grown and the step must be repeated (self.overflowed)."""

@@ -397,3 +397,23 @@ def test_low_count_filter(mode, k, p, np_, refine, split, min_count):
     # builder (same table buffers) is exact
     b.prm.min_count = b.min_count = 0
     compare_vertices(b.build(d_bases, d_off).vertices, full)
+
+
+@pytest.mark.parametrize("n_batches", [1, 3, 8])
+def test_msp_overlapped_upload_equals_single_pass(n_batches):
+    """DbgBuilder.msp_overlapped (read ranges uploaded on a copy stream, MSP appended per range)
+    builds the same graph as the single upload + MSP, ragged reads included."""
+    rs = random_reads(3000, 1, 300, seed=51, n_rate=0.01)
+    b = DbgBuilder(31, 11, 16, refine=4)
+    packed = encode_reads(rs.seq, pin=True)
+    offs = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
+    db = torch.empty(packed.numel(), dtype=torch.int64, device="cuda")
+    do = torch.empty(offs.numel(), dtype=torch.int64, device="cuda")
+    b.msp_overlapped(packed, offs, db, do, n_batches)
+    assert b.sync_sizes()
+    b.plan()
+    b.reset_output(1 << 20)
+    b.step2()
+    assert _lib.dbg_sync_status(b.d_status) == 0
+    orc = oracle.graph(rs.seq, rs.offsets, 31, 11, 16, n_threads=NT)
+    compare_vertices(b.vertices(), orc)
