@@ -29,6 +29,8 @@
 // reservation per partition per tile).
 #include <cub/block/block_scan.cuh>
 
+#include <cstdlib>
+
 #include "dbg_device.cuh"
 #include "scan.cuh"
 
@@ -358,6 +360,115 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
   }
 }
 
+// Register-blocked variant for compile-time W = K - P + 1 and P <= 16 (the
+// configurations' K = 31 with P = 11..15): the van Herk blocks of W P-mer
+// values live in registers (fully unrolled), so the per-base work is the
+// rolling P-mer, one prefix minimum and, per block, the suffix minima --
+// no shared-memory row.  K-mer i's minimizer (Def. 1) is
+// min(suffix_min_prev[t], prefix_min_cur[t-1]) for i = q0 - W + t, where the
+// current block holds P-mers q0 .. q0+W-1.  Same descriptors and flush as
+// msp_kernel; reads of any length (lanes past their read end run masked).
+template <int W, int P>
+__global__ void __launch_bounds__(kMspThreads) msp_block_kernel(MspArgs a) {
+  typedef uint32_t CT;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int tid = threadIdx.x, lane = tid & 31;
+  MspSmem<CT> sm;
+  unsigned char* sp = smem_raw;
+  sm.desc_m = reinterpret_cast<CT*>(sp);
+  sp += sizeof(CT) * kMaxDesc * kMspThreads;
+  sm.desc_e = reinterpret_cast<uint32_t*>(sp);
+  sm.row = nullptr;
+  constexpr CT kMaskP = (CT)((2 * P == 32) ? ~0u : ((1u << (2 * P)) - 1));
+  constexpr CT kInf = ~(CT)0;
+  constexpr int kTopP = 2 * P - 2;
+  constexpr int K = W + P - 1;
+  const uint32_t de_a = sh_addr(sm.desc_e + tid), dm_a = sh_addr(sm.desc_m + tid);
+  constexpr uint32_t kDescStep = kMspThreads * 4;
+  const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
+  for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
+    const uint64_t r = r0 + lane;
+    uint64_t o = 0;
+    int L = 0;
+    if (r < a.n_reads) {
+      o = a.offsets[r];
+      L = (int)(a.offsets[r + 1] - o);
+    }
+    const int nk = L - K + 1;
+    if (nk <= 0) L = 0;  // reading N: no K-mers
+    const int nP = L > 0 ? L - P + 1 : 0;  // P-mers of the read
+    int nPmax = nP;
+#pragma unroll
+    for (int dlt = 16; dlt; dlt >>= 1) nPmax = max(nPmax, __shfl_xor_sync(kFull, nPmax, dlt));
+    int ndesc = 0, s_next = 0;
+    CT f = 0, rc = 0, m_cur = 0;
+    // the bases: a 64-bit window refilled every 32 bases
+    uint64_t wbuf = L > 0 ? window64(a.words, a.n_words, o) : 0;
+    int nbuf = 32, j = 0;  // bases left in wbuf, next base index
+    auto next_base = [&]() -> uint32_t {
+      if (nbuf == 0) {
+        wbuf = j < L ? window64(a.words, a.n_words, o + j) : 0;
+        nbuf = 32;
+      }
+      const uint32_t b = (uint32_t)(wbuf >> 62);
+      wbuf <<= 2;
+      --nbuf;
+      ++j;
+      return b;
+    };
+#pragma unroll
+    for (int t = 0; t < P - 1; ++t) {  // the first P-1 bases: no P-mer yet
+      const uint32_t b = next_base();
+      f = ((f << 2) | b) & kMaskP;
+      rc = (rc >> 2) | ((CT)(3u - b) << kTopP);
+    }
+    CT suf[W];
+#pragma unroll
+    for (int t = 0; t < W; ++t) suf[t] = kInf;
+    // blocks of W P-mers; one extra block of padding emits the last K-mers
+    for (int q0 = 0; q0 < nPmax + W; q0 += W) {
+      CT c[W], pre[W];
+#pragma unroll
+      for (int t = 0; t < W; ++t) {
+        CT v = kInf;
+        if (q0 + t < nP) {
+          const uint32_t b = next_base();
+          f = ((f << 2) | b) & kMaskP;
+          rc = (rc >> 2) | ((CT)(3u - b) << kTopP);
+          v = f < rc ? f : rc;  // canonical P-mer (reading D)
+        }
+        c[t] = v;
+        pre[t] = t == 0 ? v : (v < pre[t - 1] ? v : pre[t - 1]);
+      }
+      if (q0 >= W) {  // K-mers i = q0 - W + t of the previous block's windows
+#pragma unroll
+        for (int t = 0; t < W; ++t) {
+          const int i = q0 - W + t;
+          if (i < nk) {
+            const CT m = t == 0 ? suf[0] : (suf[t] < pre[t - 1] ? suf[t] : pre[t - 1]);
+            if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
+              sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(i - 1));
+              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+              ++ndesc;
+            }
+            m_cur = m;
+            if (i == nk - 1) {  // the read's last superkmer
+              sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
+              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+              ++ndesc;
+            }
+          }
+        }
+      }
+      suf[W - 1] = c[W - 1];
+#pragma unroll
+      for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
+      if (__any_sync(kFull, ndesc > kMaxDesc - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+    }
+    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+  }
+}
+
 }  // namespace dbg
 
 using namespace dbg;
@@ -375,6 +486,28 @@ bool dbg_params_ok(const dbg_params* prm) {
          prm->p <= 31 && prm->fine_p >= 0 && prm->fine_p <= prm->k && prm->fine_p <= 31 &&
          prm->num_partitions >= 1 && prm->refine >= 0 &&
          (uint64_t)prm->num_partitions * (uint64_t)(prm->refine > 1 ? prm->refine : 1) <= kMaxPid;
+}
+
+template <int W, int P>
+static cudaError_t launch_msp_block(const MspArgs& a, int grid, cudaStream_t stream) {
+  const size_t smem = (sizeof(uint32_t) + sizeof(uint32_t)) * kMaxDesc * kMspThreads;
+  cudaError_t e = cudaFuncSetAttribute(msp_block_kernel<W, P>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  msp_block_kernel<W, P><<<grid, kMspThreads, smem, stream>>>(a);
+  return cudaGetLastError();
+}
+
+// The register-blocked kernel for the configurations' K = 31 (P = 11..15), else the generic one.
+static bool msp_block_launch(const MspArgs& a, int grid, cudaStream_t stream, cudaError_t* e) {
+  if (getenv("DBG_MSP_GENERIC") || a.k != 31) return false;
+  switch (a.p) {
+    case 11: *e = launch_msp_block<21, 11>(a, grid, stream); return true;
+    case 12: *e = launch_msp_block<20, 12>(a, grid, stream); return true;
+    case 13: *e = launch_msp_block<19, 13>(a, grid, stream); return true;
+    case 14: *e = launch_msp_block<18, 14>(a, grid, stream); return true;
+    case 15: *e = launch_msp_block<17, 15>(a, grid, stream); return true;
+  }
+  return false;
 }
 
 template <typename CT>
@@ -447,8 +580,9 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       const uint64_t want = (n_reads + kMspThreads - 1) / kMspThreads;
       const uint64_t cap = (uint64_t)dbg_sm_count() * 8;
       const int grid = (int)(want < cap ? want : cap);
-      const cudaError_t e = a.p <= 16 ? launch_msp<uint32_t>(a, grid, stream)
-                                         : launch_msp<uint64_t>(a, grid, stream);
+      cudaError_t e = cudaSuccess;
+      if (!msp_block_launch(a, grid, stream, &e))
+        e = a.p <= 16 ? launch_msp<uint32_t>(a, grid, stream) : launch_msp<uint64_t>(a, grid, stream);
       if (e != cudaSuccess) return DBG_ECUDA;
     }
     // d_fill is idle until pass 2 (which zeroes it): scratch for the tile sums

@@ -417,3 +417,22 @@ def test_msp_overlapped_upload_equals_single_pass(n_batches):
     assert _lib.dbg_sync_status(b.d_status) == 0
     orc = oracle.graph(rs.seq, rs.offsets, 31, 11, 16, n_threads=NT)
     compare_vertices(b.vertices(), orc)
+
+
+@pytest.mark.parametrize("p", [11, 12, 13, 14, 15])
+def test_register_blocked_msp_variants(p):
+    """K = 31, P = 11..15 run msp_block_kernel<W, P> (van Herk blocks in registers): ragged reads
+    (shorter than K, one K-mer, many blocks), N bases; MSP records vs the oracle's superkmers and
+    the whole graph vs the oracle."""
+    rs = random_reads(2500, 1, 420, seed=60 + p, n_rate=0.02)
+    _check(rs, 31, p, 13)
+    b = DbgBuilder(31, p, 13)
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    b.msp(d_bases, d_off)
+    assert b.sync_sizes()
+    torch.cuda.synchronize()
+    n = int(b.part_records.sum())
+    words = b.records[:n * b.rec_words].cpu().numpy().view(np.uint32)
+    got = occurrences_from_records(decode_records(words, b.rec_words, 31), 31)
+    sk = oracle.msp(rs.seq, rs.offsets, 31, p, 13)
+    assert got == occurrences_from_oracle_msp(sk, rs.reads(), 31)
