@@ -36,7 +36,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 8
+#define DBG_ABI_VERSION 9
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -134,6 +134,10 @@ typedef struct {
   uint32_t* d_staging;       /* staging_cap records, read order (pass 1 output, pass 2 input) */
   uint64_t staging_cap;      /* capacity of d_staging in records */
   uint32_t* d_records;       /* d_record_offset[NP] records in partition order; NULL => pass 1 */
+  uint32_t* d_scratch;       /* optional, staging_cap records (not aliasing d_staging or d_records):
+                                with more than 8192 fine partitions pass 2 then scatters in two
+                                levels -- into buckets of 2^s consecutive partitions (d_scratch),
+                                then within each bucket (d_records); NULL: one level */
 } dbg_partition_set;
 
 /* ---- sizes ------------------------------------------------------------ */
@@ -167,7 +171,9 @@ DBG_API dbg_status dbg_encode_ascii(const char* seq, uint64_t n_bases, uint64_t*
  *   d_staging while they fit.  The caller reads d_record_offset[NP] (or the
  *   sizes); if it exceeds staging_cap, it grows d_staging and repeats pass 1.
  * part->d_records != NULL: pass 2 -- scatters the staged records into
- *   partition order (d_record_offset[NP] records).
+ *   partition order (d_record_offset[NP] records), through d_scratch when it is
+ *   set (two levels; the order of the records inside a partition is not
+ *   specified either way).
  * A caller may enqueue pass 2 and Step 2 before reading the sizes back: after a
  * staging overflow (*d_staged > staging_cap) pass 2 and
  * dbg_build_subgraphs_smem do nothing, and the caller grows d_staging and

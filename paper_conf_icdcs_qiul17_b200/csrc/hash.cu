@@ -856,6 +856,17 @@ __device__ __forceinline__ uint64_t cas_shared64(uint32_t a, uint64_t want) {
   asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(a), "l"(0ull), "l"(want) : "memory");
   return old;
 }
+// Predicated CAS: cur = atom.cas(a, 0, want) when p, unchanged otherwise.
+__device__ __forceinline__ void cas_shared64_if(bool p, uint32_t a, uint64_t want, uint64_t& cur) {
+  asm volatile(
+      "{ .reg .pred q; setp.ne.u32 q, %1, 0; @q atom.shared.cas.b64 %0, [%2], %3, %4; }"
+      : "+l"(cur)
+      : "r"((uint32_t)p), "r"(a), "l"(0ull), "l"(want)
+      : "memory");
+}
+__device__ __forceinline__ void red_shared_or(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 __device__ __forceinline__ void red_shared_add(uint32_t a, uint32_t v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
@@ -1111,12 +1122,16 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
   char* keys = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
   uint32_t* fld = reinterpret_cast<uint32_t*>(keys + a.slots * KB);
-  const uint32_t keys_s = smem_addr(keys), fld_s = smem_addr(fld);
+  // occupancy bitmap of the table (bit s = slot s holds a vertex): extraction reads one word
+  // per 32 slots instead of 32 keys
+  uint32_t* occ = fld + a.slots * FW;
+  const uint32_t keys_s = smem_addr(keys), fld_s = smem_addr(fld), occ_s = smem_addr(occ);
   const int K = a.k;
   {  // the table starts clean; extraction keeps it clean (slots is a multiple of 64)
     uint4* z = reinterpret_cast<uint4*>(keys);
     for (uint64_t q = threadIdx.x; q < a.slots * SmemSlot<KW>::kBytes / 16; q += kSmemThreads)
       z[q] = make_uint4(0, 0, 0, 0);
+    for (uint64_t q = threadIdx.x; q < a.slots / 32; q += kSmemThreads) occ[q] = 0;
   }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
@@ -1245,10 +1260,15 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         Code fwd, rc;
         int pred, succ;
         if constexpr (R == 4) {
-          const int q = b >> 4;  // the words holding bases b .. b + 47 - 16q
-          const uint32_t a1 = w[(1 + q) * S], a2 = q < 2 ? w[(2 + q) * S] : 0u, a3 = q == 0 ? w[3 * S] : 0u;
-          const int pb = b - 1;  // the predecessor base
-          pred = b > 0 ? (int)((w[(1 + (pb >> 4)) * S] >> (30 - 2 * (pb & 15))) & 3u) : -1;
+          // the three data words, loaded unconditionally and selected (no branches): a1..a3
+          // hold bases b .. b + 47 - 16q
+          const uint32_t d1 = w[S], d2 = w[2 * S], d3 = w[3 * S];
+          const int q = b >> 4;
+          const uint32_t a1 = q == 0 ? d1 : (q == 1 ? d2 : d3), a2 = q == 0 ? d2 : (q == 1 ? d3 : 0u),
+                         a3 = q == 0 ? d3 : 0u;
+          const int pb = b - 1, pq = pb >> 4;  // the predecessor base
+          const uint32_t pw = pq <= 0 ? d1 : (pq == 1 ? d2 : d3);
+          pred = b > 0 ? (int)((pw >> (30 - 2 * (pb & 15))) & 3u) : -1;
           if constexpr (sizeof(Code) == 8) {
             // 64 bits of the record from base b: two 32-bit funnel shifts
             const uint32_t sh = 2 * (b & 15);
@@ -1278,35 +1298,56 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         // one insertion, multiple updates: probe rounds until every lane has
         // found or claimed its slot, then the counter updates, warp-converged
         const typename KO::T key = KO::make(code);
-        uint32_t idx = __umulhi(smem_hash(code), cap), probes = 0;
-        uint32_t pend = want, inserted = 0;
+        uint32_t idx = __umulhi(smem_hash(code), cap);
+        uint32_t inserted = 0;
         const uint32_t kaddr = keys_s + t0 * KB;
-        while (__any_sync(kFull, pend)) {
-          if (pend) {
-            typename KO::T cur;
-            if constexpr (KW == 1) {
-              const uint32_t ka = kaddr + idx * KB;
-              cur = lds64(ka);
-              if (cur == 0) cur = cas_shared64(ka, key);
-            } else {
-              cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);  // 16-B shared-memory CAS: read-or-claim
-            }
-            inserted = KO::empty(cur);
-            if (inserted | KO::same(cur, key)) {
-              pend = 0;
-            } else {
-              idx = idx + 1 == cap ? 0 : idx + 1;
-              if (++probes == cap) {  // wrapped: table full (reading O)
+        if constexpr (KW == 1) {
+          // every lane runs every probe round (predicated, no divergent branch): a lane with
+          // nothing pending re-reads its current slot and keeps its state
+          const uint32_t idx0 = idx;
+          bool pend = want;
+          for (;;) {
+            const uint32_t ka = kaddr + idx * KB;
+            uint64_t cur = lds64(ka);
+            cas_shared64_if(pend && cur == 0, ka, key, cur);
+            const bool hit = cur == 0 || cur == key;
+            inserted |= (uint32_t)(pend && cur == 0);
+            const bool adv = pend && !hit;
+            const uint32_t nx = idx + 1 == cap ? 0u : idx + 1;
+            idx = adv ? nx : idx;
+            pend = adv && nx != idx0;
+            if (adv && nx == idx0) ok = false;  // wrapped: table full (reading O)
+            if (!__any_sync(kFull, pend)) break;
+          }
+          if (!ok && want) {
+            const uint64_t cur = lds64(kaddr + idx * KB);
+            if (cur != key) idx = ~0u;  // this occurrence found no slot
+          }
+        } else {
+          uint32_t probes = 0, pend = want;
+          while (__any_sync(kFull, pend)) {
+            if (pend) {
+              const typename KO::T cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);  // 16-B CAS: read-or-claim
+              inserted = KO::empty(cur);
+              if (inserted | KO::same(cur, key)) {
                 pend = 0;
-                ok = false;
-                idx = ~0u;
+              } else {
+                idx = idx + 1 == cap ? 0 : idx + 1;
+                if (++probes == cap) {  // wrapped: table full (reading O)
+                  pend = 0;
+                  ok = false;
+                  idx = ~0u;
+                }
               }
             }
           }
         }
         if (want && idx != ~0u) {  // the multiple updates: 16-bit fields, two per word
           const uint32_t fa = fld_s + (t0 + idx) * (FW * 4);
-          if (inserted) sts32(fa + 20, w[0] >> 10);
+          if (inserted) {
+            sts32(fa + 20, w[0] >> 10);
+            red_shared_or(occ_s + 4 * ((t0 + idx) >> 5), 1u << ((t0 + idx) & 31u));
+          }
           const int fo = o < 4 ? o : 8;
           red_shared_add(fa + 4 * (fo >> 1), 1u << (16 * (fo & 1)));
           if (i >= 0) red_shared_add(fa + 4 * ((4 + i) >> 1), 1u << (16 * (i & 1)));
@@ -1329,7 +1370,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         uint32_t qn = 0;
         for (uint32_t c = sub; c < se; c += 32) {
           const uint32_t s = c + lane;
-          bool keep = s < se && (lds64(keys_s + s * KB) & kOccupied);
+          bool keep = ((se - c >= 32 ? occ[c >> 5] : occ[c >> 5] & ((1u << (se - c)) - 1u)) >> lane) & 1u;
           if (keep && oa.min_count > 1) {  // row f4: a low-count vertex is cleaned, never emitted
             const uint32_t* f = fld + s * FW;
             const uint32_t f0 = f[0], f1 = f[1];
@@ -1347,6 +1388,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           if (keep) queue[qn + __popc(bal & ((1u << lane) - 1u))] = (uint16_t)s;
           qn += __popc(bal);
         }
+        for (uint32_t c = (sub >> 5) + lane; c < (se + 31) >> 5; c += 32) occ[c] = 0;
         unsigned long long pos = 0;
         if (lane == 0 && qn) pos = atomicAdd(oa.n_out, (unsigned long long)qn);
         pos = __shfl_sync(kFull, pos, 0);
@@ -1557,7 +1599,7 @@ template <int R, int T>
 static uint64_t smem_slots_for(int k, int ctas) {
   const uint64_t avail = (227u * 1024u) / ctas - smem_fixed_bytes<R, T>() - 1024u;
   const uint32_t sb = k <= 31 ? SmemSlot<1>::kBytes : SmemSlot<2>::kBytes;
-  const uint64_t n = (avail / sb) & ~(uint64_t)63;
+  const uint64_t n = (8 * avail / (8 * sb + 1)) & ~(uint64_t)63;  // slot + 1 bit of occupancy bitmap
   return n < kSmemMaxSlots ? n : kSmemMaxSlots;
 }
 
@@ -1579,7 +1621,7 @@ extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
 template <typename Code, int R, int T, int C>
 static cudaError_t launch_smem_t(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes;
+  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes + a.slots / 8;  // + occupancy bitmap
   cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   if (e != cudaSuccess) return e;

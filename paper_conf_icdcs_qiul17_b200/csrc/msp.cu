@@ -29,6 +29,7 @@
 // reservation per partition per tile).
 #include <cub/block/block_scan.cuh>
 
+#include <algorithm>
 #include <cstdlib>
 
 #include "dbg_device.cuh"
@@ -39,6 +40,7 @@ namespace dbg {
 constexpr int kMspThreads = 128;
 constexpr int kMaxDesc = 40;             // descriptors per thread between flushes (>= 34)
 constexpr int kSmemHistMaxNp = 8192;
+constexpr int kTwoLevelBins = 512;  // level-1 bins of the two-level scatter
 
 struct MspArgs {
   const uint64_t* words;
@@ -142,23 +144,55 @@ __device__ __forceinline__ T in_reg(T v) {
   }
 }
 
-// Warp-collective flush of the per-thread descriptor lists: partition ids,
-// size histograms, one staging reservation per warp, record writes.
+// Records of a superkmer of n K-mers (pieces of at most nmax K-mers); the
+// common case n <= nmax needs no division.
+__device__ __forceinline__ uint32_t record_pieces(int n, int nmax) {
+  return n <= nmax ? 1u : (uint32_t)((n + nmax - 1) / nmax);
+}
+
+// Writes one record for K-mers [ps, pe] of the read at stream offset o, length
+// L, when it has 4 words (K <= 39): header + bases bs .. bs + 47, taken from
+// the three stream words that hold them (one bounds check each).
+__device__ __forceinline__ void write_record4(const MspArgs& a, uint32_t* dst, uint64_t o, int L, int ps, int pe,
+                                              uint32_t pid) {
+  const uint32_t hl = ps > 0 ? 1u : 0u;  // reading H
+  const uint32_t hr = pe + a.k < L ? 1u : 0u;
+  const int nb = (int)hl + (pe - ps + 1) + a.k - 1 + (int)hr;  // <= 48
+  const uint64_t pos = o + (uint64_t)(ps - (int)hl);
+  const uint64_t wi = pos >> 5;
+  const uint32_t sh = (uint32_t)(pos & 31) * 2;
+  const uint64_t x0 = wi < a.n_words ? __ldg(a.words + wi) : 0, x1 = wi + 1 < a.n_words ? __ldg(a.words + wi + 1) : 0;
+  const uint64_t x2 = sh > 32 && wi + 2 < a.n_words ? __ldg(a.words + wi + 2) : 0;
+  // bases 0..31 and 32..47 of the record (before masking)
+  const uint64_t v0 = sh ? (x0 << sh) | (x1 >> (64 - sh)) : x0;
+  const uint64_t v1 = sh ? (x1 << sh) | (x2 >> (64 - sh)) : x1;
+  const uint64_t m0 = nb >= 32 ? ~0ull : ~(~0ull >> (2 * nb));
+  const uint32_t m1 = nb >= 48 ? ~0u : (nb <= 32 ? 0u : ~(~0u >> (2 * (nb - 32))));
+  const uint64_t b0 = v0 & m0;
+  const uint32_t b1 = (uint32_t)(v1 >> 32) & m1;
+  reinterpret_cast<uint4*>(dst)[0] =
+      make_uint4((uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10), (uint32_t)(b0 >> 32), (uint32_t)b0, b1);
+}
+
+// Warp-collective flush of the per-thread descriptor lists: partition ids
+// (computed once per descriptor and kept in place of the minimizer), size
+// histograms, one staging reservation per warp, record writes.
 template <typename CT>
 __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
                                                   int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
   const int nmax = (int)a.max_kmers;
-  auto pid_of = [&](int d) -> uint32_t {
-    const uint64_t m = (uint64_t)sm.desc_m[d * kMspThreads + tid];
-    return a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
-  };
+  constexpr CT kSkip = ~(CT)0;  // a superkmer of another pass's partition (row f2)
   uint32_t my_records = 0;
   {
     int s = s_next;
     for (int d = 0; d < ndesc; ++d) {
       const int e = (int)sm.desc_e[d * kMspThreads + tid];
-      if (!a.ranged || (pid_of(d) - a.pid_lo < a.pid_hi - a.pid_lo)) my_records += (uint32_t)((e - s + nmax) / nmax);
+      CT& dm = sm.desc_m[d * kMspThreads + tid];
+      const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64((uint64_t)dm));
+      const bool in = !a.ranged || (pid - a.pid_lo < a.pid_hi - a.pid_lo);
+      dm = in ? (CT)pid : kSkip;
+      if (in) my_records += record_pieces(e - s + 1, nmax);
       s = e + 1;
     }
   }
@@ -178,18 +212,22 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
   int s = s_next;
   for (int d = 0; d < ndesc; ++d) {
     const int e = (int)sm.desc_e[d * kMspThreads + tid];
-    const uint32_t pid = pid_of(d);
-    if (a.ranged && pid - a.pid_lo >= a.pid_hi - a.pid_lo) {  // another pass's partition (row f2)
+    const CT dm = sm.desc_m[d * kMspThreads + tid];
+    if (dm == kSkip) {
       s = e + 1;
       continue;
     }
+    const uint32_t pid = (uint32_t)dm;
     const int n = e - s + 1;
-    const uint32_t pieces = (uint32_t)((n + nmax - 1) / nmax);
-    atomicAdd(a.n_records + pid, (unsigned long long)pieces);
+    atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
     for (int ps = s; ps <= e; ps += nmax, ++slot) {
-      if (slot < a.staging_cap)
-        write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
+      if (slot < a.staging_cap) {
+        if (a.rec_words == 4)
+          write_record4(a, a.staging + slot * 4, o, L, ps, min(e, ps + nmax - 1), pid);
+        else
+          write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
+      }
     }
     s = e + 1;
   }
@@ -288,7 +326,12 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   }
 }
 
-// Pass 3: scatter staged records into partition order.
+// Pass 3: scatter staged records into partition order.  A record's bin is
+// pid >> shift and its bin starts at record offset rec_off[bin << shift]
+// (shift = 0: one bin per partition; two-level scatter, level 1: bins of 2^shift
+// consecutive partitions, whose records are contiguous in partition order).
+// nb bins; with nb <= kSmemHistMaxNp a CTA tile ranks its records in shared
+// memory and reserves once per bin, else one global atomic per record.
 constexpr int kScatterThreads = 256;
 constexpr int kScatterPer = 8;  // records per thread per tile
 template <int R>
@@ -297,17 +340,17 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
                                                                   uint64_t staging_cap,
                                                                   const uint64_t* __restrict__ rec_off,
                                                                   unsigned long long* fill,
-                                                                  uint32_t* __restrict__ records, int np) {
-  extern __shared__ unsigned long long sh_base[];  // [np] global bases (per tile), then [np] counts
-  uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_base + np);
+                                                                  uint32_t* __restrict__ records, int nb, int shift) {
+  extern __shared__ unsigned long long sh_base[];  // [nb] global bases (per tile), then [nb] counts
+  uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_base + nb);
   const uint64_t n = *staged;
   if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
-  const bool smem = np <= kSmemHistMaxNp;
+  const bool smem = nb <= kSmemHistMaxNp;
   constexpr int kPer = R >= 16 ? 2 : kScatterPer;
   constexpr int kTile = kScatterThreads * kPer;
   for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile) {
     if (smem) {
-      for (int i = threadIdx.x; i < np; i += kScatterThreads) sh_cnt[i] = 0;
+      for (int i = threadIdx.x; i < nb; i += kScatterThreads) sh_cnt[i] = 0;
       __syncthreads();
     }
     uint4 rec[kPer][R / 4];
@@ -328,20 +371,20 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       rank[v] = 0;
       if (idx < n) {
-        const uint32_t pid = rec[v][0].x >> 10;
-        if (smem) rank[v] = atomicAdd(sh_cnt + pid, 1u);
-        else rank[v] = (uint32_t)atomicAdd(fill + pid, 1ull);
+        const uint32_t bin = (rec[v][0].x >> 10) >> shift;
+        if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
+        else rank[v] = (uint32_t)atomicAdd(fill + bin, 1ull);
       }
     }
     uint64_t base[kPer];
 #pragma unroll
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
-      base[v] = idx < n ? __ldg(rec_off + (rec[v][0].x >> 10)) : 0;
+      base[v] = idx < n ? __ldg(rec_off + (((rec[v][0].x >> 10) >> shift) << shift)) : 0;
     }
     if (smem) {
       __syncthreads();
-      for (int i = threadIdx.x; i < np; i += kScatterThreads)
+      for (int i = threadIdx.x; i < nb; i += kScatterThreads)
         if (sh_cnt[i]) sh_base[i] = atomicAdd(fill + i, (unsigned long long)sh_cnt[i]);
       __syncthreads();
     }
@@ -349,14 +392,68 @@ __global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       if (idx < n) {
-        const uint32_t pid = rec[v][0].x >> 10;
-        const uint64_t pos = base[v] + (smem ? sh_base[pid] + rank[v] : rank[v]);
+        const uint32_t bin = (rec[v][0].x >> 10) >> shift;
+        const uint64_t pos = base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
         uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
 #pragma unroll
         for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];
       }
     }
     if (smem) __syncthreads();
+  }
+}
+
+// Two-level scatter, level 2: one CTA per bucket of 2^shift consecutive
+// partitions (grid-stride over buckets).  The bucket's records are
+// contiguous in src (level 1); each is ranked inside its partition with a
+// shared-memory atomic and written to rec_off[pid] + rank in dst.  The
+// bucket's partition offsets are staged in shared memory.
+constexpr int kBucketThreads = 512;
+constexpr int kBucketPer = 4;
+template <int R>
+__global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const uint32_t* __restrict__ src,
+                                                                        const unsigned long long* staged,
+                                                                        uint64_t staging_cap,
+                                                                        const uint64_t* __restrict__ rec_off,
+                                                                        uint32_t* __restrict__ dst, int np, int shift) {
+  extern __shared__ unsigned long long sh_off[];  // [2^shift + 1] offsets, then [2^shift] counts
+  const int bw = 1 << shift;
+  uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_off + bw + 1);
+  if (*staged > staging_cap) return;
+  const int nbk = (np + bw - 1) >> shift;
+  constexpr int kTile = kBucketThreads * kBucketPer;
+  for (int bk = blockIdx.x; bk < nbk; bk += gridDim.x) {
+    const int p0 = bk << shift, np_b = min(bw, np - p0);
+    for (int i = threadIdx.x; i <= np_b; i += kBucketThreads) {
+      sh_off[i] = rec_off[p0 + i];
+      if (i < np_b) sh_cnt[i] = 0;
+    }
+    __syncthreads();
+    const uint64_t r0 = sh_off[0], r1 = sh_off[np_b];
+    for (uint64_t t0 = r0; t0 < r1; t0 += kTile) {
+      uint4 rec[kBucketPer][R / 4];
+#pragma unroll
+      for (int v = 0; v < kBucketPer; ++v) {
+        const uint64_t idx = t0 + v * kBucketThreads + threadIdx.x;
+        if (idx < r1) {
+          const uint4* s4 = reinterpret_cast<const uint4*>(src + idx * R);
+#pragma unroll
+          for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(s4 + c);
+        }
+      }
+#pragma unroll
+      for (int v = 0; v < kBucketPer; ++v) {
+        const uint64_t idx = t0 + v * kBucketThreads + threadIdx.x;
+        if (idx < r1) {
+          const uint32_t lp = (rec[v][0].x >> 10) - (uint32_t)p0;
+          const uint64_t pos = sh_off[lp] + atomicAdd(sh_cnt + lp, 1u);
+          uint4* d4 = reinterpret_cast<uint4*>(dst + pos * R);
+#pragma unroll
+          for (int c = 0; c < R / 4; ++c) d4[c] = rec[v][c];
+        }
+      }
+    }
+    __syncthreads();
   }
 }
 
@@ -592,25 +689,41 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
   } else {
     // pass 3: scatter (a no-op after a staging overflow, *d_staged > staging_cap)
     if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
-    if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * np, stream) != cudaSuccess) return DBG_ECUDA;
-    const size_t smem = np <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * np : 0;
+    if (part->d_scratch && (part->d_scratch == part->d_staging || part->d_scratch == part->d_records))
+      return DBG_EINVAL;
+    const bool two = part->d_scratch && np > kSmemHistMaxNp;
+    int shift = 0;
+    // level 1 into at most 512 bins, so that a tile of 2048 records ranks several records per
+    // bin in shared memory and reserves once per bin
+    while (two && ((np + (1 << shift) - 1) >> shift) > kTwoLevelBins) ++shift;
+    const int nb = (np + (1 << shift) - 1) >> shift;
+    if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) return DBG_ECUDA;
+    const size_t smem = nb <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * nb : 0;
     const int grid = dbg_sm_count() * 4;
+    uint32_t* lvl1 = two ? part->d_scratch : part->d_records;
+    const unsigned long long* staged = reinterpret_cast<const unsigned long long*>(part->d_staged);
+    unsigned long long* fill = reinterpret_cast<unsigned long long*>(part->d_fill);
+    const size_t smem2 = (sizeof(unsigned long long) * ((1u << shift) + 1) + sizeof(uint32_t) * (1u << shift));
+    const int grid2 = (int)std::min<int64_t>((int64_t)nb, (int64_t)dbg_sm_count() * 4);
+#define DBG_SCATTER(RW)                                                                                         \
+  cudaFuncSetAttribute(scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
+  scatter_kernel<RW><<<grid, kScatterThreads, smem, stream>>>(part->d_staging, staged, part->staging_cap,       \
+                                                              part->d_record_offset, fill, lvl1, nb, shift);    \
+  if (two) {                                                                                                    \
+    cudaFuncSetAttribute(bucket_scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);   \
+    bucket_scatter_kernel<RW><<<grid2, kBucketThreads, smem2, stream>>>(part->d_scratch, staged,               \
+                                                                        part->staging_cap,                     \
+                                                                        part->d_record_offset,                 \
+                                                                        part->d_records, np, shift);           \
+  }
     if (R == 4) {
-      cudaFuncSetAttribute(scatter_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      scatter_kernel<4><<<grid, kScatterThreads, smem, stream>>>(
-          part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
-          part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
+      DBG_SCATTER(4)
     } else if (R == 8) {
-      cudaFuncSetAttribute(scatter_kernel<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      scatter_kernel<8><<<grid, kScatterThreads, smem, stream>>>(
-          part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
-          part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
+      DBG_SCATTER(8)
     } else {
-      cudaFuncSetAttribute(scatter_kernel<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      scatter_kernel<16><<<grid, kScatterThreads, smem, stream>>>(
-          part->d_staging, reinterpret_cast<const unsigned long long*>(part->d_staged), part->staging_cap,
-          part->d_record_offset, reinterpret_cast<unsigned long long*>(part->d_fill), part->d_records, np);
+      DBG_SCATTER(16)
     }
+#undef DBG_SCATTER
   }
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }

@@ -24,6 +24,8 @@ from __future__ import annotations
 
 from dataclasses import dataclass, field
 
+import os
+
 import numpy as np
 import torch
 
@@ -113,6 +115,9 @@ class DbgBuilder:
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
         self.records = torch.empty(0, dtype=torch.int32, device=dev)
+        # two-level scatter (pass 2) above 8192 fine partitions: a third record buffer
+        self.scratch = torch.empty(0, dtype=torch.int32, device=dev)
+        self.two_level = NP > 8192 and os.environ.get("DBG_SCATTER_ONE_LEVEL") is None
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
         self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
         self.work = torch.empty(0, dtype=torch.uint8, device=dev)
@@ -162,9 +167,13 @@ class DbgBuilder:
 
     # ------------------------------------------------------------------ a2-a4
     def part_set(self, with_records: bool) -> _lib.dbg_partition_set:
+        scratch = None
+        if with_records and self.two_level:
+            self.scratch = _grow(self.scratch, self.records.numel(), torch.int32, self.device)
+            scratch = self.scratch
         return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill, self.d_staged,
                                   self.staging, self.staging.numel() // self.rec_words,
-                                  self.records if with_records else None)
+                                  self.records if with_records else None, scratch)
 
     def _staging_estimate(self, n_kmers_upper: int, n_reads: int) -> int:
         w = self.k - self.p + 1

@@ -436,3 +436,38 @@ def test_register_blocked_msp_variants(p):
     got = occurrences_from_records(decode_records(words, b.rec_words, 31), 31)
     sk = oracle.msp(rs.seq, rs.offsets, 31, p, 13)
     assert got == occurrences_from_oracle_msp(sk, rs.reads(), 31)
+
+
+@pytest.mark.parametrize("refine", [1024, 4096, 40000])
+def test_two_level_scatter_partition_order(refine, monkeypatch):
+    """More than 8192 fine partitions: pass 2 scatters through d_scratch in two levels (buckets of
+    2^s consecutive partitions, then within each bucket).  Every record must land in its own
+    partition's range [rec_off[p], rec_off[p+1]), the per-partition record multisets must equal the
+    one-level scatter's, and the graph must equal the oracle's."""
+    rs = ReadSet(*make_reads(genome(60_000, 5), 6000, 100, 0.01, 105))
+    np_ = 16
+    _check(rs, 31, 11, np_, refine=refine)
+
+    def records(two):
+        if not two:
+            monkeypatch.setenv("DBG_SCATTER_ONE_LEVEL", "1")
+        else:
+            monkeypatch.delenv("DBG_SCATTER_ONE_LEVEL", raising=False)
+        b = DbgBuilder(31, 11, np_, refine=refine)
+        assert b.two_level == two
+        d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+        b.msp(d_bases, d_off)
+        assert b.sync_sizes()
+        torch.cuda.synchronize()
+        n = int(b.part_records.sum())
+        w = b.records[:n * b.rec_words].cpu().numpy().view(np.uint32).reshape(n, b.rec_words)
+        off = np.concatenate([[0], np.cumsum(b.part_records)])
+        pid = w[:, 0] >> 10
+        assert np.array_equal(pid, np.repeat(np.arange(len(b.part_records)), b.part_records))
+        rows = [tuple(r) for r in w]
+        return off, sorted(rows)
+
+    off2, rows2 = records(True)
+    off1, rows1 = records(False)
+    assert np.array_equal(off1, off2)
+    assert rows1 == rows2
