@@ -14,7 +14,8 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "lib", "libdbg.so")
+# DBG_LIB_PATH: an A/B kernel-variant build (tools/build_variants.py); default: the in-tree build
+LIB_PATH = os.environ.get("DBG_LIB_PATH") or os.path.join(_PKG, "lib", "libdbg.so")
 
 DBG_OK, DBG_EINVAL, DBG_ENOSPACE, DBG_ETABLEFULL, DBG_ECUDA = range(5)
 

@@ -47,6 +47,17 @@
 #include "dbg_device.cuh"
 #include "scan.cuh"
 
+// Kernel variants (A/B builds: tools/build_variants.py); the defaults are the measured winners.
+#ifndef DBG_WORDSEL
+#define DBG_WORDSEL 1
+#endif
+#ifndef DBG_PROBE_PRED
+#define DBG_PROBE_PRED 1
+#endif
+#ifndef DBG_BITMAP
+#define DBG_BITMAP 0
+#endif
+
 int dbg_sm_count();
 bool dbg_params_ok(const dbg_params* prm);
 // row f3 (wide.cu): K > 63 in the resident tables, with the locked-state protocol
@@ -1024,6 +1035,58 @@ __global__ void __launch_bounds__(kTileThreads) smem_plan_apply_kernel(SmemArgs 
   }
 }
 
+// C': greedy packing (replaces C's group-start flags and their tile counts):
+// inside each run of kGroupParts consecutive partitions, partitions are packed
+// in order into groups while their grouped capacities fit one CTA table
+// (span <= slots), so a group fills the table instead of one H-window of it;
+// a split or global partition (capacity, nothing grouped) stays alone with
+// span 0, as does an empty run.  One CTA per scan tile: the tile's N^i_kmer go
+// to shared memory, then one thread per run packs it sequentially.
+constexpr int kRunsPerTile = kTileSize / kGroupParts;
+static_assert(kTileSize % kGroupParts == 0, "a scan tile holds whole group runs");
+__global__ void __launch_bounds__(kTileThreads) smem_plan_pack_kernel(SmemArgs a) {
+  typedef cub::BlockReduce<unsigned int, kTileThreads> Red;
+  __shared__ uint32_t gc[kTileSize];  // grouped capacity; ~0u: alone (split or global)
+  __shared__ uint8_t fl[kTileSize];
+  __shared__ typename Red::TempStorage tmp;
+  const int base = blockIdx.x * kTileSize;
+  for (int q = threadIdx.x; q < kTileSize; q += kTileThreads) {
+    const int p = base + q;
+    uint32_t v = 0;
+    if (p < a.n_fine) {
+      const OnChip o = on_chip(a, a.n_kmers[a.pid0 + p]);
+      v = o.gc ? (uint32_t)o.gc : (o.cap ? ~0u : 0u);
+    }
+    gc[q] = v;
+  }
+  __syncthreads();
+  if (threadIdx.x < kRunsPerTile) {
+    const int q0 = threadIdx.x * kGroupParts;
+    uint64_t acc = 0;
+    bool prev_alone = true;
+    for (int q = q0; q < q0 + kGroupParts; ++q) {
+      const uint32_t v = gc[q];
+      const bool alone = v == ~0u;
+      const uint32_t c = alone ? 0u : v;
+      const bool f = q == q0 || alone || prev_alone || acc + c > a.slots;
+      acc = f ? c : acc + c;
+      prev_alone = alone;
+      fl[q] = f;
+    }
+  }
+  __syncthreads();
+  unsigned int nflag = 0;
+  for (int q = threadIdx.x; q < kTileSize; q += kTileThreads) {
+    const int p = base + q;
+    if (p < a.n_fine) {
+      a.flag[p] = fl[q];
+      nflag += fl[q];
+    }
+  }
+  nflag = Red(tmp).Sum(nflag);
+  if (threadIdx.x == 0) a.t_fl[blockIdx.x] = nflag;
+}
+
 __global__ void __launch_bounds__(kTileThreads) smem_plan_groups_kernel(SmemArgs a) {
   typedef cub::BlockScan<unsigned int, kTileThreads> Scan;
   __shared__ typename Scan::TempStorage tmp;
@@ -1131,7 +1194,8 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
     uint4* z = reinterpret_cast<uint4*>(keys);
     for (uint64_t q = threadIdx.x; q < a.slots * SmemSlot<KW>::kBytes / 16; q += kSmemThreads)
       z[q] = make_uint4(0, 0, 0, 0);
-    for (uint64_t q = threadIdx.x; q < a.slots / 32; q += kSmemThreads) occ[q] = 0;
+    if (DBG_BITMAP)
+      for (uint64_t q = threadIdx.x; q < a.slots / 32; q += kSmemThreads) occ[q] = 0;
   }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
@@ -1260,6 +1324,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         Code fwd, rc;
         int pred, succ;
         if constexpr (R == 4) {
+#if DBG_WORDSEL
           // the three data words, loaded unconditionally and selected (no branches): a1..a3
           // hold bases b .. b + 47 - 16q
           const uint32_t d1 = w[S], d2 = w[2 * S], d3 = w[3 * S];
@@ -1269,6 +1334,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           const int pb = b - 1, pq = pb >> 4;  // the predecessor base
           const uint32_t pw = pq <= 0 ? d1 : (pq == 1 ? d2 : d3);
           pred = b > 0 ? (int)((pw >> (30 - 2 * (pb & 15))) & 3u) : -1;
+#else
+          const int q = b >> 4;  // the words holding bases b .. b + 47 - 16q
+          const uint32_t a1 = w[(1 + q) * S], a2 = q < 2 ? w[(2 + q) * S] : 0u, a3 = q == 0 ? w[3 * S] : 0u;
+          const int pb = b - 1;  // the predecessor base
+          pred = b > 0 ? (int)((w[(1 + (pb >> 4)) * S] >> (30 - 2 * (pb & 15))) & 3u) : -1;
+#endif
           if constexpr (sizeof(Code) == 8) {
             // 64 bits of the record from base b: two 32-bit funnel shifts
             const uint32_t sh = 2 * (b & 15);
@@ -1301,6 +1372,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         uint32_t idx = __umulhi(smem_hash(code), cap);
         uint32_t inserted = 0;
         const uint32_t kaddr = keys_s + t0 * KB;
+#if DBG_PROBE_PRED
         if constexpr (KW == 1) {
           // every lane runs every probe round (predicated, no divergent branch): a lane with
           // nothing pending re-reads its current slot and keeps its state
@@ -1323,6 +1395,28 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             const uint64_t cur = lds64(kaddr + idx * KB);
             if (cur != key) idx = ~0u;  // this occurrence found no slot
           }
+#else
+        if constexpr (KW == 1) {
+          uint32_t probes = 0, pend = want;
+          while (__any_sync(kFull, pend)) {
+            if (pend) {
+              const uint32_t ka = kaddr + idx * KB;
+              uint64_t cur = lds64(ka);
+              if (cur == 0) cur = cas_shared64(ka, key);
+              inserted = cur == 0;
+              if (inserted | (cur == key)) {
+                pend = 0;
+              } else {
+                idx = idx + 1 == cap ? 0 : idx + 1;
+                if (++probes == cap) {  // wrapped: table full (reading O)
+                  pend = 0;
+                  ok = false;
+                  idx = ~0u;
+                }
+              }
+            }
+          }
+#endif
         } else {
           uint32_t probes = 0, pend = want;
           while (__any_sync(kFull, pend)) {
@@ -1346,7 +1440,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           const uint32_t fa = fld_s + (t0 + idx) * (FW * 4);
           if (inserted) {
             sts32(fa + 20, w[0] >> 10);
-            red_shared_or(occ_s + 4 * ((t0 + idx) >> 5), 1u << ((t0 + idx) & 31u));
+            if (DBG_BITMAP) red_shared_or(occ_s + 4 * ((t0 + idx) >> 5), 1u << ((t0 + idx) & 31u));
           }
           const int fo = o < 4 ? o : 8;
           red_shared_add(fa + 4 * (fo >> 1), 1u << (16 * (fo & 1)));
@@ -1370,7 +1464,11 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         uint32_t qn = 0;
         for (uint32_t c = sub; c < se; c += 32) {
           const uint32_t s = c + lane;
+#if DBG_BITMAP
           bool keep = ((se - c >= 32 ? occ[c >> 5] : occ[c >> 5] & ((1u << (se - c)) - 1u)) >> lane) & 1u;
+#else
+          bool keep = s < se && (lds64(keys_s + s * KB) & kOccupied);
+#endif
           if (keep && oa.min_count > 1) {  // row f4: a low-count vertex is cleaned, never emitted
             const uint32_t* f = fld + s * FW;
             const uint32_t f0 = f[0], f1 = f[1];
@@ -1388,7 +1486,8 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           if (keep) queue[qn + __popc(bal & ((1u << lane) - 1u))] = (uint16_t)s;
           qn += __popc(bal);
         }
-        for (uint32_t c = (sub >> 5) + lane; c < (se + 31) >> 5; c += 32) occ[c] = 0;
+        if (DBG_BITMAP)
+          for (uint32_t c = (sub >> 5) + lane; c < (se + 31) >> 5; c += 32) occ[c] = 0;
         unsigned long long pos = 0;
         if (lane == 0 && qn) pos = atomicAdd(oa.n_out, (unsigned long long)qn);
         pos = __shfl_sync(kFull, pos, 0);
@@ -1599,7 +1698,7 @@ template <int R, int T>
 static uint64_t smem_slots_for(int k, int ctas) {
   const uint64_t avail = (227u * 1024u) / ctas - smem_fixed_bytes<R, T>() - 1024u;
   const uint32_t sb = k <= 31 ? SmemSlot<1>::kBytes : SmemSlot<2>::kBytes;
-  const uint64_t n = (8 * avail / (8 * sb + 1)) & ~(uint64_t)63;  // slot + 1 bit of occupancy bitmap
+  const uint64_t n = (8 * avail / (8 * sb + (DBG_BITMAP ? 1 : 0))) & ~(uint64_t)63;  // (+ 1 bit of bitmap)
   return n < kSmemMaxSlots ? n : kSmemMaxSlots;
 }
 
@@ -1621,7 +1720,7 @@ extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
 template <typename Code, int R, int T, int C>
 static cudaError_t launch_smem_t(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes + a.slots / 8;  // + occupancy bitmap
+  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes + (DBG_BITMAP ? a.slots / 8 : 0);
   cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   if (e != cudaSuccess) return e;
@@ -1716,6 +1815,7 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_gc, tiles);
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_sp, tiles);
   smem_plan_apply_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
+  if (!getenv("DBG_GROUPS_WINDOW")) smem_plan_pack_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_fl, tiles);
   smem_plan_groups_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
   smem_plan_desc_kernel<<<(a.n_fine + 255) / 256 < dbg_sm_count() * 8 ? (a.n_fine + 255) / 256 : dbg_sm_count() * 8,

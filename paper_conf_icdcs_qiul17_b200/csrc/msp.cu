@@ -39,6 +39,8 @@ namespace dbg {
 
 constexpr int kMspThreads = 128;
 constexpr int kMaxDesc = 40;             // descriptors per thread between flushes (>= 34)
+constexpr int kMaxDescBlock = 32;        // msp_block_kernel (>= W + 3)
+constexpr int kMspBlockCtas = 7;         // resident CTAs per SM (registers <= 73, 32 KB shared memory each)
 constexpr int kSmemHistMaxNp = 8192;
 constexpr int kTwoLevelBins = 512;  // level-1 bins of the two-level scatter
 
@@ -466,14 +468,14 @@ __global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const ui
 // current block holds P-mers q0 .. q0+W-1.  Same descriptors and flush as
 // msp_kernel; reads of any length (lanes past their read end run masked).
 template <int W, int P>
-__global__ void __launch_bounds__(kMspThreads) msp_block_kernel(MspArgs a) {
+__global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(MspArgs a) {
   typedef uint32_t CT;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int tid = threadIdx.x, lane = tid & 31;
   MspSmem<CT> sm;
   unsigned char* sp = smem_raw;
   sm.desc_m = reinterpret_cast<CT*>(sp);
-  sp += sizeof(CT) * kMaxDesc * kMspThreads;
+  sp += sizeof(CT) * kMaxDescBlock * kMspThreads;
   sm.desc_e = reinterpret_cast<uint32_t*>(sp);
   sm.row = nullptr;
   constexpr CT kMaskP = (CT)((2 * P == 32) ? ~0u : ((1u << (2 * P)) - 1));
@@ -519,14 +521,33 @@ __global__ void __launch_bounds__(kMspThreads) msp_block_kernel(MspArgs a) {
       f = ((f << 2) | b) & kMaskP;
       rc = (rc >> 2) | ((CT)(3u - b) << kTopP);
     }
-    CT suf[W];
+    CT suf[W];  // suffix minima of the previous block
 #pragma unroll
     for (int t = 0; t < W; ++t) suf[t] = kInf;
-    // blocks of W P-mers; one extra block of padding emits the last K-mers
+    // blocks of W P-mers; one extra block of padding emits the last K-mers.  K-mer
+    // i = q0 - W + t is complete once P-mer q0 + t - 1 is read: its minimizer is
+    // min(suf[t], prefix minimum of the current block's first t values) -- the
+    // prefix is a running scalar, the block's values are kept for its suffix minima.
     for (int q0 = 0; q0 < nPmax + W; q0 += W) {
-      CT c[W], pre[W];
+      CT c[W];
+      CT pre = kInf;
 #pragma unroll
       for (int t = 0; t < W; ++t) {
+        const int i = q0 - W + t;
+        if (q0 >= W && i < nk) {
+          const CT m = suf[t] < pre ? suf[t] : pre;
+          if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
+            sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(i - 1));
+            sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+            ++ndesc;
+          }
+          m_cur = m;
+          if (i == nk - 1) {  // the read's last superkmer
+            sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
+            sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+            ++ndesc;
+          }
+        }
         CT v = kInf;
         if (q0 + t < nP) {
           const uint32_t b = next_base();
@@ -535,32 +556,12 @@ __global__ void __launch_bounds__(kMspThreads) msp_block_kernel(MspArgs a) {
           v = f < rc ? f : rc;  // canonical P-mer (reading D)
         }
         c[t] = v;
-        pre[t] = t == 0 ? v : (v < pre[t - 1] ? v : pre[t - 1]);
-      }
-      if (q0 >= W) {  // K-mers i = q0 - W + t of the previous block's windows
-#pragma unroll
-        for (int t = 0; t < W; ++t) {
-          const int i = q0 - W + t;
-          if (i < nk) {
-            const CT m = t == 0 ? suf[0] : (suf[t] < pre[t - 1] ? suf[t] : pre[t - 1]);
-            if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
-              sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(i - 1));
-              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
-              ++ndesc;
-            }
-            m_cur = m;
-            if (i == nk - 1) {  // the read's last superkmer
-              sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
-              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
-              ++ndesc;
-            }
-          }
-        }
+        pre = v < pre ? v : pre;
       }
       suf[W - 1] = c[W - 1];
 #pragma unroll
       for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
-      if (__any_sync(kFull, ndesc > kMaxDesc - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+      if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
     }
     if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
   }
@@ -587,7 +588,7 @@ bool dbg_params_ok(const dbg_params* prm) {
 
 template <int W, int P>
 static cudaError_t launch_msp_block(const MspArgs& a, int grid, cudaStream_t stream) {
-  const size_t smem = (sizeof(uint32_t) + sizeof(uint32_t)) * kMaxDesc * kMspThreads;
+  const size_t smem = (sizeof(uint32_t) + sizeof(uint32_t)) * kMaxDescBlock * kMspThreads;
   cudaError_t e = cudaFuncSetAttribute(msp_block_kernel<W, P>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   msp_block_kernel<W, P><<<grid, kMspThreads, smem, stream>>>(a);

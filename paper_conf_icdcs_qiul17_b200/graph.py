@@ -115,9 +115,11 @@ class DbgBuilder:
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
         self.records = torch.empty(0, dtype=torch.int32, device=dev)
-        # two-level scatter (pass 2) above 8192 fine partitions: a third record buffer
+        # two-level scatter (pass 2) above 8192 fine partitions through a third record buffer:
+        # opt-in (DBG_SCATTER_TWO_LEVEL=1) -- measured slower than one level with global rank
+        # atomics on E. coli and chr14 (profiles/r01d_ab.txt)
         self.scratch = torch.empty(0, dtype=torch.int32, device=dev)
-        self.two_level = NP > 8192 and os.environ.get("DBG_SCATTER_ONE_LEVEL") is None
+        self.two_level = NP > 8192 and os.environ.get("DBG_SCATTER_TWO_LEVEL") == "1"
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
         self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
         self.work = torch.empty(0, dtype=torch.uint8, device=dev)

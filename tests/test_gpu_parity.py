@@ -446,13 +446,14 @@ def test_two_level_scatter_partition_order(refine, monkeypatch):
     one-level scatter's, and the graph must equal the oracle's."""
     rs = ReadSet(*make_reads(genome(60_000, 5), 6000, 100, 0.01, 105))
     np_ = 16
+    monkeypatch.setenv("DBG_SCATTER_TWO_LEVEL", "1")
     _check(rs, 31, 11, np_, refine=refine)
 
     def records(two):
-        if not two:
-            monkeypatch.setenv("DBG_SCATTER_ONE_LEVEL", "1")
+        if two:
+            monkeypatch.setenv("DBG_SCATTER_TWO_LEVEL", "1")
         else:
-            monkeypatch.delenv("DBG_SCATTER_ONE_LEVEL", raising=False)
+            monkeypatch.delenv("DBG_SCATTER_TWO_LEVEL", raising=False)
         b = DbgBuilder(31, 11, np_, refine=refine)
         assert b.two_level == two
         d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
