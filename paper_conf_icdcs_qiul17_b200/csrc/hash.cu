@@ -54,6 +54,12 @@
 #ifndef DBG_PROBE_PRED
 #define DBG_PROBE_PRED 1
 #endif
+#ifndef DBG_SLOT28
+#define DBG_SLOT28 1
+#endif
+#ifndef DBG_RB4
+#define DBG_RB4 1024  // records of 4 words per on-chip batch (T >= 512)
+#endif
 #ifndef DBG_BITMAP
 #define DBG_BITMAP 0
 #endif
@@ -797,7 +803,7 @@ constexpr uint64_t kSmemMaxSlots = 65535;
 template <int KW>
 struct SmemSlot {
   static constexpr uint32_t kKeyBytes = KW == 1 ? 8 : 16;
-  static constexpr uint32_t kFieldWords = 6;
+  static constexpr uint32_t kFieldWords = DBG_SLOT28 ? 5 : 6;  // (DBG_SLOT28: no fine-pid field)
   static constexpr uint32_t kBytes = kKeyBytes + 4 * kFieldWords;
 };
 
@@ -817,7 +823,7 @@ constexpr int kGroupParts = 256;  // partitions per group at most (plan rule)
 // Records per batch: 1024 four-word or 512 eight-word records (16 KB) from 512
 // threads up; fewer for smaller CTAs.
 template <int R, int T>
-__host__ __device__ constexpr int smem_rec_batch() { return (T >= 512 ? 1024 : 2 * T) * 4 / R; }
+__host__ __device__ constexpr int smem_rec_batch() { return (T >= 512 ? DBG_RB4 : 2 * T) * 4 / R; }
 
 template <int R, int T>
 struct SmemStage {
@@ -1439,7 +1445,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         if (want && idx != ~0u) {  // the multiple updates: 16-bit fields, two per word
           const uint32_t fa = fld_s + (t0 + idx) * (FW * 4);
           if (inserted) {
-            sts32(fa + 20, w[0] >> 10);
+            if (!DBG_SLOT28) sts32(fa + 20, w[0] >> 10);
             if (DBG_BITMAP) red_shared_or(occ_s + 4 * ((t0 + idx) >> 5), 1u << ((t0 + idx) & 31u));
           }
           const int fo = o < 4 ? o : 8;
@@ -1510,7 +1516,22 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
           v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
           // fine pid recorded by the inserting thread, mod NP (or from the P-minimizer, reading V)
-          v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, f[5]);
+          uint32_t fpid;
+          if (DBG_SLOT28) {  // the fine partition owning slot s: last x with Pq[x] - P0 <= s
+            fpid = I.first;
+            if (sub_n == 1) {
+              uint32_t lo = 0, n = I.last - I.first;
+              while (n > 1) {
+                const uint32_t h = n >> 1;
+                if (Pq[lo + h] - I.P0 <= s) lo += h, n -= h;
+                else n = h;
+              }
+              fpid += lo;
+            }
+          } else {
+            fpid = f[FW - 1];
+          }
+          v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, fpid);
           kp[0] = 0;  // clean-on-extract
           if (KW == 2) kp[1] = 0;
 #pragma unroll

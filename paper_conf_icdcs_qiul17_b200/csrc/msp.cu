@@ -39,8 +39,18 @@ namespace dbg {
 
 constexpr int kMspThreads = 128;
 constexpr int kMaxDesc = 40;             // descriptors per thread between flushes (>= 34)
-constexpr int kMaxDescBlock = 32;        // msp_block_kernel (>= W + 3)
-constexpr int kMspBlockCtas = 7;         // resident CTAs per SM (registers <= 73, 32 KB shared memory each)
+// msp_block_kernel variants (A/B builds, tools/build_variants.py)
+#ifndef DBG_MSP_FUSED
+#define DBG_MSP_FUSED 0   // 1: running prefix minimum interleaved with the K-mer emission
+#endif
+#ifndef DBG_MSP_DESC
+#define DBG_MSP_DESC 40   // descriptors per thread between flushes (>= W + 3)
+#endif
+#ifndef DBG_MSP_CTAS
+#define DBG_MSP_CTAS 1    // __launch_bounds__ min CTAs per SM (1: no register cap)
+#endif
+constexpr int kMaxDescBlock = DBG_MSP_DESC;
+constexpr int kMspBlockCtas = DBG_MSP_CTAS;
 constexpr int kSmemHistMaxNp = 8192;
 constexpr int kTwoLevelBins = 512;  // level-1 bins of the two-level scatter
 
@@ -334,10 +344,19 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 // consecutive partitions, whose records are contiguous in partition order).
 // nb bins; with nb <= kSmemHistMaxNp a CTA tile ranks its records in shared
 // memory and reserves once per bin, else one global atomic per record.
+#ifndef DBG_SCATTER_PER
+#define DBG_SCATTER_PER 8
+#endif
+#ifndef DBG_SCATTER_GRID
+#define DBG_SCATTER_GRID 0  // CTAs per SM (0: the occupancy limit)
+#endif
+#ifndef DBG_SCATTER_MINB
+#define DBG_SCATTER_MINB 1
+#endif
 constexpr int kScatterThreads = 256;
-constexpr int kScatterPer = 8;  // records per thread per tile
+constexpr int kScatterPer = DBG_SCATTER_PER;  // records per thread per tile
 template <int R>
-__global__ void __launch_bounds__(kScatterThreads) scatter_kernel(const uint32_t* __restrict__ staging,
+__global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_kernel(const uint32_t* __restrict__ staging,
                                                                   const unsigned long long* staged,
                                                                   uint64_t staging_cap,
                                                                   const uint64_t* __restrict__ rec_off,
@@ -528,6 +547,7 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
     // i = q0 - W + t is complete once P-mer q0 + t - 1 is read: its minimizer is
     // min(suf[t], prefix minimum of the current block's first t values) -- the
     // prefix is a running scalar, the block's values are kept for its suffix minima.
+#if DBG_MSP_FUSED
     for (int q0 = 0; q0 < nPmax + W; q0 += W) {
       CT c[W];
       CT pre = kInf;
@@ -563,6 +583,47 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
       for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
       if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
     }
+#else
+    for (int q0 = 0; q0 < nPmax + W; q0 += W) {
+      CT c[W], pre[W];
+#pragma unroll
+      for (int t = 0; t < W; ++t) {
+        CT v = kInf;
+        if (q0 + t < nP) {
+          const uint32_t b = next_base();
+          f = ((f << 2) | b) & kMaskP;
+          rc = (rc >> 2) | ((CT)(3u - b) << kTopP);
+          v = f < rc ? f : rc;  // canonical P-mer (reading D)
+        }
+        c[t] = v;
+        pre[t] = t == 0 ? v : (v < pre[t - 1] ? v : pre[t - 1]);
+      }
+      if (q0 >= W) {  // K-mers i = q0 - W + t of the previous block's windows
+#pragma unroll
+        for (int t = 0; t < W; ++t) {
+          const int i = q0 - W + t;
+          if (i < nk) {
+            const CT m = t == 0 ? suf[0] : (suf[t] < pre[t - 1] ? suf[t] : pre[t - 1]);
+            if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
+              sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(i - 1));
+              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+              ++ndesc;
+            }
+            m_cur = m;
+            if (i == nk - 1) {  // the read's last superkmer
+              sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
+              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+              ++ndesc;
+            }
+          }
+        }
+      }
+      suf[W - 1] = c[W - 1];
+#pragma unroll
+      for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
+      if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+    }
+#endif
     if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
   }
 }
@@ -700,7 +761,15 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     const int nb = (np + (1 << shift) - 1) >> shift;
     if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) return DBG_ECUDA;
     const size_t smem = nb <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * nb : 0;
-    const int grid = dbg_sm_count() * 4;
+    // one full wave: the kernel is grid-stride, a partial second wave would idle SMs
+    auto scatter_grid = [&](const void* fn) {
+      int per_sm = 0;
+      if (DBG_SCATTER_GRID > 0 ||
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kScatterThreads, smem) != cudaSuccess ||
+          per_sm < 1)
+        per_sm = DBG_SCATTER_GRID > 0 ? DBG_SCATTER_GRID : 4;
+      return dbg_sm_count() * per_sm;
+    };
     uint32_t* lvl1 = two ? part->d_scratch : part->d_records;
     const unsigned long long* staged = reinterpret_cast<const unsigned long long*>(part->d_staged);
     unsigned long long* fill = reinterpret_cast<unsigned long long*>(part->d_fill);
@@ -708,7 +777,7 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     const int grid2 = (int)std::min<int64_t>((int64_t)nb, (int64_t)dbg_sm_count() * 4);
 #define DBG_SCATTER(RW)                                                                                         \
   cudaFuncSetAttribute(scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
-  scatter_kernel<RW><<<grid, kScatterThreads, smem, stream>>>(part->d_staging, staged, part->staging_cap,       \
+  scatter_kernel<RW><<<scatter_grid((const void*)scatter_kernel<RW>), kScatterThreads, smem, stream>>>(part->d_staging, staged, part->staging_cap,       \
                                                               part->d_record_offset, fill, lvl1, nb, shift);    \
   if (two) {                                                                                                    \
     cudaFuncSetAttribute(bucket_scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);   \
