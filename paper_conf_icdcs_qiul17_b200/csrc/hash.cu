@@ -54,6 +54,9 @@
 #ifndef DBG_PROBE_PRED
 #define DBG_PROBE_PRED 1
 #endif
+#ifndef DBG_BUCKET2
+#define DBG_BUCKET2 0
+#endif
 #ifndef DBG_SLOT28
 #define DBG_SLOT28 1
 #endif
@@ -936,7 +939,7 @@ __device__ __forceinline__ OnChip on_chip(const SmemArgs& a, uint64_t nk) {
   OnChip o;
   o.cap = table_capacity(a.ratio, nk);
   const uint32_t t = onchip_tables(nk, o.cap, a.slots, a.max_split);
-  o.gc = t == 1 ? o.cap : 0;
+  o.gc = t == 1 ? (DBG_BUCKET2 ? (o.cap + 1) & ~1ull : o.cap) : 0;  // (DBG_BUCKET2: even, 16-B aligned pairs)
   o.ns = t >= 2 ? t : 0;
   return o;
 }
@@ -1378,7 +1381,37 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         uint32_t idx = __umulhi(smem_hash(code), cap);
         uint32_t inserted = 0;
         const uint32_t kaddr = keys_s + t0 * KB;
-#if DBG_PROBE_PRED
+#if DBG_BUCKET2
+        if constexpr (KW == 1) {
+          // buckets of two slots (the table's capacity and offset are even): one 16-byte
+          // load reads both keys; a lane claims the first empty one with a CAS and re-reads
+          // the bucket if it lost the race; a full bucket without its key moves it on
+          const uint32_t nbk = cap >> 1, b0 = __umulhi(smem_hash(code), nbk);
+          uint32_t bk = b0, sl = 0;
+          bool pend = want;
+          for (;;) {
+            const uint32_t ka = kaddr + bk * 16;
+            uint64_t k0, k1;
+            asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(k0), "=l"(k1) : "r"(ka) : "memory");
+            const bool m0 = k0 == key, m1 = k1 == key, e0 = k0 == 0, e1 = k1 == 0;
+            const bool found = m0 || m1;
+            const bool claim = pend && !found && (e0 || e1);
+            const uint32_t cs = e0 ? 0u : 1u;
+            uint64_t cur = 1;
+            cas_shared64_if(claim, ka + 8 * cs, key, cur);
+            const bool won = claim && cur == 0, same = claim && cur == key;
+            inserted |= (uint32_t)won;
+            sl = pend ? (found ? (m0 ? 0u : 1u) : cs) : sl;
+            const bool adv = pend && !found && !e0 && !e1;
+            const uint32_t nx = bk + 1 == nbk ? 0u : bk + 1;
+            bk = adv ? nx : bk;
+            if (adv && nx == b0) ok = false;  // wrapped: table full (reading O)
+            pend = pend && !found && !won && !same && !(adv && nx == b0);
+            if (!__any_sync(kFull, pend)) break;
+          }
+          idx = 2 * bk + sl;
+          if (!ok && want && lds64(kaddr + idx * KB) != key) idx = ~0u;  // this occurrence found no slot
+#elif DBG_PROBE_PRED
         if constexpr (KW == 1) {
           // every lane runs every probe round (predicated, no divergent branch): a lane with
           // nothing pending re-reads its current slot and keeps its state

@@ -345,13 +345,13 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 // nb bins; with nb <= kSmemHistMaxNp a CTA tile ranks its records in shared
 // memory and reserves once per bin, else one global atomic per record.
 #ifndef DBG_SCATTER_PER
-#define DBG_SCATTER_PER 8
+#define DBG_SCATTER_PER 4
 #endif
 #ifndef DBG_SCATTER_GRID
 #define DBG_SCATTER_GRID 0  // CTAs per SM (0: the occupancy limit)
 #endif
 #ifndef DBG_SCATTER_MINB
-#define DBG_SCATTER_MINB 1
+#define DBG_SCATTER_MINB 6
 #endif
 constexpr int kScatterThreads = 256;
 constexpr int kScatterPer = DBG_SCATTER_PER;  // records per thread per tile
@@ -520,20 +520,24 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
     for (int dlt = 16; dlt; dlt >>= 1) nPmax = max(nPmax, __shfl_xor_sync(kFull, nPmax, dlt));
     int ndesc = 0, s_next = 0;
     CT f = 0, rc = 0, m_cur = 0;
-    // the bases: a 64-bit window refilled every 32 bases
-    uint64_t wbuf = L > 0 ? window64(a.words, a.n_words, o) : 0;
-    int nbuf = 32, j = 0;  // bases left in wbuf, next base index
-    auto next_base = [&]() -> uint32_t {
-      if (nbuf == 0) {
+    // the bases: a 64-bit window of the stream at base j, reloaded before a run of
+    // bases that could exhaust it (one reload per block, no per-base check)
+    int j = 0, nbuf = 0;
+    uint64_t wbuf = 0;
+    auto refill = [&](int need) {
+      if (nbuf < need) {
         wbuf = j < L ? window64(a.words, a.n_words, o + j) : 0;
         nbuf = 32;
       }
+    };
+    auto next_base = [&]() -> uint32_t {
       const uint32_t b = (uint32_t)(wbuf >> 62);
       wbuf <<= 2;
       --nbuf;
       ++j;
       return b;
     };
+    refill(P - 1);
 #pragma unroll
     for (int t = 0; t < P - 1; ++t) {  // the first P-1 bases: no P-mer yet
       const uint32_t b = next_base();
@@ -551,6 +555,7 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
     for (int q0 = 0; q0 < nPmax + W; q0 += W) {
       CT c[W];
       CT pre = kInf;
+      refill(W);
 #pragma unroll
       for (int t = 0; t < W; ++t) {
         const int i = q0 - W + t;
@@ -583,9 +588,11 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
       for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
       if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
     }
+    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
 #else
     for (int q0 = 0; q0 < nPmax + W; q0 += W) {
       CT c[W], pre[W];
+      refill(W);
 #pragma unroll
       for (int t = 0; t < W; ++t) {
         CT v = kInf;
@@ -621,10 +628,12 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
       suf[W - 1] = c[W - 1];
 #pragma unroll
       for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
-      if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+      // one flush site (the code is inlined once): lists nearly full, or the reads' end
+      const bool last = q0 + W >= nPmax + W;
+      if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2 || (last && ndesc > 0)))
+        flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
     }
 #endif
-    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
   }
 }
 
