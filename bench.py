@@ -30,7 +30,7 @@ METRIC = "K-mers hashed/sec (graph build, device-timed) at 1/2/4/8 B200; HBM roo
 UNIT = "kmers/s"
 # version tag of the on-chip kernel: profiles/traffic.json (ncu --set full) is quoted only when it
 # was captured on this version
-KERNEL_VERSION = "smem-v6"
+KERNEL_VERSION = "smem-v7"
 
 
 def _peaks():
@@ -365,11 +365,12 @@ def run_ours(args):
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
     scan = 1 if b.np <= 16384 else 3  # scan.cuh: one CTA, or tile sums + tile scan + apply
-    # msp_kernel + its scan + scatter_kernel, then Step 2: the on-chip plan (7 kernels) + the on-chip
-    # kernel (+ per global-tier batch: its plan scan once, hash_build_list + extract_kernel)
+    # msp_block_kernel + its scan + scatter_kernel (+ bucket_scatter_kernel when two-level), then
+    # Step 2: the on-chip plan (8 kernels incl. the greedy group packing) + the on-chip kernel
+    # (+ per global-tier batch: its plan scan once, hash_build_list + extract_kernel)
     nb = len(b.batches)
-    launches_per_step = 2 + scan + {"fused": scan + 2, "resident": scan + 2 * nb,
-                                    "smem": 8 + 2 * nb + (scan if nb else 0)}[args.mode]
+    launches_per_step = 2 + scan + int(b.two_level) + {"fused": scan + 2, "resident": scan + 2 * nb,
+                                                       "smem": 9 + 2 * nb + (scan if nb else 0)}[args.mode]
     placement = _placement(b) if args.mode == "smem" else None
     # Fig. 6 / Table II analogue (row f1): the paper's partitions (fine pid mod NP) -- skew and the
     # table size lambda/(4 alpha) N^i_kmer x slot bytes of the largest one

@@ -57,8 +57,17 @@
 #ifndef DBG_BUCKET2
 #define DBG_BUCKET2 0
 #endif
+#ifndef DBG_SLOT26
+#define DBG_SLOT26 0  // implies no fine-pid field (DBG_SLOT28)
+#endif
 #ifndef DBG_SLOT28
 #define DBG_SLOT28 1
+#endif
+#if DBG_SLOT26 && !DBG_SLOT28
+#error DBG_SLOT26 needs DBG_SLOT28
+#endif
+#if DBG_SLOT26 && DBG_BITMAP
+#error DBG_SLOT26 excludes DBG_BITMAP
 #endif
 #ifndef DBG_RB4
 #define DBG_RB4 1024  // records of 4 words per on-chip batch (T >= 512)
@@ -807,7 +816,9 @@ template <int KW>
 struct SmemSlot {
   static constexpr uint32_t kKeyBytes = KW == 1 ? 8 : 16;
   static constexpr uint32_t kFieldWords = DBG_SLOT28 ? 5 : 6;  // (DBG_SLOT28: no fine-pid field)
-  static constexpr uint32_t kBytes = kKeyBytes + 4 * kFieldWords;
+  // DBG_SLOT26: the nine 16-bit fields packed at 18 bytes per slot (field f of slot s is
+  // half 9s + f of the field array)
+  static constexpr uint32_t kBytes = kKeyBytes + (DBG_SLOT26 ? 18 : 4 * kFieldWords);
 };
 
 // Decoded work item (32 B): records [r0, r0 + nrec) of partitions [first, last);
@@ -1476,14 +1487,20 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           }
         }
         if (want && idx != ~0u) {  // the multiple updates: 16-bit fields, two per word
+          const int fo = o < 4 ? o : 8;
+#if DBG_SLOT26
+          const uint32_t h0 = (t0 + idx) * 9u, ho = h0 + (uint32_t)fo, hi = h0 + 4u + (uint32_t)i;
+          red_shared_add(fld_s + (ho >> 1) * 4, 1u << (16 * (ho & 1)));
+          if (i >= 0) red_shared_add(fld_s + (hi >> 1) * 4, 1u << (16 * (hi & 1)));
+#else
           const uint32_t fa = fld_s + (t0 + idx) * (FW * 4);
           if (inserted) {
             if (!DBG_SLOT28) sts32(fa + 20, w[0] >> 10);
             if (DBG_BITMAP) red_shared_or(occ_s + 4 * ((t0 + idx) >> 5), 1u << ((t0 + idx) & 31u));
           }
-          const int fo = o < 4 ? o : 8;
           red_shared_add(fa + 4 * (fo >> 1), 1u << (16 * (fo & 1)));
           if (i >= 0) red_shared_add(fa + 4 * ((4 + i) >> 1), 1u << (16 * (i & 1)));
+#endif
         }
       }
     }
@@ -1509,6 +1526,17 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           bool keep = s < se && (lds64(keys_s + s * KB) & kOccupied);
 #endif
           if (keep && oa.min_count > 1) {  // row f4: a low-count vertex is cleaned, never emitted
+#if DBG_SLOT26
+            uint16_t* f16 = reinterpret_cast<uint16_t*>(fld) + s * 9;
+            if ((uint32_t)f16[0] + f16[1] + f16[2] + f16[3] + f16[8] < oa.min_count) {
+              keep = false;
+              unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+              kp[0] = 0;
+              if (KW == 2) kp[1] = 0;
+#pragma unroll
+              for (int q = 0; q < 9; ++q) f16[q] = 0;
+            }
+#else
             const uint32_t* f = fld + s * FW;
             const uint32_t f0 = f[0], f1 = f[1];
             if ((f0 & 0xffffu) + (f0 >> 16) + (f1 & 0xffffu) + (f1 >> 16) + (f[4] & 0xffffu) < oa.min_count) {
@@ -1520,6 +1548,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
 #pragma unroll
               for (uint32_t q = 0; q < FW; ++q) fz[q] = 0;
             }
+#endif
           }
           const uint32_t bal = __ballot_sync(kFull, keep);
           if (keep) queue[qn + __popc(bal & ((1u << lane) - 1u))] = (uint16_t)s;
@@ -1544,10 +1573,20 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             v.kmer_hi = kw0 & kCodeMask;
             v.kmer_lo = kp[1];
           }
+#if DBG_SLOT26
+          uint16_t* f16 = reinterpret_cast<uint16_t*>(fld) + s * 9;
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            v.out[q] = f16[q];
+            v.in[q] = f16[4 + q];
+          }
+          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + f16[8];  // count = sum(out) + t_out
+#else
           const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
           v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
           v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
           v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
+#endif
           // fine pid recorded by the inserting thread, mod NP (or from the P-minimizer, reading V)
           uint32_t fpid;
           if (DBG_SLOT28) {  // the fine partition owning slot s: last x with Pq[x] - P0 <= s
@@ -1567,8 +1606,13 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, fpid);
           kp[0] = 0;  // clean-on-extract
           if (KW == 2) kp[1] = 0;
+#if DBG_SLOT26
+#pragma unroll
+          for (int q = 0; q < 9; ++q) f16[q] = 0;
+#else
 #pragma unroll
           for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
+#endif
           const uint64_t my = pos + e;
           if (my < oa.out_cap) oa.out[my] = v;
           else atomicOr(oa.status, kStatusNoSpace);
