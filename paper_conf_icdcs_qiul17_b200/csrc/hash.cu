@@ -58,7 +58,7 @@
 #define DBG_BUCKET2 0
 #endif
 #ifndef DBG_SLOT26
-#define DBG_SLOT26 0  // implies no fine-pid field (DBG_SLOT28)
+#define DBG_SLOT26 1  // implies no fine-pid field (DBG_SLOT28)
 #endif
 #ifndef DBG_SLOT28
 #define DBG_SLOT28 1

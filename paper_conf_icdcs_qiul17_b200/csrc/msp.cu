@@ -189,11 +189,13 @@ __device__ __forceinline__ void write_record4(const MspArgs& a, uint32_t* dst, u
 // Warp-collective flush of the per-thread descriptor lists: partition ids
 // (computed once per descriptor and kept in place of the minimizer), size
 // histograms, one staging reservation per warp, record writes.
-template <typename CT>
+// kK > 0: compile-time K (record geometry and pieces without runtime division).
+template <typename CT, int kK = 0>
 __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
                                                   int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
-  const int nmax = (int)a.max_kmers;
+  const int nmax = kK > 0 ? (int)(16u * (record_words(kK) - 1u) - (uint32_t)kK - 1u) : (int)a.max_kmers;
+  const bool r4 = kK > 0 ? record_words(kK) == 4 : a.rec_words == 4;
   constexpr CT kSkip = ~(CT)0;  // a superkmer of another pass's partition (row f2)
   uint32_t my_records = 0;
   {
@@ -235,7 +237,7 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
     for (int ps = s; ps <= e; ps += nmax, ++slot) {
       if (slot < a.staging_cap) {
-        if (a.rec_words == 4)
+        if (r4)
           write_record4(a, a.staging + slot * 4, o, L, ps, min(e, ps + nmax - 1), pid);
         else
           write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
@@ -631,7 +633,7 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
       // one flush site (the code is inlined once): lists nearly full, or the reads' end
       const bool last = q0 + W >= nPmax + W;
       if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2 || (last && ndesc > 0)))
-        flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+        flush_descriptors<CT, K>(a, sm, ndesc, s_next, o, L);
     }
 #endif
   }
