@@ -349,6 +349,9 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 #ifndef DBG_SCATTER_PER
 #define DBG_SCATTER_PER 4
 #endif
+#ifndef DBG_SCATTER_A32
+#define DBG_SCATTER_A32 0  // 32-bit rank atomics
+#endif
 #ifndef DBG_SCATTER_GRID
 #define DBG_SCATTER_GRID 0  // CTAs per SM (0: the occupancy limit)
 #endif
@@ -396,7 +399,10 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
       if (idx < n) {
         const uint32_t bin = (rec[v][0].x >> 10) >> shift;
         if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
-        else rank[v] = (uint32_t)atomicAdd(fill + bin, 1ull);
+        else if (DBG_SCATTER_A32)  // the low half of the (zeroed) 64-bit cursor: counts < 2^32
+          rank[v] = atomicAdd(reinterpret_cast<unsigned int*>(fill + bin), 1u);
+        else
+          rank[v] = (uint32_t)atomicAdd(fill + bin, 1ull);
       }
     }
     uint64_t base[kPer];
