@@ -57,6 +57,9 @@
 #ifndef DBG_BUCKET2
 #define DBG_BUCKET2 0
 #endif
+#ifndef DBG_VSTORE
+#define DBG_VSTORE 0  // 16-byte vertex stores
+#endif
 #ifndef DBG_SLOT26
 #define DBG_SLOT26 1  // implies no fine-pid field (DBG_SLOT28)
 #endif
@@ -1192,6 +1195,33 @@ __device__ __forceinline__ uint32_t sub_table(Code code, uint32_t n) {
   return __umulhi((uint32_t)(fmix64(x) >> 32), n);
 }
 
+// A 56-byte vertex record with 16-byte stores where aligned: record i starts at 56 i, which is
+// 16-aligned for even i (words 0-11 as three 16-B stores, 12-13 as one 8-B store) and 8 past a
+// 16-B boundary for odd i (words 0-1 as 8 B, 2-13 as three 16-B stores): five predicated store
+// instructions per warp instead of seven 8-byte ones, with the same bytes.
+__device__ __forceinline__ void store_vertex16(dbg_vertex* dst, const dbg_vertex& v, bool odd) {
+  uint32_t w[14];
+  w[0] = (uint32_t)v.kmer_hi; w[1] = (uint32_t)(v.kmer_hi >> 32);
+  w[2] = (uint32_t)v.kmer_lo; w[3] = (uint32_t)(v.kmer_lo >> 32);
+  w[4] = v.count;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    w[5 + q] = v.out[q];
+    w[9 + q] = v.in[q];
+  }
+  w[13] = v.pid;
+  char* base = reinterpret_cast<char*>(dst);
+  const int sh = odd ? 2 : 0;  // first word of the 16-B run
+#pragma unroll
+  for (int c = 0; c < 3; ++c) {
+    const int q = 4 * c;
+    const uint4 x = odd ? make_uint4(w[q + 2], w[q + 3], w[q + 4], w[q + 5]) : make_uint4(w[q], w[q + 1], w[q + 2], w[q + 3]);
+    *reinterpret_cast<uint4*>(base + 4 * (q + sh)) = x;
+  }
+  const int r = odd ? 0 : 12;  // the 8-byte remainder
+  *reinterpret_cast<uint2*>(base + 4 * r) = odd ? make_uint2(w[0], w[1]) : make_uint2(w[12], w[13]);
+}
+
 // A group of consecutive fine partitions shares one CTA table: each partition
 // p owns slots [P[p] - P[first], P[p+1] - P[first]).
 template <typename Code, int R, int kSmemThreads, int kMinCtas>
@@ -1614,7 +1644,13 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
 #endif
           const uint64_t my = pos + e;
-          if (my < oa.out_cap) oa.out[my] = v;
+          if (my < oa.out_cap) {
+#if DBG_VSTORE
+            store_vertex16(oa.out + my, v, (my & 1) != 0);
+#else
+            oa.out[my] = v;
+#endif
+          }
           else atomicOr(oa.status, kStatusNoSpace);
           st_n += 1;
           st_count += v.count;

@@ -664,11 +664,26 @@ bool dbg_params_ok(const dbg_params* prm) {
          (uint64_t)prm->num_partitions * (uint64_t)(prm->refine > 1 ? prm->refine : 1) <= kMaxPid;
 }
 
+// Grid of the grid-stride MSP kernels: at most one wave of resident CTAs (a partial second
+// wave would start its reads only when first-wave CTAs finish theirs).
+#ifndef DBG_MSP_GRID
+#define DBG_MSP_GRID 0  // CTAs per SM (0: the occupancy limit)
+#endif
+static int msp_grid(const void* fn, int want, size_t smem) {
+  int per_sm = 0;
+  if (DBG_MSP_GRID > 0 || cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kMspThreads, smem) != cudaSuccess ||
+      per_sm < 1)
+    per_sm = DBG_MSP_GRID > 0 ? DBG_MSP_GRID : 8;
+  const int cap = dbg_sm_count() * per_sm;
+  return want < cap ? want : cap;
+}
+
 template <int W, int P>
 static cudaError_t launch_msp_block(const MspArgs& a, int grid, cudaStream_t stream) {
   const size_t smem = (sizeof(uint32_t) + sizeof(uint32_t)) * kMaxDescBlock * kMspThreads;
   cudaError_t e = cudaFuncSetAttribute(msp_block_kernel<W, P>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
+  grid = msp_grid((const void*)msp_block_kernel<W, P>, grid, smem);
   msp_block_kernel<W, P><<<grid, kMspThreads, smem, stream>>>(a);
   return cudaGetLastError();
 }
@@ -691,6 +706,7 @@ static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
   const size_t smem = (sizeof(CT) + sizeof(uint32_t)) * kMaxDesc * kMspThreads + sizeof(CT) * a.w * kMspThreads;
   cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
+  grid = msp_grid((const void*)msp_kernel<CT>, grid, smem);
   msp_kernel<CT><<<grid, kMspThreads, smem, stream>>>(a);
   return cudaGetLastError();
 }
@@ -754,7 +770,7 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       return DBG_ECUDA;
     if (n_reads) {
       const uint64_t want = (n_reads + kMspThreads - 1) / kMspThreads;
-      const uint64_t cap = (uint64_t)dbg_sm_count() * 8;
+      const uint64_t cap = (uint64_t)dbg_sm_count() * 32;  // launch_msp* cap it at one resident wave
       const int grid = (int)(want < cap ? want : cap);
       cudaError_t e = cudaSuccess;
       if (!msp_block_launch(a, grid, stream, &e))
