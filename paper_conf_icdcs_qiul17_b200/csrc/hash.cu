@@ -57,8 +57,11 @@
 #ifndef DBG_BUCKET2
 #define DBG_BUCKET2 0
 #endif
+#ifndef DBG_SADDR
+#define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
+#endif
 #ifndef DBG_VSTORE
-#define DBG_VSTORE 0  // 16-byte vertex stores
+#define DBG_VSTORE 1  // 16-byte vertex stores
 #endif
 #ifndef DBG_SLOT26
 #define DBG_SLOT26 1  // implies no fine-pid field (DBG_SLOT28)
@@ -885,6 +888,21 @@ __device__ __forceinline__ uint64_t lds64(uint32_t a) {
   asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
   return v;
 }
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+  uint16_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint2 lds_u2(uint32_t a) {
+  uint2 v;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+  return v;
+}
 __device__ __forceinline__ uint64_t cas_shared64(uint32_t a, uint64_t want) {
   uint64_t old;
   asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(a), "l"(0ull), "l"(want) : "memory");
@@ -1355,18 +1373,34 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       constexpr int S = RB;  // staging stride
       constexpr uint32_t kWarps = kSmemThreads / 32;
       typedef KeyOf<Code> KO;
+#if DBG_SADDR
+      // 32-bit shared-window addresses of the batch arrays, formed once per batch
+      const uint32_t rwin_s = smem_addr(st.rwin), pre_s = smem_addr(st.pre), desc_s = smem_addr(st.desc),
+                     wb_s = smem_addr(&st.w[bb][0][0]);
+#endif
       for (uint32_t m = warp; 32 * m < total; m += kWarps) {
         const uint32_t kb = 32 * m, kid = kb + lane;
         const bool act = kid < total;
+#if DBG_SADDR
+        const uint32_t rb = lds_u16(rwin_s + 2 * m);
+        const uint32_t nxt = rb + 1 + lane;
+        const uint32_t x0 = nxt < nc ? lds32(pre_s + 4 * nxt) : total;
+#else
         const uint32_t rb = st.rwin[m];
         // records starting inside the window: one bit each at their first K-mer
         const uint32_t nxt = rb + 1 + lane;
         const uint32_t x0 = nxt < nc ? st.pre[nxt] : total;
+#endif
         const uint32_t starts = __reduce_or_sync(kFull, x0 < kb + 32 ? 1u << (x0 - kb) : 0u);
         const uint32_t c = rb + __popc(starts & ((2u << lane) - 1u));
         const uint32_t cc = act ? c : rb;
+#if DBG_SADDR
+        const uint2 d = lds_u2(desc_s + 8 * cc);
+        const int t = (int)(kid - lds32(pre_s + 4 * cc));
+#else
         const uint2 d = st.desc[cc];
         const int t = (int)(kid - st.pre[cc]);
+#endif
         const int j = d.x & 1023u, n = (d.x >> 10) & 255u, hl = (d.x >> 18) & 1u, hr = (d.x >> 19) & 1u;
         const uint32_t t0 = d.y & 0xffffu, cap = d.y >> 16;
         const uint32_t* w = &st.w[bb][0][j];
@@ -1377,7 +1411,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
 #if DBG_WORDSEL
           // the three data words, loaded unconditionally and selected (no branches): a1..a3
           // hold bases b .. b + 47 - 16q
+#if DBG_SADDR
+          const uint32_t wj = wb_s + 4 * (uint32_t)j;
+          const uint32_t d1 = lds32(wj + 4 * S), d2 = lds32(wj + 8 * S), d3 = lds32(wj + 12 * S);
+#else
           const uint32_t d1 = w[S], d2 = w[2 * S], d3 = w[3 * S];
+#endif
           const int q = b >> 4;
           const uint32_t a1 = q == 0 ? d1 : (q == 1 ? d2 : d3), a2 = q == 0 ? d2 : (q == 1 ? d3 : 0u),
                          a3 = q == 0 ? d3 : 0u;
