@@ -57,6 +57,9 @@
 #ifndef DBG_BUCKET2
 #define DBG_BUCKET2 0
 #endif
+#ifndef DBG_KW2_LOAD
+#define DBG_KW2_LOAD 0  // two-word keys: load, CAS only on an empty-looking entry
+#endif
 #ifndef DBG_SADDR
 #define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
 #endif
@@ -1540,7 +1543,18 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
           uint32_t probes = 0, pend = want;
           while (__any_sync(kFull, pend)) {
             if (pend) {
+#if DBG_KW2_LOAD
+              // load first, CAS only on an empty-looking entry: a 16-B shared load is not
+              // single-copy atomic, but entries only go (0, 0) -> key, and every key's hi word
+              // has OCC set, so a torn read is (0, lo), (hi, 0) or the key; (x, 0) / (0, x)
+              // are treated as empty and the CAS returns the entry atomically
+              const uint32_t ka = kaddr + idx * KB;
+              typename KO::T cur;
+              asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(cur.x), "=l"(cur.y) : "r"(ka) : "memory");
+              if (cur.x == 0 || cur.y == 0) cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);
+#else
               const typename KO::T cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);  // 16-B CAS: read-or-claim
+#endif
               inserted = KO::empty(cur);
               if (inserted | KO::same(cur, key)) {
                 pend = 0;

@@ -43,6 +43,9 @@ constexpr int kMaxDesc = 40;             // descriptors per thread between flush
 #ifndef DBG_MSP_FUSED
 #define DBG_MSP_FUSED 0   // 1: running prefix minimum interleaved with the K-mer emission
 #endif
+#ifndef DBG_MSP_NOBR
+#define DBG_MSP_NOBR 0  // 1: branch-free base consumption (padding past the read end)
+#endif
 #ifndef DBG_MSP_DESC
 #define DBG_MSP_DESC 40   // descriptors per thread between flushes (>= W + 3)
 #endif
@@ -601,6 +604,19 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
     for (int q0 = 0; q0 < nPmax + W; q0 += W) {
       CT c[W], pre[W];
       refill(W);
+#if DBG_MSP_NOBR
+      // every lane shifts W bases out of its window (past its read's end they are padding and
+      // their P-mers are masked to +inf): no per-base branch
+      const int rem = nP - q0;
+#pragma unroll
+      for (int t = 0; t < W; ++t) {
+        const uint32_t b = (uint32_t)(wbuf >> 62);
+        wbuf <<= 2;
+        f = ((f << 2) | b) & kMaskP;
+        rc = (rc >> 2) | ((CT)(b ^ 3u) << kTopP);
+        const CT v = t < rem ? (f < rc ? f : rc) : kInf;  // canonical P-mer (reading D)
+        c[t] = v;
+#else
 #pragma unroll
       for (int t = 0; t < W; ++t) {
         CT v = kInf;
@@ -611,8 +627,13 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
           v = f < rc ? f : rc;  // canonical P-mer (reading D)
         }
         c[t] = v;
+#endif
         pre[t] = t == 0 ? v : (v < pre[t - 1] ? v : pre[t - 1]);
       }
+#if DBG_MSP_NOBR
+      nbuf -= W;
+      j += W;
+#endif
       if (q0 >= W) {  // K-mers i = q0 - W + t of the previous block's windows
 #pragma unroll
         for (int t = 0; t < W; ++t) {
