@@ -60,6 +60,9 @@
 #ifndef DBG_KW2_LOAD
 #define DBG_KW2_LOAD 0  // two-word keys: load, CAS only on an empty-looking entry
 #endif
+#ifndef DBG_XSCAN
+#define DBG_XSCAN 1  // extraction scan: sign bit of the key's high word, shared addresses hoisted
+#endif
 #ifndef DBG_SADDR
 #define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
 #endif
@@ -901,6 +904,9 @@ __device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
   asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
   return v;
 }
+__device__ __forceinline__ void sts16(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((uint16_t)v) : "memory");
+}
 __device__ __forceinline__ uint2 lds_u2(uint32_t a) {
   uint2 v;
   asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
@@ -1601,6 +1607,30 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       for (uint32_t sub = ws0; sub < ws1; sub += kQ) {
         const uint32_t se = min(ws1, sub + kQ);
         uint32_t qn = 0;
+#if DBG_XSCAN
+        if (oa.min_count <= 1) {
+          // occupied slots: the sign bit of the key's high 32-bit word (OCC); 32-bit shared
+          // addresses formed once; two 32-slot chunks per iteration
+          const uint32_t q_s = smem_addr(queue), lt = (1u << lane) - 1u;
+          uint32_t c = sub;
+          for (; c + 64 <= se; c += 64) {
+            const uint32_t s0 = c + lane, s1 = s0 + 32;
+            const bool k0 = (int)lds32(keys_s + s0 * KB + 4) < 0, k1 = (int)lds32(keys_s + s1 * KB + 4) < 0;
+            const uint32_t b0 = __ballot_sync(kFull, k0), b1 = __ballot_sync(kFull, k1);
+            if (k0) sts16(q_s + 2 * (qn + __popc(b0 & lt)), s0);
+            qn += __popc(b0);
+            if (k1) sts16(q_s + 2 * (qn + __popc(b1 & lt)), s1);
+            qn += __popc(b1);
+          }
+          for (; c < se; c += 32) {
+            const uint32_t s0 = c + lane;
+            const bool k0 = s0 < se && (int)lds32(keys_s + s0 * KB + 4) < 0;
+            const uint32_t b0 = __ballot_sync(kFull, k0);
+            if (k0) sts16(q_s + 2 * (qn + __popc(b0 & lt)), s0);
+            qn += __popc(b0);
+          }
+        } else
+#endif
         for (uint32_t c = sub; c < se; c += 32) {
           const uint32_t s = c + lane;
 #if DBG_BITMAP
