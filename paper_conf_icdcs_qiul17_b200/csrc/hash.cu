@@ -63,6 +63,9 @@
 #ifndef DBG_XSCAN
 #define DBG_XSCAN 1  // extraction scan: sign bit of the key's high word, shared addresses hoisted
 #endif
+#ifndef DBG_XEMIT
+#define DBG_XEMIT 0  // extraction emission with explicit shared addresses
+#endif
 #ifndef DBG_SADDR
 #define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
 #endif
@@ -904,6 +907,9 @@ __device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
   asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
   return v;
 }
+__device__ __forceinline__ void sts64(uint32_t a, uint64_t v) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
 __device__ __forceinline__ void sts16(uint32_t a, uint32_t v) {
   asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((uint16_t)v) : "memory");
 }
@@ -1673,7 +1679,45 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         if (lane == 0 && qn) pos = atomicAdd(oa.n_out, (unsigned long long)qn);
         pos = __shfl_sync(kFull, pos, 0);
         __syncwarp();
+#if DBG_XEMIT && DBG_SLOT26
+        const uint32_t qe_s = smem_addr(queue);
+#endif
         for (uint32_t e = lane; e < qn; e += 32) {
+#if DBG_XEMIT && DBG_SLOT26
+          // explicit 32-bit shared addresses (formed from hoisted bases), 16-bit field loads
+          const uint32_t s = lds_u16(qe_s + 2 * e);
+          const uint32_t ka = keys_s + s * KB, fa = fld_s + 18u * s;
+          const uint64_t kw0 = lds64(ka);
+          dbg_vertex v;
+          if (KW == 1) {
+            v.kmer_hi = 0;
+            v.kmer_lo = kw0 & kCodeMask;
+          } else {
+            v.kmer_hi = kw0 & kCodeMask;
+            v.kmer_lo = lds64(ka + 8);
+          }
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            v.out[q] = lds_u16(fa + 2 * q);
+            v.in[q] = lds_u16(fa + 8 + 2 * q);
+          }
+          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + lds_u16(fa + 16);  // count = sum(out) + t_out
+          uint32_t fpid = I.first;  // the fine partition owning slot s: last x with Pq[x] - P0 <= s
+          if (sub_n == 1) {
+            uint32_t lo = 0, n = I.last - I.first;
+            while (n > 1) {
+              const uint32_t h = n >> 1;
+              if (Pq[lo + h] - I.P0 <= s) lo += h, n -= h;
+              else n = h;
+            }
+            fpid += lo;
+          }
+          v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, fpid);
+          sts64(ka, 0);  // clean-on-extract
+          if (KW == 2) sts64(ka + 8, 0);
+#pragma unroll
+          for (int q = 0; q < 9; ++q) sts16(fa + 2 * q, 0);
+#else
           const uint32_t s = queue[e];
           unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
           const uint64_t kw0 = kp[0];
@@ -1726,6 +1770,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
 #pragma unroll
           for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
 #endif
+#endif  // DBG_XEMIT
           const uint64_t my = pos + e;
           if (my < oa.out_cap) {
 #if DBG_VSTORE

@@ -43,6 +43,9 @@ constexpr int kMaxDesc = 40;             // descriptors per thread between flush
 #ifndef DBG_MSP_FUSED
 #define DBG_MSP_FUSED 0   // 1: running prefix minimum interleaved with the K-mer emission
 #endif
+#ifndef DBG_MSP_TAIL
+#define DBG_MSP_TAIL 0  // 1: the read's last superkmer appended after the block loop
+#endif
 #ifndef DBG_MSP_NOBR
 #define DBG_MSP_NOBR 0  // 1: branch-free base consumption (padding past the read end)
 #endif
@@ -646,11 +649,13 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
               ++ndesc;
             }
             m_cur = m;
+#if !DBG_MSP_TAIL
             if (i == nk - 1) {  // the read's last superkmer
               sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
               sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
               ++ndesc;
             }
+#endif
           }
         }
       }
@@ -659,6 +664,13 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
       for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
       // one flush site (the code is inlined once): lists nearly full, or the reads' end
       const bool last = q0 + W >= nPmax + W;
+#if DBG_MSP_TAIL
+      if (last && nk > 0) {  // the read's last superkmer, appended once after its last K-mer
+        sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(nk - 1));
+        sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+        ++ndesc;
+      }
+#endif
       if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2 || (last && ndesc > 0)))
         flush_descriptors<CT, K>(a, sm, ndesc, s_next, o, L);
     }
