@@ -36,7 +36,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 9
+#define DBG_ABI_VERSION 10
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -138,6 +138,11 @@ typedef struct {
                                 with more than 8192 fine partitions pass 2 then scatters in two
                                 levels -- into buckets of 2^s consecutive partitions (d_scratch),
                                 then within each bucket (d_records); NULL: one level */
+  uint32_t* d_rank;          /* optional, staging_cap entries: pass 1 writes each staged record's
+                                rank inside its partition (from the per-partition record counter),
+                                and pass 2 places record j at d_record_offset[pid] + d_rank[j]
+                                without rank atomics.  Pass 2 may use it only for records staged by
+                                pass 1 of this partition set (NULL e.g. after a record exchange) */
 } dbg_partition_set;
 
 /* ---- sizes ------------------------------------------------------------ */

@@ -37,7 +37,7 @@ class dbg_partition_set(ctypes.Structure):
                 ("d_record_offset", ctypes.c_void_p), ("d_fill", ctypes.c_void_p),
                 ("d_staged", ctypes.c_void_p), ("d_staging", ctypes.c_void_p),
                 ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p),
-                ("d_scratch", ctypes.c_void_p)]
+                ("d_scratch", ctypes.c_void_p), ("d_rank", ctypes.c_void_p)]
 
 
 # dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
@@ -90,7 +90,7 @@ SIGNATURES = {
 }
 
 _lib = None
-ABI_VERSION = 9
+ABI_VERSION = 10
 
 
 def load():
@@ -146,9 +146,9 @@ def fine_partitions(prm: dbg_params) -> int:
 
 
 def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
-                  records=None, scratch=None) -> dbg_partition_set:
+                  records=None, scratch=None, rank=None) -> dbg_partition_set:
     return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(staged),
-                             _ptr(staging), staging_cap, _ptr(records), _ptr(scratch))
+                             _ptr(staging), staging_cap, _ptr(records), _ptr(scratch), _ptr(rank))
 
 
 # --------------------------------------------------------------------------- entry points

@@ -73,6 +73,7 @@ struct MspArgs {
   uint32_t* staging;              // records in read order
   uint64_t staging_cap;           // records
   unsigned long long* staged;     // cursor (records reserved)
+  uint32_t* rank;                 // [staging_cap] record rank inside its partition, or null
   uint32_t pid_lo, pid_hi;        // only superkmers of fine partitions [pid_lo, pid_hi) are counted and staged
   bool ranged;                    // pid_lo > 0 or pid_hi < np
 };
@@ -239,10 +240,16 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     }
     const uint32_t pid = (uint32_t)dm;
     const int n = e - s + 1;
-    atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
+    // the record counter's old value ranks this superkmer's pieces inside the partition (d_rank)
+    uint32_t r = 0;
+    if (a.rank)
+      r = (uint32_t)atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
+    else
+      atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
-    for (int ps = s; ps <= e; ps += nmax, ++slot) {
+    for (int ps = s; ps <= e; ps += nmax, ++slot, ++r) {
       if (slot < a.staging_cap) {
+        if (a.rank) a.rank[slot] = r;
         if (r4)
           write_record4(a, a.staging + slot * 4, o, L, ps, min(e, ps + nmax - 1), pid);
         else
@@ -435,6 +442,44 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
       }
     }
     if (smem) __syncthreads();
+  }
+}
+
+// Pass 3 with pass-1 ranks (dbg_partition_set.d_rank): record j goes to
+// rec_off[pid] + rank[j] -- no rank atomics, a pure gather/scatter of 16-B
+// (or wider) records.
+template <int R>
+__global__ void __launch_bounds__(256) scatter_rank_kernel(const uint32_t* __restrict__ staging,
+                                                           const uint32_t* __restrict__ rank,
+                                                           const unsigned long long* staged, uint64_t staging_cap,
+                                                           const uint64_t* __restrict__ rec_off,
+                                                           uint32_t* __restrict__ records) {
+  const uint64_t n = *staged;
+  if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
+  constexpr int kPer = 4;
+  for (uint64_t t0 = (uint64_t)blockIdx.x * 256 * kPer; t0 < n; t0 += (uint64_t)gridDim.x * 256 * kPer) {
+    uint4 rec[kPer][R / 4];
+    uint32_t rk[kPer];
+#pragma unroll
+    for (int v = 0; v < kPer; ++v) {
+      const uint64_t idx = t0 + v * 256 + threadIdx.x;
+      if (idx < n) {
+        const uint4* src = reinterpret_cast<const uint4*>(staging + idx * R);
+#pragma unroll
+        for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(src + c);
+        rk[v] = __ldcs(rank + idx);
+      }
+    }
+#pragma unroll
+    for (int v = 0; v < kPer; ++v) {
+      const uint64_t idx = t0 + v * 256 + threadIdx.x;
+      if (idx < n) {
+        const uint64_t pos = __ldg(rec_off + (rec[v][0].x >> 10)) + rk[v];
+        uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
+#pragma unroll
+        for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];
+      }
+    }
   }
 }
 
@@ -794,6 +839,7 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     a.staging = part->d_staging;
     a.staging_cap = part->staging_cap;
     a.staged = reinterpret_cast<unsigned long long*>(part->d_staged);
+    a.rank = part->d_staging && part->staging_cap ? part->d_rank : nullptr;
     a.pid_lo = (uint32_t)pid_lo;
     a.pid_hi = (uint32_t)pid_hi;
     a.ranged = pid_lo > 0 || pid_hi < np;
@@ -819,6 +865,24 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
     if (part->d_scratch && (part->d_scratch == part->d_staging || part->d_scratch == part->d_records))
       return DBG_EINVAL;
+    if (part->d_rank) {  // ranks from pass 1: one pass, no atomics
+      const unsigned long long* stg = reinterpret_cast<const unsigned long long*>(part->d_staged);
+      int per_sm = 0;
+      const int grid = dbg_sm_count() * 8;
+#define DBG_SCATTER_RANK(RW)                                                                                   \
+  scatter_rank_kernel<RW><<<grid, 256, 0, stream>>>(part->d_staging, part->d_rank, stg, part->staging_cap,      \
+                                                   part->d_record_offset, part->d_records);
+      (void)per_sm;
+      if (R == 4) {
+        DBG_SCATTER_RANK(4)
+      } else if (R == 8) {
+        DBG_SCATTER_RANK(8)
+      } else {
+        DBG_SCATTER_RANK(16)
+      }
+#undef DBG_SCATTER_RANK
+      return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
+    }
     const bool two = part->d_scratch && np > kSmemHistMaxNp;
     int shift = 0;
     // level 1 into at most 512 bins, so that a tile of 2048 records ranks several records per

@@ -120,6 +120,10 @@ class DbgBuilder:
         # atomics on E. coli and chr14 (profiles/r01d_ab.txt)
         self.scratch = torch.empty(0, dtype=torch.int32, device=dev)
         self.two_level = NP > 8192 and os.environ.get("DBG_SCATTER_TWO_LEVEL") == "1"
+        # pass-1 ranks (dbg_partition_set.d_rank): pass 2 without rank atomics
+        self.use_rank = os.environ.get("DBG_MSP_RANK", "0") == "1"
+        self.rank = torch.empty(0, dtype=torch.int32, device=dev)
+        self._rank_valid = False
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
         self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
         self.work = torch.empty(0, dtype=torch.uint8, device=dev)
@@ -173,9 +177,14 @@ class DbgBuilder:
         if with_records and self.two_level:
             self.scratch = _grow(self.scratch, self.records.numel(), torch.int32, self.device)
             scratch = self.scratch
+        rank = None
+        cap = self.staging.numel() // self.rec_words
+        if self.use_rank and (not with_records or self._rank_valid):
+            self.rank = _grow(self.rank, cap, torch.int32, self.device)
+            rank = self.rank
+            self._rank_valid = True  # pass 1 writes them; invalidated by load_exchanged
         return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill, self.d_staged,
-                                  self.staging, self.staging.numel() // self.rec_words,
-                                  self.records if with_records else None, scratch)
+                                  self.staging, cap, self.records if with_records else None, scratch, rank)
 
     def _staging_estimate(self, n_kmers_upper: int, n_reads: int) -> int:
         w = self.k - self.p + 1
@@ -294,6 +303,7 @@ class DbgBuilder:
             self.d_rec_off.copy_(torch.from_numpy(off), non_blocking=True)
             self.d_staged.fill_(n_received)
         self.staging = received
+        self._rank_valid = False  # the received records were not ranked by this set's pass 1
         self.records = _grow(self.records, n_received * self.rec_words, torch.int32, self.device, 1.05)
         _lib.dbg_msp_partition(self.prm, 1, 1, self.d_rec_off, 0, self.part_set(True), stream)
 

@@ -36,7 +36,7 @@ def test_exports_every_declared_symbol(lib):
 
 
 def test_abi_and_sizes(lib):
-    assert lib.dbg_abi_version() == 9
+    assert lib.dbg_abi_version() == 10
     p31 = lib.params(31, 11, 16)
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
