@@ -249,11 +249,11 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
     for (int ps = s; ps <= e; ps += nmax, ++slot, ++r) {
       if (slot < a.staging_cap) {
-        if (a.rank) a.rank[slot] = r;
         if (r4)
           write_record4(a, a.staging + slot * 4, o, L, ps, min(e, ps + nmax - 1), pid);
         else
           write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
+        if (a.rank) a.rank[slot] = r;  // after the record: its loads overlap the atomic's latency
       }
     }
     s = e + 1;
