@@ -362,6 +362,9 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 #ifndef DBG_SCATTER_PER
 #define DBG_SCATTER_PER 4
 #endif
+#ifndef DBG_SCATTER_ABS
+#define DBG_SCATTER_ABS 0  // global-path cursors start at the record offsets
+#endif
 #ifndef DBG_SCATTER_A32
 #define DBG_SCATTER_A32 0  // 32-bit rank atomics
 #endif
@@ -379,7 +382,10 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
                                                                   uint64_t staging_cap,
                                                                   const uint64_t* __restrict__ rec_off,
                                                                   unsigned long long* fill,
-                                                                  uint32_t* __restrict__ records, int nb, int shift) {
+                                                                  uint32_t* __restrict__ records, int nb, int shift,
+                                                                  bool abs_pos) {
+  // abs_pos (global path, shift 0): the cursors start at the partitions' record offsets, so the
+  // rank atomic returns the record's final position (no offset load)
   extern __shared__ unsigned long long sh_base[];  // [nb] global bases (per tile), then [nb] counts
   uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_base + nb);
   const uint64_t n = *staged;
@@ -394,6 +400,7 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
     }
     uint4 rec[kPer][R / 4];
     uint32_t rank[kPer];
+    uint64_t apos[kPer];
     // all loads of the tile first, then all rank atomics, then all stores: kPer records of
     // each thread in flight at every stage (the kernel is latency-bound)
 #pragma unroll
@@ -409,9 +416,11 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       rank[v] = 0;
+      apos[v] = 0;
       if (idx < n) {
         const uint32_t bin = (rec[v][0].x >> 10) >> shift;
-        if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
+        if (abs_pos) apos[v] = atomicAdd(fill + bin, 1ull);
+        else if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
         else if (DBG_SCATTER_A32)  // the low half of the (zeroed) 64-bit cursor: counts < 2^32
           rank[v] = atomicAdd(reinterpret_cast<unsigned int*>(fill + bin), 1u);
         else
@@ -422,7 +431,7 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
 #pragma unroll
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
-      base[v] = idx < n ? __ldg(rec_off + (((rec[v][0].x >> 10) >> shift) << shift)) : 0;
+      base[v] = idx < n && !abs_pos ? __ldg(rec_off + (((rec[v][0].x >> 10) >> shift) << shift)) : 0;
     }
     if (smem) {
       __syncthreads();
@@ -435,7 +444,7 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       if (idx < n) {
         const uint32_t bin = (rec[v][0].x >> 10) >> shift;
-        const uint64_t pos = base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
+        const uint64_t pos = abs_pos ? apos[v] : base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
         uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
 #pragma unroll
         for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];
@@ -889,7 +898,14 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     // bin in shared memory and reserves once per bin
     while (two && ((np + (1 << shift) - 1) >> shift) > kTwoLevelBins) ++shift;
     const int nb = (np + (1 << shift) - 1) >> shift;
-    if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) return DBG_ECUDA;
+    const bool abs_pos = DBG_SCATTER_ABS && nb > kSmemHistMaxNp && shift == 0;
+    if (abs_pos) {  // cursors = the partitions' record offsets
+      if (cudaMemcpyAsync(part->d_fill, part->d_record_offset, sizeof(uint64_t) * nb, cudaMemcpyDeviceToDevice,
+                          stream) != cudaSuccess)
+        return DBG_ECUDA;
+    } else if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) {
+      return DBG_ECUDA;
+    }
     const size_t smem = nb <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * nb : 0;
     // one full wave: the kernel is grid-stride, a partial second wave would idle SMs
     auto scatter_grid = [&](const void* fn) {
@@ -908,7 +924,8 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
 #define DBG_SCATTER(RW)                                                                                         \
   cudaFuncSetAttribute(scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
   scatter_kernel<RW><<<scatter_grid((const void*)scatter_kernel<RW>), kScatterThreads, smem, stream>>>(part->d_staging, staged, part->staging_cap,       \
-                                                              part->d_record_offset, fill, lvl1, nb, shift);    \
+                                                              part->d_record_offset, fill, lvl1, nb, shift,     \
+                                                              abs_pos);                                          \
   if (two) {                                                                                                    \
     cudaFuncSetAttribute(bucket_scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);   \
     bucket_scatter_kernel<RW><<<grid2, kBucketThreads, smem2, stream>>>(part->d_scratch, staged,               \
