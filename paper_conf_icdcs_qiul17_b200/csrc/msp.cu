@@ -43,6 +43,9 @@ constexpr int kMaxDesc = 40;             // descriptors per thread between flush
 #ifndef DBG_MSP_FUSED
 #define DBG_MSP_FUSED 0   // 1: running prefix minimum interleaved with the K-mer emission
 #endif
+#ifndef DBG_MSP_STCS
+#define DBG_MSP_STCS 0  // evict-first staging stores
+#endif
 #ifndef DBG_MSP_TAIL
 #define DBG_MSP_TAIL 0  // 1: the read's last superkmer appended after the block loop
 #endif
@@ -189,8 +192,10 @@ __device__ __forceinline__ void write_record4(const MspArgs& a, uint32_t* dst, u
   const uint32_t m1 = nb >= 48 ? ~0u : (nb <= 32 ? 0u : ~(~0u >> (2 * (nb - 32))));
   const uint64_t b0 = v0 & m0;
   const uint32_t b1 = (uint32_t)(v1 >> 32) & m1;
-  reinterpret_cast<uint4*>(dst)[0] =
-      make_uint4((uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10), (uint32_t)(b0 >> 32), (uint32_t)b0, b1);
+  const uint4 rec = make_uint4((uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10), (uint32_t)(b0 >> 32),
+                               (uint32_t)b0, b1);
+  if (DBG_MSP_STCS) __stcs(reinterpret_cast<uint4*>(dst), rec);
+  else reinterpret_cast<uint4*>(dst)[0] = rec;
 }
 
 // Warp-collective flush of the per-thread descriptor lists: partition ids
@@ -362,6 +367,9 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 #ifndef DBG_SCATTER_PER
 #define DBG_SCATTER_PER 4
 #endif
+#ifndef DBG_SCATTER_STCS
+#define DBG_SCATTER_STCS 0  // evict-first record stores
+#endif
 #ifndef DBG_SCATTER_ABS
 #define DBG_SCATTER_ABS 0  // global-path cursors start at the record offsets
 #endif
@@ -372,7 +380,7 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 #define DBG_SCATTER_GRID 0  // CTAs per SM (0: the occupancy limit)
 #endif
 #ifndef DBG_SCATTER_MINB
-#define DBG_SCATTER_MINB 6
+#define DBG_SCATTER_MINB 4
 #endif
 constexpr int kScatterThreads = 256;
 constexpr int kScatterPer = DBG_SCATTER_PER;  // records per thread per tile
@@ -447,7 +455,10 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
         const uint64_t pos = abs_pos ? apos[v] : base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
         uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
 #pragma unroll
-        for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];
+        for (int c = 0; c < R / 4; ++c) {
+          if (DBG_SCATTER_STCS) __stcs(dst + c, rec[v][c]);
+          else dst[c] = rec[v][c];
+        }
       }
     }
     if (smem) __syncthreads();
