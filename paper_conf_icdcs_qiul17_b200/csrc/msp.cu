@@ -887,12 +887,10 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       return DBG_EINVAL;
     if (part->d_rank) {  // ranks from pass 1: one pass, no atomics
       const unsigned long long* stg = reinterpret_cast<const unsigned long long*>(part->d_staged);
-      int per_sm = 0;
       const int grid = dbg_sm_count() * 8;
 #define DBG_SCATTER_RANK(RW)                                                                                   \
   scatter_rank_kernel<RW><<<grid, 256, 0, stream>>>(part->d_staging, part->d_rank, stg, part->staging_cap,      \
                                                    part->d_record_offset, part->d_records);
-      (void)per_sm;
       if (R == 4) {
         DBG_SCATTER_RANK(4)
       } else if (R == 8) {
