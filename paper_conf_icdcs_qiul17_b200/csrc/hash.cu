@@ -66,6 +66,9 @@
 #ifndef DBG_XEMIT
 #define DBG_XEMIT 0  // extraction emission with explicit shared addresses
 #endif
+#ifndef DBG_KCONST
+#define DBG_KCONST 0  // on-chip kernel specialised for K = 31 / 63
+#endif
 #ifndef DBG_SADDR
 #define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
 #endif
@@ -1257,7 +1260,7 @@ __device__ __forceinline__ void store_vertex16(dbg_vertex* dst, const dbg_vertex
 
 // A group of consecutive fine partitions shares one CTA table: each partition
 // p owns slots [P[p] - P[first], P[p+1] - P[first]).
-template <typename Code, int R, int kSmemThreads, int kMinCtas>
+template <typename Code, int R, int kSmemThreads, int kMinCtas, int KC = 0>
 __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   constexpr uint32_t KB = SmemSlot<KW>::kKeyBytes, FW = SmemSlot<KW>::kFieldWords;
@@ -1272,7 +1275,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   // per 32 slots instead of 32 keys
   uint32_t* occ = fld + a.slots * FW;
   const uint32_t keys_s = smem_addr(keys), fld_s = smem_addr(fld), occ_s = smem_addr(occ);
-  const int K = a.k;
+  const int K = KC ? KC : a.k;  // KC: compile-time K (shifts by constants)
   {  // the table starts clean; extraction keeps it clean (slots is a multiple of 64)
     uint4* z = reinterpret_cast<uint4*>(keys);
     for (uint64_t q = threadIdx.x; q < a.slots * SmemSlot<KW>::kBytes / 16; q += kSmemThreads)
@@ -1979,21 +1982,25 @@ extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
   return smem_slots(prm->k, smem_ctas());
 }
 
-template <typename Code, int R, int T, int C>
+template <typename Code, int R, int T, int C, int KC = 0>
 static cudaError_t launch_smem_t(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
   const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes + (DBG_BITMAP ? a.slots / 8 : 0);
-  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C>,
+  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C, KC>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   if (e != cudaSuccess) return e;
-  smem_subgraph_kernel<Code, R, T, C><<<dbg_sm_count() * C, T, bytes, stream>>>(a, oa);
+  smem_subgraph_kernel<Code, R, T, C, KC><<<dbg_sm_count() * C, T, bytes, stream>>>(a, oa);
   return cudaGetLastError();
 }
 
 template <typename Code, int R>
 static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
   switch (smem_ctas()) {
-    case 0: return launch_smem_t<Code, R, 1024, 1>(a, oa, stream);
+    case 0:
+      // the configurations' K (31, 63) as a compile-time constant in the default variant
+      if (DBG_KCONST && sizeof(Code) == 8 && R == 4 && a.k == 31) return launch_smem_t<Code, R, 1024, 1, 31>(a, oa, stream);
+      if (DBG_KCONST && sizeof(Code) == 16 && R == 8 && a.k == 63) return launch_smem_t<Code, R, 1024, 1, 63>(a, oa, stream);
+      return launch_smem_t<Code, R, 1024, 1>(a, oa, stream);
     case 1: return launch_smem_t<Code, R, 512, 1>(a, oa, stream);
     case 2: return launch_smem_t<Code, R, 256, 2>(a, oa, stream);
     default: return launch_smem_t<Code, R, 128, 4>(a, oa, stream);
