@@ -1998,8 +1998,10 @@ static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_
   switch (smem_ctas()) {
     case 0:
       // the configurations' K (31, 63) as a compile-time constant in the default variant
-      if (DBG_KCONST && sizeof(Code) == 8 && R == 4 && a.k == 31) return launch_smem_t<Code, R, 1024, 1, 31>(a, oa, stream);
-      if (DBG_KCONST && sizeof(Code) == 16 && R == 8 && a.k == 63) return launch_smem_t<Code, R, 1024, 1, 63>(a, oa, stream);
+      if constexpr (DBG_KCONST && sizeof(Code) == 8 && R == 4)
+        if (a.k == 31) return launch_smem_t<Code, R, 1024, 1, 31>(a, oa, stream);
+      if constexpr (DBG_KCONST && sizeof(Code) == 16 && R == 8)
+        if (a.k == 63) return launch_smem_t<Code, R, 1024, 1, 63>(a, oa, stream);
       return launch_smem_t<Code, R, 1024, 1>(a, oa, stream);
     case 1: return launch_smem_t<Code, R, 512, 1>(a, oa, stream);
     case 2: return launch_smem_t<Code, R, 256, 2>(a, oa, stream);
