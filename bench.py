@@ -30,7 +30,7 @@ METRIC = "K-mers hashed/sec (graph build, device-timed) at 1/2/4/8 B200; HBM roo
 UNIT = "kmers/s"
 # version tag of the on-chip kernel: profiles/traffic.json (ncu --set full) is quoted only when it
 # was captured on this version
-KERNEL_VERSION = "smem-v10"
+KERNEL_VERSION = "smem-v11"
 
 
 def _peaks():

@@ -67,7 +67,7 @@
 #define DBG_XEMIT 0  // extraction emission with explicit shared addresses
 #endif
 #ifndef DBG_KCONST
-#define DBG_KCONST 0  // on-chip kernel specialised for K = 31 / 63
+#define DBG_KCONST 1  // on-chip kernel specialised for K = 31 / 63 (default: -1.2 % E. coli, -1.8 % K = 63)
 #endif
 #ifndef DBG_SADDR
 #define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
