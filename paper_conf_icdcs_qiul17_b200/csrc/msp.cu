@@ -267,6 +267,16 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
   ndesc = 0;
 }
 
+#ifndef DBG_MSP_U64_FLUSH
+#define DBG_MSP_U64_FLUSH 0  // 64-bit P-mer codes: flush vote every 16 bases, 18 descriptors (3 CTAs/SM)
+#endif
+// Bases between flush votes and the descriptor capacity: a run of B bases closes
+// at most one superkmer per K-mer plus the read's last one (capacity >= B + 2).
+template <typename CT>
+constexpr int msp_flush_bases() { return (sizeof(CT) == 8 && DBG_MSP_U64_FLUSH) ? 16 : 32; }
+template <typename CT>
+constexpr int msp_max_desc() { return msp_flush_bases<CT>() == 32 ? kMaxDesc : msp_flush_bases<CT>() + 2; }
+
 // kMaxDesc >= 32 + 2: a 32-base chunk closes at most one superkmer per K-mer
 // plus the read's last one, so the flush vote is needed once per chunk.
 template <typename CT>
@@ -276,9 +286,10 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   MspSmem<CT> sm;
   unsigned char* sp = smem_raw;
   sm.desc_m = reinterpret_cast<CT*>(sp);
-  sp += sizeof(CT) * kMaxDesc * kMspThreads;
+  constexpr int kDesc = msp_max_desc<CT>(), kFB = msp_flush_bases<CT>();
+  sp += sizeof(CT) * kDesc * kMspThreads;
   sm.desc_e = reinterpret_cast<uint32_t*>(sp);
-  sp += sizeof(uint32_t) * kMaxDesc * kMspThreads;
+  sp += sizeof(uint32_t) * kDesc * kMspThreads;
   sm.row = reinterpret_cast<CT*>(sp);
 
   const int K = a.k, P = in_reg(a.p), w = in_reg(a.w);
@@ -311,7 +322,9 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
     for (int c0 = 0; c0 < Lmax; c0 += 32) {
       uint64_t wbuf = c0 < L ? window64(a.words, a.n_words, o + c0) : 0;
       const int jn = min(32, L - c0);  // bases of this read in the chunk (<= 0: none)
-      for (int jj = 0; jj < jn; ++jj) {
+#pragma unroll 1
+      for (int h = 0; h < 32; h += kFB) {
+      for (int jj = h; jj < min(jn, h + kFB); ++jj) {
         const int j = c0 + jj;
         const uint32_t b = (uint32_t)(wbuf >> 62);
         wbuf <<= 2;
@@ -352,7 +365,8 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
           ++u;
         }
       }
-      if (__any_sync(kFull, ndesc > kMaxDesc - 34)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+      if (__any_sync(kFull, ndesc > kDesc - (kFB + 2))) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+      }
     }
     if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
   }
@@ -801,7 +815,7 @@ static bool msp_block_launch(const MspArgs& a, int grid, cudaStream_t stream, cu
 
 template <typename CT>
 static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
-  const size_t smem = (sizeof(CT) + sizeof(uint32_t)) * kMaxDesc * kMspThreads + sizeof(CT) * a.w * kMspThreads;
+  const size_t smem = (sizeof(CT) + sizeof(uint32_t)) * msp_max_desc<CT>() * kMspThreads + sizeof(CT) * a.w * kMspThreads;
   cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   grid = msp_grid((const void*)msp_kernel<CT>, grid, smem);
