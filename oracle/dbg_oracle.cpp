@@ -16,12 +16,16 @@
 // SURVEY.md Sec. 8(c) and DESIGN.md "Readings" (letters A..T below).
 //
 // Deliberately slow and obvious: strings are reverse-complemented character
-// by character, every P-mer of every window is re-encoded from characters
-// (Definition 1 by brute force), and counting goes through std::map.
+// by character, every P-mer is encoded from characters (Definition 1: the
+// canonical value of each P-mer, then the minimum over each K-mer's window),
+// and counting goes through std::map.
 //
 // Parity pins for this file: tests/test_oracle_pins.py (Fig. 1 worked
 // example, Python string brute force, (K+1)-mer closed form, invariants
-// I1..I6, Fig. 4 encoding example).
+// I1..I6, Fig. 4 encoding example; fmix64 by SMHasher's published
+// MurmurHash3_x64_128 verification value; oracle_checksum by its per-field
+// closed form over the pinned fmix64; the pid / key filters by the
+// unfiltered graph restricted).
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -136,6 +140,31 @@ uint64_t canonical_minimizer(const std::string& read, size_t i, int K, int P) {
   return (uint64_t)best;  // P <= 31 so the code fits 62 bits
 }
 
+// Definition 1 written in its two steps: first every
+// P-mer position j of the read gets its canonical value
+// c_j = min(enc(S[j..j+P-1]), enc(rc(S[j..j+P-1]))) (reading D), each encoded
+// from characters as above; then the minimizer of the K-mer at i is
+// min_{j in [i, i+K-P]} c_j (window_minimum).  The same values as
+// canonical_minimizer(S, i, K, P), without re-encoding each P-mer K-P+1 times.
+std::vector<uint64_t> canonical_pmer_values(const std::string& read, int P) {
+  std::vector<uint64_t> c;
+  for (size_t j = 0; j + P <= read.size(); ++j) {
+    u128 f = 0, r = 0;
+    for (int t = 0; t < P; ++t) f = (f << 2) | (u128)code_of(read[j + t]);  // enc(s_j)
+    for (int t = P - 1; t >= 0; --t)                                          // enc(rc(s_j))
+      r = (r << 2) | (u128)code_of(complement(read[j + t]));
+    c.push_back((uint64_t)(f < r ? f : r));
+  }
+  return c;
+}
+
+uint64_t window_minimum(const std::vector<uint64_t>& c, size_t i, int K, int P) {
+  uint64_t best = ~(uint64_t)0;
+  for (size_t j = i; j <= i + (size_t)(K - P); ++j)
+    if (c[j] < best) best = c[j];
+  return best;
+}
+
 uint32_t partition_of(uint64_t minimizer, int NP) {
   return (uint32_t)(fmix64(minimizer) % (uint64_t)NP);
 }
@@ -229,7 +258,10 @@ int oracle_graph_filtered(const char* seq, const uint64_t* offs, uint64_t n_read
     for (uint64_t r = r0; r < r1; ++r) {
       std::string S = read_string(seq, offs, r);
       if (S.size() < (size_t)K) continue;  // reading N: no K-mers
+      const std::vector<uint64_t> c = canonical_pmer_values(S, P);
       for (size_t i = 0; i + K <= S.size(); ++i) {
+        const uint32_t pid = partition_of(window_minimum(c, i, K, P), NP);
+        if (pid_filter && !pid_filter[pid]) continue;
         if (key_filter) {
           std::string x = S.substr(i, K);
           u128 fx = encode(x), ry = encode(reverse_complement(x));
@@ -244,8 +276,6 @@ int oracle_graph_filtered(const char* seq, const uint64_t* offs, uint64_t n_read
           }
           if (a == n_keys || key_filter[2 * a] != hi || key_filter[2 * a + 1] != lo) continue;
         }
-        uint32_t pid = partition_of(canonical_minimizer(S, i, K, P), NP);
-        if (pid_filter && !pid_filter[pid]) continue;
         add_occurrence(S, i, K, maps[t][pid]);
       }
     }

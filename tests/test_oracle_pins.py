@@ -297,6 +297,118 @@ def test_checksum_order_independent(oracle_lib):
     assert brute.fmix64(0) == 0
 
 
+def _murmur3_x64_128(data: bytes, seed: int, fmix, c1: int, c2: int) -> bytes:
+    """MurmurHash3_x64_128 (Appleby, SMHasher) with its finaliser taken from the oracle: body
+    blocks of 16 bytes, tail, length, then fmix64 of both halves.  Only fmix64 is the oracle's."""
+    M = (1 << 64) - 1
+
+    def rotl(x, r):
+        return ((x << r) | (x >> (64 - r))) & M
+
+    n, nb = len(data), len(data) // 16
+    h1 = h2 = seed
+    for i in range(nb):
+        k1 = int.from_bytes(data[16 * i:16 * i + 8], "little")
+        k2 = int.from_bytes(data[16 * i + 8:16 * i + 16], "little")
+        k1 = (rotl((k1 * c1) & M, 31) * c2) & M
+        h1 ^= k1
+        h1 = (((rotl(h1, 27) + h2) & M) * 5 + 0x52DCE729) & M
+        k2 = (rotl((k2 * c2) & M, 33) * c1) & M
+        h2 ^= k2
+        h2 = (((rotl(h2, 31) + h1) & M) * 5 + 0x38495AB5) & M
+    tail = data[16 * nb:]
+    if len(tail) > 8:
+        h2 ^= (rotl((int.from_bytes(tail[8:], "little") * c2) & M, 33) * c1) & M
+    if len(tail) > 0:
+        h1 ^= (rotl((int.from_bytes(tail[:8], "little") * c1) & M, 31) * c2) & M
+    h1 ^= n
+    h2 ^= n
+    h1 = (h1 + h2) & M
+    h2 = (h2 + h1) & M
+    h1, h2 = fmix(h1), fmix(h2)
+    h1 = (h1 + h2) & M
+    h2 = (h2 + h1) & M
+    return h1.to_bytes(8, "little") + h2.to_bytes(8, "little")
+
+
+def test_fmix64_pinned_by_murmurhash3_verification_value(oracle_lib):
+    """Reading I: the partition hash is MurmurHash3's finaliser fmix64.  Pinned by SMHasher's
+    published verification value of MurmurHash3_x64_128 (tests/golden/murmur3_verification.txt),
+    computed here with the oracle's fmix64 as the finaliser."""
+    g = dict(l.split() for l in open(os.path.join(GOLD, "murmur3_verification.txt")) if l.strip() and l[0] != "#")
+    c1, c2 = int(g["C1"], 16), int(g["C2"], 16)
+    key = bytearray(256)
+    hashes = b""
+    for i in range(256):
+        key[i] = i
+        hashes += _murmur3_x64_128(bytes(key[:i]), 256 - i, oracle_lib.fmix64, c1, c2)
+    final = _murmur3_x64_128(hashes, 0, oracle_lib.fmix64, c1, c2)
+    assert int.from_bytes(final[:4], "little") == int(g["VERIFICATION"], 16)
+    assert oracle_lib.fmix64(0) == 0  # the fixed point the checksum closed form below relies on
+
+
+def test_checksum_closed_form_pins_field_order(oracle_lib):
+    """SURVEY.md 8(d) checksum: per record h = 0, then h = fmix64(h ^ field) over the 11 fields
+    key_hi, key_lo, count, out[0..3], in[0..3]; the checksum is the sum of h mod 2^64.  Because
+    fmix64(0) = 0 (pinned above), a record whose only nonzero field is field j (0-based) with
+    value x has h = fmix64 applied 11 - j times to x -- so the position of every field, the number
+    of fields and the exclusion of pid are fixed by iterating the pinned fmix64, not by the
+    checksum code.  Two nonzero fields i < j combine as fmix^(11-j)(fmix^(j-i)(a) ^ b)."""
+
+    def it(x, n):
+        for _ in range(n):
+            x = oracle_lib.fmix64(x)
+        return x
+
+    slots = [("key_hi", None), ("key_lo", None), ("count", None)] + [("out", c) for c in range(4)] + \
+            [("in", c) for c in range(4)]
+
+    def rec(vals):
+        r = np.zeros(1, dtype=oracle_lib.VERTEX_DTYPE)
+        for j, v in vals.items():
+            name, c = slots[j]
+            if c is None:
+                r[name] = v
+            else:
+                r[name][0, c] = v
+        return r
+
+    assert oracle_lib.checksum(np.zeros(3, dtype=oracle_lib.VERTEX_DTYPE)) == 0
+    for j in range(11):
+        x = 0x1234 + 977 * j
+        assert oracle_lib.checksum(rec({j: x})) == it(x, 11 - j), j
+    M = (1 << 64) - 1
+    for i, j in ((0, 1), (1, 2), (2, 6), (3, 7), (6, 10), (0, 10)):
+        a, b = 0xABCDEF + i, 0x31337 + j
+        assert oracle_lib.checksum(rec({i: a, j: b})) == it(it(a, j - i) ^ b, 11 - j), (i, j)
+    r = rec({0: 5, 2: 7})
+    r2 = r.copy()
+    r2["pid"] = 12345
+    assert oracle_lib.checksum(r2) == oracle_lib.checksum(r)          # pid is not a checksum field
+    both = np.concatenate([rec({1: 9}), rec({4: 3})])
+    assert oracle_lib.checksum(both) == (it(9, 10) + it(3, 7)) & M    # sum over records mod 2^64
+
+
+def test_oracle_filters_equal_the_unfiltered_graph_restricted(oracle_lib):
+    """The pid and key filters (sampled parity at full size) only drop occurrences: the filtered
+    graph is exactly the unfiltered graph restricted to those partitions / vertices."""
+    rs = random_reads(400, 20, 150, seed=91, n_rate=0.01)
+    K, P, NP = 21, 7, 16
+    full = oracle_lib.graph(rs.seq, rs.offsets, K, P, NP, n_threads=3)
+    for pids in ([], [0], [3, 7, 11], list(range(NP))):
+        got = oracle_lib.graph(rs.seq, rs.offsets, K, P, NP, n_threads=2, pids=pids)
+        assert got.tobytes() == full[np.isin(full["pid"], pids)].tobytes(), pids
+    rng = np.random.default_rng(5)
+    pick = full[rng.choice(len(full), 50, replace=False)]
+    keys = np.stack([pick["key_hi"], pick["key_lo"]], 1)
+    absent = np.array([[0, (1 << 42) + 12345], [0, 7]], dtype=np.uint64)  # codes not in the graph
+    absent = absent[~np.isin(absent[:, 1], full["key_lo"])]
+    got = oracle_lib.graph(rs.seq, rs.offsets, K, P, NP, keys=np.concatenate([keys, absent]))
+    assert got.tobytes() == np.sort(pick, order=["key_hi", "key_lo"]).tobytes()
+    both = oracle_lib.graph(rs.seq, rs.offsets, K, P, NP, pids=[int(pick["pid"][0])], keys=keys)
+    assert both.tobytes() == np.sort(pick[pick["pid"] == pick["pid"][0]], order=["key_hi", "key_lo"]).tobytes()
+
+
 # ---------------------------------------------------------------- row f4: low-count filtering
 
 
