@@ -7,9 +7,9 @@ fallback -- if libdbg.so is missing, calls raise.
 from . import _lib
 from ._lib import VERTEX_DTYPE, DbgError, load
 from .stream import StreamingBuilder, build_graph_streamed, plan_ranges
-from .graph import (DbgBuilder, GraphResult, auto_fine_p, auto_refine, build_graph, encode_reads, read_graph,
+from .graph import (DbgBuilder, GraphResult, auto_fine_p, auto_refine, build_graph, encode_reads, launch_builder, read_graph,
                     write_graph)
 
 __all__ = ["_lib", "VERTEX_DTYPE", "DbgError", "load", "DbgBuilder", "GraphResult", "auto_fine_p", "auto_refine",
-           "build_graph", "encode_reads", "read_graph", "write_graph",
+           "build_graph", "encode_reads", "launch_builder", "read_graph", "write_graph",
            "StreamingBuilder", "build_graph_streamed", "plan_ranges"]

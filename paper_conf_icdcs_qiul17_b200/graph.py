@@ -195,6 +195,18 @@ class DbgBuilder:
         asynchronously, pass 2 (scatter).  Nothing here waits for the device: sync_sizes() reads
         the sizes when the host needs them, after the device work behind them is enqueued."""
         stream = stream or torch.cuda.current_stream(self.device)
+        self.msp_pass1(d_bases, d_offsets, stream)
+        # room for every staged record: after an overflow pass 2 and Step 2 do nothing (dbg.h)
+        self.records = _grow(self.records, self.staging.numel(), torch.int32, self.device)
+        ev = self._mark("msp_scatter", stream)
+        _lib.dbg_msp_partition(self.prm, d_bases, d_bases.numel(), d_offsets, d_offsets.numel() - 1,
+                               self.part_set(True), stream)
+        self._done(ev, stream)
+
+    def msp_pass1(self, d_bases: torch.Tensor, d_offsets: torch.Tensor, stream=None):
+        """Pass 1 of Step 1 only (minimizers, superkmers into the staging, per-partition sizes),
+        and the asynchronous copy of the sizes (sync_sizes)."""
+        stream = stream or torch.cuda.current_stream(self.device)
         n_reads = d_offsets.numel() - 1
         n_words = d_bases.numel()
         if self.staging.numel() == 0:
@@ -211,11 +223,6 @@ class DbgBuilder:
             self._h_sizes[self.np:].copy_(self.d_n_kmers, non_blocking=True)
         self._sizes_ev.record(stream)
         self._sizes_pending = True
-        # room for every staged record: after an overflow pass 2 and Step 2 do nothing (dbg.h)
-        self.records = _grow(self.records, self.staging.numel(), torch.int32, self.device)
-        ev = self._mark("msp_scatter", stream)
-        _lib.dbg_msp_partition(self.prm, d_bases, n_words, d_offsets, n_reads, self.part_set(True), stream)
-        self._done(ev, stream)
 
     def msp_overlapped(self, h_packed: torch.Tensor, h_offsets: torch.Tensor, d_bases: torch.Tensor,
                        d_offsets: torch.Tensor, n_batches: int = 8, stream=None, copy_stream=None):
@@ -278,34 +285,6 @@ class DbgBuilder:
             self.staging = _grow(self.staging, total * self.rec_words, torch.int32, self.device, 1.05)
             self.overflowed = True
         return not self.overflowed
-
-    def load_exchanged(self, received: torch.Tensor, n_received: int, global_records: np.ndarray,
-                       global_kmers: np.ndarray, owned: tuple[int, int], stream=None) -> None:
-        """Multi-GPU: after the record exchange, make this builder's partition set describe only
-        the owned fine partitions [lo, hi) (records received from every rank, scattered into
-        partition order by dbg_msp_partition pass 2; sizes summed over ranks)."""
-        stream = stream or torch.cuda.current_stream(self.device)
-        lo, hi = owned
-        self.owned = (lo, hi)
-        rec = np.zeros(self.np, dtype=np.int64)
-        kmr = np.zeros(self.np, dtype=np.int64)
-        rec[lo:hi] = global_records[lo:hi]
-        kmr[lo:hi] = global_kmers[lo:hi]
-        off = np.zeros(self.np + 1, dtype=np.int64)
-        off[1:] = np.cumsum(rec)
-        assert int(off[-1]) == n_received, (int(off[-1]), n_received)
-        self.part_records, self.part_kmers = rec, kmr
-        self._sizes_pending = False
-        self.overflowed = False
-        with torch.cuda.stream(stream):
-            self.d_n_records.copy_(torch.from_numpy(rec), non_blocking=True)
-            self.d_n_kmers.copy_(torch.from_numpy(kmr), non_blocking=True)
-            self.d_rec_off.copy_(torch.from_numpy(off), non_blocking=True)
-            self.d_staged.fill_(n_received)
-        self.staging = received
-        self._rank_valid = False  # the received records were not ranked by this set's pass 1
-        self.records = _grow(self.records, n_received * self.rec_words, torch.int32, self.device, 1.05)
-        _lib.dbg_msp_partition(self.prm, 1, 1, self.d_rec_off, 0, self.part_set(True), stream)
 
     # ------------------------------------------------------------------ a5
     def plan(self, stream=None) -> list[tuple[int, int]]:
@@ -573,6 +552,17 @@ def auto_fine_p(n_kmers: int, k: int, p: int, lam: float = 2.0, alpha: float = 0
         if 4.0 ** q >= 4.0 * (k - q + 1) * n_kmers * ratio / slots:
             return q
     return min(k, 31)
+
+
+def launch_builder(k: int, p: int, num_partitions: int, n_kmers: int, lam: float = 2.0, alpha: float = 0.5,
+                   device="cuda", min_count: int = 0, **kw) -> DbgBuilder:
+    """The builder in the launch configuration bench.py times: on-chip Step 2 with the automatic
+    refinement F (auto_refine) and device minimizer length P' (auto_fine_p) for a workload of
+    n_kmers K-mers.  The full-size parity tests use the same function."""
+    refine = kw.pop("refine", None) or auto_refine(n_kmers, k, p, num_partitions, lam, alpha)
+    fine_p = kw.pop("fine_p", None) or auto_fine_p(n_kmers, k, p, lam, alpha)
+    return DbgBuilder(k, p, num_partitions, lam, alpha, device, refine=refine, fine_p=fine_p, min_count=min_count,
+                      **kw)
 
 
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,

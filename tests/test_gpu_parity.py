@@ -254,97 +254,6 @@ def test_strand_symmetry_on_gpu():
     assert a.vertices.tobytes() == b.vertices.tobytes()
 
 
-def _mirror_violations(v, k):
-    """I3 on a vertex array: every out-edge has its mirror in-edge (or out-edge) at the neighbour."""
-    code = v["kmer_lo"].astype(object) + (v["kmer_hi"].astype(object) << 64)
-    idx = {int(c): i for i, c in enumerate(code)}
-    mask = (1 << (2 * k)) - 1
-    bad = 0
-    for i in range(0, len(v), max(1, len(v) // 3000)):
-        c = int(code[i])
-        first = c >> (2 * k - 2)
-        for b in range(4):
-            m = int(v["out"][i][b])
-            if not m:
-                continue
-            w = ((c << 2) | b) & mask
-            rcw = 0
-            x = w
-            for _ in range(k):
-                rcw = (rcw << 2) | (3 - (x & 3))
-                x >>= 2
-            if w <= rcw:
-                bad += int(v["in"][idx[w]][first] != m)
-            else:
-                bad += int(v["out"][idx[rcw]][3 - first] != m)
-    return bad
-
-
-@pytest.mark.parametrize("name", ["ecoli"])
-def test_full_size_config_sampled(name):
-    """BASELINE configs[1] at full size, in the launch configuration bench.py times: invariants at
-    any size (I1, I2, I3 mirror on a sample) and oracle parity on 4000 sampled vertices."""
-    rs = make_config(name)
-    k, p, np_ = rs.k, rs.p, rs.num_partitions
-    res = build_graph(rs.seq, rs.offsets, k, p, np_)
-    v = res.vertices
-    L = rs.lengths()
-    assert res.stats["sum_count"] == int(np.maximum(L - k + 1, 0).sum())             # I1
-    assert res.stats["sum_edges"] == 2 * int(np.maximum(L - k, 0).sum())             # I2
-    assert res.stats["distinct"] == len(v)
-    assert np.all(v["kmer_lo"][1:] > v["kmer_lo"][:-1])                               # sorted, unique
-    assert _mirror_violations(v, k) == 0                                               # I3
-    rng = np.random.default_rng(17)
-    sel = v[np.sort(rng.choice(len(v), size=4000, replace=False))]
-    orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT,
-                       keys=np.stack([sel["kmer_hi"], sel["kmer_lo"]], 1))
-    compare_vertices(sel, orc)
-
-
-def test_sharded_path_two_logical_ranks_one_gpu():
-    """Row e on one GPU: two 'ranks' each run MSP on half of the reads, records are routed to the
-    owners of their fine partitions exactly as multi.exchange_records does (slices in partition
-    order), each owner builds its partitions -- the union equals the oracle on all reads."""
-    from paper_conf_icdcs_qiul17_b200.multi import owner_bounds, send_counts
-
-    g = genome(40_000, seed=9)
-    seq, offs = make_reads(g, 6000, 100, 0.01, seed=10)
-    rs = ReadSet(seq, offs)
-    k, p, np_, refine = 31, 11, 8, 8
-    halves = [rs.subset(0, 3000), rs.subset(3000, 6000)]
-    bs = []
-    for h in halves:
-        b = DbgBuilder(k, p, np_, refine=refine)
-        d_bases, d_off = b.upload(encode_reads(h.seq), h.offsets)
-        b.msp(d_bases, d_off)
-        assert b.sync_sizes()
-        bs.append(b)
-    n_fine = bs[0].np
-    bounds = owner_bounds(n_fine, 2)
-    g_rec = bs[0].part_records + bs[1].part_records
-    g_kmr = bs[0].part_kmers + bs[1].part_kmers
-    R = bs[0].rec_words
-    outs = []
-    for owner in range(2):
-        parts = []
-        for b in bs:
-            sc = np.concatenate([[0], np.cumsum(send_counts(b.part_records, bounds))])
-            parts.append(b.records[sc[owner] * R: sc[owner + 1] * R])
-        recv = torch.cat(parts)
-        n = recv.numel() // R
-        ob = DbgBuilder(k, p, np_, refine=refine)
-        ob.load_exchanged(recv, n, g_rec, g_kmr, (int(bounds[owner]), int(bounds[owner + 1])))
-        ob.plan()
-        ob.reset_output(max(n * 16, 1024))
-        ob.step2()
-        assert _lib.dbg_sync_status(ob.d_status) == 0
-        outs.append(ob.vertices(sort=False))
-    allv = np.concatenate(outs)
-    allv = allv[np.lexsort((allv["kmer_lo"], allv["kmer_hi"]))]
-    orc = oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT)
-    compare_vertices(allv, orc)
-
-
 def test_smem_global_tier_in_several_batches():
     """Oversize partitions whose global tables do not fit the table budget at once are built in
     several batches (each batch's table block starts at its first partition)."""
