@@ -1,22 +1,34 @@
 #!/usr/bin/env python
 """Benchmark of the ParaHash hot path on B200: K-mers hashed per second (graph build, device-timed).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config ecoli] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config chr14] [--impl ours|reference]
 
-One step = one pass of the whole hot path over the synthetic read set
-of the chosen configuration: MSP count pass -> size readback -> MSP emit pass -> table plan ->
-table zero-fill -> hash build.  Extraction (a7) is timed separately (``extract_ms``) and is part of
-the ``e2e`` number, which also includes the H2D of the packed reads and the D2H of the stats.
+One step = one pass of the whole hot path over the configuration's
+synthetic reads, resident in HBM: MSP pass 1 -> size readback -> MSP pass 2 (scatter into
+partition order) -> on-chip Step 2 (table sizing, hashing, extraction of the vertex records) ->
+global-table tier for the partitions too large for one SM.  The default workload is chr14
+(BASELINE.json configs[2], the largest configuration that fits one GPU).
 
-Prints ONE JSON line (rank 0).  See DESIGN.md Sec. 7 for the roofline arithmetic.
+``value`` is device-timed (CUDA events on the launching stream, L2 flushed before every step).
+``e2e`` is the same workload through the public API with the paper's timing scope (P:L979-987:
+"ends at the time all the subgraphs are constructed in main memory", transfers included): H2D of
+the packed reads from pinned memory (overlapped with MSP), the device path, and the D2H of every
+vertex record into pinned host memory.
+
+N > 1 (``--gpus N``; re-launches itself under torch.distributed.run when started without it):
+strong scaling -- the configuration's reads are split into N contiguous ranges, one per rank; each
+step is multi.ShardedBuilder.step (local MSP, emission of the records into their owners' buffers
+through peer pointers, Step 2 of the owned partitions); times are the max over ranks.
+
+Prints ONE JSON line (rank 0).  DESIGN.md Sec. 7 has the roofline arithmetic.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
-import subprocess
 import sys
 import threading
 import time
@@ -28,18 +40,22 @@ sys.path.insert(0, ROOT)
 
 METRIC = "K-mers hashed/sec (graph build, device-timed) at 1/2/4/8 B200; HBM roofline %"
 UNIT = "kmers/s"
+# algorithmic bytes per K-mer occurrence of the hot path -- one 32-B sector read +
+# write-back of the vertex's table entry (64 B, the random-access HBM table the north star's
+# roofline assumes) + ~4 B of streaming (packed reads, superkmer records written and read back)
+ALG_BYTES_PER_KMER = 68
 # version tag of the on-chip kernel: profiles/traffic.json (ncu --set full) is quoted only when it
-# was captured on this version
-KERNEL_VERSION = "smem-v11"
+# was captured on this version and workload
+KERNEL_VERSION = "smem-v12"
 
 
 def _peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             d = json.load(f)
-        return float(d["hbm_gbs"]), "measured"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
     except Exception:
-        return 6650.0, "fallback"
+        return 6650.0, "fallback (B200_PROFILING.md)"
 
 
 class ClockSampler:
@@ -112,23 +128,36 @@ def _dist():
     return ws, rank, local
 
 
-def _workload(args):
-    from synth import make_config
+def _relaunch_under_torchrun(n: int) -> int:
+    """`python bench.py --gpus N` without a launcher: start N ranks (one per GPU) ourselves."""
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    import subprocess
 
-    t = time.time()
-    rs = make_config(args.config, scale=args.scale, num_partitions=args.np)
-    if args.p is not None:
-        rs.p = args.p
-    return rs, time.time() - t
+    return subprocess.call(cmd)
 
 
-def _config_json(rs, args, extra=None):
-    c = {"workload": rs.name, "genome_bp": rs.meta["genome"], "reads": rs.n_reads,
+def _config_kmers(name: str, scale: float) -> tuple[int, int]:
+    """(reads, K-mer occurrences) of a configuration without generating it (fixed read length)."""
+    from synth import CONFIGS
+
+    c = CONFIGS[name]
+    n = max(int(c["reads"] * scale), 1)
+    return n, n * max(c["read_len"] - c["k"] + 1, 0)
+
+
+def _config_json(rs, args, n_reads_total: int, n_kmers_total: int, extra=None):
+    c = {"workload": rs.name, "desc": rs.meta["desc"], "genome_bp": rs.meta["genome"], "reads": n_reads_total,
          "read_len": rs.meta["read_len"], "error_rate": rs.meta["error"], "k": rs.k, "p": rs.p,
          "num_partitions": rs.num_partitions, "lambda": args.lam, "alpha": args.alpha,
-         "kmers_per_step": rs.n_kmers(), "scale": args.scale,
+         "kmers_per_step": n_kmers_total, "scale": args.scale,
          "l2": "flushed between timed steps (512 MiB write); step working set > L2",
-         "parallelism": f"partitions sharded over {args.gpus} GPU(s)"}
+         "parallelism": "one GPU" if args.gpus == 1 else
+         f"dp{args.gpus}: reads split by range, fine partitions owned by rank (emission into peer buffers)"}
     if extra:
         c.update(extra)
     return c
@@ -145,7 +174,6 @@ def _oracle_rate(rs, seconds: float, threads: int):
     sub = rs.subset(0, n)
     oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
     dt = max(time.time() - t, 1e-3)
-    rate = sub.n_kmers() / dt
     n2 = int(min(rs.n_reads, max(n, n * seconds / dt)))
     sub = rs.subset(0, n2)
     t = time.time()
@@ -154,11 +182,23 @@ def _oracle_rate(rs, seconds: float, threads: int):
     return sub.n_kmers() / dt, sub, dt
 
 
+def _oracle_single_thread_ecoli(seconds: float = 4.0) -> dict:
+    """the oracle's single-thread K-mer rate on the E. coli-shaped config (configs[1])."""
+    from synth import make_config
+
+    rs = make_config("ecoli")
+    rate, sub, dt = _oracle_rate(rs, seconds, 1)
+    return {"value": rate, "unit": UNIT, "cores": 1, "workload": "ecoli",
+            "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
+
+
 def run_reference(args):
     ws, rank, _ = _dist()
     if rank != 0:
         return 0
-    rs, _ = _workload(args)
+    from synth import make_config
+
+    rs = make_config(args.config, scale=args.scale, num_partitions=args.np)
     threads = os.cpu_count() or 1
     import oracle
 
@@ -177,8 +217,8 @@ def run_reference(args):
     sample = f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers) per step"
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
-            "data": "synthetic", "config": _config_json(rs, args),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic", "config": _config_json(rs, args, rs.n_reads, rs.n_kmers()),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -200,75 +240,77 @@ def _placement(b) -> dict:
             "global": float(pk[place == 0].sum()) / tot, "split_ctas": int(place[place >= 2].sum())}
 
 
+def _profile_facts(workload: str) -> dict:
+    """ncu facts of the dominant kernel for this workload (profiles/traffic.json, written from a
+    committed `ncu --set full` capture); stale=True when captured on another kernel version."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            tr = json.load(f).get(workload)
+    except Exception:
+        tr = None
+    if not tr:
+        return {"stale": True, "source": None}
+    return dict(tr, stale=tr.get("kernel_version") != KERNEL_VERSION)
+
+
 def run_ours(args):
-    """Our arm.  N = 1: the whole path on one GPU.  N > 1 (torchrun): one process per GPU, weak
-    scaling -- every rank owns a read set of the configuration's size (same genome, its own reads);
-    a step is multi.distributed_step (local MSP, one record exchange to the partition owners,
-    owned-partition Step 2, NCCL reduces), timed on each rank's stream, max over ranks."""
+    """Our arm (module docstring)."""
     import torch
 
     ws, rank, local = _dist()
+    if ws != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={ws}: launch with torchrun --nproc-per-node {args.gpus}")
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    from paper_conf_icdcs_qiul17_b200 import DbgBuilder, auto_fine_p, auto_refine, encode_reads, _lib
+    from paper_conf_icdcs_qiul17_b200 import encode_reads, launch_builder, _lib
+    from synth import make_config
 
     dist = None
     if ws > 1:
         import torch.distributed as dist
-        from paper_conf_icdcs_qiul17_b200 import multi
+        from paper_conf_icdcs_qiul17_b200.multi import ShardedBuilder
 
         dist.init_process_group("nccl", device_id=dev)
+    n_reads_total, n_kmers_total = _config_kmers(args.config, args.scale)
     t = time.time()
-    from synth import make_config
-
-    rs = make_config(args.config, scale=args.scale, num_partitions=args.np, read_seed_offset=7919 * rank)
-    if args.p is not None:
-        rs.p = args.p
+    rs = make_config(args.config, scale=args.scale, num_partitions=args.np, shard=(rank, ws) if ws > 1 else None)
     gen_s = time.time() - t
     packed = encode_reads(rs.seq, pin=True)
     offsets = torch.from_numpy(rs.offsets.view(np.int64)).pin_memory()
-    n_kmers = rs.n_kmers()
     stream = torch.cuda.current_stream(dev)
-    refine = args.refine
-    if refine is None:
-        refine = auto_refine(n_kmers, rs.k, rs.p, rs.num_partitions, args.lam, args.alpha) if args.mode == "smem" else 1
-    fine_p = args.fine_p
-    if fine_p is None:
-        fine_p = auto_fine_p(n_kmers, rs.k, rs.p, args.lam, args.alpha) if args.mode == "smem" else 0
-    if ws > 1 and args.mode != "smem":
-        raise SystemExit("multi-GPU runs use mode smem")
-    b = DbgBuilder(rs.k, rs.p, rs.num_partitions, args.lam, args.alpha, dev, args.table_budget, args.mode,
-                   args.group_slots, refine, args.smem_split, fine_p, args.min_count)
-    d_bases, d_off = b.upload(packed, offsets, stream)
+    kw = {}
+    if args.refine:
+        kw["refine"] = args.refine
+    if args.fine_p:
+        kw["fine_p"] = args.fine_p
+    if ws > 1:
+        sb = ShardedBuilder(rs.k, rs.p, rs.num_partitions, n_kmers_total, dev, lam=args.lam, alpha=args.alpha,
+                            min_count=args.min_count, **kw)
+        src, b = sb.src, sb.dst
+    else:
+        b = src = launch_builder(rs.k, rs.p, rs.num_partitions, n_kmers_total, args.lam, args.alpha, device=dev,
+                                 min_count=args.min_count, **kw)
+    d_bases, d_off = src.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
     # output capacity: distinct vertices <= K-mers; 0.4 x covers the configs' error rates (a build
     # that overflows it reports DBG_ENOSPACE and the invariant check fails loudly)
-    out_cap = int(args.out_frac * n_kmers) + 1024
-
-    host_ms = {"msp": [], "plan": [], "reset": [], "step2": []}
+    out_cap = int(args.out_frac * n_kmers_total / ws) + (1 << 20)
 
     def step(db, do):
-        """One pass of rows a2-a7 (MSP, sizing, on-chip / global Step 2) on this rank."""
+        """One pass of rows a2-a7 on this rank."""
         if ws > 1:
-            multi.distributed_step(b, db, do, stream, out_cap)
+            sb.step(db, do, stream, out_cap)
             return
-        t = time.perf_counter()
         b.msp(db, do, stream)
-        t1 = time.perf_counter()
         b.plan(stream)
-        t2 = time.perf_counter()
         b.reset_output(out_cap, stream)
-        t3 = time.perf_counter()
         b.step2(stream)
-        t4 = time.perf_counter()
-        for k, v in zip(("msp", "plan", "reset", "step2"), (t1 - t, t2 - t1, t3 - t2, t4 - t3)):
-            host_ms[k].append(1e3 * v)
 
     def barrier():
         torch.cuda.synchronize()
         if dist is not None:
-            dist.barrier()
+            dist.barrier(device_ids=[local])
 
     def max_over_ranks(x: float) -> float:
         if dist is None:
@@ -282,7 +324,7 @@ def run_ours(args):
     st = _lib.dbg_sync_status(b.d_status, stream)
     assert st == 0, _lib.dbg_status_string(st)
 
-    b.timer = {}
+    src.timer = b.timer = {}
     step_ms = []
     with ClockSampler(local) as clk:
         for _ in range(args.steps):
@@ -295,29 +337,38 @@ def run_ours(args):
             barrier()
             step_ms.append(e0.elapsed_time(e1))
     phases = {k: statistics.mean(a.elapsed_time(c) for a, c in v) for k, v in b.timer.items()}
-    b.timer = None
+    src.timer = b.timer = None
     st = _lib.dbg_sync_status(b.d_status, stream)
     stats = b.stats()
+    n_out = int(b.d_n_out.item())
     L = rs.lengths()
-    tot = torch.tensor([n_kmers, stats["sum_count"], stats["sum_edges"], stats["distinct"],
-                        2 * int(np.maximum(L - rs.k, 0).sum()), int(st == 0)], dtype=torch.int64, device=dev)
+    tot = torch.tensor([rs.n_kmers(), stats["sum_count"], stats["sum_edges"], stats["distinct"],
+                        2 * int(np.maximum(L - rs.k, 0).sum()), int(st == 0),
+                        int(np.array(stats["checksum"], dtype=np.uint64).view(np.int64))],
+                       dtype=torch.int64, device=dev)
     if dist is not None:
-        dist.all_reduce(tot)
-    total_kmers, sum_count, sum_edges, distinct, want_edges, ok_ranks = (int(x) for x in tot.cpu())
+        dist.all_reduce(tot)  # int64 sums wrap: the checksum sum stays exact mod 2^64
+    total_kmers, sum_count, sum_edges, distinct, want_edges, ok_ranks, checksum = (int(x) for x in tot.cpu())
+    checksum &= (1 << 64) - 1
+    assert total_kmers == n_kmers_total, (total_kmers, n_kmers_total)
     inv_ok = ok_ranks == ws and sum_count == total_kmers and sum_edges == want_edges
 
-    # e2e through the public API: H2D of the packed reads (pinned) + path + D2H of the stats.
-    # N = 1: DbgBuilder.msp_overlapped uploads the reads in 8 read ranges on a copy stream and
-    # starts MSP on each range as soon as it has arrived (the f2 overlap of transfer and compute).
-    e2e_ms, h2d_ms = [], []
+    # e2e through the public API with the paper's timing scope: H2D of the packed reads (pinned;
+    # N = 1: overlapped with MSP, DbgBuilder.msp_overlapped), the path, the readback of the vertex
+    # count, and the D2H of every vertex record (n_out x 56 B) into pinned host memory
+    e2e_ms, h2d_ms, d2h_ms = [], [], []
     db = torch.empty_like(d_bases)
     do = torch.empty_like(d_off)
+    vbytes = b.vdtype.itemsize
+    host_out = torch.empty(int(n_out * 1.02 + 1024) * vbytes, dtype=torch.uint8, pin_memory=True)
+    host_n = torch.empty(1, dtype=torch.int64, pin_memory=True)
     host_stats = torch.empty(4, dtype=torch.int64, pin_memory=True)
     cs = torch.cuda.Stream(dev)
+    d2h_bytes = 0
     for _ in range(max(3, min(args.steps, 5))):
         flush.zero_()
         barrier()
-        e0, e1, eh = E(), E(), E()
+        e0, e1, eh, ed = E(), E(), E(), E()
         e0.record(stream)
         if ws == 1:
             b.msp_overlapped(packed, offsets, db, do, 8, stream, cs)
@@ -326,102 +377,105 @@ def run_ours(args):
             b.reset_output(out_cap, stream)
             b.step2(stream)
         else:
-            db.copy_(packed, non_blocking=True)   # H2D of the step's input from pinned memory
+            db.copy_(packed, non_blocking=True)   # H2D of this rank's reads from pinned memory
             do.copy_(offsets, non_blocking=True)
             eh.record(stream)
             step(db, do)
-        host_stats.copy_(b.d_stats, non_blocking=True)  # D2H of the step's result
+        host_n.copy_(b.d_n_out, non_blocking=True)
+        stream.synchronize()                      # the host needs the vertex count to size the copy
+        n = int(host_n.item())
+        ed.record(stream)
+        if n * vbytes > host_out.numel():
+            raise RuntimeError(f"{n} vertices exceed the pinned output buffer")
+        host_out[:n * vbytes].copy_(b.out[:n * vbytes], non_blocking=True)   # the subgraphs in host memory
+        host_stats.copy_(b.d_stats, non_blocking=True)
         e1.record(stream)
         barrier()
         e2e_ms.append(max_over_ranks(e0.elapsed_time(e1)))
         h2d_ms.append(e0.elapsed_time(eh))
+        d2h_ms.append(ed.elapsed_time(e1))
+        d2h_bytes = n * vbytes + 8 + 32
     h2d = packed.numel() * 8 + offsets.numel() * 8
-    d2h = 32
 
     ms = max_over_ranks(statistics.mean(step_ms))
-    key = {"fused": "step2", "resident": "hash_build", "smem": "step2_smem"}[args.mode]
-    hash_ms = phases.get(key, float("nan")) + (phases.get("hash_build", 0.0) + phases.get("extract", 0.0)
-                                               if args.mode == "smem" else 0.0)
-    # this rank's Step-2 work (after the exchange: the K-mers of its own partitions)
-    my_kmers = int(b.part_kmers.sum())
+    hash_ms = phases.get("step2_smem", 0.0) + phases.get("hash_build", 0.0) + phases.get("extract", 0.0)
+    my_kmers = int(b.part_kmers.sum())         # this rank's Step-2 K-mers (its owned partitions)
     n_records = int(b.part_records.sum())
-    # one 32-B sector read + write-back per K-mer occurrence (the paper's
-    # random-access table RMW) + the records read + the vertex records written
-    alg_bytes = my_kmers * 64 + n_records * 4 * b.rec_words + stats["distinct"] * 56
     peak, peak_kind = _peaks()
+    alg_bytes = ALG_BYTES_PER_KMER * my_kmers
     achieved = alg_bytes / (hash_ms * 1e-3) / 1e9
-    traffic = None
-    try:
-        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            tr = json.load(f).get(rs.name, {})
-            if ws == 1 and tr.get("kernel_version") == KERNEL_VERSION:
-                traffic = tr.get("dram_bytes_per_launch")
-    except Exception:
-        pass
+    # the r01 byte model (table RMW + records read + vertex records written), kept for comparison
+    detailed = my_kmers * 64 + n_records * 4 * b.rec_words + n_out * 56
+    prof = _profile_facts(rs.name) if ws == 1 else {"stale": True, "source": None}
     cpu = None
     if not args.no_cpu_baseline and ws == 1:
         threads = os.cpu_count() or 1
         rate, sub, dt = _oracle_rate(rs, args.cpu_seconds, threads)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
-               "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s"}
+               "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s",
+               "single_thread_ecoli": _oracle_single_thread_ecoli()}
     scan = 1 if b.np <= 16384 else 3  # scan.cuh: one CTA, or tile sums + tile scan + apply
-    # msp_block_kernel + its scan + scatter_kernel (+ bucket_scatter_kernel when two-level), then
-    # Step 2: the on-chip plan (8 kernels incl. the greedy group packing) + the on-chip kernel
-    # (+ per global-tier batch: its plan scan once, hash_build_list + extract_kernel)
+    # Step 1: msp kernel + its scan + scatter; Step 2: the on-chip plan (8 kernels incl. the greedy
+    # group packing) + the on-chip kernel (+ per global-tier batch: its plan scan once,
+    # hash_build_list + extract_kernel); multi-GPU adds the exchange plan (scan + 1)
     nb = len(b.batches)
-    launches_per_step = 2 + scan + int(b.two_level) + {"fused": scan + 2, "resident": scan + 2 * nb,
-                                                       "smem": 9 + 2 * nb + (scan if nb else 0)}[args.mode]
-    placement = _placement(b) if args.mode == "smem" else None
+    launches_per_step = 2 + scan + 9 + 2 * nb + (scan if nb else 0) + (scan + 1 if ws > 1 else 0)
+    placement = _placement(b)
     # Fig. 6 / Table II analogue (row f1): the paper's partitions (fine pid mod NP) -- skew and the
     # table size lambda/(4 alpha) N^i_kmer x slot bytes of the largest one
     paper_parts = np.bincount(np.arange(b.np) % rs.num_partitions, weights=b.part_kmers,
                               minlength=rs.num_partitions)
     psizes = {"max_over_mean": float(paper_parts.max() / max(paper_parts.mean(), 1e-9)),
               "max_kmers": int(paper_parts.max()), "mean_kmers": float(paper_parts.mean()),
-              "max_table_mb": _lib.dbg_table_capacity(b.prm, int(paper_parts.max())) * b.slot_bytes / 1e6,
+              "max_table_mb": _lib.dbg_table_bytes(b.prm, int(paper_parts.max())) / 1e6,
               "fine_max_over_mean": float(b.part_kmers.max() / max(b.part_kmers.mean(), 1e-9))}
     if rank != 0:
-        dist.barrier()
+        dist.barrier(device_ids=[local])
         dist.destroy_process_group()
         return 0
-    cfg_extra = {"mode": args.mode, "batches": len(b.batches), "group_slots": args.group_slots, "refine": refine,
-                 "fine_partitions": b.np, "smem_split": args.smem_split, "fine_p": fine_p or rs.p,
+    cfg_extra = {"refine": b.refine, "fine_partitions": b.np, "fine_p": b.fine_p or rs.p,
                  "smem_slots": _lib.dbg_smem_table_slots(b.prm), "kmer_placement": placement,
                  "kernel_version": KERNEL_VERSION, "partition_sizes": psizes}
     if ws > 1:
-        cfg_extra.update({"reads_per_rank": rs.n_reads, "kmers_total": total_kmers,
-                          "parallelism": f"reads sharded; fine partitions owned by rank (one all_to_all of "
-                                         f"records over NCCL); {ws} GPUs"})
+        cfg_extra["reads_per_rank"] = rs.n_reads
     if args.min_count > 1:
         cfg_extra["min_count"] = args.min_count
+    onchip = {k: prof.get(k) for k in ("issue_active_pct", "warp_inst_per_kmer", "dram_bytes_per_kmer",
+                                       "l2_hit_pct", "bank_conflict_pct", "source", "kernel_version")}
+    onchip["stale"] = prof.get("stale", True)
     line = {
         "metric": METRIC, "value": total_kmers / (ms * 1e-3), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": _config_json(rs, args, cfg_extra),
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic (seeded genome + reads, DESIGN.md Sec. 4)",
+        "config": _config_json(rs, args, n_reads_total, n_kmers_total, cfg_extra),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic,
-                     "kernel": {"fused": "subgraph_kernel", "resident": "hash_build_kernel",
-                                "smem": "smem_subgraph_kernel"}[args.mode],
-                     "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
-                     "kernel_ms": hash_ms, "kernel_kmers_per_s": my_kmers / (hash_ms * 1e-3),
-                     "rank": 0},
+                     "frac": achieved / peak,
+                     "traffic": None if prof.get("stale", True) else prof.get("dram_bytes_per_launch"),
+                     "kernel": "smem_subgraph_kernel (+ global tier)", "peak_kind": peak_kind,
+                     "model": f"random-access HBM table, {ALG_BYTES_PER_KMER} B per K-mer occurrence "
+                              "(SURVEY.md 8(d)) x this rank's Step-2 K-mers / Step-2 kernel time; the tables "
+                              "are on chip, so measured DRAM traffic is far below the model (onchip)",
+                     "alg_bytes_per_launch": alg_bytes, "kernel_ms": hash_ms,
+                     "kernel_kmers_per_s": my_kmers / (hash_ms * 1e-3),
+                     "detailed_model_frac": detailed / (hash_ms * 1e-3) / 1e9 / peak,
+                     "onchip": onchip, "rank": 0},
         "cpu_baseline": cpu,
         "e2e": {"value": total_kmers / (statistics.median(e2e_ms) * 1e-3), "unit": UNIT,
-                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "ms": statistics.median(e2e_ms),
-                "h2d_ms": statistics.median(h2d_ms), "all_ms": [round(x, 3) for x in e2e_ms],
-                "h2d_overlap": "8 read ranges H2D on a copy stream, MSP per range as it arrives" if ws == 1 else None},
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h_bytes, "ms": statistics.median(e2e_ms),
+                "h2d_ms": statistics.median(h2d_ms), "d2h_ms": statistics.median(d2h_ms),
+                "all_ms": [round(x, 3) for x in e2e_ms],
+                "scope": "H2D of the packed reads + path + D2H of all vertex records to pinned host memory "
+                         "(P:L979-987)" + (", H2D overlapped with MSP in 8 read ranges" if ws == 1 else "")},
         "gpu_launches": args.steps * launches_per_step,
         "clocks": clk.summary(),
         "breakdown_ms": phases,
-        "host_ms": {k: round(statistics.mean(v[-args.steps:]), 3) for k, v in host_ms.items() if v},
         "stats": {"distinct": distinct, "sum_count": sum_count, "sum_edges": sum_edges,
-                  "checksum": stats["checksum"] if ws == 1 else None},
+                  "checksum": checksum},
         "invariants_ok": bool(inv_ok), "gen_s": gen_s,
     }
     print(json.dumps(line), flush=True)
     if dist is not None:
-        dist.barrier()
+        dist.barrier(device_ids=[local])
         dist.destroy_process_group()
     return 0
 
@@ -429,28 +483,24 @@ def run_ours(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", default="ecoli")
+    ap.add_argument("--config", default="chr14")
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--np", type=int, default=None, help="override the number of partitions")
-    ap.add_argument("--p", type=int, default=None, help="override the minimizer length P")
     ap.add_argument("--lam", type=float, default=2.0)
     ap.add_argument("--alpha", type=float, default=0.5)
-    ap.add_argument("--table-budget", type=int, default=None)
-    ap.add_argument("--mode", choices=["smem", "fused", "resident"], default="smem")
     ap.add_argument("--refine", type=int, default=None, help="fine partitions per partition (default: auto)")
-    ap.add_argument("--group-slots", type=int, default=1 << 19)
     ap.add_argument("--fine-p", type=int, default=None,
                     help="minimizer length of the fine partitioning (default: auto; dbg_params.fine_p)")
-    ap.add_argument("--smem-split", type=int, default=0,
-                    help="most CTAs an oversize partition is split over on chip (0: default, 1: none)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--out-frac", type=float, default=0.4, help="output capacity / K-mers")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--min-count", type=int, default=0, help="row f4 low-count filter (0: the full graph)")
     args = ap.parse_args()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return _relaunch_under_torchrun(args.gpus)
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

@@ -36,7 +36,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 10
+#define DBG_ABI_VERSION 11
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -143,6 +143,15 @@ typedef struct {
                                 and pass 2 places record j at d_record_offset[pid] + d_rank[j]
                                 without rank atomics.  Pass 2 may use it only for records staged by
                                 pass 1 of this partition set (NULL e.g. after a record exchange) */
+  /* Multi-GPU emission: with n_peers > 0, pass 2 writes
+     each record of fine partition f into the partition buffer of f's owner GPU o -- the o with
+     d_peer_bounds[o] <= f < d_peer_bounds[o+1] -- at record slot d_record_offset[f] + rank, i.e.
+     straight into peer memory over NVLink (IPC-mapped device pointers).  d_record_offset must
+     then hold dbg_exchange_plan's d_dest_offset; d_records is not written.  Only the one-level
+     scatter supports peers (d_rank and d_scratch must be NULL).  n_peers = 0: local pass 2. */
+  uint32_t* const* d_peer_records; /* [n_peers] device array of the owners' record buffers */
+  const int32_t* d_peer_bounds;    /* [n_peers+1] device array, owner o owns [b[o], b[o+1]) */
+  int32_t n_peers;
 } dbg_partition_set;
 
 /* ---- sizes ------------------------------------------------------------ */
@@ -159,6 +168,10 @@ DBG_API uint32_t dbg_key_bytes(const dbg_params* prm);
 /* Table capacity for a partition with n_kmers K-mers: ceil(lambda/(4 alpha) * n_kmers)
  * (Sec. IV-A), at least 1 when n_kmers > 0 (Property 1 sizing). */
 DBG_API uint64_t dbg_table_capacity(const dbg_params* prm, uint64_t n_kmers);
+/* Bytes of the global (resident) hash table of such a partition: dbg_table_capacity slots of
+ * dbg_slot_bytes each (the d_table block dbg_hash_build takes for it; Table II, P:L1005-1013,
+ * prints the paper's analogue at 32 B per entry).  0 for invalid params. */
+DBG_API uint64_t dbg_table_bytes(const dbg_params* prm, uint64_t n_kmers);
 /* uint64 words of the packed 2-bit stream for n_bases bases, including one pad word. */
 DBG_API uint64_t dbg_packed_words(uint64_t n_bases);
 
@@ -202,6 +215,27 @@ DBG_API dbg_status dbg_msp_partition_range(const dbg_params* prm, const uint64_t
                                    const uint64_t* d_offsets, uint64_t n_reads,
                                    const dbg_partition_set* part, int32_t pid_lo, int32_t pid_hi,
                                    int append, cudaStream_t stream);
+
+/* ---- e: multi-GPU exchange plan (Sec. III-A) -----
+ * world ranks split the reads by range; rank r's pass 1 gives its records per fine partition,
+ * and d_counts[world * NP] holds every rank's d_n_records (gathered: rank q's row is
+ * d_counts[q*NP .. q*NP+NP)).  Fine partition f is owned by the rank o with
+ * d_bounds[o] <= f < d_bounds[o+1] (d_bounds: world+1 int32, device).  In the owner's buffer the
+ * records are in partition order, and inside a partition in source-rank order.  Writes:
+ *   d_dest_offset[NP]          where THIS rank's records of f start in owner(f)'s buffer (records;
+ *                              pass 2 with peers uses it as d_record_offset);
+ *   d_owned_n_records[NP]      sum over ranks of d_counts for the partitions this rank owns, 0
+ *                              for the others;
+ *   d_owned_n_kmers[NP]        d_kmers_sum (the K-mers per partition summed over ranks) for the
+ *                              owned partitions, 0 for the others (may alias d_kmers_sum);
+ *   d_owned_record_offset[NP+1] exclusive prefix sum of d_owned_n_records: the partition set of
+ *                              this rank's Step 2 (its last entry = records this rank receives).
+ * d_prefix: NP+1 uint64 and d_scratch: NP uint64 of caller memory (no alias with the outputs). */
+DBG_API dbg_status dbg_exchange_plan(const dbg_params* prm, const uint64_t* d_counts, const uint64_t* d_kmers_sum,
+                                     int32_t world, int32_t rank, const int32_t* d_bounds,
+                                     uint64_t* d_dest_offset, uint64_t* d_owned_n_records,
+                                     uint64_t* d_owned_n_kmers, uint64_t* d_owned_record_offset,
+                                     uint64_t* d_prefix, uint64_t* d_scratch, cudaStream_t stream);
 
 /* ---- a5: sizing (Property 1; Sec. IV-A) ----------------------
  * d_table_offset[NP+1] = exclusive prefix sum of dbg_table_capacity(N^i_kmer)

@@ -37,7 +37,8 @@ class dbg_partition_set(ctypes.Structure):
                 ("d_record_offset", ctypes.c_void_p), ("d_fill", ctypes.c_void_p),
                 ("d_staged", ctypes.c_void_p), ("d_staging", ctypes.c_void_p),
                 ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p),
-                ("d_scratch", ctypes.c_void_p), ("d_rank", ctypes.c_void_p)]
+                ("d_scratch", ctypes.c_void_p), ("d_rank", ctypes.c_void_p),
+                ("d_peer_records", ctypes.c_void_p), ("d_peer_bounds", ctypes.c_void_p), ("n_peers", ctypes.c_int32)]
 
 
 # dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
@@ -64,6 +65,8 @@ SIGNATURES = {
     "dbg_slot_bytes": (ctypes.c_uint32, [_PRM]),
     "dbg_key_bytes": (ctypes.c_uint32, [_PRM]),
     "dbg_table_capacity": (_U64, [_PRM, _U64]),
+    "dbg_table_bytes": (_U64, [_PRM, _U64]),
+    "dbg_exchange_plan": (ctypes.c_int, [_PRM, _P, _P, _I32, _I32, _P, _P, _P, _P, _P, _P, _P, _P]),
     "dbg_packed_words": (_U64, [_U64]),
     "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
@@ -90,7 +93,7 @@ SIGNATURES = {
 }
 
 _lib = None
-ABI_VERSION = 10
+ABI_VERSION = 11
 
 
 def load():
@@ -146,9 +149,11 @@ def fine_partitions(prm: dbg_params) -> int:
 
 
 def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
-                  records=None, scratch=None, rank=None) -> dbg_partition_set:
+                  records=None, scratch=None, rank=None, peer_records=None, peer_bounds=None,
+                  n_peers: int = 0) -> dbg_partition_set:
     return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(staged),
-                             _ptr(staging), staging_cap, _ptr(records), _ptr(scratch), _ptr(rank))
+                             _ptr(staging), staging_cap, _ptr(records), _ptr(scratch), _ptr(rank),
+                             _ptr(peer_records), _ptr(peer_bounds), n_peers)
 
 
 # --------------------------------------------------------------------------- entry points
@@ -176,6 +181,18 @@ def dbg_key_bytes(prm: dbg_params) -> int:
 
 def dbg_table_capacity(prm: dbg_params, n_kmers: int) -> int:
     return load().dbg_table_capacity(ctypes.byref(prm), n_kmers)
+
+
+def dbg_table_bytes(prm: dbg_params, n_kmers: int) -> int:
+    return load().dbg_table_bytes(ctypes.byref(prm), n_kmers)
+
+
+def dbg_exchange_plan(prm, d_counts, d_kmers_sum, world: int, rank: int, d_bounds, d_dest_offset, d_owned_n_records,
+                      d_owned_n_kmers, d_owned_record_offset, d_prefix, d_scratch, stream=None) -> None:
+    _check("dbg_exchange_plan", load().dbg_exchange_plan(
+        ctypes.byref(prm), _ptr(d_counts), _ptr(d_kmers_sum), world, rank, _ptr(d_bounds), _ptr(d_dest_offset),
+        _ptr(d_owned_n_records), _ptr(d_owned_n_kmers), _ptr(d_owned_record_offset), _ptr(d_prefix),
+        _ptr(d_scratch), _stream(stream)))
 
 
 def dbg_packed_words(n_bases: int) -> int:

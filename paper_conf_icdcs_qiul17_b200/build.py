@@ -28,7 +28,8 @@ def _stale() -> bool:
     if not os.path.exists(LIB):
         return True
     t = os.path.getmtime(LIB)
-    deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS] + [__file__]
+    cuh = [f for f in os.listdir(CSRC) if f.endswith(".cuh")]   # every device header (scan.cuh, ...)
+    deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS + cuh] + [__file__]
     return any(os.path.getmtime(d) > t for d in deps)
 
 

@@ -32,6 +32,13 @@ extern "C" uint64_t dbg_table_capacity(const dbg_params* prm, uint64_t n_kmers) 
   return c < 1.0 ? 1ull : (uint64_t)c;
 }
 
+extern "C" uint32_t dbg_slot_bytes(const dbg_params* prm);
+
+extern "C" uint64_t dbg_table_bytes(const dbg_params* prm, uint64_t n_kmers) {
+  if (!prm || prm->k < 1 || prm->k > 127) return 0;
+  return dbg_table_capacity(prm, n_kmers) * (uint64_t)dbg_slot_bytes(prm);
+}
+
 extern "C" uint64_t dbg_packed_words(uint64_t n_bases) { return (n_bases + 31) / 32 + 1; }
 
 // Sec. II-A: characters are transformed into {A,C,G,T}, unknown

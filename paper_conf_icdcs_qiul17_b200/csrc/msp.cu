@@ -405,7 +405,8 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
                                                                   const uint64_t* __restrict__ rec_off,
                                                                   unsigned long long* fill,
                                                                   uint32_t* __restrict__ records, int nb, int shift,
-                                                                  bool abs_pos) {
+                                                                  bool abs_pos, uint32_t* const* peer_records,
+                                                                  const int32_t* peer_bounds, int n_peers) {
   // abs_pos (global path, shift 0): the cursors start at the partitions' record offsets, so the
   // rank atomic returns the record's final position (no offset load)
   extern __shared__ unsigned long long sh_base[];  // [nb] global bases (per tile), then [nb] counts
@@ -467,7 +468,14 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
       if (idx < n) {
         const uint32_t bin = (rec[v][0].x >> 10) >> shift;
         const uint64_t pos = abs_pos ? apos[v] : base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
-        uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
+        uint32_t* out = records;
+        if (n_peers) {  // multi-GPU emission: the owner's buffer, through its IPC-mapped pointer
+          const int32_t pid = (int32_t)(rec[v][0].x >> 10);
+          int o = 0;
+          while (o + 1 < n_peers && pid >= __ldg(peer_bounds + o + 1)) ++o;
+          out = peer_records[o];
+        }
+        uint4* dst = reinterpret_cast<uint4*>(out + pos * R);
 #pragma unroll
         for (int c = 0; c < R / 4; ++c) {
           if (DBG_SCATTER_STCS) __stcs(dst + c, rec[v][c]);
@@ -899,6 +907,9 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     if (!part->d_fill || !part->d_staging) return DBG_EINVAL;
     if (part->d_scratch && (part->d_scratch == part->d_staging || part->d_scratch == part->d_records))
       return DBG_EINVAL;
+    if (part->n_peers < 0 ||
+        (part->n_peers > 0 && (!part->d_peer_records || !part->d_peer_bounds || part->d_rank || part->d_scratch)))
+      return DBG_EINVAL;
     if (part->d_rank) {  // ranks from pass 1: one pass, no atomics
       const unsigned long long* stg = reinterpret_cast<const unsigned long long*>(part->d_staged);
       const int grid = dbg_sm_count() * 8;
@@ -948,7 +959,8 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
   cudaFuncSetAttribute(scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
   scatter_kernel<RW><<<scatter_grid((const void*)scatter_kernel<RW>), kScatterThreads, smem, stream>>>(part->d_staging, staged, part->staging_cap,       \
                                                               part->d_record_offset, fill, lvl1, nb, shift,     \
-                                                              abs_pos);                                          \
+                                                              abs_pos, part->d_peer_records,                    \
+                                                              part->d_peer_bounds, part->n_peers);              \
   if (two) {                                                                                                    \
     cudaFuncSetAttribute(bucket_scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);   \
     bucket_scatter_kernel<RW><<<grid2, kBucketThreads, smem2, stream>>>(part->d_scratch, staged,               \
@@ -988,4 +1000,63 @@ extern "C" dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t
                                            uint64_t* d_scratch, cudaStream_t stream) {
   if (!prm || prm->k > 63) return DBG_EINVAL;
   return table_plan(prm, d_n_kmers, dbg_smem_table_slots(prm), d_table_offset, d_scratch, stream);
+}
+
+// ---- multi-GPU exchange plan (dbg.h dbg_exchange_plan) ----------------
+// Entry i: records of fine partition i summed over the world ranks' rows of the gathered counts.
+struct GatheredSumOp {
+  const uint64_t* counts;
+  int np, world;
+  __device__ __forceinline__ unsigned long long operator()(int i) const {
+    unsigned long long s = 0;
+    for (int r = 0; r < world; ++r) s += counts[(size_t)r * np + i];
+    return s;
+  }
+};
+
+// prefix = exclusive scan of the summed counts over ALL partitions; partition f of owner o
+// starts at prefix[f] - prefix[bounds[o]] in o's buffer, and this rank's share of it after the
+// records of the lower ranks.
+__global__ void exchange_plan_kernel(const uint64_t* __restrict__ counts, const uint64_t* kmers_sum, int np,
+                                     int world, int rank, const int32_t* __restrict__ bounds,
+                                     const uint64_t* __restrict__ prefix, uint64_t* __restrict__ dest,
+                                     uint64_t* __restrict__ own_n, uint64_t* own_k, uint64_t* __restrict__ own_off) {
+  const int lo = bounds[rank], hi = bounds[rank + 1];
+  for (int f = blockIdx.x * blockDim.x + threadIdx.x; f <= np; f += gridDim.x * blockDim.x) {
+    if (f < np) {
+      int o = 0;
+      while (o + 1 < world && f >= bounds[o + 1]) ++o;
+      uint64_t d = prefix[f] - prefix[bounds[o]];
+      for (int r = 0; r < rank; ++r) d += counts[(size_t)r * np + f];
+      dest[f] = d;
+      const bool mine = f >= lo && f < hi;
+      own_n[f] = mine ? prefix[f + 1] - prefix[f] : 0;
+      const uint64_t k = kmers_sum[f];
+      own_k[f] = mine ? k : 0;
+    }
+    const int c = f < lo ? lo : (f > hi ? hi : f);
+    own_off[f] = prefix[c] - prefix[lo];
+  }
+}
+
+extern "C" dbg_status dbg_exchange_plan(const dbg_params* prm, const uint64_t* d_counts, const uint64_t* d_kmers_sum,
+                                        int32_t world, int32_t rank, const int32_t* d_bounds,
+                                        uint64_t* d_dest_offset, uint64_t* d_owned_n_records,
+                                        uint64_t* d_owned_n_kmers, uint64_t* d_owned_record_offset,
+                                        uint64_t* d_prefix, uint64_t* d_scratch, cudaStream_t stream) {
+  if (!dbg_params_ok(prm) || !d_counts || !d_kmers_sum || !d_bounds || !d_dest_offset || !d_owned_n_records ||
+      !d_owned_n_kmers || !d_owned_record_offset || !d_prefix || world < 1 || rank < 0 || rank >= world)
+    return DBG_EINVAL;
+  if (d_prefix == d_owned_record_offset || d_prefix == d_dest_offset || d_prefix == d_owned_n_records ||
+      (d_scratch && (d_scratch == d_prefix || d_scratch == d_owned_record_offset)))
+    return DBG_EINVAL;
+  const int np = fine_partitions(prm);
+  if (exclusive_scan(GatheredSumOp{d_counts, np, world}, np, d_prefix,
+                     reinterpret_cast<unsigned long long*>(d_scratch), stream) != cudaSuccess)
+    return DBG_ECUDA;
+  const int grid = (int)std::min<int64_t>(((int64_t)np + 256) / 256, (int64_t)dbg_sm_count() * 8);
+  exchange_plan_kernel<<<grid, 256, 0, stream>>>(d_counts, d_kmers_sum, np, world, rank, d_bounds, d_prefix,
+                                                 d_dest_offset, d_owned_n_records, d_owned_n_kmers,
+                                                 d_owned_record_offset);
+  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }

@@ -81,8 +81,9 @@ class StreamingBuilder:
         self.resident = resident
         dev = builder.device
         self.compute = torch.cuda.current_stream(dev)
-        self.copy = torch.cuda.Stream(dev)
-        self.h2d_bytes = 0
+        self.copy = torch.cuda.Stream(dev)   # H2D of the read batches
+        self.d2h = torch.cuda.Stream(dev)    # D2H of the ranges' vertices (its own stream, so the next
+        self.h2d_bytes = 0                   # range's H2D does not queue behind it)
 
     # -- input stage: batch i into device slot i % 2 (or its resident copy)
     def _inputs(self, batches):
@@ -192,10 +193,10 @@ class StreamingBuilder:
             # range's Step 1
             host = torch.empty(n_out * VERTEX_DTYPE.itemsize, dtype=torch.uint8, pin_memory=True)
             done = torch.cuda.Event()
-            self.copy.wait_stream(self.compute)
-            with torch.cuda.stream(self.copy):
+            self.d2h.wait_stream(self.compute)
+            with torch.cuda.stream(self.d2h):
                 host.copy_(b.out[:n_out * VERTEX_DTYPE.itemsize], non_blocking=True)
-            done.record(self.copy)
+            done.record(self.d2h)
             pending = (host.numpy().view(VERTEX_DTYPE), done, n_out)
         if pending is not None:
             pending[1].synchronize()

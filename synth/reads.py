@@ -81,12 +81,18 @@ def genome(length: int, seed: int, repeat_families: int = 0, repeat_len: int = 3
 
 
 def make_reads(g: np.ndarray, n_reads: int, read_len: int, error_rate: float, seed: int,
-               both_strands: bool = True, n_rate: float = 0.0) -> tuple[np.ndarray, np.ndarray]:
+               both_strands: bool = True, n_rate: float = 0.0,
+               read_range: tuple[int, int] | None = None) -> tuple[np.ndarray, np.ndarray]:
+    """Reads [r0, r1) of the n_reads-read set (default: all of them).  Chunks are seeded by their
+    index, so a read range is the same reads whether it is drawn alone or as part of the set
+    (multi-GPU strong scaling: each rank draws only its own range)."""
     G = len(g)
     assert G >= read_len
-    seq = np.empty(n_reads * read_len, dtype=np.uint8)
+    r0, r1 = read_range if read_range is not None else (0, n_reads)
+    assert 0 <= r0 <= r1 <= n_reads
+    seq = np.empty((r1 - r0) * read_len, dtype=np.uint8)
     cols = np.arange(read_len, dtype=np.int64)
-    for c0 in range(0, n_reads, CHUNK):
+    for c0 in range((r0 // CHUNK) * CHUNK, r1, CHUNK):
         c1 = min(n_reads, c0 + CHUNK)
         n = c1 - c0
         rng = np.random.Generator(np.random.PCG64(np.random.SeedSequence([seed, c0 // CHUNK])))
@@ -107,8 +113,9 @@ def make_reads(g: np.ndarray, n_reads: int, read_len: int, error_rate: float, se
         if n_rate > 0:
             nm = rng.random((n, read_len)) < n_rate
             r[nm] = ord("N")
-        seq[c0 * read_len:c1 * read_len] = r.reshape(-1)
-    offsets = np.arange(n_reads + 1, dtype=np.uint64) * np.uint64(read_len)
+        a, z = max(c0, r0), min(c1, r1)
+        seq[(a - r0) * read_len:(z - r0) * read_len] = r[a - c0:z - c0].reshape(-1)
+    offsets = np.arange(r1 - r0 + 1, dtype=np.uint64) * np.uint64(read_len)
     return seq, offsets
 
 
@@ -155,16 +162,22 @@ CONFIGS = {
 
 
 def make_config(name: str, scale: float = 1.0, num_partitions: int | None = None,
-                read_seed_offset: int = 0) -> ReadSet:
+                read_seed_offset: int = 0, shard: tuple[int, int] | None = None) -> ReadSet:
     """The named configuration; ``scale`` < 1 shrinks genome and read count together
     (same coverage, error rate and read length) for quick runs; ``read_seed_offset`` draws a
-    different read set from the same genome (multi-GPU weak scaling)."""
+    different read set from the same genome; ``shard`` = (rank, world) draws only the contiguous
+    read range [rank N / world, (rank+1) N / world) of the configuration (multi-GPU strong
+    scaling: the ranks' ranges together are exactly the configuration's reads)."""
     c = CONFIGS[name]
     G = max(int(c["genome"] * scale), c["read_len"] * 4)
     n = max(int(c["reads"] * scale), 1)
+    rng_ = None
+    if shard is not None:
+        r, w = shard
+        rng_ = (n * r // w, n * (r + 1) // w)
     g = genome(G, c["gseed"])
-    seq, offsets = make_reads(g, n, c["read_len"], c["error"], c["rseed"] + read_seed_offset)
+    seq, offsets = make_reads(g, n, c["read_len"], c["error"], c["rseed"] + read_seed_offset, read_range=rng_)
     return ReadSet(seq, offsets, name=name, k=c["k"], p=c["p"],
                    num_partitions=num_partitions or c["np"],
                    meta=dict(genome=G, reads=n, read_len=c["read_len"], error=c["error"],
-                             scale=scale, desc=c["desc"]))
+                             scale=scale, desc=c["desc"], read_range=rng_ or (0, n)))

@@ -28,7 +28,7 @@ def _declared():
 
 def test_exports_every_declared_symbol(lib):
     names = _declared()
-    assert len(names) == 28
+    assert sorted(names) == sorted(lib.SIGNATURES)   # the binding mirrors the header exactly
     raw = lib.load()
     for n in names:
         assert hasattr(raw, n), n
@@ -36,7 +36,7 @@ def test_exports_every_declared_symbol(lib):
 
 
 def test_abi_and_sizes(lib):
-    assert lib.dbg_abi_version() == 10
+    assert lib.dbg_abi_version() == 11
     p31 = lib.params(31, 11, 16)
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
@@ -65,6 +65,11 @@ def test_table2_sizing_pin(lib):
     assert lib.dbg_table_capacity(lib.params(31, 11, 16, 1.0, 0.5), 1001) == 501
     assert lib.dbg_table_capacity(prm, 0) == 0
     assert lib.dbg_table_capacity(lib.params(31, 11, 16, 0.001, 0.5), 10) == 1
+    # dbg_table_bytes = capacity x slot bytes (the d_table block dbg_hash_build takes)
+    for k, n in ((31, 1000), (63, 12345), (27, 2725 * 10 ** 6 // 512)):
+        q = lib.params(k, 11, 16, 2.0, 0.8)
+        assert lib.dbg_table_bytes(q, n) == lib.dbg_table_capacity(q, n) * lib.dbg_slot_bytes(q)
+    assert lib.dbg_table_bytes(prm, 0) == 0
 
 
 def test_onchip_placement_rule(lib):

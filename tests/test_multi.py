@@ -1,8 +1,8 @@
-"""Multi-GPU host logic on CPU: owner bounds, split sizes and the record exchange with gloo, world size 2.
+"""Multi-GPU host logic on CPU (gloo, world size 2): owner bounds, the histogram collectives, the
+peer-buffer handle protocol, and the read shards of strong scaling.
 
-The exchange is the one data-path collective of the sharded path; here each rank
-owns synthetic partition-ordered "records" whose words encode (source rank, partition, index), and
-the test checks every rank receives exactly the records of the partitions it owns, from every rank.
+The data path itself (emission into peer buffers through IPC pointers) needs a GPU: it is covered
+by tests/test_gpu_multi.py (two processes on one GPU).
 """
 import os
 import socket
@@ -25,58 +25,77 @@ def _free_port():
     return p
 
 
-def test_owner_bounds_and_send_counts():
+def test_owner_bounds():
     sys.path.insert(0, ROOT)
-    from paper_conf_icdcs_qiul17_b200.multi import owner_bounds, send_counts
+    from paper_conf_icdcs_qiul17_b200.multi import owner_bounds
 
     b = owner_bounds(10, 3)
     assert b.tolist() == [0, 3, 6, 10]
-    pr = np.array([1, 0, 2, 5, 0, 0, 1, 1, 1, 4])
-    assert send_counts(pr, b).tolist() == [3, 5, 7]
     assert owner_bounds(5, 8)[-1] == 5 and np.all(np.diff(owner_bounds(5, 8)) >= 0)
+    for n, w in ((1_579_008, 8), (7, 2), (1, 1)):
+        b = owner_bounds(n, w)
+        assert b[0] == 0 and b[-1] == n and np.all(np.diff(b) >= 0) and np.diff(b).max() - np.diff(b).min() <= 1
 
 
-def _worker(rank, world, port, n_fine, R, q):
+def _worker(rank, world, port, q):
     sys.path.insert(0, ROOT)
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    from paper_conf_icdcs_qiul17_b200.multi import exchange_records, owner_bounds
+    from paper_conf_icdcs_qiul17_b200.multi import PeerBuffers, all_reduce_sum, gather_rows
 
-    rng = np.random.default_rng(100 + rank)
-    part_records = rng.integers(0, 4, size=n_fine)
-    rows = []
-    for p in range(n_fine):
-        for i in range(part_records[p]):
-            rows.append([rank, p, i] + [7] * (R - 3))
-    recs = torch.tensor(np.array(rows, dtype=np.int32).reshape(-1)) if rows else torch.zeros(0, dtype=torch.int32)
-    bounds = owner_bounds(n_fine, world)
-    out, n, per_src = exchange_records(recs, part_records, bounds, R)
-    got = out[: n * R].view(n, R).numpy()
-    # expected: records of owned partitions from every source, in source order, partition order within
-    lo, hi = bounds[rank], bounds[rank + 1]
-    exp = []
-    for src in range(world):
-        pr = np.random.default_rng(100 + src).integers(0, 4, size=n_fine)
-        for p in range(lo, hi):
-            for i in range(pr[p]):
-                exp.append([src, p, i] + [7] * (R - 3))
-    q.put((rank, got.tolist() == exp, int(n), per_src.tolist()))
+    res = {}
+    t = torch.arange(5, dtype=torch.int64) + 10 * rank
+    res["gather"] = gather_rows(t).tolist()
+    u = torch.full((3,), rank + 1, dtype=torch.int64)
+    res["sum"] = all_reduce_sum(u).tolist()
+    # handle protocol with fake IPC: a handle names (rank, generation); opening one "maps" it
+    opened = []
+    pb = PeerBuffers(export=lambda x: ("h", rank, x.numel()),
+                     open_=lambda h, n: (None, 1000 * h[1] + h[2]) if not opened.append(h) else None)
+    bufs = [torch.zeros(4, dtype=torch.int32), None, torch.zeros(9, dtype=torch.int32)]
+    bufs[1] = bufs[0]
+    trace = []
+    for step in range(3):
+        # rank 1 reallocates its buffer at step 2 only; rank 0 never does
+        b = bufs[step] if rank == 1 else bufs[0]
+        ptrs = pb.update(b)
+        trace.append((ptrs[1 - rank], len(opened)))
+    res["trace"] = trace
+    q.put((rank, res))
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("n_fine,R", [(37, 4), (5, 8)])
-def test_exchange_records_gloo_world2(n_fine, R):
+def test_collectives_and_peer_handle_protocol_gloo_world2():
     world = 2
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, n_fine, R, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
-    res = [q.get(timeout=120) for _ in range(world)]
+    res = dict(q.get(timeout=120) for _ in range(world))
     for p in procs:
         p.join(timeout=60)
-    assert all(ok for _, ok, _, _ in res), res
+    for r in range(world):
+        assert res[r]["gather"] == [0, 1, 2, 3, 4, 10, 11, 12, 13, 14]
+        assert res[r]["sum"] == [3, 3, 3]
+    # rank 0 sees rank 1's buffer: opened at step 0 (4 words), unchanged at step 1 (no reopen),
+    # reopened at step 2 (9 words)
+    assert res[0]["trace"] == [(1004, 1), (1004, 1), (1009, 2)]
+    # rank 1 opens rank 0's buffer once
+    assert [n for _, n in res[1]["trace"]] == [1, 1, 1] and res[1]["trace"][0][0] == 4
+
+
+def test_read_shards_concatenate_to_the_configuration():
+    """Strong scaling: the ranks' read ranges are exactly the configuration's reads."""
+    sys.path.insert(0, ROOT)
+    from synth import make_config
+
+    full = make_config("ecoli", scale=0.6)     # 1.66 M reads: two generator chunks
+    for w in (2, 3):
+        parts = [make_config("ecoli", scale=0.6, shard=(r, w)) for r in range(w)]
+        assert sum(p.n_reads for p in parts) == full.n_reads
+        assert np.array_equal(np.concatenate([p.seq for p in parts]), full.seq)
 
 
 def test_stream_plan_ranges():
