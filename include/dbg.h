@@ -136,13 +136,9 @@ typedef struct {
   uint32_t* d_records;       /* d_record_offset[NP] records in partition order; NULL => pass 1 */
   uint32_t* d_scratch;       /* optional, staging_cap records (not aliasing d_staging or d_records):
                                 with more than 8192 fine partitions pass 2 then scatters in two
-                                levels -- into buckets of 2^s consecutive partitions (d_scratch),
-                                then within each bucket (d_records); NULL: one level */
-  uint32_t* d_rank;          /* optional, staging_cap entries: pass 1 writes each staged record's
-                                rank inside its partition (from the per-partition record counter),
-                                and pass 2 places record j at d_record_offset[pid] + d_rank[j]
-                                without rank atomics.  Pass 2 may use it only for records staged by
-                                pass 1 of this partition set (NULL e.g. after a record exchange) */
+                                levels -- into buckets of 8 consecutive partitions (d_scratch),
+                                then within each bucket (d_records) -- which avoids a DRAM
+                                read-modify-write per 16-byte record; NULL: one level */
   /* Multi-GPU emission: with n_peers > 0, pass 2 writes
      each record of fine partition f into the partition buffer of f's owner GPU o -- the o with
      d_peer_bounds[o] <= f < d_peer_bounds[o+1] -- at record slot d_record_offset[f] + rank, i.e.

@@ -37,7 +37,7 @@ class dbg_partition_set(ctypes.Structure):
                 ("d_record_offset", ctypes.c_void_p), ("d_fill", ctypes.c_void_p),
                 ("d_staged", ctypes.c_void_p), ("d_staging", ctypes.c_void_p),
                 ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p),
-                ("d_scratch", ctypes.c_void_p), ("d_rank", ctypes.c_void_p),
+                ("d_scratch", ctypes.c_void_p),
                 ("d_peer_records", ctypes.c_void_p), ("d_peer_bounds", ctypes.c_void_p), ("n_peers", ctypes.c_int32)]
 
 
@@ -149,10 +149,10 @@ def fine_partitions(prm: dbg_params) -> int:
 
 
 def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
-                  records=None, scratch=None, rank=None, peer_records=None, peer_bounds=None,
+                  records=None, scratch=None, peer_records=None, peer_bounds=None,
                   n_peers: int = 0) -> dbg_partition_set:
     return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(staged),
-                             _ptr(staging), staging_cap, _ptr(records), _ptr(scratch), _ptr(rank),
+                             _ptr(staging), staging_cap, _ptr(records), _ptr(scratch),
                              _ptr(peer_records), _ptr(peer_bounds), n_peers)
 
 

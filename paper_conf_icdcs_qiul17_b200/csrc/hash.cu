@@ -48,51 +48,6 @@
 #include "scan.cuh"
 
 // Kernel variants (A/B builds: tools/build_variants.py); the defaults are the measured winners.
-#ifndef DBG_WORDSEL
-#define DBG_WORDSEL 1
-#endif
-#ifndef DBG_PROBE_PRED
-#define DBG_PROBE_PRED 1
-#endif
-#ifndef DBG_BUCKET2
-#define DBG_BUCKET2 0
-#endif
-#ifndef DBG_KW2_LOAD
-#define DBG_KW2_LOAD 0  // two-word keys: load, CAS only on an empty-looking entry
-#endif
-#ifndef DBG_XSCAN
-#define DBG_XSCAN 1  // extraction scan: sign bit of the key's high word, shared addresses hoisted
-#endif
-#ifndef DBG_XEMIT
-#define DBG_XEMIT 0  // extraction emission with explicit shared addresses
-#endif
-#ifndef DBG_KCONST
-#define DBG_KCONST 1  // on-chip kernel specialised for K = 31 / 63 (default: -1.2 % E. coli, -1.8 % K = 63)
-#endif
-#ifndef DBG_SADDR
-#define DBG_SADDR 0  // explicit 32-bit shared addresses in the window loop
-#endif
-#ifndef DBG_VSTORE
-#define DBG_VSTORE 1  // 16-byte vertex stores
-#endif
-#ifndef DBG_SLOT26
-#define DBG_SLOT26 1  // implies no fine-pid field (DBG_SLOT28)
-#endif
-#ifndef DBG_SLOT28
-#define DBG_SLOT28 1
-#endif
-#if DBG_SLOT26 && !DBG_SLOT28
-#error DBG_SLOT26 needs DBG_SLOT28
-#endif
-#if DBG_SLOT26 && DBG_BITMAP
-#error DBG_SLOT26 excludes DBG_BITMAP
-#endif
-#ifndef DBG_RB4
-#define DBG_RB4 1024  // records of 4 words per on-chip batch (T >= 512)
-#endif
-#ifndef DBG_BITMAP
-#define DBG_BITMAP 0
-#endif
 
 int dbg_sm_count();
 bool dbg_params_ok(const dbg_params* prm);
@@ -423,6 +378,24 @@ __device__ __forceinline__ uint32_t kmer_partition(uint64_t hi, uint64_t lo, con
     m = oa.p <= 16 ? kmer_minimizer128<uint32_t>(code, oa.k, oa.p) : kmer_minimizer128<uint64_t>(code, oa.k, oa.p);
   }
   return fast_mod(oa.np_mod, fmix64(m));
+}
+
+// kmer_partition with compile-time K <= 31 and P <= 16 (the chr14 launch: K = 31, P = 11 under a
+// longer device minimizer): the K - P + 1 canonical P-mers of the K-mer as 32-bit values taken
+// with constant funnel shifts, min-reduced three at a time -- the same minimizer as
+// kmer_minimizer64 (the vertex's P-minimizer, reading V) at about half the instructions.
+template <int KC, int PC>
+__device__ __forceinline__ uint32_t kmer_partition_c(uint64_t lo, const OutArgs& oa) {
+  static_assert(KC <= 31 && PC >= 1 && PC <= 16, "one-word K-mer, 32-bit P-mer");
+  const uint64_t rc = revcomp64(lo, KC);
+  constexpr uint32_t mask = (uint32_t)((2ull << (2 * PC - 1)) - 1);
+  uint32_t m = ~0u;
+#pragma unroll
+  for (int q = 0; q <= KC - PC; ++q) {
+    const uint32_t f = (uint32_t)(lo >> (2 * (KC - PC - q))) & mask, r = (uint32_t)(rc >> (2 * q)) & mask;
+    m = min(m, min(f, r));
+  }
+  return fast_mod(oa.np_mod, fmix64((uint64_t)m));
 }
 
 struct XShared {
@@ -833,10 +806,10 @@ constexpr uint64_t kSmemMaxSlots = 65535;
 template <int KW>
 struct SmemSlot {
   static constexpr uint32_t kKeyBytes = KW == 1 ? 8 : 16;
-  static constexpr uint32_t kFieldWords = DBG_SLOT28 ? 5 : 6;  // (DBG_SLOT28: no fine-pid field)
-  // DBG_SLOT26: the nine 16-bit fields packed at 18 bytes per slot (field f of slot s is
-  // half 9s + f of the field array)
-  static constexpr uint32_t kBytes = kKeyBytes + (DBG_SLOT26 ? 18 : 4 * kFieldWords);
+  static constexpr uint32_t kFieldWords = 5;
+  // the nine 16-bit fields packed at 18 bytes per slot (field f of slot s is half 9s + f of
+  // the field array); the fine partition of a slot is found from the plan at extraction
+  static constexpr uint32_t kBytes = kKeyBytes + 18;
 };
 
 // Decoded work item (32 B): records [r0, r0 + nrec) of partitions [first, last);
@@ -855,7 +828,7 @@ constexpr int kGroupParts = 256;  // partitions per group at most (plan rule)
 // Records per batch: 1024 four-word or 512 eight-word records (16 KB) from 512
 // threads up; fewer for smaller CTAs.
 template <int R, int T>
-__host__ __device__ constexpr int smem_rec_batch() { return (T >= 512 ? DBG_RB4 : 2 * T) * 4 / R; }
+__host__ __device__ constexpr int smem_rec_batch() { return (T >= 512 ? 1024 : 2 * T) * 4 / R; }
 
 template <int R, int T>
 struct SmemStage {
@@ -989,7 +962,7 @@ __device__ __forceinline__ OnChip on_chip(const SmemArgs& a, uint64_t nk) {
   OnChip o;
   o.cap = table_capacity(a.ratio, nk);
   const uint32_t t = onchip_tables(nk, o.cap, a.slots, a.max_split);
-  o.gc = t == 1 ? (DBG_BUCKET2 ? (o.cap + 1) & ~1ull : o.cap) : 0;  // (DBG_BUCKET2: even, 16-B aligned pairs)
+  o.gc = t == 1 ? o.cap : 0;
   o.ns = t >= 2 ? t : 0;
   return o;
 }
@@ -1260,10 +1233,10 @@ __device__ __forceinline__ void store_vertex16(dbg_vertex* dst, const dbg_vertex
 
 // A group of consecutive fine partitions shares one CTA table: each partition
 // p owns slots [P[p] - P[first], P[p+1] - P[first]).
-template <typename Code, int R, int kSmemThreads, int kMinCtas, int KC = 0>
+template <typename Code, int R, int kSmemThreads, int kMinCtas, int KC = 0, int PC = 0>
 __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(SmemArgs a, OutArgs oa) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  constexpr uint32_t KB = SmemSlot<KW>::kKeyBytes, FW = SmemSlot<KW>::kFieldWords;
+  constexpr uint32_t KB = SmemSlot<KW>::kKeyBytes;
   constexpr int RB = SmemStage<R, kSmemThreads>::RB;
   constexpr int kRPT = RB >= kSmemThreads ? RB / kSmemThreads : 1;  // records per thread per batch
   typedef cub::BlockScan<uint32_t, kSmemThreads> Scan;
@@ -1271,17 +1244,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
   SmemStage<R, kSmemThreads>& st = *reinterpret_cast<SmemStage<R, kSmemThreads>*>(smem);
   char* keys = reinterpret_cast<char*>(smem + smem_fixed_bytes<R, kSmemThreads>());
   uint32_t* fld = reinterpret_cast<uint32_t*>(keys + a.slots * KB);
-  // occupancy bitmap of the table (bit s = slot s holds a vertex): extraction reads one word
-  // per 32 slots instead of 32 keys
-  uint32_t* occ = fld + a.slots * FW;
-  const uint32_t keys_s = smem_addr(keys), fld_s = smem_addr(fld), occ_s = smem_addr(occ);
+  const uint32_t keys_s = smem_addr(keys), fld_s = smem_addr(fld);
   const int K = KC ? KC : a.k;  // KC: compile-time K (shifts by constants)
   {  // the table starts clean; extraction keeps it clean (slots is a multiple of 64)
     uint4* z = reinterpret_cast<uint4*>(keys);
     for (uint64_t q = threadIdx.x; q < a.slots * SmemSlot<KW>::kBytes / 16; q += kSmemThreads)
       z[q] = make_uint4(0, 0, 0, 0);
-    if (DBG_BITMAP)
-      for (uint64_t q = threadIdx.x; q < a.slots / 32; q += kSmemThreads) occ[q] = 0;
   }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned long long st_n = 0, st_count = 0, st_edges = 0;
@@ -1391,34 +1359,18 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       constexpr int S = RB;  // staging stride
       constexpr uint32_t kWarps = kSmemThreads / 32;
       typedef KeyOf<Code> KO;
-#if DBG_SADDR
-      // 32-bit shared-window addresses of the batch arrays, formed once per batch
-      const uint32_t rwin_s = smem_addr(st.rwin), pre_s = smem_addr(st.pre), desc_s = smem_addr(st.desc),
-                     wb_s = smem_addr(&st.w[bb][0][0]);
-#endif
       for (uint32_t m = warp; 32 * m < total; m += kWarps) {
         const uint32_t kb = 32 * m, kid = kb + lane;
         const bool act = kid < total;
-#if DBG_SADDR
-        const uint32_t rb = lds_u16(rwin_s + 2 * m);
-        const uint32_t nxt = rb + 1 + lane;
-        const uint32_t x0 = nxt < nc ? lds32(pre_s + 4 * nxt) : total;
-#else
         const uint32_t rb = st.rwin[m];
         // records starting inside the window: one bit each at their first K-mer
         const uint32_t nxt = rb + 1 + lane;
         const uint32_t x0 = nxt < nc ? st.pre[nxt] : total;
-#endif
         const uint32_t starts = __reduce_or_sync(kFull, x0 < kb + 32 ? 1u << (x0 - kb) : 0u);
         const uint32_t c = rb + __popc(starts & ((2u << lane) - 1u));
         const uint32_t cc = act ? c : rb;
-#if DBG_SADDR
-        const uint2 d = lds_u2(desc_s + 8 * cc);
-        const int t = (int)(kid - lds32(pre_s + 4 * cc));
-#else
         const uint2 d = st.desc[cc];
         const int t = (int)(kid - st.pre[cc]);
-#endif
         const int j = d.x & 1023u, n = (d.x >> 10) & 255u, hl = (d.x >> 18) & 1u, hr = (d.x >> 19) & 1u;
         const uint32_t t0 = d.y & 0xffffu, cap = d.y >> 16;
         const uint32_t* w = &st.w[bb][0][j];
@@ -1426,27 +1378,15 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         Code fwd, rc;
         int pred, succ;
         if constexpr (R == 4) {
-#if DBG_WORDSEL
           // the three data words, loaded unconditionally and selected (no branches): a1..a3
           // hold bases b .. b + 47 - 16q
-#if DBG_SADDR
-          const uint32_t wj = wb_s + 4 * (uint32_t)j;
-          const uint32_t d1 = lds32(wj + 4 * S), d2 = lds32(wj + 8 * S), d3 = lds32(wj + 12 * S);
-#else
           const uint32_t d1 = w[S], d2 = w[2 * S], d3 = w[3 * S];
-#endif
           const int q = b >> 4;
           const uint32_t a1 = q == 0 ? d1 : (q == 1 ? d2 : d3), a2 = q == 0 ? d2 : (q == 1 ? d3 : 0u),
                          a3 = q == 0 ? d3 : 0u;
           const int pb = b - 1, pq = pb >> 4;  // the predecessor base
           const uint32_t pw = pq <= 0 ? d1 : (pq == 1 ? d2 : d3);
           pred = b > 0 ? (int)((pw >> (30 - 2 * (pb & 15))) & 3u) : -1;
-#else
-          const int q = b >> 4;  // the words holding bases b .. b + 47 - 16q
-          const uint32_t a1 = w[(1 + q) * S], a2 = q < 2 ? w[(2 + q) * S] : 0u, a3 = q == 0 ? w[3 * S] : 0u;
-          const int pb = b - 1;  // the predecessor base
-          pred = b > 0 ? (int)((w[(1 + (pb >> 4)) * S] >> (30 - 2 * (pb & 15))) & 3u) : -1;
-#endif
           if constexpr (sizeof(Code) == 8) {
             // 64 bits of the record from base b: two 32-bit funnel shifts
             const uint32_t sh = 2 * (b & 15);
@@ -1479,37 +1419,6 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         uint32_t idx = __umulhi(smem_hash(code), cap);
         uint32_t inserted = 0;
         const uint32_t kaddr = keys_s + t0 * KB;
-#if DBG_BUCKET2
-        if constexpr (KW == 1) {
-          // buckets of two slots (the table's capacity and offset are even): one 16-byte
-          // load reads both keys; a lane claims the first empty one with a CAS and re-reads
-          // the bucket if it lost the race; a full bucket without its key moves it on
-          const uint32_t nbk = cap >> 1, b0 = __umulhi(smem_hash(code), nbk);
-          uint32_t bk = b0, sl = 0;
-          bool pend = want;
-          for (;;) {
-            const uint32_t ka = kaddr + bk * 16;
-            uint64_t k0, k1;
-            asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(k0), "=l"(k1) : "r"(ka) : "memory");
-            const bool m0 = k0 == key, m1 = k1 == key, e0 = k0 == 0, e1 = k1 == 0;
-            const bool found = m0 || m1;
-            const bool claim = pend && !found && (e0 || e1);
-            const uint32_t cs = e0 ? 0u : 1u;
-            uint64_t cur = 1;
-            cas_shared64_if(claim, ka + 8 * cs, key, cur);
-            const bool won = claim && cur == 0, same = claim && cur == key;
-            inserted |= (uint32_t)won;
-            sl = pend ? (found ? (m0 ? 0u : 1u) : cs) : sl;
-            const bool adv = pend && !found && !e0 && !e1;
-            const uint32_t nx = bk + 1 == nbk ? 0u : bk + 1;
-            bk = adv ? nx : bk;
-            if (adv && nx == b0) ok = false;  // wrapped: table full (reading O)
-            pend = pend && !found && !won && !same && !(adv && nx == b0);
-            if (!__any_sync(kFull, pend)) break;
-          }
-          idx = 2 * bk + sl;
-          if (!ok && want && lds64(kaddr + idx * KB) != key) idx = ~0u;  // this occurrence found no slot
-#elif DBG_PROBE_PRED
         if constexpr (KW == 1) {
           // every lane runs every probe round (predicated, no divergent branch): a lane with
           // nothing pending re-reads its current slot and keeps its state
@@ -1532,44 +1441,11 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             const uint64_t cur = lds64(kaddr + idx * KB);
             if (cur != key) idx = ~0u;  // this occurrence found no slot
           }
-#else
-        if constexpr (KW == 1) {
-          uint32_t probes = 0, pend = want;
-          while (__any_sync(kFull, pend)) {
-            if (pend) {
-              const uint32_t ka = kaddr + idx * KB;
-              uint64_t cur = lds64(ka);
-              if (cur == 0) cur = cas_shared64(ka, key);
-              inserted = cur == 0;
-              if (inserted | (cur == key)) {
-                pend = 0;
-              } else {
-                idx = idx + 1 == cap ? 0 : idx + 1;
-                if (++probes == cap) {  // wrapped: table full (reading O)
-                  pend = 0;
-                  ok = false;
-                  idx = ~0u;
-                }
-              }
-            }
-          }
-#endif
         } else {
           uint32_t probes = 0, pend = want;
           while (__any_sync(kFull, pend)) {
             if (pend) {
-#if DBG_KW2_LOAD
-              // load first, CAS only on an empty-looking entry: a 16-B shared load is not
-              // single-copy atomic, but entries only go (0, 0) -> key, and every key's hi word
-              // has OCC set, so a torn read is (0, lo), (hi, 0) or the key; (x, 0) / (0, x)
-              // are treated as empty and the CAS returns the entry atomically
-              const uint32_t ka = kaddr + idx * KB;
-              typename KO::T cur;
-              asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(cur.x), "=l"(cur.y) : "r"(ka) : "memory");
-              if (cur.x == 0 || cur.y == 0) cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);
-#else
               const typename KO::T cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);  // 16-B CAS: read-or-claim
-#endif
               inserted = KO::empty(cur);
               if (inserted | KO::same(cur, key)) {
                 pend = 0;
@@ -1586,19 +1462,9 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         }
         if (want && idx != ~0u) {  // the multiple updates: 16-bit fields, two per word
           const int fo = o < 4 ? o : 8;
-#if DBG_SLOT26
           const uint32_t h0 = (t0 + idx) * 9u, ho = h0 + (uint32_t)fo, hi = h0 + 4u + (uint32_t)i;
           red_shared_add(fld_s + (ho >> 1) * 4, 1u << (16 * (ho & 1)));
           if (i >= 0) red_shared_add(fld_s + (hi >> 1) * 4, 1u << (16 * (hi & 1)));
-#else
-          const uint32_t fa = fld_s + (t0 + idx) * (FW * 4);
-          if (inserted) {
-            if (!DBG_SLOT28) sts32(fa + 20, w[0] >> 10);
-            if (DBG_BITMAP) red_shared_or(occ_s + 4 * ((t0 + idx) >> 5), 1u << ((t0 + idx) & 31u));
-          }
-          red_shared_add(fa + 4 * (fo >> 1), 1u << (16 * (fo & 1)));
-          if (i >= 0) red_shared_add(fa + 4 * ((4 + i) >> 1), 1u << (16 * (i & 1)));
-#endif
         }
       }
     }
@@ -1616,7 +1482,6 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
       for (uint32_t sub = ws0; sub < ws1; sub += kQ) {
         const uint32_t se = min(ws1, sub + kQ);
         uint32_t qn = 0;
-#if DBG_XSCAN
         if (oa.min_count <= 1) {
           // occupied slots: the sign bit of the key's high 32-bit word (OCC); 32-bit shared
           // addresses formed once; two 32-slot chunks per iteration
@@ -1639,16 +1504,10 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             qn += __popc(b0);
           }
         } else
-#endif
         for (uint32_t c = sub; c < se; c += 32) {
           const uint32_t s = c + lane;
-#if DBG_BITMAP
-          bool keep = ((se - c >= 32 ? occ[c >> 5] : occ[c >> 5] & ((1u << (se - c)) - 1u)) >> lane) & 1u;
-#else
           bool keep = s < se && (lds64(keys_s + s * KB) & kOccupied);
-#endif
           if (keep && oa.min_count > 1) {  // row f4: a low-count vertex is cleaned, never emitted
-#if DBG_SLOT26
             uint16_t* f16 = reinterpret_cast<uint16_t*>(fld) + s * 9;
             if ((uint32_t)f16[0] + f16[1] + f16[2] + f16[3] + f16[8] < oa.min_count) {
               keep = false;
@@ -1658,54 +1517,37 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
 #pragma unroll
               for (int q = 0; q < 9; ++q) f16[q] = 0;
             }
-#else
-            const uint32_t* f = fld + s * FW;
-            const uint32_t f0 = f[0], f1 = f[1];
-            if ((f0 & 0xffffu) + (f0 >> 16) + (f1 & 0xffffu) + (f1 >> 16) + (f[4] & 0xffffu) < oa.min_count) {
-              keep = false;
-              unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
-              kp[0] = 0;
-              if (KW == 2) kp[1] = 0;
-              uint32_t* fz = fld + s * FW;
-#pragma unroll
-              for (uint32_t q = 0; q < FW; ++q) fz[q] = 0;
-            }
-#endif
           }
           const uint32_t bal = __ballot_sync(kFull, keep);
           if (keep) queue[qn + __popc(bal & ((1u << lane) - 1u))] = (uint16_t)s;
           qn += __popc(bal);
         }
-        if (DBG_BITMAP)
-          for (uint32_t c = (sub >> 5) + lane; c < (se + 31) >> 5; c += 32) occ[c] = 0;
         unsigned long long pos = 0;
         if (lane == 0 && qn) pos = atomicAdd(oa.n_out, (unsigned long long)qn);
         pos = __shfl_sync(kFull, pos, 0);
         __syncwarp();
-#if DBG_XEMIT && DBG_SLOT26
-        const uint32_t qe_s = smem_addr(queue);
-#endif
         for (uint32_t e = lane; e < qn; e += 32) {
-#if DBG_XEMIT && DBG_SLOT26
-          // explicit 32-bit shared addresses (formed from hoisted bases), 16-bit field loads
-          const uint32_t s = lds_u16(qe_s + 2 * e);
-          const uint32_t ka = keys_s + s * KB, fa = fld_s + 18u * s;
-          const uint64_t kw0 = lds64(ka);
+          const uint32_t s = queue[e];
+          unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
+          const uint64_t kw0 = kp[0];
           dbg_vertex v;
           if (KW == 1) {
             v.kmer_hi = 0;
             v.kmer_lo = kw0 & kCodeMask;
           } else {
             v.kmer_hi = kw0 & kCodeMask;
-            v.kmer_lo = lds64(ka + 8);
+            v.kmer_lo = kp[1];
           }
+          uint16_t* f16 = reinterpret_cast<uint16_t*>(fld) + s * 9;
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
-            v.out[q] = lds_u16(fa + 2 * q);
-            v.in[q] = lds_u16(fa + 8 + 2 * q);
+            v.out[q] = f16[q];
+            v.in[q] = f16[4 + q];
           }
-          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + lds_u16(fa + 16);  // count = sum(out) + t_out
-          uint32_t fpid = I.first;  // the fine partition owning slot s: last x with Pq[x] - P0 <= s
+          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + f16[8];  // count = sum(out) + t_out
+          // the fine partition owning slot s (last x with Pq[x] - P0 <= s), mod NP -- or the
+          // paper's partition from the vertex's P-minimizer (reading V)
+          uint32_t fpid = I.first;
           if (sub_n == 1) {
             uint32_t lo = 0, n = I.last - I.first;
             while (n > 1) {
@@ -1715,72 +1557,17 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             }
             fpid += lo;
           }
-          v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, fpid);
-          sts64(ka, 0);  // clean-on-extract
-          if (KW == 2) sts64(ka + 8, 0);
-#pragma unroll
-          for (int q = 0; q < 9; ++q) sts16(fa + 2 * q, 0);
-#else
-          const uint32_t s = queue[e];
-          unsigned long long* kp = reinterpret_cast<unsigned long long*>(keys + s * KB);
-          const uint64_t kw0 = kp[0];
-          uint32_t* f = fld + s * FW;
-          dbg_vertex v;
-          if (KW == 1) {
-            v.kmer_hi = 0;
-            v.kmer_lo = kw0 & kCodeMask;
-          } else {
-            v.kmer_hi = kw0 & kCodeMask;
-            v.kmer_lo = kp[1];
-          }
-#if DBG_SLOT26
-          uint16_t* f16 = reinterpret_cast<uint16_t*>(fld) + s * 9;
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            v.out[q] = f16[q];
-            v.in[q] = f16[4 + q];
-          }
-          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + f16[8];  // count = sum(out) + t_out
-#else
-          const uint32_t f0 = f[0], f1 = f[1], f2 = f[2], f3 = f[3], f4 = f[4];
-          v.out[0] = f0 & 0xffffu; v.out[1] = f0 >> 16; v.out[2] = f1 & 0xffffu; v.out[3] = f1 >> 16;
-          v.in[0] = f2 & 0xffffu; v.in[1] = f2 >> 16; v.in[2] = f3 & 0xffffu; v.in[3] = f3 >> 16;
-          v.count = v.out[0] + v.out[1] + v.out[2] + v.out[3] + (f4 & 0xffffu);  // count = sum(out) + t_out
-#endif
-          // fine pid recorded by the inserting thread, mod NP (or from the P-minimizer, reading V)
-          uint32_t fpid;
-          if (DBG_SLOT28) {  // the fine partition owning slot s: last x with Pq[x] - P0 <= s
-            fpid = I.first;
-            if (sub_n == 1) {
-              uint32_t lo = 0, n = I.last - I.first;
-              while (n > 1) {
-                const uint32_t h = n >> 1;
-                if (Pq[lo + h] - I.P0 <= s) lo += h, n -= h;
-                else n = h;
-              }
-              fpid += lo;
-            }
-          } else {
-            fpid = f[FW - 1];
-          }
-          v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, fpid);
+          if constexpr (PC > 0)  // compile-time (K, P) of the launch, fine_p != P (reading V)
+            v.pid = kmer_partition_c<KC, PC>(v.kmer_lo, oa);
+          else
+            v.pid = oa.kmer_pid ? kmer_partition(v.kmer_hi, v.kmer_lo, oa) : fast_mod(a.np_mod, fpid);
           kp[0] = 0;  // clean-on-extract
           if (KW == 2) kp[1] = 0;
-#if DBG_SLOT26
 #pragma unroll
           for (int q = 0; q < 9; ++q) f16[q] = 0;
-#else
-#pragma unroll
-          for (uint32_t q = 0; q < FW; ++q) f[q] = 0;
-#endif
-#endif  // DBG_XEMIT
           const uint64_t my = pos + e;
           if (my < oa.out_cap) {
-#if DBG_VSTORE
             store_vertex16(oa.out + my, v, (my & 1) != 0);
-#else
-            oa.out[my] = v;
-#endif
           }
           else atomicOr(oa.status, kStatusNoSpace);
           st_n += 1;
@@ -1945,68 +1732,48 @@ extern "C" dbg_status dbg_extract_graph(const dbg_params* prm, void* d_table, co
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 
-// CTAs per SM of the on-chip kernel (env DBG_SMEM_CTAS):
-// several CTAs overlap one partition's load/scan/extract latencies with
-// another's hashing; the table per CTA shrinks accordingly.
-// 0 = one CTA of 1024 threads per SM (the default), 1/2/4 = that many CTAs of
-// 512/256/128 threads.
-static int smem_ctas() {
-  static int v = [] {
-    const char* e = getenv("DBG_SMEM_CTAS");
-    const int x = e ? atoi(e) : 0;
-    return (x == 0 || x == 1 || x == 2 || x == 4) ? x : 0;
-  }();
-  return v;
-}
-
 template <int R, int T>
 static uint64_t smem_slots_for(int k, int ctas) {
   const uint64_t avail = (227u * 1024u) / ctas - smem_fixed_bytes<R, T>() - 1024u;
   const uint32_t sb = k <= 31 ? SmemSlot<1>::kBytes : SmemSlot<2>::kBytes;
-  const uint64_t n = (8 * avail / (8 * sb + (DBG_BITMAP ? 1 : 0))) & ~(uint64_t)63;  // (+ 1 bit of bitmap)
+  const uint64_t n = (avail / sb) & ~(uint64_t)63;
   return n < kSmemMaxSlots ? n : kSmemMaxSlots;
 }
 
-static uint64_t smem_slots(int k, int ctas) {
-  const bool r4 = record_words(k) == 4;
-  switch (ctas) {
-    case 0: return r4 ? smem_slots_for<4, 1024>(k, 1) : smem_slots_for<8, 1024>(k, 1);
-    case 1: return r4 ? smem_slots_for<4, 512>(k, 1) : smem_slots_for<8, 512>(k, 1);
-    case 2: return r4 ? smem_slots_for<4, 256>(k, 2) : smem_slots_for<8, 256>(k, 2);
-    default: return r4 ? smem_slots_for<4, 128>(k, 4) : smem_slots_for<8, 128>(k, 4);
-  }
+// One persistent CTA of 1024 threads per SM (several smaller CTAs per SM measured slower,
+// profiles/r01d_ab.txt).
+static uint64_t smem_slots(int k) {
+  return record_words(k) == 4 ? smem_slots_for<4, 1024>(k, 1) : smem_slots_for<8, 1024>(k, 1);
 }
 
 extern "C" uint64_t dbg_smem_table_slots(const dbg_params* prm) {
   if (!prm || prm->k > 63) return 0;
-  return smem_slots(prm->k, smem_ctas());
+  return smem_slots(prm->k);
 }
 
-template <typename Code, int R, int T, int C, int KC = 0>
+template <typename Code, int R, int T, int C, int KC = 0, int PC = 0>
 static cudaError_t launch_smem_t(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
   constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes + (DBG_BITMAP ? a.slots / 8 : 0);
-  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C, KC>,
+  const size_t bytes = smem_fixed_bytes<R, T>() + a.slots * SmemSlot<KW>::kBytes;
+  cudaError_t e = cudaFuncSetAttribute(smem_subgraph_kernel<Code, R, T, C, KC, PC>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   if (e != cudaSuccess) return e;
-  smem_subgraph_kernel<Code, R, T, C, KC><<<dbg_sm_count() * C, T, bytes, stream>>>(a, oa);
+  smem_subgraph_kernel<Code, R, T, C, KC, PC><<<dbg_sm_count() * C, T, bytes, stream>>>(a, oa);
   return cudaGetLastError();
 }
 
 template <typename Code, int R>
 static cudaError_t launch_smem(const SmemArgs& a, const OutArgs& oa, cudaStream_t stream) {
-  switch (smem_ctas()) {
-    case 0:
-      // the configurations' K (31, 63) as a compile-time constant in the default variant
-      if constexpr (DBG_KCONST && sizeof(Code) == 8 && R == 4)
-        if (a.k == 31) return launch_smem_t<Code, R, 1024, 1, 31>(a, oa, stream);
-      if constexpr (DBG_KCONST && sizeof(Code) == 16 && R == 8)
-        if (a.k == 63) return launch_smem_t<Code, R, 1024, 1, 63>(a, oa, stream);
-      return launch_smem_t<Code, R, 1024, 1>(a, oa, stream);
-    case 1: return launch_smem_t<Code, R, 512, 1>(a, oa, stream);
-    case 2: return launch_smem_t<Code, R, 256, 2>(a, oa, stream);
-    default: return launch_smem_t<Code, R, 128, 4>(a, oa, stream);
-  }
+  // the configurations' K (31, 63) as a compile-time constant (shifts and masks by constants)
+  if constexpr (sizeof(Code) == 8 && R == 4)
+    if (a.k == 31) {
+      if (oa.kmer_pid && oa.p == 11)  // chr14's launch: P = 11 vertex partitions under fine_p > P
+        return launch_smem_t<Code, R, 1024, 1, 31, 11>(a, oa, stream);
+      return launch_smem_t<Code, R, 1024, 1, 31>(a, oa, stream);
+    }
+  if constexpr (sizeof(Code) == 16 && R == 8)
+    if (a.k == 63) return launch_smem_t<Code, R, 1024, 1, 63>(a, oa, stream);
+  return launch_smem_t<Code, R, 1024, 1>(a, oa, stream);
 }
 
 extern "C" int32_t dbg_smem_onchip(const dbg_params* prm, uint64_t n_kmers) {
@@ -2086,7 +1853,7 @@ extern "C" dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_gc, tiles);
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_sp, tiles);
   smem_plan_apply_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
-  if (!getenv("DBG_GROUPS_WINDOW")) smem_plan_pack_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
+  smem_plan_pack_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
   tile_scan_kernel<<<1, kTileScanThreads, 0, stream>>>(a.t_fl, tiles);
   smem_plan_groups_kernel<<<tiles, kTileThreads, 0, stream>>>(a);
   smem_plan_desc_kernel<<<(a.n_fine + 255) / 256 < dbg_sm_count() * 8 ? (a.n_fine + 255) / 256 : dbg_sm_count() * 8,

@@ -30,6 +30,7 @@
 #include <cub/block/block_scan.cuh>
 
 #include <algorithm>
+#include <type_traits>
 #include <cstdlib>
 
 #include "dbg_device.cuh"
@@ -38,30 +39,10 @@
 namespace dbg {
 
 constexpr int kMspThreads = 128;
-constexpr int kMaxDesc = 40;             // descriptors per thread between flushes (>= 34)
 // msp_block_kernel variants (A/B builds, tools/build_variants.py)
-#ifndef DBG_MSP_FUSED
-#define DBG_MSP_FUSED 0   // 1: running prefix minimum interleaved with the K-mer emission
-#endif
-#ifndef DBG_MSP_STCS
-#define DBG_MSP_STCS 0  // evict-first staging stores
-#endif
-#ifndef DBG_MSP_TAIL
-#define DBG_MSP_TAIL 0  // 1: the read's last superkmer appended after the block loop
-#endif
-#ifndef DBG_MSP_NOBR
-#define DBG_MSP_NOBR 0  // 1: branch-free base consumption (padding past the read end)
-#endif
-#ifndef DBG_MSP_DESC
-#define DBG_MSP_DESC 40   // descriptors per thread between flushes (>= W + 3)
-#endif
-#ifndef DBG_MSP_CTAS
-#define DBG_MSP_CTAS 1    // __launch_bounds__ min CTAs per SM (1: no register cap)
-#endif
-constexpr int kMaxDescBlock = DBG_MSP_DESC;
-constexpr int kMspBlockCtas = DBG_MSP_CTAS;
+constexpr int kMaxDescBlock = 40;  // descriptors per thread between flushes (>= W + 3)
 constexpr int kSmemHistMaxNp = 8192;
-constexpr int kTwoLevelBins = 512;  // level-1 bins of the two-level scatter
+constexpr int kBucketShift = 3;  // two-level scatter: buckets of 8 consecutive fine partitions (r02f: 3 < 4 < 5 < 6)
 
 struct MspArgs {
   const uint64_t* words;
@@ -76,7 +57,6 @@ struct MspArgs {
   uint32_t* staging;              // records in read order
   uint64_t staging_cap;           // records
   unsigned long long* staged;     // cursor (records reserved)
-  uint32_t* rank;                 // [staging_cap] record rank inside its partition, or null
   uint32_t pid_lo, pid_hi;        // only superkmers of fine partitions [pid_lo, pid_hi) are counted and staged
   bool ranged;                    // pid_lo > 0 or pid_hi < np
 };
@@ -194,15 +174,16 @@ __device__ __forceinline__ void write_record4(const MspArgs& a, uint32_t* dst, u
   const uint32_t b1 = (uint32_t)(v1 >> 32) & m1;
   const uint4 rec = make_uint4((uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10), (uint32_t)(b0 >> 32),
                                (uint32_t)b0, b1);
-  if (DBG_MSP_STCS) __stcs(reinterpret_cast<uint4*>(dst), rec);
-  else reinterpret_cast<uint4*>(dst)[0] = rec;
+  reinterpret_cast<uint4*>(dst)[0] = rec;
 }
 
 // Warp-collective flush of the per-thread descriptor lists: partition ids
 // (computed once per descriptor and kept in place of the minimizer), size
 // histograms, one staging reservation per warp, record writes.
 // kK > 0: compile-time K (record geometry and pieces without runtime division).
-template <typename CT, int kK = 0>
+// kPid: the descriptors already hold the partition id (or kSkip), computed when the superkmer
+// closed (msp_kernel), instead of the minimizer.
+template <typename CT, int kK = 0, bool kPid = false>
 __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
                                                   int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
@@ -215,9 +196,12 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     for (int d = 0; d < ndesc; ++d) {
       const int e = (int)sm.desc_e[d * kMspThreads + tid];
       CT& dm = sm.desc_m[d * kMspThreads + tid];
-      const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64((uint64_t)dm));
-      const bool in = !a.ranged || (pid - a.pid_lo < a.pid_hi - a.pid_lo);
-      dm = in ? (CT)pid : kSkip;
+      bool in = dm != kSkip;
+      if constexpr (!kPid) {
+        const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64((uint64_t)dm));
+        in = !a.ranged || (pid - a.pid_lo < a.pid_hi - a.pid_lo);
+        dm = in ? (CT)pid : kSkip;
+      }
       if (in) my_records += record_pieces(e - s + 1, nmax);
       s = e + 1;
     }
@@ -245,20 +229,14 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     }
     const uint32_t pid = (uint32_t)dm;
     const int n = e - s + 1;
-    // the record counter's old value ranks this superkmer's pieces inside the partition (d_rank)
-    uint32_t r = 0;
-    if (a.rank)
-      r = (uint32_t)atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
-    else
-      atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
+    atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
     atomicAdd(a.n_kmers + pid, (unsigned long long)n);
-    for (int ps = s; ps <= e; ps += nmax, ++slot, ++r) {
+    for (int ps = s; ps <= e; ps += nmax, ++slot) {
       if (slot < a.staging_cap) {
         if (r4)
           write_record4(a, a.staging + slot * 4, o, L, ps, min(e, ps + nmax - 1), pid);
         else
           write_record(a, a.staging + slot * a.rec_words, o, L, ps, min(e, ps + nmax - 1), pid);
-        if (a.rank) a.rank[slot] = r;  // after the record: its loads overlap the atomic's latency
       }
     }
     s = e + 1;
@@ -267,41 +245,79 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
   ndesc = 0;
 }
 
-#ifndef DBG_MSP_U64_FLUSH
-#define DBG_MSP_U64_FLUSH 0  // 64-bit P-mer codes: flush vote every 16 bases, 18 descriptors (3 CTAs/SM)
-#endif
-// Bases between flush votes and the descriptor capacity: a run of B bases closes
-// at most one superkmer per K-mer plus the read's last one (capacity >= B + 2).
-template <typename CT>
-constexpr int msp_flush_bases() { return (sizeof(CT) == 8 && DBG_MSP_U64_FLUSH) ? 16 : 32; }
-template <typename CT>
-constexpr int msp_max_desc() { return msp_flush_bases<CT>() == 32 ? kMaxDesc : msp_flush_bases<CT>() + 2; }
+// The generic kernel flushes its descriptor lists when a vote every kMspFlushBases bases finds one
+// with more than kMspDesc - (kMspFlushBases + 2) entries: a run of B bases closes at most one
+// superkmer per K-mer plus the read's last one.  A descriptor is (last K-mer, partition id), the
+// id computed when the superkmer closes, so a list costs 8 bytes per entry.  The shared memory per
+// thread (the van Herk row of w codes + the list) sets the occupancy of this latency-bound kernel:
+// 24 entries and a vote every 8 bases instead of 40 entries of (end, minimizer) and a vote every
+// 32 bases take K = 63 (P = 19, 64-bit codes) from 107.5 KB to 70.7 KB per CTA, 2 -> 3 CTAs/SM.
+constexpr int kMspFlushBases = 8, kMspDesc = 24;
+static_assert(kMspDesc >= kMspFlushBases + 2, "one vote interval must fit an empty list");
 
-// kMaxDesc >= 32 + 2: a 32-base chunk closes at most one superkmer per K-mer
-// plus the read's last one, so the flush vote is needed once per chunk.
-template <typename CT>
+// One thread's column of the van Herk row in shared memory.  kRow40: 64-bit codes of P <= 20
+// (< 2^40) kept as a 32-bit high part (bits 8..39) and an 8-bit low part -- 5 instead of 8 bytes
+// per entry, which for K = 63, P = 19 takes the CTA from 70.7 KB to 53.4 KB (3 -> 4 CTAs/SM).
+template <typename CT, bool kRow40>
+struct RowIO {
+  uint32_t hi_a, lo_a;
+  static constexpr uint32_t kStep = kMspThreads * (kRow40 ? 4u : (uint32_t)sizeof(CT));
+  __device__ __forceinline__ CT ld(int u) const {
+    if constexpr (kRow40) {
+      uint32_t h, l;
+      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(h) : "r"(hi_a + (uint32_t)u * kStep) : "memory");
+      asm volatile("ld.shared.u8 %0, [%1];" : "=r"(l) : "r"(lo_a + (uint32_t)u * kMspThreads) : "memory");
+      return ((CT)h << 8) | (CT)l;
+    } else {
+      return sh_ld(hi_a + (uint32_t)u * kStep, (CT)0);
+    }
+  }
+  __device__ __forceinline__ void st(int u, CT v) const {
+    if constexpr (kRow40) {
+      sh_st(hi_a + (uint32_t)u * kStep, (uint32_t)(v >> 8));
+      asm volatile("st.shared.u8 [%0], %1;" ::"r"(lo_a + (uint32_t)u * kMspThreads), "r"((uint32_t)v & 255u)
+                   : "memory");
+    } else {
+      sh_st(hi_a + (uint32_t)u * kStep, v);
+    }
+  }
+  static size_t bytes(int w) { return (size_t)w * kMspThreads * (kRow40 ? 5u : sizeof(CT)); }
+};
+
+__device__ __forceinline__ uint32_t desc_pid(const MspArgs& a, uint64_t m) {
+  const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
+  return (!a.ranged || pid - a.pid_lo < a.pid_hi - a.pid_lo) ? pid : ~0u;
+}
+
+template <typename CT, bool kRow40>
 __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int tid = threadIdx.x, lane = tid & 31;
-  MspSmem<CT> sm;
+  MspSmem<uint32_t> sm;  // descriptors: end + partition id
   unsigned char* sp = smem_raw;
-  sm.desc_m = reinterpret_cast<CT*>(sp);
-  constexpr int kDesc = msp_max_desc<CT>(), kFB = msp_flush_bases<CT>();
-  sp += sizeof(CT) * kDesc * kMspThreads;
+  sm.desc_m = reinterpret_cast<uint32_t*>(sp);
+  constexpr int kDesc = kMspDesc, kFB = kMspFlushBases;
+  sp += sizeof(uint32_t) * kDesc * kMspThreads;
   sm.desc_e = reinterpret_cast<uint32_t*>(sp);
   sp += sizeof(uint32_t) * kDesc * kMspThreads;
-  sm.row = reinterpret_cast<CT*>(sp);
+  sm.row = nullptr;
+  CT* row0 = reinterpret_cast<CT*>(sp);
 
   const int K = a.k, P = in_reg(a.p), w = in_reg(a.w);
   const CT maskP = in_reg((CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1)));
   const int topP = in_reg(2 * P - 2);
   const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
-  CT* row = sm.row + tid;
   // shared-window addresses of this thread's column of the van Herk block and descriptors
-  const uint32_t row_a = in_reg(sh_addr(row)), de_a = in_reg(sh_addr(sm.desc_e + tid)),
-                 dm_a = in_reg(sh_addr(sm.desc_m + tid));
-  constexpr uint32_t kRowStep = kMspThreads * sizeof(CT), kDescStepE = kMspThreads * 4,
-                     kDescStepM = kMspThreads * sizeof(CT);
+  RowIO<CT, kRow40> row;
+  if constexpr (kRow40) {
+    row.hi_a = in_reg(sh_addr(reinterpret_cast<uint32_t*>(row0) + tid));
+    row.lo_a = in_reg(sh_addr(reinterpret_cast<unsigned char*>(row0) + 4 * (size_t)a.w * kMspThreads + tid));
+  } else {
+    row.hi_a = in_reg(sh_addr(row0 + tid));
+    row.lo_a = 0;
+  }
+  const uint32_t de_a = in_reg(sh_addr(sm.desc_e + tid)), dm_a = in_reg(sh_addr(sm.desc_m + tid));
+  constexpr uint32_t kDescStepE = kMspThreads * 4, kDescStepM = kMspThreads * 4;
   // all lanes of a warp iterate together; a warp covers 32 consecutive reads
   for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
     const uint64_t r = r0 + lane;
@@ -318,6 +334,9 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
     for (int dlt = 16; dlt; dlt >>= 1) Lmax = max(Lmax, __shfl_xor_sync(kFull, Lmax, dlt));
     int ndesc = 0, s_next = 0;
     CT f = 0, rc = 0, pre = 0, m_cur = 0;
+    // nxt = row[u + 1], loaded one P-mer ahead so that the shared-memory latency is off the
+    // per-base dependency chain (in the read's first block it is never used)
+    CT nxt = 0;
     int u = 0;  // position within the current van Herk block
     for (int c0 = 0; c0 < Lmax; c0 += 32) {
       uint64_t wbuf = c0 < L ? window64(a.words, a.n_words, o + c0) : 0;
@@ -332,43 +351,54 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
         rc = (rc >> 2) | ((CT)(3u - b) << topP);
         if (j < P - 1) continue;
         const int q = j - P + 1;  // P-mer index
+        const CT snext = nxt;
+        if (u + 2 < w) nxt = row.ld(u + 2);  // for the next P-mer
         const CT c = f < rc ? f : rc;
-        const uint32_t ua = row_a + (uint32_t)u * kRowStep;
-        const CT snext = (u + 1 < w) ? sh_ld(ua + kRowStep, (CT)0) : (CT)0;
-        sh_st(ua, c);
+        row.st(u, c);
         pre = (u == 0 || c < pre) ? c : pre;
         if (q >= w - 1) {  // K-mer i = q-w+1 is complete
           const int i = q - w + 1;
           const CT m = (u == w - 1 || pre < snext) ? pre : snext;
           if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
             sh_st(de_a + (uint32_t)ndesc * kDescStepE, (uint32_t)(i - 1));
-            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, m_cur);
+            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, desc_pid(a, (uint64_t)m_cur));
             ++ndesc;
           }
           m_cur = m;
           if (i == nk - 1) {  // the read's last superkmer
             sh_st(de_a + (uint32_t)ndesc * kDescStepE, (uint32_t)i);
-            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, m_cur);
+            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, desc_pid(a, (uint64_t)m_cur));
             ++ndesc;
           }
         }
-        if (u == w - 1) {  // block complete: suffix minima in place
-          CT y = sh_ld(row_a + (uint32_t)(w - 1) * kRowStep, (CT)0);
-          for (int t = w - 2; t >= 0; --t) {
-            const uint32_t ta = row_a + (uint32_t)t * kRowStep;
-            const CT x = sh_ld(ta, (CT)0);
-            if (y < x) sh_st(ta, y);
+        if (u == w - 1) {  // block complete: suffix minima in place, loads issued 8 at a time
+          CT y = row.ld(w - 1);
+          int t = w - 2;
+          for (; t >= 7; t -= 8) {
+            CT x[8];
+#pragma unroll
+            for (int v = 0; v < 8; ++v) x[v] = row.ld(t - v);
+#pragma unroll
+            for (int v = 0; v < 8; ++v) {
+              if (y < x[v]) row.st(t - v, y);
+              else y = x[v];
+            }
+          }
+          for (; t >= 0; --t) {
+            const CT x = row.ld(t);
+            if (y < x) row.st(t, y);
             else y = x;
           }
           u = 0;
+          if (w > 1) nxt = row.ld(1);
         } else {
           ++u;
         }
       }
-      if (__any_sync(kFull, ndesc > kDesc - (kFB + 2))) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+      if (__any_sync(kFull, ndesc > kDesc - (kFB + 2))) flush_descriptors<uint32_t, 0, true>(a, sm, ndesc, s_next, o, L);
       }
     }
-    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
+    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<uint32_t, 0, true>(a, sm, ndesc, s_next, o, L);
   }
 }
 
@@ -378,42 +408,60 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
 // consecutive partitions, whose records are contiguous in partition order).
 // nb bins; with nb <= kSmemHistMaxNp a CTA tile ranks its records in shared
 // memory and reserves once per bin, else one global atomic per record.
-#ifndef DBG_SCATTER_PER
-#define DBG_SCATTER_PER 4
-#endif
-#ifndef DBG_SCATTER_STCS
-#define DBG_SCATTER_STCS 0  // evict-first record stores
-#endif
-#ifndef DBG_SCATTER_ABS
-#define DBG_SCATTER_ABS 0  // global-path cursors start at the record offsets
-#endif
-#ifndef DBG_SCATTER_A32
-#define DBG_SCATTER_A32 0  // 32-bit rank atomics
-#endif
-#ifndef DBG_SCATTER_GRID
-#define DBG_SCATTER_GRID 0  // CTAs per SM (0: the occupancy limit)
-#endif
-#ifndef DBG_SCATTER_MINB
-#define DBG_SCATTER_MINB 4
-#endif
+// L2 cache policies of the scatter: the staged records stream through once (evict first); the
+// partitions' open sectors, their cursors and offsets stay (evict last), so a 32-byte sector
+// that receives a 16-byte record is still in L2 when its other half arrives and is written back
+// whole -- without it every record store costs a DRAM read-modify-write of its sector.
+__device__ __forceinline__ uint64_t l2_policy_last() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_first() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint4 ld_stream16(const uint4* p, uint64_t pol) {
+  uint4 v;
+  asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ void st_keep16(uint4* p, uint4 v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;"
+               :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_keep8(const uint64_t* p, uint64_t pol) {
+  uint64_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ unsigned long long atom_add_keep(unsigned long long* p, unsigned long long v,
+                                                            uint64_t pol) {
+  unsigned long long r;
+  asm volatile("atom.global.add.L2::cache_hint.u64 %0, [%1], %2, %3;" : "=l"(r) : "l"(p), "l"(v), "l"(pol)
+               : "memory");
+  return r;
+}
+
 constexpr int kScatterThreads = 256;
-constexpr int kScatterPer = DBG_SCATTER_PER;  // records per thread per tile
+constexpr int kScatterPer = 4;  // records per thread per tile
 template <int R>
-__global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_kernel(const uint32_t* __restrict__ staging,
+__global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint32_t* __restrict__ staging,
                                                                   const unsigned long long* staged,
                                                                   uint64_t staging_cap,
                                                                   const uint64_t* __restrict__ rec_off,
                                                                   unsigned long long* fill,
                                                                   uint32_t* __restrict__ records, int nb, int shift,
-                                                                  bool abs_pos, uint32_t* const* peer_records,
+                                                                  uint32_t* const* peer_records,
                                                                   const int32_t* peer_bounds, int n_peers) {
-  // abs_pos (global path, shift 0): the cursors start at the partitions' record offsets, so the
-  // rank atomic returns the record's final position (no offset load)
   extern __shared__ unsigned long long sh_base[];  // [nb] global bases (per tile), then [nb] counts
   uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_base + nb);
   const uint64_t n = *staged;
   if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
   const bool smem = nb <= kSmemHistMaxNp;
+  const uint64_t pol_first = l2_policy_first(), pol_last = l2_policy_last();
   constexpr int kPer = R >= 16 ? 2 : kScatterPer;
   constexpr int kTile = kScatterThreads * kPer;
   for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile) {
@@ -423,7 +471,6 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
     }
     uint4 rec[kPer][R / 4];
     uint32_t rank[kPer];
-    uint64_t apos[kPer];
     // all loads of the tile first, then all rank atomics, then all stores: kPer records of
     // each thread in flight at every stage (the kernel is latency-bound)
 #pragma unroll
@@ -432,29 +479,25 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
       if (idx < n) {
         const uint4* src = reinterpret_cast<const uint4*>(staging + idx * R);
 #pragma unroll
-        for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(src + c);
+        for (int c = 0; c < R / 4; ++c) rec[v][c] = ld_stream16(src + c, pol_first);
       }
     }
 #pragma unroll
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       rank[v] = 0;
-      apos[v] = 0;
       if (idx < n) {
         const uint32_t bin = (rec[v][0].x >> 10) >> shift;
-        if (abs_pos) apos[v] = atomicAdd(fill + bin, 1ull);
-        else if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
-        else if (DBG_SCATTER_A32)  // the low half of the (zeroed) 64-bit cursor: counts < 2^32
-          rank[v] = atomicAdd(reinterpret_cast<unsigned int*>(fill + bin), 1u);
-        else
-          rank[v] = (uint32_t)atomicAdd(fill + bin, 1ull);
+        if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
+        else rank[v] = (uint32_t)atom_add_keep(fill + bin, 1ull, pol_last);
       }
     }
     uint64_t base[kPer];
 #pragma unroll
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
-      base[v] = idx < n && !abs_pos ? __ldg(rec_off + (((rec[v][0].x >> 10) >> shift) << shift)) : 0;
+      const uint64_t* op = rec_off + (((rec[v][0].x >> 10) >> shift) << shift);
+      base[v] = idx < n ? ld_keep8(op, pol_last) : 0;
     }
     if (smem) {
       __syncthreads();
@@ -467,7 +510,7 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       if (idx < n) {
         const uint32_t bin = (rec[v][0].x >> 10) >> shift;
-        const uint64_t pos = abs_pos ? apos[v] : base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
+        const uint64_t pos = base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
         uint32_t* out = records;
         if (n_peers) {  // multi-GPU emission: the owner's buffer, through its IPC-mapped pointer
           const int32_t pid = (int32_t)(rec[v][0].x >> 10);
@@ -477,59 +520,20 @@ __global__ void __launch_bounds__(kScatterThreads, DBG_SCATTER_MINB) scatter_ker
         }
         uint4* dst = reinterpret_cast<uint4*>(out + pos * R);
 #pragma unroll
-        for (int c = 0; c < R / 4; ++c) {
-          if (DBG_SCATTER_STCS) __stcs(dst + c, rec[v][c]);
-          else dst[c] = rec[v][c];
-        }
+        for (int c = 0; c < R / 4; ++c) st_keep16(dst + c, rec[v][c], pol_last);
       }
     }
     if (smem) __syncthreads();
   }
 }
 
-// Pass 3 with pass-1 ranks (dbg_partition_set.d_rank): record j goes to
-// rec_off[pid] + rank[j] -- no rank atomics, a pure gather/scatter of 16-B
-// (or wider) records.
-template <int R>
-__global__ void __launch_bounds__(256) scatter_rank_kernel(const uint32_t* __restrict__ staging,
-                                                           const uint32_t* __restrict__ rank,
-                                                           const unsigned long long* staged, uint64_t staging_cap,
-                                                           const uint64_t* __restrict__ rec_off,
-                                                           uint32_t* __restrict__ records) {
-  const uint64_t n = *staged;
-  if (n > staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
-  constexpr int kPer = 4;
-  for (uint64_t t0 = (uint64_t)blockIdx.x * 256 * kPer; t0 < n; t0 += (uint64_t)gridDim.x * 256 * kPer) {
-    uint4 rec[kPer][R / 4];
-    uint32_t rk[kPer];
-#pragma unroll
-    for (int v = 0; v < kPer; ++v) {
-      const uint64_t idx = t0 + v * 256 + threadIdx.x;
-      if (idx < n) {
-        const uint4* src = reinterpret_cast<const uint4*>(staging + idx * R);
-#pragma unroll
-        for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(src + c);
-        rk[v] = __ldcs(rank + idx);
-      }
-    }
-#pragma unroll
-    for (int v = 0; v < kPer; ++v) {
-      const uint64_t idx = t0 + v * 256 + threadIdx.x;
-      if (idx < n) {
-        const uint64_t pos = __ldg(rec_off + (rec[v][0].x >> 10)) + rk[v];
-        uint4* dst = reinterpret_cast<uint4*>(records + pos * R);
-#pragma unroll
-        for (int c = 0; c < R / 4; ++c) dst[c] = rec[v][c];
-      }
-    }
-  }
-}
-
 // Two-level scatter, level 2: one CTA per bucket of 2^shift consecutive
 // partitions (grid-stride over buckets).  The bucket's records are
 // contiguous in src (level 1); each is ranked inside its partition with a
-// shared-memory atomic and written to rec_off[pid] + rank in dst.  The
-// bucket's partition offsets are staged in shared memory.
+// shared-memory atomic and written to rec_off[pid] + rank in dst (or, with
+// peers, in the owner's buffer).  The bucket's output range is small (about
+// 2^shift x 190 records on chr14), so its 32-byte sectors are completed while
+// they are in L2 and written back whole.
 constexpr int kBucketThreads = 512;
 constexpr int kBucketPer = 4;
 template <int R>
@@ -537,11 +541,14 @@ __global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const ui
                                                                         const unsigned long long* staged,
                                                                         uint64_t staging_cap,
                                                                         const uint64_t* __restrict__ rec_off,
-                                                                        uint32_t* __restrict__ dst, int np, int shift) {
+                                                                        uint32_t* __restrict__ dst, int np, int shift,
+                                                                        uint32_t* const* peer_records,
+                                                                        const int32_t* peer_bounds, int n_peers) {
   extern __shared__ unsigned long long sh_off[];  // [2^shift + 1] offsets, then [2^shift] counts
   const int bw = 1 << shift;
   uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_off + bw + 1);
   if (*staged > staging_cap) return;
+  const uint64_t pol_first = l2_policy_first();
   const int nbk = (np + bw - 1) >> shift;
   constexpr int kTile = kBucketThreads * kBucketPer;
   for (int bk = blockIdx.x; bk < nbk; bk += gridDim.x) {
@@ -560,16 +567,22 @@ __global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const ui
         if (idx < r1) {
           const uint4* s4 = reinterpret_cast<const uint4*>(src + idx * R);
 #pragma unroll
-          for (int c = 0; c < R / 4; ++c) rec[v][c] = __ldcs(s4 + c);
+          for (int c = 0; c < R / 4; ++c) rec[v][c] = ld_stream16(s4 + c, pol_first);
         }
       }
 #pragma unroll
       for (int v = 0; v < kBucketPer; ++v) {
         const uint64_t idx = t0 + v * kBucketThreads + threadIdx.x;
         if (idx < r1) {
-          const uint32_t lp = (rec[v][0].x >> 10) - (uint32_t)p0;
+          const uint32_t pid = rec[v][0].x >> 10, lp = pid - (uint32_t)p0;
           const uint64_t pos = sh_off[lp] + atomicAdd(sh_cnt + lp, 1u);
-          uint4* d4 = reinterpret_cast<uint4*>(dst + pos * R);
+          uint32_t* out = dst;
+          if (n_peers) {  // multi-GPU emission: the owner's buffer, through its IPC-mapped pointer
+            int o = 0;
+            while (o + 1 < n_peers && (int32_t)pid >= __ldg(peer_bounds + o + 1)) ++o;
+            out = peer_records[o];
+          }
+          uint4* d4 = reinterpret_cast<uint4*>(out + pos * R);
 #pragma unroll
           for (int c = 0; c < R / 4; ++c) d4[c] = rec[v][c];
         }
@@ -587,23 +600,34 @@ __global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const ui
 // min(suffix_min_prev[t], prefix_min_cur[t-1]) for i = q0 - W + t, where the
 // current block holds P-mers q0 .. q0+W-1.  Same descriptors and flush as
 // msp_kernel; reads of any length (lanes past their read end run masked).
+// P-mer codes of the register-blocked kernel: 32-bit up to P = 16, else 64-bit (K = 63, P = 19);
+// descriptor lists hold at least W + 3 entries (a block of W bases closes at most W superkmers,
+// plus the read's last one and the carry).
 template <int W, int P>
-__global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(MspArgs a) {
-  typedef uint32_t CT;
+struct MspBlockCfg {
+  typedef std::conditional_t<(P <= 16), uint32_t, uint64_t> CT;
+  static constexpr int kDesc = W + 3 > kMaxDescBlock ? W + 3 : kMaxDescBlock;
+  static constexpr size_t smem() { return (sizeof(CT) + sizeof(uint32_t)) * kDesc * kMspThreads; }
+};
+
+template <int W, int P>
+__global__ void __launch_bounds__(kMspThreads, 1) msp_block_kernel(MspArgs a) {
+  typedef typename MspBlockCfg<W, P>::CT CT;
+  constexpr int kDesc = MspBlockCfg<W, P>::kDesc;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int tid = threadIdx.x, lane = tid & 31;
   MspSmem<CT> sm;
   unsigned char* sp = smem_raw;
   sm.desc_m = reinterpret_cast<CT*>(sp);
-  sp += sizeof(CT) * kMaxDescBlock * kMspThreads;
+  sp += sizeof(CT) * kDesc * kMspThreads;
   sm.desc_e = reinterpret_cast<uint32_t*>(sp);
   sm.row = nullptr;
-  constexpr CT kMaskP = (CT)((2 * P == 32) ? ~0u : ((1u << (2 * P)) - 1));
+  constexpr CT kMaskP = (CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1));
   constexpr CT kInf = ~(CT)0;
   constexpr int kTopP = 2 * P - 2;
   constexpr int K = W + P - 1;
   const uint32_t de_a = sh_addr(sm.desc_e + tid), dm_a = sh_addr(sm.desc_m + tid);
-  constexpr uint32_t kDescStep = kMspThreads * 4;
+  constexpr uint32_t kDescStep = kMspThreads * 4, kDescStepM = kMspThreads * sizeof(CT);
   const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
   for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
     const uint64_t r = r0 + lane;
@@ -652,64 +676,13 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
     // i = q0 - W + t is complete once P-mer q0 + t - 1 is read: its minimizer is
     // min(suf[t], prefix minimum of the current block's first t values) -- the
     // prefix is a running scalar, the block's values are kept for its suffix minima.
-#if DBG_MSP_FUSED
-    for (int q0 = 0; q0 < nPmax + W; q0 += W) {
-      CT c[W];
-      CT pre = kInf;
-      refill(W);
-#pragma unroll
-      for (int t = 0; t < W; ++t) {
-        const int i = q0 - W + t;
-        if (q0 >= W && i < nk) {
-          const CT m = suf[t] < pre ? suf[t] : pre;
-          if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
-            sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(i - 1));
-            sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
-            ++ndesc;
-          }
-          m_cur = m;
-          if (i == nk - 1) {  // the read's last superkmer
-            sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
-            sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
-            ++ndesc;
-          }
-        }
-        CT v = kInf;
-        if (q0 + t < nP) {
-          const uint32_t b = next_base();
-          f = ((f << 2) | b) & kMaskP;
-          rc = (rc >> 2) | ((CT)(3u - b) << kTopP);
-          v = f < rc ? f : rc;  // canonical P-mer (reading D)
-        }
-        c[t] = v;
-        pre = v < pre ? v : pre;
-      }
-      suf[W - 1] = c[W - 1];
-#pragma unroll
-      for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
-      if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
-    }
-    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<CT>(a, sm, ndesc, s_next, o, L);
-#else
     for (int q0 = 0; q0 < nPmax + W; q0 += W) {
       CT c[W], pre[W];
-      refill(W);
-#if DBG_MSP_NOBR
-      // every lane shifts W bases out of its window (past its read's end they are padding and
-      // their P-mers are masked to +inf): no per-base branch
-      const int rem = nP - q0;
-#pragma unroll
-      for (int t = 0; t < W; ++t) {
-        const uint32_t b = (uint32_t)(wbuf >> 62);
-        wbuf <<= 2;
-        f = ((f << 2) | b) & kMaskP;
-        rc = (rc >> 2) | ((CT)(b ^ 3u) << kTopP);
-        const CT v = t < rem ? (f < rc ? f : rc) : kInf;  // canonical P-mer (reading D)
-        c[t] = v;
-#else
+      refill(W < 32 ? W : 32);  // a 64-bit window holds 32 bases: W > 32 reloads once more
 #pragma unroll
       for (int t = 0; t < W; ++t) {
         CT v = kInf;
+        if (t > 0 && t % 32 == 0) refill(W - t < 32 ? W - t : 32);
         if (q0 + t < nP) {
           const uint32_t b = next_base();
           f = ((f << 2) | b) & kMaskP;
@@ -717,13 +690,8 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
           v = f < rc ? f : rc;  // canonical P-mer (reading D)
         }
         c[t] = v;
-#endif
         pre[t] = t == 0 ? v : (v < pre[t - 1] ? v : pre[t - 1]);
       }
-#if DBG_MSP_NOBR
-      nbuf -= W;
-      j += W;
-#endif
       if (q0 >= W) {  // K-mers i = q0 - W + t of the previous block's windows
 #pragma unroll
         for (int t = 0; t < W; ++t) {
@@ -732,17 +700,15 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
             const CT m = t == 0 ? suf[0] : (suf[t] < pre[t - 1] ? suf[t] : pre[t - 1]);
             if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
               sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(i - 1));
-              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+              sh_st(dm_a + (uint32_t)ndesc * kDescStepM, m_cur);
               ++ndesc;
             }
             m_cur = m;
-#if !DBG_MSP_TAIL
             if (i == nk - 1) {  // the read's last superkmer
               sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)i);
-              sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
+              sh_st(dm_a + (uint32_t)ndesc * kDescStepM, m_cur);
               ++ndesc;
             }
-#endif
           }
         }
       }
@@ -751,17 +717,9 @@ __global__ void __launch_bounds__(kMspThreads, kMspBlockCtas) msp_block_kernel(M
       for (int t = W - 2; t >= 0; --t) suf[t] = c[t] < suf[t + 1] ? c[t] : suf[t + 1];
       // one flush site (the code is inlined once): lists nearly full, or the reads' end
       const bool last = q0 + W >= nPmax + W;
-#if DBG_MSP_TAIL
-      if (last && nk > 0) {  // the read's last superkmer, appended once after its last K-mer
-        sh_st(de_a + (uint32_t)ndesc * kDescStep, (uint32_t)(nk - 1));
-        sh_st(dm_a + (uint32_t)ndesc * kDescStep, m_cur);
-        ++ndesc;
-      }
-#endif
-      if (__any_sync(kFull, ndesc > kMaxDescBlock - W - 2 || (last && ndesc > 0)))
+      if (__any_sync(kFull, ndesc > kDesc - W - 2 || (last && ndesc > 0)))
         flush_descriptors<CT, K>(a, sm, ndesc, s_next, o, L);
     }
-#endif
   }
 }
 
@@ -786,21 +744,18 @@ bool dbg_params_ok(const dbg_params* prm) {
 
 // Grid of the grid-stride MSP kernels: at most one wave of resident CTAs (a partial second
 // wave would start its reads only when first-wave CTAs finish theirs).
-#ifndef DBG_MSP_GRID
-#define DBG_MSP_GRID 0  // CTAs per SM (0: the occupancy limit)
-#endif
 static int msp_grid(const void* fn, int want, size_t smem) {
   int per_sm = 0;
-  if (DBG_MSP_GRID > 0 || cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kMspThreads, smem) != cudaSuccess ||
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kMspThreads, smem) != cudaSuccess ||
       per_sm < 1)
-    per_sm = DBG_MSP_GRID > 0 ? DBG_MSP_GRID : 8;
+    per_sm = 8;
   const int cap = dbg_sm_count() * per_sm;
   return want < cap ? want : cap;
 }
 
 template <int W, int P>
 static cudaError_t launch_msp_block(const MspArgs& a, int grid, cudaStream_t stream) {
-  const size_t smem = (sizeof(uint32_t) + sizeof(uint32_t)) * kMaxDescBlock * kMspThreads;
+  const size_t smem = MspBlockCfg<W, P>::smem();
   cudaError_t e = cudaFuncSetAttribute(msp_block_kernel<W, P>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   grid = msp_grid((const void*)msp_block_kernel<W, P>, grid, smem);
@@ -808,9 +763,11 @@ static cudaError_t launch_msp_block(const MspArgs& a, int grid, cudaStream_t str
   return cudaGetLastError();
 }
 
-// The register-blocked kernel for the configurations' K = 31 (P = 11..15), else the generic one.
+// The register-blocked kernel for the configurations' K = 31 (P = 11..15), else the generic one
+// (for K = 63, P = 19 the 64-bit blocks of W = 45 need 255 registers and spill: measured 1.5x
+// slower than the generic kernel, profiles/r02e).
 static bool msp_block_launch(const MspArgs& a, int grid, cudaStream_t stream, cudaError_t* e) {
-  if (getenv("DBG_MSP_GENERIC") || a.k != 31) return false;
+  if (a.k != 31) return false;
   switch (a.p) {
     case 11: *e = launch_msp_block<21, 11>(a, grid, stream); return true;
     case 12: *e = launch_msp_block<20, 12>(a, grid, stream); return true;
@@ -821,13 +778,17 @@ static bool msp_block_launch(const MspArgs& a, int grid, cudaStream_t stream, cu
   return false;
 }
 
-template <typename CT>
+#ifndef DBG_MSP_ROW40
+#define DBG_MSP_ROW40 1
+#endif
+template <typename CT, bool kRow40>
 static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
-  const size_t smem = (sizeof(CT) + sizeof(uint32_t)) * msp_max_desc<CT>() * kMspThreads + sizeof(CT) * a.w * kMspThreads;
-  cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const size_t smem = 2 * sizeof(uint32_t) * kMspDesc * kMspThreads + RowIO<CT, kRow40>::bytes(a.w);
+  cudaError_t e =
+      cudaFuncSetAttribute(msp_kernel<CT, kRow40>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  grid = msp_grid((const void*)msp_kernel<CT>, grid, smem);
-  msp_kernel<CT><<<grid, kMspThreads, smem, stream>>>(a);
+  grid = msp_grid((const void*)msp_kernel<CT, kRow40>, grid, smem);
+  msp_kernel<CT, kRow40><<<grid, kMspThreads, smem, stream>>>(a);
   return cudaGetLastError();
 }
 
@@ -881,7 +842,6 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     a.staging = part->d_staging;
     a.staging_cap = part->staging_cap;
     a.staged = reinterpret_cast<unsigned long long*>(part->d_staged);
-    a.rank = part->d_staging && part->staging_cap ? part->d_rank : nullptr;
     a.pid_lo = (uint32_t)pid_lo;
     a.pid_hi = (uint32_t)pid_hi;
     a.ranged = pid_lo > 0 || pid_hi < np;
@@ -895,7 +855,9 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       const int grid = (int)(want < cap ? want : cap);
       cudaError_t e = cudaSuccess;
       if (!msp_block_launch(a, grid, stream, &e))
-        e = a.p <= 16 ? launch_msp<uint32_t>(a, grid, stream) : launch_msp<uint64_t>(a, grid, stream);
+        e = a.p <= 16 ? launch_msp<uint32_t, false>(a, grid, stream)
+                      : (DBG_MSP_ROW40 && a.p <= 20 ? launch_msp<uint64_t, true>(a, grid, stream)
+                                                    : launch_msp<uint64_t, false>(a, grid, stream));
       if (e != cudaSuccess) return DBG_ECUDA;
     }
     // d_fill is idle until pass 2 (which zeroes it): scratch for the tile sums
@@ -908,46 +870,25 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     if (part->d_scratch && (part->d_scratch == part->d_staging || part->d_scratch == part->d_records))
       return DBG_EINVAL;
     if (part->n_peers < 0 ||
-        (part->n_peers > 0 && (!part->d_peer_records || !part->d_peer_bounds || part->d_rank || part->d_scratch)))
+        (part->n_peers > 0 && (!part->d_peer_records || !part->d_peer_bounds)))
       return DBG_EINVAL;
-    if (part->d_rank) {  // ranks from pass 1: one pass, no atomics
-      const unsigned long long* stg = reinterpret_cast<const unsigned long long*>(part->d_staged);
-      const int grid = dbg_sm_count() * 8;
-#define DBG_SCATTER_RANK(RW)                                                                                   \
-  scatter_rank_kernel<RW><<<grid, 256, 0, stream>>>(part->d_staging, part->d_rank, stg, part->staging_cap,      \
-                                                   part->d_record_offset, part->d_records);
-      if (R == 4) {
-        DBG_SCATTER_RANK(4)
-      } else if (R == 8) {
-        DBG_SCATTER_RANK(8)
-      } else {
-        DBG_SCATTER_RANK(16)
-      }
-#undef DBG_SCATTER_RANK
-      return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
-    }
+    // Above kSmemHistMaxNp fine partitions a one-level scatter writes every 16-byte record to a
+    // random place of a multi-GB output: each store is a DRAM read-modify-write of its sector
+    // (chr14: 14 ms for 295 M records, ~1.85 TB/s of random sector traffic; tools/scatter_probe.py).
+    // With d_scratch the records go in two levels instead: level 1 into buckets of
+    // 2^kBucketShift consecutive partitions (bucket cursors advance sequentially; the buckets'
+    // open sectors fit L2), level 2 per bucket inside its small output range.
     const bool two = part->d_scratch && np > kSmemHistMaxNp;
-    int shift = 0;
-    // level 1 into at most 512 bins, so that a tile of 2048 records ranks several records per
-    // bin in shared memory and reserves once per bin
-    while (two && ((np + (1 << shift) - 1) >> shift) > kTwoLevelBins) ++shift;
+    const int shift = two ? kBucketShift : 0;
     const int nb = (np + (1 << shift) - 1) >> shift;
-    const bool abs_pos = DBG_SCATTER_ABS && nb > kSmemHistMaxNp && shift == 0;
-    if (abs_pos) {  // cursors = the partitions' record offsets
-      if (cudaMemcpyAsync(part->d_fill, part->d_record_offset, sizeof(uint64_t) * nb, cudaMemcpyDeviceToDevice,
-                          stream) != cudaSuccess)
-        return DBG_ECUDA;
-    } else if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) {
-      return DBG_ECUDA;
-    }
+    if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) return DBG_ECUDA;
     const size_t smem = nb <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * nb : 0;
     // one full wave: the kernel is grid-stride, a partial second wave would idle SMs
     auto scatter_grid = [&](const void* fn) {
       int per_sm = 0;
-      if (DBG_SCATTER_GRID > 0 ||
-          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kScatterThreads, smem) != cudaSuccess ||
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kScatterThreads, smem) != cudaSuccess ||
           per_sm < 1)
-        per_sm = DBG_SCATTER_GRID > 0 ? DBG_SCATTER_GRID : 4;
+        per_sm = 4;
       return dbg_sm_count() * per_sm;
     };
     uint32_t* lvl1 = two ? part->d_scratch : part->d_records;
@@ -957,16 +898,14 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     const int grid2 = (int)std::min<int64_t>((int64_t)nb, (int64_t)dbg_sm_count() * 4);
 #define DBG_SCATTER(RW)                                                                                         \
   cudaFuncSetAttribute(scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
-  scatter_kernel<RW><<<scatter_grid((const void*)scatter_kernel<RW>), kScatterThreads, smem, stream>>>(part->d_staging, staged, part->staging_cap,       \
-                                                              part->d_record_offset, fill, lvl1, nb, shift,     \
-                                                              abs_pos, part->d_peer_records,                    \
-                                                              part->d_peer_bounds, part->n_peers);              \
+  scatter_kernel<RW><<<scatter_grid((const void*)scatter_kernel<RW>), kScatterThreads, smem, stream>>>(        \
+      part->d_staging, staged, part->staging_cap, part->d_record_offset, fill, lvl1, nb, shift,                 \
+      two ? nullptr : part->d_peer_records, part->d_peer_bounds, two ? 0 : part->n_peers);                      \
   if (two) {                                                                                                    \
     cudaFuncSetAttribute(bucket_scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);   \
-    bucket_scatter_kernel<RW><<<grid2, kBucketThreads, smem2, stream>>>(part->d_scratch, staged,               \
-                                                                        part->staging_cap,                     \
-                                                                        part->d_record_offset,                 \
-                                                                        part->d_records, np, shift);           \
+    bucket_scatter_kernel<RW><<<grid2, kBucketThreads, smem2, stream>>>(                                       \
+        part->d_scratch, staged, part->staging_cap, part->d_record_offset, part->d_records, np, shift,         \
+        part->d_peer_records, part->d_peer_bounds, part->n_peers);                                             \
   }
     if (R == 4) {
       DBG_SCATTER(4)

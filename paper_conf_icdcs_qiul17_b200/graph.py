@@ -24,8 +24,6 @@ from __future__ import annotations
 
 from dataclasses import dataclass, field
 
-import os
-
 import numpy as np
 import torch
 
@@ -115,15 +113,13 @@ class DbgBuilder:
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
         self.records = torch.empty(0, dtype=torch.int32, device=dev)
-        # two-level scatter (pass 2) above 8192 fine partitions through a third record buffer:
-        # opt-in (DBG_SCATTER_TWO_LEVEL=1) -- measured slower than one level with global rank
-        # atomics on E. coli and chr14 (profiles/r01d_ab.txt)
+        # two-level scatter (pass 2) through a third record buffer (dbg_partition_set.d_scratch;
+        # msp.cu): it pays only where one level's random 16-byte record stores miss L2 -- 4-word
+        # records and a staging far larger than L2 (chr14: 14.1 -> 12.2 ms); E. coli (0.35 GB of
+        # records: 0.52 -> 1.25 ms) and 32-byte records (bumblebee: 20.1 -> 23.6 ms) lose (r02f)
         self.scratch = torch.empty(0, dtype=torch.int32, device=dev)
-        self.two_level = NP > 8192 and os.environ.get("DBG_SCATTER_TWO_LEVEL") == "1"
-        # pass-1 ranks (dbg_partition_set.d_rank): pass 2 without rank atomics
-        self.use_rank = os.environ.get("DBG_MSP_RANK", "0") == "1"
-        self.rank = torch.empty(0, dtype=torch.int32, device=dev)
-        self._rank_valid = False
+        self.two_level = NP > 8192
+        self.two_level_min_bytes = 2 << 30
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
         self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
         self.work = torch.empty(0, dtype=torch.uint8, device=dev)
@@ -174,17 +170,15 @@ class DbgBuilder:
     # ------------------------------------------------------------------ a2-a4
     def part_set(self, with_records: bool) -> _lib.dbg_partition_set:
         scratch = None
-        if with_records and self.two_level:
+        if with_records and self.use_two_level():
             self.scratch = _grow(self.scratch, self.records.numel(), torch.int32, self.device)
             scratch = self.scratch
-        rank = None
         cap = self.staging.numel() // self.rec_words
-        if self.use_rank and (not with_records or self._rank_valid):
-            self.rank = _grow(self.rank, cap, torch.int32, self.device)
-            rank = self.rank
-            self._rank_valid = True  # pass 1 writes them; invalidated by load_exchanged
         return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill, self.d_staged,
-                                  self.staging, cap, self.records if with_records else None, scratch, rank)
+                                  self.staging, cap, self.records if with_records else None, scratch)
+
+    def use_two_level(self) -> bool:
+        return self.two_level and self.rec_words == 4 and self.staging.numel() * 4 >= self.two_level_min_bytes
 
     def _staging_estimate(self, n_kmers_upper: int, n_reads: int) -> int:
         w = self.k - self.p + 1

@@ -207,8 +207,12 @@ class ShardedBuilder:
         with torch.cuda.stream(stream):
             self.d_ptrs.copy_(self._h_ptrs, non_blocking=True)
         # pass 2: every staged record into its owner's buffer (peer memory), partition order
+        scratch = None
+        if s.use_two_level():  # two-level scatter (msp.cu): level 1 locally, level 2 into the owners' buffers
+            s.scratch = _grow(s.scratch, s.staging.numel(), torch.int32, self.device)
+            scratch = s.scratch
         part = _lib.partition_set(s.d_n_records, s.d_n_kmers, self.d_dest, s.d_fill, s.d_staged, s.staging,
-                                  s.staging.numel() // R, d.records, None, None, self.d_ptrs, self.d_bounds,
+                                  s.staging.numel() // R, d.records, scratch, self.d_ptrs, self.d_bounds,
                                   self.world)
         ev = s._mark("msp_scatter", stream)
         _lib.dbg_msp_partition(s.prm, d_bases, d_bases.numel(), d_offsets, d_offsets.numel() - 1, part, stream)

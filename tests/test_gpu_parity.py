@@ -348,23 +348,19 @@ def test_register_blocked_msp_variants(p):
 
 
 @pytest.mark.parametrize("refine", [1024, 4096, 40000])
-def test_two_level_scatter_partition_order(refine, monkeypatch):
+def test_two_level_scatter_partition_order(refine):
     """More than 8192 fine partitions: pass 2 scatters through d_scratch in two levels (buckets of
-    2^s consecutive partitions, then within each bucket).  Every record must land in its own
+    16 consecutive partitions, then within each bucket).  Every record must land in its own
     partition's range [rec_off[p], rec_off[p+1]), the per-partition record multisets must equal the
     one-level scatter's, and the graph must equal the oracle's."""
     rs = ReadSet(*make_reads(genome(60_000, 5), 6000, 100, 0.01, 105))
     np_ = 16
-    monkeypatch.setenv("DBG_SCATTER_TWO_LEVEL", "1")
-    _check(rs, 31, 11, np_, refine=refine)
 
     def records(two):
-        if two:
-            monkeypatch.setenv("DBG_SCATTER_TWO_LEVEL", "1")
-        else:
-            monkeypatch.delenv("DBG_SCATTER_TWO_LEVEL", raising=False)
         b = DbgBuilder(31, 11, np_, refine=refine)
-        assert b.two_level == two
+        assert b.two_level
+        b.two_level = two
+        b.two_level_min_bytes = 0  # at every size here
         d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
         b.msp(d_bases, d_off)
         assert b.sync_sizes()
@@ -381,3 +377,9 @@ def test_two_level_scatter_partition_order(refine, monkeypatch):
     off1, rows1 = records(False)
     assert np.array_equal(off1, off2)
     assert rows1 == rows2
+    # and the graph through the two-level path
+    b = DbgBuilder(31, 11, np_, refine=refine)
+    b.two_level_min_bytes = 0
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    res = b.build(d_bases, d_off)
+    compare_vertices(res.vertices, oracle.graph(rs.seq, rs.offsets, 31, 11, np_, n_threads=NT))

@@ -128,6 +128,19 @@ def test_oracle_vs_string_brute_force(oracle_lib, k, p, np_, seed):
     assert got == want
 
 
+@pytest.mark.parametrize("k,p", [(5, 3), (31, 11), (31, 13), (63, 19), (21, 21), (9, 1)])
+def test_oracle_helpers_vs_string_brute_force(oracle_lib, k, p):
+    """oracle.kmer_minimizer (Def. 1, readings D, E) and oracle.canonical against the
+    string brute force: the lexicographically smallest of all P-substrings of the K-mer and of its
+    reverse complement, and the smaller of the K-mer and its reverse complement."""
+    rng = np.random.default_rng(k * 100 + p)
+    for _ in range(200):
+        x = "".join("ACGT"[c] for c in rng.integers(0, 4, k))
+        m = brute.minimizer_string(x, p)
+        assert oracle_lib.kmer_minimizer(x, p) == brute.code(m)
+        assert oracle_lib.canonical(x) == brute.code(brute.canonical_string(x))
+
+
 def test_oracle_threads_equal(oracle_lib):
     rs = random_reads(300, 20, 120, seed=13)
     a = oracle_lib.graph(rs.seq, rs.offsets, 11, 5, 7, n_threads=1)

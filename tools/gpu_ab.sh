@@ -1,20 +1,18 @@
-# same-box A/B of kernel variants (tools/build_variants.py) and runtime switches
-python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { cat gpurun_out/build.log; exit 1; }
-timeout 600 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "two_level or tiny or smem or low_count or overflow or auto_refine or full_size" > gpurun_out/ab_tests.log 2>&1; echo "tests rc=$?"; tail -2 gpurun_out/ab_tests.log
-run() {  # name, env...
-  local name=$1; shift
-  env "$@" timeout 300 python bench.py --steps 10 --warmup 3 --no-cpu-baseline 2>/dev/null | tail -1 > gpurun_out/ab_$name.json
-  python -c "
-import json; d=json.load(open('gpurun_out/ab_$name.json'))
-print('$name', round(d['ms_per_step'],3), 'ms', {k: round(v,3) for k,v in d['breakdown_ms'].items()}, d['invariants_ok'])"
-}
-V=paper_conf_icdcs_qiul17_b200/lib/variants
-for rep in 1 2; do
-run v0w DBG_LIB_PATH=$V/v0/libdbg.so DBG_GROUPS_WINDOW=1 DBG_SCATTER_ONE_LEVEL=1
-run v1w DBG_LIB_PATH=$V/v1/libdbg.so DBG_GROUPS_WINDOW=1 DBG_SCATTER_ONE_LEVEL=1
-run v2w DBG_LIB_PATH=$V/v2/libdbg.so DBG_GROUPS_WINDOW=1 DBG_SCATTER_ONE_LEVEL=1
-run v3w DBG_LIB_PATH=$V/v3/libdbg.so DBG_GROUPS_WINDOW=1 DBG_SCATTER_ONE_LEVEL=1
-run v1g DBG_LIB_PATH=$V/v1/libdbg.so DBG_SCATTER_ONE_LEVEL=1
-run v0g DBG_LIB_PATH=$V/v0/libdbg.so DBG_SCATTER_ONE_LEVEL=1
-run v1g2 DBG_LIB_PATH=$V/v1/libdbg.so
+#!/bin/bash
+# Same-box A/B of libdbg.so variants (tools/build_variants.py builds lib/variants/<name>/):
+#   tools/gpu_ab.sh TAG CONFIG "variant1 variant2 ..." [extra bench args]
+TAG=$1; CFG=$2; VARS=$3; shift 3
+mkdir -p gpurun_out
+for v in $VARS; do
+  DBG_LIB_PATH=paper_conf_icdcs_qiul17_b200/lib/variants/$v/libdbg.so timeout 900 python bench.py --config $CFG \
+    --no-cpu-baseline "$@" > gpurun_out/${TAG}_$v.json 2> gpurun_out/${TAG}_$v.err
+  python - "$v" gpurun_out/${TAG}_$v.json <<'PY'
+import json, sys
+try:
+    d = json.load(open(sys.argv[2]))
+    print(sys.argv[1], round(d["value"] / 1e9, 3), "G/s", round(d["ms_per_step"], 3), "ms",
+          {k: round(v, 3) for k, v in d["breakdown_ms"].items()}, "inv", d["invariants_ok"])
+except Exception as e:
+    print(sys.argv[1], "failed", e)
+PY
 done
