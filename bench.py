@@ -421,10 +421,13 @@ def run_ours(args):
     nb = len(b.batches)
     launches_per_step = 2 + scan + 9 + 2 * nb + (scan if nb else 0) + (scan + 1 if ws > 1 else 0)
     placement = _placement(b)
-    # Fig. 6 / Table II analogue (row f1): the paper's partitions (fine pid mod NP) -- skew and the
-    # table size lambda/(4 alpha) N^i_kmer x slot bytes of the largest one
-    paper_parts = np.bincount(np.arange(b.np) % rs.num_partitions, weights=b.part_kmers,
-                              minlength=rs.num_partitions)
+    # Fig. 6 / Table II analogue (row f1): the paper's partitions (the vertices' pid, reading V; K-mers
+    # = sum of their counts) -- skew and the table size lambda/(4 alpha) N^i_kmer x slot bytes of the
+    # largest one (this rank's vertices)
+    rec = b.out[:n_out * b.vdtype.itemsize].view(torch.int32).view(n_out, b.vdtype.itemsize // 4)
+    paper_parts = torch.bincount(rec[:, -1].long(), weights=rec[:, -10].double(),
+                                 minlength=rs.num_partitions).cpu().numpy()
+    del rec
     psizes = {"max_over_mean": float(paper_parts.max() / max(paper_parts.mean(), 1e-9)),
               "max_kmers": int(paper_parts.max()), "mean_kmers": float(paper_parts.mean()),
               "max_table_mb": _lib.dbg_table_bytes(b.prm, int(paper_parts.max())) / 1e6,

@@ -19,7 +19,7 @@
  *    (row f3: four-word keys, the paper's empty/locked/occupied protocol) runs
  *    only through the resident tables: dbg_msp_partition[_range],
  *    dbg_table_plan, dbg_hash_build, dbg_extract_graph (dbg_vertex_wide
- *    output); fine_p must be 0 or P; the on-chip, fused, sort and checksum
+ *    output); fine_p must be 0 or P; the on-chip, sort and checksum
  *    calls return DBG_EINVAL;
  *    1 <= num_partitions * refine <= 4,194,303.  Every per-partition array
  *    and pid range below is in FINE partitions (NP * refine of them); only
@@ -273,30 +273,6 @@ DBG_API dbg_status dbg_build_subgraphs_smem(const dbg_params* prm, const dbg_par
  * capacity 0, so resident tables cover only the rest. */
 DBG_API dbg_status dbg_table_plan_split(const dbg_params* prm, const uint64_t* d_n_kmers,
                                 uint64_t* d_table_offset, uint64_t* d_scratch, cudaStream_t stream);
-
-/* ---- a5-a7 fused: Step 2 through an L2-resident ring -----------------------
- * For partitions [pid_begin, pid_end): build each partition's table (one
- * insertion per distinct vertex, multiple updates, Sec. III-C)
- * and compact it into d_out -- all in one persistent kernel.  d_ring must be
- * all-zero when first used (extraction leaves it clean again).  Partitions are taken in groups of consecutive
- * partitions spanning about group_slots table slots (the caller picks it so
- * a few groups fit in L2: the B200 form of sizing tables for locality,
- * P:L665-675); each group's tables live in one of the ring regions of d_ring
- * (ring_bytes >= dbg_subgraph_ring_bytes(group_slots, max capacity); a
- * smaller ring sets status bit 2 -> DBG_ENOSPACE).  total_slots =
- * d_table_offset[pid_end] - d_table_offset[pid_begin] (host copy, sizes the
- * workspace: dbg_subgraph_workspace_bytes bytes of scheduling state).
- * Output appends to d_out[*d_n_out ...] and accumulates *d_stats as
- * dbg_extract_graph does. */
-DBG_API uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t group_slots, uint64_t max_capacity);
-DBG_API uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions, uint64_t total_slots,
-                                      uint64_t group_slots);
-DBG_API dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
-                               int32_t pid_end, const uint64_t* d_table_offset, uint64_t total_slots,
-                               uint64_t group_slots, void* d_ring, uint64_t ring_bytes, void* d_workspace,
-                               uint64_t workspace_bytes, dbg_vertex* d_out, uint64_t out_cap,
-                               uint64_t* d_n_out, dbg_stats* d_stats, uint32_t* d_status,
-                               cudaStream_t stream);
 
 /* ---- a6: Step 2 with resident tables (Sec. III-C) ------------
  * Inserts every K-mer occurrence of partitions [pid_begin, pid_end) into that

@@ -77,10 +77,6 @@ SIGNATURES = {
     "dbg_smem_workspace_bytes": (_U64, [_PRM]),
     "dbg_build_subgraphs_smem": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _P, _U64, _P, _P, _P, _P]),
     "dbg_table_plan_split": (ctypes.c_int, [_PRM, _P, _P, _P, _P]),
-    "dbg_subgraph_ring_bytes": (_U64, [_PRM, _U64, _U64]),
-    "dbg_subgraph_workspace_bytes": (_U64, [_PRM, _I32, _U64, _U64]),
-    "dbg_build_subgraphs": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _U64, _U64, _P, _U64, _P, _U64, _P, _U64,
-                                           _P, _P, _P, _P]),
     "dbg_hash_build": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _P, _P]),
     "dbg_hash_build_list": (ctypes.c_int, [_PRM, _PART, _I32, _I32, _P, _P, _I32, _P, _P, _P, _P]),
     "dbg_extract_graph": (ctypes.c_int, [_PRM, _P, _P, _I32, _I32, _P, _U64, _P, _P, _P, _P]),
@@ -248,23 +244,6 @@ def dbg_table_plan_split(prm, d_n_kmers, d_table_offset, d_scratch=None, stream=
     _check("dbg_table_plan_split", load().dbg_table_plan_split(ctypes.byref(prm), _ptr(d_n_kmers),
                                                                _ptr(d_table_offset), _ptr(d_scratch),
                                                                _stream(stream)))
-
-
-def dbg_subgraph_ring_bytes(prm, group_slots: int, max_capacity: int) -> int:
-    return load().dbg_subgraph_ring_bytes(ctypes.byref(prm), group_slots, max_capacity)
-
-
-def dbg_subgraph_workspace_bytes(prm, n_partitions: int, total_slots: int, group_slots: int) -> int:
-    return load().dbg_subgraph_workspace_bytes(ctypes.byref(prm), n_partitions, total_slots, group_slots)
-
-
-def dbg_build_subgraphs(prm, part, pid_begin: int, pid_end: int, d_table_offset, total_slots: int,
-                        group_slots: int, d_ring, ring_bytes: int, d_workspace, workspace_bytes: int, d_out,
-                        out_cap: int, d_n_out, d_stats, d_status, stream=None) -> None:
-    _check("dbg_build_subgraphs", load().dbg_build_subgraphs(
-        ctypes.byref(prm), ctypes.byref(part), pid_begin, pid_end, _ptr(d_table_offset), total_slots, group_slots,
-        _ptr(d_ring), ring_bytes, _ptr(d_workspace), workspace_bytes, _ptr(d_out), out_cap, _ptr(d_n_out),
-        _ptr(d_stats), _ptr(d_status), _stream(stream)))
 
 
 def dbg_hash_build(prm, part, pid_begin: int, pid_end: int, d_table, d_table_offset, d_status,

@@ -32,12 +32,11 @@
 // extraction: two reds per K-mer instead of the paper's three.
 //
 // Kernels:
-//  hash_build_kernel    resident tables of partitions [b, e) (dbg_hash_build)
+//  smem_subgraph_kernel the hot path: one persistent CTA per SM builds groups of fine partitions
+//                       in shared-memory tables and extracts them (dbg_build_subgraphs_smem)
+//  hash_build_kernel    resident tables of partitions [b, e) (dbg_hash_build): partitions too
+//                       large for one SM, and K > 63 (wide.cu)
 //  extract_kernel       compaction + clean of resident tables (dbg_extract_graph)
-//  subgraph_kernel      fused Step 2 (dbg_build_subgraphs): a persistent
-//                       kernel streams groups of partitions through a ring of
-//                       L2-sized table regions (hash a record chunk / extract
-//                       a slot chunk, claimed in a fixed global order)
 #include <cub/block/block_reduce.cuh>
 #include <cub/block/block_scan.cuh>
 #include <cub/device/device_radix_sort.cuh>
@@ -66,10 +65,8 @@ typedef unsigned __int128 u128;
 constexpr int kThreads = 256;
 constexpr uint64_t kCodeMask = (1ull << 62) - 1;
 constexpr uint64_t kSlotSeed = 0x9e3779b97f4a7c15ull;
-constexpr uint32_t kHashRecs = kThreads;  // records per hash item (32 per warp)
 constexpr int kXPer = 8;
 constexpr uint32_t kExtractSlots = kThreads * kXPer;
-constexpr uint32_t kStatusRing = 4u;
 constexpr int kJobs = 4;  // occurrences in flight per lane
 
 __host__ __device__ inline uint32_t key_bytes(int k) { return k <= 31 ? 16u : (k <= 63 ? 32u : 48u); }
@@ -582,199 +579,6 @@ __global__ void __launch_bounds__(kThreads, 4) extract_kernel(ResidentArgs a, Ou
     const uint64_t* off = a.tab_off;
     extract_tile<KW>(a.table + t0 * KE, ctr_base + t0 * 8, n,
                      [=](uint64_t s) { return (uint32_t)find_part(off, lo, hi, s0 + t0 + s); }, oa, sh);
-  }
-}
-
-// --------------------------------------------------------------- fused Step 2
-//
-// Partitions [b, e) are cut into groups of consecutive partitions: partition
-// p belongs to group floor((tab_off[p] - tab_off[b]) / group_slots), so a
-// group spans at most group_slots + max capacity slots.  Group g uses ring
-// region g % kRingGroups: key entries of the group's partitions back to back,
-// then their counter records.  The work list is a sequence of stages; stage s
-// holds H(s) (hash the records of group s) and X(s-1-kLagX) (extract group
-// s-1-kLagX), and CTAs claim items in list order.  Dependencies (per-group
-// completion counters): X(g) after H(g); H(g) after H(g-kRingGroups) and
-// X(g-kRingGroups) (ring reuse: the region is clean again; every group has
-// >= 1 hash item so the chain is transitive through empty groups).  Every
-// dependency of an item lies in an earlier stage, so the schedule cannot
-// deadlock; the lag keeps CTAs from stalling on a group's last hash items.
-
-constexpr int kLagX = 1;
-constexpr int kRingGroups = kLagX + 3;
-
-struct SubgraphArgs {
-  const uint32_t* records;
-  const uint64_t* rec_off;
-  const uint64_t* tab_off;
-  int pid_begin, pid_end, k;
-  uint64_t group_slots, n_groups_max;
-  char* ring;
-  uint64_t region_slots, region_bytes;
-  uint32_t* gfirst;               // [n_groups_max + 1] first partition of each group
-  unsigned long long* stage_off;  // [n_groups_max + kLagX + 3]
-  unsigned long long* work;       // [0] claimed-item counter, [1] n_groups
-  uint32_t* done;                 // [2][n_groups_max]: hash, extract items done
-};
-
-__device__ __forceinline__ uint64_t div_up(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
-
-struct GroupGeom {
-  int p0, p1;            // partitions [p0, p1)
-  uint64_t slot0, span;  // first slot (tab_off coordinates), slots
-  uint64_t rec0, nrec;   // records
-};
-__device__ __forceinline__ GroupGeom ggeom(const SubgraphArgs& a, int g) {
-  GroupGeom G;
-  G.p0 = (int)a.gfirst[g];
-  G.p1 = (int)a.gfirst[g + 1];
-  G.slot0 = a.tab_off[G.p0];
-  G.span = a.tab_off[G.p1] - G.slot0;
-  G.rec0 = a.rec_off[G.p0];
-  G.nrec = a.rec_off[G.p1] - G.rec0;
-  return G;
-}
-__device__ __forceinline__ uint64_t nh_items(const GroupGeom& G) { return G.nrec ? div_up(G.nrec, kHashRecs) : 1; }
-__device__ __forceinline__ uint64_t nx_items(const GroupGeom& G) { return div_up(G.span, kExtractSlots); }
-
-// Single CTA: groups, stage offsets of the work list, zeroed completion counters.
-__global__ void __launch_bounds__(kThreads) subgraph_plan_kernel(SubgraphArgs a, uint32_t* status) {
-  typedef cub::BlockScan<unsigned long long, kThreads> Scan;
-  __shared__ typename Scan::TempStorage tmp;
-  __shared__ unsigned long long carry;
-  const uint64_t base = a.tab_off[a.pid_begin];
-  const uint64_t total = a.tab_off[a.pid_end] - base;
-  uint64_t n_g = total ? div_up(total, a.group_slots) : 1;
-  if (n_g > a.n_groups_max) {
-    if (threadIdx.x == 0) atomicOr(status, kStatusRing);
-    n_g = a.n_groups_max;
-  }
-  // first partition of group g: lower bound of (tab_off[p] - base) / group_slots >= g
-  for (uint64_t g = threadIdx.x; g <= n_g; g += kThreads) {
-    int lo = a.pid_begin, hi = a.pid_end;
-    if (g == n_g) {
-      lo = a.pid_end;
-    } else {
-      while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if ((a.tab_off[mid] - base) / a.group_slots < g) lo = mid + 1;
-        else hi = mid;
-      }
-    }
-    a.gfirst[g] = (uint32_t)lo;
-  }
-  for (uint64_t i = threadIdx.x; i < 2 * n_g; i += kThreads) a.done[i] = 0;
-  if (threadIdx.x == 0) {
-    carry = 0;
-    a.work[0] = 0;
-    a.work[1] = n_g;
-  }
-  __syncthreads();
-  const int n_stage = (int)n_g + 1 + kLagX;
-  for (int s0 = 0; s0 < n_stage; s0 += kThreads) {
-    const int s = s0 + threadIdx.x;
-    unsigned long long items = 0;
-    if (s < n_stage) {
-      if (s < (int)n_g) {
-        const GroupGeom G = ggeom(a, s);
-        if (G.span > a.region_slots) atomicOr(status, kStatusRing);
-        items += nh_items(G);
-      }
-      if (s >= 1 + kLagX) items += nx_items(ggeom(a, s - 1 - kLagX));
-    }
-    unsigned long long excl, tot;
-    Scan(tmp).ExclusiveSum(items, excl, tot);
-    if (s < n_stage) a.stage_off[s] = carry + excl;
-    __syncthreads();
-    if (threadIdx.x == 0) carry += tot;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) a.stage_off[n_stage] = carry;
-}
-
-__device__ __forceinline__ void wait_count(const uint32_t* p, uint32_t need) {
-  if (need == 0) return;
-  while (ld_acquire32(p) < need) __nanosleep(64);
-}
-
-template <typename Code, int R>
-__global__ void __launch_bounds__(kThreads, 4) subgraph_kernel(SubgraphArgs a, OutArgs oa) {
-  constexpr int KW = sizeof(Code) == 8 ? 1 : 2;
-  constexpr uint32_t KE = KW == 1 ? 16 : 32;
-  __shared__ XShared sh;
-  __shared__ WarpRecs<R> shw[kThreads / 32];
-  __shared__ unsigned long long s_item;
-  const int n_g = (int)a.work[1];
-  const int n_stage = n_g + 1 + kLagX;
-  const unsigned long long total = a.stage_off[n_stage];
-  uint32_t* done_h = a.done;
-  uint32_t* done_x = a.done + n_g;
-  for (;;) {
-    if (threadIdx.x == 0) s_item = atomicAdd(a.work, 1ull);
-    __syncthreads();
-    const unsigned long long item = s_item;
-    __syncthreads();
-    if (item >= total) break;
-    int lo = 0, hi = n_stage;  // stage: last s with stage_off[s] <= item
-    while (hi - lo > 1) {
-      const int mid = (lo + hi) >> 1;
-      if (a.stage_off[mid] <= item) lo = mid;
-      else hi = mid;
-    }
-    const int s = lo;
-    uint64_t j = item - a.stage_off[s];
-    int kind = -1, g = -1;
-    GroupGeom G;
-    if (s < n_g) {
-      G = ggeom(a, s);
-      const uint64_t n = nh_items(G);
-      if (j < n) kind = 1, g = s;
-      else j -= n;
-    }
-    if (kind < 0) {
-      kind = 2;
-      g = s - 1 - kLagX;
-      G = ggeom(a, g);
-    }
-    char* keys = a.ring + (uint64_t)(g % kRingGroups) * a.region_bytes;
-    uint32_t* ctr = reinterpret_cast<uint32_t*>(keys + a.region_slots * KE);
-    if (threadIdx.x == 0) {
-      if (kind == 1 && g >= kRingGroups) {  // ring reuse: the previous user is extracted (and clean)
-        const GroupGeom Q = ggeom(a, g - kRingGroups);
-        wait_count(done_h + g - kRingGroups, (uint32_t)nh_items(Q));
-        wait_count(done_x + g - kRingGroups, (uint32_t)nx_items(Q));
-      }
-      if (kind == 2) wait_count(done_h + g, (uint32_t)nh_items(G));
-    }
-    __syncthreads();
-    if (kind == 1) {
-      const int warp = threadIdx.x >> 5;
-      const uint64_t r = j * kHashRecs + 32 * warp;
-      const int64_t n = r < G.nrec ? (int64_t)min((uint64_t)32, G.nrec - r) : 0;
-      if (n > 0) {
-        const uint64_t* off = a.tab_off;
-        const uint64_t gs0 = G.slot0;
-        auto table_of = [=](uint32_t pid, uint64_t& t0, uint64_t& cap) {
-          t0 = off[pid] - gs0;
-          cap = off[pid + 1] - off[pid];
-        };
-        if (!hash_warp<Code, R>(a.records + (G.rec0 + r) * R, n, a.k, keys, ctr, table_of, shw[warp]))
-          atomicOr(oa.status, kStatusTableFull);
-      }
-    } else {
-      const uint64_t s0 = j * kExtractSlots;
-      const uint64_t n = min((uint64_t)kExtractSlots, G.span - s0);
-      const uint64_t* off = a.tab_off;
-      const uint64_t gs0 = G.slot0;
-      const int p0 = G.p0, p1 = G.p1;
-      extract_tile<KW>(keys + s0 * KE, ctr + s0 * 8, n,
-                       [=](uint64_t sl) { return (uint32_t)find_part(off, p0, p1, gs0 + s0 + sl); }, oa, sh);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      atomicAdd(kind == 1 ? done_h + g : done_x + g, 1u);
-    }
   }
 }
 
@@ -1401,6 +1205,24 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             succ = (t < n - 1 || hr) ? (int)((uint32_t)(uint64_t)(Y >> (126 - 2 * K)) & 3u) : -1;
             rc = revcomp128(fwd, K);
           }
+        } else if constexpr (R == 8 && sizeof(Code) == 16 && KC > 48) {
+          // compile-time K in 49..63 (bumblebee's 63): the five record words holding bases
+          // b .. b + 79 are loaded once each and funnel-shifted; pred and succ come from them
+          // (pred needs the previous word only when b starts a word)
+          const int q = 1 + (b >> 4), sh = 2 * (b & 15);
+          uint32_t x[5];
+#pragma unroll
+          for (int v = 0; v < 5; ++v) x[v] = q + v < R ? w[(q + v) * S] : 0u;
+          const uint64_t A = ((uint64_t)x[0] << 32) | x[1], B = ((uint64_t)x[2] << 32) | x[3];
+          const uint64_t hi = (A << sh) | ((uint64_t)x[2] >> (32 - sh));
+          const uint64_t lo = (B << sh) | ((uint64_t)x[4] >> (32 - sh));
+          fwd = (Code)((((u128)hi << 64) | (u128)lo) >> (128 - 2 * KC));
+          rc = revcomp128(fwd, KC);
+          const uint32_t pw = (b & 15) ? x[0] : w[(q - 1) * S];
+          pred = b > 0 ? (int)((pw >> (30 - 2 * ((b - 1) & 15))) & 3u) : -1;
+          const int rel = (b & 15) + KC;  // the successor, inside the five words
+          const uint32_t sw = (rel >> 4) == 3 ? x[3] : x[4];
+          succ = (t < n - 1 || hr) ? (int)((sw >> (30 - 2 * (rel & 15))) & 3u) : -1;
         } else {
           kmer_at(w, b, K, R, fwd, rc, S);
           pred = b > 0 ? (int)rec_base(w, b - 1, S) : -1;
@@ -1873,67 +1695,6 @@ extern "C" dbg_status dbg_checksum_vertices(const dbg_params* prm, const dbg_ver
   const uint64_t want = (n + 255) / 256, cap = (uint64_t)dbg_sm_count() * 8;
   checksum_kernel<<<(int)(want < cap ? want : cap), 256, 0, stream>>>(
       d_vertices, n, reinterpret_cast<unsigned long long*>(d_stats) + 3);
-  return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
-}
-
-static uint64_t n_groups_max(uint64_t total_slots, uint64_t group_slots) {
-  return (group_slots ? total_slots / group_slots : 0) + 2;
-}
-
-extern "C" uint64_t dbg_subgraph_workspace_bytes(const dbg_params* prm, int32_t n_partitions, uint64_t total_slots,
-                                                 uint64_t group_slots) {
-  (void)prm;
-  (void)n_partitions;
-  const uint64_t g = n_groups_max(total_slots, group_slots);
-  return 4 * (g + 1) + 8 * (g + kLagX + 3) + 16 + 4 * 3 * g + 64;
-}
-
-extern "C" uint64_t dbg_subgraph_ring_bytes(const dbg_params* prm, uint64_t group_slots, uint64_t max_capacity) {
-  if (!prm) return 0;
-  const uint64_t region = (group_slots + max_capacity + 63) & ~(uint64_t)63;
-  return (uint64_t)kRingGroups * region * (key_bytes(prm->k) + kCtrBytes);
-}
-
-extern "C" dbg_status dbg_build_subgraphs(const dbg_params* prm, const dbg_partition_set* part, int32_t pid_begin,
-                                          int32_t pid_end, const uint64_t* d_table_offset, uint64_t total_slots,
-                                          uint64_t group_slots, void* d_ring, uint64_t ring_bytes,
-                                          void* d_workspace, uint64_t workspace_bytes, dbg_vertex* d_out,
-                                          uint64_t out_cap, uint64_t* d_n_out, dbg_stats* d_stats,
-                                          uint32_t* d_status, cudaStream_t stream) {
-  if (!dbg_params_ok(prm) || !part || !part->d_records || !part->d_record_offset || !d_table_offset ||
-      !d_ring || !d_workspace || !d_n_out || !d_stats || !d_status || (out_cap && !d_out) || group_slots == 0)
-    return DBG_EINVAL;
-  if (prm->k > 63) return DBG_EINVAL;  // row f3: resident tables only
-  if (pid_begin < 0 || pid_end > fine_partitions(prm) || pid_begin > pid_end) return DBG_EINVAL;
-  if (pid_begin == pid_end) return DBG_OK;
-  if (workspace_bytes < dbg_subgraph_workspace_bytes(prm, pid_end - pid_begin, total_slots, group_slots))
-    return DBG_EINVAL;
-  const uint64_t slot = key_bytes(prm->k) + kCtrBytes;
-  SubgraphArgs a;
-  a.records = part->d_records;
-  a.rec_off = part->d_record_offset;
-  a.tab_off = d_table_offset;
-  a.pid_begin = pid_begin;
-  a.pid_end = pid_end;
-  a.k = prm->k;
-  a.group_slots = group_slots;
-  a.n_groups_max = n_groups_max(total_slots, group_slots);
-  a.ring = static_cast<char*>(d_ring);
-  a.region_slots = (ring_bytes / kRingGroups / slot) & ~(uint64_t)63;
-  a.region_bytes = a.region_slots * slot;
-  if (a.region_slots == 0) return DBG_EINVAL;
-  char* ws = static_cast<char*>(d_workspace);
-  const uint64_t g = a.n_groups_max;
-  a.stage_off = reinterpret_cast<unsigned long long*>(ws);
-  a.work = reinterpret_cast<unsigned long long*>(ws + 8 * (g + kLagX + 3));
-  a.done = reinterpret_cast<uint32_t*>(ws + 8 * (g + kLagX + 3) + 16);
-  a.gfirst = a.done + 3 * g;
-  const OutArgs oa = make_out_args(prm, d_out, out_cap, d_n_out, d_stats, d_status);
-  subgraph_plan_kernel<<<1, kThreads, 0, stream>>>(a, d_status);
-  const int grid = dbg_sm_count() * 4;
-  if (prm->k <= 31) subgraph_kernel<uint64_t, 4><<<grid, kThreads, 0, stream>>>(a, oa);
-  else if (prm->k <= 39) subgraph_kernel<u128, 4><<<grid, kThreads, 0, stream>>>(a, oa);
-  else subgraph_kernel<u128, 8><<<grid, kThreads, 0, stream>>>(a, oa);
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }
 

@@ -289,7 +289,9 @@ __device__ __forceinline__ uint32_t desc_pid(const MspArgs& a, uint64_t m) {
   return (!a.ranged || pid - a.pid_lo < a.pid_hi - a.pid_lo) ? pid : ~0u;
 }
 
-template <typename CT, bool kRow40>
+// KC, PC > 0: compile-time K and P (bumblebee: 63, 19), so the rolling masks and shifts and the
+// van Herk block length W = K - P + 1 are constants.
+template <typename CT, bool kRow40, int KC = 0, int PC = 0>
 __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int tid = threadIdx.x, lane = tid & 31;
@@ -303,9 +305,10 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
   sm.row = nullptr;
   CT* row0 = reinterpret_cast<CT*>(sp);
 
-  const int K = a.k, P = in_reg(a.p), w = in_reg(a.w);
-  const CT maskP = in_reg((CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1)));
-  const int topP = in_reg(2 * P - 2);
+  const int K = KC ? KC : a.k, P = PC ? PC : in_reg(a.p), w = KC ? KC - PC + 1 : in_reg(a.w);
+  const CT maskP = PC ? (CT)((2 * PC == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * PC)) - 1))
+                      : in_reg((CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1)));
+  const int topP = PC ? 2 * PC - 2 : in_reg(2 * P - 2);
   const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
   // shared-window addresses of this thread's column of the van Herk block and descriptors
   RowIO<CT, kRow40> row;
@@ -395,10 +398,10 @@ __global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
           ++u;
         }
       }
-      if (__any_sync(kFull, ndesc > kDesc - (kFB + 2))) flush_descriptors<uint32_t, 0, true>(a, sm, ndesc, s_next, o, L);
+      if (__any_sync(kFull, ndesc > kDesc - (kFB + 2))) flush_descriptors<uint32_t, KC, true>(a, sm, ndesc, s_next, o, L);
       }
     }
-    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<uint32_t, 0, true>(a, sm, ndesc, s_next, o, L);
+    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<uint32_t, KC, true>(a, sm, ndesc, s_next, o, L);
   }
 }
 
@@ -778,17 +781,14 @@ static bool msp_block_launch(const MspArgs& a, int grid, cudaStream_t stream, cu
   return false;
 }
 
-#ifndef DBG_MSP_ROW40
-#define DBG_MSP_ROW40 1
-#endif
-template <typename CT, bool kRow40>
+template <typename CT, bool kRow40, int KC = 0, int PC = 0>
 static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
   const size_t smem = 2 * sizeof(uint32_t) * kMspDesc * kMspThreads + RowIO<CT, kRow40>::bytes(a.w);
-  cudaError_t e =
-      cudaFuncSetAttribute(msp_kernel<CT, kRow40>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT, kRow40, KC, PC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem);
   if (e != cudaSuccess) return e;
-  grid = msp_grid((const void*)msp_kernel<CT, kRow40>, grid, smem);
-  msp_kernel<CT, kRow40><<<grid, kMspThreads, smem, stream>>>(a);
+  grid = msp_grid((const void*)msp_kernel<CT, kRow40, KC, PC>, grid, smem);
+  msp_kernel<CT, kRow40, KC, PC><<<grid, kMspThreads, smem, stream>>>(a);
   return cudaGetLastError();
 }
 
@@ -855,8 +855,9 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       const int grid = (int)(want < cap ? want : cap);
       cudaError_t e = cudaSuccess;
       if (!msp_block_launch(a, grid, stream, &e))
-        e = a.p <= 16 ? launch_msp<uint32_t, false>(a, grid, stream)
-                      : (DBG_MSP_ROW40 && a.p <= 20 ? launch_msp<uint64_t, true>(a, grid, stream)
+        e = (a.k == 63 && a.p == 19) ? launch_msp<uint64_t, true, 63, 19>(a, grid, stream)
+          : a.p <= 16 ? launch_msp<uint32_t, false>(a, grid, stream)
+                      : (a.p <= 20 ? launch_msp<uint64_t, true>(a, grid, stream)
                                                     : launch_msp<uint64_t, false>(a, grid, stream));
       if (e != cudaSuccess) return DBG_ECUDA;
     }

@@ -13,8 +13,7 @@ libdbg.so kernels:
                                  over several CTAs) in shared memory, then
                                  dbg_hash_build_list + dbg_extract_graph build the remaining
                                  (oversize) partitions in global tables, in batches;
-                                 mode "resident": dbg_hash_build + dbg_extract_graph for all;
-                                 mode "fused": dbg_build_subgraphs (L2 ring of tables)
+                                 mode "resident": dbg_hash_build + dbg_extract_graph for all
     a7     DbgBuilder.vertices   dbg_sort_vertices + D2H
 
 The paper builds "one partition at a time"; here the
@@ -71,7 +70,7 @@ class DbgBuilder:
 
     def __init__(self, k: int, p: int, num_partitions: int, lam: float = 2.0, alpha: float = 0.5,
                  device: str | torch.device = "cuda", table_budget_bytes: int | None = None,
-                 mode: str = "smem", group_slots: int = 1 << 19, refine: int = 1, smem_split: int = 0,
+                 mode: str = "smem", refine: int = 1, smem_split: int = 0,
                  fine_p: int = 0, min_count: int = 0):
         if k % 2 == 0 or not 1 <= k <= 127:
             raise ValueError("K must be odd and 1..127 (DESIGN.md reading C)")
@@ -79,15 +78,13 @@ class DbgBuilder:
             raise ValueError("K > 63 (row f3) runs through the resident tables: mode='resident'")
         if not 1 <= p <= min(k, 31):
             raise ValueError("P must be in 1..min(K, 31)")
-        if mode not in ("smem", "fused", "resident"):
+        if mode not in ("smem", "resident"):
             raise ValueError(mode)
         self.k, self.p, self.mode = k, p, mode
         self.vdtype = VERTEX_WIDE_DTYPE if k > 63 else VERTEX_DTYPE  # dbg_vertex_wide for K > 63
         self.np_out = num_partitions                 # the paper's NP (dbg_vertex.pid)
         self.refine = max(1, int(refine))
         self.np = num_partitions * self.refine       # fine partitions the device works on
-        self.group_slots = int(group_slots)  # fused mode: table slots per ring group (L2 sizing)
-        self.total_slots = 0
         self.owned = (0, self.np)  # fine partitions this builder hashes (multi-GPU: a shard)
         self.smem_split = int(smem_split)  # 0: library default (dbg_params.smem_split)
         self.fine_p = int(fine_p)          # 0: P (dbg_params.fine_p)
@@ -121,7 +118,6 @@ class DbgBuilder:
         self.two_level = NP > 8192
         self.two_level_min_bytes = 2 << 30
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
-        self.ring = torch.empty(0, dtype=torch.uint8, device=dev)
         self.work = torch.empty(0, dtype=torch.uint8, device=dev)
         self.out = torch.empty(0, dtype=torch.uint8, device=dev)
         self.table_budget_bytes = table_budget_bytes
@@ -324,14 +320,6 @@ class DbgBuilder:
             self.tab_host = np.zeros(self.np + 1, dtype=np.int64)
             self.tab_host[1:] = np.cumsum(self.caps)
             self._tab_key = self._caps_key
-        if self.mode == "fused":
-            self.batches = [(0, self.np)]
-            self.total_slots = int(self.tab_host[-1])
-            ring = _lib.dbg_subgraph_ring_bytes(self.prm, self.group_slots, int(self.caps.max(initial=1)))
-            self.ring = self._clean_buffer(self.ring, ring, stream)
-            wsb = _lib.dbg_subgraph_workspace_bytes(self.prm, self.np, self.total_slots, self.group_slots)
-            self.work = _grow(self.work, wsb, torch.uint8, self.device)
-            return self.batches
         budget = self.table_budget_bytes
         if budget is None:  # once per builder: cudaMemGetInfo costs milliseconds
             free, _ = torch.cuda.mem_get_info(self.device)
@@ -398,13 +386,6 @@ class DbgBuilder:
             if not self.sync_sizes():
                 return
             self._plan_tables(stream)
-        if self.mode == "fused":
-            ev = self._mark("step2", stream)
-            _lib.dbg_build_subgraphs(self.prm, self.part_set(True), 0, self.np, self.d_tab_off, self.total_slots,
-                                     self.group_slots, self.ring, self.ring.numel(), self.work, self.work.numel(),
-                                     self.out, self.out_cap(), self.d_n_out, self.d_stats, self.d_status, stream)
-            self._done(ev, stream)
-            return
         for (b, e) in self.batches:
             ev = self._mark("hash_build", stream)
             if self.mode == "smem":  # only the oversize partitions have records to hash here
@@ -562,7 +543,7 @@ def launch_builder(k: int, p: int, num_partitions: int, n_kmers: int, lam: float
 def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partitions: int,
                 lam: float = 2.0, alpha: float = 0.5, device="cuda", sort: bool = True,
                 table_budget_bytes: int | None = None, mode: str = "smem",
-                group_slots: int = 1 << 19, refine: int | str = "auto", smem_split: int = 0,
+                refine: int | str = "auto", smem_split: int = 0,
                 fine_p: int | str = "auto", min_count: int = 0) -> GraphResult:
     """ASCII reads -> De Bruijn graph records (the public one-call API)."""
     lens = np.diff(np.asarray(offsets, dtype=np.int64))
@@ -573,7 +554,7 @@ def build_graph(seq: np.ndarray, offsets: np.ndarray, k: int, p: int, num_partit
         refine = auto_refine(n_kmers, k, p, num_partitions, lam, alpha) if mode == "smem" else 1
     if fine_p == "auto":
         fine_p = auto_fine_p(n_kmers, k, p, lam, alpha) if mode == "smem" else 0
-    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, group_slots, refine,
+    builder = DbgBuilder(k, p, num_partitions, lam, alpha, device, table_budget_bytes, mode, refine,
                          smem_split, fine_p, min_count)
     packed = encode_reads(seq)
     d_bases, d_offsets = builder.upload(packed, offsets)

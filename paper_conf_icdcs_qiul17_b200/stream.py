@@ -145,7 +145,11 @@ class StreamingBuilder:
         b._sizes_ev.record(self.compute)
         b._sizes_pending = True
 
-    def run(self, batches, sort: bool = True, out_frac: float = 0.5) -> StreamResult:
+    def run(self, batches, sort: bool = True, out_frac: float = 0.5, sink=None) -> StreamResult:
+        """sink: None -- every range's vertices go D2H and are returned; else sink(d_records, n) is
+        called per range with the range's records on the device (a uint8 view of n dbg_vertex), for
+        graphs larger than host memory (the sink copies out what it needs); the result then holds
+        no vertices, and stats["checksum"] is the order-independent checksum over all ranges."""
         b = self.b
         # sizing pass: per-partition record counts over every batch (nothing staged)
         self._pass1(batches, 0, b.np, count_only=True)
@@ -186,6 +190,14 @@ class StreamingBuilder:
             n_out = int(b.d_n_out.item())
             for k, v in zip(("distinct", "sum_count", "sum_edges"), b.d_stats[:3].cpu().numpy().view(np.uint64)):
                 stats[k] += int(v)
+            if sink is not None:
+                with torch.cuda.stream(self.compute):
+                    b.d_stats[3].zero_()
+                _lib.dbg_checksum_vertices(b.prm, b.out, n_out, b.d_stats, self.compute)
+                stats["checksum"] = (stats.get("checksum", 0) + int(b.d_stats[3:].cpu().numpy().view(np.uint64)[0])) \
+                    % (1 << 64)
+                sink(b.out[:n_out * VERTEX_DTYPE.itemsize], n_out)
+                continue
             if pending is not None:
                 pending[1].synchronize()
                 parts.append(pending[0][:pending[2]].copy())

@@ -43,7 +43,6 @@ def test_abi_and_sizes(lib):
     assert lib.dbg_record_words(p63) == 8 and lib.dbg_record_max_kmers(p63) == 48
     assert lib.dbg_slot_bytes(p31) == 48 and lib.dbg_key_bytes(p31) == 16
     assert lib.dbg_slot_bytes(p63) == 64 and lib.dbg_key_bytes(p63) == 32
-    assert lib.dbg_subgraph_ring_bytes(p31, 1000, 24) == 4 * 1024 * 48
     assert lib.dbg_packed_words(0) == 1 and lib.dbg_packed_words(32) == 2 and lib.dbg_packed_words(33) == 3
 
 

@@ -118,7 +118,7 @@ def test_msp_records_vs_oracle_superkmers():
         assert occurrences_from_records(recs, k) == occurrences_from_oracle_msp(sk, rs.reads(), k)
 
 
-@pytest.mark.parametrize("mode", ["smem", "fused", "resident"])
+@pytest.mark.parametrize("mode", ["smem", "resident"])
 def test_table_overflow_detected_and_rebuilt(mode):
     """Reading O: an undersized table (lambda/(4 alpha) << distinct/N) overflows; the status word
     reports DBG_ETABLEFULL and the builder rebuilds at capacity N^i_kmer with the same result."""
@@ -149,13 +149,6 @@ def test_resident_batches_give_same_graph():
 def test_resident_mode_parity(k, p, np_):
     rs = random_reads(300, 1, 2 * k + 100, seed=k + np_, n_rate=0.01)
     _check(rs, k, p, np_, mode="resident")
-
-
-def test_ring_with_many_small_partitions():
-    """More partitions than ring regions, many empty: the fused kernel's region reuse chain."""
-    rs = random_reads(500, 40, 160, seed=77)
-    _check(rs, 31, 11, 1000, mode="fused")
-    _check(rs, 15, 7, 37, mode="fused")
 
 
 @pytest.mark.parametrize("k,p,np_,refine", [(31, 11, 1, 1), (31, 11, 3, 1), (63, 19, 2, 1), (31, 11, 4, 8),
@@ -283,7 +276,7 @@ def test_staging_overflow_repeats_the_step():
 
 
 @pytest.mark.parametrize("mode,k,p,np_,refine,split", [("smem", 31, 11, 4, 8, 0), ("smem", 31, 11, 2, 1, 1),
-                                                       ("smem", 63, 19, 3, 2, 0), ("fused", 31, 11, 16, 1, 0),
+                                                       ("smem", 63, 19, 3, 2, 0),
                                                        ("resident", 63, 19, 8, 1, 0)])
 @pytest.mark.parametrize("min_count", [2, 3])
 def test_low_count_filter(mode, k, p, np_, refine, split, min_count):

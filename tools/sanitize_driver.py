@@ -6,9 +6,9 @@ synccheck / initcheck), each checked against the oracle:
 
   * on-chip Step 2 (smem_subgraph_kernel), K = 31 and K = 63, with split and global-tier
     partitions (small refine so some partitions exceed a CTA table);
-  * resident tables (hash_build_kernel / extract_kernel) and the fused L2-ring tier;
+  * resident tables (hash_build_kernel / extract_kernel);
   * K = 65 / 101 (wide.cu, the empty -> locked -> occupied protocol, with a hot key);
-  * the MSP kernels: register-blocked K = 31 (P = 11, 13) and K = 63 (P = 19), generic otherwise;
+  * the MSP kernels: register-blocked K = 31 (P = 11, 13), generic otherwise (K = 63: 40-bit row);
   * the two-level scatter (more than 8192 fine partitions).
 """
 import os
@@ -20,12 +20,18 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 import oracle  # noqa: E402
-from paper_conf_icdcs_qiul17_b200 import build_graph  # noqa: E402
+from paper_conf_icdcs_qiul17_b200 import DbgBuilder, build_graph, encode_reads  # noqa: E402
 from synth import ReadSet, genome, make_reads, random_reads  # noqa: E402
 
 
-def _check(tag, rs, k, p, np_, **kw):
-    res = build_graph(rs.seq, rs.offsets, k, p, np_, **kw)
+def _check(tag, rs, k, p, np_, two_level_min_bytes=None, **kw):
+    if two_level_min_bytes is None:
+        res = build_graph(rs.seq, rs.offsets, k, p, np_, **kw)
+    else:  # the two-level scatter at a size where the builder would not pick it
+        b = DbgBuilder(k, p, np_, **kw)
+        b.two_level_min_bytes = two_level_min_bytes
+        d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+        res = b.build(d_bases, d_off)
     if k > 63:
         orc = oracle.graph_wide(rs.seq, rs.offsets, k, p, np_)
         ok = len(orc) == len(res.vertices) and np.array_equal(res.vertices["kmer"], orc["key"]) and \
@@ -49,11 +55,10 @@ def main():
     ok = True
     ok &= _check("smem K=31 P=11 (register MSP, split + global tier)", rs, 31, 11, 2, refine=1)
     ok &= _check("smem K=31 P=11 fine_p 13 (reading V)", rs, 31, 11, 8, refine=4, fine_p=13)
-    ok &= _check("smem K=63 P=19 (register MSP, 64-bit)", rs, 63, 19, 4, refine=2)
+    ok &= _check("smem K=63 P=19 (generic MSP, 40-bit row)", rs, 63, 19, 4, refine=2)
     ok &= _check("smem K=41 P=17 (generic MSP)", rs, 41, 17, 4, refine=2)
-    ok &= _check("smem two-level scatter (10000 fine partitions)", rs, 31, 11, 16, refine=625)
+    ok &= _check("smem two-level scatter (10000 fine partitions)", rs, 31, 11, 16, refine=625, two_level_min_bytes=0)
     ok &= _check("resident K=31", rs, 31, 11, 4, mode="resident")
-    ok &= _check("fused K=31", rs, 31, 11, 4, mode="fused")
     ok &= _check("wide K=65 (locked state)", rs, 65, 21, 3)
     ok &= _check("wide K=101 hot key", hot, 101, 19, 2)
     ok &= _check("ragged reads K=21", random_reads(300, 1, 200, seed=33, n_rate=0.01), 21, 9, 5)
