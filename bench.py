@@ -425,9 +425,12 @@ def run_ours(args):
     # = sum of their counts) -- skew and the table size lambda/(4 alpha) N^i_kmer x slot bytes of the
     # largest one (this rank's vertices)
     rec = b.out[:n_out * b.vdtype.itemsize].view(torch.int32).view(n_out, b.vdtype.itemsize // 4)
-    paper_parts = torch.bincount(rec[:, -1].long(), weights=rec[:, -10].double(),
-                                 minlength=rs.num_partitions).cpu().numpy()
-    del rec
+    paper_parts = np.zeros(rs.num_partitions, dtype=np.float64)
+    for c0 in range(0, n_out, 1 << 26):  # chunks: the conversions of 1.8 G rows would not fit
+        c = rec[c0:c0 + (1 << 26)]
+        paper_parts += torch.bincount(c[:, -1].long(), weights=c[:, -10].double(),
+                                      minlength=rs.num_partitions).cpu().numpy()
+    del rec, c
     psizes = {"max_over_mean": float(paper_parts.max() / max(paper_parts.mean(), 1e-9)),
               "max_kmers": int(paper_parts.max()), "mean_kmers": float(paper_parts.mean()),
               "max_table_mb": _lib.dbg_table_bytes(b.prm, int(paper_parts.max())) / 1e6,

@@ -40,7 +40,10 @@ namespace dbg {
 
 constexpr int kMspThreads = 128;
 // msp_block_kernel variants (A/B builds, tools/build_variants.py)
-constexpr int kMaxDescBlock = 40;  // descriptors per thread between flushes (>= W + 3)
+#ifndef DBG_MSPB_DESC
+#define DBG_MSPB_DESC 40
+#endif
+constexpr int kMaxDescBlock = DBG_MSPB_DESC;  // descriptors per thread between flushes (>= W + 3)
 constexpr int kSmemHistMaxNp = 8192;
 constexpr int kBucketShift = 3;  // two-level scatter: buckets of 8 consecutive fine partitions (r02f: 3 < 4 < 5 < 6)
 
@@ -614,7 +617,10 @@ struct MspBlockCfg {
 };
 
 template <int W, int P>
-__global__ void __launch_bounds__(kMspThreads, 1) msp_block_kernel(MspArgs a) {
+#ifndef DBG_MSPB_MINB
+#define DBG_MSPB_MINB 1
+#endif
+__global__ void __launch_bounds__(kMspThreads, DBG_MSPB_MINB) msp_block_kernel(MspArgs a) {
   typedef typename MspBlockCfg<W, P>::CT CT;
   constexpr int kDesc = MspBlockCfg<W, P>::kDesc;
   extern __shared__ __align__(16) unsigned char smem_raw[];
