@@ -439,7 +439,8 @@ def run_ours(args):
         dist.barrier(device_ids=[local])
         dist.destroy_process_group()
         return 0
-    cfg_extra = {"refine": b.refine, "fine_partitions": b.np, "fine_p": b.fine_p or rs.p,
+    cfg_extra = {"refine": b.refine, "fine_partitions": b.np, "fine_p": b.fine_p or rs.p, "records": n_records,
+                 "vertices": n_out,
                  "smem_slots": _lib.dbg_smem_table_slots(b.prm), "kmer_placement": placement,
                  "kernel_version": KERNEL_VERSION, "partition_sizes": psizes}
     if ws > 1:

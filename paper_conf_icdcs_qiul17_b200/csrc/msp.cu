@@ -40,10 +40,9 @@ namespace dbg {
 
 constexpr int kMspThreads = 128;
 // msp_block_kernel variants (A/B builds, tools/build_variants.py)
-#ifndef DBG_MSPB_DESC
-#define DBG_MSPB_DESC 40
-#endif
-constexpr int kMaxDescBlock = DBG_MSPB_DESC;  // descriptors per thread between flushes (>= W + 3)
+// descriptors per thread between flushes of the register-blocked kernel (>= W + 3; a register cap
+// for 6-7 CTAs/SM with 28-32 descriptors was no faster on chr14, profiles/r02_ab.txt)
+constexpr int kMaxDescBlock = 40;
 constexpr int kSmemHistMaxNp = 8192;
 constexpr int kBucketShift = 3;  // two-level scatter: buckets of 8 consecutive fine partitions (r02f: 3 < 4 < 5 < 6)
 
@@ -617,10 +616,7 @@ struct MspBlockCfg {
 };
 
 template <int W, int P>
-#ifndef DBG_MSPB_MINB
-#define DBG_MSPB_MINB 1
-#endif
-__global__ void __launch_bounds__(kMspThreads, DBG_MSPB_MINB) msp_block_kernel(MspArgs a) {
+__global__ void __launch_bounds__(kMspThreads, 1) msp_block_kernel(MspArgs a) {
   typedef typename MspBlockCfg<W, P>::CT CT;
   constexpr int kDesc = MspBlockCfg<W, P>::kDesc;
   extern __shared__ __align__(16) unsigned char smem_raw[];
