@@ -46,7 +46,7 @@ UNIT = "kmers/s"
 ALG_BYTES_PER_KMER = 68
 # version tag of the on-chip kernel: profiles/traffic.json (ncu --set full) is quoted only when it
 # was captured on this version and workload
-KERNEL_VERSION = "smem-v12"
+KERNEL_VERSION = "smem-v13"
 
 
 def _peaks():
