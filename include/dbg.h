@@ -233,6 +233,11 @@ DBG_API dbg_status dbg_exchange_plan(const dbg_params* prm, const uint64_t* d_co
                                      uint64_t* d_owned_n_kmers, uint64_t* d_owned_record_offset,
                                      uint64_t* d_prefix, uint64_t* d_scratch, cudaStream_t stream);
 
+/* Peer access from the current device to peer_device (cudaDeviceEnablePeerAccess; already enabled
+ * is not an error), needed before pass 2 writes into d_peer_records that live on other GPUs.
+ * DBG_EINVAL if the devices cannot access each other. */
+DBG_API dbg_status dbg_enable_peer_access(int32_t peer_device);
+
 /* ---- a5: sizing (Property 1; Sec. IV-A) ----------------------
  * d_table_offset[NP+1] = exclusive prefix sum of dbg_table_capacity(N^i_kmer)
  * (in slots).  d_scratch: NP uint64 of caller memory for the multi-CTA scan

@@ -67,6 +67,7 @@ SIGNATURES = {
     "dbg_table_capacity": (_U64, [_PRM, _U64]),
     "dbg_table_bytes": (_U64, [_PRM, _U64]),
     "dbg_exchange_plan": (ctypes.c_int, [_PRM, _P, _P, _I32, _I32, _P, _P, _P, _P, _P, _P, _P, _P]),
+    "dbg_enable_peer_access": (ctypes.c_int, [_I32]),
     "dbg_packed_words": (_U64, [_U64]),
     "dbg_encode_ascii": (ctypes.c_int, [_P, _U64, _P]),
     "dbg_msp_partition": (ctypes.c_int, [_PRM, _P, _U64, _P, _U64, _PART, _P]),
@@ -189,6 +190,10 @@ def dbg_exchange_plan(prm, d_counts, d_kmers_sum, world: int, rank: int, d_bound
         ctypes.byref(prm), _ptr(d_counts), _ptr(d_kmers_sum), world, rank, _ptr(d_bounds), _ptr(d_dest_offset),
         _ptr(d_owned_n_records), _ptr(d_owned_n_kmers), _ptr(d_owned_record_offset), _ptr(d_prefix),
         _ptr(d_scratch), _stream(stream)))
+
+
+def dbg_enable_peer_access(peer_device: int) -> None:
+    _check("dbg_enable_peer_access", load().dbg_enable_peer_access(peer_device))
 
 
 def dbg_packed_words(n_bases: int) -> int:

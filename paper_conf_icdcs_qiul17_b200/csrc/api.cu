@@ -132,3 +132,21 @@ extern "C" const char* dbg_status_string(dbg_status s) {
   }
   return "unknown status";
 }
+
+// Multi-GPU emission (dbg_partition_set.d_peer_records): kernels of the current device write into
+// the record buffers of the other GPUs through their IPC-mapped pointers, which needs peer access
+// from this device to theirs (NVLink / NVSwitch).  Idempotent.
+extern "C" dbg_status dbg_enable_peer_access(int32_t peer_device) {
+  int cur = 0;
+  if (cudaGetDevice(&cur) != cudaSuccess) return DBG_ECUDA;
+  if (peer_device == cur) return DBG_OK;
+  int can = 0;
+  if (cudaDeviceCanAccessPeer(&can, cur, peer_device) != cudaSuccess) return DBG_ECUDA;
+  if (!can) return DBG_EINVAL;
+  const cudaError_t e = cudaDeviceEnablePeerAccess(peer_device, 0);
+  if (e == cudaErrorPeerAccessAlreadyEnabled) {
+    (void)cudaGetLastError();  // clear the (non-sticky) error
+    return DBG_OK;
+  }
+  return e == cudaSuccess ? DBG_OK : DBG_ECUDA;
+}

@@ -67,7 +67,12 @@ def _ipc_export(t: torch.Tensor):
 
 
 def _ipc_open(handle, nbytes: int, dtype=torch.int32):
-    """Maps a peer's exported storage into this process; returns (keep-alive object, device pointer)."""
+    """Maps a peer's exported storage into this process; returns (keep-alive object, device pointer).
+    The buffer lives on the peer's GPU (handle[0]); this device's kernels write it over NVLink, so
+    peer access to that GPU is enabled first (a no-op for a buffer on this GPU)."""
+    dev = int(handle[0])
+    if torch.cuda.is_available() and dev != torch.cuda.current_device():
+        _lib.dbg_enable_peer_access(dev)
     st = torch.UntypedStorage._new_shared_cuda(*handle)
     return st, st.data_ptr()
 
