@@ -170,10 +170,14 @@ def _oracle_rate(rs, seconds: float, threads: int):
 
     oracle.build()
     n = min(rs.n_reads, 2000)
-    t = time.time()
-    sub = rs.subset(0, n)
-    oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
-    dt = max(time.time() - t, 1e-3)
+    for _ in range(2):  # calibrate on a sample that takes ~10 % of the budget (thread start-up amortised)
+        t = time.time()
+        sub = rs.subset(0, n)
+        oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
+        dt = max(time.time() - t, 1e-3)
+        if dt > 0.1 * seconds or n == rs.n_reads:
+            break
+        n = int(min(rs.n_reads, n * 0.1 * seconds / dt))
     n2 = int(min(rs.n_reads, max(n, n * seconds / dt)))
     sub = rs.subset(0, n2)
     t = time.time()
@@ -203,7 +207,7 @@ def run_reference(args):
     import oracle
 
     oracle.build()
-    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    per_step = max(1.0, min(20.0, 120.0 / max(1, args.steps + args.warmup)))
     _, sub, _ = _oracle_rate(rs, per_step, threads)
     for _ in range(args.warmup):
         oracle.graph(sub.seq, sub.offsets, rs.k, rs.p, rs.num_partitions, n_threads=threads)
