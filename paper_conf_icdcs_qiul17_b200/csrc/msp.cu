@@ -204,7 +204,14 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
         in = !a.ranged || (pid - a.pid_lo < a.pid_hi - a.pid_lo);
         dm = in ? (CT)pid : kSkip;
       }
-      if (in) my_records += record_pieces(e - s + 1, nmax);
+      if (in) {
+        // the per-partition sizes here, so that the record loop below has no atomics between
+        // its loads and stores (the loads of consecutive records overlap)
+        const uint32_t pid = (uint32_t)dm, pieces = record_pieces(e - s + 1, nmax);
+        my_records += pieces;
+        atomicAdd(a.n_records + pid, (unsigned long long)pieces);
+        atomicAdd(a.n_kmers + pid, (unsigned long long)(e - s + 1));
+      }
       s = e + 1;
     }
   }
@@ -230,9 +237,6 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
       continue;
     }
     const uint32_t pid = (uint32_t)dm;
-    const int n = e - s + 1;
-    atomicAdd(a.n_records + pid, (unsigned long long)record_pieces(n, nmax));
-    atomicAdd(a.n_kmers + pid, (unsigned long long)n);
     for (int ps = s; ps <= e; ps += nmax, ++slot) {
       if (slot < a.staging_cap) {
         if (r4)
