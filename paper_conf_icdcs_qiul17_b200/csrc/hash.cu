@@ -677,6 +677,11 @@ __device__ __forceinline__ uint64_t lds64(uint32_t a) {
   asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
   return v;
 }
+__device__ __forceinline__ ulonglong2 lds_u4x(uint32_t a) {
+  ulonglong2 v;
+  asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "r"(a) : "memory");
+  return v;
+}
 __device__ __forceinline__ uint32_t lds32(uint32_t a) {
   uint32_t v;
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
@@ -1239,7 +1244,6 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         // found or claimed its slot, then the counter updates, warp-converged
         const typename KO::T key = KO::make(code);
         uint32_t idx = __umulhi(smem_hash(code), cap);
-        uint32_t inserted = 0;
         const uint32_t kaddr = keys_s + t0 * KB;
         if constexpr (KW == 1) {
           // every lane runs every probe round (predicated, no divergent branch): a lane with
@@ -1251,7 +1255,6 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             uint64_t cur = lds64(ka);
             cas_shared64_if(pend && cur == 0, ka, key, cur);
             const bool hit = cur == 0 || cur == key;
-            inserted |= (uint32_t)(pend && cur == 0);
             const bool adv = pend && !hit;
             const uint32_t nx = idx + 1 == cap ? 0u : idx + 1;
             idx = adv ? nx : idx;
@@ -1264,23 +1267,26 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
             if (cur != key) idx = ~0u;  // this occurrence found no slot
           }
         } else {
-          uint32_t probes = 0, pend = want;
-          while (__any_sync(kFull, pend)) {
-            if (pend) {
-              const typename KO::T cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);  // 16-B CAS: read-or-claim
-              inserted = KO::empty(cur);
-              if (inserted | KO::same(cur, key)) {
-                pend = 0;
-              } else {
-                idx = idx + 1 == cap ? 0 : idx + 1;
-                if (++probes == cap) {  // wrapped: table full (reading O)
-                  pend = 0;
-                  ok = false;
-                  idx = ~0u;
-                }
-              }
-            }
+          // 16-byte keys: a plain 16-byte load first; the CAS (read-or-claim) only where the
+          // entry may be empty.  A claimed entry never changes and a torn read of one being
+          // published shows a zero word, so a load with both words nonzero is a whole key; a
+          // zero word (empty, torn, or a key whose low word is 0) goes to the CAS, which
+          // returns the entry atomically.
+          const uint32_t idx0 = idx;
+          bool pend = want;
+          for (;;) {
+            const uint32_t ka = kaddr + idx * KB;
+            typename KO::T cur = lds_u4x(ka);
+            if (pend && (cur.x == 0 || cur.y == 0)) cur = KO::cas(keys + (size_t)(t0 + idx) * KB, key);
+            const bool emp = KO::empty(cur), hit = emp || KO::same(cur, key);
+            const bool adv = pend && !hit;
+            const uint32_t nx = idx + 1 == cap ? 0u : idx + 1;
+            idx = adv ? nx : idx;
+            pend = adv && nx != idx0;
+            if (adv && nx == idx0) ok = false;  // wrapped: table full (reading O)
+            if (!__any_sync(kFull, pend)) break;
           }
+          if (!ok && want && !KO::same(lds_u4x(kaddr + idx * KB), key)) idx = ~0u;  // found no slot
         }
         if (want && idx != ~0u) {  // the multiple updates: 16-bit fields, two per word
           const int fo = o < 4 ? o : 8;

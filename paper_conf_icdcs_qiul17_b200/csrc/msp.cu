@@ -1,27 +1,23 @@
 // msp.cu -- Step 1 of ParaHash on sm_100a: MSP graph partitioning
 // (Sec. III-B; Defs. 1-2), kernel (a) of the north star.
 //
-// Pass 1, msp_kernel: one thread scans one read (32 consecutive reads per
-// warp, so the 2-bit words a warp loads are contiguous).  Per base it rolls
-// the forward and reverse-complement codes of the current P-mer, takes the
-// canonical value c_q = min(code, rc code) (readings A, D, E) and feeds it to
-// a sliding-window minimum over w = K-P+1 P-mers (Definition 1: the
-// P-minimum-substring of K-mer i is min c_q over q in [i, i+K-P]).  The window
-// minimum is van Herk / Gil-Werman: blocks of w values, a running prefix
-// minimum of the current block and the suffix minima of the previous block,
-// kept in place in one per-thread shared-memory row -- O(1) per base and no
-// divergence across the lanes of a warp.  A superkmer (Def. 2, reading G) is
-// a maximal run of K-mers with equal minimizer; each is appended as a
-// descriptor (start, end, minimizer) to a per-thread shared-memory list.
-// When any list fills (or the reads end) the warp flushes: pid = fmix64(m)
-// mod NP (reading I) via a precomputed 64-bit reciprocal, a warp scan sizes
-// the records, one atomicAdd reserves a contiguous staging range, and each
-// lane writes its fixed-width records (dbg.h) with the two adjacency bases
-// (Sec. III-B).  Per-partition record/K-mer histograms are kept in
-// shared memory and flushed once per CTA (N^i_kmer).
+// Pass 1 (minimizers, superkmers, partition ids, sizes, staging), two kernels chosen by measured
+// speed (profiles/r02_ab.txt):
+//  * msp_warp_kernel (msp_warp.cuh): one WARP per read, lanes over P-mer positions -- the
+//    warp-parallel sliding minimizer, reads staged in shared memory by TMA bulk copies.  Every
+//    (K, P) except the ones below (bumblebee's K = 63, P = 19: 47.5 vs 49.2 ms for a thread per
+//    read).
+//  * msp_block_kernel: one THREAD per read (32 consecutive reads per warp), van Herk blocks of
+//    W = K-P+1 canonical P-mer codes in registers, for K = 31 with P = 11..15 (chr14: 10.8 vs
+//    15.6 ms for the warp kernel, whose per-read shuffles, ballots and descriptor ranks cost 5
+//    warp instructions per K-mer against 3.2 here).
+// Both append superkmer descriptors to shared memory and flush them per warp: pid = fmix64(m)
+// mod NP (reading I) via a precomputed 64-bit reciprocal, per-partition sizes N^i_kmer
+// (P:L972-975), one staging reservation per warp flush, fixed-width records (dbg.h) with the two
+// adjacency bases (Sec. III-B).
 //
 // The paper computed only "superkmer ids and offsets" on the GPU and left
-// the irregular copy to the CPU; here both run in this kernel.
+// the irregular copy to the CPU; here both run in these kernels.
 //
 // Pass 2, exclusive_scan (scan.cuh): record offsets per partition.
 // Pass 3, scatter_kernel: counting-sort scatter of the staged records into
@@ -65,10 +61,8 @@ struct MspArgs {
 
 template <typename CT>
 struct MspSmem {
-  // row[t * kMspThreads + tid], t < w: the van Herk block (in place)
   // desc_e[d * kMspThreads + tid]: last K-mer of descriptor d (its first is the previous
   // descriptor's last + 1, or the carried start); desc_m: its minimizer
-  CT* row;
   uint32_t* desc_e;
   CT* desc_m;
 };
@@ -117,35 +111,11 @@ __device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, ui
 // 32-bit shared-window accesses for the per-base loop (keeps generic-pointer
 // arithmetic and the shared-window base out of it).
 __device__ __forceinline__ uint32_t sh_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ uint32_t sh_ld(uint32_t a, uint32_t) {
-  uint32_t v;
-  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
-  return v;
-}
-__device__ __forceinline__ uint64_t sh_ld(uint32_t a, uint64_t) {
-  uint64_t v;
-  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
-  return v;
-}
 __device__ __forceinline__ void sh_st(uint32_t a, uint32_t v) {
   asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
 __device__ __forceinline__ void sh_st(uint32_t a, uint64_t v) {
   asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
-}
-// Pins a value in a register (the compiler may not re-derive it from the
-// constant bank inside the per-base loop).
-template <typename T>
-__device__ __forceinline__ T in_reg(T v) {
-  if constexpr (sizeof(T) == 8) {
-    uint64_t x = (uint64_t)v;
-    asm volatile("" : "+l"(x));
-    return (T)x;
-  } else {
-    uint32_t x = (uint32_t)v;
-    asm volatile("" : "+r"(x));
-    return (T)x;
-  }
 }
 
 // Records of a superkmer of n K-mers (pieces of at most nmax K-mers); the
@@ -183,9 +153,7 @@ __device__ __forceinline__ void write_record4(const MspArgs& a, uint32_t* dst, u
 // (computed once per descriptor and kept in place of the minimizer), size
 // histograms, one staging reservation per warp, record writes.
 // kK > 0: compile-time K (record geometry and pieces without runtime division).
-// kPid: the descriptors already hold the partition id (or kSkip), computed when the superkmer
-// closed (msp_kernel), instead of the minimizer.
-template <typename CT, int kK = 0, bool kPid = false>
+template <typename CT, int kK = 0>
 __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
                                                   int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
@@ -198,12 +166,9 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
     for (int d = 0; d < ndesc; ++d) {
       const int e = (int)sm.desc_e[d * kMspThreads + tid];
       CT& dm = sm.desc_m[d * kMspThreads + tid];
-      bool in = dm != kSkip;
-      if constexpr (!kPid) {
-        const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64((uint64_t)dm));
-        in = !a.ranged || (pid - a.pid_lo < a.pid_hi - a.pid_lo);
-        dm = in ? (CT)pid : kSkip;
-      }
+      const uint32_t pid0 = a.np == 1 ? 0u : fast_mod(a.mod, fmix64((uint64_t)dm));
+      const bool in = !a.ranged || (pid0 - a.pid_lo < a.pid_hi - a.pid_lo);
+      dm = in ? (CT)pid0 : kSkip;
       if (in) {
         // the per-partition sizes here, so that the record loop below has no atomics between
         // its loads and stores (the loads of consecutive records overlap)
@@ -249,166 +214,6 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
   }
   s_next = s;
   ndesc = 0;
-}
-
-// The generic kernel flushes its descriptor lists when a vote every kMspFlushBases bases finds one
-// with more than kMspDesc - (kMspFlushBases + 2) entries: a run of B bases closes at most one
-// superkmer per K-mer plus the read's last one.  A descriptor is (last K-mer, partition id), the
-// id computed when the superkmer closes, so a list costs 8 bytes per entry.  The shared memory per
-// thread (the van Herk row of w codes + the list) sets the occupancy of this latency-bound kernel:
-// 24 entries and a vote every 8 bases instead of 40 entries of (end, minimizer) and a vote every
-// 32 bases take K = 63 (P = 19, 64-bit codes) from 107.5 KB to 70.7 KB per CTA, 2 -> 3 CTAs/SM.
-constexpr int kMspFlushBases = 8, kMspDesc = 24;
-static_assert(kMspDesc >= kMspFlushBases + 2, "one vote interval must fit an empty list");
-
-// One thread's column of the van Herk row in shared memory.  kRow40: 64-bit codes of P <= 20
-// (< 2^40) kept as a 32-bit high part (bits 8..39) and an 8-bit low part -- 5 instead of 8 bytes
-// per entry, which for K = 63, P = 19 takes the CTA from 70.7 KB to 53.4 KB (3 -> 4 CTAs/SM).
-template <typename CT, bool kRow40>
-struct RowIO {
-  uint32_t hi_a, lo_a;
-  static constexpr uint32_t kStep = kMspThreads * (kRow40 ? 4u : (uint32_t)sizeof(CT));
-  __device__ __forceinline__ CT ld(int u) const {
-    if constexpr (kRow40) {
-      uint32_t h, l;
-      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(h) : "r"(hi_a + (uint32_t)u * kStep) : "memory");
-      asm volatile("ld.shared.u8 %0, [%1];" : "=r"(l) : "r"(lo_a + (uint32_t)u * kMspThreads) : "memory");
-      return ((CT)h << 8) | (CT)l;
-    } else {
-      return sh_ld(hi_a + (uint32_t)u * kStep, (CT)0);
-    }
-  }
-  __device__ __forceinline__ void st(int u, CT v) const {
-    if constexpr (kRow40) {
-      sh_st(hi_a + (uint32_t)u * kStep, (uint32_t)(v >> 8));
-      asm volatile("st.shared.u8 [%0], %1;" ::"r"(lo_a + (uint32_t)u * kMspThreads), "r"((uint32_t)v & 255u)
-                   : "memory");
-    } else {
-      sh_st(hi_a + (uint32_t)u * kStep, v);
-    }
-  }
-  static size_t bytes(int w) { return (size_t)w * kMspThreads * (kRow40 ? 5u : sizeof(CT)); }
-};
-
-__device__ __forceinline__ uint32_t desc_pid(const MspArgs& a, uint64_t m) {
-  const uint32_t pid = a.np == 1 ? 0u : fast_mod(a.mod, fmix64(m));
-  return (!a.ranged || pid - a.pid_lo < a.pid_hi - a.pid_lo) ? pid : ~0u;
-}
-
-// KC, PC > 0: compile-time K and P (bumblebee: 63, 19), so the rolling masks and shifts and the
-// van Herk block length W = K - P + 1 are constants.
-template <typename CT, bool kRow40, int KC = 0, int PC = 0>
-__global__ void __launch_bounds__(kMspThreads) msp_kernel(MspArgs a) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const int tid = threadIdx.x, lane = tid & 31;
-  MspSmem<uint32_t> sm;  // descriptors: end + partition id
-  unsigned char* sp = smem_raw;
-  sm.desc_m = reinterpret_cast<uint32_t*>(sp);
-  constexpr int kDesc = kMspDesc, kFB = kMspFlushBases;
-  sp += sizeof(uint32_t) * kDesc * kMspThreads;
-  sm.desc_e = reinterpret_cast<uint32_t*>(sp);
-  sp += sizeof(uint32_t) * kDesc * kMspThreads;
-  sm.row = nullptr;
-  CT* row0 = reinterpret_cast<CT*>(sp);
-
-  const int K = KC ? KC : a.k, P = PC ? PC : in_reg(a.p), w = KC ? KC - PC + 1 : in_reg(a.w);
-  const CT maskP = PC ? (CT)((2 * PC == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * PC)) - 1))
-                      : in_reg((CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1)));
-  const int topP = PC ? 2 * PC - 2 : in_reg(2 * P - 2);
-  const uint64_t stride = (uint64_t)gridDim.x * kMspThreads;
-  // shared-window addresses of this thread's column of the van Herk block and descriptors
-  RowIO<CT, kRow40> row;
-  if constexpr (kRow40) {
-    row.hi_a = in_reg(sh_addr(reinterpret_cast<uint32_t*>(row0) + tid));
-    row.lo_a = in_reg(sh_addr(reinterpret_cast<unsigned char*>(row0) + 4 * (size_t)a.w * kMspThreads + tid));
-  } else {
-    row.hi_a = in_reg(sh_addr(row0 + tid));
-    row.lo_a = 0;
-  }
-  const uint32_t de_a = in_reg(sh_addr(sm.desc_e + tid)), dm_a = in_reg(sh_addr(sm.desc_m + tid));
-  constexpr uint32_t kDescStepE = kMspThreads * 4, kDescStepM = kMspThreads * 4;
-  // all lanes of a warp iterate together; a warp covers 32 consecutive reads
-  for (uint64_t r0 = (uint64_t)blockIdx.x * kMspThreads + (tid & ~31); r0 < a.n_reads; r0 += stride) {
-    const uint64_t r = r0 + lane;
-    uint64_t o = 0;
-    int L = 0;
-    if (r < a.n_reads) {
-      o = a.offsets[r];
-      L = (int)(a.offsets[r + 1] - o);
-    }
-    const int nk = L - K + 1;
-    if (nk <= 0) L = 0;  // reading N: no K-mers
-    int Lmax = L;
-#pragma unroll
-    for (int dlt = 16; dlt; dlt >>= 1) Lmax = max(Lmax, __shfl_xor_sync(kFull, Lmax, dlt));
-    int ndesc = 0, s_next = 0;
-    CT f = 0, rc = 0, pre = 0, m_cur = 0;
-    // nxt = row[u + 1], loaded one P-mer ahead so that the shared-memory latency is off the
-    // per-base dependency chain (in the read's first block it is never used)
-    CT nxt = 0;
-    int u = 0;  // position within the current van Herk block
-    for (int c0 = 0; c0 < Lmax; c0 += 32) {
-      uint64_t wbuf = c0 < L ? window64(a.words, a.n_words, o + c0) : 0;
-      const int jn = min(32, L - c0);  // bases of this read in the chunk (<= 0: none)
-#pragma unroll 1
-      for (int h = 0; h < 32; h += kFB) {
-      for (int jj = h; jj < min(jn, h + kFB); ++jj) {
-        const int j = c0 + jj;
-        const uint32_t b = (uint32_t)(wbuf >> 62);
-        wbuf <<= 2;
-        f = ((f << 2) | (CT)b) & maskP;
-        rc = (rc >> 2) | ((CT)(3u - b) << topP);
-        if (j < P - 1) continue;
-        const int q = j - P + 1;  // P-mer index
-        const CT snext = nxt;
-        if (u + 2 < w) nxt = row.ld(u + 2);  // for the next P-mer
-        const CT c = f < rc ? f : rc;
-        row.st(u, c);
-        pre = (u == 0 || c < pre) ? c : pre;
-        if (q >= w - 1) {  // K-mer i = q-w+1 is complete
-          const int i = q - w + 1;
-          const CT m = (u == w - 1 || pre < snext) ? pre : snext;
-          if (i > 0 && m != m_cur) {  // a superkmer ends at K-mer i-1 (Def. 2)
-            sh_st(de_a + (uint32_t)ndesc * kDescStepE, (uint32_t)(i - 1));
-            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, desc_pid(a, (uint64_t)m_cur));
-            ++ndesc;
-          }
-          m_cur = m;
-          if (i == nk - 1) {  // the read's last superkmer
-            sh_st(de_a + (uint32_t)ndesc * kDescStepE, (uint32_t)i);
-            sh_st(dm_a + (uint32_t)ndesc * kDescStepM, desc_pid(a, (uint64_t)m_cur));
-            ++ndesc;
-          }
-        }
-        if (u == w - 1) {  // block complete: suffix minima in place, loads issued 8 at a time
-          CT y = row.ld(w - 1);
-          int t = w - 2;
-          for (; t >= 7; t -= 8) {
-            CT x[8];
-#pragma unroll
-            for (int v = 0; v < 8; ++v) x[v] = row.ld(t - v);
-#pragma unroll
-            for (int v = 0; v < 8; ++v) {
-              if (y < x[v]) row.st(t - v, y);
-              else y = x[v];
-            }
-          }
-          for (; t >= 0; --t) {
-            const CT x = row.ld(t);
-            if (y < x) row.st(t, y);
-            else y = x;
-          }
-          u = 0;
-          if (w > 1) nxt = row.ld(1);
-        } else {
-          ++u;
-        }
-      }
-      if (__any_sync(kFull, ndesc > kDesc - (kFB + 2))) flush_descriptors<uint32_t, KC, true>(a, sm, ndesc, s_next, o, L);
-      }
-    }
-    if (__any_sync(kFull, ndesc > 0)) flush_descriptors<uint32_t, KC, true>(a, sm, ndesc, s_next, o, L);
-  }
 }
 
 // Pass 3: scatter staged records into partition order.  A record's bin is
@@ -608,7 +413,7 @@ __global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const ui
 // no shared-memory row.  K-mer i's minimizer (Def. 1) is
 // min(suffix_min_prev[t], prefix_min_cur[t-1]) for i = q0 - W + t, where the
 // current block holds P-mers q0 .. q0+W-1.  Same descriptors and flush as
-// msp_kernel; reads of any length (lanes past their read end run masked).
+// the warp kernel; reads of any length (lanes past their read end run masked).
 // P-mer codes of the register-blocked kernel: 32-bit up to P = 16, else 64-bit (K = 63, P = 19);
 // descriptor lists hold at least W + 3 entries (a block of W bases closes at most W superkmers,
 // plus the read's last one and the carry).
@@ -630,7 +435,6 @@ __global__ void __launch_bounds__(kMspThreads, 1) msp_block_kernel(MspArgs a) {
   sm.desc_m = reinterpret_cast<CT*>(sp);
   sp += sizeof(CT) * kDesc * kMspThreads;
   sm.desc_e = reinterpret_cast<uint32_t*>(sp);
-  sm.row = nullptr;
   constexpr CT kMaskP = (CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1));
   constexpr CT kInf = ~(CT)0;
   constexpr int kTopP = 2 * P - 2;
@@ -734,6 +538,9 @@ __global__ void __launch_bounds__(kMspThreads, 1) msp_block_kernel(MspArgs a) {
 
 }  // namespace dbg
 
+int dbg_sm_count();
+#include "msp_warp.cuh"
+
 using namespace dbg;
 
 int dbg_sm_count() {
@@ -785,17 +592,6 @@ static bool msp_block_launch(const MspArgs& a, int grid, cudaStream_t stream, cu
     case 15: *e = launch_msp_block<17, 15>(a, grid, stream); return true;
   }
   return false;
-}
-
-template <typename CT, bool kRow40, int KC = 0, int PC = 0>
-static cudaError_t launch_msp(const MspArgs& a, int grid, cudaStream_t stream) {
-  const size_t smem = 2 * sizeof(uint32_t) * kMspDesc * kMspThreads + RowIO<CT, kRow40>::bytes(a.w);
-  cudaError_t e = cudaFuncSetAttribute(msp_kernel<CT, kRow40, KC, PC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)smem);
-  if (e != cudaSuccess) return e;
-  grid = msp_grid((const void*)msp_kernel<CT, kRow40, KC, PC>, grid, smem);
-  msp_kernel<CT, kRow40, KC, PC><<<grid, kMspThreads, smem, stream>>>(a);
-  return cudaGetLastError();
 }
 
 static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, uint64_t n_words,
@@ -857,14 +653,10 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
       return DBG_ECUDA;
     if (n_reads) {
       const uint64_t want = (n_reads + kMspThreads - 1) / kMspThreads;
-      const uint64_t cap = (uint64_t)dbg_sm_count() * 32;  // launch_msp* cap it at one resident wave
+      const uint64_t cap = (uint64_t)dbg_sm_count() * 32;  // the launchers cap it at one resident wave
       const int grid = (int)(want < cap ? want : cap);
       cudaError_t e = cudaSuccess;
-      if (!msp_block_launch(a, grid, stream, &e))
-        e = (a.k == 63 && a.p == 19) ? launch_msp<uint64_t, true, 63, 19>(a, grid, stream)
-          : a.p <= 16 ? launch_msp<uint32_t, false>(a, grid, stream)
-                      : (a.p <= 20 ? launch_msp<uint64_t, true>(a, grid, stream)
-                                                    : launch_msp<uint64_t, false>(a, grid, stream));
+      if (!msp_block_launch(a, grid, stream, &e)) e = launch_msp_warp_any(a, stream);
       if (e != cudaSuccess) return DBG_ECUDA;
     }
     // d_fill is idle until pass 2 (which zeroes it): scratch for the tile sums

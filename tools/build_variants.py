@@ -26,10 +26,12 @@ def build_variant(name: str, defs: list[str], rev: str | None = None) -> str:
         blob = subprocess.run(["git", "-C", ROOT, "show", f"{rev}:include/dbg.h"], check=True,
                               capture_output=True).stdout
         open(os.path.join(top, "include", "dbg.h"), "wb").write(blob)
-        for f in os.listdir(B.CSRC):
-            blob = subprocess.run(["git", "-C", ROOT, "show", f"{rev}:paper_conf_icdcs_qiul17_b200/csrc/{f}"],
-                                  check=True, capture_output=True).stdout
-            open(os.path.join(csrc, f), "wb").write(blob)
+        names = subprocess.run(["git", "-C", ROOT, "ls-tree", "--name-only", rev, "paper_conf_icdcs_qiul17_b200/csrc/"],
+                               check=True, capture_output=True, text=True).stdout.split()
+        for path in names:
+            blob = subprocess.run(["git", "-C", ROOT, "show", f"{rev}:{path}"], check=True,
+                                  capture_output=True).stdout
+            open(os.path.join(csrc, os.path.basename(path)), "wb").write(blob)
     objs = []
     for s in B.SOURCES:
         o = os.path.join(out, s.replace(".cu", ".o"))
