@@ -376,3 +376,43 @@ def test_two_level_scatter_partition_order(refine):
     d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
     res = b.build(d_bases, d_off)
     compare_vertices(res.vertices, oracle.graph(rs.seq, rs.offsets, 31, 11, np_, n_threads=NT))
+
+
+@pytest.mark.parametrize("k,p", [(63, 19), (21, 7), (45, 30)])
+def test_warp_msp_chunks_pieces_and_fallback(k, p):
+    """msp_warp_kernel (every (K, P) but K = 31 with P = 11..15): chunks of 32 reads whose words
+    fit the TMA-staged buffer next to chunks that do not (long reads: global-memory windows),
+    reads longer than one piece of 32R P-mer positions (the open superkmer carried across
+    pieces), reads of exactly K bases, superkmers longer than a record (pieces), and P + R - 1 >
+    32 (two-window codes, P = 30).  Records vs the oracle's superkmers (per-partition sizes and
+    record counts) and the whole graph vs the oracle."""
+    rng = np.random.default_rng(1000 + k + p)
+    reads = []
+    for q in range(7):  # chunks: short, long (unstaged), mixed, ...
+        for t in range(32):
+            if q == 1 or (q == 4 and t % 5 == 0):
+                n = int(rng.integers(400, 1500))
+            elif q == 5 and t % 3 == 0:
+                n = k
+            else:
+                n = int(rng.integers(k, 160))
+            reads.append("".join(rng.choice(list("ACGT"), n)))
+    reads[40] = "A" * 900          # one minimizer over the whole read: superkmer pieces
+    reads[70] = "AC" * 300
+    rs = _readset(reads)
+    _check(rs, k, p, 11)
+    b = DbgBuilder(k, p, 11)
+    d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
+    b.msp(d_bases, d_off)
+    assert b.sync_sizes()
+    torch.cuda.synchronize()
+    sk = oracle.msp(rs.seq, rs.offsets, k, p, 11)
+    nmax = _lib.dbg_record_max_kmers(b.prm)
+    want_k = np.bincount(sk["pid"], weights=sk["n_kmers"], minlength=11).astype(np.int64)
+    want_r = np.bincount(sk["pid"], weights=(sk["n_kmers"] + nmax - 1) // nmax, minlength=11).astype(np.int64)
+    assert np.array_equal(b.part_kmers, want_k)
+    assert np.array_equal(b.part_records, want_r)
+    n = int(b.part_records.sum())
+    words = b.records[:n * b.rec_words].cpu().numpy().view(np.uint32)
+    assert occurrences_from_records(decode_records(words, b.rec_words, k), k) == \
+        occurrences_from_oracle_msp(sk, rs.reads(), k)
