@@ -46,7 +46,7 @@ UNIT = "kmers/s"
 ALG_BYTES_PER_KMER = 68
 # version tag of the on-chip kernel: profiles/traffic.json (ncu --set full) is quoted only when it
 # was captured on this version and workload
-KERNEL_VERSION = "smem-v13"
+KERNEL_VERSION = "smem-v14"
 
 
 def _peaks():
@@ -294,6 +294,10 @@ def run_ours(args):
     else:
         b = src = launch_builder(rs.k, rs.p, rs.num_partitions, n_kmers_total, args.lam, args.alpha, device=dev,
                                  min_count=args.min_count, **kw)
+    if args.scatter == "one":  # A/B: pass 2 in one level
+        src.two_level = False
+    elif args.scatter == "two":  # A/B: two levels at any size and record width
+        src.two_level_words, src.two_level_min_bytes = (4, 8, 16), 0
     d_bases, d_off = src.upload(packed, offsets, stream)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     E = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
@@ -508,6 +512,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--out-frac", type=float, default=0.4, help="output capacity / K-mers")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--scatter", choices=["auto", "one", "two"], default="auto", help="A/B: pass-2 scatter levels")
     ap.add_argument("--min-count", type=int, default=0, help="row f4 low-count filter (0: the full graph)")
     args = ap.parse_args()
     if "WORLD_SIZE" not in os.environ and args.gpus > 1:

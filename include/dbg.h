@@ -21,7 +21,7 @@
  *    dbg_table_plan, dbg_hash_build, dbg_extract_graph (dbg_vertex_wide
  *    output); fine_p must be 0 or P; the on-chip, sort and checksum
  *    calls return DBG_EINVAL;
- *    1 <= num_partitions * refine <= 4,194,303.  Every per-partition array
+ *    1 <= num_partitions * refine <= 16,777,215 (2^24 - 1, the record header's pid field).  Every per-partition array
  *    and pid range below is in FINE partitions (NP * refine of them); only
  *    dbg_vertex.pid reports the paper's partition (fine pid mod NP).  Reads shorter than K contribute
  *    nothing and are not an error (reading N).
@@ -36,7 +36,7 @@
 extern "C" {
 #endif
 
-#define DBG_ABI_VERSION 11
+#define DBG_ABI_VERSION 12
 
 #if defined(__GNUC__)
 #define DBG_API __attribute__((visibility("default")))
@@ -118,7 +118,7 @@ typedef struct {
  * All arrays are device memory owned by the caller.  Records of partition i
  * occupy record slots [d_record_offset[i], d_record_offset[i+1]) of
  * d_records; one record is dbg_record_words() uint32 words:
- *   word 0: n_kmers (bits 0-7) | has_left (bit 8) | has_right (bit 9) | pid (bits 10-31)
+ *   word 0: n_kmers (bits 0-5, <= 63) | has_left (bit 6) | has_right (bit 7) | fine pid (bits 8-31)
  *   words 1..: the bases S[s-has_left .. e+K-1+has_right], 2-bit, 16 per word,
  *              first base in the most significant bits (Sec. III-B).
  * A superkmer longer than the record holds is stored as consecutive pieces,
@@ -136,19 +136,27 @@ typedef struct {
   uint32_t* d_records;       /* d_record_offset[NP] records in partition order; NULL => pass 1 */
   uint32_t* d_scratch;       /* optional, staging_cap records (not aliasing d_staging or d_records):
                                 with more than 8192 fine partitions pass 2 then scatters in two
-                                levels -- into buckets of 8 consecutive partitions (d_scratch),
-                                then within each bucket (d_records) -- which avoids a DRAM
-                                read-modify-write per 16-byte record; NULL: one level */
+                                counting-sort levels -- into buckets of 2^s consecutive partitions
+                                (d_scratch), then within each bucket (d_records / the peers) --
+                                each level ranking a tile of records in shared memory and
+                                reserving once per (tile, bin); needs d_work.  NULL: one level,
+                                one global rank atomic per record */
   /* Multi-GPU emission: with n_peers > 0, pass 2 writes
      each record of fine partition f into the partition buffer of f's owner GPU o -- the o with
      d_peer_bounds[o] <= f < d_peer_bounds[o+1] -- at record slot d_record_offset[f] + rank, i.e.
      straight into peer memory over NVLink (IPC-mapped device pointers).  d_record_offset must
-     then hold dbg_exchange_plan's d_dest_offset; d_records is not written.  Only the one-level
-     scatter supports peers (d_rank and d_scratch must be NULL).  n_peers = 0: local pass 2. */
+     then hold dbg_exchange_plan's d_dest_offset; d_records is not written.  Both scatters
+     support peers (the two-level one buckets locally from d_n_records, then writes the peers).
+     n_peers = 0: local pass 2. */
   uint32_t* const* d_peer_records; /* [n_peers] device array of the owners' record buffers */
   const int32_t* d_peer_bounds;    /* [n_peers+1] device array, owner o owns [b[o], b[o+1]) */
   int32_t n_peers;
+  uint64_t* d_work;          /* with d_scratch: dbg_scatter_work_words(prm) uint64 of caller memory
+                                (bucket offsets, cursors and tile counts of the two-level scatter) */
 } dbg_partition_set;
+
+/* uint64 words of dbg_partition_set.d_work for the two-level scatter. */
+DBG_API uint64_t dbg_scatter_work_words(const dbg_params* prm);
 
 /* ---- sizes ------------------------------------------------------------ */
 DBG_API int dbg_abi_version(void);

@@ -38,7 +38,8 @@ class dbg_partition_set(ctypes.Structure):
                 ("d_staged", ctypes.c_void_p), ("d_staging", ctypes.c_void_p),
                 ("staging_cap", ctypes.c_uint64), ("d_records", ctypes.c_void_p),
                 ("d_scratch", ctypes.c_void_p),
-                ("d_peer_records", ctypes.c_void_p), ("d_peer_bounds", ctypes.c_void_p), ("n_peers", ctypes.c_int32)]
+                ("d_peer_records", ctypes.c_void_p), ("d_peer_bounds", ctypes.c_void_p), ("n_peers", ctypes.c_int32),
+                ("d_work", ctypes.c_void_p)]
 
 
 # dbg_vertex (56 B) and dbg_stats (32 B) as numpy dtypes
@@ -62,6 +63,7 @@ SIGNATURES = {
     "dbg_abi_version": (ctypes.c_int, []),
     "dbg_record_words": (ctypes.c_uint32, [_PRM]),
     "dbg_record_max_kmers": (ctypes.c_uint32, [_PRM]),
+    "dbg_scatter_work_words": (ctypes.c_uint64, [_PRM]),
     "dbg_slot_bytes": (ctypes.c_uint32, [_PRM]),
     "dbg_key_bytes": (ctypes.c_uint32, [_PRM]),
     "dbg_table_capacity": (_U64, [_PRM, _U64]),
@@ -90,7 +92,7 @@ SIGNATURES = {
 }
 
 _lib = None
-ABI_VERSION = 11
+ABI_VERSION = 12
 
 
 def load():
@@ -147,10 +149,10 @@ def fine_partitions(prm: dbg_params) -> int:
 
 def partition_set(n_records, n_kmers, record_offset, fill, staged, staging=None, staging_cap: int = 0,
                   records=None, scratch=None, peer_records=None, peer_bounds=None,
-                  n_peers: int = 0) -> dbg_partition_set:
+                  n_peers: int = 0, work=None) -> dbg_partition_set:
     return dbg_partition_set(_ptr(n_records), _ptr(n_kmers), _ptr(record_offset), _ptr(fill), _ptr(staged),
                              _ptr(staging), staging_cap, _ptr(records), _ptr(scratch),
-                             _ptr(peer_records), _ptr(peer_bounds), n_peers)
+                             _ptr(peer_records), _ptr(peer_bounds), n_peers, _ptr(work))
 
 
 # --------------------------------------------------------------------------- entry points
@@ -166,6 +168,10 @@ def dbg_record_words(prm: dbg_params) -> int:
 
 def dbg_record_max_kmers(prm: dbg_params) -> int:
     return load().dbg_record_max_kmers(ctypes.byref(prm))
+
+
+def dbg_scatter_work_words(prm: dbg_params) -> int:
+    return load().dbg_scatter_work_words(ctypes.byref(prm))
 
 
 def dbg_slot_bytes(prm: dbg_params) -> int:

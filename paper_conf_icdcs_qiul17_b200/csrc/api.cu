@@ -21,6 +21,16 @@ extern "C" uint32_t dbg_record_max_kmers(const dbg_params* prm) {
   return prm ? record_max_kmers(prm->k) : 0u;
 }
 
+// Two-level scatter workspace (msp.cu ts_*): cursors, offsets and tile counts of <= 4096 buckets.
+extern "C" uint64_t dbg_scatter_work_words(const dbg_params* prm) {
+  if (!prm || prm->num_partitions < 1) return 0;
+  const int64_t np = (int64_t)prm->num_partitions * (prm->refine > 1 ? prm->refine : 1);
+  int s = 0;
+  while (s < 12 && ((np + (1ll << s) - 1) >> s) > 2048) ++s;
+  const uint64_t nb = (uint64_t)((np + (1ll << s) - 1) >> s);
+  return 3 * nb + 2;
+}
+
 // Sec. IV-A: "we use [N^i_kmer] with a load ratio alpha to set the
 // hash table size as lambda/(4 alpha) N^i_kmer"; lambda = 2, alpha = 0.5 by
 // default, which makes the capacity N^i_kmer (Table II).

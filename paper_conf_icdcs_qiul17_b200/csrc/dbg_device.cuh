@@ -10,7 +10,18 @@ namespace dbg {
 
 constexpr int kWarp = 32;
 constexpr uint32_t kFull = 0xffffffffu;
-constexpr uint32_t kMaxPid = (1u << 22) - 1;
+// Record header (dbg.h): n_kmers (bits 0-5, <= 63) | has_left (bit 6) | has_right (bit 7) |
+// fine pid (bits 8-31): up to 2^24 - 1 fine partitions.
+constexpr uint32_t kMaxPid = (1u << 24) - 1;
+constexpr int kHdrPidShift = 8;
+constexpr uint32_t kHdrNMask = 63u;
+__host__ __device__ __forceinline__ uint32_t rec_header(uint32_t n, uint32_t hl, uint32_t hr, uint32_t pid) {
+  return n | hl << 6 | hr << 7 | pid << kHdrPidShift;
+}
+__host__ __device__ __forceinline__ uint32_t hdr_n(uint32_t h) { return h & kHdrNMask; }
+__host__ __device__ __forceinline__ uint32_t hdr_hl(uint32_t h) { return (h >> 6) & 1u; }
+__host__ __device__ __forceinline__ uint32_t hdr_hr(uint32_t h) { return (h >> 7) & 1u; }
+__host__ __device__ __forceinline__ uint32_t hdr_pid(uint32_t h) { return h >> kHdrPidShift; }
 constexpr uint64_t kOccupied = 1ull << 63;
 
 // Status bits (dbg_sync_status).
@@ -21,8 +32,9 @@ constexpr uint32_t kStatusNoSpace = 2u;
 // K <= 63, 16 (240 bases) for K <= 127 (row f3).
 __host__ __device__ inline uint32_t record_words(int k) { return k <= 39 ? 4u : (k <= 63 ? 8u : 16u); }
 __host__ __device__ inline uint32_t record_max_kmers(int k) {
-  // bases = 16 * (R - 1) >= has_left + n + K - 1 + has_right
-  return 16u * (record_words(k) - 1u) - (uint32_t)k - 1u;
+  // bases = 16 * (R - 1) >= has_left + n + K - 1 + has_right, and n fits the header's 6 bits
+  const uint32_t n = 16u * (record_words(k) - 1u) - (uint32_t)k - 1u;
+  return n < kHdrNMask ? n : kHdrNMask;
 }
 
 // Number of fine partitions the device works on (dbg.h: num_partitions * refine).

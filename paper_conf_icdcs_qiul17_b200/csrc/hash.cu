@@ -196,7 +196,7 @@ __device__ __forceinline__ Job<Code> make_job(const WarpRecs<R>& sm, uint32_t ki
   while (sm.pre[r + 1] <= kid) ++r;
   const uint32_t* w = sm.w[r];
   const uint32_t hdr = w[0];
-  const int n = hdr & 255u, hl = (hdr >> 8) & 1u, hr = (hdr >> 9) & 1u;
+  const int n = hdr_n(hdr), hl = hdr_hl(hdr), hr = hdr_hr(hdr);
   const int t = (int)(kid - sm.pre[r]);
   const int b = hl + t;  // first base of the K-mer in the record
   Code fwd, rc;
@@ -245,8 +245,8 @@ __device__ __forceinline__ bool hash_warp(const uint32_t* recs, int64_t n_recs, 
     }
     const uint32_t hdr = sm.w[lane][0];
     uint64_t t0, cap;
-    table_of(hdr >> 10, t0, cap);
-    n = cap ? hdr & 255u : 0u;  // capacity 0: the partition is built elsewhere (on chip)
+    table_of(hdr_pid(hdr), t0, cap);
+    n = cap ? hdr_n(hdr) : 0u;  // capacity 0: the partition is built elsewhere (on chip)
     sm.t0[lane] = t0;
     sm.cap[lane] = cap;
   }
@@ -378,21 +378,25 @@ __device__ __forceinline__ uint32_t kmer_partition(uint64_t hi, uint64_t lo, con
 }
 
 // kmer_partition with compile-time K <= 31 and P <= 16 (the chr14 launch: K = 31, P = 11 under a
-// longer device minimizer): the K - P + 1 canonical P-mers of the K-mer as 32-bit values taken
-// with constant funnel shifts, min-reduced three at a time -- the same minimizer as
-// kmer_minimizer64 (the vertex's P-minimizer, reading V) at about half the instructions.
+// longer device minimizer).  Each P-mer is taken TOP-aligned in a 32-bit word -- its 2P bits
+// followed by the next bases of the K-mer (or zeros) -- with one funnel shift, and the words are
+// min-reduced three at a time: the top 2P bits of the minimum word are the minimum P-mer (a
+// numeric minimum is decided by the leading bits first), on either strand, so no masks are needed.
+// The same minimizer as kmer_minimizer64 (the vertex's P-minimizer, reading V).
 template <int KC, int PC>
 __device__ __forceinline__ uint32_t kmer_partition_c(uint64_t lo, const OutArgs& oa) {
   static_assert(KC <= 31 && PC >= 1 && PC <= 16, "one-word K-mer, 32-bit P-mer");
   const uint64_t rc = revcomp64(lo, KC);
-  constexpr uint32_t mask = (uint32_t)((2ull << (2 * PC - 1)) - 1);
+  // forward P-mer q = bits [2(K-P-q), 2(K-q)) of lo; reverse one = bits [2q, 2q+2P) of rc
+  const uint64_t fa = lo << (64 - 2 * KC);  // the K-mer's first base at bit 63
   uint32_t m = ~0u;
 #pragma unroll
   for (int q = 0; q <= KC - PC; ++q) {
-    const uint32_t f = (uint32_t)(lo >> (2 * (KC - PC - q))) & mask, r = (uint32_t)(rc >> (2 * q)) & mask;
+    const uint32_t f = (uint32_t)((fa << (2 * q)) >> 32);
+    const uint32_t r = (uint32_t)((rc << (64 - 2 * q - 2 * PC)) >> 32);
     m = min(m, min(f, r));
   }
-  return fast_mod(oa.np_mod, fmix64((uint64_t)m));
+  return fast_mod(oa.np_mod, fmix64((uint64_t)(m >> (32 - 2 * PC))));
 }
 
 struct XShared {
@@ -641,7 +645,7 @@ struct SmemStage {
   unsigned long long Pq[2][kGroupParts + 2];  // P[first .. last] of the current and the next item
   uint32_t pre[RB + 1];                       // K-mer offsets of the records with on-chip K-mers
   uint2 desc[RB];                             // their descriptors: x = batch position | n << 10 |
-                                              // hl << 18 | hr << 19, y = table offset | capacity << 16
+                                              // hl << 16 | hr << 17, y = table offset | capacity << 16
   uint16_t rwin[(RB * (16 * (R - 1) - 1) + 31) / 32 + 1];  // record of the first K-mer of each warp window
   ItemDesc it[4];                             // items i .. i+3 (ring)
   typename cub::BlockScan<uint32_t, T>::TempStorage scan;
@@ -1128,10 +1132,10 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         const uint32_t w0 = st.w[bb][0][j];
         uint32_t c;
         if (split) {
-          c = w0 & 255u;
+          c = hdr_n(w0);
         } else {
-          const uint32_t x = (w0 >> 10) - I.first;
-          c = Pq[x + 1] != Pq[x] ? w0 & 255u : 0u;  // off-chip partition: skipped here
+          const uint32_t x = hdr_pid(w0) - I.first;
+          c = Pq[x + 1] != Pq[x] ? hdr_n(w0) : 0u;  // off-chip partition: skipped here
         }
         cnt[v] = c ? c | 1u << 16 : 0u;
       }
@@ -1149,12 +1153,12 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         const uint32_t w0 = st.w[bb][0][jj];
         uint32_t t0 = 0, cp = (uint32_t)a.slots;
         if (!split) {
-          const uint32_t x = (w0 >> 10) - I.first;
+          const uint32_t x = hdr_pid(w0) - I.first;
           t0 = (uint32_t)(Pq[x] - I.P0);
           cp = (uint32_t)(Pq[x + 1] - Pq[x]);
         }
         st.pre[c] = e;
-        st.desc[c] = make_uint2((uint32_t)jj | (w0 & 1023u) << 10, t0 | cp << 16);
+        st.desc[c] = make_uint2((uint32_t)jj | (w0 & 255u) << 10, t0 | cp << 16);
         for (uint32_t m = (e + 31) >> 5; 32 * m < e + n; ++m) st.rwin[m] = (uint16_t)c;
       }
     }
@@ -1180,7 +1184,7 @@ __global__ void __launch_bounds__(kSmemThreads, kMinCtas) smem_subgraph_kernel(S
         const uint32_t cc = act ? c : rb;
         const uint2 d = st.desc[cc];
         const int t = (int)(kid - st.pre[cc]);
-        const int j = d.x & 1023u, n = (d.x >> 10) & 255u, hl = (d.x >> 18) & 1u, hr = (d.x >> 19) & 1u;
+        const int j = d.x & 1023u, n = (d.x >> 10) & kHdrNMask, hl = (d.x >> 16) & 1u, hr = (d.x >> 17) & 1u;
         const uint32_t t0 = d.y & 0xffffu, cap = d.y >> 16;
         const uint32_t* w = &st.w[bb][0][j];
         const int b = hl + t;

@@ -40,7 +40,6 @@ constexpr int kMspThreads = 128;
 // for 6-7 CTAs/SM with 28-32 descriptors was no faster on chr14, profiles/r02_ab.txt)
 constexpr int kMaxDescBlock = 40;
 constexpr int kSmemHistMaxNp = 8192;
-constexpr int kBucketShift = 3;  // two-level scatter: buckets of 8 consecutive fine partitions (r02f: 3 < 4 < 5 < 6)
 
 struct MspArgs {
   const uint64_t* words;
@@ -92,7 +91,7 @@ __device__ __forceinline__ void write_record(const MspArgs& a, uint32_t* dst, ui
           v = window64(a.words, a.n_words, o + bs);
           if (left < 32) v &= ~(~0ull >> (2 * left));
         }
-        w[0] = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
+        w[0] = rec_header((uint32_t)(pe - ps + 1), hl, hr, pid);
         w[1] = (uint32_t)(v >> 32);  // bases 0..15
         continue;
       }
@@ -144,7 +143,7 @@ __device__ __forceinline__ void write_record4(const MspArgs& a, uint32_t* dst, u
   const uint32_t m1 = nb >= 48 ? ~0u : (nb <= 32 ? 0u : ~(~0u >> (2 * (nb - 32))));
   const uint64_t b0 = v0 & m0;
   const uint32_t b1 = (uint32_t)(v1 >> 32) & m1;
-  const uint4 rec = make_uint4((uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10), (uint32_t)(b0 >> 32),
+  const uint4 rec = make_uint4(rec_header((uint32_t)(pe - ps + 1), hl, hr, pid), (uint32_t)(b0 >> 32),
                                (uint32_t)b0, b1);
   reinterpret_cast<uint4*>(dst)[0] = rec;
 }
@@ -157,7 +156,7 @@ template <typename CT, int kK = 0>
 __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSmem<CT>& sm, int& ndesc,
                                                   int& s_next, uint64_t o, int L) {
   const int tid = threadIdx.x, lane = tid & 31;
-  const int nmax = kK > 0 ? (int)(16u * (record_words(kK) - 1u) - (uint32_t)kK - 1u) : (int)a.max_kmers;
+  const int nmax = kK > 0 ? (int)record_max_kmers(kK) : (int)a.max_kmers;
   const bool r4 = kK > 0 ? record_words(kK) == 4 : a.rec_words == 4;
   constexpr CT kSkip = ~(CT)0;  // a superkmer of another pass's partition (row f2)
   uint32_t my_records = 0;
@@ -216,12 +215,9 @@ __device__ __forceinline__ void flush_descriptors(const MspArgs& a, const MspSme
   ndesc = 0;
 }
 
-// Pass 3: scatter staged records into partition order.  A record's bin is
-// pid >> shift and its bin starts at record offset rec_off[bin << shift]
-// (shift = 0: one bin per partition; two-level scatter, level 1: bins of 2^shift
-// consecutive partitions, whose records are contiguous in partition order).
-// nb bins; with nb <= kSmemHistMaxNp a CTA tile ranks its records in shared
-// memory and reserves once per bin, else one global atomic per record.
+// Pass 3 (one level): scatter staged records into partition order, record of partition pid at
+// rec_off[pid] + rank.  With nb <= kSmemHistMaxNp partitions a CTA tile ranks its records in
+// shared memory and reserves once per partition, else one global atomic per record.
 // L2 cache policies of the scatter: the staged records stream through once (evict first); the
 // partitions' open sectors, their cursors and offsets stay (evict last), so a 32-byte sector
 // that receives a 16-byte record is still in L2 when its other half arrives and is written back
@@ -267,7 +263,7 @@ __global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint3
                                                                   uint64_t staging_cap,
                                                                   const uint64_t* __restrict__ rec_off,
                                                                   unsigned long long* fill,
-                                                                  uint32_t* __restrict__ records, int nb, int shift,
+                                                                  uint32_t* __restrict__ records, int nb,
                                                                   uint32_t* const* peer_records,
                                                                   const int32_t* peer_bounds, int n_peers) {
   extern __shared__ unsigned long long sh_base[];  // [nb] global bases (per tile), then [nb] counts
@@ -301,7 +297,7 @@ __global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint3
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       rank[v] = 0;
       if (idx < n) {
-        const uint32_t bin = (rec[v][0].x >> 10) >> shift;
+        const uint32_t bin = hdr_pid(rec[v][0].x);
         if (smem) rank[v] = atomicAdd(sh_cnt + bin, 1u);
         else rank[v] = (uint32_t)atom_add_keep(fill + bin, 1ull, pol_last);
       }
@@ -310,7 +306,7 @@ __global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint3
 #pragma unroll
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
-      const uint64_t* op = rec_off + (((rec[v][0].x >> 10) >> shift) << shift);
+      const uint64_t* op = rec_off + hdr_pid(rec[v][0].x);
       base[v] = idx < n ? ld_keep8(op, pol_last) : 0;
     }
     if (smem) {
@@ -323,11 +319,11 @@ __global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint3
     for (int v = 0; v < kPer; ++v) {
       const uint64_t idx = t0 + v * kScatterThreads + threadIdx.x;
       if (idx < n) {
-        const uint32_t bin = (rec[v][0].x >> 10) >> shift;
+        const uint32_t bin = hdr_pid(rec[v][0].x);
         const uint64_t pos = base[v] + (smem ? sh_base[bin] + rank[v] : rank[v]);
         uint32_t* out = records;
         if (n_peers) {  // multi-GPU emission: the owner's buffer, through its IPC-mapped pointer
-          const int32_t pid = (int32_t)(rec[v][0].x >> 10);
+          const int32_t pid = (int32_t)hdr_pid(rec[v][0].x);
           int o = 0;
           while (o + 1 < n_peers && pid >= __ldg(peer_bounds + o + 1)) ++o;
           out = peer_records[o];
@@ -341,68 +337,226 @@ __global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint3
   }
 }
 
-// Two-level scatter, level 2: one CTA per bucket of 2^shift consecutive
-// partitions (grid-stride over buckets).  The bucket's records are
-// contiguous in src (level 1); each is ranked inside its partition with a
-// shared-memory atomic and written to rec_off[pid] + rank in dst (or, with
-// peers, in the owner's buffer).  The bucket's output range is small (about
-// 2^shift x 190 records on chr14), so its 32-byte sectors are completed while
-// they are in L2 and written back whole.
-constexpr int kBucketThreads = 512;
-constexpr int kBucketPer = 4;
+// Two-level scatter (pass 3 with d_scratch): two counting-sort passes over tiles of records.
+// Level A ranks a tile of staged records by BUCKET (2^s consecutive fine partitions, <= 2048
+// buckets) in shared memory, reserves once per (tile, non-empty bucket) from a global bucket
+// cursor and writes the tile into the buckets' contiguous ranges of d_scratch (bucket b starts at
+// the local prefix of this rank's counts).  Level B takes tiles inside one bucket, ranks them by
+// partition in shared memory, reserves once per (tile, partition) from d_fill and writes each
+// record to d_record_offset[pid] + rank -- in d_records or the owner's buffer.  A record costs a
+// shared-memory atomic per level and ~0.1-0.4 global atomics, instead of one returning global
+// atomic in a dependent chain (the one-level scatter above, latency-bound at ~36 G records/s).
+constexpr int kTsThreads = 1024;
+constexpr int kTsMaxBins = 4096;  // bins of one tile pass (buckets in level A, partitions in level B)
 template <int R>
-__global__ void __launch_bounds__(kBucketThreads) bucket_scatter_kernel(const uint32_t* __restrict__ src,
-                                                                        const unsigned long long* staged,
-                                                                        uint64_t staging_cap,
-                                                                        const uint64_t* __restrict__ rec_off,
-                                                                        uint32_t* __restrict__ dst, int np, int shift,
-                                                                        uint32_t* const* peer_records,
-                                                                        const int32_t* peer_bounds, int n_peers) {
-  extern __shared__ unsigned long long sh_off[];  // [2^shift + 1] offsets, then [2^shift] counts
-  const int bw = 1 << shift;
-  uint32_t* sh_cnt = reinterpret_cast<uint32_t*>(sh_off + bw + 1);
-  if (*staged > staging_cap) return;
+__host__ __device__ constexpr int ts_per() { return R == 4 ? 6 : (R == 8 ? 3 : 1); }
+template <int R>
+__host__ __device__ constexpr int ts_tile() { return kTsThreads * ts_per<R>(); }  // <= 96 KB of records
+// log2 of the bucket width: the smallest s with <= 2048 buckets, at most 12 (4096 partitions a
+// bucket; <= 4096 buckets for the 2^24 - 1 fine partitions of dbg.h)
+__host__ __device__ inline int ts_shift(int np) {
+  int s = 0;
+  while (s < 12 && ((np + (1 << s) - 1) >> s) > 2048) ++s;
+  return s;
+}
+// d_work layout (uint64): fill[nb] | boff[nb + 1] | tiles[nb + 1]
+struct TsArgs {
+  const uint32_t* src;
+  uint32_t* dst;
+  const unsigned long long* staged;
+  uint64_t staging_cap;
+  unsigned long long* fill;  // level A: bucket cursors (work); level B: partition cursors (d_fill)
+  const uint64_t* boff;      // [nb + 1] local bucket offsets
+  const uint64_t* tiles;     // [nb + 1] level B tiles before bucket b
+  const uint64_t* rec_off;   // level B: d_record_offset (or the exchange plan's destinations)
+  int nb, s, np;
+  uint32_t* const* peer_records;
+  const int32_t* peer_bounds;
+  int n_peers;
+};
+
+// Per bucket: this rank's records in it (sum of d_n_records over its partitions).
+__global__ void __launch_bounds__(256) ts_bucket_count_kernel(const uint64_t* __restrict__ n_records, int np, int s,
+                                                             uint64_t* __restrict__ boff) {
+  typedef cub::BlockReduce<unsigned long long, 256> Red;
+  __shared__ typename Red::TempStorage tmp;
+  const int b = blockIdx.x, f0 = b << s, f1 = min(np, (b + 1) << s);
+  unsigned long long c = 0;
+  for (int f = f0 + threadIdx.x; f < f1; f += 256) c += n_records[f];
+  c = Red(tmp).Sum(c);
+  if (threadIdx.x == 0) boff[b] = c;
+}
+
+// boff: counts -> exclusive prefix (boff[nb] = total); tiles: exclusive prefix of ceil(count / tile);
+// fill = 0.  One CTA, nb <= 4096.
+__global__ void __launch_bounds__(1024) ts_bucket_scan_kernel(uint64_t* work, int nb, int tile) {
+  typedef cub::BlockScan<unsigned long long, 1024> Scan;
+  __shared__ typename Scan::TempStorage tmp;
+  unsigned long long* fill = reinterpret_cast<unsigned long long*>(work);
+  uint64_t* boff = work + nb;
+  uint64_t* tiles = boff + nb + 1;
+  unsigned long long c[4], t[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const int i = 4 * threadIdx.x + q;
+    c[q] = i < nb ? boff[i] : 0ull;
+    t[q] = (c[q] + tile - 1) / tile;
+    if (i < nb) fill[i] = 0;
+  }
+  unsigned long long ct, tt;
+  Scan(tmp).ExclusiveSum(c, c, ct);
+  __syncthreads();
+  Scan(tmp).ExclusiveSum(t, t, tt);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const int i = 4 * threadIdx.x + q;
+    if (i < nb) {
+      boff[i] = c[q];
+      tiles[i] = t[q];
+    }
+  }
+  if (threadIdx.x == 0) {
+    boff[nb] = ct;
+    tiles[nb] = tt;
+  }
+}
+
+// One tile [r0, r1) of a.src (a counting sort of the tile, onesweep-style): records ranked by bin
+// in shared memory, the tile's bin counts scanned (local offsets) and reserved once per non-empty
+// bin (base_of(bin, count)), the records placed in bin order in shared memory, then written out
+// by consecutive threads to consecutive slots of each bin's global range -- coalesced stores of
+// whole 32-byte sectors instead of one scattered 16-byte store per record.
+template <int R, class BinFn, class BaseFn, class DstFn>
+__device__ __forceinline__ void ts_tile_pass(const TsArgs& a, uint64_t r0, uint64_t r1, int nbins, uint32_t* srec,
+                                             unsigned long long* gbase, uint32_t* hist, uint32_t* lbase,
+                                             BinFn bin_of, BaseFn base_of, DstFn dst_of, uint64_t pol_first) {
+  constexpr int kPer = ts_per<R>(), kItems = kTsMaxBins / kTsThreads;
+  typedef cub::BlockScan<uint32_t, kTsThreads> Scan;
+  __shared__ typename Scan::TempStorage scan_tmp;
+  for (int i = threadIdx.x; i < nbins; i += kTsThreads) hist[i] = 0;
+  __syncthreads();
+  uint4 rec[kPer][R / 4];
+  uint32_t bin[kPer], rank[kPer];
+#pragma unroll
+  for (int v = 0; v < kPer; ++v) {
+    const uint64_t idx = r0 + (uint64_t)v * kTsThreads + threadIdx.x;
+    if (idx < r1) {
+      const uint4* s4 = reinterpret_cast<const uint4*>(a.src + idx * R);
+#pragma unroll
+      for (int c = 0; c < R / 4; ++c) rec[v][c] = ld_stream16(s4 + c, pol_first);
+    }
+  }
+#pragma unroll
+  for (int v = 0; v < kPer; ++v) {
+    const uint64_t idx = r0 + (uint64_t)v * kTsThreads + threadIdx.x;
+    if (idx < r1) {
+      bin[v] = bin_of(hdr_pid(rec[v][0].x));
+      rank[v] = atomicAdd(hist + bin[v], 1u);
+    }
+  }
+  __syncthreads();
+  {
+    uint32_t c[kItems], ex[kItems];
+#pragma unroll
+    for (int q = 0; q < kItems; ++q) {
+      const int i = kItems * threadIdx.x + q;
+      c[q] = i < nbins ? hist[i] : 0u;
+    }
+    Scan(scan_tmp).ExclusiveSum(c, ex);
+#pragma unroll
+    for (int q = 0; q < kItems; ++q) {
+      const int i = kItems * threadIdx.x + q;
+      if (i < nbins) {
+        lbase[i] = ex[q];
+        if (c[q]) gbase[i] = base_of(i, c[q]);
+      }
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int v = 0; v < kPer; ++v) {
+    const uint64_t idx = r0 + (uint64_t)v * kTsThreads + threadIdx.x;
+    if (idx < r1) {
+      uint4* d4 = reinterpret_cast<uint4*>(srec + (size_t)(lbase[bin[v]] + rank[v]) * R);
+#pragma unroll
+      for (int c = 0; c < R / 4; ++c) d4[c] = rec[v][c];
+    }
+  }
+  __syncthreads();
+  const uint32_t nt = (uint32_t)(r1 - r0);
+  for (uint32_t p = threadIdx.x; p < nt; p += kTsThreads) {
+    const uint4* sp = reinterpret_cast<const uint4*>(srec + (size_t)p * R);
+    const uint4 x0 = sp[0];
+    const uint32_t pid = hdr_pid(x0.x), b = bin_of(pid);
+    uint4* d4 = reinterpret_cast<uint4*>(dst_of(pid) + (gbase[b] + (p - lbase[b])) * R);
+    d4[0] = x0;
+#pragma unroll
+    for (int c = 1; c < R / 4; ++c) d4[c] = sp[c];
+  }
+  __syncthreads();
+}
+
+// Dynamic shared memory of a tile pass: records, then bases, counts and local offsets of nbins.
+template <int R>
+__host__ __device__ constexpr size_t ts_rec_bytes() { return (size_t)ts_tile<R>() * R * 4; }
+inline size_t ts_bin_bytes(int nbins) { return (size_t)nbins * (8 + 4 + 4); }
+
+template <int R>
+__global__ void __launch_bounds__(kTsThreads) ts_level_a_kernel(TsArgs a) {
+  extern __shared__ __align__(16) unsigned char ts_smem[];
+  uint32_t* srec = reinterpret_cast<uint32_t*>(ts_smem);
+  unsigned long long* gbase = reinterpret_cast<unsigned long long*>(ts_smem + ts_rec_bytes<R>());
+  uint32_t* hist = reinterpret_cast<uint32_t*>(gbase + a.nb);
+  uint32_t* lbase = hist + a.nb;
+  const uint64_t n = *a.staged;
+  if (n > a.staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
   const uint64_t pol_first = l2_policy_first();
-  const int nbk = (np + bw - 1) >> shift;
-  constexpr int kTile = kBucketThreads * kBucketPer;
-  for (int bk = blockIdx.x; bk < nbk; bk += gridDim.x) {
-    const int p0 = bk << shift, np_b = min(bw, np - p0);
-    for (int i = threadIdx.x; i <= np_b; i += kBucketThreads) {
-      sh_off[i] = rec_off[p0 + i];
-      if (i < np_b) sh_cnt[i] = 0;
+  constexpr int kTile = ts_tile<R>();
+  const int s = a.s;
+  for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile)
+    ts_tile_pass<R>(a, t0, min(n, t0 + kTile), a.nb, srec, gbase, hist, lbase,
+                    [s](uint32_t pid) { return pid >> s; },
+                    [&](int b, uint32_t c) { return a.boff[b] + atomicAdd(a.fill + b, (unsigned long long)c); },
+                    [&](uint32_t) { return a.dst; }, pol_first);
+}
+
+template <int R>
+__global__ void __launch_bounds__(kTsThreads) ts_level_b_kernel(TsArgs a) {
+  extern __shared__ __align__(16) unsigned char ts_smem[];
+  const int w = 1 << a.s;
+  uint32_t* srec = reinterpret_cast<uint32_t*>(ts_smem);
+  unsigned long long* gbase = reinterpret_cast<unsigned long long*>(ts_smem + ts_rec_bytes<R>());
+  unsigned long long* tiles = gbase + w;  // [nb + 1] tile prefix
+  uint32_t* hist = reinterpret_cast<uint32_t*>(tiles + a.nb + 1);
+  uint32_t* lbase = hist + w;
+  if (*a.staged > a.staging_cap) return;
+  for (int i = threadIdx.x; i <= a.nb; i += kTsThreads) tiles[i] = a.tiles[i];
+  __syncthreads();
+  const uint64_t pol_first = l2_policy_first();
+  constexpr int kTile = ts_tile<R>();
+  const uint64_t n_tiles = tiles[a.nb];
+  for (uint64_t g = blockIdx.x; g < n_tiles; g += gridDim.x) {
+    int b = 0, cnt = a.nb;  // the bucket of tile g: last b with tiles[b] <= g (shared-memory search)
+    while (cnt > 1) {
+      const int h = cnt >> 1;
+      if (tiles[b + h] <= g) b += h, cnt -= h;
+      else cnt = h;
     }
-    __syncthreads();
-    const uint64_t r0 = sh_off[0], r1 = sh_off[np_b];
-    for (uint64_t t0 = r0; t0 < r1; t0 += kTile) {
-      uint4 rec[kBucketPer][R / 4];
-#pragma unroll
-      for (int v = 0; v < kBucketPer; ++v) {
-        const uint64_t idx = t0 + v * kBucketThreads + threadIdx.x;
-        if (idx < r1) {
-          const uint4* s4 = reinterpret_cast<const uint4*>(src + idx * R);
-#pragma unroll
-          for (int c = 0; c < R / 4; ++c) rec[v][c] = ld_stream16(s4 + c, pol_first);
-        }
-      }
-#pragma unroll
-      for (int v = 0; v < kBucketPer; ++v) {
-        const uint64_t idx = t0 + v * kBucketThreads + threadIdx.x;
-        if (idx < r1) {
-          const uint32_t pid = rec[v][0].x >> 10, lp = pid - (uint32_t)p0;
-          const uint64_t pos = sh_off[lp] + atomicAdd(sh_cnt + lp, 1u);
-          uint32_t* out = dst;
-          if (n_peers) {  // multi-GPU emission: the owner's buffer, through its IPC-mapped pointer
-            int o = 0;
-            while (o + 1 < n_peers && (int32_t)pid >= __ldg(peer_bounds + o + 1)) ++o;
-            out = peer_records[o];
-          }
-          uint4* d4 = reinterpret_cast<uint4*>(out + pos * R);
-#pragma unroll
-          for (int c = 0; c < R / 4; ++c) d4[c] = rec[v][c];
-        }
-      }
-    }
-    __syncthreads();
+    const uint32_t f0 = (uint32_t)b << a.s;
+    const uint64_t r0 = a.boff[b] + (g - tiles[b]) * kTile, r1 = min(a.boff[b + 1], r0 + kTile);
+    const int nbins = min(w, a.np - (int)f0);
+    ts_tile_pass<R>(
+        a, r0, r1, nbins, srec, gbase, hist, lbase, [f0](uint32_t pid) { return pid - f0; },
+        [&](int i, uint32_t c) {
+          return a.rec_off[f0 + i] + atomicAdd(a.fill + f0 + i, (unsigned long long)c);
+        },
+        [&](uint32_t pid) -> uint32_t* {
+          if (!a.n_peers) return a.dst;  // multi-GPU emission: the owner's buffer, through its IPC pointer
+          int o = 0;
+          while (o + 1 < a.n_peers && (int32_t)pid >= __ldg(a.peer_bounds + o + 1)) ++o;
+          return a.peer_records[o];
+        },
+        pol_first);
   }
 }
 
@@ -671,49 +825,87 @@ static dbg_status msp_partition(const dbg_params* prm, const uint64_t* d_bases, 
     if (part->n_peers < 0 ||
         (part->n_peers > 0 && (!part->d_peer_records || !part->d_peer_bounds)))
       return DBG_EINVAL;
-    // Above kSmemHistMaxNp fine partitions a one-level scatter writes every 16-byte record to a
-    // random place of a multi-GB output: each store is a DRAM read-modify-write of its sector
-    // (chr14: 14 ms for 295 M records, ~1.85 TB/s of random sector traffic; tools/scatter_probe.py).
-    // With d_scratch the records go in two levels instead: level 1 into buckets of
-    // 2^kBucketShift consecutive partitions (bucket cursors advance sequentially; the buckets'
-    // open sectors fit L2), level 2 per bucket inside its small output range.
-    const bool two = part->d_scratch && np > kSmemHistMaxNp;
-    const int shift = two ? kBucketShift : 0;
-    const int nb = (np + (1 << shift) - 1) >> shift;
-    if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * nb, stream) != cudaSuccess) return DBG_ECUDA;
-    const size_t smem = nb <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * nb : 0;
-    // one full wave: the kernel is grid-stride, a partial second wave would idle SMs
-    auto scatter_grid = [&](const void* fn) {
-      int per_sm = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kScatterThreads, smem) != cudaSuccess ||
-          per_sm < 1)
-        per_sm = 4;
-      return dbg_sm_count() * per_sm;
-    };
-    uint32_t* lvl1 = two ? part->d_scratch : part->d_records;
+    // Above kSmemHistMaxNp fine partitions a one-level scatter writes every record to a random
+    // place of a multi-GB output with one returning global atomic each (chr14: ~36 G records/s,
+    // latency-bound); with d_scratch and d_work the records go in two counting-sort levels
+    // (ts_level_a/b_kernel).
+    const bool two = part->d_scratch && part->d_work && np > kSmemHistMaxNp;
+    if (part->d_scratch && !part->d_work && np > kSmemHistMaxNp) return DBG_EINVAL;
+    if (cudaMemsetAsync(part->d_fill, 0, sizeof(uint64_t) * np, stream) != cudaSuccess) return DBG_ECUDA;
     const unsigned long long* staged = reinterpret_cast<const unsigned long long*>(part->d_staged);
     unsigned long long* fill = reinterpret_cast<unsigned long long*>(part->d_fill);
-    const size_t smem2 = (sizeof(unsigned long long) * ((1u << shift) + 1) + sizeof(uint32_t) * (1u << shift));
-    const int grid2 = (int)std::min<int64_t>((int64_t)nb, (int64_t)dbg_sm_count() * 4);
+    if (!two) {
+      const size_t smem = np <= kSmemHistMaxNp ? (sizeof(unsigned long long) + sizeof(uint32_t)) * np : 0;
+      // one full wave: the kernel is grid-stride, a partial second wave would idle SMs
+      auto scatter_grid = [&](const void* fn) {
+        int per_sm = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kScatterThreads, smem) != cudaSuccess ||
+            per_sm < 1)
+          per_sm = 4;
+        return dbg_sm_count() * per_sm;
+      };
 #define DBG_SCATTER(RW)                                                                                         \
   cudaFuncSetAttribute(scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
   scatter_kernel<RW><<<scatter_grid((const void*)scatter_kernel<RW>), kScatterThreads, smem, stream>>>(        \
-      part->d_staging, staged, part->staging_cap, part->d_record_offset, fill, lvl1, nb, shift,                 \
-      two ? nullptr : part->d_peer_records, part->d_peer_bounds, two ? 0 : part->n_peers);                      \
-  if (two) {                                                                                                    \
-    cudaFuncSetAttribute(bucket_scatter_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);   \
-    bucket_scatter_kernel<RW><<<grid2, kBucketThreads, smem2, stream>>>(                                       \
-        part->d_scratch, staged, part->staging_cap, part->d_record_offset, part->d_records, np, shift,         \
-        part->d_peer_records, part->d_peer_bounds, part->n_peers);                                             \
-  }
-    if (R == 4) {
-      DBG_SCATTER(4)
-    } else if (R == 8) {
-      DBG_SCATTER(8)
-    } else {
-      DBG_SCATTER(16)
-    }
+      part->d_staging, staged, part->staging_cap, part->d_record_offset, fill, part->d_records, np,             \
+      part->d_peer_records, part->d_peer_bounds, part->n_peers);
+      if (R == 4) {
+        DBG_SCATTER(4)
+      } else if (R == 8) {
+        DBG_SCATTER(8)
+      } else {
+        DBG_SCATTER(16)
+      }
 #undef DBG_SCATTER
+    } else {
+      const int s = ts_shift(np), nb = (np + (1 << s) - 1) >> s;
+      TsArgs ta;
+      ta.staged = staged;
+      ta.staging_cap = part->staging_cap;
+      ta.boff = part->d_work + nb;
+      ta.tiles = part->d_work + 2 * nb + 1;
+      ta.rec_off = part->d_record_offset;
+      ta.nb = nb;
+      ta.s = s;
+      ta.np = np;
+      ta.peer_records = part->d_peer_records;
+      ta.peer_bounds = part->d_peer_bounds;
+      ta.n_peers = part->n_peers;
+      const int tile = R == 4 ? ts_tile<4>() : (R == 8 ? ts_tile<8>() : ts_tile<16>());
+      ts_bucket_count_kernel<<<nb, 256, 0, stream>>>(part->d_n_records, np, s, part->d_work + nb);
+      ts_bucket_scan_kernel<<<1, 1024, 0, stream>>>(part->d_work, nb, tile);
+      const size_t rec_bytes = R == 4 ? ts_rec_bytes<4>() : (R == 8 ? ts_rec_bytes<8>() : ts_rec_bytes<16>());
+      const size_t smem_a = rec_bytes + ts_bin_bytes(nb);
+      const size_t smem_b = rec_bytes + ts_bin_bytes(1 << s) + sizeof(unsigned long long) * (nb + 1);
+      auto ts_grid = [&](const void* fn, size_t smem) {
+        int per_sm = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kTsThreads, smem) != cudaSuccess || per_sm < 1)
+          per_sm = 1;
+        return dbg_sm_count() * per_sm;
+      };
+#define DBG_TS(RW)                                                                                              \
+  {                                                                                                             \
+    TsArgs x = ta;                                                                                              \
+    x.src = part->d_staging;                                                                                    \
+    x.dst = part->d_scratch;                                                                                    \
+    x.fill = reinterpret_cast<unsigned long long*>(part->d_work);                                               \
+    cudaFuncSetAttribute(ts_level_a_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_a);     \
+    ts_level_a_kernel<RW><<<ts_grid((const void*)ts_level_a_kernel<RW>, smem_a), kTsThreads, smem_a, stream>>>(x); \
+    x.src = part->d_scratch;                                                                                    \
+    x.dst = part->d_records;                                                                                    \
+    x.fill = fill;                                                                                              \
+    cudaFuncSetAttribute(ts_level_b_kernel<RW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_b);     \
+    ts_level_b_kernel<RW><<<ts_grid((const void*)ts_level_b_kernel<RW>, smem_b), kTsThreads, smem_b, stream>>>(x); \
+  }
+      if (R == 4) {
+        DBG_TS(4)
+      } else if (R == 8) {
+        DBG_TS(8)
+      } else {
+        DBG_TS(16)
+      }
+#undef DBG_TS
+    }
   }
   return cudaPeekAtLastError() == cudaSuccess ? DBG_OK : DBG_ECUDA;
 }

@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(kWarpMspThreads, 3) msp_warp_kernel(MspArgs a)
   const CT maskP = (CT)((2 * P == 8 * (int)sizeof(CT)) ? ~(CT)0 : (((CT)1 << (2 * P)) - 1));
   const int cap = 32 * R - w + 1;  // K-mers per piece (the launcher checks w <= 32R)
   const bool two_win = P + R - 1 > 32;
-  const int nmax = KC ? (int)(16u * (record_words(KC) - 1u) - (uint32_t)KC - 1u) : (int)a.max_kmers;
+  const int nmax = KC ? (int)record_max_kmers(KC) : (int)a.max_kmers;
   const uint32_t rw = KC ? record_words(KC) : a.rec_words;
   // lanes l + 1 .. l + D (D = d - 1 <= Dmax) from a sparse table of lane minima
   const int Dmax = (R - 1 + w - 1) / R - 1;
@@ -211,7 +211,7 @@ __global__ void __launch_bounds__(kWarpMspThreads, 3) msp_warp_kernel(MspArgs a)
             const int nb = (int)hl + (pe - ps + 1) + K - 1 + (int)hr;
             const uint64_t pos = o + (uint64_t)(ps - (int)hl);
             uint4* d4 = reinterpret_cast<uint4*>(a.staging + slot * rw);
-            const uint32_t hdr = (uint32_t)(pe - ps + 1) | (hl << 8) | (hr << 9) | (pid << 10);
+            const uint32_t hdr = rec_header((uint32_t)(pe - ps + 1), hl, hr, pid);
             // data word q (1 .. rw-1) holds bases 16(q-1) .. 16q-1: 32-base window u = (q-1)/2,
             // high half for odd q
             for (int c4 = 0; c4 < (int)rw / 4; ++c4) {

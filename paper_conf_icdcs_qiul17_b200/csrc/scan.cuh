@@ -1,10 +1,10 @@
 // scan.cuh -- exclusive prefix sums over the fine partitions, multi-CTA.
 //
 // The per-partition arrays (records, K-mers, table capacities; PAPER.md
-// Sec. IV-A P:L783-788 sizes the tables from them) have up to 4,194,303
+// Sec. IV-A P:L783-788 sizes the tables from them) have up to 16,777,215
 // entries, far more than one CTA scans quickly, so the sums run in three
 // launches: per-tile totals (one CTA per 4096 entries), one CTA scanning the
-// <= 1024 tile totals in place, and per-tile block scans offset by their
+// <= 4096 tile totals in place, and per-tile block scans offset by their
 // tile's prefix.  Small arrays take one single-CTA launch instead.
 #pragma once
 #include <cub/block/block_reduce.cuh>
@@ -17,7 +17,7 @@
 namespace dbg {
 
 constexpr int kTileThreads = 512, kTileItems = 8, kTileSize = kTileThreads * kTileItems;
-constexpr int kTileScanThreads = 1024, kTileScanItems = 4;  // <= 4096 tiles: NP*refine <= 4,194,303
+constexpr int kTileScanThreads = 1024, kTileScanItems = 4;  // <= 4096 tiles of 4096: NP*refine <= 2^24 - 1
 constexpr int kSingleCtaMax = 4 * kTileSize;                 // one launch up to this many entries
 
 __host__ __device__ inline int scan_tiles(int n) { return (n + kTileSize - 1) / kTileSize; }

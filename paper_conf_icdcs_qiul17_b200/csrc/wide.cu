@@ -142,8 +142,8 @@ __global__ void __launch_bounds__(kWideThreads) wide_hash_kernel(WideArgs a) {
        r += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t* w = a.records + r * R;
     const uint32_t w0 = w[0];
-    const int n = w0 & 255u, hl = (w0 >> 8) & 1u, hr = (w0 >> 9) & 1u;
-    const uint32_t pid = w0 >> 10;
+    const int n = hdr_n(w0), hl = hdr_hl(w0), hr = hdr_hr(w0);
+    const uint32_t pid = hdr_pid(w0);
     const uint64_t t0 = __ldg(a.tab_off + pid) - s0, cap = __ldg(a.tab_off + pid + 1) - __ldg(a.tab_off + pid);
     auto base = [&](int q) { return (__ldg(w + 1 + (q >> 4)) >> (30 - 2 * (q & 15))) & 3u; };
     W4 fwd = {{0, 0, 0, 0}}, rc = {{0, 0, 0, 0}};

@@ -29,6 +29,9 @@ import torch
 from . import _lib
 from ._lib import VERTEX_DTYPE, VERTEX_WIDE_DTYPE, STATS_FIELDS
 
+# dbg.h: NP * refine <= 2^24 - 1 (the fine pid field of the record header)
+MAX_FINE_PARTITIONS = (1 << 24) - 1
+
 
 def encode_reads(seq: np.ndarray, pin: bool = False) -> torch.Tensor:
     """Row a0: ASCII reads (concatenated) -> packed 2-bit words (uint64 as int64 tensor)."""
@@ -110,13 +113,16 @@ class DbgBuilder:
         self.d_stats = torch.zeros(4, **i64)
         self.staging = torch.empty(0, dtype=torch.int32, device=dev)
         self.records = torch.empty(0, dtype=torch.int32, device=dev)
-        # two-level scatter (pass 2) through a third record buffer (dbg_partition_set.d_scratch;
-        # msp.cu): it pays only where one level's random 16-byte record stores miss L2 -- 4-word
-        # records and a staging far larger than L2 (chr14: 14.1 -> 12.2 ms); E. coli (0.35 GB of
-        # records: 0.52 -> 1.25 ms) and 32-byte records (bumblebee: 20.1 -> 23.6 ms) lose (r02f)
+        # two-level counting-sort scatter (pass 2) through a third record buffer
+        # (dbg_partition_set.d_scratch + d_work; msp.cu ts_level_a/b): above 8192 fine partitions
+        # the one-level scatter pays one returning global atomic per record; with a staging
+        # beyond L2 two levels win (r02z1: chr14 8.82 vs 14.14 ms, bumblebee 17.61 vs 19.61 ms),
+        # on E. coli's 0.35 GB they lose (0.65 vs 0.51 ms)
         self.scratch = torch.empty(0, dtype=torch.int32, device=dev)
+        self.scatter_work = torch.zeros(_lib.dbg_scatter_work_words(self.prm), **i64)
         self.two_level = NP > 8192
         self.two_level_min_bytes = 2 << 30
+        self.two_level_words = (4, 8, 16)  # record widths that take it
         self.table = torch.empty(0, dtype=torch.uint8, device=dev)
         self.work = torch.empty(0, dtype=torch.uint8, device=dev)
         self.out = torch.empty(0, dtype=torch.uint8, device=dev)
@@ -171,10 +177,12 @@ class DbgBuilder:
             scratch = self.scratch
         cap = self.staging.numel() // self.rec_words
         return _lib.partition_set(self.d_n_records, self.d_n_kmers, self.d_rec_off, self.d_fill, self.d_staged,
-                                  self.staging, cap, self.records if with_records else None, scratch)
+                                  self.staging, cap, self.records if with_records else None, scratch,
+                                  work=self.scatter_work if scratch is not None else None)
 
     def use_two_level(self) -> bool:
-        return self.two_level and self.rec_words == 4 and self.staging.numel() * 4 >= self.two_level_min_bytes
+        return (self.two_level and self.rec_words in self.two_level_words
+                and self.staging.numel() * 4 >= self.two_level_min_bytes)
 
     def _staging_estimate(self, n_kmers_upper: int, n_reads: int) -> int:
         w = self.k - self.p + 1
@@ -512,7 +520,7 @@ def auto_refine(n_kmers: int, k: int, p: int, num_partitions: int, lam: float = 
     slots = _lib.dbg_smem_table_slots(prm)
     per_part = max(1.0, fill * slots / max(lam / (4 * alpha), 1e-9))
     f = max(1, int(np.ceil(n_kmers / (num_partitions * per_part))))
-    return max(1, min(f, 4_194_303 // num_partitions))
+    return max(1, min(f, MAX_FINE_PARTITIONS // num_partitions))
 
 
 def auto_fine_p(n_kmers: int, k: int, p: int, lam: float = 2.0, alpha: float = 0.5) -> int:

@@ -218,7 +218,7 @@ class ShardedBuilder:
             scratch = s.scratch
         part = _lib.partition_set(s.d_n_records, s.d_n_kmers, self.d_dest, s.d_fill, s.d_staged, s.staging,
                                   s.staging.numel() // R, d.records, scratch, self.d_ptrs, self.d_bounds,
-                                  self.world)
+                                  self.world, work=s.scatter_work if scratch is not None else None)
         ev = s._mark("msp_scatter", stream)
         _lib.dbg_msp_partition(s.prm, d_bases, d_bases.numel(), d_offsets, d_offsets.numel() - 1, part, stream)
         s._done(ev, stream)

@@ -23,7 +23,7 @@ def decode_records(words: np.ndarray, rec_words: int, k: int):
     out = []
     for row in w:
         hdr = int(row[0])
-        n, hl, hr, pid = hdr & 255, (hdr >> 8) & 1, (hdr >> 9) & 1, hdr >> 10
+        n, hl, hr, pid = hdr & 63, (hdr >> 6) & 1, (hdr >> 7) & 1, hdr >> 8
         nb = hl + n + k - 1 + hr
         bases = []
         for i in range(nb):

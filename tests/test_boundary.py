@@ -36,7 +36,7 @@ def test_exports_every_declared_symbol(lib):
 
 
 def test_abi_and_sizes(lib):
-    assert lib.dbg_abi_version() == 11
+    assert lib.dbg_abi_version() == 12
     p31 = lib.params(31, 11, 16)
     p63 = lib.params(63, 19, 16)
     assert lib.dbg_record_words(p31) == 4 and lib.dbg_record_max_kmers(p31) == 16
@@ -44,6 +44,14 @@ def test_abi_and_sizes(lib):
     assert lib.dbg_slot_bytes(p31) == 48 and lib.dbg_key_bytes(p31) == 16
     assert lib.dbg_slot_bytes(p63) == 64 and lib.dbg_key_bytes(p63) == 32
     assert lib.dbg_packed_words(0) == 1 and lib.dbg_packed_words(32) == 2 and lib.dbg_packed_words(33) == 3
+    # the record header's 6-bit K-mer count caps long records at 63 K-mers (dbg.h)
+    assert lib.dbg_record_words(lib.params(41, 11, 16)) == 8 and lib.dbg_record_max_kmers(lib.params(41, 11, 16)) == 63
+    assert lib.dbg_record_words(lib.params(65, 11, 16)) == 16 and lib.dbg_record_max_kmers(lib.params(65, 11, 16)) == 63
+    # fine partitions: NP * refine <= 2^24 - 1 (the header's 24-bit pid field); whole human (65.1 G
+    # K-mers, NP = 960) wants ~39 M and is clamped there
+    from paper_conf_icdcs_qiul17_b200.graph import MAX_FINE_PARTITIONS, auto_refine
+    assert MAX_FINE_PARTITIONS == (1 << 24) - 1
+    assert auto_refine(65_100_000_000, 31, 11, 960) == MAX_FINE_PARTITIONS // 960
 
 
 def test_table2_sizing_pin(lib):
@@ -146,7 +154,7 @@ def test_invalid_arguments_return_before_launch(lib):
     assert lib.dbg_status_string(lib.DBG_ETABLEFULL).startswith("hash table full")
     # row f3: K > 63 runs through the resident tables only
     p65 = lib.params(65, 21, 4)
-    assert lib.dbg_record_words(p65) == 16 and lib.dbg_record_max_kmers(p65) == 240 - 65 - 1
+    assert lib.dbg_record_words(p65) == 16 and lib.dbg_record_max_kmers(p65) == 63  # 6-bit header count
     assert lib.dbg_key_bytes(p65) == 48 and lib.dbg_slot_bytes(p65) == 80
     assert lib.dbg_smem_onchip(p65, 100) == 0 and lib.dbg_smem_table_slots(p65) == 0
     with pytest.raises(DbgError) as e:

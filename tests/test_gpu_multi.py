@@ -47,7 +47,7 @@ def _reads(n=20_000, seed=9):
     return ReadSet(seq, offs)
 
 
-def _rank(rank, world, port, k, p, np_, refine, n_reads, q):
+def _rank(rank, world, port, k, p, np_, refine, n_reads, q, two_level=False):
     sys.path.insert(0, ROOT)
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     import torch.distributed as dist
@@ -61,6 +61,9 @@ def _rank(rank, world, port, k, p, np_, refine, n_reads, q):
     total = rs.n_kmers(k)
     mine = rs.subset(n_reads * rank // world, n_reads * (rank + 1) // world)
     sb = ShardedBuilder(k, p, np_, total, "cuda:0", refine=refine)
+    if two_level:  # pass 2 through the two-level scatter at this size: buckets locally, then the peers
+        sb.src.two_level_min_bytes, sb.src.two_level_words = 0, (4, 8, 16)
+        assert sb.src.use_two_level() or sb.src.staging.numel() == 0
     d_bases, d_off = sb.src.upload(encode_reads(mine.seq), mine.offsets)
     stream = torch.cuda.current_stream()
     outs = []
@@ -73,15 +76,17 @@ def _rank(rank, world, port, k, p, np_, refine, n_reads, q):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("k,p,np_,refine", [(31, 11, 16, 64), (63, 19, 8, 16)])
-def test_sharded_builder_two_ranks_one_gpu_equals_oracle(k, p, np_, refine):
+@pytest.mark.parametrize("k,p,np_,refine,two_level", [(31, 11, 16, 64, False), (63, 19, 8, 16, False),
+                                                      (31, 11, 16, 1024, True), (63, 19, 8, 2048, True)])
+def test_sharded_builder_two_ranks_one_gpu_equals_oracle(k, p, np_, refine, two_level):
     import torch.multiprocessing as mp
 
     world, n_reads = 2, 20_000
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank, args=(r, world, port, k, p, np_, refine, n_reads, q)) for r in range(world)]
+    procs = [ctx.Process(target=_rank, args=(r, world, port, k, p, np_, refine, n_reads, q, two_level))
+             for r in range(world)]
     for pr in procs:
         pr.start()
     res = dict(q.get(timeout=600) for _ in range(world))

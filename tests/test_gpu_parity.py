@@ -340,20 +340,22 @@ def test_register_blocked_msp_variants(p):
     assert got == occurrences_from_oracle_msp(sk, rs.reads(), 31)
 
 
-@pytest.mark.parametrize("refine", [1024, 4096, 40000])
-def test_two_level_scatter_partition_order(refine):
-    """More than 8192 fine partitions: pass 2 scatters through d_scratch in two levels (buckets of
-    16 consecutive partitions, then within each bucket).  Every record must land in its own
+@pytest.mark.parametrize("k,p,refine", [(31, 11, 1024), (31, 11, 4096), (31, 11, 40000), (31, 11, 1_000_000),
+                                         (63, 19, 4096), (63, 19, 300_000)])
+def test_two_level_scatter_partition_order(k, p, refine):
+    """More than 8192 fine partitions: pass 2 scatters through d_scratch in two counting-sort
+    levels (buckets of 2^s consecutive partitions, <= 2048 buckets; then partitions inside a
+    bucket, up to 8192 per bucket at 16 M fine partitions).  Every record must land in its own
     partition's range [rec_off[p], rec_off[p+1]), the per-partition record multisets must equal the
     one-level scatter's, and the graph must equal the oracle's."""
     rs = ReadSet(*make_reads(genome(60_000, 5), 6000, 100, 0.01, 105))
     np_ = 16
 
     def records(two):
-        b = DbgBuilder(31, 11, np_, refine=refine)
+        b = DbgBuilder(k, p, np_, refine=refine)
         assert b.two_level
         b.two_level = two
-        b.two_level_min_bytes = 0  # at every size here
+        b.two_level_min_bytes, b.two_level_words = 0, (4, 8, 16)  # at every size here
         d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
         b.msp(d_bases, d_off)
         assert b.sync_sizes()
@@ -361,7 +363,7 @@ def test_two_level_scatter_partition_order(refine):
         n = int(b.part_records.sum())
         w = b.records[:n * b.rec_words].cpu().numpy().view(np.uint32).reshape(n, b.rec_words)
         off = np.concatenate([[0], np.cumsum(b.part_records)])
-        pid = w[:, 0] >> 10
+        pid = w[:, 0] >> 8
         assert np.array_equal(pid, np.repeat(np.arange(len(b.part_records)), b.part_records))
         rows = [tuple(r) for r in w]
         return off, sorted(rows)
@@ -371,11 +373,11 @@ def test_two_level_scatter_partition_order(refine):
     assert np.array_equal(off1, off2)
     assert rows1 == rows2
     # and the graph through the two-level path
-    b = DbgBuilder(31, 11, np_, refine=refine)
-    b.two_level_min_bytes = 0
+    b = DbgBuilder(k, p, np_, refine=refine)
+    b.two_level_min_bytes, b.two_level_words = 0, (4, 8, 16)
     d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
     res = b.build(d_bases, d_off)
-    compare_vertices(res.vertices, oracle.graph(rs.seq, rs.offsets, 31, 11, np_, n_threads=NT))
+    compare_vertices(res.vertices, oracle.graph(rs.seq, rs.offsets, k, p, np_, n_threads=NT))
 
 
 @pytest.mark.parametrize("k,p", [(63, 19), (21, 7), (45, 30)])
@@ -416,3 +418,13 @@ def test_warp_msp_chunks_pieces_and_fallback(k, p):
     words = b.records[:n * b.rec_words].cpu().numpy().view(np.uint32)
     assert occurrences_from_records(decode_records(words, b.rec_words, k), k) == \
         occurrences_from_oracle_msp(sk, rs.reads(), k)
+
+
+@pytest.mark.parametrize("k,p,np_,refine", [(31, 13, 16, 300_000), (63, 19, 7, 2_396_745)])
+def test_fine_pids_beyond_22_bits(k, p, np_, refine):
+    """dbg.h: the record header's 24-bit fine pid -- NP * refine above 2^22 (4.8 M and 16.8 M - 1
+    fine partitions, almost all empty): multi-tile scans, the on-chip plan over millions of
+    partitions, the two-level scatter, and the paper's pid (fine pid mod NP) of every vertex."""
+    g = genome(30_000, seed=k + 1)
+    seq, offs = make_reads(g, 3000, 120, 0.01, seed=k + 2)
+    _check(ReadSet(seq, offs), k, p, np_, refine=refine)

@@ -2,7 +2,7 @@
 # Round-closing measurements: build + smoke, every GPU test, bench lines (chr14 with cpu_baseline,
 # bumblebee, E. coli, the reference arm), the chr14 launch list, ncu full captures of the step's
 # kernels (chr14, bumblebee), compute-sanitizer over every tier.   tools/gpu_final.sh TAG
-T=${1:-r02n}
+T=${1:-r02z}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/${T}_smoke.log 2>&1; echo smoke=$?; tail -1 gpurun_out/${T}_smoke.log
 timeout 2400 python -m pytest tests -m gpu -q --durations=15 > gpurun_out/${T}_pytest.log 2>&1; echo pytest=$?; tail -3 gpurun_out/${T}_pytest.log
@@ -16,7 +16,7 @@ for k in smem_subgraph msp_block scatter_kernel bucket_scatter; do
   timeout 1200 ncu --set full --import-source on --clock-control none -k regex:$k -s 3 -c 1 -o gpurun_out/${T}_chr14_$k -f \
     python bench.py --steps 1 --warmup 3 --no-cpu-baseline > gpurun_out/${T}_ncu_chr14_$k.log 2>&1; echo "ncu chr14 $k=$?"
 done
-for k in smem_subgraph msp_kernel; do
+for k in smem_subgraph msp_warp; do
   timeout 1500 ncu --set full --import-source on --clock-control none -k regex:$k -s 3 -c 1 -o gpurun_out/${T}_bbee_$k -f \
     python bench.py --config bumblebee --steps 1 --warmup 3 --no-cpu-baseline > gpurun_out/${T}_ncu_bbee_$k.log 2>&1; echo "ncu bbee $k=$?"
 done
