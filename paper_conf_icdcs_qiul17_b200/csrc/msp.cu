@@ -349,9 +349,9 @@ __global__ void __launch_bounds__(kScatterThreads, 4) scatter_kernel(const uint3
 constexpr int kTsThreads = 1024;
 constexpr int kTsMaxBins = 4096;  // bins of one tile pass (buckets in level A, partitions in level B)
 template <int R>
-__host__ __device__ constexpr int ts_per() { return R == 4 ? 6 : (R == 8 ? 3 : 1); }
+__host__ __device__ constexpr int ts_per() { return R == 4 ? 8 : (R == 8 ? 4 : 1); }
 template <int R>
-__host__ __device__ constexpr int ts_tile() { return kTsThreads * ts_per<R>(); }  // <= 96 KB of records
+__host__ __device__ constexpr int ts_tile() { return kTsThreads * ts_per<R>(); }  // <= 128 KB of records
 // log2 of the bucket width: the smallest s with <= 2048 buckets, at most 12 (4096 partitions a
 // bucket; <= 4096 buckets for the 2^24 - 1 fine partitions of dbg.h)
 __host__ __device__ inline int ts_shift(int np) {
@@ -496,10 +496,11 @@ __device__ __forceinline__ void ts_tile_pass(const TsArgs& a, uint64_t r0, uint6
   __syncthreads();
 }
 
-// Dynamic shared memory of a tile pass: records, then bases, counts and local offsets of nbins.
+// Dynamic shared memory of a tile pass: records, then the bases and the counts (overwritten in
+// place by their local offsets) of nbins.
 template <int R>
 __host__ __device__ constexpr size_t ts_rec_bytes() { return (size_t)ts_tile<R>() * R * 4; }
-inline size_t ts_bin_bytes(int nbins) { return (size_t)nbins * (8 + 4 + 4); }
+inline size_t ts_bin_bytes(int nbins) { return (size_t)nbins * (8 + 4); }
 
 template <int R>
 __global__ void __launch_bounds__(kTsThreads) ts_level_a_kernel(TsArgs a) {
@@ -507,17 +508,17 @@ __global__ void __launch_bounds__(kTsThreads) ts_level_a_kernel(TsArgs a) {
   uint32_t* srec = reinterpret_cast<uint32_t*>(ts_smem);
   unsigned long long* gbase = reinterpret_cast<unsigned long long*>(ts_smem + ts_rec_bytes<R>());
   uint32_t* hist = reinterpret_cast<uint32_t*>(gbase + a.nb);
-  uint32_t* lbase = hist + a.nb;
+  uint32_t* lbase = hist;  // each thread reads its counts before writing their offsets
   const uint64_t n = *a.staged;
   if (n > a.staging_cap) return;  // pass 1 overflowed the staging: the caller repeats it (dbg.h)
-  const uint64_t pol_first = l2_policy_first();
   constexpr int kTile = ts_tile<R>();
   const int s = a.s;
+  auto bin_of = [s](uint32_t pid) { return pid >> s; };
+  auto base_of = [&](int b, uint32_t c) { return a.boff[b] + atomicAdd(a.fill + b, (unsigned long long)c); };
+  auto dst_of = [&](uint32_t) { return a.dst; };
+  const uint64_t pol_first = l2_policy_first();
   for (uint64_t t0 = (uint64_t)blockIdx.x * kTile; t0 < n; t0 += (uint64_t)gridDim.x * kTile)
-    ts_tile_pass<R>(a, t0, min(n, t0 + kTile), a.nb, srec, gbase, hist, lbase,
-                    [s](uint32_t pid) { return pid >> s; },
-                    [&](int b, uint32_t c) { return a.boff[b] + atomicAdd(a.fill + b, (unsigned long long)c); },
-                    [&](uint32_t) { return a.dst; }, pol_first);
+    ts_tile_pass<R>(a, t0, min(n, t0 + kTile), a.nb, srec, gbase, hist, lbase, bin_of, base_of, dst_of, pol_first);
 }
 
 template <int R>
@@ -528,11 +529,11 @@ __global__ void __launch_bounds__(kTsThreads) ts_level_b_kernel(TsArgs a) {
   unsigned long long* gbase = reinterpret_cast<unsigned long long*>(ts_smem + ts_rec_bytes<R>());
   unsigned long long* tiles = gbase + w;  // [nb + 1] tile prefix
   uint32_t* hist = reinterpret_cast<uint32_t*>(tiles + a.nb + 1);
-  uint32_t* lbase = hist + w;
+  uint32_t* lbase = hist;  // each thread reads its counts before writing their offsets
   if (*a.staged > a.staging_cap) return;
   for (int i = threadIdx.x; i <= a.nb; i += kTsThreads) tiles[i] = a.tiles[i];
-  __syncthreads();
   const uint64_t pol_first = l2_policy_first();
+  __syncthreads();
   constexpr int kTile = ts_tile<R>();
   const uint64_t n_tiles = tiles[a.nb];
   for (uint64_t g = blockIdx.x; g < n_tiles; g += gridDim.x) {
@@ -545,18 +546,17 @@ __global__ void __launch_bounds__(kTsThreads) ts_level_b_kernel(TsArgs a) {
     const uint32_t f0 = (uint32_t)b << a.s;
     const uint64_t r0 = a.boff[b] + (g - tiles[b]) * kTile, r1 = min(a.boff[b + 1], r0 + kTile);
     const int nbins = min(w, a.np - (int)f0);
-    ts_tile_pass<R>(
-        a, r0, r1, nbins, srec, gbase, hist, lbase, [f0](uint32_t pid) { return pid - f0; },
-        [&](int i, uint32_t c) {
-          return a.rec_off[f0 + i] + atomicAdd(a.fill + f0 + i, (unsigned long long)c);
-        },
-        [&](uint32_t pid) -> uint32_t* {
-          if (!a.n_peers) return a.dst;  // multi-GPU emission: the owner's buffer, through its IPC pointer
-          int o = 0;
-          while (o + 1 < a.n_peers && (int32_t)pid >= __ldg(a.peer_bounds + o + 1)) ++o;
-          return a.peer_records[o];
-        },
-        pol_first);
+    auto bin_of = [f0](uint32_t pid) { return pid - f0; };
+    auto base_of = [&](int i, uint32_t c) {
+      return a.rec_off[f0 + i] + atomicAdd(a.fill + f0 + i, (unsigned long long)c);
+    };
+    auto dst_of = [&](uint32_t pid) -> uint32_t* {
+      if (!a.n_peers) return a.dst;  // multi-GPU emission: the owner's buffer, through its IPC pointer
+      int o = 0;
+      while (o + 1 < a.n_peers && (int32_t)pid >= __ldg(a.peer_bounds + o + 1)) ++o;
+      return a.peer_records[o];
+    };
+    ts_tile_pass<R>(a, r0, r1, nbins, srec, gbase, hist, lbase, bin_of, base_of, dst_of, pol_first);
   }
 }
 

@@ -44,29 +44,6 @@ struct alignas(16) WarpMspSmem {  // one warp's shared memory
   uint8_t dt[DESC];             // its read within the chunk
 };
 
-__device__ __forceinline__ void mbar_init(uint64_t* m, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sh_addr(m)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_tx(uint64_t* m, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sh_addr(m)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* m) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sh_addr(m)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* m, uint32_t parity) {
-  uint32_t done;
-  do {
-    asm volatile(
-        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
-        : "=r"(done) : "r"(sh_addr(m)), "r"(parity) : "memory");
-  } while (!done);
-}
-// 1-D TMA: bytes (multiple of 16) from global src (16-byte aligned) into shared dst.
-__device__ __forceinline__ void tma_bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* m) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               ::"r"(sh_addr(dst)), "l"(src), "r"(bytes), "r"(sh_addr(m)) : "memory");
-}
-
 // Reverse complement of all 32 bases of a 64-bit window (reading A: complement = 3 - c).
 __device__ __forceinline__ uint64_t revcomp32(uint64_t x) {
   const uint64_t y = __brevll(~x);

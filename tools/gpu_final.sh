@@ -12,7 +12,7 @@ timeout 600 python bench.py --config ecoli --no-cpu-baseline > gpurun_out/${T}_b
 timeout 900 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/${T}_reference.json 2> gpurun_out/${T}_reference.err; echo ref=$?
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/${T}_launches.csv \
   python bench.py --steps 2 --warmup 3 --no-cpu-baseline > /dev/null 2>&1; echo launches=$?
-for k in smem_subgraph msp_block scatter_kernel bucket_scatter; do
+for k in smem_subgraph msp_block ts_level_a ts_level_b; do
   timeout 1200 ncu --set full --import-source on --clock-control none -k regex:$k -s 3 -c 1 -o gpurun_out/${T}_chr14_$k -f \
     python bench.py --steps 1 --warmup 3 --no-cpu-baseline > gpurun_out/${T}_ncu_chr14_$k.log 2>&1; echo "ncu chr14 $k=$?"
 done
@@ -20,6 +20,7 @@ for k in smem_subgraph msp_warp; do
   timeout 1500 ncu --set full --import-source on --clock-control none -k regex:$k -s 3 -c 1 -o gpurun_out/${T}_bbee_$k -f \
     python bench.py --config bumblebee --steps 1 --warmup 3 --no-cpu-baseline > gpurun_out/${T}_ncu_bbee_$k.log 2>&1; echo "ncu bbee $k=$?"
 done
+timeout 1200 python tools/human_run.py > gpurun_out/${T}_human.json 2> gpurun_out/${T}_human.err; echo human=$?; tail -c 400 gpurun_out/${T}_human.json
 for tool in memcheck racecheck synccheck initcheck; do
   timeout 1500 compute-sanitizer --tool $tool --print-limit 50 python tools/sanitize_driver.py > gpurun_out/${T}_san_$tool.log 2>&1
   echo "$tool rc=$?"; tail -1 gpurun_out/${T}_san_$tool.log

@@ -29,7 +29,7 @@ def _check(tag, rs, k, p, np_, two_level_min_bytes=None, **kw):
         res = build_graph(rs.seq, rs.offsets, k, p, np_, **kw)
     else:  # the two-level scatter at a size where the builder would not pick it
         b = DbgBuilder(k, p, np_, **kw)
-        b.two_level_min_bytes = two_level_min_bytes
+        b.two_level_min_bytes, b.two_level_words = two_level_min_bytes, (4, 8, 16)
         d_bases, d_off = b.upload(encode_reads(rs.seq), rs.offsets)
         res = b.build(d_bases, d_off)
     if k > 63:
@@ -55,9 +55,10 @@ def main():
     ok = True
     ok &= _check("smem K=31 P=11 (register MSP, split + global tier)", rs, 31, 11, 2, refine=1)
     ok &= _check("smem K=31 P=11 fine_p 13 (reading V)", rs, 31, 11, 8, refine=4, fine_p=13)
-    ok &= _check("smem K=63 P=19 (generic MSP, 40-bit row)", rs, 63, 19, 4, refine=2)
-    ok &= _check("smem K=41 P=17 (generic MSP)", rs, 41, 17, 4, refine=2)
+    ok &= _check("smem K=63 P=19 (warp MSP, TMA-staged reads)", rs, 63, 19, 4, refine=2)
+    ok &= _check("smem K=41 P=17 (warp MSP)", rs, 41, 17, 4, refine=2)
     ok &= _check("smem two-level scatter (10000 fine partitions)", rs, 31, 11, 16, refine=625, two_level_min_bytes=0)
+    ok &= _check("smem two-level scatter, 8-word records", rs, 63, 19, 16, refine=625, two_level_min_bytes=0)
     ok &= _check("resident K=31", rs, 31, 11, 4, mode="resident")
     ok &= _check("wide K=65 (locked state)", rs, 65, 21, 3)
     ok &= _check("wide K=101 hot key", hot, 101, 19, 2)
