@@ -423,11 +423,13 @@ def run_ours(args):
                "sample": f"first {sub.n_reads} of {rs.n_reads} reads ({sub.n_kmers()} K-mers), {dt:.1f} s",
                "single_thread_ecoli": _oracle_single_thread_ecoli()}
     scan = 1 if b.np <= 16384 else 3  # scan.cuh: one CTA, or tile sums + tile scan + apply
-    # Step 1: msp kernel + its scan + scatter; Step 2: the on-chip plan (8 kernels incl. the greedy
-    # group packing) + the on-chip kernel (+ per global-tier batch: its plan scan once,
-    # hash_build_list + extract_kernel); multi-GPU adds the exchange plan (scan + 1)
+    # Step 1: msp kernel + its scan + the scatter (one kernel, or the two-level one: bucket counts,
+    # bucket scan, level A, level B); Step 2: the on-chip plan (8 kernels incl. the greedy group
+    # packing) + the on-chip kernel (+ per global-tier batch: its plan scan once, hash_build_list +
+    # extract_kernel); multi-GPU adds the exchange plan (scan + 1)
     nb = len(b.batches)
-    launches_per_step = 2 + scan + 9 + 2 * nb + (scan if nb else 0) + (scan + 1 if ws > 1 else 0)
+    scatter = 4 if src.use_two_level() else 1
+    launches_per_step = 1 + scan + scatter + 9 + 2 * nb + (scan if nb else 0) + (scan + 1 if ws > 1 else 0)
     placement = _placement(b)
     # Fig. 6 / Table II analogue (row f1): the paper's partitions (the vertices' pid, reading V; K-mers
     # = sum of their counts) -- skew and the table size lambda/(4 alpha) N^i_kmer x slot bytes of the

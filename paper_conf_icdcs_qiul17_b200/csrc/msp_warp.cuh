@@ -55,7 +55,13 @@ __device__ __forceinline__ T tmin(T x, T y) { return y < x ? y : x; }
 
 // R: P-mer positions per lane; KC, PC > 0: compile-time K and P; DESC: descriptor list length.
 template <typename CT, int R, int KC, int PC, int DESC>
-__global__ void __launch_bounds__(kWarpMspThreads, 3) msp_warp_kernel(MspArgs a) {
+#ifndef DBG_MSPW_MINB
+#define DBG_MSPW_MINB 3
+#endif
+#ifndef DBG_MSPW_DESC64
+#define DBG_MSPW_DESC64 256
+#endif
+__global__ void __launch_bounds__(kWarpMspThreads, DBG_MSPW_MINB) msp_warp_kernel(MspArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   typedef WarpMspSmem<CT, DESC> S;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -404,7 +410,7 @@ static cudaError_t launch_msp_warp_any(const MspArgs& a, cudaStream_t stream) {
       case 15: return launch_msp_warp<uint32_t, 3, 31, 15, 384>(a, stream);
     }
   }
-  if (a.k == 63 && a.p == 19) return launch_msp_warp<uint64_t, 4, 63, 19, 256>(a, stream);
+  if (a.k == 63 && a.p == 19) return launch_msp_warp<uint64_t, 4, 63, 19, DBG_MSPW_DESC64>(a, stream);
   return a.p <= 16 ? launch_msp_warp<uint32_t, 4, 0, 0, 384>(a, stream)
                    : launch_msp_warp<uint64_t, 4, 0, 0, 256>(a, stream);
 }
