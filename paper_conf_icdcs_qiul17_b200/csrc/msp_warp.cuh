@@ -53,15 +53,11 @@ __device__ __forceinline__ uint64_t revcomp32(uint64_t x) {
 template <typename T>
 __device__ __forceinline__ T tmin(T x, T y) { return y < x ? y : x; }
 
-// R: P-mer positions per lane; KC, PC > 0: compile-time K and P; DESC: descriptor list length.
-template <typename CT, int R, int KC, int PC, int DESC>
-#ifndef DBG_MSPW_MINB
-#define DBG_MSPW_MINB 3
-#endif
-#ifndef DBG_MSPW_DESC64
-#define DBG_MSPW_DESC64 256
-#endif
-__global__ void __launch_bounds__(kWarpMspThreads, DBG_MSPW_MINB) msp_warp_kernel(MspArgs a) {
+// R: P-mer positions per lane; KC, PC > 0: compile-time K and P; DESC: descriptor list length;
+// MINB: CTAs per SM the registers are capped for (K = 63: 4 CTAs x 8 warps with <= 64 registers and
+// 192 descriptors, 46.8 vs 47.4 ms with 3 CTAs, profiles/r02_ab.txt; runtime K, P: 3, no spills).
+template <typename CT, int R, int KC, int PC, int DESC, int MINB>
+__global__ void __launch_bounds__(kWarpMspThreads, MINB) msp_warp_kernel(MspArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   typedef WarpMspSmem<CT, DESC> S;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -381,10 +377,10 @@ __global__ void __launch_bounds__(kWarpMspThreads, DBG_MSPW_MINB) msp_warp_kerne
   }
 }
 
-template <typename CT, int R, int KC, int PC, int DESC>
+template <typename CT, int R, int KC, int PC, int DESC, int MINB>
 static cudaError_t launch_msp_warp(const MspArgs& a, cudaStream_t stream) {
   const size_t smem = sizeof(WarpMspSmem<CT, DESC>) * kWarpMspWarps;
-  auto fn = msp_warp_kernel<CT, R, KC, PC, DESC>;
+  auto fn = msp_warp_kernel<CT, R, KC, PC, DESC, MINB>;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int per_sm = 0;
@@ -397,22 +393,13 @@ static cudaError_t launch_msp_warp(const MspArgs& a, cudaStream_t stream) {
   return cudaGetLastError();
 }
 
-// Compile-time (K, P) for the configurations (K = 31 with P = 11..15: 32-bit codes, 3 positions
-// per lane = 78 K-mers per piece for w = 19; K = 63, P = 19: 64-bit codes, 4 positions per lane),
-// else runtime K, P with 4 positions per lane (w <= 128 for every K <= 127).
+// Compile-time (K, P) = (63, 19) for bumblebee (64-bit codes, 4 positions per lane), else runtime
+// K, P with 4 positions per lane (w <= 128 for every K <= 127).  K = 31 with P = 11..15 never gets
+// here: msp_block_kernel is faster for it (msp.cu).
 static cudaError_t launch_msp_warp_any(const MspArgs& a, cudaStream_t stream) {
-  if (a.k == 31) {
-    switch (a.p) {
-      case 11: return launch_msp_warp<uint32_t, 3, 31, 11, 384>(a, stream);
-      case 12: return launch_msp_warp<uint32_t, 3, 31, 12, 384>(a, stream);
-      case 13: return launch_msp_warp<uint32_t, 3, 31, 13, 384>(a, stream);
-      case 14: return launch_msp_warp<uint32_t, 3, 31, 14, 384>(a, stream);
-      case 15: return launch_msp_warp<uint32_t, 3, 31, 15, 384>(a, stream);
-    }
-  }
-  if (a.k == 63 && a.p == 19) return launch_msp_warp<uint64_t, 4, 63, 19, DBG_MSPW_DESC64>(a, stream);
-  return a.p <= 16 ? launch_msp_warp<uint32_t, 4, 0, 0, 384>(a, stream)
-                   : launch_msp_warp<uint64_t, 4, 0, 0, 256>(a, stream);
+  if (a.k == 63 && a.p == 19) return launch_msp_warp<uint64_t, 4, 63, 19, 192, 4>(a, stream);
+  return a.p <= 16 ? launch_msp_warp<uint32_t, 4, 0, 0, 384, 3>(a, stream)
+                   : launch_msp_warp<uint64_t, 4, 0, 0, 256, 3>(a, stream);
 }
 
 }  // namespace dbg
