@@ -26,7 +26,7 @@ extern "C" uint64_t dbg_scatter_work_words(const dbg_params* prm) {
   if (!prm || prm->num_partitions < 1) return 0;
   const int64_t np = (int64_t)prm->num_partitions * (prm->refine > 1 ? prm->refine : 1);
   int s = 0;
-  while (s < 12 && ((np + (1ll << s) - 1) >> s) > 2048) ++s;
+  while (s < 12 && ((np + (1ll << s) - 1) >> s) > 2048) ++s;  // msp.cu ts_shift's rule
   const uint64_t nb = (uint64_t)((np + (1ll << s) - 1) >> s);
   return 3 * nb + 2;
 }

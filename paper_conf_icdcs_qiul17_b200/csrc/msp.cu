@@ -354,7 +354,7 @@ template <int R>
 __host__ __device__ constexpr int ts_tile() { return kTsThreads * ts_per<R>(); }  // <= 128 KB of records
 // log2 of the bucket width: the smallest s with <= 2048 buckets, at most 12 (4096 partitions a
 // bucket; <= 4096 buckets for the 2^24 - 1 fine partitions of dbg.h)
-__host__ __device__ inline int ts_shift(int np) {
+__host__ __device__ inline int ts_shift(int np) {  // (r02z6: 1024 / 4096 buckets: mixed / slower)
   int s = 0;
   while (s < 12 && ((np + (1 << s) - 1) >> s) > 2048) ++s;
   return s;

@@ -49,6 +49,17 @@ def test_abi_and_sizes(lib):
     assert lib.dbg_record_words(lib.params(65, 11, 16)) == 16 and lib.dbg_record_max_kmers(lib.params(65, 11, 16)) == 63
     # fine partitions: NP * refine <= 2^24 - 1 (the header's 24-bit pid field); whole human (65.1 G
     # K-mers, NP = 960) wants ~39 M and is clamped there
+    # two-level scatter workspace: fill, offsets and tile counts of the <= 2048 buckets (<= 4096 at
+    # 2^24 - 1 fine partitions, 4096 partitions a bucket) that msp.cu's ts_shift picks
+    def buckets(np_):
+        sh = 0
+        while sh < 12 and -(-np_ // (1 << sh)) > 2048:
+            sh += 1
+        return -(-np_ // (1 << sh))
+    for np_, ref in ((16, 1), (16, 625), (512, 3084), (512, 7444), (960, 17476)):
+        nb = buckets(np_ * ref)
+        assert nb <= 4096
+        assert lib.dbg_scatter_work_words(lib.params(31, 11, np_, refine=ref)) == 3 * nb + 2
     from paper_conf_icdcs_qiul17_b200.graph import MAX_FINE_PARTITIONS, auto_refine
     assert MAX_FINE_PARTITIONS == (1 << 24) - 1
     assert auto_refine(65_100_000_000, 31, 11, 960) == MAX_FINE_PARTITIONS // 960
